@@ -1,0 +1,54 @@
+/*
+ * oracle.h -- CPU oracle for the NBA IPsec ESP hot path.  TEST INFRASTRUCTURE
+ * ONLY (see oracle.c header).  Independent of include/nba_ipsec.h: nothing
+ * here is shared with the CUDA library and neither side includes the other.
+ */
+#ifndef NBA_ORACLE_H
+#define NBA_ORACLE_H
+#include <stddef.h>
+#include <stdint.h>
+
+#define ORACLE_MIN_DATAGRAM 20u    /* A15: smallest IPv4 datagram */
+#define ORACLE_MAX_DATAGRAM 1500u  /* A15: paper's largest size */
+
+#define ORACLE_EFORMAT  -1
+#define ORACLE_ECSUM    -2
+#define ORACLE_EICV     -3
+#define ORACLE_ETRAILER -4
+
+typedef struct {
+    uint32_t spi;
+    uint32_t tunnel_src, tunnel_dst;
+    uint8_t  aes_key[16];
+    uint8_t  ctr_nonce[4];
+    uint8_t  hmac_key[20];
+    uint32_t seq;                 /* last sequence number used */
+} oracle_sa;
+
+typedef struct { uint64_t pkts_ok, pkts_dropped, bytes_in, bytes_out, batches; } oracle_counters;
+
+void     oracle_init(void);
+uint8_t  oracle_sbox(uint8_t x);
+void     oracle_aes128_expand_key(const uint8_t key[16], uint8_t w[176]);
+void     oracle_aes128_encrypt_w(const uint8_t w[176], const uint8_t in[16], uint8_t out[16]);
+void     oracle_aes128_encrypt(const uint8_t key[16], const uint8_t in[16], uint8_t out[16]);
+void     oracle_ctr_xcrypt(const uint8_t key[16], const uint8_t icb[16], const uint8_t *in,
+                           size_t len, uint8_t *out);
+void     oracle_sha1(const uint8_t *msg, size_t len, uint8_t out[20]);
+void     oracle_hmac_sha1(const uint8_t *key, size_t klen, const uint8_t *msg, size_t mlen,
+                          uint8_t out[20]);
+uint16_t oracle_ipv4_checksum(const uint8_t *hdr, size_t len);
+uint32_t oracle_esp_encap(const oracle_sa *sa, uint32_t q, const uint8_t *P, uint32_t D,
+                          uint8_t *out);
+void     oracle_process_batch(oracle_sa *sas, uint32_t n_sa, const uint8_t *in_buf,
+                              const uint32_t *in_off, const uint16_t *in_len,
+                              const uint32_t *sa_idx, uint8_t *out_buf, const uint32_t *out_off,
+                              uint16_t *out_len, uint32_t n, oracle_counters *ctr);
+int      oracle_process_batch_mt(oracle_sa *sas, uint32_t n_sa, const uint8_t *in_buf,
+                                 const uint32_t *in_off, const uint16_t *in_len,
+                                 const uint32_t *sa_idx, uint8_t *out_buf,
+                                 const uint32_t *out_off, uint16_t *out_len, uint32_t n,
+                                 oracle_counters *ctr, int n_threads);
+int      oracle_decap(const oracle_sa *sa, const uint8_t *pkt, uint32_t len, uint8_t *inner,
+                      uint32_t *inner_len, uint32_t *seq_out);
+#endif

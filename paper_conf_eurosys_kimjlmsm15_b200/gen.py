@@ -1,0 +1,203 @@
+"""Seeded synthetic workload generator (SA tables + packet batches).
+
+This module holds NONE of the method's arithmetic (no AES, SHA-1, HMAC, ESP
+framing or outer-header logic).  It only synthesises inputs, and it is the one
+piece of code shared by the CUDA path's tests/bench and the oracle.
+
+Workload recipe:
+  * "randomly generated IP traffic with UDP payloads", IPv4 headers for IPsec
+    (§4.1 "Workloads");
+  * packet sizes 64..1514 B frames (Fig. 12(c) x-axis), IMIX
+    64/594/1514 at 7:4:1 (BASELINE.json configs[3]);
+  * 1024 SAs, random keys (BASELINE.json north_star; per-flow contexts
+    PAPER.md:395).
+Frame length L excludes the FCS; the library sees only the inner IPv4
+datagram, D = L - 14 (reading A2).
+"""
+from __future__ import annotations
+
+import dataclasses
+
+import numpy as np
+
+SEED = 20150421
+SLOT = 2048          # packet-pool slot stride (bytes)
+HEADROOM = 128       # headroom before the Ethernet header in each slot
+ETH = 14
+IMIX_SIZES = (64, 594, 1514)
+IMIX_WEIGHTS = (7, 4, 1)
+TUN_SRC = (192 << 24) | (0 << 16) | (2 << 8) | 1          # 192.0.2.1 (RFC 5737)
+TUN_DST_BASE = (198 << 24) | (51 << 16) | (100 << 8)      # 198.51.100.0/24
+
+
+def rng_for(cfg_id: int, rank: int = 0, batch: int = 0, salt: int = 0) -> np.random.Generator:
+    return np.random.default_rng([SEED, cfg_id, rank, batch, salt])
+
+
+@dataclasses.dataclass
+class SAParams:
+    """SoA security-association parameters (host order integers)."""
+    spi: np.ndarray          # u32[n]
+    tunnel_src: np.ndarray   # u32[n]
+    tunnel_dst: np.ndarray   # u32[n]
+    aes_key: np.ndarray      # u8[n,16]
+    ctr_nonce: np.ndarray    # u8[n,4]
+    hmac_key: np.ndarray     # u8[n,20]
+    seq: np.ndarray          # u32[n]
+
+    def __len__(self):
+        return int(self.spi.shape[0])
+
+    def copy(self) -> "SAParams":
+        return SAParams(*(np.array(getattr(self, f.name)) for f in dataclasses.fields(self)))
+
+
+@dataclasses.dataclass
+class Batch:
+    n: int
+    in_buf: np.ndarray       # u8[pool]
+    in_off: np.ndarray       # u32[n]  offset of the inner IPv4 datagram
+    in_len: np.ndarray       # u16[n]  D
+    sa_idx: np.ndarray       # u32[n]
+    out_off: np.ndarray      # u32[n]
+    out_pool_bytes: int
+    frame_len: np.ndarray    # u32[n]  L (for Gbps accounting, reading A18)
+
+
+def make_sas(n_sa: int, cfg_id: int = 0, rank: int = 0, world: int = 1,
+             seq0: int | np.ndarray = 0) -> SAParams:
+    """SA table for one rank: global SA ids s = rank + world*j (SA-hash shard)."""
+    r = rng_for(cfg_id, rank, 0, salt=1)
+    gid = rank + world * np.arange(n_sa, dtype=np.int64)
+    seq = np.full(n_sa, 0, np.uint32) if np.isscalar(seq0) else np.asarray(seq0, np.uint32)
+    if np.isscalar(seq0):
+        seq[:] = np.uint32(seq0)
+    return SAParams(
+        spi=(0x100 + gid).astype(np.uint32),
+        tunnel_src=np.full(n_sa, TUN_SRC, np.uint32),
+        tunnel_dst=(TUN_DST_BASE + (gid % 254) + 1).astype(np.uint32),
+        aes_key=r.integers(0, 256, (n_sa, 16), dtype=np.uint8),
+        ctr_nonce=r.integers(0, 256, (n_sa, 4), dtype=np.uint8),
+        hmac_key=r.integers(0, 256, (n_sa, 20), dtype=np.uint8),
+        seq=seq,
+    )
+
+
+def frame_sizes(n: int, size, r: np.random.Generator) -> np.ndarray:
+    """Frame lengths L for n packets: an int, 'imix', or an explicit array."""
+    if isinstance(size, str):
+        assert size == "imix"
+        w = np.array(IMIX_WEIGHTS, np.int64)
+        counts = (n * w) // w.sum()
+        for j in range(int(n - counts.sum())):           # leftovers to the largest sizes
+            counts[len(w) - 1 - j] += 1                   # (65536 -> 38229/21845/5462)
+        L = np.repeat(np.array(IMIX_SIZES, np.uint32), counts)
+        return L[r.permutation(n)]                          # Fisher-Yates shuffle
+    if np.isscalar(size):
+        return np.full(n, int(size), np.uint32)
+    a = np.asarray(size, np.uint32)
+    assert a.shape == (n,)
+    return a
+
+
+def _csum16(words: np.ndarray) -> np.ndarray:
+    """Input synthesis only: inner IPv4 header checksum for realism."""
+    s = words.astype(np.uint64).sum(axis=1)
+    while np.any(s >> 16):
+        s = (s & 0xFFFF) + (s >> 16)
+    return (~s & 0xFFFF).astype(np.uint16)
+
+
+def make_batch(n: int, size, n_sa: int, cfg_id: int = 0, rank: int = 0, batch: int = 0,
+               locality: int = 1, layout: str = "slots", in_len_override=None,
+               sa_idx_override=None) -> Batch:
+    """Synthesise one batch of n packets.
+
+    layout="slots": slot stride 2048, headroom 128 -> in_off = 2048 i + 142
+    (≡ 14 mod 16, deliberately unaligned), same formula for out_off in a
+    separate pool.  layout="packed": datagrams back to back (for host I/O).
+    locality=k: SA chosen per run of k consecutive packets (flow locality)."""
+    r = rng_for(cfg_id, rank, batch)
+    L = frame_sizes(n, size, r)
+    D = (L.astype(np.int64) - ETH)
+    if in_len_override is not None:
+        D = np.asarray(in_len_override, np.int64)
+        assert D.shape == (n,)
+    Dc = np.clip(D, 0, SLOT - HEADROOM - ETH)
+    runs = (n + locality - 1) // max(locality, 1)
+    sa = np.repeat(r.integers(0, max(n_sa, 1), runs, dtype=np.int64), locality)[:n]
+    if sa_idx_override is not None:
+        sa = np.asarray(sa_idx_override, np.int64)
+    if layout == "slots":
+        in_off = (SLOT * np.arange(n, dtype=np.int64) + HEADROOM + ETH)
+        out_off = in_off.copy()
+        pool = SLOT * max(n, 1)
+        out_pool = pool
+    elif layout == "packed":
+        in_off = np.concatenate([[0], np.cumsum(Dc)[:-1]]) if n else np.zeros(0, np.int64)
+        pool = int(Dc.sum()) + 16
+        cap = Dc + 64
+        out_off = np.concatenate([[0], np.cumsum(cap)[:-1]]) if n else np.zeros(0, np.int64)
+        out_pool = int(cap.sum()) + 16
+    else:
+        raise ValueError(layout)
+
+    buf = np.zeros(pool, np.uint8)
+    if n:
+        maxD = int(Dc.max())
+        # random datagram bytes, then overwrite the IPv4/UDP headers
+        pk = r.integers(0, 256, (n, max(maxD, 28)), dtype=np.uint8)
+        hdr = np.zeros((n, 28), np.uint8)
+        hdr[:, 0] = 0x45
+        hdr[:, 1] = 0                                    # TOS 0
+        hdr[:, 2] = (Dc >> 8) & 0xFF
+        hdr[:, 3] = Dc & 0xFF
+        hdr[:, 4:6] = r.integers(0, 256, (n, 2), dtype=np.uint8)   # ID
+        hdr[:, 6] = 0x40                                 # DF
+        hdr[:, 8] = 64                                   # TTL
+        hdr[:, 9] = 17                                   # UDP
+        hdr[:, 12] = 10
+        hdr[:, 13:16] = r.integers(0, 256, (n, 3), dtype=np.uint8)
+        hdr[:, 16] = 10
+        hdr[:, 17:20] = r.integers(0, 256, (n, 3), dtype=np.uint8)
+        words = (hdr[:, 0:20:2].astype(np.uint32) << 8) | hdr[:, 1:20:2]
+        cs = _csum16(words)
+        hdr[:, 10] = cs >> 8
+        hdr[:, 11] = cs & 0xFF
+        ports = r.integers(1024, 65536, (n, 2), dtype=np.int64)
+        hdr[:, 20] = ports[:, 0] >> 8
+        hdr[:, 21] = ports[:, 0] & 0xFF
+        hdr[:, 22] = ports[:, 1] >> 8
+        hdr[:, 23] = ports[:, 1] & 0xFF
+        ulen = np.clip(Dc - 20, 0, 65535)
+        hdr[:, 24] = (ulen >> 8) & 0xFF
+        hdr[:, 25] = ulen & 0xFF
+        pk[:, :28] = hdr
+        W = pk.shape[1]
+        mask = np.arange(W)[None, :] < Dc[:, None]
+        if layout == "slots":
+            pool2d = buf.reshape(n, SLOT)
+            view = pool2d[:, HEADROOM + ETH:HEADROOM + ETH + W]
+            view[mask[:, :view.shape[1]]] = pk[:, :view.shape[1]][mask[:, :view.shape[1]]]
+            # Ethernet header in front of the datagram (random MACs, type 0x0800)
+            eth = r.integers(0, 256, (n, ETH), dtype=np.uint8)
+            eth[:, 12] = 0x08
+            eth[:, 13] = 0x00
+            pool2d[:, HEADROOM:HEADROOM + ETH] = eth
+        else:
+            flat = pk[mask]                                  # row-major = back to back
+            buf[:flat.size] = flat
+    return Batch(n=n, in_buf=buf, in_off=in_off.astype(np.uint32),
+                 in_len=np.asarray(D, np.int64).astype(np.uint16), sa_idx=sa.astype(np.uint32),
+                 out_off=out_off.astype(np.uint32), out_pool_bytes=int(out_pool),
+                 frame_len=L.astype(np.uint32))
+
+
+# BASELINE.json configs, in order (configs[0..4]).
+CONFIGS = {
+    1: dict(name="c1_64x64B_1sa", n=64, size=64, n_sa=1),
+    2: dict(name="c2_64B_1024sa", n=65536, size=64, n_sa=1024),
+    3: dict(name="c3_1514B_1024sa", n=65536, size=1514, n_sa=1024),
+    4: dict(name="c4_imix_1024sa", n=65536, size="imix", n_sa=1024),
+}
+SWEEP_SIZES = (64, 128, 256, 512, 1024, 1514, "imix")   # configs[4]
