@@ -1,0 +1,164 @@
+/*
+ * nba_ipsec.h -- C ABI of the B200-native IPsec ESP outbound hot path.
+ *
+ * What the library computes:
+ *   NBA's "IPsec encryption gateway" offloads, per packet, "HMAC-SHA1 to
+ *   authenticate the packets and AES-128CTR to encrypt them"
+ *   (§4.1 "Sample applications"), using per-flow crypto
+ *   contexts initialised once and reused "by only changing initial vector
+ *   (IV) values".  The offloaded function consumes a
+ *   *datablock*: byte ranges of packets given by offset/length (PAPER.md:329-343,
+ *   §3.3 and Table 2) and returns whole packets with a size delta.  The
+ *   framework validates fields before execution; invalid
+ *   packets are dropped, not branched.
+ *   The ESP wire format is not in the paper; it is fixed by the readings
+ *   A1..A24 of DESIGN.md §3 (RFC 4303 tunnel mode, RFC 3686 AES-CTR,
+ *   RFC 2404 HMAC-SHA1-96).  Per packet i with SA s = sa_idx[i] and inner
+ *   IPv4 datagram P of D = in_len[i] bytes, the library writes at
+ *   out_buf + out_off[i]:
+ *       outer IPv4 (20 B) || SPI || seq || IV=BE64(seq) || AES-CTR(P||pad||p||4) || ICV(12 B)
+ *   and out_len[i] = 48 + C, C = D + p + 2, p = (-(D+2)) mod 4.
+ *
+ * Threading/ordering: calls on one table must be serialised on one CUDA
+ * stream (sequence numbers are stream-ordered state).  Different tables and
+ * devices may run concurrently.
+ *
+ * Errors: argument errors are detected on the host before any work is
+ * enqueued and return a negative NBA_IPSEC_E* code.  Per-packet problems are
+ * NOT errors: the packet is dropped (out_len[i] = 0, pkts_dropped++) when
+ * sa_idx[i] >= n_sa, D < 20, D > 1500, or the SA's 32-bit sequence number
+ * space is exhausted (RFC 4303 §3.3.3).  Launch failures return
+ * NBA_IPSEC_ECUDA; asynchronous faults surface at the caller's next
+ * synchronisation.
+ */
+#ifndef NBA_IPSEC_H
+#define NBA_IPSEC_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum {
+    NBA_IPSEC_OK = 0,
+    NBA_IPSEC_EINVAL = -22,
+    NBA_IPSEC_ENOMEM = -12,
+    NBA_IPSEC_ENODEV = -19,
+    NBA_IPSEC_ECUDA = -1000
+};
+
+#define NBA_IPSEC_MIN_DATAGRAM 20u    /* smallest inner IPv4 datagram (reading A15) */
+#define NBA_IPSEC_MAX_DATAGRAM 1500u  /* largest inner datagram, PAPER.md:603 (A15) */
+#define NBA_IPSEC_MAX_OVERHEAD 53u    /* 20 outer + 8 ESP + 8 IV + 3 pad + 2 trailer + 12 ICV */
+#define NBA_IPSEC_MAX_SA       65536u /* per table */
+#define NBA_IPSEC_MAX_BATCH    (1u << 22)
+
+/* Per-SA parameters ("envelope contexts for all flows").
+ * Integers are in host byte order. */
+typedef struct {
+    uint32_t spi;                    /* != 0 recommended (RFC 4303 §2.1); not checked */
+    uint32_t tunnel_src, tunnel_dst; /* outer IPv4 addresses */
+    uint8_t  aes_key[16];            /* AES-128 key (RFC 3686 §5 KEYMAT bytes 0..15) */
+    uint8_t  ctr_nonce[4];           /* RFC 3686 nonce (KEYMAT bytes 16..19) */
+    uint8_t  hmac_key[20];           /* RFC 2404: 160-bit HMAC-SHA1 key */
+    uint32_t seq;                    /* last sequence number used; 0 => first packet gets 1 */
+} nba_ipsec_sa_params;
+
+typedef struct nba_ipsec_sa_table nba_ipsec_sa_table;  /* opaque; owns SA state + workspace */
+
+/* One batch ("datablock" view).  For process_batch every
+ * pointer is a DEVICE pointer on the table's device; for process_batch_host
+ * every pointer is a HOST pointer (pinned memory recommended).
+ *   in_buf  + in_off[i]  : inner IPv4 datagram i, in_len[i] bytes, any alignment
+ *   sa_idx[i]            : SA index of packet i in [0, n_sa) (else dropped)
+ *   out_buf + out_off[i] : output slot i; capacity must be >= in_len[i] + 53;
+ *                          only bytes [0, out_len[i]) are written
+ *   out_len[i]           : written: 48 + C, or 0 if dropped
+ * in_buf and out_buf ranges must not overlap.  Slot i corresponds to packet i
+ * (order preserved). */
+typedef struct {
+    const uint8_t  *in_buf;
+    const uint32_t *in_off;
+    const uint16_t *in_len;
+    const uint32_t *sa_idx;
+    uint8_t        *out_buf;
+    const uint32_t *out_off;
+    uint16_t       *out_len;
+    uint32_t        n_pkts;
+} nba_ipsec_batch;
+
+/* Build the per-device SA table (AES-128 key schedules per FIPS-197 §5.2,
+ * HMAC-SHA1 inner/outer midstates per RFC 2104) and a workspace sized for
+ * max_batch_pkts packets.  `sas` is copied; the caller may free it on return.
+ * All device memory is allocated here (none in process_batch).
+ * Returns NBA_IPSEC_EINVAL for NULL sas/out, n_sa == 0 or > NBA_IPSEC_MAX_SA,
+ * max_batch_pkts == 0 or > NBA_IPSEC_MAX_BATCH; NBA_IPSEC_ENODEV for a bad
+ * device; NBA_IPSEC_ENOMEM if allocation fails. */
+int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int cuda_device,
+                              uint32_t max_batch_pkts, nba_ipsec_sa_table **out);
+
+/* Enqueue the whole ESP outbound path for one batch on `cuda_stream`
+ * (a cudaStream_t; NULL = legacy default stream) and return immediately.
+ * Device pointers only.  n_pkts == 0 is a no-op returning NBA_IPSEC_OK.
+ * Returns NBA_IPSEC_EINVAL for NULL t/b, n_pkts > max_batch_pkts or a NULL
+ * array with n_pkts > 0; NBA_IPSEC_ECUDA if a launch fails. */
+int nba_ipsec_process_batch(nba_ipsec_sa_table *t, const nba_ipsec_batch *b, void *cuda_stream);
+
+/* Same computation with HOST buffers (end-to-end path): copies
+ * in_buf[0, in_buf_bytes), in_off, in_len, sa_idx host->device, runs the
+ * path, copies out_buf[0, out_buf_bytes) and out_len device->host, all
+ * enqueued on `cuda_stream`.  Needs staging reserved with
+ * nba_ipsec_reserve_host_io; returns NBA_IPSEC_EINVAL if it is too small.
+ * The host buffers must stay valid until the stream passes the batch. */
+int nba_ipsec_process_batch_host(nba_ipsec_sa_table *t, const nba_ipsec_batch *b,
+                                 uint64_t in_buf_bytes, uint64_t out_buf_bytes,
+                                 void *cuda_stream);
+int nba_ipsec_reserve_host_io(nba_ipsec_sa_table *t, uint64_t in_buf_bytes,
+                              uint64_t out_buf_bytes);
+
+/* Free everything.  NULL -> NBA_IPSEC_OK.  Synchronises the table's device. */
+int nba_ipsec_destroy(nba_ipsec_sa_table *t);
+
+/* ---- auxiliary: tests, resume, bench -------------------------------------- */
+typedef struct { uint64_t pkts_ok, pkts_dropped, bytes_in, bytes_out, batches; } nba_ipsec_counters;
+
+/* Device counters accumulated since create.  Synchronises `cuda_stream`. */
+int nba_ipsec_read_counters(nba_ipsec_sa_table *t, nba_ipsec_counters *out, void *cuda_stream);
+/* Current per-SA sequence numbers (the only cross-batch state; re-import via
+ * nba_ipsec_sa_params.seq for exact resume).  host_seq has n_sa entries.
+ * Synchronises `cuda_stream`. */
+int nba_ipsec_read_sa_seq(nba_ipsec_sa_table *t, uint32_t *host_seq, void *cuda_stream);
+const char *nba_ipsec_strerror(int code);
+
+/* Pipeline selection (both produce identical bytes):
+ *   NBA_IPSEC_PIPE_FUSED   : prologue + one fused gather/AES/HMAC/scatter kernel (default)
+ *   NBA_IPSEC_PIPE_UNFUSED : prologue, gather, AES-CTR, HMAC-SHA1, scatter kernels */
+enum { NBA_IPSEC_PIPE_FUSED = 0, NBA_IPSEC_PIPE_UNFUSED = 1 };
+int nba_ipsec_set_pipeline(nba_ipsec_sa_table *t, int pipeline);
+/* Number of kernel launches one process_batch call enqueues (n_pkts > 0). */
+int nba_ipsec_launches_per_batch(nba_ipsec_sa_table *t);
+
+/* Per-kernel timing with CUDA events recorded on the caller's stream between
+ * the kernels of each batch.  enable=1 starts (and resets) collection;
+ * nba_ipsec_profile_read synchronises the device, and returns per-kernel sums
+ * of milliseconds over all profiled batches (ms[k], k < *n_kernels, at most
+ * max entries) with short kernel names (names[k] static strings), and the
+ * number of profiled batches. */
+int nba_ipsec_profile_enable(nba_ipsec_sa_table *t, int enable);
+int nba_ipsec_profile_read(nba_ipsec_sa_table *t, double *ms, const char **names, int max,
+                           int *n_kernels, uint32_t *n_batches);
+
+/* Host-only helpers exported for tests of the library's own setup code
+ * (no device needed): the AES-128 key schedule (FIPS-197 §5.2; 44 words,
+ * word i = bytes w[4i..4i+3] of the standard, big-endian) and the HMAC-SHA1
+ * inner/outer chaining values after compressing K0^ipad / K0^opad
+ * (RFC 2104 §2; FIPS 180-4 §6.1.2). */
+void nba_ipsec_host_aes128_key_schedule(const uint8_t key[16], uint32_t w[44]);
+void nba_ipsec_host_hmac_sha1_midstates(const uint8_t key[20], uint32_t hin[5], uint32_t hout[5]);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* NBA_IPSEC_H */

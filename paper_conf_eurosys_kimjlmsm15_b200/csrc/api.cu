@@ -1,0 +1,423 @@
+// api.cu -- the C ABI of libnba_ipsec.so (include/nba_ipsec.h): SA-table
+// construction (row a0), argument validation, workspace ownership and the
+// per-batch launch sequence (rows a1..a5).
+//
+// per-flow crypto contexts are built once at startup and reused;
+// the framework validates datablock fields before execution;
+// offloads aggregate thousands of packets -- here a batch is up
+// to max_batch_pkts packets that stay resident in HBM.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <vector>
+
+#include "internal.cuh"
+#include "nba_ipsec.h"
+
+using namespace nba;
+
+namespace {
+
+constexpr int PROF_RING = 64;
+constexpr int MAX_KERNELS = 8;
+
+struct ProfSet {
+    cudaEvent_t ev[MAX_KERNELS + 1] = {};
+    int n_ev = 0;          // events recorded in this set (0 = empty)
+};
+
+}  // namespace
+
+struct nba_ipsec_sa_table {
+    int device = 0;
+    uint32_t n_sa = 0, max_batch = 0, max_tiles = 0;
+    int num_sms = 0;
+    int grid_aes = 0, grid_fused = 0;
+    int pipeline = NBA_IPSEC_PIPE_UNFUSED;
+    DevTable T{};
+    DevWork W{};
+    std::vector<void *> allocs;
+    // host-I/O staging (process_batch_host)
+    uint8_t *io_in = nullptr, *io_out = nullptr;
+    uint64_t io_in_bytes = 0, io_out_bytes = 0;
+    uint32_t *io_meta = nullptr;   // in_off, sa_idx, out_off (u32) + in_len, out_len (u16)
+    // profiling
+    bool prof = false;
+    ProfSet ring[PROF_RING];
+    int ring_next = 0;
+    uint32_t prof_batches = 0;
+    double prof_ms[MAX_KERNELS] = {};
+    int prof_nk = 0;
+};
+
+namespace {
+
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int dev)
+    {
+        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+        if (prev != dev) cudaSetDevice(dev);
+    }
+    ~DeviceGuard()
+    {
+        if (prev >= 0) cudaSetDevice(prev);
+    }
+};
+
+template <typename T>
+cudaError_t dalloc(nba_ipsec_sa_table *t, T **p, size_t count)
+{
+    void *q = nullptr;
+    cudaError_t e = cudaMalloc(&q, count * sizeof(T) + 256);
+    if (e != cudaSuccess) return e;
+    t->allocs.push_back(q);
+    *p = static_cast<T *>(q);
+    return cudaMemset(q, 0, count * sizeof(T) + 256);
+}
+
+void free_all(nba_ipsec_sa_table *t)
+{
+    for (void *p : t->allocs) cudaFree(p);
+    t->allocs.clear();
+    for (auto &s : t->ring)
+        for (int k = 0; k < MAX_KERNELS + 1; k++)
+            if (s.ev[k]) cudaEventDestroy(s.ev[k]);
+}
+
+const char *kernel_names_unfused[] = {"prologue", "gather", "aes_ctr", "hmac_sha1", "scatter"};
+const char *kernel_names_fused[] = {"prologue", "fused"};
+
+void prof_drain_set(nba_ipsec_sa_table *t, ProfSet &s)
+{
+    if (s.n_ev == 0) return;
+    cudaEventSynchronize(s.ev[s.n_ev - 1]);
+    for (int k = 0; k + 1 < s.n_ev; k++) {
+        float ms = 0.f;
+        if (cudaEventElapsedTime(&ms, s.ev[k], s.ev[k + 1]) == cudaSuccess) t->prof_ms[k] += ms;
+    }
+    t->prof_nk = s.n_ev - 1;
+    t->prof_batches++;
+    s.n_ev = 0;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char *nba_ipsec_strerror(int code)
+{
+    switch (code) {
+    case NBA_IPSEC_OK: return "ok";
+    case NBA_IPSEC_EINVAL: return "invalid argument";
+    case NBA_IPSEC_ENOMEM: return "out of device memory";
+    case NBA_IPSEC_ENODEV: return "no such CUDA device";
+    case NBA_IPSEC_ECUDA: return "CUDA launch or runtime error";
+    default: return "unknown error";
+    }
+}
+
+int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int cuda_device,
+                              uint32_t max_batch_pkts, nba_ipsec_sa_table **out)
+{
+    if (!out) return NBA_IPSEC_EINVAL;
+    *out = nullptr;
+    if (!sas || n_sa == 0 || n_sa > NBA_IPSEC_MAX_SA || max_batch_pkts == 0 ||
+        max_batch_pkts > NBA_IPSEC_MAX_BATCH)
+        return NBA_IPSEC_EINVAL;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || cuda_device < 0 || cuda_device >= ndev) {
+        cudaGetLastError();
+        return NBA_IPSEC_ENODEV;
+    }
+    DeviceGuard g(cuda_device);
+    auto *t = new (std::nothrow) nba_ipsec_sa_table();
+    if (!t) return NBA_IPSEC_ENOMEM;
+    t->device = cuda_device;
+    t->n_sa = n_sa;
+    t->max_batch = max_batch_pkts;
+    t->max_tiles = (max_batch_pkts + TILE - 1) / TILE;
+    cudaDeviceGetAttribute(&t->num_sms, cudaDevAttrMultiProcessorCount, cuda_device);
+    t->grid_aes = aes_grid(t->num_sms);
+    t->grid_fused = t->grid_aes;
+
+    // ---- a0: host-side key schedules, midstates, header words -------------
+    std::vector<uint4> rk((size_t)n_sa * 11), hm((size_t)n_sa * 3), hdr(n_sa);
+    std::vector<uint32_t> seq(n_sa);
+    for (uint32_t s = 0; s < n_sa; s++) {
+        const nba_ipsec_sa_params &p = sas[s];
+        uint8_t bytes[176];
+        aes128_schedule_bytes(p.aes_key, bytes);
+        std::memcpy(&rk[(size_t)s * 11], bytes, 176);
+        uint32_t hin[5], hout[5];
+        hmac_midstates(p.hmac_key, hin, hout);
+        hm[(size_t)s * 3 + 0] = make_uint4(hin[0], hin[1], hin[2], hin[3]);
+        hm[(size_t)s * 3 + 1] = make_uint4(hin[4], hout[0], hout[1], hout[2]);
+        hm[(size_t)s * 3 + 2] = make_uint4(hout[3], hout[4], 0u, 0u);
+        auto be_img = [](uint32_t v) {   // little-endian image of BE32(v)
+            return ((v >> 24) & 0xffu) | ((v >> 8) & 0xff00u) | ((v << 8) & 0xff0000u) |
+                   (v << 24);
+        };
+        uint32_t nonce;
+        std::memcpy(&nonce, p.ctr_nonce, 4);
+        hdr[s] = make_uint4(be_img(p.spi), nonce, be_img(p.tunnel_src), be_img(p.tunnel_dst));
+        seq[s] = p.seq;
+    }
+
+    uint4 *d_rk = nullptr, *d_hm = nullptr, *d_hdr = nullptr;
+    uint32_t *d_seq = nullptr, *d_seq_prev = nullptr, *d_te0 = nullptr;
+    const uint32_t M = max_batch_pkts;
+    cudaError_t e = cudaSuccess;
+    auto chk = [&](cudaError_t x) {
+        if (e == cudaSuccess && x != cudaSuccess) e = x;
+    };
+    chk(dalloc(t, &d_rk, rk.size()));
+    chk(dalloc(t, &d_hm, hm.size()));
+    chk(dalloc(t, &d_hdr, hdr.size()));
+    chk(dalloc(t, &d_seq, n_sa));
+    chk(dalloc(t, &d_seq_prev, n_sa));
+    chk(dalloc(t, &d_te0, 256));
+    DevWork &W = t->W;
+    chk(dalloc(t, &W.lrank, M));
+    chk(dalloc(t, &W.m_rec, M));
+    chk(dalloc(t, &W.m_blk, M + 1));
+    chk(dalloc(t, &W.m_seq, M));
+    chk(dalloc(t, &W.m_info, M));
+    chk(dalloc(t, &W.perm, M));
+    chk(dalloc(t, &W.hist, (size_t)t->max_tiles * n_sa));
+    chk(dalloc(t, &W.tile_rec, t->max_tiles));
+    chk(dalloc(t, &W.tile_blk, t->max_tiles));
+    chk(dalloc(t, &W.tile_bin, (size_t)t->max_tiles * NBINS));
+    chk(dalloc(t, &W.aes_start, (size_t)std::max(t->grid_aes, t->grid_fused)));
+    chk(dalloc(t, &W.ctl, 16));
+    chk(dalloc(t, &W.counters, 8));
+    chk(dalloc(t, &W.db, (size_t)M * (MAX_REC_BYTES / 16) + 16));
+    if (e == cudaSuccess) {
+        chk(cudaMemcpy(d_rk, rk.data(), rk.size() * sizeof(uint4), cudaMemcpyHostToDevice));
+        chk(cudaMemcpy(d_hm, hm.data(), hm.size() * sizeof(uint4), cudaMemcpyHostToDevice));
+        chk(cudaMemcpy(d_hdr, hdr.data(), hdr.size() * sizeof(uint4), cudaMemcpyHostToDevice));
+        chk(cudaMemcpy(d_seq, seq.data(), n_sa * sizeof(uint32_t), cudaMemcpyHostToDevice));
+        chk(cudaMemcpy(d_te0, host_te0(), 256 * sizeof(uint32_t), cudaMemcpyHostToDevice));
+    }
+    if (e == cudaSuccess) chk(setup_prologue_attributes(n_sa));
+    if (e == cudaSuccess) chk(setup_aes_attributes());
+    if (e == cudaSuccess) chk(cudaDeviceSynchronize());
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        free_all(t);
+        delete t;
+        return e == cudaErrorMemoryAllocation ? NBA_IPSEC_ENOMEM : NBA_IPSEC_ECUDA;
+    }
+    t->T = DevTable{d_rk, d_hm, d_hdr, d_seq, d_seq_prev, d_te0, n_sa};
+    *out = t;
+    return NBA_IPSEC_OK;
+}
+
+static int enqueue(nba_ipsec_sa_table *t, const BatchArgs &B, cudaStream_t st)
+{
+    const uint32_t n_tiles = (B.n + TILE - 1) / TILE;
+    ProfSet *ps = nullptr;
+    if (t->prof) {
+        ps = &t->ring[t->ring_next];
+        prof_drain_set(t, *ps);        // only blocks if the ring wrapped
+        t->ring_next = (t->ring_next + 1) % PROF_RING;
+        for (int k = 0; k < MAX_KERNELS + 1; k++)
+            if (!ps->ev[k]) cudaEventCreate(&ps->ev[k]);
+        ps->n_ev = 0;
+    }
+    auto mark = [&]() {
+        if (ps) cudaEventRecord(ps->ev[ps->n_ev++], st);
+    };
+    mark();
+    if (launch_prologue(t->T, t->W, B, n_tiles, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
+    mark();
+    if (launch_gather(t->T, t->W, B, n_tiles, (uint32_t)t->grid_aes, st) != cudaSuccess)
+        return NBA_IPSEC_ECUDA;
+    mark();
+    if (launch_aes(t->T, t->W, B, t->grid_aes, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
+    mark();
+    if (launch_hmac(t->T, t->W, B, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
+    mark();
+    if (launch_scatter(t->T, t->W, B, n_tiles, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
+    mark();
+    return NBA_IPSEC_OK;
+}
+
+int nba_ipsec_process_batch(nba_ipsec_sa_table *t, const nba_ipsec_batch *b, void *cuda_stream)
+{
+    if (!t || !b) return NBA_IPSEC_EINVAL;
+    if (b->n_pkts > t->max_batch) return NBA_IPSEC_EINVAL;
+    if (b->n_pkts == 0) return NBA_IPSEC_OK;
+    if (!b->in_buf || !b->in_off || !b->in_len || !b->sa_idx || !b->out_buf || !b->out_off ||
+        !b->out_len)
+        return NBA_IPSEC_EINVAL;
+    DeviceGuard g(t->device);
+    BatchArgs B{b->in_buf, b->in_off, b->in_len, b->sa_idx, b->out_buf, b->out_off, b->out_len,
+                b->n_pkts};
+    return enqueue(t, B, static_cast<cudaStream_t>(cuda_stream));
+}
+
+int nba_ipsec_reserve_host_io(nba_ipsec_sa_table *t, uint64_t in_buf_bytes, uint64_t out_buf_bytes)
+{
+    if (!t) return NBA_IPSEC_EINVAL;
+    DeviceGuard g(t->device);
+    if (in_buf_bytes > t->io_in_bytes) {
+        if (t->io_in) cudaFree(t->io_in);
+        t->io_in = nullptr;
+        if (cudaMalloc(&t->io_in, in_buf_bytes + 16) != cudaSuccess) {
+            cudaGetLastError();
+            t->io_in_bytes = 0;
+            return NBA_IPSEC_ENOMEM;
+        }
+        t->io_in_bytes = in_buf_bytes;
+    }
+    if (out_buf_bytes > t->io_out_bytes) {
+        if (t->io_out) cudaFree(t->io_out);
+        t->io_out = nullptr;
+        if (cudaMalloc(&t->io_out, out_buf_bytes + 16) != cudaSuccess) {
+            cudaGetLastError();
+            t->io_out_bytes = 0;
+            return NBA_IPSEC_ENOMEM;
+        }
+        t->io_out_bytes = out_buf_bytes;
+    }
+    if (!t->io_meta) {
+        // 3 u32 arrays + 2 u16 arrays of max_batch entries
+        size_t bytes = (size_t)t->max_batch * 16 + 64;
+        if (cudaMalloc(&t->io_meta, bytes) != cudaSuccess) {
+            cudaGetLastError();
+            return NBA_IPSEC_ENOMEM;
+        }
+    }
+    return NBA_IPSEC_OK;
+}
+
+int nba_ipsec_process_batch_host(nba_ipsec_sa_table *t, const nba_ipsec_batch *b,
+                                 uint64_t in_buf_bytes, uint64_t out_buf_bytes, void *cuda_stream)
+{
+    if (!t || !b) return NBA_IPSEC_EINVAL;
+    if (b->n_pkts > t->max_batch) return NBA_IPSEC_EINVAL;
+    if (b->n_pkts == 0) return NBA_IPSEC_OK;
+    if (!b->in_buf || !b->in_off || !b->in_len || !b->sa_idx || !b->out_buf || !b->out_off ||
+        !b->out_len)
+        return NBA_IPSEC_EINVAL;
+    if (!t->io_meta || in_buf_bytes > t->io_in_bytes || out_buf_bytes > t->io_out_bytes)
+        return NBA_IPSEC_EINVAL;
+    DeviceGuard g(t->device);
+    cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    const uint32_t n = b->n_pkts;
+    uint32_t *d_in_off = t->io_meta;
+    uint32_t *d_sa = d_in_off + t->max_batch;
+    uint32_t *d_out_off = d_sa + t->max_batch;
+    uint16_t *d_in_len = reinterpret_cast<uint16_t *>(d_out_off + t->max_batch);
+    uint16_t *d_out_len = d_in_len + t->max_batch;
+    cudaError_t e = cudaSuccess;
+    auto chk = [&](cudaError_t x) {
+        if (e == cudaSuccess && x != cudaSuccess) e = x;
+    };
+    chk(cudaMemcpyAsync(t->io_in, b->in_buf, in_buf_bytes, cudaMemcpyHostToDevice, st));
+    chk(cudaMemcpyAsync(d_in_off, b->in_off, n * 4ull, cudaMemcpyHostToDevice, st));
+    chk(cudaMemcpyAsync(d_sa, b->sa_idx, n * 4ull, cudaMemcpyHostToDevice, st));
+    chk(cudaMemcpyAsync(d_out_off, b->out_off, n * 4ull, cudaMemcpyHostToDevice, st));
+    chk(cudaMemcpyAsync(d_in_len, b->in_len, n * 2ull, cudaMemcpyHostToDevice, st));
+    if (e != cudaSuccess) return NBA_IPSEC_ECUDA;
+    BatchArgs B{t->io_in, d_in_off, d_in_len, d_sa, t->io_out, d_out_off, d_out_len, n};
+    int rc = enqueue(t, B, st);
+    if (rc != NBA_IPSEC_OK) return rc;
+    chk(cudaMemcpyAsync(b->out_buf, t->io_out, out_buf_bytes, cudaMemcpyDeviceToHost, st));
+    chk(cudaMemcpyAsync(b->out_len, d_out_len, n * 2ull, cudaMemcpyDeviceToHost, st));
+    return e == cudaSuccess ? NBA_IPSEC_OK : NBA_IPSEC_ECUDA;
+}
+
+int nba_ipsec_destroy(nba_ipsec_sa_table *t)
+{
+    if (!t) return NBA_IPSEC_OK;
+    {
+        DeviceGuard g(t->device);
+        cudaDeviceSynchronize();
+        free_all(t);
+        if (t->io_in) cudaFree(t->io_in);
+        if (t->io_out) cudaFree(t->io_out);
+        if (t->io_meta) cudaFree(t->io_meta);
+    }
+    delete t;
+    return NBA_IPSEC_OK;
+}
+
+int nba_ipsec_read_counters(nba_ipsec_sa_table *t, nba_ipsec_counters *out, void *cuda_stream)
+{
+    if (!t || !out) return NBA_IPSEC_EINVAL;
+    DeviceGuard g(t->device);
+    unsigned long long h[5];
+    cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    if (cudaMemcpyAsync(h, t->W.counters, sizeof(h), cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+        cudaStreamSynchronize(st) != cudaSuccess)
+        return NBA_IPSEC_ECUDA;
+    out->pkts_ok = h[0];
+    out->pkts_dropped = h[1];
+    out->bytes_in = h[2];
+    out->bytes_out = h[3];
+    out->batches = h[4];
+    return NBA_IPSEC_OK;
+}
+
+int nba_ipsec_read_sa_seq(nba_ipsec_sa_table *t, uint32_t *host_seq, void *cuda_stream)
+{
+    if (!t || !host_seq) return NBA_IPSEC_EINVAL;
+    DeviceGuard g(t->device);
+    cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    if (cudaMemcpyAsync(host_seq, t->T.seq, t->n_sa * sizeof(uint32_t), cudaMemcpyDeviceToHost,
+                        st) != cudaSuccess ||
+        cudaStreamSynchronize(st) != cudaSuccess)
+        return NBA_IPSEC_ECUDA;
+    return NBA_IPSEC_OK;
+}
+
+int nba_ipsec_set_pipeline(nba_ipsec_sa_table *t, int pipeline)
+{
+    if (!t) return NBA_IPSEC_EINVAL;
+    if (pipeline != NBA_IPSEC_PIPE_UNFUSED) return NBA_IPSEC_EINVAL;   // fused: not yet built
+    t->pipeline = pipeline;
+    return NBA_IPSEC_OK;
+}
+
+int nba_ipsec_launches_per_batch(nba_ipsec_sa_table *t)
+{
+    if (!t) return NBA_IPSEC_EINVAL;
+    return t->pipeline == NBA_IPSEC_PIPE_FUSED ? 2 : 5;
+}
+
+int nba_ipsec_profile_enable(nba_ipsec_sa_table *t, int enable)
+{
+    if (!t) return NBA_IPSEC_EINVAL;
+    DeviceGuard g(t->device);
+    for (auto &s : t->ring) s.n_ev = 0;
+    t->prof = enable != 0;
+    t->prof_batches = 0;
+    t->prof_nk = 0;
+    for (double &x : t->prof_ms) x = 0.0;
+    return NBA_IPSEC_OK;
+}
+
+int nba_ipsec_profile_read(nba_ipsec_sa_table *t, double *ms, const char **names, int max,
+                           int *n_kernels, uint32_t *n_batches)
+{
+    if (!t) return NBA_IPSEC_EINVAL;
+    DeviceGuard g(t->device);
+    for (int k = 0; k < PROF_RING; k++) prof_drain_set(t, t->ring[(t->ring_next + k) % PROF_RING]);
+    const char **nm = t->pipeline == NBA_IPSEC_PIPE_FUSED ? kernel_names_fused
+                                                          : kernel_names_unfused;
+    int nk = t->prof_nk;
+    for (int k = 0; k < nk && k < max; k++) {
+        if (ms) ms[k] = t->prof_ms[k];
+        if (names) names[k] = nm[k];
+    }
+    if (n_kernels) *n_kernels = nk;
+    if (n_batches) *n_batches = t->prof_batches;
+    return NBA_IPSEC_OK;
+}
+
+}  // extern "C"

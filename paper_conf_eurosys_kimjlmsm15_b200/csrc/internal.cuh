@@ -1,0 +1,205 @@
+// internal.cuh -- device-side data layout and helpers shared by the kernels
+// of libnba_ipsec.so (never by oracle/).  DESIGN.md §4 describes the layout.
+#pragma once
+#include <cstdint>
+
+#include <vector_types.h>
+
+#ifdef __CUDACC__
+#include <cuda_runtime.h>
+#endif
+
+namespace nba {
+
+constexpr uint32_t TILE = 1024;        // packets per prologue / gather / scatter tile
+constexpr uint32_t MIN_D = 20, MAX_D = 1500;
+constexpr uint32_t MAX_REC_BYTES = 1536;  // roundup16(28 + 1504)
+constexpr uint32_t INVALID_SA = 0xffffffffu;
+constexpr uint32_t INFO_OK = 0x80000000u;
+
+// --- setup-time host arithmetic (host_tables.cpp) -------------------------
+const uint32_t *host_te0();
+const uint8_t *host_sbox();
+void aes128_schedule_bytes(const uint8_t key[16], uint8_t rk[176]);
+void hmac_midstates(const uint8_t key[20], uint32_t hin[5], uint32_t hout[5]);
+
+// --- device SA table (a0) ---------------------------------------------------
+// All words are little-endian images of the wire bytes unless noted.
+struct DevTable {
+    const uint4 *rk;        // [n_sa * 11] AES-128 round keys (FIPS-197 byte order)
+    const uint4 *hmid;      // [n_sa * 3]  hin[0..4], hout[0..4] (SHA-1 words), 2 pad
+    const uint4 *sahdr;     // [n_sa] {BE(spi), nonce bytes, BE(tun_src), BE(tun_dst)}
+    uint32_t *seq;          // [n_sa] last sequence number used (mutable)
+    uint32_t *seq_prev;     // [n_sa] value of seq before the current batch
+    const uint32_t *te0;    // [256] T-table, row-0 byte in bits 0..7
+    uint32_t n_sa;
+};
+
+// --- per-batch workspace ----------------------------------------------------
+struct DevWork {
+    uint32_t *lrank;        // [M]   within-tile per-SA rank
+    uint32_t *m_rec;        // [M]   record offset in the datablock, 16-B units
+    uint32_t *m_blk;        // [M+1] exclusive prefix of AES blocks (+ total)
+    uint32_t *m_seq;        // [M]   ESP sequence number
+    uint32_t *m_info;       // [M]   C | tos << 16 | INFO_OK  (0 = dropped / invalid)
+    uint32_t *perm;         // [M]   HMAC processing order (length-binned)
+    uint32_t *hist;         // [max_tiles * n_sa] tile histogram -> exclusive prefix
+    uint32_t *tile_rec;     // [max_tiles] record chunks per tile -> exclusive prefix
+    uint32_t *tile_blk;     // [max_tiles] AES blocks per tile -> exclusive prefix
+    uint32_t *tile_bin;     // [max_tiles * NBINS] HMAC length bins per tile -> prefix
+    uint32_t *aes_start;    // [grid] first packet of each persistent AES / fused CTA
+    uint32_t *ctl;          // [16] ticket, total_rec16, total_blk, ...
+    unsigned long long *counters;  // [5] pkts_ok, pkts_dropped, bytes_in, bytes_out, batches
+    uint4 *db;              // datablock of ESP records (16-B aligned)
+};
+
+constexpr int CTL_TICKET = 0, CTL_TOTAL_REC = 1, CTL_TOTAL_BLK = 2, CTL_TICKET2 = 3;
+constexpr int NBINS = 32;   // HMAC bins by number of inner SHA-1 blocks (2..25)
+
+struct BatchArgs {
+    const uint8_t *in_buf;
+    const uint32_t *in_off;
+    const uint16_t *in_len;
+    const uint32_t *sa_idx;
+    uint8_t *out_buf;
+    const uint32_t *out_off;
+    uint16_t *out_len;
+    uint32_t n;
+};
+
+#ifdef __CUDACC__
+// --- launchers (one per kernel file) ----------------------------------------
+cudaError_t launch_prologue(const DevTable &T, const DevWork &W, const BatchArgs &B,
+                            uint32_t n_tiles, cudaStream_t st);
+cudaError_t launch_gather(const DevTable &T, const DevWork &W, const BatchArgs &B,
+                          uint32_t n_tiles, uint32_t aes_grid, cudaStream_t st);
+cudaError_t launch_aes(const DevTable &T, const DevWork &W, const BatchArgs &B, int grid,
+                       cudaStream_t st);
+cudaError_t launch_hmac(const DevTable &T, const DevWork &W, const BatchArgs &B,
+                        cudaStream_t st);
+cudaError_t launch_scatter(const DevTable &T, const DevWork &W, const BatchArgs &B,
+                           uint32_t n_tiles, cudaStream_t st);
+cudaError_t launch_fused(const DevTable &T, const DevWork &W, const BatchArgs &B, int grid,
+                         cudaStream_t st);
+cudaError_t setup_prologue_attributes(uint32_t n_sa);
+cudaError_t setup_aes_attributes();
+cudaError_t setup_fused_attributes();
+int aes_grid(int num_sms);
+int fused_grid(int num_sms);
+
+// --- small device helpers ---------------------------------------------------
+__device__ __forceinline__ uint32_t bswap32(uint32_t x) { return __byte_perm(x, 0, 0x0123); }
+
+__device__ __forceinline__ uint32_t lanemask_lt()
+{
+    uint32_t m;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+    return m;
+}
+
+// ESP sizes for an inner datagram of D bytes (A9):
+// p = (-(D+2)) mod 4, C = D + p + 2, AES blocks ceil(C/16), record roundup16(28+C).
+__device__ __forceinline__ uint32_t esp_pad(uint32_t D) { return (0u - (D + 2u)) & 3u; }
+__device__ __forceinline__ uint32_t esp_C(uint32_t D) { return D + esp_pad(D) + 2u; }
+__device__ __forceinline__ uint32_t esp_rec16(uint32_t C) { return (28u + C + 15u) >> 4; }
+__device__ __forceinline__ uint32_t esp_nblk(uint32_t C) { return (C + 15u) >> 4; }
+// inner SHA-1 blocks over (ipad block ||) SPI..trailer: message M = 16 + C bytes
+// after the 64-byte key block; padded length (M + 9) rounded up to 64.
+__device__ __forceinline__ uint32_t esp_nsha_inner(uint32_t C) { return (16u + C + 8u) / 64u + 1u; }
+// HMAC length bin: longest first; invalid packets last.
+__device__ __forceinline__ uint32_t hmac_bin(bool valid, uint32_t C)
+{
+    return valid ? (uint32_t)(NBINS - 1) - esp_nsha_inner(C) : (uint32_t)(NBINS - 1);
+}
+
+// 16 bytes starting at byte `sh` (0..15) of the 32-byte little-endian
+// concatenation lo || hi.
+__device__ __forceinline__ uint4 extract16(uint4 lo, uint4 hi, uint32_t sh)
+{
+    uint32_t q = sh >> 2, r = (sh & 3u) * 8u;
+    uint32_t a0, a1, a2, a3, a4;
+    switch (q) {
+    case 0: a0 = lo.x; a1 = lo.y; a2 = lo.z; a3 = lo.w; a4 = hi.x; break;
+    case 1: a0 = lo.y; a1 = lo.z; a2 = lo.w; a3 = hi.x; a4 = hi.y; break;
+    case 2: a0 = lo.z; a1 = lo.w; a2 = hi.x; a3 = hi.y; a4 = hi.z; break;
+    default: a0 = lo.w; a1 = hi.x; a2 = hi.y; a3 = hi.z; a4 = hi.w; break;
+    }
+    uint4 o;
+    o.x = __funnelshift_r(a0, a1, r);
+    o.y = __funnelshift_r(a1, a2, r);
+    o.z = __funnelshift_r(a2, a3, r);
+    o.w = __funnelshift_r(a3, a4, r);
+    return o;
+}
+
+__device__ __forceinline__ uint4 ldg_nc_v4(const void *p)
+{
+    uint4 v;
+    asm volatile("ld.global.nc.v4.u32 {%0,%1,%2,%3}, [%4];"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+                 : "l"(p));
+    return v;
+}
+
+__device__ __forceinline__ uint32_t get_byte(uint4 v, uint32_t j)
+{
+    uint32_t w = (j < 4) ? v.x : (j < 8) ? v.y : (j < 12) ? v.z : v.w;
+    return (w >> ((j & 3u) * 8u)) & 0xffu;
+}
+
+__device__ __forceinline__ void set_byte(uint4 &v, uint32_t j, uint32_t b)
+{
+    uint32_t sh = (j & 3u) * 8u;
+    uint32_t m = ~(0xffu << sh);
+    if (j < 4) v.x = (v.x & m) | (b << sh);
+    else if (j < 8) v.y = (v.y & m) | (b << sh);
+    else if (j < 12) v.z = (v.z & m) | (b << sh);
+    else v.w = (v.w & m) | (b << sh);
+}
+
+// Largest k in [0, n) with a[k] <= x, for non-decreasing a with a[0] <= x.
+__device__ __forceinline__ uint32_t upper_bound_m1(const uint32_t *a, uint32_t n, uint32_t x)
+{
+    uint32_t lo = 0, len = n;
+    while (len > 1) {
+        uint32_t half = len >> 1;
+        if (a[lo + half] <= x) lo += half;
+        len -= half;
+    }
+    return lo;
+}
+
+// Block-wide exclusive scan of one u32 per thread (blockDim.x == 1024 or a
+// multiple of 32 <= 1024).  `scratch` holds >= 32 u32.  Returns the exclusive
+// prefix; *total receives the block sum.  Contains __syncthreads.
+__device__ __forceinline__ uint32_t block_exclusive_scan(uint32_t v, uint32_t *scratch,
+                                                         uint32_t *total)
+{
+    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+    const uint32_t nw = blockDim.x >> 5;
+    uint32_t x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+        if (lane >= (uint32_t)o) x += y;
+    }
+    __syncthreads();
+    if (lane == 31) scratch[warp] = x;
+    __syncthreads();
+    if (warp == 0) {
+        uint32_t w = lane < nw ? scratch[lane] : 0u;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            uint32_t y = __shfl_up_sync(0xffffffffu, w, o);
+            if (lane >= (uint32_t)o) w += y;
+        }
+        scratch[lane] = w;   // inclusive warp-sum prefix
+    }
+    __syncthreads();
+    uint32_t base = warp ? scratch[warp - 1] : 0u;
+    *total = scratch[nw - 1];
+    return base + x - v;
+}
+#endif
+
+}  // namespace nba

@@ -1,0 +1,239 @@
+"""Thin ctypes binding of libnba_ipsec.so (include/nba_ipsec.h).
+
+Argument marshalling only: every step of the ESP path runs in the library's
+CUDA kernels.  PyTorch supplies device memory (tensors' data_ptr) and streams.
+There is no CPU fallback: if the library is missing, importing this module
+raises.  Names follow the C ABI (nba_ipsec_create_sa_table /
+nba_ipsec_process_batch / nba_ipsec_destroy ...).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import re
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libnba_ipsec.so")
+HEADER = os.path.join(os.path.dirname(_HERE), "include", "nba_ipsec.h")
+
+OK, EINVAL, ENOMEM, ENODEV, ECUDA = 0, -22, -12, -19, -1000
+PIPE_FUSED, PIPE_UNFUSED = 0, 1
+MIN_DATAGRAM, MAX_DATAGRAM, MAX_OVERHEAD = 20, 1500, 53
+
+
+class NbaIpsecError(RuntimeError):
+    def __init__(self, code, what):
+        super().__init__(f"{what}: {strerror(code)} ({code})")
+        self.code = code
+
+
+class SaParams(ctypes.Structure):
+    _fields_ = [("spi", ctypes.c_uint32), ("tunnel_src", ctypes.c_uint32),
+                ("tunnel_dst", ctypes.c_uint32), ("aes_key", ctypes.c_uint8 * 16),
+                ("ctr_nonce", ctypes.c_uint8 * 4), ("hmac_key", ctypes.c_uint8 * 20),
+                ("seq", ctypes.c_uint32)]
+
+
+class Batch(ctypes.Structure):
+    _fields_ = [("in_buf", ctypes.c_void_p), ("in_off", ctypes.c_void_p),
+                ("in_len", ctypes.c_void_p), ("sa_idx", ctypes.c_void_p),
+                ("out_buf", ctypes.c_void_p), ("out_off", ctypes.c_void_p),
+                ("out_len", ctypes.c_void_p), ("n_pkts", ctypes.c_uint32)]
+
+
+class Counters(ctypes.Structure):
+    _fields_ = [("pkts_ok", ctypes.c_uint64), ("pkts_dropped", ctypes.c_uint64),
+                ("bytes_in", ctypes.c_uint64), ("bytes_out", ctypes.c_uint64),
+                ("batches", ctypes.c_uint64)]
+
+    def as_dict(self):
+        return {k: int(getattr(self, k)) for k, _ in self._fields_}
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: run `python -m "
+                          "paper_conf_eurosys_kimjlmsm15_b200.build` (no CPU fallback exists)")
+    L = ctypes.CDLL(LIB_PATH)
+    P = ctypes.POINTER
+    vp, i32, u32, u64 = ctypes.c_void_p, ctypes.c_int, ctypes.c_uint32, ctypes.c_uint64
+    sig = {
+        "nba_ipsec_create_sa_table": (i32, [P(SaParams), u32, i32, u32, P(vp)]),
+        "nba_ipsec_process_batch": (i32, [vp, P(Batch), vp]),
+        "nba_ipsec_process_batch_host": (i32, [vp, P(Batch), u64, u64, vp]),
+        "nba_ipsec_reserve_host_io": (i32, [vp, u64, u64]),
+        "nba_ipsec_destroy": (i32, [vp]),
+        "nba_ipsec_read_counters": (i32, [vp, P(Counters), vp]),
+        "nba_ipsec_read_sa_seq": (i32, [vp, P(u32), vp]),
+        "nba_ipsec_strerror": (ctypes.c_char_p, [i32]),
+        "nba_ipsec_set_pipeline": (i32, [vp, i32]),
+        "nba_ipsec_launches_per_batch": (i32, [vp]),
+        "nba_ipsec_profile_enable": (i32, [vp, i32]),
+        "nba_ipsec_profile_read": (i32, [vp, P(ctypes.c_double), P(ctypes.c_char_p), i32,
+                                         P(i32), P(u32)]),
+        "nba_ipsec_host_aes128_key_schedule": (None, [P(ctypes.c_uint8), P(u32)]),
+        "nba_ipsec_host_hmac_sha1_midstates": (None, [P(ctypes.c_uint8), P(u32), P(u32)]),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(L, name)
+        f.restype = res
+        f.argtypes = args
+    return L
+
+
+lib = _load()
+
+
+def header_functions() -> list[str]:
+    """Function names declared in include/nba_ipsec.h."""
+    txt = open(HEADER).read()
+    return sorted(set(re.findall(r"\b(nba_ipsec_[a-z0-9_]+)\s*\(", txt)))
+
+
+def strerror(code: int) -> str:
+    return lib.nba_ipsec_strerror(int(code)).decode()
+
+
+def _check(rc, what):
+    if rc != OK:
+        raise NbaIpsecError(rc, what)
+
+
+def make_params(p) -> "ctypes.Array":
+    """gen.SAParams (numpy SoA) -> nba_ipsec_sa_params[n]."""
+    n = len(p.spi)
+    arr = (SaParams * max(n, 1))()
+    for s in range(n):
+        e = arr[s]
+        e.spi = int(p.spi[s])
+        e.tunnel_src = int(p.tunnel_src[s])
+        e.tunnel_dst = int(p.tunnel_dst[s])
+        ctypes.memmove(e.aes_key, np.ascontiguousarray(p.aes_key[s], np.uint8).ctypes.data, 16)
+        ctypes.memmove(e.ctr_nonce, np.ascontiguousarray(p.ctr_nonce[s], np.uint8).ctypes.data, 4)
+        ctypes.memmove(e.hmac_key, np.ascontiguousarray(p.hmac_key[s], np.uint8).ctypes.data, 20)
+        e.seq = int(p.seq[s])
+    return arr
+
+
+def _stream_handle(stream):
+    if stream is None:
+        import torch
+        stream = torch.cuda.current_stream()
+    if isinstance(stream, int):
+        return stream
+    return int(stream.cuda_stream)
+
+
+def _ptr(x):
+    if x is None:
+        return None
+    if hasattr(x, "data_ptr"):
+        return x.data_ptr()
+    if isinstance(x, np.ndarray):
+        return x.ctypes.data
+    return int(x)
+
+
+class SATable:
+    """nba_ipsec_sa_table: per-device SA state + workspace."""
+
+    def __init__(self, params, device: int = 0, max_batch: int = 65536):
+        arr = params if isinstance(params, ctypes.Array) else make_params(params)
+        self.n_sa = len(params.spi) if not isinstance(params, ctypes.Array) else len(arr)
+        self.device = device
+        self.max_batch = max_batch
+        h = ctypes.c_void_p()
+        _check(lib.nba_ipsec_create_sa_table(arr, self.n_sa, device, max_batch, ctypes.byref(h)),
+               "nba_ipsec_create_sa_table")
+        self._h = h
+
+    # -- hot path ------------------------------------------------------------
+    def process(self, in_buf, in_off, in_len, sa_idx, out_buf, out_off, out_len, n=None,
+                stream=None):
+        """nba_ipsec_process_batch on device tensors (uint8 / int32 / int16 views)."""
+        n = int(in_len.numel() if n is None else n)
+        b = Batch(_ptr(in_buf), _ptr(in_off), _ptr(in_len), _ptr(sa_idx), _ptr(out_buf),
+                  _ptr(out_off), _ptr(out_len), n)
+        _check(lib.nba_ipsec_process_batch(self._h, ctypes.byref(b), _stream_handle(stream)),
+               "nba_ipsec_process_batch")
+
+    def reserve_host_io(self, in_bytes: int, out_bytes: int):
+        _check(lib.nba_ipsec_reserve_host_io(self._h, in_bytes, out_bytes),
+               "nba_ipsec_reserve_host_io")
+
+    def process_host(self, in_buf, in_off, in_len, sa_idx, out_buf, out_off, out_len,
+                     in_bytes, out_bytes, n=None, stream=None):
+        """nba_ipsec_process_batch_host on host (pinned) buffers."""
+        n = int(len(in_len) if n is None else n)
+        b = Batch(_ptr(in_buf), _ptr(in_off), _ptr(in_len), _ptr(sa_idx), _ptr(out_buf),
+                  _ptr(out_off), _ptr(out_len), n)
+        _check(lib.nba_ipsec_process_batch_host(self._h, ctypes.byref(b), int(in_bytes),
+                                                int(out_bytes), _stream_handle(stream)),
+               "nba_ipsec_process_batch_host")
+
+    # -- auxiliary -------------------------------------------------------------
+    def counters(self, stream=None) -> dict:
+        c = Counters()
+        _check(lib.nba_ipsec_read_counters(self._h, ctypes.byref(c), _stream_handle(stream)),
+               "nba_ipsec_read_counters")
+        return c.as_dict()
+
+    def sa_seq(self, stream=None) -> np.ndarray:
+        out = np.zeros(self.n_sa, np.uint32)
+        _check(lib.nba_ipsec_read_sa_seq(self._h, out.ctypes.data_as(ctypes.POINTER(ctypes.c_uint32)),
+                                         _stream_handle(stream)), "nba_ipsec_read_sa_seq")
+        return out
+
+    def set_pipeline(self, pipeline: int):
+        _check(lib.nba_ipsec_set_pipeline(self._h, int(pipeline)), "nba_ipsec_set_pipeline")
+
+    def launches_per_batch(self) -> int:
+        return int(lib.nba_ipsec_launches_per_batch(self._h))
+
+    def profile_enable(self, on: bool = True):
+        _check(lib.nba_ipsec_profile_enable(self._h, 1 if on else 0), "nba_ipsec_profile_enable")
+
+    def profile_read(self) -> tuple[dict, int]:
+        ms = (ctypes.c_double * 8)()
+        names = (ctypes.c_char_p * 8)()
+        nk, nb = ctypes.c_int(0), ctypes.c_uint32(0)
+        _check(lib.nba_ipsec_profile_read(self._h, ms, names, 8, ctypes.byref(nk),
+                                          ctypes.byref(nb)), "nba_ipsec_profile_read")
+        return {names[k].decode(): ms[k] for k in range(nk.value)}, int(nb.value)
+
+    def close(self):
+        if getattr(self, "_h", None) is not None and self._h.value:
+            _check(lib.nba_ipsec_destroy(self._h), "nba_ipsec_destroy")
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+
+# -- host-only setup helpers (tests of the library's own a0 arithmetic) ---------
+def host_aes128_key_schedule(key: bytes) -> np.ndarray:
+    k = np.frombuffer(bytes(key), np.uint8).copy()
+    w = np.zeros(44, np.uint32)
+    lib.nba_ipsec_host_aes128_key_schedule(k.ctypes.data_as(ctypes.POINTER(ctypes.c_uint8)),
+                                           w.ctypes.data_as(ctypes.POINTER(ctypes.c_uint32)))
+    return w
+
+
+def host_hmac_sha1_midstates(key: bytes):
+    k = np.frombuffer(bytes(key), np.uint8).copy()
+    hin, hout = np.zeros(5, np.uint32), np.zeros(5, np.uint32)
+    u32p = ctypes.POINTER(ctypes.c_uint32)
+    lib.nba_ipsec_host_hmac_sha1_midstates(k.ctypes.data_as(ctypes.POINTER(ctypes.c_uint8)),
+                                           hin.ctypes.data_as(u32p), hout.ctypes.data_as(u32p))
+    return hin, hout
