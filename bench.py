@@ -1,0 +1,492 @@
+#!/usr/bin/env python
+"""Benchmark: IPsec ESP outbound throughput (Gbps, Mpps) on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config 2|3|4] [--impl ours|reference]
+    python -m torch.distributed.run --nproc-per-node N --master-addr 127.0.0.1 bench.py --gpus N
+
+One step = one batch of 65,536 packets per GPU through the whole hot path
+(prologue, gather+ESP encapsulation, AES-128-CTR, HMAC-SHA1-96, scatter) via
+the C ABI (nba_ipsec_process_batch), inputs resident in HBM.  Default workload
+is BASELINE.json configs[1] (64 B frames, 1024 SAs); configs[2] (1514 B) and
+configs[3] (IMIX) are measured too and reported under "per_size".  Multi-GPU:
+SA-hash sharding (GPU g owns SAs s = g mod N), weak scaling, no data-path
+collective; NCCL only reduces counters and takes the max elapsed time.
+
+Gbps = 8 * sum(frame bytes L) / t (reading A18, frames excluding FCS);
+Mpps = packets / t.  L2 is flushed (256 MiB write) before every timed step and
+each step is timed with CUDA events on the launching stream.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+from paper_conf_eurosys_kimjlmsm15_b200 import gen, shard  # noqa: E402
+
+METRIC = "IPsec ESP throughput Gbps & Mpps per packet size at 1/2/4/8 B200; % roofline"
+N_SA_TOTAL = 1024
+PKTS_PER_GPU = 65536
+CFG_SIZE = {2: 64, 3: 1514, 4: "imix"}
+SM_COUNT = 148
+
+
+# --------------------------------------------------------------------------- utils
+def load_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return {"hbm_gbs": float(d["hbm_gbs"]), "sm_max_mhz": float(d.get("sm_max_mhz", 1965.0)),
+                "source": "measured (MEASURED_PEAKS.json)"}
+    except Exception:
+        return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0,
+                "source": "fallback (B200_PROFILING.md)"}
+
+
+class ClockSampler:
+    """Samples SM clock + throttle reasons with NVML during the timed region."""
+
+    def __init__(self, gpu_index: int, period_s: float = 0.002):
+        self.idx, self.period = gpu_index, period_s
+        self.samples, self.reasons = [], set()
+        self._stop = threading.Event()
+        self.max_mhz = None
+        self._t = None
+
+    def __enter__(self):
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            h = pynvml.nvmlDeviceGetHandleByIndex(self.idx)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(h, pynvml.NVML_CLOCK_SM)
+            names = {
+                "hw_slowdown": getattr(pynvml, "nvmlClocksEventReasonHwSlowdown", 0x8),
+                "hw_thermal_slowdown": getattr(pynvml, "nvmlClocksEventReasonHwThermalSlowdown", 0x40),
+                "sw_thermal_slowdown": getattr(pynvml, "nvmlClocksEventReasonSwThermalSlowdown", 0x20),
+                "sw_power_cap": getattr(pynvml, "nvmlClocksEventReasonSwPowerCap", 0x4),
+                "hw_power_brake_slowdown": getattr(pynvml, "nvmlClocksEventReasonHwPowerBrakeSlowdown", 0x80),
+            }
+
+            def run():
+                while not self._stop.is_set():
+                    try:
+                        self.samples.append(pynvml.nvmlDeviceGetClockInfo(h, pynvml.NVML_CLOCK_SM))
+                        r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(h)
+                        for k, bit in names.items():
+                            if r & bit:
+                                self.reasons.add(k)
+                    except Exception:
+                        pass
+                    time.sleep(self.period)
+
+            self._t = threading.Thread(target=run, daemon=True)
+            self._t.start()
+        except Exception as e:  # NVML unavailable: record why
+            self.reasons.add(f"nvml_unavailable:{type(e).__name__}")
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join()
+
+    def summary(self):
+        return {"sm_mhz": float(statistics.median(self.samples)) if self.samples else None,
+                "sm_max_mhz": float(self.max_mhz) if self.max_mhz else None,
+                "samples": len(self.samples), "reasons": sorted(self.reasons)}
+
+
+def frame_bits(b):
+    return 8.0 * float(np.asarray(b.frame_len, np.float64).sum())
+
+
+def work_model(b):
+    """Algorithmic work of one batch: per valid packet
+    AES blocks ceil(C/16), SHA-1 compressions (inner ceil((C+25)/64) + outer 1,
+    the ipad/opad blocks are precomputed), bytes read D and written 48+C."""
+    D = b.in_len.astype(np.int64)
+    ok = (D >= 20) & (D <= 1500) & (b.sa_idx < 2**31)
+    D = D[ok]
+    C = D + ((-(D + 2)) % 4) + 2
+    return {
+        "packets": int(ok.sum()),
+        "aes_blocks": int(((C + 15) // 16).sum()),
+        "sha1_compressions": int(((16 + C + 8) // 64 + 1 + 1).sum()),
+        "bytes_in": int(D.sum()),
+        "bytes_out": int((48 + C).sum()),
+        "rec_bytes": int((((28 + C + 15) // 16) * 16).sum()),
+    }
+
+
+# Per-kernel roofline model.  Integer-pipe peaks from the
+# microarchitecture guide's unit counts at the max SM clock: shared-memory
+# LSU 32 x 4-B lookups/clk/SM; ALU pipe (LOP3/SHF/IADD3) 64 lanes/clk/SM.
+AES_LOOKUPS_PER_BLOCK = 160
+SHA1_OPS_PER_COMPRESSION = 597
+
+
+def kernel_roofline(name, ms_per_launch, w, peaks):
+    f = peaks["sm_max_mhz"] * 1e6
+    s = ms_per_launch * 1e-3
+    if name in ("aes_ctr",):
+        achieved = w["aes_blocks"] * AES_LOOKUPS_PER_BLOCK / s / 1e9
+        peak = SM_COUNT * 32 * f / 1e9
+        return {"bound": "alu", "unit": "Glookup/s", "achieved": achieved, "peak": peak,
+                "peak_basis": "shared-memory LSU: 32 x 4-B T-table lookups/clk/SM x 148 SMs x "
+                              f"{peaks['sm_max_mhz']:.0f} MHz (160 lookups per AES block)"}
+    if name in ("hmac_sha1",):
+        achieved = w["sha1_compressions"] * SHA1_OPS_PER_COMPRESSION / s / 1e9
+        peak = SM_COUNT * 64 * f / 1e9
+        return {"bound": "alu", "unit": "Gop/s", "achieved": achieved, "peak": peak,
+                "peak_basis": "ALU pipe: 64 int32 lanes/clk/SM x 148 SMs x "
+                              f"{peaks['sm_max_mhz']:.0f} MHz (597 ops per SHA-1 compression)"}
+    if name == "fused":
+        # lower bound = max(LSU time of AES, ALU time of SHA-1 + AES ALU share, HBM time)
+        t_lsu = w["aes_blocks"] * AES_LOOKUPS_PER_BLOCK / (SM_COUNT * 32 * f)
+        t_alu = w["sha1_compressions"] * SHA1_OPS_PER_COMPRESSION / (SM_COUNT * 64 * f)
+        t_hbm = (w["bytes_in"] + w["bytes_out"]) / (peaks["hbm_gbs"] * 1e9)
+        t_lb = max(t_lsu, t_alu, t_hbm)
+        return {"bound": "alu", "unit": "fraction-of-lower-bound", "achieved": t_lb / s,
+                "peak": 1.0,
+                "peak_basis": "max(AES LSU time, SHA-1 ALU time, HBM time) at max SM clock"}
+    # memory-bound kernels: algorithmic bytes
+    if name == "gather":
+        byts = w["bytes_in"] + w["rec_bytes"]
+    elif name == "scatter":
+        byts = (w["rec_bytes"]) + w["bytes_out"]
+    else:  # prologue: read sa_idx + in_len, write rank
+        byts = w["packets"] * 10
+    return {"bound": "hbm", "unit": "GB/s", "achieved": byts / s / 1e9, "peak": peaks["hbm_gbs"],
+            "peak_basis": "measured HBM copy bandwidth"}
+
+
+def load_traffic(kernel):
+    """dram bytes per launch of `kernel` from the committed ncu summary, if any."""
+    p = os.path.join(ROOT, "profiles", "ncu_kernels.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return d.get(kernel, {}).get("dram_bytes_per_launch")
+    except Exception:
+        return None
+
+
+# --------------------------------------------------------------------------- ours
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    peaks = load_peaks()
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+
+    def barrier():
+        if world > 1:
+            dist.barrier(device_ids=[local])
+
+    def measure(cfg_id, steps, warmup, profile=True):
+        size = CFG_SIZE[cfg_id]
+        p, b = shard.rank_workload(cfg_id, PKTS_PER_GPU, size, N_SA_TOTAL, rank, world)
+        t = nba_ipsec.SATable(p, device=local, max_batch=PKTS_PER_GPU)
+        if args.pipeline is not None:
+            t.set_pipeline(args.pipeline)
+        db = device.to_device(b, dev)
+        run = lambda: t.process(*db.args(), n=b.n)  # noqa: E731
+        for _ in range(warmup):
+            flush.zero_()
+            run()
+        torch.cuda.synchronize()
+        t_end = time.time() + 0.3          # settle clocks: >= 0.3 s of back-to-back work
+        while time.time() < t_end:
+            for _ in range(20):
+                run()
+            torch.cuda.synchronize()
+        torch.cuda.synchronize()
+        barrier()
+        if profile:
+            t.profile_enable(True)
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+              for _ in range(steps)]
+        with ClockSampler(local) as clk:
+            torch.cuda.synchronize()
+            for k in range(steps):
+                flush.zero_()
+                ev[k][0].record()
+                run()
+                ev[k][1].record()
+            torch.cuda.synchronize()
+        barrier()
+        step_ms = [a.elapsed_time(c) for a, c in ev]
+        tot_ms = float(sum(step_ms))
+        kern, nb = t.profile_read() if profile else ({}, 0)
+        t.profile_enable(False)
+        launches = t.launches_per_batch() * steps
+        ctr = t.counters()
+        t.close()
+        return dict(b=b, p=p, tot_ms=tot_ms, step_ms=step_ms, kern=kern, nb=nb, clk=clk,
+                    launches=launches, ctr=ctr)
+
+    def aggregate(res, steps):
+        tot_ms_max = shard.max_over_ranks(res["tot_ms"], device=dev)
+        bits = shard.reduce_counters({"pkts_ok": frame_bits(res["b"]) / 8.0, "pkts_dropped": 0,
+                                      "bytes_in": res["b"].n, "bytes_out": 0, "batches": 0},
+                                     device=dev)
+        frame_bytes_all, pkts_all = bits["pkts_ok"], bits["bytes_in"]
+        s = tot_ms_max * 1e-3
+        return {"gbps": 8.0 * frame_bytes_all * steps / s / 1e9,
+                "mpps": pkts_all * steps / s / 1e6,
+                "ms_per_step": tot_ms_max / steps}
+
+    main_cfg = args.config
+    res = measure(main_cfg, args.steps, args.warmup)
+    agg = aggregate(res, args.steps)
+
+    # per-kernel breakdown and roofline of the dominant kernel (this rank)
+    w = work_model(res["b"])
+    kern_avg = {k: v / max(res["nb"], 1) for k, v in res["kern"].items()}
+    dom = max(kern_avg, key=kern_avg.get) if kern_avg else None
+    roof = None
+    kern_roofs = {}
+    for k, ms in kern_avg.items():
+        r = kernel_roofline(k, ms, w, peaks)
+        r["frac"] = r["achieved"] / r["peak"]
+        r["ms_per_launch"] = ms
+        kern_roofs[k] = r
+    if dom:
+        r = kern_roofs[dom]
+        roof = {"kernel": dom, "bound": r["bound"], "achieved": r["achieved"], "peak": r["peak"],
+                "unit": r["unit"], "frac": r["frac"], "traffic": load_traffic(dom),
+                "peak_basis": r["peak_basis"], "peak_source": peaks["source"],
+                "share_of_step": kern_avg[dom] / max(sum(kern_avg.values()), 1e-12)}
+
+    # ---- e2e: host buffers through nba_ipsec_process_batch_host ---------------
+    e2e = run_e2e(args, rank, world, local, dev, barrier)
+
+    # ---- other packet sizes (same protocol, fewer steps) ------------------------
+    per_size = {}
+    if not args.no_sweep:
+        for cfg_id in (2, 3, 4):
+            if cfg_id == main_cfg:
+                per_size[str(CFG_SIZE[cfg_id])] = {"gbps": agg["gbps"], "mpps": agg["mpps"],
+                                                   "ms_per_step": agg["ms_per_step"]}
+                continue
+            r2 = measure(cfg_id, max(10, args.steps // 2), max(3, args.warmup // 2))
+            a2 = aggregate(r2, max(10, args.steps // 2))
+            kk = {k: v / max(r2["nb"], 1) for k, v in r2["kern"].items()}
+            w2 = work_model(r2["b"])
+            rr = {}
+            for k, ms in kk.items():
+                x = kernel_roofline(k, ms, w2, peaks)
+                rr[k] = {"ms": ms, "frac": x["achieved"] / x["peak"], "unit": x["unit"]}
+            per_size[str(CFG_SIZE[cfg_id])] = {"gbps": a2["gbps"], "mpps": a2["mpps"],
+                                               "ms_per_step": a2["ms_per_step"], "kernels": rr}
+
+    # ---- CPU baseline: the oracle on host cores (rank 0, N = 1 only) ----------
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cpu = cpu_baseline(res["p"], res["b"], budget_s=args.cpu_seconds,
+                           label=gen.CONFIGS[main_cfg]["name"])
+
+    ctr_all = shard.reduce_counters(res["ctr"], device=dev)
+    if rank == 0:
+        clk = res["clk"].summary()
+        out = {
+            "metric": METRIC,
+            "value": agg["gbps"],
+            "unit": "Gbps",
+            "mpps": agg["mpps"],
+            "n_gpus": world,
+            "steps": args.steps,
+            "warmup": args.warmup,
+            "ms_per_step": agg["ms_per_step"],
+            "higher_is_better": True,
+            "scaling": "weak",
+            "vs_baseline": None,
+            "dtype": "u8",
+            "data": "synthetic (seeded random IPv4/UDP, random SA keys; PAPER.md:395 workload shape)",
+            "config": {"workload": f"configs[{main_cfg - 1}]: {gen.CONFIGS[main_cfg]['name']}",
+                       "frame_bytes": CFG_SIZE[main_cfg], "packets_per_gpu": PKTS_PER_GPU,
+                       "n_sa_total": N_SA_TOTAL, "global_batch": PKTS_PER_GPU * world,
+                       "parallelism": f"sa-hash shard x{world} (no data-path collective)",
+                       "l2": "flushed before every timed step (256 MiB device write, untimed)",
+                       "timing": "CUDA events per step on the launching stream, sum over steps, max over ranks",
+                       "pipeline": "fused" if args.pipeline in (None, 0) and res["launches"] // args.steps == 2 else "unfused"},
+            "roofline": roof,
+            "kernels": {k: {"ms_per_launch": v["ms_per_launch"], "frac": v["frac"], "unit": v["unit"],
+                            "achieved": v["achieved"]} for k, v in kern_roofs.items()},
+            "work_per_step_per_gpu": w,
+            "per_size": per_size,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": res["launches"],
+            "counters": ctr_all,
+            "clocks": clk,
+        }
+        print(json.dumps(out), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def run_e2e(args, rank, world, local, dev, barrier):
+    """Same metric through nba_ipsec_process_batch_host: every step copies the
+    step's inputs from pinned host memory and reads back the results."""
+    import torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import nba_ipsec
+    size = CFG_SIZE[args.config]
+    p, b = shard.rank_workload(args.config, PKTS_PER_GPU, size, N_SA_TOTAL, rank, world,
+                               layout="packed")
+    t = nba_ipsec.SATable(p, device=local, max_batch=PKTS_PER_GPU)
+    if args.pipeline is not None:
+        t.set_pipeline(args.pipeline)
+    in_bytes = int(b.in_off[-1]) + int(b.in_len[-1])
+    out_bytes = int(b.out_pool_bytes)
+    t.reserve_host_io(in_bytes, out_bytes)
+    pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()  # noqa: E731
+    h_in = pin(b.in_buf)
+    h_off, h_len, h_sa = pin(b.in_off.view(np.int32)), pin(b.in_len.view(np.int16)), pin(b.sa_idx.view(np.int32))
+    h_ooff = pin(b.out_off.view(np.int32))
+    h_out = torch.empty(out_bytes, dtype=torch.uint8).pin_memory()
+    h_olen = torch.empty(b.n, dtype=torch.int16).pin_memory()
+    st = torch.cuda.current_stream(dev)
+
+    def step():
+        t.process_host(h_in, h_off, h_len, h_sa, h_out, h_ooff, h_olen, in_bytes, out_bytes,
+                       n=b.n, stream=st)
+
+    for _ in range(max(3, args.warmup)):
+        step()
+    torch.cuda.synchronize()
+    barrier()
+    steps = max(5, args.steps // 2)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(steps):
+        step()
+    e1.record()
+    torch.cuda.synchronize()
+    barrier()
+    ms = shard.max_over_ranks(e0.elapsed_time(e1), device=dev)
+    tot = shard.reduce_counters({"pkts_ok": frame_bits(b) / 8.0, "pkts_dropped": 0, "bytes_in": b.n,
+                                 "bytes_out": 0, "batches": 0}, device=dev)
+    t.close()
+    h2d = in_bytes + b.n * (4 + 2 + 4 + 4)
+    d2h = out_bytes + b.n * 2
+    return {"value": 8.0 * tot["pkts_ok"] * steps / (ms * 1e-3) / 1e9, "unit": "Gbps",
+            "mpps": tot["bytes_in"] * steps / (ms * 1e-3) / 1e6,
+            "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
+            "steps": steps, "ms_per_step": ms / steps,
+            "note": "nba_ipsec_process_batch_host: pinned H2D of packed datagrams + metadata, "
+                    "kernels, D2H of output pool + out_len, one stream, no overlap across steps"}
+
+
+def cpu_baseline(p, b, budget_s=3.0, threads=None, label=""):
+    """The oracle as it stands (plain C, -O2) on the host's cores: full batches
+    repeated until `budget_s` of wall time, SAs partitioned s mod T over T threads."""
+    import oracle
+    T = threads or len(os.sched_getaffinity(0))
+    sas = oracle.make_sas(p)
+    n_sa = len(p.spi)
+    out = np.zeros(b.out_pool_bytes, np.uint8)
+    t0 = time.perf_counter()
+    reps = 0
+    while True:
+        oracle.process_batch(sas, n_sa, b, n_threads=T, out_buf=out)
+        reps += 1
+        el = time.perf_counter() - t0
+        if el >= budget_s:
+            break
+    gbps = frame_bits(b) * reps / el / 1e9
+    return {"value": gbps, "unit": "Gbps", "mpps": b.n * reps / el / 1e6, "cores": T,
+            "kind": "oracle",
+            "sample": f"{reps} full batch(es) of {b.n} packets ({label}, the benchmarked batch), "
+                      f"{el:.2f} s wall on {T} threads (~{el * T:.0f} CPU-s)"}
+
+
+# --------------------------------------------------------------------------- reference arm
+def run_reference(args):
+    """The oracle (this tier's reference arm) on the host cores, same metric and
+    config as our arm.  Under torchrun only rank 0 works; others exit 0."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import oracle
+    size = CFG_SIZE[args.config]
+    p, b = shard.rank_workload(args.config, PKTS_PER_GPU, size, N_SA_TOTAL, 0, 1)
+    T = len(os.sched_getaffinity(0))
+    sas = oracle.make_sas(p)
+    out = np.zeros(b.out_pool_bytes, np.uint8)
+    # bounded sample per step: as many packets as ~0.5 s of all-core work
+    probe = min(b.n, 4096)
+    sub = gen.Batch(n=probe, in_buf=b.in_buf, in_off=b.in_off[:probe], in_len=b.in_len[:probe],
+                    sa_idx=b.sa_idx[:probe], out_off=b.out_off[:probe],
+                    out_pool_bytes=b.out_pool_bytes, frame_len=b.frame_len[:probe])
+    t0 = time.perf_counter()
+    oracle.process_batch(sas, len(p.spi), sub, n_threads=T, out_buf=out)
+    per_pkt = (time.perf_counter() - t0) / probe
+    m = int(max(1024, min(b.n, 0.5 / max(per_pkt, 1e-9))))
+    sb = gen.Batch(n=m, in_buf=b.in_buf, in_off=b.in_off[:m], in_len=b.in_len[:m],
+                   sa_idx=b.sa_idx[:m], out_off=b.out_off[:m], out_pool_bytes=b.out_pool_bytes,
+                   frame_len=b.frame_len[:m])
+    for _ in range(args.warmup):
+        oracle.process_batch(sas, len(p.spi), sb, n_threads=T, out_buf=out)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle.process_batch(sas, len(p.spi), sb, n_threads=T, out_buf=out)
+    el = time.perf_counter() - t0
+    gbps = frame_bits(sb) * args.steps / el / 1e9
+    line = {
+        "impl": "reference",
+        "metric": METRIC, "value": gbps, "unit": "Gbps", "mpps": m * args.steps / el / 1e6,
+        "n_gpus": int(os.environ.get("WORLD_SIZE", "1")), "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": el * 1e3 / args.steps, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+        "config": {"workload": f"configs[{args.config - 1}]: {gen.CONFIGS[args.config]['name']}",
+                   "frame_bytes": CFG_SIZE[args.config], "packets_per_gpu": PKTS_PER_GPU,
+                   "n_sa_total": N_SA_TOTAL},
+        "cpu_baseline": {"value": gbps, "unit": "Gbps", "cores": T, "kind": "oracle",
+                         "sample": f"first {m} packets of the {b.n}-packet batch per step "
+                                   f"(~0.5 s all-core work), {args.steps} steps"},
+        "e2e": {"value": gbps, "unit": "Gbps", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--config", type=int, default=2, choices=[2, 3, 4])
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--pipeline", type=int, default=None, help="0 fused, 1 unfused")
+    ap.add_argument("--no-sweep", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=3.0)
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -150,6 +150,13 @@ int nba_ipsec_profile_enable(nba_ipsec_sa_table *t, int enable);
 int nba_ipsec_profile_read(nba_ipsec_sa_table *t, double *ms, const char **names, int max,
                            int *n_kernels, uint32_t *n_batches);
 
+/* Debug: per-CTA phase timestamps (%globaltimer ns) of the last fused batch,
+ * 8 words per CTA: start, metadata done, AES done, HMAC done, first group
+ * ready, last group ready.  Only when the table was created with the
+ * environment variable NBA_IPSEC_TRACE set; otherwise NBA_IPSEC_EINVAL.
+ * Synchronises the device. */
+int nba_ipsec_debug_trace(nba_ipsec_sa_table *t, uint64_t *host, uint32_t n_words);
+
 /* Host-only helpers exported for tests of the library's own setup code
  * (no device needed): the AES-128 key schedule (FIPS-197 §5.2; 44 words,
  * word i = bytes w[4i..4i+3] of the standard, big-endian) and the HMAC-SHA1

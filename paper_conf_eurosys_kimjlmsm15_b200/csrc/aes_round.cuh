@@ -22,13 +22,26 @@ constexpr uint32_t AES_TABLE_BYTES = 2u * 65536u;
 __device__ __forceinline__ void aes_tables_to_smem(uint8_t *smem, const uint32_t *te0)
 {
     uint32_t *tw = reinterpret_cast<uint32_t *>(smem);
-    for (uint32_t e = threadIdx.x; e < 256u * 32u; e += blockDim.x) {
-        uint32_t x = e >> 5, l = e & 31u;
-        uint32_t v = __ldg(&te0[x]);
-        tw[x * 64u + l] = v;
-        tw[x * 64u + 32u + l] = __funnelshift_l(v, v, 8);
-        tw[16384u + x * 64u + l] = __funnelshift_l(v, v, 16);
-        tw[16384u + x * 64u + 32u + l] = __funnelshift_l(v, v, 24);
+    // all base-table loads first (independent), then the replicated stores
+    constexpr uint32_t NE = 256u * 32u;
+    for (uint32_t e0 = 0; e0 < NE; e0 += 8u * blockDim.x) {
+        uint32_t v[8];
+#pragma unroll
+        for (int u = 0; u < 8; u++) {
+            uint32_t e = e0 + threadIdx.x + u * blockDim.x;
+            v[u] = e < NE ? __ldg(&te0[e >> 5]) : 0u;
+        }
+#pragma unroll
+        for (int u = 0; u < 8; u++) {
+            uint32_t e = e0 + threadIdx.x + u * blockDim.x;
+            if (e < NE) {
+                uint32_t x = e >> 5, l = e & 31u;
+                tw[x * 64u + l] = v[u];
+                tw[x * 64u + 32u + l] = __funnelshift_l(v[u], v[u], 8);
+                tw[16384u + x * 64u + l] = __funnelshift_l(v[u], v[u], 16);
+                tw[16384u + x * 64u + 32u + l] = __funnelshift_l(v[u], v[u], 24);
+            }
+        }
     }
 }
 

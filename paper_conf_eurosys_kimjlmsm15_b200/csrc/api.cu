@@ -10,6 +10,7 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <vector>
@@ -36,7 +37,7 @@ struct nba_ipsec_sa_table {
     uint32_t n_sa = 0, max_batch = 0, max_tiles = 0;
     int num_sms = 0;
     int grid_aes = 0, grid_fused = 0;
-    int pipeline = NBA_IPSEC_PIPE_UNFUSED;
+    int pipeline = NBA_IPSEC_PIPE_FUSED;
     DevTable T{};
     DevWork W{};
     std::vector<void *> allocs;
@@ -187,14 +188,17 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
     chk(dalloc(t, &W.m_seq, M));
     chk(dalloc(t, &W.m_info, M));
     chk(dalloc(t, &W.perm, M));
-    chk(dalloc(t, &W.hist, (size_t)t->max_tiles * n_sa));
+    chk(dalloc(t, &W.hist16, (size_t)t->max_tiles * n_sa));
+    chk(dalloc(t, &W.hpfx, (size_t)t->max_tiles * n_sa));
     chk(dalloc(t, &W.tile_rec, t->max_tiles));
     chk(dalloc(t, &W.tile_blk, t->max_tiles));
     chk(dalloc(t, &W.tile_bin, (size_t)t->max_tiles * NBINS));
     chk(dalloc(t, &W.aes_start, (size_t)std::max(t->grid_aes, t->grid_fused)));
     chk(dalloc(t, &W.ctl, 16));
     chk(dalloc(t, &W.counters, 8));
-    chk(dalloc(t, &W.db, (size_t)M * (MAX_REC_BYTES / 16) + 16));
+    chk(dalloc(t, &W.db, (size_t)M * DB_SLOT16 + 16));
+    if (std::getenv("NBA_IPSEC_TRACE")) chk(dalloc(t, &W.trace, (size_t)t->grid_fused * 8 + 64));
+    W.trace_pro = (uint32_t)t->grid_fused * 8;
     if (e == cudaSuccess) {
         chk(cudaMemcpy(d_rk, rk.data(), rk.size() * sizeof(uint4), cudaMemcpyHostToDevice));
         chk(cudaMemcpy(d_hm, hm.data(), hm.size() * sizeof(uint4), cudaMemcpyHostToDevice));
@@ -202,8 +206,9 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
         chk(cudaMemcpy(d_seq, seq.data(), n_sa * sizeof(uint32_t), cudaMemcpyHostToDevice));
         chk(cudaMemcpy(d_te0, host_te0(), 256 * sizeof(uint32_t), cudaMemcpyHostToDevice));
     }
-    if (e == cudaSuccess) chk(setup_prologue_attributes(n_sa));
+    if (e == cudaSuccess) chk(setup_prologue_attributes(n_sa, t->max_tiles));
     if (e == cudaSuccess) chk(setup_aes_attributes());
+    if (e == cudaSuccess) chk(setup_fused_attributes());
     if (e == cudaSuccess) chk(cudaDeviceSynchronize());
     if (e != cudaSuccess) {
         cudaGetLastError();
@@ -231,9 +236,25 @@ static int enqueue(nba_ipsec_sa_table *t, const BatchArgs &B, cudaStream_t st)
     auto mark = [&]() {
         if (ps) cudaEventRecord(ps->ev[ps->n_ev++], st);
     };
+    const bool unfused = t->pipeline == NBA_IPSEC_PIPE_UNFUSED;
+    if (t->W.trace) {   // debug only: reset the phase trace (mins start at ~0)
+        static std::vector<unsigned long long> init;
+        size_t nw = (size_t)t->grid_fused * 8 + 8;
+        if (init.size() != nw) {
+            init.assign(nw, 0ull);
+            for (size_t c = 0; c < nw / 8; c++) init[c * 8 + 4] = ~0ull;
+            init[nw - 8] = ~0ull;
+        }
+        cudaMemcpyAsync(t->W.trace, init.data(), nw * 8, cudaMemcpyHostToDevice, st);
+    }
     mark();
-    if (launch_prologue(t->T, t->W, B, n_tiles, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
+    if (launch_prologue(t->T, t->W, B, n_tiles, unfused, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
     mark();
+    if (!unfused) {
+        if (launch_fused(t->T, t->W, B, t->grid_fused, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
+        mark();
+        return NBA_IPSEC_OK;
+    }
     if (launch_gather(t->T, t->W, B, n_tiles, (uint32_t)t->grid_aes, st) != cudaSuccess)
         return NBA_IPSEC_ECUDA;
     mark();
@@ -376,10 +397,23 @@ int nba_ipsec_read_sa_seq(nba_ipsec_sa_table *t, uint32_t *host_seq, void *cuda_
     return NBA_IPSEC_OK;
 }
 
+int nba_ipsec_debug_trace(nba_ipsec_sa_table *t, uint64_t *host, uint32_t n_words)
+{
+    if (!t || !host) return NBA_IPSEC_EINVAL;
+    if (!t->W.trace) return NBA_IPSEC_EINVAL;
+    DeviceGuard g(t->device);
+    size_t n = std::min<size_t>(n_words, (size_t)t->grid_fused * 8 + 64);
+    if (cudaDeviceSynchronize() != cudaSuccess ||
+        cudaMemcpy(host, t->W.trace, n * 8, cudaMemcpyDeviceToHost) != cudaSuccess)
+        return NBA_IPSEC_ECUDA;
+    return NBA_IPSEC_OK;
+}
+
 int nba_ipsec_set_pipeline(nba_ipsec_sa_table *t, int pipeline)
 {
     if (!t) return NBA_IPSEC_EINVAL;
-    if (pipeline != NBA_IPSEC_PIPE_UNFUSED) return NBA_IPSEC_EINVAL;   // fused: not yet built
+    if (pipeline != NBA_IPSEC_PIPE_UNFUSED && pipeline != NBA_IPSEC_PIPE_FUSED)
+        return NBA_IPSEC_EINVAL;
     t->pipeline = pipeline;
     return NBA_IPSEC_OK;
 }

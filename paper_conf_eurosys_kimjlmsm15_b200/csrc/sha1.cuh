@@ -77,31 +77,34 @@ __device__ __forceinline__ void hmac_sha1_96(const uint32_t hin[5], const uint32
     const uint32_t bitlen = (64u + M) * 8u;   // the ipad block counts in the length
     uint32_t st[5] = {hin[0], hin[1], hin[2], hin[3], hin[4]};
     uint32_t w[16];
-    for (uint32_t b = 0; b < nblocks; b++) {
-        if (b <= nfull) load_block(w, b);
-        if (b >= nfull) {                     // FIPS 180-4 §5.1.1 padding
-            const uint32_t cut = (b == nfull) ? remw : 0u;
+    // blocks 0..nblocks-1: inner hash; block nblocks: outer hash of the inner
+    // digest (one SHA-1 compression body for both keeps the code compact)
+    for (uint32_t b = 0; b <= nblocks; b++) {
+        if (b < nblocks) {
+            if (b <= nfull) load_block(w, b);
+            if (b >= nfull) {                 // FIPS 180-4 §5.1.1 padding
+                const uint32_t cut = (b == nfull) ? remw : 0u;
 #pragma unroll
-            for (uint32_t j = 0; j < 16; j++)
-                w[j] = j < cut ? w[j] : ((b == nfull && j == cut) ? 0x80000000u : 0u);
-            if (b == nblocks - 1u) w[15] = bitlen;
+                for (uint32_t j = 0; j < 16; j++)
+                    w[j] = j < cut ? w[j] : ((b == nfull && j == cut) ? 0x80000000u : 0u);
+                if (b == nblocks - 1u) w[15] = bitlen;
+            }
+        } else {
+#pragma unroll
+            for (int j = 0; j < 5; j++) {
+                w[j] = st[j];
+                st[j] = hout[j];
+            }
+            w[5] = 0x80000000u;
+#pragma unroll
+            for (int j = 6; j < 15; j++) w[j] = 0u;
+            w[15] = (64u + 20u) * 8u;
         }
         sha1_compress(st, w);
     }
-    uint32_t o[5] = {hout[0], hout[1], hout[2], hout[3], hout[4]};
-    w[0] = st[0];
-    w[1] = st[1];
-    w[2] = st[2];
-    w[3] = st[3];
-    w[4] = st[4];
-    w[5] = 0x80000000u;
-#pragma unroll
-    for (int j = 6; j < 15; j++) w[j] = 0u;
-    w[15] = (64u + 20u) * 8u;
-    sha1_compress(o, w);
-    icv[0] = o[0];
-    icv[1] = o[1];
-    icv[2] = o[2];
+    icv[0] = st[0];
+    icv[1] = st[1];
+    icv[2] = st[2];
 }
 
 }  // namespace nba

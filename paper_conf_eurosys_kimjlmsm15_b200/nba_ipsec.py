@@ -73,6 +73,7 @@ def _load():
         "nba_ipsec_profile_enable": (i32, [vp, i32]),
         "nba_ipsec_profile_read": (i32, [vp, P(ctypes.c_double), P(ctypes.c_char_p), i32,
                                          P(i32), P(u32)]),
+        "nba_ipsec_debug_trace": (i32, [vp, P(u64), u32]),
         "nba_ipsec_host_aes128_key_schedule": (None, [P(ctypes.c_uint8), P(u32)]),
         "nba_ipsec_host_hmac_sha1_midstates": (None, [P(ctypes.c_uint8), P(u32), P(u32)]),
     }
@@ -202,6 +203,13 @@ class SATable:
         _check(lib.nba_ipsec_profile_read(self._h, ms, names, 8, ctypes.byref(nk),
                                           ctypes.byref(nb)), "nba_ipsec_profile_read")
         return {names[k].decode(): ms[k] for k in range(nk.value)}, int(nb.value)
+
+    def debug_trace(self, n_cta: int = 148) -> np.ndarray:
+        """(n_cta + 1, 8) timestamps; the last row is the prologue's."""
+        out = np.zeros(n_cta * 8 + 8, np.uint64)
+        _check(lib.nba_ipsec_debug_trace(self._h, out.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)),
+                                         out.size), "nba_ipsec_debug_trace")
+        return out.reshape(n_cta + 1, 8)
 
     def close(self):
         if getattr(self, "_h", None) is not None and self._h.value:

@@ -11,7 +11,7 @@ from paper_conf_eurosys_kimjlmsm15_b200 import gen
 
 pytestmark = pytest.mark.gpu
 
-PIPES = [1]      # NBA_IPSEC_PIPE_UNFUSED (fused pipeline added with f1)
+PIPES = [0, 1]   # NBA_IPSEC_PIPE_FUSED, NBA_IPSEC_PIPE_UNFUSED
 
 
 @pytest.mark.parametrize("pipe", PIPES)

@@ -1,0 +1,40 @@
+"""Per-CTA phase timeline of the fused kernel (needs NBA_IPSEC_TRACE=1)."""
+import os
+import sys
+
+os.environ.setdefault("NBA_IPSEC_TRACE", "1")
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+from paper_conf_eurosys_kimjlmsm15_b200 import device, gen, nba_ipsec  # noqa: E402
+
+for cfg in (2, 3, 4):
+    c = gen.CONFIGS[cfg]
+    p = gen.make_sas(c["n_sa"], cfg_id=cfg)
+    b = gen.make_batch(c["n"], c["size"], c["n_sa"], cfg_id=cfg)
+    t = nba_ipsec.SATable(p, max_batch=c["n"])
+    db = device.to_device(b, "cuda")
+    for _ in range(5):
+        t.process(*db.args(), n=b.n)
+    torch.cuda.synchronize()
+    full = t.debug_trace(148).astype(np.int64)
+    pro = full[-1]
+    tr = full[:-1]
+    live = tr[:, 0] > 0
+    tr = tr[live]
+    t0 = pro[0]
+    print("prologue: first start 0, tiles done %.2f, last-CTA start %.2f, end %.2f us" %
+          ((pro[1] - t0) / 1e3, (pro[2] - t0) / 1e3, (pro[3] - t0) / 1e3))
+    rel = (tr - t0) / 1000.0
+    names = ["start", "meta_done", "aes_done", "hmac_done", "first_ready", "last_ready"]
+    print(f"config {cfg} ({c['name']}), {live.sum()} CTAs, times in us from first CTA start")
+    for k, nm in enumerate(names):
+        col = rel[:, k]
+        print(f"  {nm:12s} min {col.min():8.2f}  med {np.median(col):8.2f}  max {col.max():8.2f}")
+    from paper_conf_eurosys_kimjlmsm15_b200 import nba_ipsec as nbm
+    import ctypes
+    raw = np.zeros(148 * 8 + 64, np.uint64)
+    nbm.lib.nba_ipsec_debug_trace(t._h, raw.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)), raw.size)
+    print("  chunk0 cycles: meta %d  rounds %d  final %d  stores %d" % tuple(int(x) for x in raw[148*8+8:148*8+12]))
+    t.close()
