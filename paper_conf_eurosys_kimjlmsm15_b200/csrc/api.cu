@@ -38,6 +38,7 @@ struct nba_ipsec_sa_table {
     int num_sms = 0;
     int grid_aes = 0, grid_fused = 0;
     int pipeline = NBA_IPSEC_PIPE_FUSED;
+    bool gridsync = false;     // prologue phase 2 on all CTAs (grid barrier)
     DevTable T{};
     DevWork W{};
     std::vector<void *> allocs;
@@ -140,7 +141,7 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
     t->device = cuda_device;
     t->n_sa = n_sa;
     t->max_batch = max_batch_pkts;
-    t->max_tiles = (max_batch_pkts + TILE - 1) / TILE;
+    t->max_tiles = (max_batch_pkts + PTILE - 1) / PTILE;
     cudaDeviceGetAttribute(&t->num_sms, cudaDevAttrMultiProcessorCount, cuda_device);
     t->grid_aes = aes_grid(t->num_sms);
     t->grid_fused = t->grid_aes;
@@ -206,7 +207,7 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
         chk(cudaMemcpy(d_seq, seq.data(), n_sa * sizeof(uint32_t), cudaMemcpyHostToDevice));
         chk(cudaMemcpy(d_te0, host_te0(), 256 * sizeof(uint32_t), cudaMemcpyHostToDevice));
     }
-    if (e == cudaSuccess) chk(setup_prologue_attributes(n_sa, t->max_tiles));
+    if (e == cudaSuccess) chk(setup_prologue_attributes(n_sa, t->max_tiles, t->num_sms, &t->gridsync));
     if (e == cudaSuccess) chk(setup_aes_attributes());
     if (e == cudaSuccess) chk(setup_fused_attributes());
     if (e == cudaSuccess) chk(cudaDeviceSynchronize());
@@ -223,7 +224,8 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
 
 static int enqueue(nba_ipsec_sa_table *t, const BatchArgs &B, cudaStream_t st)
 {
-    const uint32_t n_tiles = (B.n + TILE - 1) / TILE;
+    const uint32_t n_tiles = (B.n + PTILE - 1) / PTILE;      // prologue / gather tiles
+    const uint32_t n_stiles = (B.n + TILE - 1) / TILE;       // scatter tiles
     ProfSet *ps = nullptr;
     if (t->prof) {
         ps = &t->ring[t->ring_next];
@@ -248,7 +250,8 @@ static int enqueue(nba_ipsec_sa_table *t, const BatchArgs &B, cudaStream_t st)
         cudaMemcpyAsync(t->W.trace, init.data(), nw * 8, cudaMemcpyHostToDevice, st);
     }
     mark();
-    if (launch_prologue(t->T, t->W, B, n_tiles, unfused, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
+    if (launch_prologue(t->T, t->W, B, n_tiles, unfused, t->gridsync, st) != cudaSuccess)
+        return NBA_IPSEC_ECUDA;
     mark();
     if (!unfused) {
         if (launch_fused(t->T, t->W, B, t->grid_fused, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
@@ -262,7 +265,7 @@ static int enqueue(nba_ipsec_sa_table *t, const BatchArgs &B, cudaStream_t st)
     mark();
     if (launch_hmac(t->T, t->W, B, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
     mark();
-    if (launch_scatter(t->T, t->W, B, n_tiles, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
+    if (launch_scatter(t->T, t->W, B, n_stiles, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
     mark();
     return NBA_IPSEC_OK;
 }

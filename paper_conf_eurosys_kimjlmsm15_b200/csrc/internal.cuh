@@ -11,7 +11,8 @@
 
 namespace nba {
 
-constexpr uint32_t TILE = 1024;        // packets per prologue / gather / scatter tile
+constexpr uint32_t TILE = 1024;        // packets per scatter tile (unfused)
+constexpr uint32_t PTILE = 256;        // packets per prologue / gather tile
 constexpr uint32_t MIN_D = 20, MAX_D = 1500;
 constexpr uint32_t MAX_REC_BYTES = 1536;  // roundup16(28 + 1504)
 constexpr uint32_t DB_SLOT16 = 100;       // datablock uint4s per packet (>= fused slot of 1600 B)
@@ -44,8 +45,8 @@ struct DevWork {
     uint32_t *m_seq;        // [M]   ESP sequence number
     uint32_t *m_info;       // [M]   C | tos << 16 | INFO_OK  (0 = dropped / invalid)
     uint32_t *perm;         // [M]   HMAC processing order (length-binned)
-    uint16_t *hist16;       // [max_tiles * n_sa] per-tile per-SA packet counts
-    uint32_t *hpfx;         // [max_tiles * n_sa] exclusive prefix of hist16 down each SA column
+    uint16_t *hist16;       // [max_ptiles * n_sa] per-prologue-tile per-SA packet counts
+    uint32_t *hpfx;         // [max_ptiles * n_sa] exclusive prefix of hist16 down each SA column
     uint32_t *tile_rec;     // [max_tiles] record chunks per tile -> exclusive prefix
     uint32_t *tile_blk;     // [max_tiles] AES blocks per tile -> exclusive prefix
     uint32_t *tile_bin;     // [max_tiles * NBINS] HMAC length bins per tile -> prefix
@@ -57,7 +58,8 @@ struct DevWork {
     uint4 *db;              // datablock of ESP records (16-B aligned)
 };
 
-constexpr int CTL_TICKET = 0, CTL_TOTAL_REC = 1, CTL_TOTAL_BLK = 2, CTL_WORK = 3;
+constexpr int CTL_TICKET = 0, CTL_TOTAL_REC = 1, CTL_TOTAL_BLK = 2, CTL_WORK = 3,
+              CTL_BAR_COUNT = 4, CTL_BAR_GEN = 5;
 constexpr int NBINS = 32;   // HMAC bins by number of inner SHA-1 blocks (2..25)
 
 struct BatchArgs {
@@ -74,7 +76,7 @@ struct BatchArgs {
 #ifdef __CUDACC__
 // --- launchers (one per kernel file) ----------------------------------------
 cudaError_t launch_prologue(const DevTable &T, const DevWork &W, const BatchArgs &B,
-                            uint32_t n_tiles, bool unfused, cudaStream_t st);
+                            uint32_t n_tiles, bool unfused, bool gridsync, cudaStream_t st);
 cudaError_t launch_gather(const DevTable &T, const DevWork &W, const BatchArgs &B,
                           uint32_t n_tiles, uint32_t aes_grid, cudaStream_t st);
 cudaError_t launch_aes(const DevTable &T, const DevWork &W, const BatchArgs &B, int grid,
@@ -85,7 +87,7 @@ cudaError_t launch_scatter(const DevTable &T, const DevWork &W, const BatchArgs 
                            uint32_t n_tiles, cudaStream_t st);
 cudaError_t launch_fused(const DevTable &T, const DevWork &W, const BatchArgs &B, int grid,
                          cudaStream_t st);
-cudaError_t setup_prologue_attributes(uint32_t n_sa, uint32_t max_tiles);
+cudaError_t setup_prologue_attributes(uint32_t n_sa, uint32_t max_tiles, int num_sms, bool *gridsync);
 cudaError_t setup_aes_attributes();
 cudaError_t setup_fused_attributes();
 int aes_grid(int num_sms);

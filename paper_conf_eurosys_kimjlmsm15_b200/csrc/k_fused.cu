@@ -52,7 +52,7 @@ struct FusedLo {
     uint4 pre0[F_SUPER];           // X0, Z0, Z1, Z2 (CTR precompute)
     uint32_t pre1[F_SUPER];        // Z3
     uint8_t pre2[F_SUPER];         // byte 3 of round-key word rk0.w
-    uint4 rkA[F_SUPER][4];         // round keys 3..6
+    uint4 rkA[4][F_SUPER];         // round keys 3..6, round-major (conflict-free LDS.128)
     uint32_t gneed[F_GROUPS];      // AES pairs per HMAC group
     unsigned long long gbar[F_GROUPS];   // mbarrier per HMAC group
     uint32_t aes_next;             // next 32-pair AES chunk to claim
@@ -63,7 +63,7 @@ struct FusedLo {
 };
 
 struct FusedHi {
-    uint4 rkB[F_SUPER][4];         // round keys 7..10
+    uint4 rkB[4][F_SUPER];         // round keys 7..10, round-major
     uint16_t chunkpos[F_CHUNKS];   // first position of every 32-pair chunk
 };
 
@@ -311,9 +311,11 @@ __device__ __forceinline__ void aes_pair_chunk(const BatchArgs &B, FusedLo &L, F
              a3 = TL(ta, 1, 1) ^ Z3;
     uint32_t b0 = TL(tb, 0, 0) ^ pre.y, b1 = TL(tb, 3, 3) ^ pre.z, b2 = TL(tb, 2, 2) ^ pre.w,
              b3 = TL(tb, 1, 1) ^ Z3;
-#pragma unroll
+    // rounds 3..9 as a rolled loop: keeps the hot code within the instruction cache
+    // alongside the SHA-1 compression that other warps run concurrently
+#pragma unroll 1
     for (int r = 3; r < 10; r++) {
-        const uint4 rk = r < 7 ? L.rkA[pk][r - 3] : H.rkB[pk][r - 7];
+        const uint4 rk = r < 7 ? L.rkA[r - 3][pk] : H.rkB[r - 7][pk];
         const uint32_t u0 = TL(a0, 0, 0) ^ TL(a1, 1, 1) ^ TL(a2, 2, 2) ^ TL(a3, 3, 3) ^ rk.x;
         const uint32_t u1 = TL(a1, 0, 0) ^ TL(a2, 1, 1) ^ TL(a3, 2, 2) ^ TL(a0, 3, 3) ^ rk.y;
         const uint32_t u2 = TL(a2, 0, 0) ^ TL(a3, 1, 1) ^ TL(a0, 2, 2) ^ TL(a1, 3, 3) ^ rk.z;
@@ -325,7 +327,7 @@ __device__ __forceinline__ void aes_pair_chunk(const BatchArgs &B, FusedLo &L, F
         a0 = u0; a1 = u1; a2 = u2; a3 = u3;
         b0 = v0; b1 = v1; b2 = v2; b3 = v3;
     }
-    const uint4 rk = H.rkB[pk][3];
+    const uint4 rk = H.rkB[3][pk];
     long long ck2 = clock64();
     // final round: S[x] is byte (j+2)&3 of Tj[x]
 #define NBA_FINAL(s0, s1, s2, s3)                                                               \
@@ -478,31 +480,54 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc)
 
     aes_tables_to_smem(tabs, T.te0);
     if (tid < 4) L.cnt[tid] = 0ull;
-    // Programmatic dependent launch: everything above overlapped the prologue;
-    // its outputs (ranks, per-SA prefixes, seq_prev) are visible after this.
-    asm volatile("griddepcontrol.wait;" ::: "memory");
 
     const uint32_t p_begin = blockIdx.x * ppc;
     const uint32_t p_end = min(B.n, p_begin + ppc);
+    static_assert(F_SUPER <= F_THREADS, "one packet per thread in the metadata phase");
 
     for (uint32_t base = p_begin; base < p_end; base += F_SUPER) {
         const uint32_t cnt_pk = min((uint32_t)F_SUPER, p_end - base);
         // ---- 1. metadata (thread j <-> packet base + j) ---------------------
         if (tid < NBINS) L.bins[tid] = 0;
+        const uint32_t j = tid;
+        const uint32_t i = base + j;
+        // 1a. everything that does not depend on the prologue (overlaps it
+        //     under programmatic dependent launch on the first round)
+        uint32_t sa = INVALID_SA, D = 0, inoff = 0, tos = 0, nonce = 0;
+        bool cand = false;
+        uint4 r0 = make_uint4(0, 0, 0, 0), r1 = r0, r2 = r0;
+        if (j < cnt_pk) {
+            sa = B.sa_idx[i];
+            D = B.in_len[i];
+            inoff = B.in_off[i];
+            L.outoff[j] = B.out_off[i];
+            cand = sa < n_sa && D >= MIN_D && D <= MAX_D;
+            if (cand) {
+                tos = B.in_buf[inoff + 1];
+                const uint4 *rks = T.rk + (size_t)sa * 11u;
+                r0 = __ldg(&rks[0]);
+                r1 = __ldg(&rks[1]);
+                r2 = __ldg(&rks[2]);
+                nonce = __ldg(&T.sahdr[sa].y);
+#pragma unroll
+                for (int r = 0; r < 4; r++) {
+                    L.rkA[r][j] = __ldg(&rks[3 + r]);
+                    H.rkB[r][j] = __ldg(&rks[7 + r]);
+                }
+            }
+        }
+        // Programmatic dependent launch: the prologue's outputs (ranks, per-SA
+        // prefixes, seq_prev) are complete and visible after this.
+        if (base == p_begin) asm volatile("griddepcontrol.wait;" ::: "memory");
         __syncthreads();   // also publishes the T-tables on the first round
-        for (uint32_t j = tid; j < cnt_pk; j += F_THREADS) {
-            const uint32_t i = base + j;
-            uint32_t info = 0, bin = NBINS - 1;
-            const uint32_t sa = B.sa_idx[i];
-            const uint32_t D = B.in_len[i];
-            const uint32_t inoff = B.in_off[i];
-            uint32_t q32 = 0;
-            if (sa < n_sa && D >= MIN_D && D <= MAX_D) {
+        // 1b. sequence number, drop decision, CTR precompute
+        if (j < cnt_pk) {
+            uint32_t info = 0, bin = NBINS - 1, q32 = 0;
+            if (cand) {
                 const unsigned long long q = (unsigned long long)T.seq_prev[sa] + 1ull +
-                                             W.hpfx[(size_t)(i / TILE) * n_sa + sa] + W.lrank[i];
+                                             W.hpfx[(size_t)(i / PTILE) * n_sa + sa] + W.lrank[i];
                 if (q <= 0xffffffffull) {   // RFC 4303 §3.3.3: never cycle
                     q32 = (uint32_t)q;
-                    const uint32_t tos = B.in_buf[inoff + 1];
                     info = D | (tos << 16) | INFO_OK;
                     bin = hmac_bin(true, esp_C(D));
                     // CTR precompute (FIPS-197 Cipher() rounds 1-2 on the counter block
@@ -510,9 +535,7 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc)
                     // column 3 varies, so after round 1 only column 0 varies, through
                     // one T3 lookup: t0 = T3[r3 ^ (k+1)] ^ X0, and round 2 is
                     // u_c = T[row(t0)] ^ Z_c with one lookup per column.
-                    const uint4 *rks = T.rk + (size_t)sa * 11u;
-                    const uint4 r0 = __ldg(&rks[0]), r1 = __ldg(&rks[1]), r2 = __ldg(&rks[2]);
-                    const uint32_t s0 = __ldg(&T.sahdr[sa].y) ^ r0.x;
+                    const uint32_t s0 = nonce ^ r0.x;
                     const uint32_t s1 = r0.y;
                     const uint32_t s2 = bswap32(q32) ^ r0.z;
                     const uint32_t s3 = r0.w;     // byte 3 is XORed with (k+1) per block
@@ -527,18 +550,12 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc)
                     L.pre0[j] = make_uint4(X0, Z0, Z1, Z2);
                     L.pre1[j] = Z3;
                     L.pre2[j] = (uint8_t)(s3 >> 24);
-#pragma unroll
-                    for (int r = 0; r < 4; r++) {
-                        L.rkA[j][r] = __ldg(&rks[3 + r]);
-                        H.rkB[j][r] = __ldg(&rks[7 + r]);
-                    }
                 }
             }
             L.sa[j] = (uint16_t)sa;
             L.seq[j] = q32;
             L.info[j] = info;
             L.inoff[j] = inoff;
-            L.outoff[j] = B.out_off[i];
             atomicAdd(&L.bins[bin], 1u);
         }
         __syncthreads();

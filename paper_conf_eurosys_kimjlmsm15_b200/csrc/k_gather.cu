@@ -53,18 +53,18 @@ __device__ __forceinline__ uint4 build_payload_chunk(const uint8_t *src, uint32_
     return v;
 }
 
-__global__ void __launch_bounds__(1024, 1)
+__global__ void __launch_bounds__(PTILE)
 k_gather(DevTable T, DevWork W, BatchArgs B, uint32_t aes_grid)
 {
-    __shared__ uint32_t s_pref[TILE + 1];   // record-chunk prefix within the tile
-    __shared__ uint32_t s_D[TILE];          // D | INFO_OK-bit
-    __shared__ uint32_t s_sa[TILE];
-    __shared__ uint32_t s_seq[TILE];
+    __shared__ uint32_t s_pref[PTILE + 1];   // record-chunk prefix within the tile
+    __shared__ uint32_t s_D[PTILE];          // D | INFO_OK-bit
+    __shared__ uint32_t s_sa[PTILE];
+    __shared__ uint32_t s_seq[PTILE];
     __shared__ uint32_t s_scr[32];
     __shared__ uint32_t s_bin[NBINS];
     const uint32_t tid = threadIdx.x;
     const uint32_t tile = blockIdx.x;
-    const uint32_t i = tile * TILE + tid;
+    const uint32_t i = tile * PTILE + tid;
     const uint32_t n_sa = T.n_sa;
     if (tid < NBINS) s_bin[tid] = 0;
 
@@ -110,15 +110,15 @@ k_gather(DevTable T, DevWork W, BatchArgs B, uint32_t aes_grid)
         }
     }
     s_pref[tid] = my_rec;
-    if (tid == TILE - 1) s_pref[TILE] = tot_rec;
+    if (tid == PTILE - 1) s_pref[PTILE] = tot_rec;
     s_D[tid] = D | (info ? INFO_OK : 0u);
     s_sa[tid] = s;
     s_seq[tid] = q32;
     __syncthreads();
 
-    const uint32_t tile_first = tile * TILE;
+    const uint32_t tile_first = tile * PTILE;
     for (uint32_t c = tid; c < tot_rec; c += blockDim.x) {
-        uint32_t j = upper_bound_m1(s_pref, TILE, c);
+        uint32_t j = upper_bound_m1(s_pref, PTILE, c);
         uint32_t k = c - s_pref[j];
         uint32_t dd = s_D[j];
         if (!(dd & INFO_OK)) continue;            // dropped: record never read
@@ -139,7 +139,7 @@ k_gather(DevTable T, DevWork W, BatchArgs B, uint32_t aes_grid)
 cudaError_t launch_gather(const DevTable &T, const DevWork &W, const BatchArgs &B,
                           uint32_t n_tiles, uint32_t aes_grid, cudaStream_t st)
 {
-    k_gather<<<n_tiles, TILE, 0, st>>>(T, W, B, aes_grid);
+    k_gather<<<n_tiles, PTILE, 0, st>>>(T, W, B, aes_grid);
     return cudaGetLastError();
 }
 

@@ -1,6 +1,7 @@
 // k_prologue.cu -- row a1 of the hot path: per-packet validity and sizes,
-// deterministic per-SA ranks (-> ESP sequence numbers), per-SA counter advance,
-// and the tile-level exclusive scans that place records and AES blocks.
+// deterministic per-SA ranks (-> ESP sequence numbers), the per-SA counter
+// advance, and (unfused pipeline only) the tile-level scans that place records
+// and AES blocks in the datablock.
 //
 // PAPER.md:329 (§3.3): "the framework validates packet data and datablock
 // fields prior to execution"; invalid packets are masked, not
@@ -8,28 +9,113 @@
 // never cycling) applied in batch-index order (reading A5), so the result is
 // exactly that of the sequential oracle loop.
 //
-// One CTA per tile of 1024 packets.  Within a warp, __match_any_sync groups
-// lanes with the same SA; the per-warp groups are then merged in warp order
-// through a shared histogram (deterministic: no atomics decide ranks).  The
-// last CTA to finish (ticket) scans the tile histograms per SA, advances the
-// SA sequence counters and scans the per-tile record / block totals.
+// Phase 1, one CTA per tile of PTILE = 256 packets: __match_any_sync groups
+// the lanes of a warp by SA; the 8 warps' groups are merged in warp order
+// through a shared histogram (deterministic: no atomic decides a rank).  The
+// tile writes its per-SA counts (u16) and each packet's within-tile rank.
+// Phase 2, after a grid-wide barrier (all tiles are co-resident: 256-thread
+// CTAs with a 2 KB histogram): one warp per SA scans that SA's column of tile
+// counts with shuffles (-> per-tile exclusive prefixes) and advances the SA's
+// sequence counter.  If the grid could not be co-resident (very many SAs),
+// the last CTA to finish does phase 2 alone instead.
 #include "internal.cuh"
 
 namespace nba {
 
-// Dynamic shared memory of the prologue: the tile histogram (u16 per SA), or
-// -- when it fits -- the whole [tiles x SAs] u16 histogram for the last CTA's
-// column scan.
-static size_t prologue_smem(uint32_t n_sa, uint32_t n_tiles)
+static size_t prologue_smem(uint32_t n_sa) { return ((size_t)n_sa * 2 + 15) & ~(size_t)15; }
+
+// Sense-reversing grid barrier over gridDim.x co-resident CTAs.
+__device__ __forceinline__ void grid_barrier(uint32_t *count, uint32_t *gen)
 {
-    size_t tile = ((size_t)n_sa * 2 + 15) & ~(size_t)15;
-    size_t all = ((size_t)n_sa * n_tiles * 2 + 15) & ~(size_t)15;
-    const size_t cap = 200u * 1024u;
-    return all <= cap ? (all > tile ? all : tile) : tile;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        const uint32_t g = *reinterpret_cast<volatile uint32_t *>(gen);
+        __threadfence();
+        if (atomicAdd(count, 1u) == gridDim.x - 1u) {
+            *reinterpret_cast<volatile uint32_t *>(count) = 0;
+            __threadfence();
+            atomicAdd(gen, 1u);
+        } else {
+            while (*reinterpret_cast<volatile uint32_t *>(gen) == g) __nanosleep(32);
+        }
+        __threadfence();
+    }
+    __syncthreads();
 }
 
-__global__ void __launch_bounds__(1024, 1)
-k_prologue(DevTable T, DevWork W, BatchArgs B, uint32_t n_tiles, bool unfused, uint32_t smem_bytes)
+// Exclusive prefix of the tile counts down SA column `sa` by one warp, then the
+// SA counter advance (only the first (2^32-1 - seq) packets get numbers).
+__device__ __forceinline__ void scan_sa_column(const DevTable &T, const DevWork &W, uint32_t sa,
+                                               uint32_t n_tiles, uint32_t n_sa, uint32_t lane)
+{
+    uint32_t carry = 0;
+    for (uint32_t t0 = 0; t0 < n_tiles; t0 += 128) {
+        uint32_t h[4];
+#pragma unroll
+        for (int u = 0; u < 4; u++) {
+            const uint32_t t = t0 + 32u * u + lane;
+            h[u] = t < n_tiles ? __ldcg(&W.hist16[(size_t)t * n_sa + sa]) : 0u;
+        }
+#pragma unroll
+        for (int u = 0; u < 4; u++) {
+            uint32_t x = h[u];
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+                if (lane >= (uint32_t)o) x += y;
+            }
+            const uint32_t t = t0 + 32u * u + lane;
+            if (t < n_tiles) W.hpfx[(size_t)t * n_sa + sa] = carry + x - h[u];
+            carry += __shfl_sync(0xffffffffu, x, 31);
+        }
+    }
+    if (lane == 0) {
+        const uint32_t old = T.seq[sa];
+        T.seq_prev[sa] = old;
+        const uint32_t room = 0xffffffffu - old;
+        T.seq[sa] = old + (carry < room ? carry : room);
+    }
+}
+
+// Unfused pipeline only: exclusive scans of the per-tile record / AES-block
+// totals and of the HMAC length bins (bin-major, tile-minor).
+__device__ __forceinline__ void scan_tile_totals(const DevWork &W, uint32_t n_tiles, uint32_t *s_scr)
+{
+    const uint32_t tid = threadIdx.x;
+    uint32_t carry_rec = 0, carry_blk = 0;
+    for (uint32_t t0 = 0; t0 < n_tiles; t0 += blockDim.x) {
+        const uint32_t t = t0 + tid;
+        const uint32_t vr = t < n_tiles ? __ldcg(&W.tile_rec[t]) : 0u;
+        const uint32_t vb = t < n_tiles ? __ldcg(&W.tile_blk[t]) : 0u;
+        uint32_t sr, sb;
+        const uint32_t er = block_exclusive_scan(vr, s_scr, &sr);
+        const uint32_t eb = block_exclusive_scan(vb, s_scr, &sb);
+        if (t < n_tiles) {
+            W.tile_rec[t] = carry_rec + er;
+            W.tile_blk[t] = carry_blk + eb;
+        }
+        carry_rec += sr;
+        carry_blk += sb;
+    }
+    const uint32_t tot = n_tiles * NBINS;
+    uint32_t carry = 0;
+    for (uint32_t e0 = 0; e0 < tot; e0 += blockDim.x) {
+        const uint32_t e = e0 + tid;
+        const uint32_t b = e / n_tiles, t = e % n_tiles;
+        const uint32_t v = e < tot ? __ldcg(&W.tile_bin[t * NBINS + b]) : 0u;
+        uint32_t s;
+        const uint32_t ex = block_exclusive_scan(v, s_scr, &s);
+        if (e < tot) W.tile_bin[t * NBINS + b] = carry + ex;
+        carry += s;
+    }
+    if (tid == 0) {
+        W.ctl[CTL_TOTAL_REC] = carry_rec;
+        W.ctl[CTL_TOTAL_BLK] = carry_blk;
+    }
+}
+
+__global__ void __launch_bounds__(PTILE)
+k_prologue(DevTable T, DevWork W, BatchArgs B, uint32_t n_tiles, bool unfused, bool gridsync)
 {
     extern __shared__ uint16_t s_hist[];             // [n_sa] counts in this tile
     __shared__ uint32_t s_scr[32];
@@ -37,36 +123,35 @@ k_prologue(DevTable T, DevWork W, BatchArgs B, uint32_t n_tiles, bool unfused, u
     __shared__ uint32_t s_bin[NBINS];
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
     const uint32_t tile = blockIdx.x;
-    const uint32_t i = tile * TILE + tid;
+    const uint32_t i = tile * PTILE + tid;
     const uint32_t n_sa = T.n_sa;
-
     unsigned long long *tr = W.trace ? W.trace + (size_t)W.trace_pro : nullptr;
     if (tr && tid == 0) atomicMin(&tr[0], gtimer());
-    for (uint32_t k = tid; k < n_sa; k += blockDim.x) s_hist[k] = 0;
+
+    for (uint32_t k = tid; k < n_sa; k += PTILE) s_hist[k] = 0;
     if (tid < NBINS) s_bin[tid] = 0;
 
-    uint32_t s = INVALID_SA, rec16 = 0, nblk = 0;
+    uint32_t s = INVALID_SA, rec16 = 0, nblk = 0, C = 0;
     if (i < B.n) {
-        uint32_t sa = B.sa_idx[i];
-        uint32_t D = B.in_len[i];
+        const uint32_t sa = B.sa_idx[i];
+        const uint32_t D = B.in_len[i];
         if (sa < n_sa && D >= MIN_D && D <= MAX_D) {
             s = sa;
-            uint32_t C = esp_C(D);
+            C = esp_C(D);
             rec16 = esp_rec16(C);
             nblk = esp_nblk(C);
         }
     }
-    uint32_t C_ = (s != INVALID_SA) ? esp_C(B.in_len[i]) : 0u;
-    const uint32_t bin = hmac_bin(s != INVALID_SA, C_);
     const uint32_t peers = __match_any_sync(0xffffffffu, s);
     const uint32_t leader = __ffs(peers) - 1;
     const uint32_t wrank = __popc(peers & lanemask_lt());
     const uint32_t wcnt = __popc(peers);
     __syncthreads();
 
-    // merge warp groups in warp order (deterministic ranks)
+    // merge the warps' groups in warp order (deterministic ranks)
     uint32_t base = 0;
-    for (uint32_t w = 0; w < blockDim.x / 32u; w++) {
+#pragma unroll 1
+    for (uint32_t w = 0; w < PTILE / 32u; w++) {
         if (warp == w) {
             if (s != INVALID_SA && lane == leader) {
                 base = s_hist[s];
@@ -76,150 +161,75 @@ k_prologue(DevTable T, DevWork W, BatchArgs B, uint32_t n_tiles, bool unfused, u
         }
         __syncthreads();
     }
-    if (i < B.n) {
-        W.lrank[i] = base + wrank;
-        atomicAdd(&s_bin[bin], 1u);
-    }
+    if (i < B.n) W.lrank[i] = base + wrank;
+    for (uint32_t k = tid; k < n_sa; k += PTILE) W.hist16[(size_t)tile * n_sa + k] = s_hist[k];
 
-    for (uint32_t k = tid; k < n_sa; k += blockDim.x)
-        W.hist16[(size_t)tile * n_sa + k] = s_hist[k];
-    // let the dependent (fused) kernel launch and build its tables meanwhile;
-    // it waits for this grid's completion before reading our outputs
-    asm volatile("griddepcontrol.launch_dependents;");
-
-    uint32_t tot_rec, tot_blk;
-    block_exclusive_scan(rec16, s_scr, &tot_rec);
-    block_exclusive_scan(nblk, s_scr, &tot_blk);
     if (unfused) {
+        if (i < B.n) atomicAdd(&s_bin[hmac_bin(s != INVALID_SA, C)], 1u);
+        uint32_t tot_rec, tot_blk;
+        block_exclusive_scan(rec16, s_scr, &tot_rec);
+        block_exclusive_scan(nblk, s_scr, &tot_blk);
         if (tid == 0) {
             W.tile_rec[tile] = tot_rec;
             W.tile_blk[tile] = tot_blk;
         }
         if (tid < NBINS) W.tile_bin[tile * NBINS + tid] = s_bin[tid];
     }
-
-    // ---- last CTA: per-SA scan over tiles, seq advance, tile scans ----------
-    __threadfence();
-    __syncthreads();
     if (tr && tid == 0) atomicMax(&tr[1], gtimer());
-    if (tid == 0) s_last = (atomicAdd(&W.ctl[CTL_TICKET], 1u) == n_tiles - 1u) ? 1u : 0u;
-    __syncthreads();
-    if (!s_last) return;
-    __threadfence();
-    if (tr && tid == 0) tr[2] = gtimer();
 
-    // per-SA exclusive scan down the tile columns -> hpfx, and the SA counter advance
-    const size_t cells = (size_t)n_tiles * n_sa;
-    if (cells * 2 <= smem_bytes) {
-        // whole histogram into shared memory with 16-byte loads, then scan there
-        uint16_t *m = s_hist;
-        const size_t n16 = cells / 8;                  // cells is a multiple of 8 (n_sa even)
-        const uint4 *src = reinterpret_cast<const uint4 *>(W.hist16);
-        for (size_t e0 = 0; e0 < n16; e0 += 4u * blockDim.x) {
-            uint4 v[4];
-#pragma unroll
-            for (int u = 0; u < 4; u++) {
-                size_t e = e0 + tid + (size_t)u * blockDim.x;
-                v[u] = e < n16 ? __ldcg(&src[e]) : make_uint4(0, 0, 0, 0);
-            }
-#pragma unroll
-            for (int u = 0; u < 4; u++) {
-                size_t e = e0 + tid + (size_t)u * blockDim.x;
-                if (e < n16) reinterpret_cast<uint4 *>(m)[e] = v[u];
-            }
-        }
-        for (size_t e = n16 * 8 + tid; e < cells; e += blockDim.x) m[e] = __ldcg(&W.hist16[e]);
-        __syncthreads();
-        for (uint32_t sa = tid; sa < n_sa; sa += blockDim.x) {
-            uint32_t run = 0;
-            for (uint32_t t = 0; t < n_tiles; t++) {
-                const uint32_t h = m[(size_t)t * n_sa + sa];
-                W.hpfx[(size_t)t * n_sa + sa] = run;
-                run += h;
-            }
-            const uint32_t old = T.seq[sa];
-            T.seq_prev[sa] = old;
-            const uint32_t room = 0xffffffffu - old;
-            T.seq[sa] = old + (run < room ? run : room);
-        }
+    if (gridsync) {
+        // ---- phase 2 on every CTA: one warp per SA column -------------------
+        grid_barrier(&W.ctl[CTL_BAR_COUNT], &W.ctl[CTL_BAR_GEN]);
+        if (tr && tid == 0 && tile == 0) tr[2] = gtimer();
+        // let the dependent (fused) kernel launch and stage its tables; it waits
+        // for this grid's completion before reading our outputs
+        asm volatile("griddepcontrol.launch_dependents;");
+        const uint32_t nwarps = gridDim.x * (PTILE / 32u);
+        for (uint32_t col = tile * (PTILE / 32u) + warp; col < n_sa; col += nwarps)
+            scan_sa_column(T, W, col, n_tiles, n_sa, lane);
+        if (unfused && tile == 0) scan_tile_totals(W, n_tiles, s_scr);
     } else {
-        for (uint32_t sa = tid; sa < n_sa; sa += blockDim.x) {
-            uint32_t run = 0;
-            for (uint32_t t0 = 0; t0 < n_tiles; t0 += 16) {
-                uint32_t h[16];
-#pragma unroll
-                for (int u = 0; u < 16; u++)
-                    h[u] = (t0 + u < n_tiles) ? __ldcg(&W.hist16[(size_t)(t0 + u) * n_sa + sa]) : 0u;
-#pragma unroll
-                for (int u = 0; u < 16; u++) {
-                    if (t0 + u < n_tiles) W.hpfx[(size_t)(t0 + u) * n_sa + sa] = run;
-                    run += h[u];
-                }
-            }
-            const uint32_t old = T.seq[sa];
-            T.seq_prev[sa] = old;
-            const uint32_t room = 0xffffffffu - old;
-            T.seq[sa] = old + (run < room ? run : room);
-        }
-    }
-    __syncthreads();
-
-    uint32_t carry_rec = 0, carry_blk = 0;
-    if (unfused) {
-        for (uint32_t t0 = 0; t0 < n_tiles; t0 += blockDim.x) {
-            uint32_t t = t0 + tid;
-            uint32_t vr = t < n_tiles ? __ldcg(&W.tile_rec[t]) : 0u;
-            uint32_t vb = t < n_tiles ? __ldcg(&W.tile_blk[t]) : 0u;
-            uint32_t sr, sb;
-            uint32_t er = block_exclusive_scan(vr, s_scr, &sr);
-            uint32_t eb = block_exclusive_scan(vb, s_scr, &sb);
-            if (t < n_tiles) {
-                W.tile_rec[t] = carry_rec + er;
-                W.tile_blk[t] = carry_blk + eb;
-            }
-            carry_rec += sr;
-            carry_blk += sb;
-        }
-        // HMAC length bins, bin-major / tile-minor order: one flattened block scan
-        const uint32_t tot = n_tiles * NBINS;
-        uint32_t carry = 0;
-        for (uint32_t e0 = 0; e0 < tot; e0 += blockDim.x) {
-            uint32_t e = e0 + tid;
-            uint32_t b = e / n_tiles, t = e % n_tiles;
-            uint32_t v = e < tot ? __ldcg(&W.tile_bin[t * NBINS + b]) : 0u;
-            uint32_t s;
-            uint32_t ex = block_exclusive_scan(v, s_scr, &s);
-            if (e < tot) W.tile_bin[t * NBINS + b] = carry + ex;
-            carry += s;
-        }
-    }
-    if (tid == 0) {
-        W.ctl[CTL_TOTAL_REC] = carry_rec;
-        W.ctl[CTL_TOTAL_BLK] = carry_blk;
-        W.ctl[CTL_TICKET] = 0;            // re-arm for the next batch (stream-ordered)
-        W.ctl[CTL_WORK] = 0;              // fused kernel's work counter
+        // ---- phase 2 on the last CTA to finish phase 1 -----------------------
+        __threadfence();
+        __syncthreads();
+        if (tid == 0) s_last = (atomicAdd(&W.ctl[CTL_TICKET], 1u) == n_tiles - 1u) ? 1u : 0u;
+        __syncthreads();
+        asm volatile("griddepcontrol.launch_dependents;");
+        if (!s_last) return;
+        __threadfence();
+        if (tr && tid == 0) tr[2] = gtimer();
+        for (uint32_t col = warp; col < n_sa; col += PTILE / 32u)
+            scan_sa_column(T, W, col, n_tiles, n_sa, lane);
+        if (unfused) scan_tile_totals(W, n_tiles, s_scr);
+        __syncthreads();
+        if (tid == 0) W.ctl[CTL_TICKET] = 0;            // re-arm for the next batch
     }
     if (tr) {
         __syncthreads();
-        if (tid == 0) tr[3] = gtimer();
+        if (tid == 0) atomicMax(&tr[3], gtimer());
     }
 }
 
 cudaError_t launch_prologue(const DevTable &T, const DevWork &W, const BatchArgs &B,
-                            uint32_t n_tiles, bool unfused, cudaStream_t st)
+                            uint32_t n_tiles, bool unfused, bool gridsync, cudaStream_t st)
 {
-    size_t smem = prologue_smem(T.n_sa, n_tiles);
-    k_prologue<<<n_tiles, TILE, smem, st>>>(T, W, B, n_tiles, unfused, (uint32_t)smem);
+    k_prologue<<<n_tiles, PTILE, prologue_smem(T.n_sa), st>>>(T, W, B, n_tiles, unfused, gridsync);
     return cudaGetLastError();
 }
 
-cudaError_t setup_prologue_attributes(uint32_t n_sa, uint32_t max_tiles)
+cudaError_t setup_prologue_attributes(uint32_t n_sa, uint32_t max_tiles, int num_sms, bool *gridsync)
 {
-    size_t smem = prologue_smem(n_sa, max_tiles);
-    if (smem < 200u * 1024u && (size_t)n_sa * max_tiles * 2 > smem) smem = 200u * 1024u;
-    if (smem > 48 * 1024)
-        return cudaFuncSetAttribute(k_prologue, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                    (int)smem);
+    const size_t smem = prologue_smem(n_sa);
+    if (smem > 48 * 1024) {
+        cudaError_t e = cudaFuncSetAttribute(k_prologue, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             (int)smem);
+        if (e != cudaSuccess) return e;
+    }
+    int per_sm = 0;
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_prologue, PTILE, smem);
+    if (e != cudaSuccess) return e;
+    // grid-wide barrier only if every tile of the largest batch is co-resident
+    *gridsync = (uint64_t)per_sm * (uint64_t)num_sms >= (uint64_t)max_tiles;
     return cudaSuccess;
 }
 
