@@ -56,7 +56,7 @@ def load_peaks():
 class ClockSampler:
     """Samples SM clock + throttle reasons with NVML during the timed region."""
 
-    def __init__(self, gpu_index: int, period_s: float = 0.002):
+    def __init__(self, gpu_index: int, period_s: float = 0.001):
         self.idx, self.period = gpu_index, period_s
         self.samples, self.reasons = [], set()
         self._stop = threading.Event()
@@ -128,37 +128,45 @@ def work_model(b):
     }
 
 
-# Per-kernel roofline model.  Integer-pipe peaks from the
-# microarchitecture guide's unit counts at the max SM clock: shared-memory
-# LSU 32 x 4-B lookups/clk/SM; ALU pipe (LOP3/SHF/IADD3) 64 lanes/clk/SM.
-AES_LOOKUPS_PER_BLOCK = 160
-SHA1_OPS_PER_COMPRESSION = 597
+# Per-kernel roofline model.
+#
+# The path is integer work: AES-128 T-table rounds (shared-memory lookups plus
+# ALU byte-permutes / XORs) and SHA-1 compressions (ALU rotates / logic / adds).
+# Its roofline is the SM's integer ALU pipe: 64 int32 lanes/clk/SM (4 SMSPs x 16;
+# B300_MICROARCH.md "Pipe rates", re-measured on B200 by tools/microbench.cu:
+# 63.9 lanes/clk/SM for LOP3 / PRMT / SHF / IADD3) x 148 SMs x the max SM clock.
+# Algorithmic ALU work:
+#   AES-128-CTR block (T-table method with the per-packet round-1/2 CTR
+#   precompute): 133 table lookups, each one byte-select/address op, plus the
+#   XOR merges -> AES_ALU_OPS_PER_BLOCK = 220
+#   SHA-1 compression (FIPS 180-4 §6.1.2): 80 rounds x 5 (f, rotl5, rotl30,
+#   two 3-input adds) + 64 x 3 schedule ops -> SHA1_ALU_OPS_PER_COMPRESSION = 592
+# The shared-memory LSU (32 lookups/clk/SM) is reported alongside for AES.
+AES_ALU_OPS_PER_BLOCK = 220
+AES_LOOKUPS_PER_BLOCK = 133
+SHA1_ALU_OPS_PER_COMPRESSION = 592
+ALU_LANES_PER_CLK_SM = 64
+LDS_LANES_PER_CLK_SM = 32
 
 
 def kernel_roofline(name, ms_per_launch, w, peaks):
     f = peaks["sm_max_mhz"] * 1e6
     s = ms_per_launch * 1e-3
-    if name in ("aes_ctr",):
-        achieved = w["aes_blocks"] * AES_LOOKUPS_PER_BLOCK / s / 1e9
-        peak = SM_COUNT * 32 * f / 1e9
-        return {"bound": "alu", "unit": "Glookup/s", "achieved": achieved, "peak": peak,
-                "peak_basis": "shared-memory LSU: 32 x 4-B T-table lookups/clk/SM x 148 SMs x "
-                              f"{peaks['sm_max_mhz']:.0f} MHz (160 lookups per AES block)"}
-    if name in ("hmac_sha1",):
-        achieved = w["sha1_compressions"] * SHA1_OPS_PER_COMPRESSION / s / 1e9
-        peak = SM_COUNT * 64 * f / 1e9
-        return {"bound": "alu", "unit": "Gop/s", "achieved": achieved, "peak": peak,
-                "peak_basis": "ALU pipe: 64 int32 lanes/clk/SM x 148 SMs x "
-                              f"{peaks['sm_max_mhz']:.0f} MHz (597 ops per SHA-1 compression)"}
-    if name == "fused":
-        # lower bound = max(LSU time of AES, ALU time of SHA-1 + AES ALU share, HBM time)
-        t_lsu = w["aes_blocks"] * AES_LOOKUPS_PER_BLOCK / (SM_COUNT * 32 * f)
-        t_alu = w["sha1_compressions"] * SHA1_OPS_PER_COMPRESSION / (SM_COUNT * 64 * f)
-        t_hbm = (w["bytes_in"] + w["bytes_out"]) / (peaks["hbm_gbs"] * 1e9)
-        t_lb = max(t_lsu, t_alu, t_hbm)
-        return {"bound": "alu", "unit": "fraction-of-lower-bound", "achieved": t_lb / s,
-                "peak": 1.0,
-                "peak_basis": "max(AES LSU time, SHA-1 ALU time, HBM time) at max SM clock"}
+    alu_peak = SM_COUNT * ALU_LANES_PER_CLK_SM * f / 1e9            # Gop/s
+    aes_ops = w["aes_blocks"] * AES_ALU_OPS_PER_BLOCK
+    sha_ops = w["sha1_compressions"] * SHA1_ALU_OPS_PER_COMPRESSION
+    if name in ("fused", "aes_ctr", "hmac_sha1"):
+        ops = {"fused": aes_ops + sha_ops, "aes_ctr": aes_ops, "hmac_sha1": sha_ops}[name]
+        r = {"bound": "alu", "unit": "Gop/s", "achieved": ops / s / 1e9, "peak": alu_peak,
+             "peak_basis": f"integer ALU pipe: {ALU_LANES_PER_CLK_SM} lanes/clk/SM x {SM_COUNT} SMs x "
+                           f"{peaks['sm_max_mhz']:.0f} MHz (microbenchmarked 63.9 lanes/clk/SM); "
+                           f"work = {AES_ALU_OPS_PER_BLOCK} ops/AES block + "
+                           f"{SHA1_ALU_OPS_PER_COMPRESSION} ops/SHA-1 compression"}
+        if name in ("fused", "aes_ctr"):
+            lds = w["aes_blocks"] * AES_LOOKUPS_PER_BLOCK / s / 1e9
+            r["lds_lookups_gps"] = lds
+            r["lds_frac"] = lds / (SM_COUNT * LDS_LANES_PER_CLK_SM * f / 1e9)
+        return r
     # memory-bound kernels: algorithmic bytes
     if name == "gather":
         byts = w["bytes_in"] + w["rec_bytes"]
@@ -170,13 +178,14 @@ def kernel_roofline(name, ms_per_launch, w, peaks):
             "peak_basis": "measured HBM copy bandwidth"}
 
 
-def load_traffic(kernel):
+def load_traffic(kernel, cfg_name=None):
     """dram bytes per launch of `kernel` from the committed ncu summary, if any."""
     p = os.path.join(ROOT, "profiles", "ncu_kernels.json")
     try:
         with open(p) as f:
             d = json.load(f)
-        return d.get(kernel, {}).get("dram_bytes_per_launch")
+        key = f"{kernel}:{cfg_name}" if cfg_name else kernel
+        return d.get(key, d.get(kernel, {})).get("dram_bytes_per_launch")
     except Exception:
         return None
 
@@ -272,7 +281,9 @@ def run_ours(args):
     if dom:
         r = kern_roofs[dom]
         roof = {"kernel": dom, "bound": r["bound"], "achieved": r["achieved"], "peak": r["peak"],
-                "unit": r["unit"], "frac": r["frac"], "traffic": load_traffic(dom),
+                "unit": r["unit"], "frac": r["frac"],
+                "traffic": load_traffic(dom, gen.CONFIGS[main_cfg]["name"]),
+                "traffic_unit": "bytes per launch (ncu dram__bytes_read.sum + dram__bytes_write.sum)",
                 "peak_basis": r["peak_basis"], "peak_source": peaks["source"],
                 "share_of_step": kern_avg[dom] / max(sum(kern_avg.values()), 1e-12)}
 
@@ -287,14 +298,15 @@ def run_ours(args):
                 per_size[str(CFG_SIZE[cfg_id])] = {"gbps": agg["gbps"], "mpps": agg["mpps"],
                                                    "ms_per_step": agg["ms_per_step"]}
                 continue
-            r2 = measure(cfg_id, max(10, args.steps // 2), max(3, args.warmup // 2))
-            a2 = aggregate(r2, max(10, args.steps // 2))
+            r2 = measure(cfg_id, max(10, args.steps // 4), max(3, args.warmup // 2))
+            a2 = aggregate(r2, max(10, args.steps // 4))
             kk = {k: v / max(r2["nb"], 1) for k, v in r2["kern"].items()}
             w2 = work_model(r2["b"])
             rr = {}
             for k, ms in kk.items():
                 x = kernel_roofline(k, ms, w2, peaks)
-                rr[k] = {"ms": ms, "frac": x["achieved"] / x["peak"], "unit": x["unit"]}
+                rr[k] = {"ms": ms, "frac": x["achieved"] / x["peak"], "unit": x["unit"],
+                         "achieved": x["achieved"], "bound": x["bound"]}
             per_size[str(CFG_SIZE[cfg_id])] = {"gbps": a2["gbps"], "mpps": a2["mpps"],
                                                "ms_per_step": a2["ms_per_step"], "kernels": rr}
 
@@ -471,8 +483,8 @@ def run_reference(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=50)
-    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--config", type=int, default=2, choices=[2, 3, 4])
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--pipeline", type=int, default=None, help="0 fused, 1 unfused")
