@@ -48,16 +48,19 @@ __device__ __forceinline__ void grid_barrier(uint32_t *count, uint32_t *gen)
 __device__ __forceinline__ void scan_sa_column(const DevTable &T, const DevWork &W, uint32_t sa,
                                                uint32_t n_tiles, uint32_t n_sa, uint32_t lane)
 {
+    // all loads of the column first (one L2 round trip), then the shuffle scans
+    constexpr int U = 8;                       // 8 x 32 = 256 tiles per pass
     uint32_t carry = 0;
-    for (uint32_t t0 = 0; t0 < n_tiles; t0 += 128) {
-        uint32_t h[4];
+    for (uint32_t t0 = 0; t0 < n_tiles; t0 += 32u * U) {
+        uint32_t h[U];
 #pragma unroll
-        for (int u = 0; u < 4; u++) {
+        for (int u = 0; u < U; u++) {
             const uint32_t t = t0 + 32u * u + lane;
             h[u] = t < n_tiles ? __ldcg(&W.hist16[(size_t)t * n_sa + sa]) : 0u;
         }
 #pragma unroll
-        for (int u = 0; u < 4; u++) {
+        for (int u = 0; u < U; u++) {
+            if (t0 + 32u * u >= n_tiles) break;
             uint32_t x = h[u];
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {

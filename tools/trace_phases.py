@@ -36,5 +36,7 @@ for cfg in (2, 3, 4):
     import ctypes
     raw = np.zeros(148 * 8 + 64, np.uint64)
     nbm.lib.nba_ipsec_debug_trace(t._h, raw.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)), raw.size)
-    print("  chunk0 cycles: meta %d  rounds %d  final %d  stores %d" % tuple(int(x) for x in raw[148*8+8:148*8+12]))
+    for k, nm in ((0, "tid0 (shortest)"), (8, "last (longest)")):
+        v = [int(x) for x in raw[148*8+8+k:148*8+8+k+5]]
+        print("  lane %s cycles: setup %d  aes0 %d  emit0 %d  sha0 %d  rest %d" % (nm, *v))
     t.close()
