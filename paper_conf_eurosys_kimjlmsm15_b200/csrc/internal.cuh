@@ -45,8 +45,9 @@ struct DevWork {
     uint32_t *m_seq;        // [M]   ESP sequence number
     uint32_t *m_info;       // [M]   C | tos << 16 | INFO_OK  (0 = dropped / invalid)
     uint32_t *perm;         // [M]   HMAC processing order (length-binned)
-    uint16_t *hist16;       // [max_ptiles * n_sa] per-prologue-tile per-SA packet counts
-    uint32_t *hpfx;         // [max_ptiles * n_sa] exclusive prefix of hist16 down each SA column
+    uint16_t *hist16;       // [n_sa][n_tiles] per-SA per-prologue-tile packet counts (SA-major;
+                            //   all-zero between batches)
+    uint32_t *hpfx;         // [n_sa][n_tiles] exclusive prefix of hist16 along each SA row
     uint32_t *tile_rec;     // [max_tiles] record chunks per tile -> exclusive prefix
     uint32_t *tile_blk;     // [max_tiles] AES blocks per tile -> exclusive prefix
     uint32_t *tile_bin;     // [max_tiles * NBINS] HMAC length bins per tile -> prefix

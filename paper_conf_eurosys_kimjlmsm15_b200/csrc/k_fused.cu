@@ -471,6 +471,20 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc)
     FusedHi &H = *reinterpret_cast<FusedHi *>(smem + toff + AES_TABLE_BYTES);
     const uint32_t lane4r = (lane * 4u) | (smem_u32(tabs) & 0xffff0000u);
 
+    // warm L2 with the SA table (round keys, midstates, header words) while the
+    // prologue runs: each CTA prefetches a slice of the 128-byte lines
+    {
+        const uint32_t nl_rk = (T.n_sa * 176u + 127u) >> 7;
+        const uint32_t nl_hm = (T.n_sa * 48u + 127u) >> 7;
+        const uint32_t nl_hd = (T.n_sa * 16u + 127u) >> 7;
+        const uint32_t nl = nl_rk + nl_hm + nl_hd;
+        for (uint32_t l = blockIdx.x * blockDim.x + tid; l < nl; l += gridDim.x * blockDim.x) {
+            const uint8_t *a = l < nl_rk ? reinterpret_cast<const uint8_t *>(T.rk) + 128u * l
+                             : l < nl_rk + nl_hm ? reinterpret_cast<const uint8_t *>(T.hmid) + 128u * (l - nl_rk)
+                                                 : reinterpret_cast<const uint8_t *>(T.sahdr) + 128u * (l - nl_rk - nl_hm);
+            prefetch_l2(a);
+        }
+    }
     aes_tables_to_smem(tabs, T.te0);
     if (tid < 4) L.cnt[tid] = 0ull;
 
@@ -505,7 +519,7 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc)
             uint32_t info = 0, bin = NBINS - 1, q32 = 0;
             if (cand) {
                 const unsigned long long q = (unsigned long long)T.seq_prev[sa] + 1ull +
-                                             W.hpfx[(size_t)(i / PTILE) * n_sa + sa] + W.lrank[i];
+                                             W.hpfx[(size_t)sa * ((B.n + PTILE - 1) / PTILE) + i / PTILE] + W.lrank[i];
                 if (q <= 0xffffffffull) {   // RFC 4303 §3.3.3: never cycle
                     q32 = (uint32_t)q;
                     info = D | (tos << 16) | INFO_OK;

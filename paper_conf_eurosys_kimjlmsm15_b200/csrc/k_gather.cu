@@ -78,7 +78,7 @@ k_gather(DevTable T, DevWork W, BatchArgs B, uint32_t aes_grid)
             rec16 = esp_rec16(C);
             nblk = esp_nblk(C);
             unsigned long long q = (unsigned long long)T.seq_prev[s] + 1ull +
-                                   W.hpfx[(size_t)tile * n_sa + s] + W.lrank[i];
+                                   W.hpfx[(size_t)s * gridDim.x + tile] + W.lrank[i];
             q32 = (uint32_t)q;
             uint32_t tos = B.in_buf[B.in_off[i] + 1];
             info = C | (tos << 16) | (q <= 0xffffffffull ? INFO_OK : 0u);

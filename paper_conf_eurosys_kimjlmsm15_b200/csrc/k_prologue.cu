@@ -46,17 +46,19 @@ __device__ __forceinline__ void grid_barrier(uint32_t *count, uint32_t *gen)
 // Exclusive prefix of the tile counts down SA column `sa` by one warp, then the
 // SA counter advance (only the first (2^32-1 - seq) packets get numbers).
 __device__ __forceinline__ void scan_sa_column(const DevTable &T, const DevWork &W, uint32_t sa,
-                                               uint32_t n_tiles, uint32_t n_sa, uint32_t lane)
+                                               uint32_t n_tiles, uint32_t lane)
 {
-    // all loads of the column first (one L2 round trip), then the shuffle scans
+    // the column is contiguous (SA-major): coalesced loads, all issued first
     constexpr int U = 8;                       // 8 x 32 = 256 tiles per pass
+    uint16_t *col = W.hist16 + (size_t)sa * n_tiles;
+    uint32_t *pfx = W.hpfx + (size_t)sa * n_tiles;
     uint32_t carry = 0;
     for (uint32_t t0 = 0; t0 < n_tiles; t0 += 32u * U) {
         uint32_t h[U];
 #pragma unroll
         for (int u = 0; u < U; u++) {
             const uint32_t t = t0 + 32u * u + lane;
-            h[u] = t < n_tiles ? __ldcg(&W.hist16[(size_t)t * n_sa + sa]) : 0u;
+            h[u] = t < n_tiles ? __ldcg(&col[t]) : 0u;
         }
 #pragma unroll
         for (int u = 0; u < U; u++) {
@@ -68,7 +70,10 @@ __device__ __forceinline__ void scan_sa_column(const DevTable &T, const DevWork 
                 if (lane >= (uint32_t)o) x += y;
             }
             const uint32_t t = t0 + 32u * u + lane;
-            if (t < n_tiles) W.hpfx[(size_t)t * n_sa + sa] = carry + x - h[u];
+            if (t < n_tiles) {
+                pfx[t] = carry + x - h[u];
+                if (h[u]) col[t] = 0;            // re-arm for the next batch
+            }
             carry += __shfl_sync(0xffffffffu, x, 31);
         }
     }
@@ -165,7 +170,11 @@ k_prologue(DevTable T, DevWork W, BatchArgs B, uint32_t n_tiles, bool unfused, b
         __syncthreads();
     }
     if (i < B.n) W.lrank[i] = base + wrank;
-    for (uint32_t k = tid; k < n_sa; k += PTILE) W.hist16[(size_t)tile * n_sa + k] = s_hist[k];
+    // SA-major tile counts, nonzero entries only (the column scan re-zeroes what
+    // it reads, so the matrix is all-zero between batches): the packet with the
+    // tile's highest rank for its SA writes that SA's count
+    if (s != INVALID_SA && base + wrank + 1u == s_hist[s])
+        W.hist16[(size_t)s * n_tiles + tile] = s_hist[s];
 
     if (unfused) {
         if (i < B.n) atomicAdd(&s_bin[hmac_bin(s != INVALID_SA, C)], 1u);
@@ -189,7 +198,7 @@ k_prologue(DevTable T, DevWork W, BatchArgs B, uint32_t n_tiles, bool unfused, b
         asm volatile("griddepcontrol.launch_dependents;");
         const uint32_t nwarps = gridDim.x * (PTILE / 32u);
         for (uint32_t col = tile * (PTILE / 32u) + warp; col < n_sa; col += nwarps)
-            scan_sa_column(T, W, col, n_tiles, n_sa, lane);
+            scan_sa_column(T, W, col, n_tiles, lane);
         if (unfused && tile == 0) scan_tile_totals(W, n_tiles, s_scr);
     } else {
         // ---- phase 2 on the last CTA to finish phase 1 -----------------------
@@ -202,7 +211,7 @@ k_prologue(DevTable T, DevWork W, BatchArgs B, uint32_t n_tiles, bool unfused, b
         __threadfence();
         if (tr && tid == 0) tr[2] = gtimer();
         for (uint32_t col = warp; col < n_sa; col += PTILE / 32u)
-            scan_sa_column(T, W, col, n_tiles, n_sa, lane);
+            scan_sa_column(T, W, col, n_tiles, lane);
         if (unfused) scan_tile_totals(W, n_tiles, s_scr);
         __syncthreads();
         if (tid == 0) W.ctl[CTL_TICKET] = 0;            // re-arm for the next batch
