@@ -60,6 +60,25 @@ class Counters(ctypes.Structure):
         return {k: int(getattr(self, k)) for k, _ in self._fields_}
 
 
+IN_OK, IN_DROP_SA, IN_DROP_FORMAT, IN_DROP_REPLAY, IN_DROP_AUTH, IN_DROP_TRAILER = range(6)
+REPLAY_WINDOW = 64
+
+
+class Replay(ctypes.Structure):
+    _fields_ = [("top", ctypes.c_uint32), ("pad_", ctypes.c_uint32), ("bitmap", ctypes.c_uint64)]
+
+
+class InCounters(ctypes.Structure):
+    _fields_ = [("pkts_ok", ctypes.c_uint64), ("drop_sa", ctypes.c_uint64),
+                ("drop_format", ctypes.c_uint64), ("drop_replay", ctypes.c_uint64),
+                ("drop_auth", ctypes.c_uint64), ("drop_trailer", ctypes.c_uint64),
+                ("bytes_in", ctypes.c_uint64), ("bytes_out", ctypes.c_uint64),
+                ("batches", ctypes.c_uint64)]
+
+    def as_dict(self):
+        return {k: int(getattr(self, k)) for k, _ in self._fields_}
+
+
 def lib():
     global _lib
     with _lock:
@@ -87,6 +106,12 @@ def lib():
             L.oracle_process_batch_mt.argtypes = batch_args + [ctypes.c_int]
             L.oracle_decap.restype = ctypes.c_int
             L.oracle_decap.argtypes = [P(SA), u8p, ctypes.c_uint32, u8p, u32p, u32p]
+            L.oracle_replay_init.restype = None
+            L.oracle_replay_init.argtypes = [P(SA), P(Replay)]
+            L.oracle_process_inbound.restype = None
+            L.oracle_process_inbound.argtypes = [P(SA), P(Replay), ctypes.c_uint32, u8p, u32p, u16p,
+                                                 u32p, u8p, u32p, u16p, u8p, ctypes.c_uint32,
+                                                 P(InCounters)]
             L.oracle_init()
             _lib = L
     return _lib
@@ -217,3 +242,44 @@ def decap(sas, s: int, pkt: bytes):
     rc = lib().oracle_decap(ctypes.byref(sas[s]), _ptr(p), p.size, _ptr(inner),
                             ctypes.byref(ilen), ctypes.byref(seq))
     return rc, inner[:ilen.value].tobytes(), seq.value
+
+
+# --- ESP inbound -------------------------------------------
+
+def make_windows(sas, n_sa: int) -> "ctypes.Array":
+    """Per-SA anti-replay windows initialised from the SAs' ``seq`` (reading B6)."""
+    arr = (Replay * max(n_sa, 1))()
+    for s in range(n_sa):
+        lib().oracle_replay_init(ctypes.byref(sas[s]), ctypes.byref(arr[s]))
+    return arr
+
+
+def window_state(win, n_sa: int):
+    top = np.array([win[s].top for s in range(n_sa)], dtype=np.uint32)
+    bmp = np.array([win[s].bitmap for s in range(n_sa)], dtype=np.uint64)
+    return top, bmp
+
+
+def process_inbound(sas, win, n_sa: int, batch, out_pool_bytes: int | None = None,
+                    counters: InCounters | None = None):
+    """Sequential ESP inbound over ``batch`` (a gen.Batch whose in_buf holds ESP
+    tunnel packets).  ``win`` is updated in place.  Returns
+    (out_buf, out_len, status, counters); only out_buf[out_off[i] : +out_len[i]]
+    is defined."""
+    n = int(batch.n)
+    in_buf = np.ascontiguousarray(batch.in_buf, np.uint8)
+    in_off = np.ascontiguousarray(batch.in_off, np.uint32)
+    in_len = np.ascontiguousarray(batch.in_len, np.uint16)
+    sa_idx = np.ascontiguousarray(batch.sa_idx, np.uint32)
+    out_off = np.ascontiguousarray(batch.out_off, np.uint32)
+    size = out_pool_bytes if out_pool_bytes is not None else batch.out_pool_bytes
+    out_buf = np.zeros(max(size, 1), np.uint8)
+    out_len = np.zeros(max(n, 1), np.uint16)
+    status = np.zeros(max(n, 1), np.uint8)
+    ctr = counters if counters is not None else InCounters()
+    lib().oracle_process_inbound(sas, win, n_sa, _ptr(in_buf), _ptr(in_off, ctypes.c_uint32),
+                                 _ptr(in_len, ctypes.c_uint16), _ptr(sa_idx, ctypes.c_uint32),
+                                 _ptr(out_buf), _ptr(out_off, ctypes.c_uint32),
+                                 _ptr(out_len, ctypes.c_uint16), _ptr(status), n,
+                                 ctypes.byref(ctr))
+    return out_buf, out_len[:n], status[:n], ctr

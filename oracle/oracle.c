@@ -485,3 +485,133 @@ int oracle_decap(const oracle_sa *sa, const uint8_t *pkt, uint32_t len,
     free(T);
     return rc;
 }
+
+/* ------------------------------------------------------------------------ */
+/* ESP inbound, sequential.  RFC 4303 §3.4 in its order:    */
+/* §3.4.1 no fragments, §3.4.2 SA (caller's sa_idx, SPI must match),         */
+/* §3.4.3 sequence number / anti-replay check, §3.4.4.1 ICV check, then the  */
+/* receive window update ("only if the integrity verification succeeds"),   */
+/* §3.4.4.2 decryption, §2.4 / §2.6 trailer checks, output of the inner      */
+/* datagram.  Readings B1..B9 are listed in DESIGN.md.                       */
+/* ------------------------------------------------------------------------ */
+
+/* B6: the window starts at the SA's `seq` with everything at or below it
+ * counted as received (a resumed SA); seq = 0 gives an empty window. */
+void oracle_replay_init(const oracle_sa *sa, oracle_replay *w)
+{
+    w->top = sa->seq;
+    w->pad_ = 0;
+    w->bitmap = sa->seq ? ~(uint64_t)0 : 0;
+}
+
+/* RFC 4303 §3.4.3: right edge `top` = highest authenticated number; bit d of
+ * the bitmap records number top - d (d < 64).  Zero is never sent (§3.3.3). */
+static int replay_check(const oracle_replay *w, uint32_t q)
+{
+    if (q == 0) return 0;
+    if (q > w->top) return 1;                       /* right of the window: new */
+    uint32_t d = w->top - q;
+    if (d >= ORACLE_REPLAY_WINDOW) return 0;        /* left of the window: too old */
+    return ((w->bitmap >> d) & 1u) ? 0 : 1;         /* inside: not seen before */
+}
+
+static void replay_update(oracle_replay *w, uint32_t q)
+{
+    if (q > w->top) {                               /* slide the window right */
+        uint32_t shift = q - w->top;
+        w->bitmap = shift >= ORACLE_REPLAY_WINDOW ? 0 : (w->bitmap << shift);
+        w->bitmap |= 1u;
+        w->top = q;
+    } else {
+        w->bitmap |= (uint64_t)1 << (w->top - q);
+    }
+}
+
+static uint32_t be32_at(const uint8_t *p)
+{
+    return ((uint32_t)p[0] << 24) | ((uint32_t)p[1] << 16) | ((uint32_t)p[2] << 8) | p[3];
+}
+
+/* One packet; returns its ORACLE_IN_* status and the inner length in *D_out. */
+static int inbound_one(const oracle_sa *sa, oracle_replay *w, const uint8_t *pkt, uint32_t L,
+                       uint8_t *out, uint32_t *D_out)
+{
+    /* B2: outer IPv4 without options, not a fragment (§3.4.1), protocol ESP,
+     * total length = the caller's length, valid header checksum (RFC 1071) */
+    if (L < 48u + 24u || L > 48u + 1504u || (L - 48u) % 4u != 0) return ORACLE_IN_DROP_FORMAT;
+    if (pkt[0] != 0x45 || pkt[9] != 50) return ORACLE_IN_DROP_FORMAT;
+    if ((((uint32_t)pkt[2] << 8) | pkt[3]) != L) return ORACLE_IN_DROP_FORMAT;
+    if (((((uint32_t)pkt[6] << 8) | pkt[7]) & 0x3fffu) != 0) return ORACLE_IN_DROP_FORMAT;
+    if (oracle_ipv4_checksum(pkt, 20) != 0) return ORACLE_IN_DROP_FORMAT;
+    const uint8_t *H = pkt + 20;                     /* SPI || seq || IV */
+    if (be32_at(H) != sa->spi) return ORACLE_IN_DROP_FORMAT;     /* §3.4.2 */
+    const uint32_t C = L - 48u;
+    const uint32_t q = be32_at(H + 4);
+
+    /* §3.4.3: sequence number check before the ICV */
+    if (!replay_check(w, q)) return ORACLE_IN_DROP_REPLAY;
+
+    /* §3.4.4.1: ICV = HMAC-SHA1(H || E)[0:12], compared without early exit */
+    uint8_t mac[20];
+    oracle_hmac_sha1(sa->hmac_key, 20, H, 16u + C, mac);
+    uint8_t diff = 0;
+    for (int j = 0; j < 12; j++) diff |= (uint8_t)(mac[j] ^ H[16u + C + (uint32_t)j]);
+    if (diff) return ORACLE_IN_DROP_AUTH;
+
+    /* §3.4.3: the window advances only for authenticated packets */
+    replay_update(w, q);
+
+    /* §3.4.4.2: T = E xor keystream; counter block nonce || IV(from packet) || BE32(1..) */
+    uint8_t icb[16];
+    memcpy(icb, sa->ctr_nonce, 4);
+    memcpy(icb + 4, H + 8, 8);
+    put_be32(icb + 12, 1);
+    uint8_t *T = (uint8_t *)malloc(C);
+    if (!T) return ORACLE_IN_DROP_FORMAT;
+    oracle_ctr_xcrypt(sa->aes_key, icb, H + 16, C, T);
+
+    /* B4: next header 4 (tunnel mode), pad bytes 1..p (§2.4), D >= 20 */
+    int rc = ORACLE_IN_OK;
+    const uint32_t p = T[C - 2];
+    if (T[C - 1] != 4 || p + 2u + ORACLE_MIN_DATAGRAM > C) rc = ORACLE_IN_DROP_TRAILER;
+    const uint32_t D = C - 2u - p;
+    for (uint32_t j = 1; rc == ORACLE_IN_OK && j <= p; j++)
+        if (T[D + j - 1] != (uint8_t)j) rc = ORACLE_IN_DROP_TRAILER;
+    if (rc == ORACLE_IN_OK) {
+        memcpy(out, T, D);
+        *D_out = D;
+    }
+    free(T);
+    return rc;
+}
+
+void oracle_process_inbound(const oracle_sa *sas, oracle_replay *win, uint32_t n_sa,
+                            const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
+                            const uint32_t *sa_idx, uint8_t *out_buf, const uint32_t *out_off,
+                            uint16_t *out_len, uint8_t *status, uint32_t n,
+                            oracle_in_counters *ctr)
+{
+    sbox_init();
+    for (uint32_t i = 0; i < n; i++) {
+        const uint32_t s = sa_idx[i];
+        uint32_t D = 0;
+        int rc = s < n_sa ? inbound_one(&sas[s], &win[s], in_buf + in_off[i], in_len[i],
+                                        out_buf + out_off[i], &D)
+                          : ORACLE_IN_DROP_SA;
+        status[i] = (uint8_t)rc;
+        out_len[i] = rc == ORACLE_IN_OK ? (uint16_t)D : 0;
+        switch (rc) {
+        case ORACLE_IN_OK:
+            ctr->pkts_ok++;
+            ctr->bytes_in += in_len[i];
+            ctr->bytes_out += D;
+            break;
+        case ORACLE_IN_DROP_SA: ctr->drop_sa++; break;
+        case ORACLE_IN_DROP_FORMAT: ctr->drop_format++; break;
+        case ORACLE_IN_DROP_REPLAY: ctr->drop_replay++; break;
+        case ORACLE_IN_DROP_AUTH: ctr->drop_auth++; break;
+        default: ctr->drop_trailer++; break;
+        }
+    }
+    if (n) ctr->batches++;
+}

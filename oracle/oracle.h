@@ -51,4 +51,26 @@ int      oracle_process_batch_mt(oracle_sa *sas, uint32_t n_sa, const uint8_t *i
                                  oracle_counters *ctr, int n_threads);
 int      oracle_decap(const oracle_sa *sa, const uint8_t *pkt, uint32_t len, uint8_t *inner,
                       uint32_t *inner_len, uint32_t *seq_out);
+
+/* ---- ESP inbound (readings B1..B9) ------------ */
+#define ORACLE_IN_OK           0
+#define ORACLE_IN_DROP_SA      1   /* sa_idx >= n_sa                              */
+#define ORACLE_IN_DROP_FORMAT  2   /* outer header / length / SPI                 */
+#define ORACLE_IN_DROP_REPLAY  3   /* RFC 4303 §3.4.3 sequence number check       */
+#define ORACLE_IN_DROP_AUTH    4   /* RFC 4303 §3.4.4.1 ICV mismatch              */
+#define ORACLE_IN_DROP_TRAILER 5   /* pad contents / pad length / next header     */
+#define ORACLE_REPLAY_WINDOW  64u  /* RFC 4303 §3.4.3: 64 SHOULD be the default   */
+
+typedef struct { uint32_t top; uint32_t pad_; uint64_t bitmap; } oracle_replay;
+typedef struct {
+    uint64_t pkts_ok, drop_sa, drop_format, drop_replay, drop_auth, drop_trailer;
+    uint64_t bytes_in, bytes_out, batches;
+} oracle_in_counters;
+
+void     oracle_replay_init(const oracle_sa *sa, oracle_replay *w);
+void     oracle_process_inbound(const oracle_sa *sas, oracle_replay *win, uint32_t n_sa,
+                                const uint8_t *in_buf, const uint32_t *in_off,
+                                const uint16_t *in_len, const uint32_t *sa_idx, uint8_t *out_buf,
+                                const uint32_t *out_off, uint16_t *out_len, uint8_t *status,
+                                uint32_t n, oracle_in_counters *ctr);
 #endif

@@ -487,6 +487,8 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc)
     }
     aes_tables_to_smem(tabs, T.te0);
     if (tid < 4) L.cnt[tid] = 0ull;
+    if (tid < NBINS) L.bins[tid] = 0;   // re-zeroed after each use (below)
+    __syncthreads();
 
     const uint32_t p_begin = blockIdx.x * ppc;
     const uint32_t p_end = min(B.n, p_begin + ppc);
@@ -496,7 +498,6 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc)
     for (uint32_t base = p_begin; base < p_end; base += F_SUPER) {
         const uint32_t cnt_pk = min((uint32_t)F_SUPER, p_end - base);
         // ---- 1. metadata (thread j <-> packet base + j) ---------------------
-        if (tid < NBINS) L.bins[tid] = 0;
         const uint32_t j = tid;
         const uint32_t i = base + j;
         // 1a. everything that does not depend on the prologue (overlaps it under
@@ -549,6 +550,7 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc)
             L.perm[atomicAdd(&L.bins[bin], 1u)] = (uint16_t)j;
         }
         __syncthreads();
+        if (tid < NBINS) L.bins[tid] = 0;   // next round's counts (after its barrier)
         if (tr && tid == 0 && base == p_begin) tr[1] = gtimer();
 
         // ---- 2. one lane per packet; the longest packets go to the HIGHEST warps

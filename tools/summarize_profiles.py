@@ -83,7 +83,9 @@ def main(tag):
                   "| kernel | us | DRAM rd MB | DRAM wr MB | issue % | ALU % | FMA % | LSU % | smem wavefronts | bank conflicts | warp inst | regs |",
                   "|---|---|---|---|---|---|---|---|---|---|---|---|"]
         for k, ds in agg.items():
-            d = ds[-1]
+            d = collections.defaultdict(lambda: float("nan"))
+            d.update({m: (v if isinstance(v, float) else float("nan")) for m, v in ds[-1].items()
+                      if m != "kernel"})
             lines.append(
                 f"| {k} | {d['duration'] * 1e6:.1f} | {d['dram_read'] / 1e6:.2f} | {d['dram_write'] / 1e6:.2f} | "
                 f"{d['issue_active_pct']:.1f} | {d['alu_pipe_pct']:.1f} | {d['fma_pipe_pct']:.1f} | "
@@ -98,7 +100,10 @@ def main(tag):
         lines += ["## c3_1514B_1024sa (unfused ablation: gather / AES / HMAC / scatter)", "",
                   "| kernel | us | DRAM rd MB | DRAM wr MB | issue % | ALU % | LSU % | bank conflicts |",
                   "|---|---|---|---|---|---|---|---|"]
-        for d in raw(rep):
+        for d0 in raw(rep):
+            d = collections.defaultdict(lambda: float("nan"))
+            d.update({m: (v if isinstance(v, float) else float("nan")) for m, v in d0.items()})
+            d["kernel"] = d0["kernel"]
             lines.append(f"| {d['kernel']} | {d['duration'] * 1e6:.1f} | {d['dram_read'] / 1e6:.2f} | "
                          f"{d['dram_write'] / 1e6:.2f} | {d['issue_active_pct']:.1f} | "
                          f"{d['alu_pipe_pct']:.1f} | {d['lsu_inst_pct']:.1f} | {d['shared_bank_conflicts']:.3g} |")
