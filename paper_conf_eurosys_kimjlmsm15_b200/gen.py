@@ -201,3 +201,65 @@ CONFIGS = {
     4: dict(name="c4_imix_1024sa", n=65536, size="imix", n_sa=1024),
 }
 SWEEP_SIZES = (64, 128, 256, 512, 1024, 1514, "imix")   # configs[4]
+
+
+# --- inbound (ESP decapsulation) traffic -------------------
+# An inbound batch is a sequence of ESP tunnel packets.  They are produced by an
+# OUTBOUND run (the oracle's in tests, the library's own in bench.py); this
+# module only rearranges those bytes -- arrival order, replays, corruption --
+# and holds no ESP arithmetic.
+
+def arrival_order(n_src: int, n: int, r: np.random.Generator, reorder: int = 0,
+                  dup: float = 0.0, old: float = 0.0, old_span: int = 4096) -> np.ndarray:
+    """Indices into the source packets for n arrivals: the source order, with
+    local reordering inside windows of `reorder` packets, a fraction `dup`
+    replaced by a recent earlier arrival (replayed duplicates) and a fraction
+    `old` by one from up to `old_span` arrivals back (stale replays)."""
+    idx = np.arange(n, dtype=np.int64) % max(n_src, 1)
+    if reorder > 1:
+        for s in range(0, n, reorder):
+            seg = idx[s:s + reorder]
+            idx[s:s + reorder] = seg[r.permutation(seg.size)]
+    pos = np.arange(n, dtype=np.int64)
+    u = r.random(n)
+    d = (u < dup) & (pos > 0)
+    idx[d] = idx[pos[d] - r.integers(1, 1 + np.minimum(pos[d], 256))]
+    o = (u >= dup) & (u < dup + old) & (pos > 0)
+    idx[o] = idx[pos[o] - r.integers(1, 1 + np.minimum(pos[o], old_span))]
+    return idx
+
+
+def esp_batch(src_buf: np.ndarray, src_off: np.ndarray, src_len: np.ndarray,
+              src_sa: np.ndarray, order: np.ndarray, corrupt: float = 0.0,
+              r: np.random.Generator | None = None, layout: str = "slots") -> Batch:
+    """Inbound batch whose packet j is source packet order[j] copied verbatim
+    (slot layout as make_batch: in_off = 2048 j + 142, same for out_off).  A
+    fraction `corrupt` of the packets gets one random byte XOR-ed with a random
+    nonzero value.  frame_len = in_len + 14 (Ethernet, reading A2)."""
+    order = np.asarray(order, np.int64)
+    n = int(order.size)
+    L = np.asarray(src_len, np.int64)[order]
+    if layout == "slots":
+        in_off = SLOT * np.arange(n, dtype=np.int64) + HEADROOM + ETH
+        pool = SLOT * max(n, 1)
+        out_off, out_pool = in_off.copy(), pool
+    elif layout == "packed":
+        in_off = np.concatenate([[0], np.cumsum(L)[:-1]]) if n else np.zeros(0, np.int64)
+        pool = int(L.sum()) + 16
+        out_off, out_pool = in_off.copy(), pool
+    else:
+        raise ValueError(layout)
+    buf = np.zeros(pool, np.uint8)
+    so = np.asarray(src_off, np.int64)[order]
+    for j in range(n):
+        buf[in_off[j]:in_off[j] + L[j]] = src_buf[so[j]:so[j] + L[j]]
+    if corrupt > 0 and n:
+        r = r if r is not None else rng_for(0, salt=7)
+        hit = np.nonzero(r.random(n) < corrupt)[0]
+        for j in hit:
+            if L[j] > 0:
+                buf[in_off[j] + int(r.integers(0, L[j]))] ^= np.uint8(r.integers(1, 256))
+    return Batch(n=n, in_buf=buf, in_off=in_off.astype(np.uint32), in_len=L.astype(np.uint16),
+                 sa_idx=np.asarray(src_sa, np.int64)[order].astype(np.uint32),
+                 out_off=out_off.astype(np.uint32), out_pool_bytes=int(out_pool),
+                 frame_len=(L + ETH).astype(np.uint32))
