@@ -165,6 +165,79 @@ int nba_ipsec_debug_trace(nba_ipsec_sa_table *t, uint64_t *host, uint32_t n_word
 void nba_ipsec_host_aes128_key_schedule(const uint8_t key[16], uint32_t w[44]);
 void nba_ipsec_host_hmac_sha1_midstates(const uint8_t key[20], uint32_t hin[5], uint32_t hout[5]);
 
+/* ---- ESP inbound: the mirror of the path ------------------
+ *
+ * RFC 4303 §3.4 receive processing in tunnel mode on the same SA table (the
+ * SAs' keys; the receive state is separate from the outbound counter).  Per
+ * packet i with s = sa_idx[i] and the outer IPv4 datagram of L = in_len[i]
+ * bytes at in_buf + in_off[i] (readings B1..B9):
+ *   1. s >= n_sa                                           -> DROP_SA
+ *   2. format (§3.4.1-§3.4.2): 72 <= L <= 1552, C = L - 48 = 0 mod 4, version/IHL
+ *      0x45, total length L, not a fragment, protocol 50, header checksum
+ *      valid (RFC 1071), SPI = spi_s                       -> else DROP_FORMAT
+ *   3. anti-replay (§3.4.3), window of NBA_IPSEC_REPLAY_WINDOW = 64 numbers:
+ *      q = 0, q left of the window or already received     -> DROP_REPLAY
+ *   4. ICV (§3.4.4.1): HMAC-SHA1-96 over SPI..ciphertext   -> else DROP_AUTH
+ *   5. the window records q (only authenticated packets move it)
+ *   6. decrypt (§3.4.4.2): AES-128-CTR, counter block nonce || IV (from the
+ *      packet) || BE32(k+1) (RFC 3686)
+ *   7. trailer: next header 4, pad bytes 1..p (§2.4), D = C - 2 - p >= 20
+ *                                                          -> else DROP_TRAILER
+ *   8. out_buf + out_off[i] <- the inner datagram (D bytes), out_len[i] = D.
+ * The batch result equals processing the packets one by one in index order.
+ * Window start (reading B6): an SA created with seq = s0 > 0 counts every
+ * number <= s0 as received; s0 = 0 gives an empty window.
+ * Slots: capacity >= in_len[i] - 48.  The library may write bytes [0, in_len[i]
+ * - 48) of EVERY slot whose packet passes step 2 (decryption runs in parallel
+ * with the ICV check, RFC 4303 §3.4.4.1); only [0, out_len[i]) is defined and
+ * out_len[i] = 0 marks a dropped packet.  status (optional, may be NULL)
+ * receives the NBA_IPSEC_IN_* code per packet. */
+enum {
+    NBA_IPSEC_IN_OK = 0,
+    NBA_IPSEC_IN_DROP_SA = 1,
+    NBA_IPSEC_IN_DROP_FORMAT = 2,
+    NBA_IPSEC_IN_DROP_REPLAY = 3,
+    NBA_IPSEC_IN_DROP_AUTH = 4,
+    NBA_IPSEC_IN_DROP_TRAILER = 5
+};
+#define NBA_IPSEC_REPLAY_WINDOW 64u
+
+typedef struct {
+    const uint8_t  *in_buf;
+    const uint32_t *in_off;
+    const uint16_t *in_len;     /* outer datagram length L */
+    const uint32_t *sa_idx;
+    uint8_t        *out_buf;
+    const uint32_t *out_off;
+    uint16_t       *out_len;    /* written: D, or 0 if dropped */
+    uint8_t        *status;     /* written if not NULL */
+    uint32_t        n_pkts;
+} nba_ipsec_in_batch;
+
+typedef struct {
+    uint64_t pkts_ok, drop_sa, drop_format, drop_replay, drop_auth, drop_trailer;
+    uint64_t bytes_in, bytes_out, batches;
+} nba_ipsec_in_counters;
+
+/* Allocate the inbound state (receive windows initialised from the SAs' seq)
+ * and workspace for max_batch_pkts packets.  Synchronous; idempotent.
+ * NBA_IPSEC_ENOMEM if allocation fails. */
+int nba_ipsec_enable_inbound(nba_ipsec_sa_table *t);
+/* Enqueue ESP inbound for one batch (DEVICE pointers) on `cuda_stream`; three
+ * kernel launches (decrypt+verify, replay scan, decide).  Same ordering rules
+ * as process_batch.  NBA_IPSEC_EINVAL if inbound is not enabled, for NULL
+ * arrays with n_pkts > 0 or n_pkts > max_batch_pkts. */
+int nba_ipsec_process_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batch *b, void *cuda_stream);
+/* Inbound counters since enable.  Synchronises `cuda_stream`. */
+int nba_ipsec_read_in_counters(nba_ipsec_sa_table *t, nba_ipsec_in_counters *out, void *cuda_stream);
+/* Receive windows: top[s] = highest authenticated number, bitmap[s] bit d set
+ * iff number top[s] - d was received.  n_sa entries each.  Synchronises. */
+int nba_ipsec_read_replay_window(nba_ipsec_sa_table *t, uint32_t *top, uint64_t *bitmap,
+                                 void *cuda_stream);
+/* As nba_ipsec_profile_read, for the inbound kernels (in_fused, in_replay, in_decide). */
+int nba_ipsec_profile_read_inbound(nba_ipsec_sa_table *t, double *ms, const char **names, int max,
+                                   int *n_kernels, uint32_t *n_batches);
+
 #ifdef __cplusplus
 }
 #endif

@@ -28,6 +28,7 @@ constexpr int MAX_KERNELS = 8;
 struct ProfSet {
     cudaEvent_t ev[MAX_KERNELS + 1] = {};
     int n_ev = 0;          // events recorded in this set (0 = empty)
+    bool inbound = false;
 };
 
 }  // namespace
@@ -53,6 +54,13 @@ struct nba_ipsec_sa_table {
     uint32_t prof_batches = 0;
     double prof_ms[MAX_KERNELS] = {};
     int prof_nk = 0;
+    // ESP inbound (nba_ipsec_enable_inbound)
+    std::vector<uint32_t> seq0;     // the SAs' initial seq (window start, reading B6)
+    bool in_enabled = false, in_gridsync = false;
+    uint32_t in_hcap = 0;
+    InState S{};
+    double prof_in_ms[3] = {};
+    uint32_t prof_in_batches = 0;
 };
 
 namespace {
@@ -99,10 +107,19 @@ void prof_drain_set(nba_ipsec_sa_table *t, ProfSet &s)
     cudaEventSynchronize(s.ev[s.n_ev - 1]);
     for (int k = 0; k + 1 < s.n_ev; k++) {
         float ms = 0.f;
-        if (cudaEventElapsedTime(&ms, s.ev[k], s.ev[k + 1]) == cudaSuccess) t->prof_ms[k] += ms;
+        if (cudaEventElapsedTime(&ms, s.ev[k], s.ev[k + 1]) != cudaSuccess) continue;
+        if (s.inbound) {
+            if (k < 3) t->prof_in_ms[k] += ms;
+        } else {
+            t->prof_ms[k] += ms;
+        }
     }
-    t->prof_nk = s.n_ev - 1;
-    t->prof_batches++;
+    if (s.inbound) {
+        t->prof_in_batches++;
+    } else {
+        t->prof_nk = s.n_ev - 1;
+        t->prof_batches++;
+    }
     s.n_ev = 0;
 }
 
@@ -168,6 +185,7 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
         hdr[s] = make_uint4(be_img(p.spi), nonce, be_img(p.tunnel_src), be_img(p.tunnel_dst));
         seq[s] = p.seq;
     }
+    t->seq0 = seq;
 
     uint4 *d_rk = nullptr, *d_hm = nullptr, *d_hdr = nullptr;
     uint32_t *d_seq = nullptr, *d_seq_prev = nullptr, *d_te0 = nullptr;
@@ -234,6 +252,7 @@ static int enqueue(nba_ipsec_sa_table *t, const BatchArgs &B, cudaStream_t st)
         for (int k = 0; k < MAX_KERNELS + 1; k++)
             if (!ps->ev[k]) cudaEventCreate(&ps->ev[k]);
         ps->n_ev = 0;
+        ps->inbound = false;
     }
     auto mark = [&]() {
         if (ps) cudaEventRecord(ps->ev[ps->n_ev++], st);
@@ -436,6 +455,8 @@ int nba_ipsec_profile_enable(nba_ipsec_sa_table *t, int enable)
     t->prof_batches = 0;
     t->prof_nk = 0;
     for (double &x : t->prof_ms) x = 0.0;
+    for (double &x : t->prof_in_ms) x = 0.0;
+    t->prof_in_batches = 0;
     return NBA_IPSEC_OK;
 }
 
@@ -454,6 +475,142 @@ int nba_ipsec_profile_read(nba_ipsec_sa_table *t, double *ms, const char **names
     }
     if (n_kernels) *n_kernels = nk;
     if (n_batches) *n_batches = t->prof_batches;
+    return NBA_IPSEC_OK;
+}
+
+// ---- ESP inbound -----------------------------------------
+
+int nba_ipsec_enable_inbound(nba_ipsec_sa_table *t)
+{
+    if (!t) return NBA_IPSEC_EINVAL;
+    if (t->in_enabled) return NBA_IPSEC_OK;
+    DeviceGuard g(t->device);
+    const uint32_t n_sa = t->n_sa, M = t->max_batch;
+    uint32_t hcap = 1024;
+    while (hcap < 2ull * M) hcap <<= 1;
+    InState &S = t->S;
+    cudaError_t e = cudaSuccess;
+    auto chk = [&](cudaError_t x) {
+        if (e == cudaSuccess && x != cudaSuccess) e = x;
+    };
+    chk(dalloc(t, &S.top, n_sa));
+    chk(dalloc(t, &S.top_prev, n_sa));
+    chk(dalloc(t, &S.bmp, n_sa));
+    chk(dalloc(t, &S.bmp_prev, n_sa));
+    chk(dalloc(t, &S.flags, M));
+    chk(dalloc(t, &S.seq, M));
+    chk(dalloc(t, &S.lmax, M));
+    chk(dalloc(t, &S.hmax, (size_t)t->max_tiles * n_sa));
+    chk(dalloc(t, &S.pmx, (size_t)t->max_tiles * n_sa));
+    chk(dalloc(t, &S.hkey, hcap));
+    chk(dalloc(t, &S.hval, hcap));
+    chk(dalloc(t, &S.counters, N_IN_COUNTERS));
+    chk(dalloc(t, &S.ctl, 8));
+    if (e == cudaSuccess) {
+        // reading B6: the window starts at the SA's seq, everything <= seq seen
+        std::vector<unsigned long long> bmp(n_sa);
+        for (uint32_t s = 0; s < n_sa; s++) bmp[s] = t->seq0[s] ? ~0ull : 0ull;
+        chk(cudaMemcpy(S.top, t->seq0.data(), n_sa * 4ull, cudaMemcpyHostToDevice));
+        chk(cudaMemcpy(S.bmp, bmp.data(), n_sa * 8ull, cudaMemcpyHostToDevice));
+    }
+    if (e == cudaSuccess) chk(setup_inbound_attributes(n_sa, t->max_tiles, t->num_sms, &t->in_gridsync));
+    if (e == cudaSuccess) chk(cudaDeviceSynchronize());
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return e == cudaErrorMemoryAllocation ? NBA_IPSEC_ENOMEM : NBA_IPSEC_ECUDA;
+    }
+    t->in_hcap = hcap;
+    t->in_enabled = true;
+    return NBA_IPSEC_OK;
+}
+
+int nba_ipsec_process_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batch *b, void *cuda_stream)
+{
+    if (!t || !b) return NBA_IPSEC_EINVAL;
+    if (!t->in_enabled || b->n_pkts > t->max_batch) return NBA_IPSEC_EINVAL;
+    if (b->n_pkts == 0) return NBA_IPSEC_OK;
+    if (!b->in_buf || !b->in_off || !b->in_len || !b->sa_idx || !b->out_buf || !b->out_off ||
+        !b->out_len)
+        return NBA_IPSEC_EINVAL;
+    DeviceGuard g(t->device);
+    cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    const uint32_t n = b->n_pkts;
+    uint32_t hmask = 1023;
+    while (hmask + 1ull < 2ull * n) hmask = hmask * 2 + 1;
+    const uint32_t n_tiles = (n + PTILE - 1) / PTILE;
+    InBatchArgs B{b->in_buf, b->in_off, b->in_len, b->sa_idx, b->out_buf, b->out_off, b->out_len,
+                  b->status, n};
+    ProfSet *ps = nullptr;
+    if (t->prof) {
+        ps = &t->ring[t->ring_next];
+        prof_drain_set(t, *ps);
+        t->ring_next = (t->ring_next + 1) % PROF_RING;
+        for (int k = 0; k < MAX_KERNELS + 1; k++)
+            if (!ps->ev[k]) cudaEventCreate(&ps->ev[k]);
+        ps->n_ev = 0;
+        ps->inbound = true;
+    }
+    auto mark = [&]() {
+        if (ps) cudaEventRecord(ps->ev[ps->n_ev++], st);
+    };
+    mark();
+    if (launch_in_fused(t->T, t->S, B, t->grid_fused, hmask, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
+    mark();
+    if (launch_in_replay(t->T, t->S, B, n_tiles, hmask, t->in_gridsync, st) != cudaSuccess)
+        return NBA_IPSEC_ECUDA;
+    mark();
+    if (launch_in_decide(t->T, t->S, B, n_tiles, hmask, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
+    mark();
+    return NBA_IPSEC_OK;
+}
+
+int nba_ipsec_read_in_counters(nba_ipsec_sa_table *t, nba_ipsec_in_counters *out, void *cuda_stream)
+{
+    if (!t || !out || !t->in_enabled) return NBA_IPSEC_EINVAL;
+    DeviceGuard g(t->device);
+    unsigned long long h[N_IN_COUNTERS];
+    cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    if (cudaMemcpyAsync(h, t->S.counters, sizeof(h), cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+        cudaStreamSynchronize(st) != cudaSuccess)
+        return NBA_IPSEC_ECUDA;
+    out->pkts_ok = h[0];
+    out->drop_sa = h[1];
+    out->drop_format = h[2];
+    out->drop_replay = h[3];
+    out->drop_auth = h[4];
+    out->drop_trailer = h[5];
+    out->bytes_in = h[6];
+    out->bytes_out = h[7];
+    out->batches = h[8];
+    return NBA_IPSEC_OK;
+}
+
+int nba_ipsec_read_replay_window(nba_ipsec_sa_table *t, uint32_t *top, uint64_t *bitmap,
+                                 void *cuda_stream)
+{
+    if (!t || !top || !bitmap || !t->in_enabled) return NBA_IPSEC_EINVAL;
+    DeviceGuard g(t->device);
+    cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    if (cudaMemcpyAsync(top, t->S.top, t->n_sa * 4ull, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+        cudaMemcpyAsync(bitmap, t->S.bmp, t->n_sa * 8ull, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+        cudaStreamSynchronize(st) != cudaSuccess)
+        return NBA_IPSEC_ECUDA;
+    return NBA_IPSEC_OK;
+}
+
+int nba_ipsec_profile_read_inbound(nba_ipsec_sa_table *t, double *ms, const char **names, int max,
+                                   int *n_kernels, uint32_t *n_batches)
+{
+    static const char *nm[3] = {"in_fused", "in_replay", "in_decide"};
+    if (!t) return NBA_IPSEC_EINVAL;
+    DeviceGuard g(t->device);
+    for (int k = 0; k < PROF_RING; k++) prof_drain_set(t, t->ring[(t->ring_next + k) % PROF_RING]);
+    for (int k = 0; k < 3 && k < max; k++) {
+        if (ms) ms[k] = t->prof_in_ms[k];
+        if (names) names[k] = nm[k];
+    }
+    if (n_kernels) *n_kernels = 3;
+    if (n_batches) *n_batches = t->prof_in_batches;
     return NBA_IPSEC_OK;
 }
 

@@ -74,6 +74,44 @@ struct BatchArgs {
     uint32_t n;
 };
 
+// --- ESP inbound (readings B1..B9) ---------------
+constexpr uint32_t IN_MIN_LEN = 48u + 24u;      // outer 20 + ESP 16 + C >= 24 + ICV 12
+constexpr uint32_t IN_MAX_LEN = 48u + 1504u;
+constexpr uint32_t REPLAY_W = 64u;              // RFC 4303 §3.4.3 default window
+// per-packet flags written by k_in_fused: bits 0..15 inner length D
+constexpr uint32_t INF_FMT = 1u << 31, INF_ICV = 1u << 30, INF_TRL = 1u << 29;
+enum : uint8_t { ST_OK = 0, ST_DROP_SA = 1, ST_DROP_FORMAT = 2, ST_DROP_REPLAY = 3,
+                 ST_DROP_AUTH = 4, ST_DROP_TRAILER = 5 };
+constexpr int N_IN_COUNTERS = 9;   // ok, 5 drop kinds, bytes_in, bytes_out, batches
+
+struct InState {                    // per-SA receive windows + per-batch workspace
+    uint32_t *top;                  // [n_sa] right edge (highest authenticated number)
+    uint32_t *top_prev;             // [n_sa] before the current batch
+    unsigned long long *bmp;        // [n_sa] bit d <-> number top - d
+    unsigned long long *bmp_prev;   // [n_sa]
+    uint32_t *flags;                // [M] INF_* | D
+    uint32_t *seq;                  // [M] sequence number field
+    uint32_t *lmax;                 // [M] max authenticated seq of the SA earlier in the tile
+    uint32_t *hmax;                 // [n_sa][n_tiles] per-tile max (SA-major, zero between batches)
+    uint32_t *pmx;                  // [n_sa][n_tiles] exclusive prefix max along each SA row
+    unsigned long long *hkey;       // [hcap] (sa << 32 | seq) of authenticated packets
+    uint32_t *hval;                 // [hcap] smallest packet index with that key
+    unsigned long long *counters;   // [N_IN_COUNTERS]
+    uint32_t *ctl;                  // [8] ticket, barrier count / generation
+};
+
+struct InBatchArgs {
+    const uint8_t *in_buf;
+    const uint32_t *in_off;
+    const uint16_t *in_len;
+    const uint32_t *sa_idx;
+    uint8_t *out_buf;
+    const uint32_t *out_off;
+    uint16_t *out_len;
+    uint8_t *status;                // may be null
+    uint32_t n;
+};
+
 #ifdef __CUDACC__
 // --- launchers (one per kernel file) ----------------------------------------
 cudaError_t launch_prologue(const DevTable &T, const DevWork &W, const BatchArgs &B,
@@ -93,6 +131,13 @@ cudaError_t setup_aes_attributes();
 cudaError_t setup_fused_attributes();
 int aes_grid(int num_sms);
 int fused_grid(int num_sms);
+cudaError_t launch_in_fused(const DevTable &T, const InState &S, const InBatchArgs &B, int grid,
+                            uint32_t hmask, cudaStream_t st);
+cudaError_t launch_in_replay(const DevTable &T, const InState &S, const InBatchArgs &B,
+                             uint32_t n_tiles, uint32_t hmask, bool gridsync, cudaStream_t st);
+cudaError_t launch_in_decide(const DevTable &T, const InState &S, const InBatchArgs &B,
+                             uint32_t n_tiles, uint32_t hmask, cudaStream_t st);
+cudaError_t setup_inbound_attributes(uint32_t n_sa, uint32_t max_tiles, int num_sms, bool *gridsync);
 
 // --- small device helpers ---------------------------------------------------
 __device__ __forceinline__ uint32_t bswap32(uint32_t x) { return __byte_perm(x, 0, 0x0123); }

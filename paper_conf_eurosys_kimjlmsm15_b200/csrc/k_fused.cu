@@ -25,205 +25,9 @@
 // (byte r of the state word in bits 8..15, lane*4 in bits 0..7, the table base
 // in bits 16..31) -- no address add per lookup.  Per-thread round keys and the
 // packet metadata live below (FusedLo) and above (FusedHi) the tables.
-#include "aes_round.cuh"
-#include "sha1.cuh"
+#include "fused_common.cuh"
 
 namespace nba {
-
-constexpr int F_THREADS = 512;            // 16 warps -> up to 128 registers
-constexpr int F_SUPER = 512;              // packets per super-round (one per thread)
-
-struct FusedLo {
-    uint32_t sa[F_SUPER];          // by packet index in the super-round
-    uint32_t info[F_SUPER];        // D | tos << 16 | INFO_OK  (0: dropped)
-    uint32_t seq[F_SUPER];
-    uint32_t inoff[F_SUPER];
-    uint32_t outoff[F_SUPER];
-    uint16_t perm[F_SUPER];        // position -> packet index (length-sorted)
-    uint4 rkA[4][F_THREADS];       // round keys 3..6 of the thread's current packet
-    uint32_t bins[NBINS];
-    unsigned long long cnt[4];
-};
-
-struct FusedHi {
-    uint4 rkB[4][F_THREADS];       // round keys 7..10
-};
-
-// Dynamic shared memory: [Lo | pad][tables 128 KB][Hi].  With the usual 1 KB of
-// reserved shared memory the tables start at shared address 0x10000.
-constexpr uint32_t F_TOFF_MAX = 0xFC00u;
-constexpr size_t F_SMEM = F_TOFF_MAX + AES_TABLE_BYTES + sizeof(FusedHi);
-static_assert(sizeof(FusedLo) <= F_TOFF_MAX, "FusedLo must fit below the tables");
-static_assert(F_SMEM <= 232448, "exceeds 227 KB of shared memory per block");
-
-// -------------------------------------------------------------------- helpers
-__device__ __forceinline__ uint32_t smem_u32(const void *p)
-{
-    return (uint32_t)__cvta_generic_to_shared(p);
-}
-
-template <uint32_t OFF>
-__device__ __forceinline__ uint32_t lds_abs(uint32_t a)
-{
-    uint32_t v;
-    asm volatile("ld.shared.u32 %0, [%1+%2];" : "=r"(v) : "r"(a), "n"(OFF));
-    return v;
-}
-
-// T-table lookup: table `tbl`, row `row` of state word `reg`; lane4r holds
-// lane*4 in bits 0..7 and the 64 KB-aligned table base in bits 16..31.
-#define TL(reg, row, tbl)                                                                  \
-    lds_abs<((tbl) >> 1) * 0x10000u + ((tbl) & 1u) * 0x80u>(                               \
-        __byte_perm((reg), lane4r, 0x7604u | ((row) << 4)))
-
-__device__ __forceinline__ uint32_t trailer_byte_f(uint32_t b, uint32_t D, uint32_t p)
-{
-    if (b < D + p) return b - D + 1u;
-    if (b == D + p) return p;
-    if (b == D + p + 1u) return 4u;
-    return 0u;
-}
-
-__device__ __forceinline__ void prefetch_l2(const void *p)
-{
-    asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
-}
-
-__device__ __forceinline__ void stg_v4(void *p, uint32_t a, uint32_t b, uint32_t c, uint32_t d)
-{
-    asm volatile("st.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(a), "r"(b), "r"(c), "r"(d)
-                 : "memory");
-}
-
-// Bytes [lo, hi) of the 16-byte image (w0..w3) to chunk + [lo, hi); chunk 16-B aligned.
-__device__ __forceinline__ void store_chunk_range(uint8_t *chunk, uint32_t w0, uint32_t w1,
-                                                  uint32_t w2, uint32_t w3, uint32_t lo, uint32_t hi)
-{
-    if (lo == 0 && hi == 16) {
-        stg_v4(chunk, w0, w1, w2, w3);
-        return;
-    }
-    uint32_t x = lo;
-    while (x < hi) {
-        const uint32_t wi = x >> 2;
-        const uint32_t w = wi == 0 ? w0 : wi == 1 ? w1 : wi == 2 ? w2 : w3;
-        if ((x & 3u) == 0 && x + 4 <= hi) {
-            asm volatile("st.global.u32 [%0], %1;" ::"l"(chunk + x), "r"(w) : "memory");
-            x += 4;
-        } else if ((x & 1u) == 0 && x + 2 <= hi) {
-            asm volatile("st.global.u16 [%0], %1;" ::"l"(chunk + x),
-                         "h"((unsigned short)(w >> ((x & 3u) * 8u)))
-                         : "memory");
-            x += 2;
-        } else {
-            asm volatile("st.global.u8 [%0], %1;" ::"l"(chunk + x),
-                         "h"((unsigned short)((w >> ((x & 3u) * 8u)) & 0xffu))
-                         : "memory");
-            x += 1;
-        }
-    }
-}
-
-// Streams the output packet (outer IPv4 || ESP header || ciphertext || ICV) as
-// 32-bit words, in order, into destination-aligned 16-byte stores.  Output word
-// w lands at byte e + 4w of the aligned chunk sequence starting at cp (e = the
-// slot's misalignment); dest word k = funnel(out[k-q-1], out[k-q]) by r bits.
-struct OutStream {
-    uint8_t *cp;           // current 16-B aligned destination chunk
-    uint32_t a0, a1, a2, a3;
-    uint32_t p;            // next word position in the chunk (0..3)
-    uint32_t prev;         // previous output word (for the funnel shift)
-    uint32_t r;            // 8 * (e & 3)
-    uint32_t lo;           // first byte of the current chunk that is ours
-
-    __device__ __forceinline__ void init(uint8_t *dst)
-    {
-        const uintptr_t a = reinterpret_cast<uintptr_t>(dst);
-        const uint32_t e = (uint32_t)(a & 15u);
-        cp = reinterpret_cast<uint8_t *>(a - e);
-        a0 = a1 = a2 = a3 = 0;
-        p = e >> 2;
-        prev = 0;
-        r = (e & 3u) * 8u;
-        lo = e;
-    }
-    __device__ __forceinline__ void place(uint32_t d)
-    {
-        a0 = p == 0 ? d : a0;
-        a1 = p == 1 ? d : a1;
-        a2 = p == 2 ? d : a2;
-        a3 = p == 3 ? d : a3;
-    }
-    __device__ __forceinline__ void put(uint32_t v)
-    {
-        const uint32_t d = __funnelshift_l(prev, v, r);
-        prev = v;
-        place(d);
-        if (++p == 4) {
-            store_chunk_range(cp, a0, a1, a2, a3, lo, 16);
-            cp += 16;
-            p = 0;
-            lo = 0;
-        }
-    }
-    // 16 words whose dest words start at chunk position p (any): the whole
-    // step without per-word selects.
-    __device__ __forceinline__ void put16(const uint32_t (&v)[16])
-    {
-        uint32_t d[16];
-#pragma unroll
-        for (int i = 0; i < 16; i++) {
-            d[i] = __funnelshift_l(i ? v[i - 1] : prev, v[i], r);
-        }
-        prev = v[15];
-#define NBA_PUT16(P)                                                                             \
-    {                                                                                            \
-        uint32_t c[4] = {a0, a1, a2, a3};                                                        \
-        _Pragma("unroll") for (int i = 0; i < 4 - (P); i++) c[(P) + i] = d[i];                   \
-        store_chunk_range(cp, c[0], c[1], c[2], c[3], lo, 16);                                   \
-        stg_v4(cp + 16, d[4 - (P)], d[5 - (P)], d[6 - (P)], d[7 - (P)]);                         \
-        stg_v4(cp + 32, d[8 - (P)], d[9 - (P)], d[10 - (P)], d[11 - (P)]);                       \
-        stg_v4(cp + 48, d[12 - (P)], d[13 - (P)], d[14 - (P)], d[15 - (P)]);                     \
-        cp += 64;                                                                                \
-        if ((P) > 0) a0 = d[16 - (P)];                                                           \
-        if ((P) > 1) a1 = d[17 - (P)];                                                           \
-        if ((P) > 2) a2 = d[18 - (P)];                                                           \
-    }
-        switch (p) {
-        case 0: {
-            stg_v4(cp, d[0], d[1], d[2], d[3]);
-            stg_v4(cp + 16, d[4], d[5], d[6], d[7]);
-            stg_v4(cp + 32, d[8], d[9], d[10], d[11]);
-            stg_v4(cp + 48, d[12], d[13], d[14], d[15]);
-            cp += 64;
-            break;
-        }
-        case 1: NBA_PUT16(1) break;
-        case 2: NBA_PUT16(2) break;
-        default: NBA_PUT16(3) break;
-        }
-#undef NBA_PUT16
-        lo = 0;
-    }
-    // after the last word: the spill-over dest word (if r) and the final partial chunk
-    __device__ __forceinline__ void finish(const uint8_t *end)
-    {
-        if (r) {
-            place(__funnelshift_l(prev, 0u, r));
-            if (++p == 4) {
-                // the spill-over word completed a chunk: it ends inside it
-                const uint32_t hi = (uint32_t)(end - cp);
-                store_chunk_range(cp, a0, a1, a2, a3, lo, hi < 16u ? hi : 16u);
-                cp += 16;
-                p = 0;
-                lo = 0;
-                return;
-            }
-        }
-        const intptr_t hi = end - cp;
-        if (hi > 0) store_chunk_range(cp, a0, a1, a2, a3, lo, (uint32_t)hi);
-    }
-};
 
 // ---------------------------------------------- one packet, one lane
 __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B, FusedLo &L,
@@ -252,16 +56,7 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
     // round keys 3..10 were staged into L.rkA / H.rkB by the warp (coalesced)
     const uint4 hd = __ldg(&T.sahdr[sa]);
     const uint32_t qbe = bswap32(q32);
-    const uint32_t s0 = hd.y ^ r0.x, s1 = r0.y, s2 = qbe ^ r0.z, s3 = r0.w;
-    const uint32_t X0 = TL(s0, 0, 0) ^ TL(s1, 1, 1) ^ TL(s2, 2, 2) ^ r1.x;
-    const uint32_t Y1 = TL(s1, 0, 0) ^ TL(s2, 1, 1) ^ TL(s3, 2, 2) ^ TL(s0, 3, 3) ^ r1.y;
-    const uint32_t Y2 = TL(s2, 0, 0) ^ TL(s3, 1, 1) ^ TL(s0, 2, 2) ^ TL(s1, 3, 3) ^ r1.z;
-    const uint32_t Y3 = TL(s3, 0, 0) ^ TL(s0, 1, 1) ^ TL(s1, 2, 2) ^ TL(s2, 3, 3) ^ r1.w;
-    const uint32_t Z0 = TL(Y1, 1, 1) ^ TL(Y2, 2, 2) ^ TL(Y3, 3, 3) ^ r2.x;
-    const uint32_t Z1 = TL(Y1, 0, 0) ^ TL(Y2, 1, 1) ^ TL(Y3, 2, 2) ^ r2.y;
-    const uint32_t Z2 = TL(Y2, 0, 0) ^ TL(Y3, 1, 1) ^ TL(Y1, 3, 3) ^ r2.z;
-    const uint32_t Z3 = TL(Y3, 0, 0) ^ TL(Y1, 2, 2) ^ TL(Y2, 3, 3) ^ r2.w;
-    const uint32_t R3 = s3 >> 24;
+    const CtrPre cp = ctr_precompute(lane4r, r0, r1, r2, hd.y, 0u, qbe);   // IV = BE64(q), A6
 
     // outer IPv4 header (reading A13) + ESP header + IV: output words 0..8
     OutStream os;
@@ -298,7 +93,6 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
     // metadata phase); each step prefetches two steps ahead
     if (D > 64u) prefetch_l2(src + 64);
     if (D > 128u) prefetch_l2(src + 128);
-    const uint4 z4 = make_uint4(0, 0, 0, 0);
 
     // ---- one SHA-1 compression per iteration; AES steps feed the first nsteps
 #pragma unroll 1
@@ -309,71 +103,14 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
         if (it < nsteps) {
             // payload words of T bytes [64 it, 64 it + 64), realigned
             if (64u * it + 192u < D) prefetch_l2(src + 64u * it + 192u);
-            const uintptr_t a = reinterpret_cast<uintptr_t>(src) + 64u * it;
-            const uintptr_t abase = a & ~(uintptr_t)15;
-            const uint32_t sh = (uint32_t)(a & 15u);
-            uint4 c[5];
-#pragma unroll
-            for (int i = 0; i < 5; i++) {
-                const uintptr_t qa = abase + 16u * i;
-                c[i] = qa < src_end ? ldg_nc_v4(reinterpret_cast<const void *>(qa)) : z4;
-            }
-            // AES-128 of counter blocks 4 it + 1 .. 4 it + 4 (rounds 3..10)
+            Raw5 raw;
+            load_raw5(reinterpret_cast<uintptr_t>(src) + 64u * it, src_end, raw);
+            // AES-128 of counter blocks 4 it + 1 .. 4 it + 4
             uint32_t ks[16];
-            {
-                uint32_t x[4][4];
-#pragma unroll
-                for (int b = 0; b < 4; b++) {
-                    const uint32_t t0 = TL((R3 ^ (4u * it + 1u + b)) << 24, 3, 3) ^ X0;
-                    x[b][0] = TL(t0, 0, 0) ^ Z0;
-                    x[b][1] = TL(t0, 3, 3) ^ Z1;
-                    x[b][2] = TL(t0, 2, 2) ^ Z2;
-                    x[b][3] = TL(t0, 1, 1) ^ Z3;
-                }
-#pragma unroll 1
-                for (int r = 0; r < 7; r++) {
-                    const uint4 rk = r < 4 ? L.rkA[r][tid] : H.rkB[r - 4][tid];
-#pragma unroll
-                    for (int b = 0; b < 4; b++) {
-                        const uint32_t u0 = TL(x[b][0], 0, 0) ^ TL(x[b][1], 1, 1) ^ TL(x[b][2], 2, 2) ^ TL(x[b][3], 3, 3) ^ rk.x;
-                        const uint32_t u1 = TL(x[b][1], 0, 0) ^ TL(x[b][2], 1, 1) ^ TL(x[b][3], 2, 2) ^ TL(x[b][0], 3, 3) ^ rk.y;
-                        const uint32_t u2 = TL(x[b][2], 0, 0) ^ TL(x[b][3], 1, 1) ^ TL(x[b][0], 2, 2) ^ TL(x[b][1], 3, 3) ^ rk.z;
-                        const uint32_t u3 = TL(x[b][3], 0, 0) ^ TL(x[b][0], 1, 1) ^ TL(x[b][1], 2, 2) ^ TL(x[b][2], 3, 3) ^ rk.w;
-                        x[b][0] = u0;
-                        x[b][1] = u1;
-                        x[b][2] = u2;
-                        x[b][3] = u3;
-                    }
-                }
-                const uint4 rk = H.rkB[3][tid];
-#define NBA_FINAL(s0, s1, s2, s3)                                                               \
-    ((TL(s0, 0, 2) & 0x000000ffu) | (TL(s1, 1, 3) & 0x0000ff00u) | (TL(s2, 2, 0) & 0x00ff0000u) | \
-     (TL(s3, 3, 1) & 0xff000000u))
-#pragma unroll
-                for (int b = 0; b < 4; b++) {
-                    ks[4 * b + 0] = rk.x ^ NBA_FINAL(x[b][0], x[b][1], x[b][2], x[b][3]);
-                    ks[4 * b + 1] = rk.y ^ NBA_FINAL(x[b][1], x[b][2], x[b][3], x[b][0]);
-                    ks[4 * b + 2] = rk.z ^ NBA_FINAL(x[b][2], x[b][3], x[b][0], x[b][1]);
-                    ks[4 * b + 3] = rk.w ^ NBA_FINAL(x[b][3], x[b][0], x[b][1], x[b][2]);
-                }
-#undef NBA_FINAL
-            }
+            aes4_keystream(lane4r, cp, it, L, H, tid, ks);
             // plaintext T = P || pad || p || 4, XOR keystream
             {
-                uint32_t v[20] = {c[0].x, c[0].y, c[0].z, c[0].w, c[1].x, c[1].y, c[1].z, c[1].w,
-                                  c[2].x, c[2].y, c[2].z, c[2].w, c[3].x, c[3].y, c[3].z, c[3].w,
-                                  c[4].x, c[4].y, c[4].z, c[4].w};
-                const uint32_t rr = (sh & 3u) * 8u;
-#define NBA_PT_CASE(Q)                                                                    \
-    _Pragma("unroll") for (int w = 0; w < 16; w++) ct[w] =                                \
-        __funnelshift_r(v[(Q) + w], v[(Q) + w + 1], rr);
-                switch (sh >> 2) {
-                case 0: NBA_PT_CASE(0) break;
-                case 1: NBA_PT_CASE(1) break;
-                case 2: NBA_PT_CASE(2) break;
-                default: NBA_PT_CASE(3) break;
-                }
-#undef NBA_PT_CASE
+                extract16(raw, ct);
                 // trailer: T ends on a word boundary (C = 0 mod 4), so it touches only
                 // the last word (and the one before when p = 3):
                 //   p=0 [P P 0 4]  p=1 [P 1 1 4]  p=2 [1 2 2 4]  p=3 [.. 1][2 3 3 4]
@@ -562,19 +299,8 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc)
             const uint32_t info = have ? L.info[pk] : 0u;
             const uint32_t pkt = base + pk;
             const uint32_t sa_me = (info & INFO_OK) ? L.sa[pk] : INVALID_SA;
-            // warp-cooperative, coalesced staging of round keys 3..10: load m of
-            // the warp covers 128 contiguous bytes of 4 lanes' SAs
-#pragma unroll
-            for (int k = 0; k < 8; k++) {
-                const uint32_t m = 32u * k + lane, owner = m >> 3, r = m & 7u;
-                const uint32_t s = __shfl_sync(0xffffffffu, sa_me, owner);
-                if (s != INVALID_SA) {
-                    const uint4 v = __ldg(&T.rk[(size_t)s * 11u + 3u + r]);
-                    const uint32_t slot = (warp << 5) + owner;
-                    if (r < 4) L.rkA[r][slot] = v;
-                    else H.rkB[r - 4][slot] = v;
-                }
-            }
+            // warp-cooperative, coalesced staging of round keys 3..10
+            stage_round_keys(T.rk, L, H, sa_me, warp, lane);
             __syncwarp();
             if (!have) {
             } else if (info & INFO_OK) {

@@ -1,0 +1,272 @@
+// k_in_fused.cu -- ESP inbound, step 1 of 3: per packet, in
+// ONE pass over its bytes, the format checks, the ICV verification and the
+// AES-CTR decryption.  The mirror of k_fused.cu (same SM layout: one 512-thread
+// CTA per SM, 128 KB bank-replicated T-tables, one lane per packet, length-
+// sorted lanes, AES and SHA-1 interleaved every 64 bytes).
+//
+// RFC 4303 §3.4.4.1 allows the ICV check and the decryption to run in parallel
+// as long as the packet is not released before both are done: the plaintext is
+// written to the caller's slot here, but out_len stays 0 (= dropped) until
+// k_in_decide has combined the ICV result with the anti-replay decision
+// (§3.4.3), which needs the authenticated sequence numbers of all earlier
+// packets of the SA (k_in_replay).
+//
+// Per packet i (SA s = sa_idx[i], L = in_len[i], reading B2):
+//   format: 72 <= L <= 1552, C = L - 48 = 0 mod 4, outer 0x45, tot_len = L,
+//           no fragment, protocol 50, header checksum valid, SPI = spi_s;
+//   ICV:    HMAC-SHA1-96 over SPI .. ciphertext (midstates of the SA), compared
+//           with the 12 received bytes;
+//   decrypt: counter block nonce_s || IV (from the packet, RFC 3686 §3.1) ||
+//           BE32(k+1); T = E xor keystream streamed to out_buf + out_off[i];
+//   trailer: next header 4, pad length p with D = C - 2 - p >= 20, pad bytes 1..p.
+// Output: flags[i] = INF_FMT | INF_ICV | INF_TRL | D, seq[i].
+#include "fused_common.cuh"
+
+namespace nba {
+
+__device__ __forceinline__ uint32_t esp_in_packet(const DevTable &T, const InBatchArgs &B,
+                                                  const FusedLo &L, const FusedHi &H,
+                                                  uint32_t lane4r, uint32_t tid, uint32_t sa,
+                                                  uint32_t C, uint32_t q32, uint32_t iv0,
+                                                  uint32_t iv1, uint32_t inoff, uint32_t outoff)
+{
+    const uint32_t Cw = C >> 2;                  // ciphertext words
+    const uint32_t Mw = 4u + Cw;                 // MAC input words (ESP hdr + ciphertext)
+    const uint32_t nsteps = (Cw + 15u) >> 4;     // 64-byte AES steps
+    const uint32_t nb_in = (4u * Mw + 8u) / 64u + 1u;   // inner SHA-1 blocks
+    const uint32_t bitlen = (64u + 4u * Mw) * 8u;
+
+    const uint4 *rks = T.rk + (size_t)sa * 11u;
+    const uint4 r0 = __ldg(&rks[0]), r1 = __ldg(&rks[1]), r2 = __ldg(&rks[2]);
+    const uint4 hd = __ldg(&T.sahdr[sa]);
+    const CtrPre cp = ctr_precompute(lane4r, r0, r1, r2, hd.y, iv0, iv1);
+
+    OutStream os;
+    os.init(B.out_buf + outoff);
+    // SHA-1 message words 0..3 = SPI || seq || IV (big-endian words of the wire bytes)
+    uint32_t carry[4] = {bswap32(hd.x), q32, bswap32(iv0), bswap32(iv1)};
+    uint32_t st[5];
+    {
+        const uint4 h0 = __ldg(&T.hmid[(size_t)sa * 3 + 0]);
+        const uint4 h1 = __ldg(&T.hmid[(size_t)sa * 3 + 1]);
+        st[0] = h0.x; st[1] = h0.y; st[2] = h0.z; st[3] = h0.w; st[4] = h1.x;
+    }
+    const uint8_t *src = B.in_buf + inoff + 36u;          // ciphertext E
+    const uintptr_t src_end = reinterpret_cast<uintptr_t>(src) + C;
+    if (C > 64u) prefetch_l2(src + 64);
+    if (C > 128u) prefetch_l2(src + 128);
+    uint32_t lastw = 0, prevw = 0;               // plaintext words Cw-1 and Cw-2
+
+#pragma unroll 1
+    for (uint32_t it = 0; it <= nb_in; it++) {
+        uint32_t ct[16];
+#pragma unroll
+        for (int w = 0; w < 16; w++) ct[w] = 0u;
+        if (it < nsteps) {
+            if (64u * it + 192u < C) prefetch_l2(src + 64u * it + 192u);
+            Raw5 raw;
+            load_raw5(reinterpret_cast<uintptr_t>(src) + 64u * it, src_end, raw);
+            uint32_t ks[16];
+            aes4_keystream(lane4r, cp, it, L, H, tid, ks);
+            extract16(raw, ct);                  // ciphertext words (beyond C: ignored)
+            uint32_t pt[16];
+#pragma unroll
+            for (int w = 0; w < 16; w++) pt[w] = ct[w] ^ ks[w];
+            const uint32_t lw = Cw - 1u - 16u * it;
+#pragma unroll
+            for (int w = 0; w < 16; w++) {
+                if ((uint32_t)w == lw) lastw = pt[w];
+                if ((uint32_t)w + 1u == lw) prevw = pt[w];
+            }
+            if (16u * it + 16u <= Cw) {
+                os.put16(pt);
+            } else {
+#pragma unroll
+                for (int w = 0; w < 16; w++)
+                    if (16u * it + w < Cw) os.put(pt[w]);
+            }
+        }
+        // SHA-1 block: inner block `it` over SPI || seq || IV || E (FIPS 180-4
+        // §5.1.1 padding), or the outer hash of the inner digest (RFC 2104)
+        uint32_t W[16];
+        if (it < nb_in) {
+            const uint32_t m0 = 16u * it;
+#pragma unroll
+            for (int i = 0; i < 16; i++) {
+                const uint32_t m = m0 + i;
+                const uint32_t msg = i < 4 ? carry[i] : bswap32(ct[i - 4]);
+                W[i] = m < Mw ? msg : (m == Mw ? 0x80000000u : 0u);
+            }
+            if (it == nb_in - 1u) W[15] = bitlen;
+#pragma unroll
+            for (int i = 0; i < 4; i++) carry[i] = bswap32(ct[12 + i]);
+        } else {
+#pragma unroll
+            for (int i = 0; i < 5; i++) W[i] = st[i];
+            W[5] = 0x80000000u;
+#pragma unroll
+            for (int i = 6; i < 15; i++) W[i] = 0u;
+            W[15] = (64u + 20u) * 8u;
+            const uint4 h1 = __ldg(&T.hmid[(size_t)sa * 3 + 1]);
+            const uint4 h2 = __ldg(&T.hmid[(size_t)sa * 3 + 2]);
+            st[0] = h1.y; st[1] = h1.z; st[2] = h1.w; st[3] = h2.x; st[4] = h2.y;
+        }
+        sha1_compress(st, W);
+    }
+    os.finish(B.out_buf + outoff + C);
+
+    // RFC 4303 §3.4.4.1 / RFC 2404: first 96 bits of the outer digest
+    uint32_t icv[3];
+    load_words<3>(src_end, src_end + 12u, icv);
+    const uint32_t diff = (bswap32(st[0]) ^ icv[0]) | (bswap32(st[1]) ^ icv[1]) |
+                          (bswap32(st[2]) ^ icv[2]);
+    uint32_t flags = diff == 0u ? INF_ICV : 0u;
+
+    // trailer (reading B4): ... pad 1..p | p | next header, T ends on a word
+    const uint32_t nh = lastw >> 24, p = (lastw >> 16) & 0xffu;
+    bool trl = nh == 4u && p + 2u + MIN_D <= C;
+    if (trl) {
+        const uint32_t D = C - 2u - p;
+        if (p <= 6u) {               // pad bytes inside the last two words
+            const unsigned long long tail = ((unsigned long long)lastw << 32) | prevw;
+            for (uint32_t j = 1; j <= p; j++)
+                trl &= ((tail >> (8u * (5u - p + j))) & 0xffu) == j;
+        } else {                     // long padding: read back this lane's own stores
+            const uint8_t *o = B.out_buf + outoff + D;
+            for (uint32_t j = 1; j <= p; j++) trl &= o[j - 1] == (uint8_t)j;
+        }
+        if (trl) flags |= INF_TRL | D;
+    }
+    return flags;
+}
+
+__global__ void __launch_bounds__(F_THREADS, 1)
+k_in_fused(DevTable T, InState S, InBatchArgs B, uint32_t ppc, uint32_t hmask)
+{
+    extern __shared__ __align__(16) uint8_t smem[];
+    const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
+    const uint32_t n_sa = T.n_sa;
+
+    const uint32_t sb = smem_u32(smem);
+    const uint32_t toff = (0x10000u - (sb & 0xffffu)) & 0xffffu;
+    uint32_t lo_off = 0;
+    if (toff < sizeof(FusedLo)) {
+        if (toff + AES_TABLE_BYTES + sizeof(FusedHi) + sizeof(FusedLo) > F_SMEM) __trap();
+        lo_off = toff + AES_TABLE_BYTES + (uint32_t)sizeof(FusedHi);
+    }
+    uint8_t *tabs = smem + toff;
+    FusedLo &L = *reinterpret_cast<FusedLo *>(smem + lo_off);
+    FusedHi &H = *reinterpret_cast<FusedHi *>(smem + toff + AES_TABLE_BYTES);
+    const uint32_t lane4r = (lane * 4u) | (smem_u32(tabs) & 0xffff0000u);
+
+    // this batch's duplicate-detection hash (read by k_in_replay / k_in_decide
+    // of this batch only; the previous batch's kernels have completed)
+    for (uint32_t k = blockIdx.x * blockDim.x + tid; k <= hmask; k += gridDim.x * blockDim.x) {
+        S.hkey[k] = ~0ull;
+        S.hval[k] = ~0u;
+    }
+    aes_tables_to_smem(tabs, T.te0);
+    if (tid < NBINS) L.bins[tid] = 0;
+    __syncthreads();
+
+    const uint32_t p_begin = blockIdx.x * ppc;
+    const uint32_t p_end = min(B.n, p_begin + ppc);
+    for (uint32_t base = p_begin; base < p_end; base += F_SUPER) {
+        const uint32_t cnt_pk = min((uint32_t)F_SUPER, p_end - base);
+        // ---- 1. metadata and format checks (thread j <-> packet base + j) ----
+        const uint32_t j = tid;
+        const uint32_t i = base + j;
+        if (j < cnt_pk) {
+            const uint32_t sa = B.sa_idx[i];
+            const uint32_t Lin = B.in_len[i];
+            const uint32_t inoff = B.in_off[i];
+            uint32_t info = 0, q = 0, iv0 = 0, iv1 = 0;
+            if (sa < n_sa && Lin >= IN_MIN_LEN && Lin <= IN_MAX_LEN && ((Lin - 48u) & 3u) == 0) {
+                const uint8_t *pk = B.in_buf + inoff;
+                uint32_t w[9];
+                load_words<9>(reinterpret_cast<uintptr_t>(pk), reinterpret_cast<uintptr_t>(pk) + Lin, w);
+                // RFC 1071: the one's complement sum over the header (checksum
+                // included) is 0xffff; byte order does not matter (§2(B))
+                uint32_t sum = 0;
+#pragma unroll
+                for (int k = 0; k < 5; k++) sum += (w[k] & 0xffffu) + (w[k] >> 16);
+                sum = (sum & 0xffffu) + (sum >> 16);
+                sum = (sum & 0xffffu) + (sum >> 16);
+                const uint32_t tot = ((w[0] >> 8) & 0xff00u) | (w[0] >> 24);
+                const bool ok = (w[0] & 0xffu) == 0x45u && tot == Lin &&
+                                (w[1] & 0xff3f0000u) == 0u &&         // MF = 0, offset 0
+                                ((w[2] >> 8) & 0xffu) == 50u && sum == 0xffffu &&
+                                w[5] == __ldg(&T.sahdr[sa]).x;        // SPI (RFC 4303 §3.4.2)
+                if (ok) {
+                    info = (Lin - 48u) | INFO_OK;
+                    q = bswap32(w[6]);
+                    iv0 = w[7];
+                    iv1 = w[8];
+                }
+            }
+            L.sa[j] = sa;
+            L.info[j] = info;
+            L.seq[j] = q;
+            L.inoff[j] = inoff;
+            L.outoff[j] = B.out_off[i];
+            L.aux0[j] = iv0;
+            L.aux1[j] = iv1;
+            atomicAdd(&L.bins[info ? hmac_bin(true, info & 0xffffu) : NBINS - 1], 1u);
+        }
+        __syncthreads();
+        if (warp == 0) {
+            uint32_t cb = L.bins[lane], x = cb;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+                if (lane >= (uint32_t)o) x += y;
+            }
+            L.bins[lane] = x - cb;
+        }
+        __syncthreads();
+        if (j < cnt_pk) {
+            const uint32_t info = L.info[j];
+            L.perm[atomicAdd(&L.bins[info ? hmac_bin(true, info & 0xffffu) : NBINS - 1], 1u)] = (uint16_t)j;
+        }
+        __syncthreads();
+        if (tid < NBINS) L.bins[tid] = 0;
+
+        // ---- 2. one lane per packet, longest packets in the highest warps ----
+        {
+            const bool have = tid < cnt_pk;
+            const uint32_t pk = have ? L.perm[cnt_pk - 1u - tid] : 0u;
+            const uint32_t info = have ? L.info[pk] : 0u;
+            const uint32_t sa_me = (info & INFO_OK) ? L.sa[pk] : INVALID_SA;
+            stage_round_keys(T.rk, L, H, sa_me, warp, lane);
+            __syncwarp();
+            if (have) {
+                uint32_t flags = 0;
+                if (info & INFO_OK)
+                    flags = INF_FMT | esp_in_packet(T, B, L, H, lane4r, tid, sa_me, info & 0xffffu,
+                                                    L.seq[pk], L.aux0[pk], L.aux1[pk], L.inoff[pk],
+                                                    L.outoff[pk]);
+                S.flags[base + pk] = flags;
+                S.seq[base + pk] = L.seq[pk];
+            }
+        }
+        __syncthreads();
+    }
+}
+
+cudaError_t launch_in_fused(const DevTable &T, const InState &S, const InBatchArgs &B, int grid,
+                            uint32_t hmask, cudaStream_t st)
+{
+    uint32_t ppc = (B.n + grid - 1) / grid;
+    ppc = (ppc + 31u) & ~31u;
+    if (ppc < 32u) ppc = 32u;
+    const uint32_t g = (B.n + ppc - 1) / ppc;
+    k_in_fused<<<g, F_THREADS, F_SMEM, st>>>(T, S, B, ppc, hmask);
+    return cudaGetLastError();
+}
+
+cudaError_t setup_in_fused_attributes()
+{
+    return cudaFuncSetAttribute(k_in_fused, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)F_SMEM);
+}
+
+}  // namespace nba

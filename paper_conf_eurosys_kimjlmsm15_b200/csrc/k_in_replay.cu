@@ -1,0 +1,329 @@
+// k_in_replay.cu -- ESP inbound, steps 2 and 3: the RFC 4303
+// §3.4.3 anti-replay decision for a whole batch at once, bit-exact with the
+// sequential receiver (oracle_process_inbound), and the per-SA window update.
+//
+// Sequential rule (window W = 64, right edge `top`, bit d <-> number top - d):
+// packet j of SA s passes iff q != 0 and (q > top, or top - q < W and q not yet
+// marked); the window is updated only for packets that pass AND authenticate.
+// Parallel form used here: let A = the packets with a
+// valid format and ICV.  Packets outside A never move the window, and a packet
+// of A that fails the check has q <= top, so the edge seen by packet j is
+//     top_j = max(top_0, max{ q_k : k < j, k in A, same SA })     (a prefix max)
+// and j passes iff q != 0 and (q > top_j, or top_j - q < W, q is not marked in
+// the window at batch start, and no k < j in A of the same SA has q_k = q).
+// (If such a k exists and passed, j is a duplicate; if it failed, it was too old
+// or itself a duplicate, and so is j.)  The first-index test uses a hash of
+// (s, q) -> min k over A.  The final window: top' = max(top_0, max over A) and
+// the start bitmap shifted by top' - top_0, OR the bits of the accepted numbers.
+//
+// k_in_replay: one CTA per tile of PTILE packets: warp-segmented prefix max by
+// SA (__match_any_sync), then each group looks up its SA among the other warps'
+// groups (earlier warps raise its prefix); per-tile per-SA max into an SA-major
+// matrix; hash inserts.  Then (grid barrier when the grid is
+// co-resident, else the last CTA) one warp per SA scans its row (exclusive
+// prefix max) and moves the window edge.
+// k_in_decide: one thread per packet: status, out_len, window bits, counters.
+#include "internal.cuh"
+
+namespace nba {
+
+__device__ __forceinline__ uint32_t hash_slot(unsigned long long key, uint32_t hmask)
+{
+    return (uint32_t)((key * 0x9E3779B97F4A7C15ull) >> 32) & hmask;
+}
+
+__device__ __forceinline__ void in_grid_barrier(uint32_t *count, uint32_t *gen)
+{
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        const uint32_t g = *reinterpret_cast<volatile uint32_t *>(gen);
+        __threadfence();
+        if (atomicAdd(count, 1u) == gridDim.x - 1u) {
+            *reinterpret_cast<volatile uint32_t *>(count) = 0;
+            __threadfence();
+            atomicAdd(gen, 1u);
+        } else {
+            while (*reinterpret_cast<volatile uint32_t *>(gen) == g) __nanosleep(32);
+        }
+        __threadfence();
+    }
+    __syncthreads();
+}
+
+// Exclusive prefix max down SA row `sa` of the tile maxima by one warp, then
+// the window edge update for the batch.
+__device__ __forceinline__ void scan_max_row(const InState &S, uint32_t sa, uint32_t n_tiles,
+                                             uint32_t lane)
+{
+    constexpr int U = 8;
+    uint32_t *row = S.hmax + (size_t)sa * n_tiles;
+    uint32_t *pfx = S.pmx + (size_t)sa * n_tiles;
+    uint32_t carry = 0;
+    for (uint32_t t0 = 0; t0 < n_tiles; t0 += 32u * U) {
+        uint32_t h[U];
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            const uint32_t t = t0 + 32u * u + lane;
+            h[u] = t < n_tiles ? __ldcg(&row[t]) : 0u;
+        }
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            if (t0 + 32u * u >= n_tiles) break;
+            uint32_t x = h[u];
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+                if (lane >= (uint32_t)o) x = max(x, y);
+            }
+            uint32_t ex = __shfl_up_sync(0xffffffffu, x, 1);
+            if (lane == 0) ex = 0;
+            const uint32_t t = t0 + 32u * u + lane;
+            if (t < n_tiles) {
+                pfx[t] = max(carry, ex);
+                if (h[u]) row[t] = 0;            // re-arm for the next batch
+            }
+            carry = max(carry, __shfl_sync(0xffffffffu, x, 31));
+        }
+    }
+    if (lane == 0) {
+        const uint32_t t0 = S.top[sa];
+        const unsigned long long b0 = S.bmp[sa];
+        S.top_prev[sa] = t0;
+        S.bmp_prev[sa] = b0;
+        const uint32_t t1 = max(t0, carry);
+        const uint32_t sh = t1 - t0;
+        S.bmp[sa] = sh >= REPLAY_W ? 0ull : (b0 << sh);
+        S.top[sa] = t1;
+    }
+}
+
+__global__ void __launch_bounds__(PTILE)
+k_in_replay(DevTable T, InState S, InBatchArgs B, uint32_t n_tiles, uint32_t hmask, bool gridsync)
+{
+    constexpr uint32_t NW = PTILE / 32u;
+    __shared__ uint32_t s_key[NW][32], s_gmax[NW][32];   // each warp's SA groups (by leader lane)
+    __shared__ uint32_t s_last;
+    const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
+    const uint32_t tile = blockIdx.x;
+    const uint32_t i = tile * PTILE + tid;
+    const uint32_t n_sa = T.n_sa;
+    // k_in_fused's flags / sequence numbers are complete after this
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+
+    // group by SA every packet that reaches the replay check (valid format);
+    // only members of A (authenticated) contribute their number, the rest 0
+    uint32_t key = INVALID_SA, q = 0;
+    bool inA = false;
+    if (i < B.n) {
+        const uint32_t f = S.flags[i];
+        if (f & INF_FMT) {
+            key = B.sa_idx[i];
+            inA = (f & INF_ICV) != 0;
+            q = inA ? S.seq[i] : 0u;
+        }
+    }
+    const uint32_t peers = __match_any_sync(0xffffffffu, key);
+    const uint32_t lt = peers & lanemask_lt();
+    uint32_t mex = 0;                                // max over earlier lanes of the group
+#pragma unroll
+    for (int l = 0; l < 32; l++) {
+        const uint32_t v = __shfl_sync(0xffffffffu, q, l);
+        if ((lt >> l) & 1u) mex = max(mex, v);
+    }
+    const uint32_t leader = __ffs(peers) - 1;
+    const uint32_t hi_lane = 31u - __clz(peers);
+    const uint32_t gmax = __shfl_sync(0xffffffffu, max(mex, q), hi_lane);
+    s_key[warp][lane] = lane == leader ? key : INVALID_SA;
+    s_gmax[warp][lane] = gmax;
+    __syncthreads();
+
+    // the same SA in the tile's other warps: earlier warps raise the prefix, a
+    // later one takes over writing the tile maximum (no per-SA shared array,
+    // so any number of SAs)
+    uint32_t base = 0;
+    bool later = false;
+    if (key != INVALID_SA) {
+#pragma unroll 1
+        for (uint32_t w = 0; w < NW; w++) {
+            if (w == warp) continue;
+#pragma unroll 8
+            for (uint32_t l = 0; l < 32; l++) {
+                if (s_key[w][l] == key) {
+                    if (w < warp) base = max(base, s_gmax[w][l]);
+                    else later = true;
+                }
+            }
+        }
+    }
+    if (i < B.n) S.lmax[i] = max(base, mex);
+    if (key != INVALID_SA) {
+        // per-tile SA maxima, nonzero only (0 is the identity: top_0 >= 0)
+        const uint32_t tmax = max(base, gmax);
+        if (!later && lane == hi_lane && tmax != 0u) S.hmax[(size_t)key * n_tiles + tile] = tmax;
+    }
+    if (inA) {
+        // (s, q) -> smallest packet index in A
+        const unsigned long long k64 = ((unsigned long long)key << 32) | q;
+        uint32_t h = hash_slot(k64, hmask);
+        while (true) {
+            const unsigned long long old = atomicCAS(&S.hkey[h], ~0ull, k64);
+            if (old == ~0ull || old == k64) {
+                atomicMin(&S.hval[h], i);
+                break;
+            }
+            h = (h + 1u) & hmask;
+        }
+    }
+
+    if (gridsync) {
+        in_grid_barrier(&S.ctl[1], &S.ctl[2]);
+        asm volatile("griddepcontrol.launch_dependents;");
+        const uint32_t nwarps = gridDim.x * (PTILE / 32u);
+        for (uint32_t sa = tile * (PTILE / 32u) + warp; sa < n_sa; sa += nwarps)
+            scan_max_row(S, sa, n_tiles, lane);
+    } else {
+        __threadfence();
+        __syncthreads();
+        if (tid == 0) s_last = (atomicAdd(&S.ctl[0], 1u) == n_tiles - 1u) ? 1u : 0u;
+        __syncthreads();
+        asm volatile("griddepcontrol.launch_dependents;");
+        if (!s_last) return;
+        __threadfence();
+        for (uint32_t sa = warp; sa < n_sa; sa += PTILE / 32u) scan_max_row(S, sa, n_tiles, lane);
+        __syncthreads();
+        if (tid == 0) S.ctl[0] = 0;
+    }
+}
+
+constexpr uint32_t DEC_THREADS = 256;
+
+__global__ void __launch_bounds__(DEC_THREADS)
+k_in_decide(DevTable T, InState S, InBatchArgs B, uint32_t n_tiles, uint32_t hmask)
+{
+    __shared__ unsigned long long s_cnt[N_IN_COUNTERS - 1];
+    const uint32_t tid = threadIdx.x, lane = tid & 31u;
+    const uint32_t i = blockIdx.x * DEC_THREADS + tid;
+    if (tid < N_IN_COUNTERS - 1) s_cnt[tid] = 0;
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    __syncthreads();
+
+    uint32_t st = 0xffu, D = 0, Lin = 0;
+    if (i < B.n) {
+        const uint32_t s = B.sa_idx[i];
+        const uint32_t f = S.flags[i];
+        if (s >= T.n_sa) {
+            st = ST_DROP_SA;
+        } else if (!(f & INF_FMT)) {
+            st = ST_DROP_FORMAT;
+        } else {
+            const uint32_t q = S.seq[i];
+            const uint32_t t0 = S.top_prev[s];
+            const unsigned long long b0 = S.bmp_prev[s];
+            const uint32_t tj = max(t0, max(S.pmx[(size_t)s * n_tiles + i / PTILE], S.lmax[i]));
+            bool pass = q != 0u;
+            if (pass && q <= tj) {
+                if (tj - q >= REPLAY_W) {
+                    pass = false;                                    // left of the window
+                } else if (q <= t0 && ((b0 >> (t0 - q)) & 1ull)) {
+                    pass = false;                                    // seen before the batch
+                } else {                                             // seen earlier in it?
+                    const unsigned long long k64 = ((unsigned long long)s << 32) | q;
+                    uint32_t h = hash_slot(k64, hmask);
+                    while (true) {
+                        const unsigned long long kk = S.hkey[h];
+                        if (kk == k64) {
+                            if (S.hval[h] < i) pass = false;
+                            break;
+                        }
+                        if (kk == ~0ull) break;
+                        h = (h + 1u) & hmask;
+                    }
+                }
+            }
+            if (!pass) {
+                st = ST_DROP_REPLAY;
+            } else if (!(f & INF_ICV)) {
+                st = ST_DROP_AUTH;
+            } else {
+                const uint32_t d = S.top[s] - q;                     // new right edge
+                if (d < REPLAY_W) atomicOr(&S.bmp[s], 1ull << d);
+                if (f & INF_TRL) {
+                    st = ST_OK;
+                    D = f & 0xffffu;
+                    Lin = B.in_len[i];
+                } else {
+                    st = ST_DROP_TRAILER;
+                }
+            }
+        }
+        B.out_len[i] = (uint16_t)D;
+        if (B.status) B.status[i] = (uint8_t)st;
+    }
+    // counters: pkts_ok, drop_sa, drop_format, drop_replay, drop_auth, drop_trailer,
+    // bytes_in, bytes_out (+ batches by block 0)
+#pragma unroll
+    for (uint32_t k = 0; k < 6; k++) {
+        const uint32_t c = __reduce_add_sync(0xffffffffu, st == k ? 1u : 0u);
+        if (lane == 0 && c) atomicAdd(&s_cnt[k], (unsigned long long)c);
+    }
+    const uint32_t bi = __reduce_add_sync(0xffffffffu, Lin);
+    const uint32_t bo = __reduce_add_sync(0xffffffffu, D);
+    if (lane == 0 && bi) atomicAdd(&s_cnt[6], (unsigned long long)bi);
+    if (lane == 0 && bo) atomicAdd(&s_cnt[7], (unsigned long long)bo);
+    __syncthreads();
+    if (tid < N_IN_COUNTERS - 1 && s_cnt[tid]) atomicAdd(&S.counters[tid], s_cnt[tid]);
+    if (tid == 0 && blockIdx.x == 0) atomicAdd(&S.counters[N_IN_COUNTERS - 1], 1ull);
+}
+
+static cudaError_t launch_pdl(const void *fn, dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                              void **args)
+{
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelExC(&cfg, fn, args);
+}
+
+cudaError_t launch_in_replay(const DevTable &T, const InState &S, const InBatchArgs &B,
+                             uint32_t n_tiles, uint32_t hmask, bool gridsync, cudaStream_t st)
+{
+    DevTable t = T;
+    InState s = S;
+    InBatchArgs b = B;
+    void *args[] = {&t, &s, &b, &n_tiles, &hmask, &gridsync};
+    return launch_pdl((const void *)k_in_replay, dim3(n_tiles), dim3(PTILE), 0, st, args);
+}
+
+cudaError_t launch_in_decide(const DevTable &T, const InState &S, const InBatchArgs &B,
+                             uint32_t n_tiles, uint32_t hmask, cudaStream_t st)
+{
+    DevTable t = T;
+    InState s = S;
+    InBatchArgs b = B;
+    void *args[] = {&t, &s, &b, &n_tiles, &hmask};
+    return launch_pdl((const void *)k_in_decide, dim3((B.n + DEC_THREADS - 1) / DEC_THREADS),
+                      dim3(DEC_THREADS), 0, st, args);
+}
+
+cudaError_t setup_in_fused_attributes();
+
+cudaError_t setup_inbound_attributes(uint32_t n_sa, uint32_t max_tiles, int num_sms, bool *gridsync)
+{
+    cudaError_t e = setup_in_fused_attributes();
+    if (e != cudaSuccess) return e;
+    (void)n_sa;
+    int per_sm = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_in_replay, PTILE, 0);
+    if (e != cudaSuccess) return e;
+    *gridsync = (uint64_t)per_sm * (uint64_t)num_sms >= (uint64_t)max_tiles;
+    return cudaSuccess;
+}
+
+}  // namespace nba

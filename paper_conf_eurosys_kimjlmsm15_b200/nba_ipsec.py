@@ -21,6 +21,8 @@ HEADER = os.path.join(os.path.dirname(_HERE), "include", "nba_ipsec.h")
 OK, EINVAL, ENOMEM, ENODEV, ECUDA = 0, -22, -12, -19, -1000
 PIPE_FUSED, PIPE_UNFUSED = 0, 1
 MIN_DATAGRAM, MAX_DATAGRAM, MAX_OVERHEAD = 20, 1500, 53
+IN_OK, IN_DROP_SA, IN_DROP_FORMAT, IN_DROP_REPLAY, IN_DROP_AUTH, IN_DROP_TRAILER = range(6)
+REPLAY_WINDOW = 64
 
 
 class NbaIpsecError(RuntimeError):
@@ -52,6 +54,25 @@ class Counters(ctypes.Structure):
         return {k: int(getattr(self, k)) for k, _ in self._fields_}
 
 
+class InBatch(ctypes.Structure):
+    _fields_ = [("in_buf", ctypes.c_void_p), ("in_off", ctypes.c_void_p),
+                ("in_len", ctypes.c_void_p), ("sa_idx", ctypes.c_void_p),
+                ("out_buf", ctypes.c_void_p), ("out_off", ctypes.c_void_p),
+                ("out_len", ctypes.c_void_p), ("status", ctypes.c_void_p),
+                ("n_pkts", ctypes.c_uint32)]
+
+
+class InCounters(ctypes.Structure):
+    _fields_ = [("pkts_ok", ctypes.c_uint64), ("drop_sa", ctypes.c_uint64),
+                ("drop_format", ctypes.c_uint64), ("drop_replay", ctypes.c_uint64),
+                ("drop_auth", ctypes.c_uint64), ("drop_trailer", ctypes.c_uint64),
+                ("bytes_in", ctypes.c_uint64), ("bytes_out", ctypes.c_uint64),
+                ("batches", ctypes.c_uint64)]
+
+    def as_dict(self):
+        return {k: int(getattr(self, k)) for k, _ in self._fields_}
+
+
 def _load():
     if not os.path.exists(LIB_PATH):
         raise ImportError(f"{LIB_PATH} is missing: run `python -m "
@@ -74,6 +95,12 @@ def _load():
         "nba_ipsec_profile_read": (i32, [vp, P(ctypes.c_double), P(ctypes.c_char_p), i32,
                                          P(i32), P(u32)]),
         "nba_ipsec_debug_trace": (i32, [vp, P(u64), u32]),
+        "nba_ipsec_enable_inbound": (i32, [vp]),
+        "nba_ipsec_process_inbound": (i32, [vp, P(InBatch), vp]),
+        "nba_ipsec_read_in_counters": (i32, [vp, P(InCounters), vp]),
+        "nba_ipsec_read_replay_window": (i32, [vp, P(u32), P(u64), vp]),
+        "nba_ipsec_profile_read_inbound": (i32, [vp, P(ctypes.c_double), P(ctypes.c_char_p), i32,
+                                                 P(i32), P(u32)]),
         "nba_ipsec_host_aes128_key_schedule": (None, [P(ctypes.c_uint8), P(u32)]),
         "nba_ipsec_host_hmac_sha1_midstates": (None, [P(ctypes.c_uint8), P(u32), P(u32)]),
     }
@@ -202,6 +229,43 @@ class SATable:
         nk, nb = ctypes.c_int(0), ctypes.c_uint32(0)
         _check(lib.nba_ipsec_profile_read(self._h, ms, names, 8, ctypes.byref(nk),
                                           ctypes.byref(nb)), "nba_ipsec_profile_read")
+        return {names[k].decode(): ms[k] for k in range(nk.value)}, int(nb.value)
+
+    # -- ESP inbound ------------------------------------------
+    def enable_inbound(self):
+        _check(lib.nba_ipsec_enable_inbound(self._h), "nba_ipsec_enable_inbound")
+
+    def process_inbound(self, in_buf, in_off, in_len, sa_idx, out_buf, out_off, out_len,
+                        status=None, n=None, stream=None):
+        """nba_ipsec_process_inbound on device tensors; status (uint8) optional."""
+        n = int(in_len.numel() if n is None else n)
+        b = InBatch(_ptr(in_buf), _ptr(in_off), _ptr(in_len), _ptr(sa_idx), _ptr(out_buf),
+                    _ptr(out_off), _ptr(out_len), _ptr(status), n)
+        _check(lib.nba_ipsec_process_inbound(self._h, ctypes.byref(b), _stream_handle(stream)),
+               "nba_ipsec_process_inbound")
+
+    def in_counters(self, stream=None) -> dict:
+        c = InCounters()
+        _check(lib.nba_ipsec_read_in_counters(self._h, ctypes.byref(c), _stream_handle(stream)),
+               "nba_ipsec_read_in_counters")
+        return c.as_dict()
+
+    def replay_window(self, stream=None):
+        top = np.zeros(self.n_sa, np.uint32)
+        bmp = np.zeros(self.n_sa, np.uint64)
+        _check(lib.nba_ipsec_read_replay_window(
+            self._h, top.ctypes.data_as(ctypes.POINTER(ctypes.c_uint32)),
+            bmp.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)), _stream_handle(stream)),
+            "nba_ipsec_read_replay_window")
+        return top, bmp
+
+    def profile_read_inbound(self) -> tuple[dict, int]:
+        ms = (ctypes.c_double * 3)()
+        names = (ctypes.c_char_p * 3)()
+        nk, nb = ctypes.c_int(0), ctypes.c_uint32(0)
+        _check(lib.nba_ipsec_profile_read_inbound(self._h, ms, names, 3, ctypes.byref(nk),
+                                                  ctypes.byref(nb)),
+               "nba_ipsec_profile_read_inbound")
         return {names[k].decode(): ms[k] for k in range(nk.value)}, int(nb.value)
 
     def debug_trace(self, n_cta: int = 148) -> np.ndarray:
