@@ -272,6 +272,82 @@ def run_ours(args):
                 "mpps": pkts_all * steps / s / 1e6,
                 "ms_per_step": tot_ms_max / steps}
 
+    def measure_inbound(cfg_id, steps, warmup):
+        """ESP inbound on the same traffic: the library's own
+        outbound output of the config's batch is decapsulated every step; the
+        receive windows are reset before each step (untimed, like the L2
+        flush) so every packet is fresh and accepted."""
+        size = CFG_SIZE[cfg_id]
+        p, b = shard.rank_workload(cfg_id, PKTS_PER_GPU, size, N_SA_TOTAL, rank, world)
+        t_out = nba_ipsec.SATable(p, device=local, max_batch=PKTS_PER_GPU)
+        db = device.to_device(b, dev)
+        t_out.process(*db.args(), n=b.n)
+        torch.cuda.synchronize()
+        esp_len = db.out_len[:b.n].cpu().numpy().view(np.uint16).astype(np.int64)
+        t_out.close()
+        t = nba_ipsec.SATable(p, device=local, max_batch=PKTS_PER_GPU)
+        t.enable_inbound()
+        inner = torch.empty_like(db.out_buf)
+        inner_len = torch.zeros_like(db.out_len)
+        args_in = (db.out_buf, db.out_off, db.out_len, db.sa_idx, inner, db.out_off, inner_len)
+        run = lambda: t.process_inbound(*args_in, n=b.n)  # noqa: E731
+        for _ in range(warmup):
+            flush.zero_()
+            t.reset_inbound()
+            run()
+        torch.cuda.synchronize()
+        barrier()
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+              for _ in range(steps)]
+        for k in range(steps):
+            flush.zero_()
+            t.reset_inbound()
+            ev[k][0].record()
+            run()
+            ev[k][1].record()
+        torch.cuda.synchronize()
+        barrier()
+        tot_ms = float(sum(a.elapsed_time(c) for a, c in ev))
+        t.profile_enable(True)
+        for k in range(max(10, steps // 4)):
+            flush.zero_()
+            t.reset_inbound()
+            run()
+        torch.cuda.synchronize()
+        kern, nb = t.profile_read_inbound()
+        t.profile_enable(False)
+        ctr = t.in_counters()
+        ok_all = ctr["pkts_ok"] == ctr["batches"] * b.n
+        same = bool(torch.equal(inner_len[:b.n].to(torch.int32), db.in_len[:b.n].to(torch.int32)))
+        t.close()
+        C = esp_len - 48
+        w = {"packets": int(b.n), "aes_blocks": int(((C + 15) // 16).sum()),
+             "sha1_compressions": int(((16 + C + 8) // 64 + 1 + 1).sum()),
+             "bytes_in": int(esp_len.sum()), "bytes_out": int(b.in_len.astype(np.int64).sum())}
+        tot_max = shard.max_over_ranks(tot_ms, device=dev)
+        red = shard.reduce_counters({"pkts_ok": frame_bits(b) / 8.0, "pkts_dropped": 0,
+                                     "bytes_in": b.n, "bytes_out": float((esp_len + 14).sum()),
+                                     "batches": 0}, device=dev)
+        sec = tot_max * 1e-3
+        kk = {k: v / max(nb, 1) for k, v in kern.items()}
+        rr = {}
+        for k, ms in kk.items():
+            if k == "in_fused":
+                x = kernel_roofline("fused", ms, w, peaks)
+            else:
+                x = {"bound": "hbm", "unit": "GB/s", "peak": peaks["hbm_gbs"],
+                     "achieved": w["packets"] * (16 if k == "in_replay" else 22) / (ms * 1e-3) / 1e9}
+            rr[k] = {"ms": ms, "frac": x["achieved"] / x["peak"], "unit": x["unit"],
+                     "achieved": x["achieved"], "bound": x["bound"]}
+            if "lds_frac" in x:
+                rr[k]["lds_frac"] = x["lds_frac"]
+        return {"gbps": 8.0 * red["pkts_ok"] * steps / sec / 1e9,
+                "gbps_esp_wire": 8.0 * red["bytes_out"] * steps / sec / 1e9,
+                "mpps": red["bytes_in"] * steps / sec / 1e6,
+                "ms_per_step": tot_max / steps, "steps": steps, "kernels": rr,
+                "all_accepted": bool(ok_all), "lengths_match_outbound_input": same,
+                "gpu_launches": 3 * steps}
+
     main_cfg = args.config
     res = measure(main_cfg, args.steps, args.warmup)
     agg = aggregate(res, args.steps)
@@ -319,6 +395,13 @@ def run_ours(args):
             per_size[str(CFG_SIZE[cfg_id])] = {"gbps": a2["gbps"], "mpps": a2["mpps"],
                                                "ms_per_step": a2["ms_per_step"], "kernels": rr}
 
+    # ---- ESP inbound on the same traffic ----------------------------
+    inbound = {}
+    if not args.no_inbound:
+        for cfg_id in (2, 3, 4):
+            inbound[str(CFG_SIZE[cfg_id])] = measure_inbound(cfg_id, max(10, args.steps // 4),
+                                                            max(3, args.warmup // 2))
+
     # ---- CPU baseline: the oracle on host cores (rank 0, N = 1 only) ----------
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
@@ -354,6 +437,7 @@ def run_ours(args):
                             "achieved": v["achieved"]} for k, v in kern_roofs.items()},
             "work_per_step_per_gpu": w,
             "per_size": per_size,
+            "inbound": inbound or None,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": res["launches"],
@@ -498,6 +582,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--pipeline", type=int, default=None, help="0 fused, 1 unfused")
     ap.add_argument("--no-sweep", action="store_true")
+    ap.add_argument("--no-inbound", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=3.0)
     args = ap.parse_args()

@@ -228,6 +228,9 @@ int nba_ipsec_enable_inbound(nba_ipsec_sa_table *t);
  * as process_batch.  NBA_IPSEC_EINVAL if inbound is not enabled, for NULL
  * arrays with n_pkts > 0 or n_pkts > max_batch_pkts. */
 int nba_ipsec_process_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batch *b, void *cuda_stream);
+/* Enqueue (on `cuda_stream`) a reset of every receive window to its initial
+ * state (reading B6), e.g. after re-keying; counters are kept. */
+int nba_ipsec_reset_inbound(nba_ipsec_sa_table *t, void *cuda_stream);
 /* Inbound counters since enable.  Synchronises `cuda_stream`. */
 int nba_ipsec_read_in_counters(nba_ipsec_sa_table *t, nba_ipsec_in_counters *out, void *cuda_stream);
 /* Receive windows: top[s] = highest authenticated number, bitmap[s] bit d set

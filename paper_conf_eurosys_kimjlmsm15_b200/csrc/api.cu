@@ -59,6 +59,8 @@ struct nba_ipsec_sa_table {
     bool in_enabled = false, in_gridsync = false;
     uint32_t in_hcap = 0;
     InState S{};
+    uint32_t *in_top0 = nullptr;              // the windows' initial state (reset)
+    unsigned long long *in_bmp0 = nullptr;
     double prof_in_ms[3] = {};
     uint32_t prof_in_batches = 0;
 };
@@ -226,6 +228,8 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
         chk(cudaMemcpy(d_te0, host_te0(), 256 * sizeof(uint32_t), cudaMemcpyHostToDevice));
     }
     if (e == cudaSuccess) chk(setup_prologue_attributes(n_sa, t->max_tiles, t->num_sms, &t->gridsync));
+    // testing: force the last-CTA (non co-resident) fallback of the per-SA scans
+    if (std::getenv("NBA_IPSEC_NO_GRIDSYNC")) t->gridsync = false;
     if (e == cudaSuccess) chk(setup_aes_attributes());
     if (e == cudaSuccess) chk(setup_fused_attributes());
     if (e == cudaSuccess) chk(cudaDeviceSynchronize());
@@ -506,14 +510,19 @@ int nba_ipsec_enable_inbound(nba_ipsec_sa_table *t)
     chk(dalloc(t, &S.hval, hcap));
     chk(dalloc(t, &S.counters, N_IN_COUNTERS));
     chk(dalloc(t, &S.ctl, 8));
+    chk(dalloc(t, &t->in_top0, n_sa));
+    chk(dalloc(t, &t->in_bmp0, n_sa));
     if (e == cudaSuccess) {
         // reading B6: the window starts at the SA's seq, everything <= seq seen
         std::vector<unsigned long long> bmp(n_sa);
         for (uint32_t s = 0; s < n_sa; s++) bmp[s] = t->seq0[s] ? ~0ull : 0ull;
         chk(cudaMemcpy(S.top, t->seq0.data(), n_sa * 4ull, cudaMemcpyHostToDevice));
         chk(cudaMemcpy(S.bmp, bmp.data(), n_sa * 8ull, cudaMemcpyHostToDevice));
+        chk(cudaMemcpy(t->in_top0, t->seq0.data(), n_sa * 4ull, cudaMemcpyHostToDevice));
+        chk(cudaMemcpy(t->in_bmp0, bmp.data(), n_sa * 8ull, cudaMemcpyHostToDevice));
     }
     if (e == cudaSuccess) chk(setup_inbound_attributes(n_sa, t->max_tiles, t->num_sms, &t->in_gridsync));
+    if (std::getenv("NBA_IPSEC_NO_GRIDSYNC")) t->in_gridsync = false;
     if (e == cudaSuccess) chk(cudaDeviceSynchronize());
     if (e != cudaSuccess) {
         cudaGetLastError();
@@ -561,6 +570,19 @@ int nba_ipsec_process_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batch *b
     mark();
     if (launch_in_decide(t->T, t->S, B, n_tiles, hmask, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
     mark();
+    return NBA_IPSEC_OK;
+}
+
+int nba_ipsec_reset_inbound(nba_ipsec_sa_table *t, void *cuda_stream)
+{
+    if (!t || !t->in_enabled) return NBA_IPSEC_EINVAL;
+    DeviceGuard g(t->device);
+    cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    if (cudaMemcpyAsync(t->S.top, t->in_top0, t->n_sa * 4ull, cudaMemcpyDeviceToDevice, st) !=
+            cudaSuccess ||
+        cudaMemcpyAsync(t->S.bmp, t->in_bmp0, t->n_sa * 8ull, cudaMemcpyDeviceToDevice, st) !=
+            cudaSuccess)
+        return NBA_IPSEC_ECUDA;
     return NBA_IPSEC_OK;
 }
 

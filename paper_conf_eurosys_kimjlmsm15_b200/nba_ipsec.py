@@ -98,6 +98,7 @@ def _load():
         "nba_ipsec_enable_inbound": (i32, [vp]),
         "nba_ipsec_process_inbound": (i32, [vp, P(InBatch), vp]),
         "nba_ipsec_read_in_counters": (i32, [vp, P(InCounters), vp]),
+        "nba_ipsec_reset_inbound": (i32, [vp, vp]),
         "nba_ipsec_read_replay_window": (i32, [vp, P(u32), P(u64), vp]),
         "nba_ipsec_profile_read_inbound": (i32, [vp, P(ctypes.c_double), P(ctypes.c_char_p), i32,
                                                  P(i32), P(u32)]),
@@ -243,6 +244,10 @@ class SATable:
                     _ptr(out_off), _ptr(out_len), _ptr(status), n)
         _check(lib.nba_ipsec_process_inbound(self._h, ctypes.byref(b), _stream_handle(stream)),
                "nba_ipsec_process_inbound")
+
+    def reset_inbound(self, stream=None):
+        _check(lib.nba_ipsec_reset_inbound(self._h, _stream_handle(stream)),
+               "nba_ipsec_reset_inbound")
 
     def in_counters(self, stream=None) -> dict:
         c = InCounters()

@@ -18,8 +18,7 @@ def _batches(b, out, ol, sizes, seed, **mix):
     bs, start = [], 0
     for n in sizes:
         order = (gen.arrival_order(b.n, n, r, **mix) + start) % b.n
-        bs.append(gen.esp_batch(out, b.out_off, ol, b.sa_idx, order,
-                                corrupt=mix.get("corrupt_", 0.0), r=r))
+        bs.append(gen.esp_batch(out, b.out_off, ol, b.sa_idx, order))
         start += n
     return bs
 
@@ -127,3 +126,45 @@ def test_empty_batch_and_errors():
     assert top.tolist() == [0] * 4 and bmp.tolist() == [0] * 4
     assert t.in_counters()["batches"] == 0
     t.close()
+
+
+def test_last_cta_scan_fallback(monkeypatch):
+    """k_in_replay's per-SA row scans on the last CTA (no grid barrier)."""
+    monkeypatch.setenv("NBA_IPSEC_NO_GRIDSYNC", "1")
+    n_sa = 40
+    p = gen.make_sas(n_sa, cfg_id=97)
+    b, out, ol = esp_source(p, 9000, "imix", 97)
+    bs = _batches(b, out, ol, [4000, 5000], 97, reorder=7, dup=0.05, old=0.04, old_span=2000)
+    assert_same_inbound(gpu_inbound_run(p, bs), oracle_inbound_run(p, bs), bs)
+
+
+def test_reset_inbound_replays_same_traffic():
+    """nba_ipsec_reset_inbound restores the initial windows: the same batch is
+    accepted again with identical output (the bench's steady-state protocol)."""
+    import torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    n_sa = 64
+    p = gen.make_sas(n_sa, cfg_id=98)
+    b, out, ol = esp_source(p, 5000, "imix", 98)
+    ib = gen.esp_batch(out, b.out_off, ol, b.sa_idx, np.arange(b.n))
+    t = nba_ipsec.SATable(p, max_batch=b.n)
+    t.enable_inbound()
+    db = device.to_device(ib, "cuda")
+    t.process_inbound(*db.args(), n=ib.n)
+    o1, l1 = device.fetch(db)
+    w1 = t.replay_window()
+    t.process_inbound(*db.args(), n=ib.n)          # all replays now
+    _, l2 = device.fetch(db)
+    assert (l2 == 0).all()
+    t.reset_inbound()
+    db.out_buf.zero_()
+    t.process_inbound(*db.args(), n=ib.n)
+    o3, l3 = device.fetch(db)
+    assert np.array_equal(l1, l3) and (l1 > 0).all()
+    assert np.array_equal(o1, o3)
+    w3 = t.replay_window()
+    assert np.array_equal(w1[0], w3[0]) and np.array_equal(w1[1], w3[1])
+    c = t.in_counters()
+    assert c["pkts_ok"] == 2 * ib.n and c["drop_replay"] == ib.n and c["batches"] == 3
+    t.close()
+    torch.cuda.synchronize()

@@ -147,3 +147,13 @@ def test_virtual_shards_union_equals_oracle():
                     o_out[b.out_off[i]:b.out_off[i] + L].tobytes()
                 seen[i] = True
         assert seen[b.sa_idx < n_sa].all()
+
+
+@pytest.mark.parametrize("pipe", PIPES)
+def test_last_cta_scan_fallback(pipe, monkeypatch):
+    """The per-SA column scans on the last CTA (the path taken when the prologue
+    grid cannot be co-resident), forced with NBA_IPSEC_NO_GRIDSYNC."""
+    monkeypatch.setenv("NBA_IPSEC_NO_GRIDSYNC", "1")
+    p = gen.make_sas(300, cfg_id=57)
+    bs = [gen.make_batch(20000, "imix", 300, cfg_id=57, batch=k) for k in range(2)]
+    assert_same(gpu_run(p, bs, pipeline=pipe), oracle_run(p, bs))
