@@ -133,11 +133,14 @@ int nba_ipsec_read_sa_seq(nba_ipsec_sa_table *t, uint32_t *host_seq, void *cuda_
 const char *nba_ipsec_strerror(int code);
 
 /* Pipeline selection (both produce identical bytes):
- *   NBA_IPSEC_PIPE_FUSED   : prologue + one fused gather/AES/HMAC/scatter kernel (default)
+ *   NBA_IPSEC_PIPE_FUSED   : one fused prologue/gather/AES/HMAC/scatter kernel when
+ *                            n_pkts <= 512 x SM count (cooperative launch, grid
+ *                            barriers), else prologue kernel + fused kernel (default)
  *   NBA_IPSEC_PIPE_UNFUSED : prologue, gather, AES-CTR, HMAC-SHA1, scatter kernels */
 enum { NBA_IPSEC_PIPE_FUSED = 0, NBA_IPSEC_PIPE_UNFUSED = 1 };
 int nba_ipsec_set_pipeline(nba_ipsec_sa_table *t, int pipeline);
-/* Number of kernel launches one process_batch call enqueues (n_pkts > 0). */
+/* Number of kernel launches the most recent process_batch call enqueued
+ * (2 before the first call). */
 int nba_ipsec_launches_per_batch(nba_ipsec_sa_table *t);
 
 /* Per-kernel timing with CUDA events recorded on the caller's stream between

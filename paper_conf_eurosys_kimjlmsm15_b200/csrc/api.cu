@@ -29,6 +29,7 @@ struct ProfSet {
     cudaEvent_t ev[MAX_KERNELS + 1] = {};
     int n_ev = 0;          // events recorded in this set (0 = empty)
     bool inbound = false;
+    const char **names = nullptr;
 };
 
 }  // namespace
@@ -40,6 +41,9 @@ struct nba_ipsec_sa_table {
     int grid_aes = 0, grid_fused = 0;
     int pipeline = NBA_IPSEC_PIPE_FUSED;
     bool gridsync = false;     // prologue phase 2 on all CTAs (grid barrier)
+    bool allow_merged = true;  // prologue inside the fused kernel when the batch fits
+    uint32_t bar_base = 0;     // arrivals so far at the fused kernel's grid barrier
+    int last_launches = 2;
     DevTable T{};
     DevWork W{};
     std::vector<void *> allocs;
@@ -54,6 +58,7 @@ struct nba_ipsec_sa_table {
     uint32_t prof_batches = 0;
     double prof_ms[MAX_KERNELS] = {};
     int prof_nk = 0;
+    const char **prof_names = nullptr;
     // ESP inbound (nba_ipsec_enable_inbound)
     std::vector<uint32_t> seq0;     // the SAs' initial seq (window start, reading B6)
     bool in_enabled = false, in_gridsync = false;
@@ -102,6 +107,7 @@ void free_all(nba_ipsec_sa_table *t)
 
 const char *kernel_names_unfused[] = {"prologue", "gather", "aes_ctr", "hmac_sha1", "scatter"};
 const char *kernel_names_fused[] = {"prologue", "fused"};
+const char *kernel_names_merged[] = {"fused"};
 
 void prof_drain_set(nba_ipsec_sa_table *t, ProfSet &s)
 {
@@ -120,6 +126,7 @@ void prof_drain_set(nba_ipsec_sa_table *t, ProfSet &s)
         t->prof_in_batches++;
     } else {
         t->prof_nk = s.n_ev - 1;
+        t->prof_names = s.names;
         t->prof_batches++;
     }
     s.n_ev = 0;
@@ -209,8 +216,10 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
     chk(dalloc(t, &W.m_seq, M));
     chk(dalloc(t, &W.m_info, M));
     chk(dalloc(t, &W.perm, M));
-    chk(dalloc(t, &W.hist16, (size_t)t->max_tiles * n_sa));
-    chk(dalloc(t, &W.hpfx, (size_t)t->max_tiles * n_sa));
+    // columns: prologue tiles, or the fused kernel's CTAs when it runs the prologue
+    const size_t cols = std::max<size_t>(t->max_tiles, (size_t)t->grid_fused);
+    chk(dalloc(t, &W.hist16, cols * n_sa));
+    chk(dalloc(t, &W.hpfx, cols * n_sa));
     chk(dalloc(t, &W.tile_rec, t->max_tiles));
     chk(dalloc(t, &W.tile_blk, t->max_tiles));
     chk(dalloc(t, &W.tile_bin, (size_t)t->max_tiles * NBINS));
@@ -230,6 +239,8 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
     if (e == cudaSuccess) chk(setup_prologue_attributes(n_sa, t->max_tiles, t->num_sms, &t->gridsync));
     // testing: force the last-CTA (non co-resident) fallback of the per-SA scans
     if (std::getenv("NBA_IPSEC_NO_GRIDSYNC")) t->gridsync = false;
+    // testing: always use the separate prologue kernel
+    if (std::getenv("NBA_IPSEC_NO_MERGE")) t->allow_merged = false;
     if (e == cudaSuccess) chk(setup_aes_attributes());
     if (e == cudaSuccess) chk(setup_fused_attributes());
     if (e == cudaSuccess) chk(cudaDeviceSynchronize());
@@ -262,6 +273,9 @@ static int enqueue(nba_ipsec_sa_table *t, const BatchArgs &B, cudaStream_t st)
         if (ps) cudaEventRecord(ps->ev[ps->n_ev++], st);
     };
     const bool unfused = t->pipeline == NBA_IPSEC_PIPE_UNFUSED;
+    const bool merged = !unfused && t->allow_merged && fused_merged_ok(B.n, t->grid_fused);
+    if (ps) ps->names = unfused ? kernel_names_unfused : merged ? kernel_names_merged : kernel_names_fused;
+    t->last_launches = unfused ? 5 : merged ? 1 : 2;
     if (t->W.trace) {   // debug only: reset the phase trace (mins start at ~0)
         static std::vector<unsigned long long> init;
         size_t nw = (size_t)t->grid_fused * 8 + 8;
@@ -273,11 +287,18 @@ static int enqueue(nba_ipsec_sa_table *t, const BatchArgs &B, cudaStream_t st)
         cudaMemcpyAsync(t->W.trace, init.data(), nw * 8, cudaMemcpyHostToDevice, st);
     }
     mark();
+    if (merged) {
+        if (launch_fused(t->T, t->W, B, t->grid_fused, true, &t->bar_base, st) != cudaSuccess)
+            return NBA_IPSEC_ECUDA;
+        mark();
+        return NBA_IPSEC_OK;
+    }
     if (launch_prologue(t->T, t->W, B, n_tiles, unfused, t->gridsync, st) != cudaSuccess)
         return NBA_IPSEC_ECUDA;
     mark();
     if (!unfused) {
-        if (launch_fused(t->T, t->W, B, t->grid_fused, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
+        if (launch_fused(t->T, t->W, B, t->grid_fused, false, &t->bar_base, st) != cudaSuccess)
+            return NBA_IPSEC_ECUDA;
         mark();
         return NBA_IPSEC_OK;
     }
@@ -447,7 +468,7 @@ int nba_ipsec_set_pipeline(nba_ipsec_sa_table *t, int pipeline)
 int nba_ipsec_launches_per_batch(nba_ipsec_sa_table *t)
 {
     if (!t) return NBA_IPSEC_EINVAL;
-    return t->pipeline == NBA_IPSEC_PIPE_FUSED ? 2 : 5;
+    return t->last_launches;
 }
 
 int nba_ipsec_profile_enable(nba_ipsec_sa_table *t, int enable)
@@ -470,8 +491,7 @@ int nba_ipsec_profile_read(nba_ipsec_sa_table *t, double *ms, const char **names
     if (!t) return NBA_IPSEC_EINVAL;
     DeviceGuard g(t->device);
     for (int k = 0; k < PROF_RING; k++) prof_drain_set(t, t->ring[(t->ring_next + k) % PROF_RING]);
-    const char **nm = t->pipeline == NBA_IPSEC_PIPE_FUSED ? kernel_names_fused
-                                                          : kernel_names_unfused;
+    const char **nm = t->prof_names ? t->prof_names : kernel_names_fused;
     int nk = t->prof_nk;
     for (int k = 0; k < nk && k < max; k++) {
         if (ms) ms[k] = t->prof_ms[k];

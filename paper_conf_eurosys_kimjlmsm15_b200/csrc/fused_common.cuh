@@ -24,6 +24,8 @@ struct FusedLo {
     uint4 rkA[4][F_THREADS];       // round keys 3..6 of the thread's current packet
     uint32_t bins[NBINS];
     unsigned long long cnt[4];
+    uint32_t hkey[2 * F_SUPER];    // merged prologue: SA of each slot of the CTA's SA hash
+    uint32_t hmask[2 * F_SUPER];   //   warps holding a group of that SA
 };
 
 struct FusedHi {

@@ -60,7 +60,7 @@ struct DevWork {
 };
 
 constexpr int CTL_TICKET = 0, CTL_TOTAL_REC = 1, CTL_TOTAL_BLK = 2, CTL_WORK = 3,
-              CTL_BAR_COUNT = 4, CTL_BAR_GEN = 5;
+              CTL_BAR_COUNT = 4, CTL_BAR_GEN = 5, CTL_BAR_MONO = 6;
 constexpr int NBINS = 32;   // HMAC bins by number of inner SHA-1 blocks (2..25)
 
 struct BatchArgs {
@@ -125,7 +125,8 @@ cudaError_t launch_hmac(const DevTable &T, const DevWork &W, const BatchArgs &B,
 cudaError_t launch_scatter(const DevTable &T, const DevWork &W, const BatchArgs &B,
                            uint32_t n_tiles, cudaStream_t st);
 cudaError_t launch_fused(const DevTable &T, const DevWork &W, const BatchArgs &B, int grid,
-                         cudaStream_t st);
+                         bool merged, uint32_t *bar_base, cudaStream_t st);
+bool fused_merged_ok(uint32_t n, int grid);
 cudaError_t setup_prologue_attributes(uint32_t n_sa, uint32_t max_tiles, int num_sms, bool *gridsync);
 cudaError_t setup_aes_attributes();
 cudaError_t setup_fused_attributes();
@@ -259,6 +260,104 @@ __device__ __forceinline__ uint32_t block_exclusive_scan(uint32_t v, uint32_t *s
     *total = scratch[nw - 1];
     return base + x - v;
 }
+
+// Grid-wide barrier for a co-resident (cooperatively launched) grid: a
+// monotonically increasing arrival counter; the host passes the count this
+// barrier waits for (previous arrivals + gridDim.x), so it never needs a reset.
+__device__ __forceinline__ void grid_sync_mono(uint32_t *count, uint32_t target)
+{
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        atomicAdd(count, 1u);
+        uint32_t v;
+        do {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(count) : "memory");
+        } while ((int)(v - target) < 0);
+        __threadfence();
+    }
+    __syncthreads();
+}
+
+// Exclusive prefix of the tile counts down SA column `sa` by one warp, then the
+// SA counter advance (only the first (2^32-1 - seq) packets get numbers).
+__device__ __forceinline__ void scan_sa_column(const DevTable &T, const DevWork &W, uint32_t sa,
+                                               uint32_t n_tiles, uint32_t lane)
+{
+    // the column is contiguous (SA-major): coalesced loads, all issued first
+    constexpr int U = 8;                       // 8 x 32 = 256 tiles per pass
+    uint16_t *col = W.hist16 + (size_t)sa * n_tiles;
+    uint32_t *pfx = W.hpfx + (size_t)sa * n_tiles;
+    uint32_t carry = 0;
+    for (uint32_t t0 = 0; t0 < n_tiles; t0 += 32u * U) {
+        uint32_t h[U];
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            const uint32_t t = t0 + 32u * u + lane;
+            h[u] = t < n_tiles ? __ldcg(&col[t]) : 0u;
+        }
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            if (t0 + 32u * u >= n_tiles) break;
+            uint32_t x = h[u];
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+                if (lane >= (uint32_t)o) x += y;
+            }
+            const uint32_t t = t0 + 32u * u + lane;
+            if (t < n_tiles) {
+                pfx[t] = carry + x - h[u];
+                if (h[u]) col[t] = 0;            // re-arm for the next batch
+            }
+            carry += __shfl_sync(0xffffffffu, x, 31);
+        }
+    }
+    if (lane == 0) {
+        const uint32_t old = T.seq[sa];
+        T.seq_prev[sa] = old;
+        const uint32_t room = 0xffffffffu - old;
+        T.seq[sa] = old + (carry < room ? carry : room);
+    }
+}
+
+
+// All SA rows, by `nslots` warps (this one is `slot`).  Long rows: one warp per
+// SA (scan_sa_column).  Short rows (small batches, n_tiles <= 32): one LANE per
+// SA, so a few warps still cover thousands of SAs in one memory round trip.
+__device__ __forceinline__ void scan_all_columns(const DevTable &T, const DevWork &W, uint32_t slot,
+                                                 uint32_t nslots, uint32_t n_tiles, uint32_t lane)
+{
+    if (n_tiles > 32u) {
+        for (uint32_t col = slot; col < T.n_sa; col += nslots) scan_sa_column(T, W, col, n_tiles, lane);
+        return;
+    }
+    for (uint32_t k0 = 0; (size_t)k0 * nslots < T.n_sa; k0 += 32u) {
+        // SA slot + k * nslots for k = k0 + lane: spread over all warps of the grid
+        const size_t sa_l = slot + (size_t)(k0 + lane) * nslots;
+        if (sa_l >= T.n_sa) continue;
+        const uint32_t sa = (uint32_t)sa_l;
+        uint16_t *col = W.hist16 + (size_t)sa * n_tiles;
+        uint32_t *pfx = W.hpfx + (size_t)sa * n_tiles;
+        uint32_t h[32];
+#pragma unroll
+        for (uint32_t t = 0; t < 32u; t++) h[t] = t < n_tiles ? __ldcg(&col[t]) : 0u;
+        uint32_t carry = 0;
+#pragma unroll
+        for (uint32_t t = 0; t < 32u; t++) {
+            if (t < n_tiles) {
+                pfx[t] = carry;
+                if (h[t]) col[t] = 0;            // re-arm for the next batch
+            }
+            carry += h[t];
+        }
+        const uint32_t old = T.seq[sa];
+        T.seq_prev[sa] = old;
+        const uint32_t room = 0xffffffffu - old;
+        T.seq[sa] = old + (carry < room ? carry : room);
+    }
+}
+
 #endif
 
 }  // namespace nba

@@ -25,9 +25,13 @@
 // (byte r of the state word in bits 8..15, lane*4 in bits 0..7, the table base
 // in bits 16..31) -- no address add per lookup.  Per-thread round keys and the
 // packet metadata live below (FusedLo) and above (FusedHi) the tables.
+#include <cstdlib>
+
 #include "fused_common.cuh"
 
 namespace nba {
+
+constexpr uint32_t INFO_TOSLOAD = 0x40000000u;   // esp_packet loads the TOS byte itself
 
 // ---------------------------------------------- one packet, one lane
 __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B, FusedLo &L,
@@ -37,7 +41,9 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
 {
     long long ck_start = clock64(), ck_setup = 0, ck_aes = 0, ck_sha = 0, ck_emit = 0;
     const uint32_t D = info & 0x7ffu;
-    const uint32_t tos = (info >> 16) & 0xffu;
+    // TOS of the inner header (outer header copies it, reading A13): from the
+    // metadata phase, or loaded here (merged prologue: off its critical path)
+    const uint32_t tos = (info & INFO_TOSLOAD) ? (uint32_t)__ldg(B.in_buf + inoff + 1) : (info >> 16) & 0xffu;
     const uint32_t pad = esp_pad(D);
     const uint32_t C = D + pad + 2u;
     const uint32_t Lb = 48u + C;
@@ -185,9 +191,68 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
     }
 }
 
+// ------------------------------------------- merged prologue (row a1 in-kernel)
+// When the whole batch fits in one super-round per CTA (n <= grid * F_SUPER),
+// the prologue runs inside this kernel: each CTA is one tile.  Per-SA ranks in
+// the CTA come from __match_any_sync groups merged across the 16 warps through
+// a small shared hash (slot per SA; per-warp group sizes); the CTA's per-SA
+// counts go to the SA-major matrix; after a grid barrier one warp per SA scans
+// its row (exclusive prefix over CTAs, SA counter advance); after a second
+// barrier every packet's sequence number is known.  Deterministic: no atomic
+// decides a rank.  Returns the packet's rank among the CTA's packets of its SA.
+__device__ __forceinline__ uint32_t merged_prologue(const DevTable &T, const DevWork &W, FusedLo &L,
+                                                    uint32_t s, uint32_t bar_base,
+                                                    unsigned long long *tr)
+{
+    constexpr uint32_t HS = 2u * F_SUPER, NW = F_THREADS / 32u;
+    const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
+    const uint32_t G = gridDim.x, cta = blockIdx.x;
+    uint16_t(*wcnt)[NW] = reinterpret_cast<uint16_t(*)[NW]>(&L.rkA[0][0]);   // [HS][NW], 32 KB
+    static_assert(sizeof(L.rkA) >= HS * NW * sizeof(uint16_t), "wcnt overlay");
+
+    const uint32_t peers = __match_any_sync(0xffffffffu, s);
+    const uint32_t leader = __ffs(peers) - 1, hi_lane = 31u - __clz(peers);
+    const uint32_t wrank = __popc(peers & lanemask_lt()), wcnt_me = __popc(peers);
+    uint32_t slot = 0;
+    if (s != INVALID_SA && lane == leader) {
+        slot = (s * 0x9E3779B1u) >> 22;                    // 10 bits -> HS = 1024
+        while (true) {
+            const uint32_t old = atomicCAS(&L.hkey[slot], INVALID_SA, s);
+            if (old == INVALID_SA || old == s) break;
+            slot = (slot + 1u) & (HS - 1u);
+        }
+        wcnt[slot][warp] = (uint16_t)wcnt_me;
+        atomicOr(&L.hmask[slot], 1u << warp);
+    }
+    slot = __shfl_sync(0xffffffffu, slot, leader);
+    __syncthreads();
+    uint32_t rank = 0;
+    if (s != INVALID_SA) {
+        const uint32_t m = L.hmask[slot];
+        uint32_t base = 0;
+#pragma unroll
+        for (uint32_t w = 0; w < NW; w++)
+            if (w < warp && ((m >> w) & 1u)) base += wcnt[slot][w];
+        rank = base + wrank;
+        // the SA's last group in the CTA writes the CTA's count (nonzero only;
+        // the row scan re-zeroes it)
+        if ((m >> (warp + 1u)) == 0u && lane == hi_lane)
+            W.hist16[(size_t)s * G + cta] = (uint16_t)(base + wcnt_me);
+    }
+    if (tr && tid == 0) tr[4] = gtimer();
+    grid_sync_mono(&W.ctl[CTL_BAR_MONO], bar_base + G);
+    if (tr && tid == 0) tr[5] = gtimer();
+    scan_all_columns(T, W, cta * NW + warp, G * NW, G, lane);
+    if (tr && tid == 0) tr[6] = gtimer();
+    grid_sync_mono(&W.ctl[CTL_BAR_MONO], bar_base + 2u * G);
+    if (tr && tid == 0) tr[7] = gtimer();
+    return rank;
+}
+
 // ---------------------------------------------------------------- the kernel
+template <bool MERGED>
 __global__ void __launch_bounds__(F_THREADS, 1)
-k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc)
+k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base)
 {
     extern __shared__ __align__(16) uint8_t smem[];
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
@@ -222,13 +287,29 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc)
             prefetch_l2(a);
         }
     }
-    aes_tables_to_smem(tabs, T.te0);
-    if (tid < 4) L.cnt[tid] = 0ull;
-    if (tid < NBINS) L.bins[tid] = 0;   // re-zeroed after each use (below)
-    __syncthreads();
-
     const uint32_t p_begin = blockIdx.x * ppc;
     const uint32_t p_end = min(B.n, p_begin + ppc);
+    // merged prologue: the packet metadata loads are issued before the table
+    // staging so their DRAM latency overlaps it
+    uint32_t pre_sa = INVALID_SA, pre_D = 0, pre_inoff = 0, pre_outoff = 0;
+    if (MERGED && p_begin + tid < p_end) {
+        pre_sa = B.sa_idx[p_begin + tid];
+        pre_D = B.in_len[p_begin + tid];
+        pre_inoff = B.in_off[p_begin + tid];
+        pre_outoff = B.out_off[p_begin + tid];
+    }
+    aes_tables_to_smem(tabs, T.te0);
+    if (tr && tid == 0) tr[2] = gtimer();
+    if (tid < 4) L.cnt[tid] = 0ull;
+    if (tid < NBINS) L.bins[tid] = 0;   // re-zeroed after each use (below)
+    if (MERGED) {
+        for (uint32_t k = tid; k < 2u * F_SUPER; k += F_THREADS) {
+            L.hkey[k] = INVALID_SA;
+            L.hmask[k] = 0;
+        }
+    }
+    __syncthreads();
+
     static_assert(F_SUPER <= F_THREADS, "one packet per thread in the metadata phase");
     uint32_t c_ok = 0, c_drop = 0, c_in = 0, c_out = 0;
 
@@ -242,25 +323,44 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc)
         uint32_t sa = INVALID_SA, D = 0, inoff = 0, tos = 0;
         bool cand = false;
         if (j < cnt_pk) {
-            sa = B.sa_idx[i];
-            D = B.in_len[i];
-            inoff = B.in_off[i];
-            L.outoff[j] = B.out_off[i];
+            if (MERGED) {
+                sa = pre_sa;
+                D = pre_D;
+                inoff = pre_inoff;
+                L.outoff[j] = pre_outoff;
+            } else {
+                sa = B.sa_idx[i];
+                D = B.in_len[i];
+                inoff = B.in_off[i];
+                L.outoff[j] = B.out_off[i];
+            }
             cand = sa < n_sa && D >= MIN_D && D <= MAX_D;
-            if (cand) tos = B.in_buf[inoff + 1];
+            if (cand && !MERGED) tos = B.in_buf[inoff + 1];
+            // merged: the lane reads the payload after the prologue; start the
+            // DRAM -> L2 transfer of its first line now
+            if (cand && MERGED) prefetch_l2(B.in_buf + inoff);
         }
-        // Programmatic dependent launch: the prologue's outputs (ranks, per-SA
-        // prefixes, seq_prev) are complete and visible after this.
-        if (base == p_begin) asm volatile("griddepcontrol.wait;" ::: "memory");
+        uint32_t rank = 0;
+        if (MERGED) {
+            // the prologue, in this kernel (single super-round per CTA)
+            rank = merged_prologue(T, W, L, cand ? sa : INVALID_SA, bar_base, tr);
+        } else if (base == p_begin) {
+            // Programmatic dependent launch: the prologue kernel's outputs (ranks,
+            // per-SA prefixes, seq_prev) are complete and visible after this.
+            asm volatile("griddepcontrol.wait;" ::: "memory");
+        }
         // 1b. sequence number, drop decision, length bin
         if (j < cnt_pk) {
             uint32_t info = 0, bin = NBINS - 1, q32 = 0;
             if (cand) {
-                const unsigned long long q = (unsigned long long)T.seq_prev[sa] + 1ull +
-                                             W.hpfx[(size_t)sa * ((B.n + PTILE - 1) / PTILE) + i / PTILE] + W.lrank[i];
+                const unsigned long long q =
+                    MERGED ? (unsigned long long)__ldcg(&T.seq_prev[sa]) + 1ull +
+                                 __ldcg(&W.hpfx[(size_t)sa * gridDim.x + blockIdx.x]) + rank
+                           : (unsigned long long)T.seq_prev[sa] + 1ull +
+                                 W.hpfx[(size_t)sa * ((B.n + PTILE - 1) / PTILE) + i / PTILE] + W.lrank[i];
                 if (q <= 0xffffffffull) {   // RFC 4303 §3.3.3: never cycle
                     q32 = (uint32_t)q;
-                    info = D | (tos << 16) | INFO_OK;
+                    info = D | (tos << 16) | INFO_OK | (MERGED ? INFO_TOSLOAD : 0u);
                     bin = hmac_bin(true, esp_C(D));
                 }
             }
@@ -347,8 +447,13 @@ uint32_t fused_ppc(uint32_t n, int grid)
     return ppc < 32u ? 32u : ppc;
 }
 
+bool fused_merged_ok(uint32_t n, int grid)
+{
+    return fused_ppc(n, grid) <= (uint32_t)F_SUPER;
+}
+
 cudaError_t launch_fused(const DevTable &T, const DevWork &W, const BatchArgs &B, int grid,
-                         cudaStream_t st)
+                         bool merged, uint32_t *bar_base, cudaStream_t st)
 {
     uint32_t ppc = fused_ppc(B.n, grid);
     uint32_t g = (B.n + ppc - 1) / ppc;
@@ -358,16 +463,31 @@ cudaError_t launch_fused(const DevTable &T, const DevWork &W, const BatchArgs &B
     cfg.dynamicSmemBytes = F_SMEM;
     cfg.stream = st;
     cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    static const bool no_coop = std::getenv("NBA_IPSEC_NO_COOP") != nullptr;   // A/B only
+    if (merged) {
+        // grid barriers inside: the driver must make all CTAs co-resident
+        attr[0].id = cudaLaunchAttributeCooperative;
+        attr[0].val.cooperative = no_coop ? 0 : 1;
+    } else {
+        attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        attr[0].val.programmaticStreamSerializationAllowed = 1;
+    }
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    return cudaLaunchKernelEx(&cfg, k_fused, T, W, B, ppc);
+    const uint32_t bb = *bar_base;
+    cudaError_t e = merged ? cudaLaunchKernelEx(&cfg, k_fused<true>, T, W, B, ppc, bb)
+                           : cudaLaunchKernelEx(&cfg, k_fused<false>, T, W, B, ppc, bb);
+    if (e == cudaSuccess && merged) *bar_base = bb + 2u * g;
+    return e;
 }
 
 cudaError_t setup_fused_attributes()
 {
-    return cudaFuncSetAttribute(k_fused, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)F_SMEM);
+    cudaError_t e = cudaFuncSetAttribute(k_fused<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)F_SMEM);
+    if (e != cudaSuccess) return e;
+    return cudaFuncSetAttribute(k_fused<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)F_SMEM);
 }
 
 }  // namespace nba

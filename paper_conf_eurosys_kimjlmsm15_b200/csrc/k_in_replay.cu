@@ -50,6 +50,18 @@ __device__ __forceinline__ void in_grid_barrier(uint32_t *count, uint32_t *gen)
     __syncthreads();
 }
 
+__device__ __forceinline__ void window_advance(const InState &S, uint32_t sa, uint32_t batch_max)
+{
+    const uint32_t t0 = S.top[sa];
+    const unsigned long long b0 = S.bmp[sa];
+    S.top_prev[sa] = t0;
+    S.bmp_prev[sa] = b0;
+    const uint32_t t1 = max(t0, batch_max);
+    const uint32_t sh = t1 - t0;
+    S.bmp[sa] = sh >= REPLAY_W ? 0ull : (b0 << sh);
+    S.top[sa] = t1;
+}
+
 // Exclusive prefix max down SA row `sa` of the tile maxima by one warp, then
 // the window edge update for the batch.
 __device__ __forceinline__ void scan_max_row(const InState &S, uint32_t sa, uint32_t n_tiles,
@@ -85,15 +97,37 @@ __device__ __forceinline__ void scan_max_row(const InState &S, uint32_t sa, uint
             carry = max(carry, __shfl_sync(0xffffffffu, x, 31));
         }
     }
-    if (lane == 0) {
-        const uint32_t t0 = S.top[sa];
-        const unsigned long long b0 = S.bmp[sa];
-        S.top_prev[sa] = t0;
-        S.bmp_prev[sa] = b0;
-        const uint32_t t1 = max(t0, carry);
-        const uint32_t sh = t1 - t0;
-        S.bmp[sa] = sh >= REPLAY_W ? 0ull : (b0 << sh);
-        S.top[sa] = t1;
+    if (lane == 0) window_advance(S, sa, carry);
+}
+
+// All SA rows by `nslots` warps (this one is `slot`): one warp per SA for long
+// rows, one lane per SA for short ones (small batches, n_tiles <= 32).
+__device__ __forceinline__ void scan_all_rows(const InState &S, uint32_t n_sa, uint32_t slot,
+                                              uint32_t nslots, uint32_t n_tiles, uint32_t lane)
+{
+    if (n_tiles > 32u) {
+        for (uint32_t sa = slot; sa < n_sa; sa += nslots) scan_max_row(S, sa, n_tiles, lane);
+        return;
+    }
+    for (uint32_t k0 = 0; (size_t)k0 * nslots < n_sa; k0 += 32u) {
+        const size_t sa_l = slot + (size_t)(k0 + lane) * nslots;
+        if (sa_l >= n_sa) continue;
+        const uint32_t sa = (uint32_t)sa_l;
+        uint32_t *row = S.hmax + (size_t)sa * n_tiles;
+        uint32_t *pfx = S.pmx + (size_t)sa * n_tiles;
+        uint32_t h[32];
+#pragma unroll
+        for (uint32_t t = 0; t < 32u; t++) h[t] = t < n_tiles ? __ldcg(&row[t]) : 0u;
+        uint32_t carry = 0;
+#pragma unroll
+        for (uint32_t t = 0; t < 32u; t++) {
+            if (t < n_tiles) {
+                pfx[t] = carry;
+                if (h[t]) row[t] = 0;
+            }
+            carry = max(carry, h[t]);
+        }
+        window_advance(S, sa, carry);
     }
 }
 
@@ -101,12 +135,19 @@ __global__ void __launch_bounds__(PTILE)
 k_in_replay(DevTable T, InState S, InBatchArgs B, uint32_t n_tiles, uint32_t hmask, bool gridsync)
 {
     constexpr uint32_t NW = PTILE / 32u;
-    __shared__ uint32_t s_key[NW][32], s_gmax[NW][32];   // each warp's SA groups (by leader lane)
+    constexpr uint32_t HS = 2u * PTILE;                  // tile hash: <= PTILE distinct SAs
+    __shared__ uint32_t s_hkey[HS];                       // SA in the slot (INVALID_SA = free)
+    __shared__ uint32_t s_hmax[HS][NW];                   // the SA's group max in warp w
+    __shared__ uint32_t s_hmask[HS];                      // warps that hold a group of the SA
     __shared__ uint32_t s_last;
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
     const uint32_t tile = blockIdx.x;
     const uint32_t i = tile * PTILE + tid;
     const uint32_t n_sa = T.n_sa;
+    for (uint32_t k = tid; k < HS; k += PTILE) {
+        s_hkey[k] = INVALID_SA;
+        s_hmask[k] = 0;
+    }
     // k_in_fused's flags / sequence numbers are complete after this
     asm volatile("griddepcontrol.wait;" ::: "memory");
 
@@ -133,27 +174,33 @@ k_in_replay(DevTable T, InState S, InBatchArgs B, uint32_t n_tiles, uint32_t hma
     const uint32_t leader = __ffs(peers) - 1;
     const uint32_t hi_lane = 31u - __clz(peers);
     const uint32_t gmax = __shfl_sync(0xffffffffu, max(mex, q), hi_lane);
-    s_key[warp][lane] = lane == leader ? key : INVALID_SA;
-    s_gmax[warp][lane] = gmax;
-    __syncthreads();
+    __syncthreads();   // tile hash initialised
 
-    // the same SA in the tile's other warps: earlier warps raise the prefix, a
-    // later one takes over writing the tile maximum (no per-SA shared array,
-    // so any number of SAs)
+    // merge the warps' groups of the same SA through a small shared hash:
+    // the group leader claims the SA's slot and records its warp's group max;
+    // earlier warps then raise the prefix, and the last warp holding the SA
+    // writes the tile maximum (any number of SAs per table)
+    uint32_t slot = 0;
+    if (key != INVALID_SA && lane == leader) {
+        slot = (key * 0x9E3779B1u) >> 23;               // 9 bits -> HS = 512 slots
+        while (true) {
+            const uint32_t old = atomicCAS(&s_hkey[slot], INVALID_SA, key);
+            if (old == INVALID_SA || old == key) break;
+            slot = (slot + 1u) & (HS - 1u);
+        }
+        s_hmax[slot][warp] = gmax;
+        atomicOr(&s_hmask[slot], 1u << warp);
+    }
+    slot = __shfl_sync(0xffffffffu, slot, leader);
+    __syncthreads();
     uint32_t base = 0;
     bool later = false;
     if (key != INVALID_SA) {
-#pragma unroll 1
-        for (uint32_t w = 0; w < NW; w++) {
-            if (w == warp) continue;
-#pragma unroll 8
-            for (uint32_t l = 0; l < 32; l++) {
-                if (s_key[w][l] == key) {
-                    if (w < warp) base = max(base, s_gmax[w][l]);
-                    else later = true;
-                }
-            }
-        }
+        const uint32_t m = s_hmask[slot];
+#pragma unroll
+        for (uint32_t w = 0; w < NW; w++)
+            if (w < warp && ((m >> w) & 1u)) base = max(base, s_hmax[slot][w]);
+        later = (m >> (warp + 1u)) != 0u;
     }
     if (i < B.n) S.lmax[i] = max(base, mex);
     if (key != INVALID_SA) {
@@ -178,9 +225,7 @@ k_in_replay(DevTable T, InState S, InBatchArgs B, uint32_t n_tiles, uint32_t hma
     if (gridsync) {
         in_grid_barrier(&S.ctl[1], &S.ctl[2]);
         asm volatile("griddepcontrol.launch_dependents;");
-        const uint32_t nwarps = gridDim.x * (PTILE / 32u);
-        for (uint32_t sa = tile * (PTILE / 32u) + warp; sa < n_sa; sa += nwarps)
-            scan_max_row(S, sa, n_tiles, lane);
+        scan_all_rows(S, n_sa, tile * (PTILE / 32u) + warp, gridDim.x * (PTILE / 32u), n_tiles, lane);
     } else {
         __threadfence();
         __syncthreads();
@@ -189,7 +234,7 @@ k_in_replay(DevTable T, InState S, InBatchArgs B, uint32_t n_tiles, uint32_t hma
         asm volatile("griddepcontrol.launch_dependents;");
         if (!s_last) return;
         __threadfence();
-        for (uint32_t sa = warp; sa < n_sa; sa += PTILE / 32u) scan_max_row(S, sa, n_tiles, lane);
+        scan_all_rows(S, n_sa, warp, PTILE / 32u, n_tiles, lane);
         __syncthreads();
         if (tid == 0) S.ctl[0] = 0;
     }

@@ -43,48 +43,6 @@ __device__ __forceinline__ void grid_barrier(uint32_t *count, uint32_t *gen)
     __syncthreads();
 }
 
-// Exclusive prefix of the tile counts down SA column `sa` by one warp, then the
-// SA counter advance (only the first (2^32-1 - seq) packets get numbers).
-__device__ __forceinline__ void scan_sa_column(const DevTable &T, const DevWork &W, uint32_t sa,
-                                               uint32_t n_tiles, uint32_t lane)
-{
-    // the column is contiguous (SA-major): coalesced loads, all issued first
-    constexpr int U = 8;                       // 8 x 32 = 256 tiles per pass
-    uint16_t *col = W.hist16 + (size_t)sa * n_tiles;
-    uint32_t *pfx = W.hpfx + (size_t)sa * n_tiles;
-    uint32_t carry = 0;
-    for (uint32_t t0 = 0; t0 < n_tiles; t0 += 32u * U) {
-        uint32_t h[U];
-#pragma unroll
-        for (int u = 0; u < U; u++) {
-            const uint32_t t = t0 + 32u * u + lane;
-            h[u] = t < n_tiles ? __ldcg(&col[t]) : 0u;
-        }
-#pragma unroll
-        for (int u = 0; u < U; u++) {
-            if (t0 + 32u * u >= n_tiles) break;
-            uint32_t x = h[u];
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-                if (lane >= (uint32_t)o) x += y;
-            }
-            const uint32_t t = t0 + 32u * u + lane;
-            if (t < n_tiles) {
-                pfx[t] = carry + x - h[u];
-                if (h[u]) col[t] = 0;            // re-arm for the next batch
-            }
-            carry += __shfl_sync(0xffffffffu, x, 31);
-        }
-    }
-    if (lane == 0) {
-        const uint32_t old = T.seq[sa];
-        T.seq_prev[sa] = old;
-        const uint32_t room = 0xffffffffu - old;
-        T.seq[sa] = old + (carry < room ? carry : room);
-    }
-}
-
 // Unfused pipeline only: exclusive scans of the per-tile record / AES-block
 // totals and of the HMAC length bins (bin-major, tile-minor).
 __device__ __forceinline__ void scan_tile_totals(const DevWork &W, uint32_t n_tiles, uint32_t *s_scr)
@@ -196,9 +154,7 @@ k_prologue(DevTable T, DevWork W, BatchArgs B, uint32_t n_tiles, bool unfused, b
         // let the dependent (fused) kernel launch and stage its tables; it waits
         // for this grid's completion before reading our outputs
         asm volatile("griddepcontrol.launch_dependents;");
-        const uint32_t nwarps = gridDim.x * (PTILE / 32u);
-        for (uint32_t col = tile * (PTILE / 32u) + warp; col < n_sa; col += nwarps)
-            scan_sa_column(T, W, col, n_tiles, lane);
+        scan_all_columns(T, W, tile * (PTILE / 32u) + warp, gridDim.x * (PTILE / 32u), n_tiles, lane);
         if (unfused && tile == 0) scan_tile_totals(W, n_tiles, s_scr);
     } else {
         // ---- phase 2 on the last CTA to finish phase 1 -----------------------
@@ -210,8 +166,7 @@ k_prologue(DevTable T, DevWork W, BatchArgs B, uint32_t n_tiles, bool unfused, b
         if (!s_last) return;
         __threadfence();
         if (tr && tid == 0) tr[2] = gtimer();
-        for (uint32_t col = warp; col < n_sa; col += PTILE / 32u)
-            scan_sa_column(T, W, col, n_tiles, lane);
+        scan_all_columns(T, W, warp, PTILE / 32u, n_tiles, lane);
         if (unfused) scan_tile_totals(W, n_tiles, s_scr);
         __syncthreads();
         if (tid == 0) W.ctl[CTL_TICKET] = 0;            // re-arm for the next batch

@@ -157,3 +157,51 @@ def test_last_cta_scan_fallback(pipe, monkeypatch):
     p = gen.make_sas(300, cfg_id=57)
     bs = [gen.make_batch(20000, "imix", 300, cfg_id=57, batch=k) for k in range(2)]
     assert_same(gpu_run(p, bs, pipeline=pipe), oracle_run(p, bs))
+
+
+@pytest.mark.parametrize("cfg", [2, 4])
+def test_two_kernel_fused_path(cfg, monkeypatch):
+    """The prologue kernel + fused kernel path (used when a batch exceeds one
+    super-round per CTA), forced with NBA_IPSEC_NO_MERGE at full size."""
+    monkeypatch.setenv("NBA_IPSEC_NO_MERGE", "1")
+    c = gen.CONFIGS[cfg]
+    p = gen.make_sas(c["n_sa"], cfg_id=cfg)
+    bs = [gen.make_batch(c["n"], c["size"], c["n_sa"], cfg_id=cfg, batch=k) for k in range(2)]
+    assert_same(gpu_run(p, bs, pipeline=0), oracle_run(p, bs))
+
+
+def test_large_batch_uses_two_kernels():
+    """n > 512 x SMs: several super-rounds per CTA behind the prologue kernel."""
+    from paper_conf_eurosys_kimjlmsm15_b200 import nba_ipsec
+    n, n_sa = 100000, 700
+    p = gen.make_sas(n_sa, cfg_id=58)
+    bs = [gen.make_batch(n, "imix", n_sa, cfg_id=58, batch=k) for k in range(2)]
+    t = nba_ipsec.SATable(p, max_batch=n)
+    g = gpu_run(p, bs, table=t)
+    assert t.launches_per_batch() == 2
+    t.close()
+    assert_same(g, oracle_run(p, bs))
+
+
+def test_concurrent_tables_on_two_streams():
+    """Two tables on two streams with interleaved launches (the merged kernel's
+    grid barriers rely on cooperative launch for co-residency)."""
+    import torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    ps = [gen.make_sas(64, cfg_id=59 + k) for k in range(2)]
+    bs = [[gen.make_batch(30000, "imix", 64, cfg_id=59 + k, batch=j) for j in range(3)]
+          for k in range(2)]
+    ts = [nba_ipsec.SATable(ps[k], max_batch=30000) for k in range(2)]
+    ss = [torch.cuda.Stream() for _ in range(2)]
+    dbs = [[device.to_device(b, "cuda") for b in bs[k]] for k in range(2)]
+    torch.cuda.synchronize()
+    for j in range(3):
+        for k in range(2):
+            with torch.cuda.stream(ss[k]):
+                ts[k].process(*dbs[k][j].args(), n=bs[k][j].n, stream=ss[k])
+    torch.cuda.synchronize()
+    for k in range(2):
+        res = [device.fetch(d) for d in dbs[k]]
+        assert ts[k].launches_per_batch() == 1
+        assert_same((res, ts[k].sa_seq(), ts[k].counters()), oracle_run(ps[k], bs[k]))
+        ts[k].close()

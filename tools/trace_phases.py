@@ -9,13 +9,17 @@ import torch  # noqa: E402
 
 from paper_conf_eurosys_kimjlmsm15_b200 import device, gen, nba_ipsec  # noqa: E402
 
-for cfg in (2, 3, 4):
+FLUSH = "--flush" in sys.argv
+flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda") if FLUSH else None
+for cfg in [int(x) for x in sys.argv[1:] if x.isdigit()] or (2, 3, 4):
     c = gen.CONFIGS[cfg]
     p = gen.make_sas(c["n_sa"], cfg_id=cfg)
     b = gen.make_batch(c["n"], c["size"], c["n_sa"], cfg_id=cfg)
     t = nba_ipsec.SATable(p, max_batch=c["n"])
     db = device.to_device(b, "cuda")
     for _ in range(5):
+        if flush is not None:
+            flush.zero_()
         t.process(*db.args(), n=b.n)
     torch.cuda.synchronize()
     full = t.debug_trace(148).astype(np.int64)
@@ -23,12 +27,14 @@ for cfg in (2, 3, 4):
     tr = full[:-1]
     live = tr[:, 0] > 0
     tr = tr[live]
-    t0 = pro[0]
+    t0 = pro[0] if pro[0] > 0 else tr[:, 0].min()
     print("prologue: first start 0, tiles done %.2f, last-CTA start %.2f, end %.2f us" %
           ((pro[1] - t0) / 1e3, (pro[2] - t0) / 1e3, (pro[3] - t0) / 1e3))
     rel = (tr - t0) / 1000.0
-    names = ["start", "meta_done", "aes_done", "hmac_done", "first_ready", "last_ready"]
-    print(f"config {cfg} ({c['name']}), {live.sum()} CTAs, times in us from first CTA start")
+    names = ["start", "meta_done", "tables_done", "lanes_done", "m_tiles_done", "m_bar1_done",
+             "m_scans_done", "m_bar2_done"]
+    print(f"config {cfg} ({c['name']}), {live.sum()} CTAs, times in us from the prologue's first "
+          f"CTA start{' (L2 flushed before the batch)' if FLUSH else ''}")
     for k, nm in enumerate(names):
         col = rel[:, k]
         print(f"  {nm:12s} min {col.min():8.2f}  med {np.median(col):8.2f}  max {col.max():8.2f}")
