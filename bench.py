@@ -338,7 +338,8 @@ def run_ours(args):
                 x = {"bound": "hbm", "unit": "GB/s", "peak": peaks["hbm_gbs"],
                      "achieved": w["packets"] * (16 if k == "in_replay" else 22) / (ms * 1e-3) / 1e9}
             rr[k] = {"ms": ms, "frac": x["achieved"] / x["peak"], "unit": x["unit"],
-                     "achieved": x["achieved"], "bound": x["bound"]}
+                     "achieved": x["achieved"], "bound": x["bound"],
+                     "traffic": load_traffic(k, gen.CONFIGS[cfg_id]["name"])}
             if "lds_frac" in x:
                 rr[k]["lds_frac"] = x["lds_frac"]
         return {"gbps": 8.0 * red["pkts_ok"] * steps / sec / 1e9,

@@ -43,6 +43,16 @@ SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "ns": 1e-9, "us": 
          "usecond": 1e-6, "msecond": 1e-3, "nsecond": 1e-9, "Ghz": 1e9, "Mhz": 1e6}
 
 
+ALIAS = {"aes": "aes_ctr", "hmac": "hmac_sha1"}
+
+
+def short_name(full):
+    """'void nba::k_fused<1>(nba::DevTable, ...)' -> 'fused' (bench.py's kernel names)."""
+    n = full.split("(")[0].replace("void ", "").replace("nba::", "").split("<")[0]
+    n = n[2:] if n.startswith("k_") else n
+    return ALIAS.get(n, n)
+
+
 def raw(rep):
     out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True,
                          text=True).stdout
@@ -52,7 +62,7 @@ def raw(rep):
     h, units, data = rows[0], rows[1], rows[2:]
     res = []
     for r in data:
-        d = {"kernel": r[h.index("Kernel Name")].split("(")[0].replace("nba::", "")}
+        d = {"kernel": short_name(r[h.index("Kernel Name")])}
         for m, short in METRICS:
             if m in h:
                 v, u = r[h.index(m)].replace(",", ""), units[h.index(m)]
@@ -94,6 +104,24 @@ def main(tag):
             kj[f"{k}:{name}"] = {"dram_bytes_per_launch": d["dram_read"] + d["dram_write"],
                                  "ncu_duration_us": d["duration"] * 1e6,
                                  "source": os.path.basename(rep)}
+        lines.append("")
+    for c, name in CFG.items():
+        rep = os.path.join(OUT, f"prof_{tag}_in_{c}.ncu-rep")
+        if not os.path.exists(rep):
+            continue
+        lines += [f"## {name} ESP inbound (k_in_fused -> k_in_replay -> k_in_decide)", "",
+                  "| kernel | us | DRAM rd MB | DRAM wr MB | issue % | ALU % | LSU % | warp inst | regs |",
+                  "|---|---|---|---|---|---|---|---|---|"]
+        for d0 in raw(rep):
+            d = collections.defaultdict(lambda: float("nan"))
+            d.update({m: (v if isinstance(v, float) else float("nan")) for m, v in d0.items()})
+            lines.append(f"| {d0['kernel']} | {d['duration'] * 1e6:.1f} | {d['dram_read'] / 1e6:.2f} | "
+                         f"{d['dram_write'] / 1e6:.2f} | {d['issue_active_pct']:.1f} | "
+                         f"{d['alu_pipe_pct']:.1f} | {d['lsu_inst_pct']:.1f} | "
+                         f"{d['warp_instructions']:.3g} | {d['registers']:.0f} |")
+            kj[f"{d0['kernel']}:{name}"] = {"dram_bytes_per_launch": d["dram_read"] + d["dram_write"],
+                                            "ncu_duration_us": d["duration"] * 1e6,
+                                            "source": os.path.basename(rep)}
         lines.append("")
     rep = os.path.join(OUT, f"prof_{tag}_unfused_c3.ncu-rep")
     if os.path.exists(rep):
@@ -141,10 +169,8 @@ def main(tag):
             pass
     with open(os.path.join(PROF, f"{tag}_ncu_summary.md"), "w") as f:
         f.write("\n".join(lines))
-    old = {}
+    old = {"_round": tag}
     pj = os.path.join(PROF, "ncu_kernels.json")
-    if os.path.exists(pj):
-        old = json.load(open(pj))
     old.update(kj)
     with open(pj, "w") as f:
         json.dump(old, f, indent=1)
