@@ -148,7 +148,7 @@ def main(tag):
         agg = collections.defaultdict(list)
         for r in rows[hdr + 1:]:
             if len(r) > vi:
-                agg[r[ki].split("(")[0]].append(float(r[vi].replace(",", "")))
+                agg[r[ki].split("(")[0].replace("void ", "")].append(float(r[vi].replace(",", "")))
         tot = sum(sum(v) for k, v in agg.items() if k.startswith("nba::"))
         lines += ["## launch list (bench.py --steps 5, `--metrics gpu__time_duration.sum`)", "",
                   "| kernel | launches | mean ns | share of our kernels |", "|---|---|---|---|"]
