@@ -108,15 +108,27 @@ int nba_ipsec_process_batch(nba_ipsec_sa_table *t, const nba_ipsec_batch *b, voi
 
 /* Same computation with HOST buffers (end-to-end path): copies
  * in_buf[0, in_buf_bytes), in_off, in_len, sa_idx host->device, runs the
- * path, copies out_buf[0, out_buf_bytes) and out_len device->host, all
- * enqueued on `cuda_stream`.  Needs staging reserved with
- * nba_ipsec_reserve_host_io; returns NBA_IPSEC_EINVAL if it is too small.
- * The host buffers must stay valid until the stream passes the batch. */
+ * path, copies out_buf[0, out_buf_bytes) and out_len device->host.  The copies
+ * and the kernels run on three internal streams with two staging slots, so
+ * consecutive calls overlap batch k+1's copy-in and batch k-1's copy-out with
+ * batch k's kernels (pinned host memory makes the copies asynchronous).
+ * Ordering: the kernels start after all work already on `cuda_stream`, and
+ * later work on `cuda_stream` waits for them (so the SA counters follow call
+ * order, also when mixed with nba_ipsec_process_batch).  The OUTPUTS reach host
+ * memory asynchronously: call nba_ipsec_host_wait(t, stream) and synchronise
+ * that stream before reading out_buf / out_len or reusing any host buffer of
+ * an earlier call.  out_buf[0, out_buf_bytes) is copied back whole: bytes
+ * outside the slots' [0, out_len[i]) receive unspecified values.  Needs staging
+ * reserved with nba_ipsec_reserve_host_io (EINVAL if it is too small). */
 int nba_ipsec_process_batch_host(nba_ipsec_sa_table *t, const nba_ipsec_batch *b,
                                  uint64_t in_buf_bytes, uint64_t out_buf_bytes,
                                  void *cuda_stream);
+/* Allocate (or grow) the two staging slots of the host path; synchronous. */
 int nba_ipsec_reserve_host_io(nba_ipsec_sa_table *t, uint64_t in_buf_bytes,
                               uint64_t out_buf_bytes);
+/* Make `cuda_stream` wait until every batch submitted so far through
+ * nba_ipsec_process_batch_host has its outputs in host memory. */
+int nba_ipsec_host_wait(nba_ipsec_sa_table *t, void *cuda_stream);
 
 /* Free everything.  NULL -> NBA_IPSEC_OK.  Synchronises the table's device. */
 int nba_ipsec_destroy(nba_ipsec_sa_table *t);

@@ -47,10 +47,20 @@ struct nba_ipsec_sa_table {
     DevTable T{};
     DevWork W{};
     std::vector<void *> allocs;
-    // host-I/O staging (process_batch_host)
-    uint8_t *io_in = nullptr, *io_out = nullptr;
+    // host-I/O pipeline (process_batch_host): IO_DEPTH staging slots, copy-in /
+    // compute / copy-out on three internal streams so batch k+1's H2D and batch
+    // k-1's D2H overlap batch k's kernels
+    static constexpr int IO_DEPTH = 2;
+    struct IoSlot {
+        uint8_t *in = nullptr, *out = nullptr;
+        uint32_t *meta = nullptr;   // in_off, sa_idx, out_off (u32) + in_len, out_len (u16)
+        cudaEvent_t in_ready = nullptr, done = nullptr, out_done = nullptr;
+    } io[IO_DEPTH];
     uint64_t io_in_bytes = 0, io_out_bytes = 0;
-    uint32_t *io_meta = nullptr;   // in_off, sa_idx, out_off (u32) + in_len, out_len (u16)
+    bool io_ready = false;
+    unsigned io_next = 0;
+    cudaStream_t s_h2d = nullptr, s_comp = nullptr, s_d2h = nullptr;
+    cudaEvent_t ev_call = nullptr;
     // profiling
     bool prof = false;
     ProfSet ring[PROF_RING];
@@ -328,38 +338,64 @@ int nba_ipsec_process_batch(nba_ipsec_sa_table *t, const nba_ipsec_batch *b, voi
     return enqueue(t, B, static_cast<cudaStream_t>(cuda_stream));
 }
 
+static void io_free(nba_ipsec_sa_table *t)
+{
+    for (auto &sl : t->io) {
+        if (sl.in) cudaFree(sl.in);
+        if (sl.out) cudaFree(sl.out);
+        if (sl.meta) cudaFree(sl.meta);
+        sl.in = sl.out = nullptr;
+        sl.meta = nullptr;
+    }
+    t->io_in_bytes = t->io_out_bytes = 0;
+}
+
 int nba_ipsec_reserve_host_io(nba_ipsec_sa_table *t, uint64_t in_buf_bytes, uint64_t out_buf_bytes)
 {
     if (!t) return NBA_IPSEC_EINVAL;
     DeviceGuard g(t->device);
-    if (in_buf_bytes > t->io_in_bytes) {
-        if (t->io_in) cudaFree(t->io_in);
-        t->io_in = nullptr;
-        if (cudaMalloc(&t->io_in, in_buf_bytes + 16) != cudaSuccess) {
-            cudaGetLastError();
-            t->io_in_bytes = 0;
-            return NBA_IPSEC_ENOMEM;
+    cudaError_t e = cudaSuccess;
+    auto chk = [&](cudaError_t x) {
+        if (e == cudaSuccess && x != cudaSuccess) e = x;
+    };
+    if (!t->s_h2d) {
+        chk(cudaStreamCreateWithFlags(&t->s_h2d, cudaStreamNonBlocking));
+        chk(cudaStreamCreateWithFlags(&t->s_comp, cudaStreamNonBlocking));
+        chk(cudaStreamCreateWithFlags(&t->s_d2h, cudaStreamNonBlocking));
+        chk(cudaEventCreateWithFlags(&t->ev_call, cudaEventDisableTiming));
+        for (auto &sl : t->io) {
+            chk(cudaEventCreateWithFlags(&sl.in_ready, cudaEventDisableTiming));
+            chk(cudaEventCreateWithFlags(&sl.done, cudaEventDisableTiming));
+            chk(cudaEventCreateWithFlags(&sl.out_done, cudaEventDisableTiming));
         }
-        t->io_in_bytes = in_buf_bytes;
-    }
-    if (out_buf_bytes > t->io_out_bytes) {
-        if (t->io_out) cudaFree(t->io_out);
-        t->io_out = nullptr;
-        if (cudaMalloc(&t->io_out, out_buf_bytes + 16) != cudaSuccess) {
+        if (e != cudaSuccess) {
             cudaGetLastError();
-            t->io_out_bytes = 0;
-            return NBA_IPSEC_ENOMEM;
-        }
-        t->io_out_bytes = out_buf_bytes;
-    }
-    if (!t->io_meta) {
-        // 3 u32 arrays + 2 u16 arrays of max_batch entries
-        size_t bytes = (size_t)t->max_batch * 16 + 64;
-        if (cudaMalloc(&t->io_meta, bytes) != cudaSuccess) {
-            cudaGetLastError();
-            return NBA_IPSEC_ENOMEM;
+            return NBA_IPSEC_ECUDA;
         }
     }
+    if (in_buf_bytes <= t->io_in_bytes && out_buf_bytes <= t->io_out_bytes && t->io_ready)
+        return NBA_IPSEC_OK;
+    // grow: wait for batches in flight, then reallocate every slot
+    cudaStreamSynchronize(t->s_h2d);
+    cudaStreamSynchronize(t->s_comp);
+    cudaStreamSynchronize(t->s_d2h);
+    const uint64_t inb = std::max(in_buf_bytes, t->io_in_bytes);
+    const uint64_t outb = std::max(out_buf_bytes, t->io_out_bytes);
+    io_free(t);
+    t->io_ready = false;
+    for (auto &sl : t->io) {
+        chk(cudaMalloc(&sl.in, inb + 16));
+        chk(cudaMalloc(&sl.out, outb + 16));
+        chk(cudaMalloc(&sl.meta, (size_t)t->max_batch * 16 + 64));
+    }
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        io_free(t);
+        return NBA_IPSEC_ENOMEM;
+    }
+    t->io_in_bytes = inb;
+    t->io_out_bytes = outb;
+    t->io_ready = true;
     return NBA_IPSEC_OK;
 }
 
@@ -372,12 +408,14 @@ int nba_ipsec_process_batch_host(nba_ipsec_sa_table *t, const nba_ipsec_batch *b
     if (!b->in_buf || !b->in_off || !b->in_len || !b->sa_idx || !b->out_buf || !b->out_off ||
         !b->out_len)
         return NBA_IPSEC_EINVAL;
-    if (!t->io_meta || in_buf_bytes > t->io_in_bytes || out_buf_bytes > t->io_out_bytes)
+    if (!t->io_ready || in_buf_bytes > t->io_in_bytes || out_buf_bytes > t->io_out_bytes)
         return NBA_IPSEC_EINVAL;
     DeviceGuard g(t->device);
     cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    auto &sl = t->io[t->io_next % nba_ipsec_sa_table::IO_DEPTH];
+    t->io_next++;
     const uint32_t n = b->n_pkts;
-    uint32_t *d_in_off = t->io_meta;
+    uint32_t *d_in_off = sl.meta;
     uint32_t *d_sa = d_in_off + t->max_batch;
     uint32_t *d_out_off = d_sa + t->max_batch;
     uint16_t *d_in_len = reinterpret_cast<uint16_t *>(d_out_off + t->max_batch);
@@ -386,17 +424,41 @@ int nba_ipsec_process_batch_host(nba_ipsec_sa_table *t, const nba_ipsec_batch *b
     auto chk = [&](cudaError_t x) {
         if (e == cudaSuccess && x != cudaSuccess) e = x;
     };
-    chk(cudaMemcpyAsync(t->io_in, b->in_buf, in_buf_bytes, cudaMemcpyHostToDevice, st));
-    chk(cudaMemcpyAsync(d_in_off, b->in_off, n * 4ull, cudaMemcpyHostToDevice, st));
-    chk(cudaMemcpyAsync(d_sa, b->sa_idx, n * 4ull, cudaMemcpyHostToDevice, st));
-    chk(cudaMemcpyAsync(d_out_off, b->out_off, n * 4ull, cudaMemcpyHostToDevice, st));
-    chk(cudaMemcpyAsync(d_in_len, b->in_len, n * 2ull, cudaMemcpyHostToDevice, st));
+    // copy-in: after this slot's previous copy-out has drained its buffers
+    chk(cudaStreamWaitEvent(t->s_h2d, sl.out_done, 0));
+    chk(cudaMemcpyAsync(sl.in, b->in_buf, in_buf_bytes, cudaMemcpyHostToDevice, t->s_h2d));
+    chk(cudaMemcpyAsync(d_in_off, b->in_off, n * 4ull, cudaMemcpyHostToDevice, t->s_h2d));
+    chk(cudaMemcpyAsync(d_sa, b->sa_idx, n * 4ull, cudaMemcpyHostToDevice, t->s_h2d));
+    chk(cudaMemcpyAsync(d_out_off, b->out_off, n * 4ull, cudaMemcpyHostToDevice, t->s_h2d));
+    chk(cudaMemcpyAsync(d_in_len, b->in_len, n * 2ull, cudaMemcpyHostToDevice, t->s_h2d));
+    chk(cudaEventRecord(sl.in_ready, t->s_h2d));
+    // compute: after the inputs and after everything the caller's stream holds
+    // (keeps the SA counters in call order with device-path batches)
+    chk(cudaEventRecord(t->ev_call, st));
+    chk(cudaStreamWaitEvent(t->s_comp, t->ev_call, 0));
+    chk(cudaStreamWaitEvent(t->s_comp, sl.in_ready, 0));
     if (e != cudaSuccess) return NBA_IPSEC_ECUDA;
-    BatchArgs B{t->io_in, d_in_off, d_in_len, d_sa, t->io_out, d_out_off, d_out_len, n};
-    int rc = enqueue(t, B, st);
+    BatchArgs B{sl.in, d_in_off, d_in_len, d_sa, sl.out, d_out_off, d_out_len, n};
+    int rc = enqueue(t, B, t->s_comp);
     if (rc != NBA_IPSEC_OK) return rc;
-    chk(cudaMemcpyAsync(b->out_buf, t->io_out, out_buf_bytes, cudaMemcpyDeviceToHost, st));
-    chk(cudaMemcpyAsync(b->out_len, d_out_len, n * 2ull, cudaMemcpyDeviceToHost, st));
+    chk(cudaEventRecord(sl.done, t->s_comp));
+    chk(cudaStreamWaitEvent(st, sl.done, 0));        // later work on the caller's stream
+    // copy-out
+    chk(cudaStreamWaitEvent(t->s_d2h, sl.done, 0));
+    chk(cudaMemcpyAsync(b->out_buf, sl.out, out_buf_bytes, cudaMemcpyDeviceToHost, t->s_d2h));
+    chk(cudaMemcpyAsync(b->out_len, d_out_len, n * 2ull, cudaMemcpyDeviceToHost, t->s_d2h));
+    chk(cudaEventRecord(sl.out_done, t->s_d2h));
+    return e == cudaSuccess ? NBA_IPSEC_OK : NBA_IPSEC_ECUDA;
+}
+
+int nba_ipsec_host_wait(nba_ipsec_sa_table *t, void *cuda_stream)
+{
+    if (!t) return NBA_IPSEC_EINVAL;
+    if (!t->s_d2h) return NBA_IPSEC_OK;
+    DeviceGuard g(t->device);
+    cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    cudaError_t e = cudaEventRecord(t->ev_call, t->s_d2h);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(st, t->ev_call, 0);
     return e == cudaSuccess ? NBA_IPSEC_OK : NBA_IPSEC_ECUDA;
 }
 
@@ -407,9 +469,16 @@ int nba_ipsec_destroy(nba_ipsec_sa_table *t)
         DeviceGuard g(t->device);
         cudaDeviceSynchronize();
         free_all(t);
-        if (t->io_in) cudaFree(t->io_in);
-        if (t->io_out) cudaFree(t->io_out);
-        if (t->io_meta) cudaFree(t->io_meta);
+        io_free(t);
+        for (auto &sl : t->io) {
+            if (sl.in_ready) cudaEventDestroy(sl.in_ready);
+            if (sl.done) cudaEventDestroy(sl.done);
+            if (sl.out_done) cudaEventDestroy(sl.out_done);
+        }
+        if (t->ev_call) cudaEventDestroy(t->ev_call);
+        if (t->s_h2d) cudaStreamDestroy(t->s_h2d);
+        if (t->s_comp) cudaStreamDestroy(t->s_comp);
+        if (t->s_d2h) cudaStreamDestroy(t->s_d2h);
     }
     delete t;
     return NBA_IPSEC_OK;

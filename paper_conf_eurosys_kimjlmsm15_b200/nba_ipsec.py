@@ -85,6 +85,7 @@ def _load():
         "nba_ipsec_process_batch": (i32, [vp, P(Batch), vp]),
         "nba_ipsec_process_batch_host": (i32, [vp, P(Batch), u64, u64, vp]),
         "nba_ipsec_reserve_host_io": (i32, [vp, u64, u64]),
+        "nba_ipsec_host_wait": (i32, [vp, vp]),
         "nba_ipsec_destroy": (i32, [vp]),
         "nba_ipsec_read_counters": (i32, [vp, P(Counters), vp]),
         "nba_ipsec_read_sa_seq": (i32, [vp, P(u32), vp]),
@@ -201,6 +202,10 @@ class SATable:
         _check(lib.nba_ipsec_process_batch_host(self._h, ctypes.byref(b), int(in_bytes),
                                                 int(out_bytes), _stream_handle(stream)),
                "nba_ipsec_process_batch_host")
+
+    def host_wait(self, stream=None):
+        """nba_ipsec_host_wait: `stream` waits for every host-path batch's outputs."""
+        _check(lib.nba_ipsec_host_wait(self._h, _stream_handle(stream)), "nba_ipsec_host_wait")
 
     # -- auxiliary -------------------------------------------------------------
     def counters(self, stream=None) -> dict:
