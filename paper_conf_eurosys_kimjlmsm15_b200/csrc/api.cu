@@ -43,6 +43,7 @@ struct nba_ipsec_sa_table {
     bool gridsync = false;     // prologue phase 2 on all CTAs (grid barrier)
     bool allow_merged = true;  // prologue inside the fused kernel when the batch fits
     uint32_t bar_base = 0;     // arrivals so far at the fused kernel's grid barrier
+    uint32_t epoch = 0;        // tag of the last in-kernel prologue's published bases
     int last_launches = 2;
     DevTable T{};
     DevWork W{};
@@ -230,6 +231,7 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
     const size_t cols = std::max<size_t>(t->max_tiles, (size_t)t->grid_fused);
     chk(dalloc(t, &W.hist16, cols * n_sa));
     chk(dalloc(t, &W.hpfx, cols * n_sa));
+    chk(dalloc(t, &W.hbase, (size_t)t->grid_fused * n_sa));
     chk(dalloc(t, &W.tile_rec, t->max_tiles));
     chk(dalloc(t, &W.tile_blk, t->max_tiles));
     chk(dalloc(t, &W.tile_bin, (size_t)t->max_tiles * NBINS));
@@ -298,7 +300,7 @@ static int enqueue(nba_ipsec_sa_table *t, const BatchArgs &B, cudaStream_t st)
     }
     mark();
     if (merged) {
-        if (launch_fused(t->T, t->W, B, t->grid_fused, true, &t->bar_base, st) != cudaSuccess)
+        if (launch_fused(t->T, t->W, B, t->grid_fused, true, &t->bar_base, &t->epoch, st) != cudaSuccess)
             return NBA_IPSEC_ECUDA;
         mark();
         return NBA_IPSEC_OK;
@@ -307,7 +309,7 @@ static int enqueue(nba_ipsec_sa_table *t, const BatchArgs &B, cudaStream_t st)
         return NBA_IPSEC_ECUDA;
     mark();
     if (!unfused) {
-        if (launch_fused(t->T, t->W, B, t->grid_fused, false, &t->bar_base, st) != cudaSuccess)
+        if (launch_fused(t->T, t->W, B, t->grid_fused, false, &t->bar_base, &t->epoch, st) != cudaSuccess)
             return NBA_IPSEC_ECUDA;
         mark();
         return NBA_IPSEC_OK;

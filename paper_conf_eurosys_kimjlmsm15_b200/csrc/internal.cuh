@@ -48,6 +48,7 @@ struct DevWork {
     uint16_t *hist16;       // [n_sa][n_tiles] per-SA per-prologue-tile packet counts (SA-major;
                             //   all-zero between batches)
     uint32_t *hpfx;         // [n_sa][n_tiles] exclusive prefix of hist16 along each SA row
+    unsigned long long *hbase;   // [n_sa][G] in-kernel prologue: epoch << 33 | (seq_prev + prefix)
     uint32_t *tile_rec;     // [max_tiles] record chunks per tile -> exclusive prefix
     uint32_t *tile_blk;     // [max_tiles] AES blocks per tile -> exclusive prefix
     uint32_t *tile_bin;     // [max_tiles * NBINS] HMAC length bins per tile -> prefix
@@ -125,7 +126,7 @@ cudaError_t launch_hmac(const DevTable &T, const DevWork &W, const BatchArgs &B,
 cudaError_t launch_scatter(const DevTable &T, const DevWork &W, const BatchArgs &B,
                            uint32_t n_tiles, cudaStream_t st);
 cudaError_t launch_fused(const DevTable &T, const DevWork &W, const BatchArgs &B, int grid,
-                         bool merged, uint32_t *bar_base, cudaStream_t st);
+                         bool merged, uint32_t *bar_base, uint32_t *epoch, cudaStream_t st);
 bool fused_merged_ok(uint32_t n, int grid);
 cudaError_t setup_prologue_attributes(uint32_t n_sa, uint32_t max_tiles, int num_sms, bool *gridsync);
 cudaError_t setup_aes_attributes();
@@ -281,13 +282,42 @@ __device__ __forceinline__ void grid_sync_mono(uint32_t *count, uint32_t target)
 
 // Exclusive prefix of the tile counts down SA column `sa` by one warp, then the
 // SA counter advance (only the first (2^32-1 - seq) packets get numbers).
-__device__ __forceinline__ void scan_sa_column(const DevTable &T, const DevWork &W, uint32_t sa,
-                                               uint32_t n_tiles, uint32_t lane)
+__device__ __forceinline__ void st_relaxed_u64(unsigned long long *p, unsigned long long v)
 {
-    // the column is contiguous (SA-major): coalesced loads, all issued first
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long *p)
+{
+    unsigned long long v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
+// Where a row scan puts its exclusive prefixes: the prologue kernel writes
+// hpfx[t] (read after a kernel boundary); the in-kernel prologue (BASE) writes
+// hbase[t] = epoch << 33 | (seq_prev + prefix) with the batch's epoch, which the
+// consuming CTA polls instead of waiting at a second grid barrier.
+template <bool BASE>
+__device__ __forceinline__ void put_prefix(const DevWork &W, size_t idx, uint32_t pfx, uint32_t old,
+                                           uint32_t epoch)
+{
+    if (BASE)
+        st_relaxed_u64(&W.hbase[idx], ((unsigned long long)epoch << 33) | ((unsigned long long)old + pfx));
+    else
+        W.hpfx[idx] = pfx;
+}
+
+// Exclusive prefix of the tile counts down SA row `sa` by one warp (coalesced:
+// the matrix is SA-major), then the SA counter advance (only the first
+// (2^32-1 - seq) packets get numbers).
+template <bool BASE>
+__device__ __forceinline__ void scan_sa_column(const DevTable &T, const DevWork &W, uint32_t sa,
+                                               uint32_t n_tiles, uint32_t lane, uint32_t epoch)
+{
     constexpr int U = 8;                       // 8 x 32 = 256 tiles per pass
     uint16_t *col = W.hist16 + (size_t)sa * n_tiles;
-    uint32_t *pfx = W.hpfx + (size_t)sa * n_tiles;
+    const uint32_t old = __shfl_sync(0xffffffffu, lane == 0 ? T.seq[sa] : 0u, 0);
     uint32_t carry = 0;
     for (uint32_t t0 = 0; t0 < n_tiles; t0 += 32u * U) {
         uint32_t h[U];
@@ -307,29 +337,30 @@ __device__ __forceinline__ void scan_sa_column(const DevTable &T, const DevWork 
             }
             const uint32_t t = t0 + 32u * u + lane;
             if (t < n_tiles) {
-                pfx[t] = carry + x - h[u];
+                put_prefix<BASE>(W, (size_t)sa * n_tiles + t, carry + x - h[u], old, epoch);
                 if (h[u]) col[t] = 0;            // re-arm for the next batch
             }
             carry += __shfl_sync(0xffffffffu, x, 31);
         }
     }
     if (lane == 0) {
-        const uint32_t old = T.seq[sa];
         T.seq_prev[sa] = old;
         const uint32_t room = 0xffffffffu - old;
         T.seq[sa] = old + (carry < room ? carry : room);
     }
 }
 
-
 // All SA rows, by `nslots` warps (this one is `slot`).  Long rows: one warp per
 // SA (scan_sa_column).  Short rows (small batches, n_tiles <= 32): one LANE per
 // SA, so a few warps still cover thousands of SAs in one memory round trip.
+template <bool BASE = false>
 __device__ __forceinline__ void scan_all_columns(const DevTable &T, const DevWork &W, uint32_t slot,
-                                                 uint32_t nslots, uint32_t n_tiles, uint32_t lane)
+                                                 uint32_t nslots, uint32_t n_tiles, uint32_t lane,
+                                                 uint32_t epoch = 0)
 {
     if (n_tiles > 32u) {
-        for (uint32_t col = slot; col < T.n_sa; col += nslots) scan_sa_column(T, W, col, n_tiles, lane);
+        for (uint32_t col = slot; col < T.n_sa; col += nslots)
+            scan_sa_column<BASE>(T, W, col, n_tiles, lane, epoch);
         return;
     }
     for (uint32_t k0 = 0; (size_t)k0 * nslots < T.n_sa; k0 += 32u) {
@@ -338,7 +369,7 @@ __device__ __forceinline__ void scan_all_columns(const DevTable &T, const DevWor
         if (sa_l >= T.n_sa) continue;
         const uint32_t sa = (uint32_t)sa_l;
         uint16_t *col = W.hist16 + (size_t)sa * n_tiles;
-        uint32_t *pfx = W.hpfx + (size_t)sa * n_tiles;
+        const uint32_t old = T.seq[sa];
         uint32_t h[32];
 #pragma unroll
         for (uint32_t t = 0; t < 32u; t++) h[t] = t < n_tiles ? __ldcg(&col[t]) : 0u;
@@ -346,12 +377,11 @@ __device__ __forceinline__ void scan_all_columns(const DevTable &T, const DevWor
 #pragma unroll
         for (uint32_t t = 0; t < 32u; t++) {
             if (t < n_tiles) {
-                pfx[t] = carry;
+                put_prefix<BASE>(W, (size_t)sa * n_tiles + t, carry, old, epoch);
                 if (h[t]) col[t] = 0;            // re-arm for the next batch
             }
             carry += h[t];
         }
-        const uint32_t old = T.seq[sa];
         T.seq_prev[sa] = old;
         const uint32_t room = 0xffffffffu - old;
         T.seq[sa] = old + (carry < room ? carry : room);

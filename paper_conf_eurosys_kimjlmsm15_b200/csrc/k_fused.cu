@@ -201,7 +201,7 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
 // barrier every packet's sequence number is known.  Deterministic: no atomic
 // decides a rank.  Returns the packet's rank among the CTA's packets of its SA.
 __device__ __forceinline__ uint32_t merged_prologue(const DevTable &T, const DevWork &W, FusedLo &L,
-                                                    uint32_t s, uint32_t bar_base,
+                                                    uint32_t s, uint32_t bar_base, uint32_t epoch,
                                                     unsigned long long *tr)
 {
     constexpr uint32_t HS = 2u * F_SUPER, NW = F_THREADS / 32u;
@@ -242,17 +242,17 @@ __device__ __forceinline__ uint32_t merged_prologue(const DevTable &T, const Dev
     if (tr && tid == 0) tr[4] = gtimer();
     grid_sync_mono(&W.ctl[CTL_BAR_MONO], bar_base + G);
     if (tr && tid == 0) tr[5] = gtimer();
-    scan_all_columns(T, W, cta * NW + warp, G * NW, G, lane);
+    // row scans publish epoch-tagged bases; no second barrier: each packet
+    // polls its own (SA, CTA) entry
+    scan_all_columns<true>(T, W, cta * NW + warp, G * NW, G, lane, epoch);
     if (tr && tid == 0) tr[6] = gtimer();
-    grid_sync_mono(&W.ctl[CTL_BAR_MONO], bar_base + 2u * G);
-    if (tr && tid == 0) tr[7] = gtimer();
     return rank;
 }
 
 // ---------------------------------------------------------------- the kernel
 template <bool MERGED>
 __global__ void __launch_bounds__(F_THREADS, 1)
-k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base)
+k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uint32_t epoch)
 {
     extern __shared__ __align__(16) uint8_t smem[];
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
@@ -343,7 +343,7 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base)
         uint32_t rank = 0;
         if (MERGED) {
             // the prologue, in this kernel (single super-round per CTA)
-            rank = merged_prologue(T, W, L, cand ? sa : INVALID_SA, bar_base, tr);
+            rank = merged_prologue(T, W, L, cand ? sa : INVALID_SA, bar_base, epoch, tr);
         } else if (base == p_begin) {
             // Programmatic dependent launch: the prologue kernel's outputs (ranks,
             // per-SA prefixes, seq_prev) are complete and visible after this.
@@ -353,11 +353,16 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base)
         if (j < cnt_pk) {
             uint32_t info = 0, bin = NBINS - 1, q32 = 0;
             if (cand) {
-                const unsigned long long q =
-                    MERGED ? (unsigned long long)__ldcg(&T.seq_prev[sa]) + 1ull +
-                                 __ldcg(&W.hpfx[(size_t)sa * gridDim.x + blockIdx.x]) + rank
-                           : (unsigned long long)T.seq_prev[sa] + 1ull +
-                                 W.hpfx[(size_t)sa * ((B.n + PTILE - 1) / PTILE) + i / PTILE] + W.lrank[i];
+                unsigned long long q;
+                if (MERGED) {
+                    const unsigned long long *pb = &W.hbase[(size_t)sa * gridDim.x + blockIdx.x];
+                    unsigned long long v = ld_relaxed_u64(pb);
+                    while ((uint32_t)(v >> 33) != epoch) v = ld_relaxed_u64(pb);
+                    q = (v & ((1ull << 33) - 1ull)) + 1ull + rank;
+                } else {
+                    q = (unsigned long long)T.seq_prev[sa] + 1ull +
+                        W.hpfx[(size_t)sa * ((B.n + PTILE - 1) / PTILE) + i / PTILE] + W.lrank[i];
+                }
                 if (q <= 0xffffffffull) {   // RFC 4303 §3.3.3: never cycle
                     q32 = (uint32_t)q;
                     info = D | (tos << 16) | INFO_OK | (MERGED ? INFO_TOSLOAD : 0u);
@@ -453,7 +458,7 @@ bool fused_merged_ok(uint32_t n, int grid)
 }
 
 cudaError_t launch_fused(const DevTable &T, const DevWork &W, const BatchArgs &B, int grid,
-                         bool merged, uint32_t *bar_base, cudaStream_t st)
+                         bool merged, uint32_t *bar_base, uint32_t *epoch, cudaStream_t st)
 {
     uint32_t ppc = fused_ppc(B.n, grid);
     uint32_t g = (B.n + ppc - 1) / ppc;
@@ -475,9 +480,14 @@ cudaError_t launch_fused(const DevTable &T, const DevWork &W, const BatchArgs &B
     cfg.attrs = attr;
     cfg.numAttrs = 1;
     const uint32_t bb = *bar_base;
-    cudaError_t e = merged ? cudaLaunchKernelEx(&cfg, k_fused<true>, T, W, B, ppc, bb)
-                           : cudaLaunchKernelEx(&cfg, k_fused<false>, T, W, B, ppc, bb);
-    if (e == cudaSuccess && merged) *bar_base = bb + 2u * g;
+    // epoch: 31-bit batch tag of the in-kernel prologue's published bases (never 0)
+    const uint32_t ep = merged ? ((*epoch % 0x7fffffffu) + 1u) : 0u;
+    cudaError_t e = merged ? cudaLaunchKernelEx(&cfg, k_fused<true>, T, W, B, ppc, bb, ep)
+                           : cudaLaunchKernelEx(&cfg, k_fused<false>, T, W, B, ppc, bb, ep);
+    if (e == cudaSuccess && merged) {
+        *bar_base = bb + g;
+        *epoch = ep;
+    }
     return e;
 }
 
