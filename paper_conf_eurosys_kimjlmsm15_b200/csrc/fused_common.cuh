@@ -4,6 +4,9 @@
 // RFC 3686 counter-block precompute and 4-block AES-128 step, and the
 // destination-aligned output stream.
 #pragma once
+#ifndef NBA_STAGE_SERIAL
+#define NBA_STAGE_SERIAL 0
+#endif
 #include "aes_round.cuh"
 #include "sha1.cuh"
 
@@ -286,6 +289,7 @@ __device__ __forceinline__ void aes4_keystream(uint32_t lane4r, const CtrPre &c,
 __device__ __forceinline__ void stage_round_keys(const uint4 *rk, FusedLo &L, FusedHi &H,
                                                  uint32_t sa_me, uint32_t warp, uint32_t lane)
 {
+#if NBA_STAGE_SERIAL
 #pragma unroll
     for (int k = 0; k < 8; k++) {
         const uint32_t m = 32u * k + lane, owner = m >> 3, r = m & 7u;
@@ -295,6 +299,26 @@ __device__ __forceinline__ void stage_round_keys(const uint4 *rk, FusedLo &L, Fu
             const uint32_t slot = (warp << 5) + owner;
             if (r < 4) L.rkA[r][slot] = v;
             else H.rkB[r - 4][slot] = v;
+        }
+    }
+    return;
+#endif
+    // all eight loads in flight before the first store
+    uint4 v[8];
+    uint32_t sv[8];
+#pragma unroll
+    for (int k = 0; k < 8; k++) {
+        const uint32_t m = 32u * k + lane, owner = m >> 3, r = m & 7u;
+        sv[k] = __shfl_sync(0xffffffffu, sa_me, owner);
+        v[k] = sv[k] != INVALID_SA ? __ldg(&rk[(size_t)sv[k] * 11u + 3u + r]) : make_uint4(0, 0, 0, 0);
+    }
+#pragma unroll
+    for (int k = 0; k < 8; k++) {
+        const uint32_t m = 32u * k + lane, owner = m >> 3, r = m & 7u;
+        if (sv[k] != INVALID_SA) {
+            const uint32_t slot = (warp << 5) + owner;
+            if (r < 4) L.rkA[r][slot] = v[k];
+            else H.rkB[r - 4][slot] = v[k];
         }
     }
 }

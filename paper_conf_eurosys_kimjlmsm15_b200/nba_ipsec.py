@@ -15,7 +15,8 @@ import re
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libnba_ipsec.so")
+# NBA_IPSEC_LIB: an A/B build variant of the same library (tools/ab_variants.py)
+LIB_PATH = os.environ.get("NBA_IPSEC_LIB") or os.path.join(_HERE, "libnba_ipsec.so")
 HEADER = os.path.join(os.path.dirname(_HERE), "include", "nba_ipsec.h")
 
 OK, EINVAL, ENOMEM, ENODEV, ECUDA = 0, -22, -12, -19, -1000
