@@ -31,9 +31,6 @@
 
 namespace nba {
 
-#ifndef NBA_HOUT_EARLY
-#define NBA_HOUT_EARLY 0
-#endif
 #ifndef NBA_PF_AHEAD          // payload prefetch distance in 64-byte steps
 #define NBA_PF_AHEAD 3
 #endif
@@ -103,9 +100,6 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
     // SHA-1 message words 0..3 = ESP header (big-endian words of the wire bytes)
     uint32_t carry[4] = {bswap32(hd.x), q32, 0u, q32};
     uint32_t st[5] = {h0.x, h0.y, h0.z, h0.w, h1.x};
-#if NBA_HOUT_EARLY
-    uint32_t ho[5] = {h1.y, h1.z, h1.w, 0u, 0u};   // outer midstate (last two words loaded later)
-#endif
     const uint8_t *src = B.in_buf + inoff;
     const uintptr_t src_end = reinterpret_cast<uintptr_t>(src) + D;
     ck_setup = clock64();
@@ -173,15 +167,7 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
                 const uint32_t msg = i < 4 ? carry[i] : bswap32(ct[i - 4]);
                 W[i] = m < Mw ? msg : (m == Mw ? 0x80000000u : 0u);
             }
-            if (it == nb_in - 1u) {
-                W[15] = bitlen;
-#if NBA_HOUT_EARLY
-                // the outer midstate's last words, in flight during this compression
-                const uint2 h2 = __ldg(reinterpret_cast<const uint2 *>(&T.hmid[(size_t)sa * 3 + 2]));
-                ho[3] = h2.x;
-                ho[4] = h2.y;
-#endif
-            }
+            if (it == nb_in - 1u) W[15] = bitlen;
 #pragma unroll
             for (int i = 0; i < 4; i++) carry[i] = bswap32(ct[12 + i]);
         } else {
@@ -191,14 +177,9 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
 #pragma unroll
             for (int i = 6; i < 15; i++) W[i] = 0u;
             W[15] = (64u + 20u) * 8u;
-#if NBA_HOUT_EARLY
-#pragma unroll
-            for (int i = 0; i < 5; i++) st[i] = ho[i];
-#else
             const uint4 g1 = __ldg(&T.hmid[(size_t)sa * 3 + 1]);
             const uint4 g2 = __ldg(&T.hmid[(size_t)sa * 3 + 2]);
             st[0] = g1.y; st[1] = g1.z; st[2] = g1.w; st[3] = g2.x; st[4] = g2.y;
-#endif
         }
         sha1_compress(st, W);
         if (it == 0) ck_sha = clock64();

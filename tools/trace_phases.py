@@ -45,4 +45,10 @@ for cfg in [int(x) for x in sys.argv[1:] if x.isdigit()] or (2, 3, 4):
     for k, nm in ((0, "tid0 (shortest)"), (8, "last (longest)")):
         v = [int(x) for x in raw[148*8+8+k:148*8+8+k+5]]
         print("  lane %s cycles: setup %d  aes0 %d  emit0 %d  sha0 %d  rest %d" % (nm, *v))
+    raw2 = np.zeros(148 * 8 + 64, np.uint64)
+    nbm.lib.nba_ipsec_debug_trace(t._h, raw2.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)), raw2.size)
+    G = int(live.sum()) if pro[0] == 0 else 148
+    wend = raw2[G * 8 + 32:G * 8 + 48].astype(np.int64)
+    st0 = int(full[0, 0])
+    print("  CTA 0 warp finish (us from its start):", " ".join(f"{(x - st0) / 1e3:.1f}" if x else "-" for x in wend))
     t.close()
