@@ -79,6 +79,15 @@ class InCounters(ctypes.Structure):
         return {k: int(getattr(self, k)) for k, _ in self._fields_}
 
 
+NO_SA = 0xFFFFFFFF
+
+
+class Flow(ctypes.Structure):
+    _fields_ = [("src", ctypes.c_uint32), ("dst", ctypes.c_uint32), ("sport", ctypes.c_uint16),
+                ("dport", ctypes.c_uint16), ("proto", ctypes.c_uint8), ("pad_", ctypes.c_uint8 * 3),
+                ("sa", ctypes.c_uint32)]
+
+
 def lib():
     global _lib
     with _lock:
@@ -112,6 +121,11 @@ def lib():
             L.oracle_process_inbound.argtypes = [P(SA), P(Replay), ctypes.c_uint32, u8p, u32p, u16p,
                                                  u32p, u8p, u32p, u16p, u8p, ctypes.c_uint32,
                                                  P(InCounters)]
+            L.oracle_flow_table_prepare.restype = ctypes.c_int
+            L.oracle_flow_table_prepare.argtypes = [P(Flow), ctypes.c_uint32]
+            L.oracle_flow_lookup.restype = None
+            L.oracle_flow_lookup.argtypes = [P(Flow), ctypes.c_uint32, u8p, u32p, u16p,
+                                             ctypes.c_uint32, u32p]
             L.oracle_init()
             _lib = L
     return _lib
@@ -283,3 +297,27 @@ def process_inbound(sas, win, n_sa: int, batch, out_pool_bytes: int | None = Non
                                  _ptr(out_len, ctypes.c_uint16), _ptr(status), n,
                                  ctypes.byref(ctr))
     return out_buf, out_len[:n], status[:n], ctr
+
+
+# --- flow -> SA lookup -------------------------------------
+
+def flow_lookup(flows, batch) -> np.ndarray:
+    """SA index per packet of ``batch`` from the exact-match 5-tuple table
+    ``flows`` (a gen.Flows); NO_SA where there is no key or no match."""
+    nf = len(flows.sa)
+    arr = (Flow * max(nf, 1))()
+    for k in range(nf):
+        f = arr[k]
+        f.src, f.dst = int(flows.src[k]), int(flows.dst[k])
+        f.sport, f.dport, f.proto = int(flows.sport[k]), int(flows.dport[k]), int(flows.proto[k])
+        f.sa = int(flows.sa[k])
+    if lib().oracle_flow_table_prepare(arr, nf) != 0:
+        raise ValueError("duplicate flow keys")
+    n = int(batch.n)
+    in_buf = np.ascontiguousarray(batch.in_buf, np.uint8)
+    in_off = np.ascontiguousarray(batch.in_off, np.uint32)
+    in_len = np.ascontiguousarray(batch.in_len, np.uint16)
+    out = np.zeros(max(n, 1), np.uint32)
+    lib().oracle_flow_lookup(arr, nf, _ptr(in_buf), _ptr(in_off, ctypes.c_uint32),
+                             _ptr(in_len, ctypes.c_uint16), n, _ptr(out, ctypes.c_uint32))
+    return out[:n]

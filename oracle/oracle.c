@@ -615,3 +615,64 @@ void oracle_process_inbound(const oracle_sa *sas, oracle_replay *win, uint32_t n
     }
     if (n) ctr->batches++;
 }
+
+/* ------------------------------------------------------------------------ */
+/* Flow -> SA lookup.  PAPER.md:395 keeps one crypto      */
+/* context per flow, initialised at startup; the lookup is an exact match   */
+/* on the inner IPv4 5-tuple (readings F1..F4 in DESIGN.md): plain parsing  */
+/* of the header and a binary search over the sorted flow list.             */
+/* ------------------------------------------------------------------------ */
+static int flow_cmp(const oracle_flow *a, const oracle_flow *b)
+{
+    if (a->src != b->src) return a->src < b->src ? -1 : 1;
+    if (a->dst != b->dst) return a->dst < b->dst ? -1 : 1;
+    if (a->proto != b->proto) return a->proto < b->proto ? -1 : 1;
+    if (a->sport != b->sport) return a->sport < b->sport ? -1 : 1;
+    if (a->dport != b->dport) return a->dport < b->dport ? -1 : 1;
+    return 0;
+}
+
+static int flow_qsort_cmp(const void *a, const void *b)
+{
+    return flow_cmp((const oracle_flow *)a, (const oracle_flow *)b);
+}
+
+int oracle_flow_table_prepare(oracle_flow *flows, uint32_t n_flows)
+{
+    qsort(flows, n_flows, sizeof(oracle_flow), flow_qsort_cmp);
+    for (uint32_t k = 1; k < n_flows; k++)
+        if (flow_cmp(&flows[k - 1], &flows[k]) == 0) return -1;
+    return 0;
+}
+
+/* F1/F2: the key of one inner datagram; returns 0 if it has none. */
+static int flow_key(const uint8_t *P, uint32_t D, oracle_flow *k)
+{
+    if (D < 20) return 0;
+    uint32_t ihl = P[0] & 0x0fu;
+    if ((P[0] >> 4) != 4 || ihl < 5 || D < 4u * ihl) return 0;
+    memset(k, 0, sizeof(*k));
+    k->src = be32_at(P + 12);
+    k->dst = be32_at(P + 16);
+    k->proto = P[9];
+    uint32_t frag_off = (((uint32_t)P[6] << 8) | P[7]) & 0x1fffu;
+    if ((k->proto == 6 || k->proto == 17) && frag_off == 0 && D >= 4u * ihl + 4u) {
+        k->sport = (uint16_t)(((uint32_t)P[4 * ihl] << 8) | P[4 * ihl + 1]);
+        k->dport = (uint16_t)(((uint32_t)P[4 * ihl + 2] << 8) | P[4 * ihl + 3]);
+    }
+    return 1;
+}
+
+void oracle_flow_lookup(const oracle_flow *sorted_flows, uint32_t n_flows,
+                        const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
+                        uint32_t n, uint32_t *sa_idx)
+{
+    for (uint32_t i = 0; i < n; i++) {
+        oracle_flow k;
+        sa_idx[i] = ORACLE_NO_SA;
+        if (!flow_key(in_buf + in_off[i], in_len[i], &k)) continue;
+        const oracle_flow *hit = (const oracle_flow *)bsearch(&k, sorted_flows, n_flows,
+                                                              sizeof(oracle_flow), flow_qsort_cmp);
+        if (hit) sa_idx[i] = hit->sa;
+    }
+}

@@ -73,4 +73,21 @@ void     oracle_process_inbound(const oracle_sa *sas, oracle_replay *win, uint32
                                 const uint16_t *in_len, const uint32_t *sa_idx, uint8_t *out_buf,
                                 const uint32_t *out_off, uint16_t *out_len, uint8_t *status,
                                 uint32_t n, oracle_in_counters *ctr);
+
+/* ---- flow -> SA lookup (readings F1..F4) -------- */
+#define ORACLE_NO_SA 0xffffffffu
+typedef struct {
+    uint32_t src, dst;        /* IPv4 addresses, host order */
+    uint16_t sport, dport;    /* 0 when the protocol has no ports (F2) */
+    uint8_t  proto;
+    uint8_t  pad_[3];
+    uint32_t sa;              /* SA index of the flow */
+} oracle_flow;
+
+/* Sorts `flows` in place (the lookup is a binary search); returns -1 if two
+ * flows have the same key. */
+int      oracle_flow_table_prepare(oracle_flow *flows, uint32_t n_flows);
+void     oracle_flow_lookup(const oracle_flow *sorted_flows, uint32_t n_flows,
+                            const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
+                            uint32_t n, uint32_t *sa_idx);
 #endif

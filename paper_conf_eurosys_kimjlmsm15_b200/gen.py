@@ -263,3 +263,68 @@ def esp_batch(src_buf: np.ndarray, src_off: np.ndarray, src_len: np.ndarray,
                  sa_idx=np.asarray(src_sa, np.int64)[order].astype(np.uint32),
                  out_off=out_off.astype(np.uint32), out_pool_bytes=int(out_pool),
                  frame_len=(L + ETH).astype(np.uint32))
+
+
+# --- flows (flow -> SA lookup) -------------------------------
+
+@dataclasses.dataclass
+class Flows:
+    """Exact-match 5-tuple -> SA table (host order; ports 0 for portless protocols)."""
+    src: np.ndarray     # u32[n]
+    dst: np.ndarray     # u32[n]
+    sport: np.ndarray   # u16[n]
+    dport: np.ndarray   # u16[n]
+    proto: np.ndarray   # u8[n]
+    sa: np.ndarray      # u32[n]
+
+
+def make_flows(n_flows: int, n_sa: int, cfg_id: int = 0, rank: int = 0) -> Flows:
+    """n_flows distinct UDP/TCP flows in 10.0.0.0/8, each bound to a random SA
+    (per-flow contexts initialised at startup)."""
+    r = rng_for(cfg_id, rank, 0, salt=21)
+    seen, rows = set(), []
+    while len(rows) < n_flows:
+        k = int(n_flows - len(rows))
+        src = (10 << 24) | r.integers(0, 1 << 24, k)
+        dst = (10 << 24) | r.integers(0, 1 << 24, k)
+        sp = r.integers(1024, 65536, k)
+        dp = r.integers(1, 65536, k)
+        pr = np.where(r.random(k) < 0.8, 17, 6)
+        for t in zip(src.tolist(), dst.tolist(), sp.tolist(), dp.tolist(), pr.tolist()):
+            if t not in seen:
+                seen.add(t)
+                rows.append(t)
+    a = np.array(rows[:n_flows], dtype=np.int64).reshape(-1, 5)
+    return Flows(src=a[:, 0].astype(np.uint32), dst=a[:, 1].astype(np.uint32),
+                 sport=a[:, 2].astype(np.uint16), dport=a[:, 3].astype(np.uint16),
+                 proto=a[:, 4].astype(np.uint8),
+                 sa=r.integers(0, max(n_sa, 1), n_flows).astype(np.uint32))
+
+
+def apply_flows(b: Batch, flows: Flows, cfg_id: int = 0, batch: int = 0, miss: float = 0.0) -> np.ndarray:
+    """Rewrite the inner IPv4 / TCP-UDP headers of every packet of ``b`` (slot
+    layout) to a random flow of ``flows``; a fraction ``miss`` gets an unknown
+    source address.  Keeps the IPv4 checksum valid.  Returns the flow index per
+    packet (-1 for a miss).  Input synthesis only: no lookup logic."""
+    r = rng_for(cfg_id, 0, batch, salt=22)
+    n = int(b.n)
+    fi = r.integers(0, len(flows.sa), n)
+    is_miss = r.random(n) < miss
+    for i in range(n):
+        D = int(b.in_len[i])
+        if D < 24:
+            continue
+        o = int(b.in_off[i])
+        k = int(fi[i])
+        P = b.in_buf[o:o + D]
+        src = int(flows.src[k]) if not is_miss[i] else (11 << 24) | int(r.integers(0, 1 << 24))
+        P[12:16] = np.frombuffer(src.to_bytes(4, "big"), np.uint8)
+        P[16:20] = np.frombuffer(int(flows.dst[k]).to_bytes(4, "big"), np.uint8)
+        P[9] = int(flows.proto[k])
+        P[20:22] = np.frombuffer(int(flows.sport[k]).to_bytes(2, "big"), np.uint8)
+        P[22:24] = np.frombuffer(int(flows.dport[k]).to_bytes(2, "big"), np.uint8)
+        P[10:12] = 0
+        words = (P[0:20:2].astype(np.uint32) << 8) | P[1:20:2]
+        cs = int(_csum16(words[None, :])[0])
+        P[10], P[11] = cs >> 8, cs & 0xFF
+    return np.where(is_miss, -1, fi)
