@@ -102,6 +102,8 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
 /* Enqueue the whole ESP outbound path for one batch on `cuda_stream`
  * (a cudaStream_t; NULL = legacy default stream) and return immediately.
  * Device pointers only.  n_pkts == 0 is a no-op returning NBA_IPSEC_OK.
+ * b->sa_idx may be NULL if a flow table is set (nba_ipsec_set_flow_table): the
+ * packets' SAs are then looked up on the GPU first.
  * Returns NBA_IPSEC_EINVAL for NULL t/b, n_pkts > max_batch_pkts or a NULL
  * array with n_pkts > 0; NBA_IPSEC_ECUDA if a launch fails. */
 int nba_ipsec_process_batch(nba_ipsec_sa_table *t, const nba_ipsec_batch *b, void *cuda_stream);
@@ -179,6 +181,41 @@ int nba_ipsec_debug_trace(nba_ipsec_sa_table *t, uint64_t *host, uint32_t n_word
  * (RFC 2104 §2; FIPS 180-4 §6.1.2). */
 void nba_ipsec_host_aes128_key_schedule(const uint8_t key[16], uint32_t w[44]);
 void nba_ipsec_host_hmac_sha1_midstates(const uint8_t key[20], uint32_t hin[5], uint32_t hout[5]);
+
+/* ---- flow -> SA lookup on the GPU --------------------------
+ *
+ * crypto contexts exist per flow and are set up at startup.  The
+ * caller registers its flows -- exact inner IPv4 5-tuples -- and the SA each
+ * one uses; the lookup then finds every packet's SA on the GPU (readings
+ * F1..F4):
+ *   key of the inner datagram P (D = in_len bytes): none unless P is IPv4 with
+ *   20 <= 4*IHL <= D; else (src, dst, protocol, sport, dport), the ports being
+ *   the 4 bytes after the IPv4 header for TCP (6) / UDP (17) when the fragment
+ *   offset is 0 and D >= 4*IHL + 4, and 0 otherwise;
+ *   sa_idx[i] = SA of the flow with that key, or NBA_IPSEC_NO_SA (no key / no
+ *   match; the path drops such a packet like any sa_idx >= n_sa). */
+#define NBA_IPSEC_NO_SA 0xffffffffu
+
+typedef struct {
+    uint32_t src, dst;       /* host order */
+    uint16_t sport, dport;   /* 0 for portless protocols / non-first fragments */
+    uint8_t  proto;
+    uint8_t  pad_[3];
+    uint32_t sa;             /* SA index, < n_sa */
+} nba_ipsec_flow;
+
+/* Build (replace) the device flow table from `flows` (copied; synchronous).
+ * NBA_IPSEC_EINVAL for NULL flows with n_flows > 0, an sa >= n_sa, duplicate
+ * keys, or n_flows > 2^26; NBA_IPSEC_ENOMEM if allocation fails.  n_flows = 0
+ * removes the table. */
+int nba_ipsec_set_flow_table(nba_ipsec_sa_table *t, const nba_ipsec_flow *flows, uint32_t n_flows);
+/* Enqueue the lookup for n packets (DEVICE pointers) on `cuda_stream`:
+ * sa_idx[i] <- the packet's SA or NBA_IPSEC_NO_SA.  NBA_IPSEC_EINVAL if no flow
+ * table is set or n > max_batch_pkts.  nba_ipsec_process_batch also accepts
+ * b->sa_idx == NULL when a flow table is set: it then runs this lookup first. */
+int nba_ipsec_lookup_sa(nba_ipsec_sa_table *t, const uint8_t *in_buf, const uint32_t *in_off,
+                        const uint16_t *in_len, uint32_t n_pkts, uint32_t *sa_idx,
+                        void *cuda_stream);
 
 /* ---- ESP inbound: the mirror of the path ------------------
  *

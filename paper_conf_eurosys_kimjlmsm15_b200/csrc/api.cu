@@ -79,6 +79,10 @@ struct nba_ipsec_sa_table {
     unsigned long long *in_bmp0 = nullptr;
     double prof_in_ms[3] = {};
     uint32_t prof_in_batches = 0;
+    // flow -> SA lookup (nba_ipsec_set_flow_table)
+    uint4 *flow_table = nullptr;
+    uint32_t flow_mask = 0;
+    uint32_t *flow_sa = nullptr;   // [max_batch] SA indices looked up for process_batch
 };
 
 namespace {
@@ -331,13 +335,21 @@ int nba_ipsec_process_batch(nba_ipsec_sa_table *t, const nba_ipsec_batch *b, voi
     if (!t || !b) return NBA_IPSEC_EINVAL;
     if (b->n_pkts > t->max_batch) return NBA_IPSEC_EINVAL;
     if (b->n_pkts == 0) return NBA_IPSEC_OK;
-    if (!b->in_buf || !b->in_off || !b->in_len || !b->sa_idx || !b->out_buf || !b->out_off ||
-        !b->out_len)
+    if (!b->in_buf || !b->in_off || !b->in_len || !b->out_buf || !b->out_off || !b->out_len)
         return NBA_IPSEC_EINVAL;
+    if (!b->sa_idx && !t->flow_table) return NBA_IPSEC_EINVAL;
     DeviceGuard g(t->device);
-    BatchArgs B{b->in_buf, b->in_off, b->in_len, b->sa_idx, b->out_buf, b->out_off, b->out_len,
+    cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    const uint32_t *sa_idx = b->sa_idx;
+    if (!sa_idx) {   // the SAs come from the flow table
+        FlowArgs A{b->in_buf, b->in_off, b->in_len, t->flow_sa, b->n_pkts};
+        if (launch_flow_lookup(t->flow_table, t->flow_mask, A, st) != cudaSuccess)
+            return NBA_IPSEC_ECUDA;
+        sa_idx = t->flow_sa;
+    }
+    BatchArgs B{b->in_buf, b->in_off, b->in_len, sa_idx, b->out_buf, b->out_off, b->out_len,
                 b->n_pkts};
-    return enqueue(t, B, static_cast<cudaStream_t>(cuda_stream));
+    return enqueue(t, B, st);
 }
 
 static void io_free(nba_ipsec_sa_table *t)
@@ -472,6 +484,8 @@ int nba_ipsec_destroy(nba_ipsec_sa_table *t)
         cudaDeviceSynchronize();
         free_all(t);
         io_free(t);
+        if (t->flow_table) cudaFree(t->flow_table);
+        if (t->flow_sa) cudaFree(t->flow_sa);
         for (auto &sl : t->io) {
             if (sl.in_ready) cudaEventDestroy(sl.in_ready);
             if (sl.done) cudaEventDestroy(sl.done);
@@ -574,6 +588,73 @@ int nba_ipsec_profile_read(nba_ipsec_sa_table *t, double *ms, const char **names
 }
 
 // ---- ESP inbound -----------------------------------------
+
+// ---- flow -> SA lookup ----------------------------------
+
+int nba_ipsec_set_flow_table(nba_ipsec_sa_table *t, const nba_ipsec_flow *flows, uint32_t n_flows)
+{
+    if (!t || (!flows && n_flows) || n_flows > (1u << 26)) return NBA_IPSEC_EINVAL;
+    DeviceGuard g(t->device);
+    if (n_flows == 0) {
+        cudaDeviceSynchronize();
+        if (t->flow_table) cudaFree(t->flow_table);
+        t->flow_table = nullptr;
+        t->flow_mask = 0;
+        return NBA_IPSEC_OK;
+    }
+    uint32_t cap = 64;
+    while (cap < 2ull * n_flows) cap <<= 1;
+    std::vector<uint4> tab(cap, make_uint4(0, 0, 0, 0));
+    for (uint32_t k = 0; k < n_flows; k++) {
+        const nba_ipsec_flow &f = flows[k];
+        if (f.sa >= t->n_sa) return NBA_IPSEC_EINVAL;
+        const uint32_t ports = ((uint32_t)f.sport << 16) | f.dport;
+        uint32_t h = flow_hash(f.src, f.dst, ports, f.proto) & (cap - 1u);
+        while (tab[h].w & FLOW_VALID) {
+            if (tab[h].x == f.src && tab[h].y == f.dst && tab[h].z == ports &&
+                (tab[h].w & 0xffu) == f.proto)
+                return NBA_IPSEC_EINVAL;   // duplicate key
+            h = (h + 1u) & (cap - 1u);
+        }
+        tab[h] = make_uint4(f.src, f.dst, ports, (uint32_t)f.proto | FLOW_VALID | (f.sa << 16));
+    }
+    cudaError_t e = cudaSuccess;
+    if (!t->flow_sa) {
+        e = cudaMalloc(&t->flow_sa, (size_t)t->max_batch * 4 + 64);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            t->flow_sa = nullptr;
+            return NBA_IPSEC_ENOMEM;
+        }
+    }
+    cudaDeviceSynchronize();   // the old table may be in use by enqueued work
+    if (t->flow_table) cudaFree(t->flow_table);
+    t->flow_table = nullptr;
+    if (cudaMalloc(&t->flow_table, cap * sizeof(uint4)) != cudaSuccess) {
+        cudaGetLastError();
+        return NBA_IPSEC_ENOMEM;
+    }
+    if (cudaMemcpy(t->flow_table, tab.data(), cap * sizeof(uint4), cudaMemcpyHostToDevice) !=
+        cudaSuccess)
+        return NBA_IPSEC_ECUDA;
+    t->flow_mask = cap - 1u;
+    return NBA_IPSEC_OK;
+}
+
+int nba_ipsec_lookup_sa(nba_ipsec_sa_table *t, const uint8_t *in_buf, const uint32_t *in_off,
+                        const uint16_t *in_len, uint32_t n_pkts, uint32_t *sa_idx,
+                        void *cuda_stream)
+{
+    if (!t || !t->flow_table || n_pkts > t->max_batch) return NBA_IPSEC_EINVAL;
+    if (n_pkts == 0) return NBA_IPSEC_OK;
+    if (!in_buf || !in_off || !in_len || !sa_idx) return NBA_IPSEC_EINVAL;
+    DeviceGuard g(t->device);
+    FlowArgs A{in_buf, in_off, in_len, sa_idx, n_pkts};
+    return launch_flow_lookup(t->flow_table, t->flow_mask, A, static_cast<cudaStream_t>(cuda_stream)) ==
+                   cudaSuccess
+               ? NBA_IPSEC_OK
+               : NBA_IPSEC_ECUDA;
+}
 
 int nba_ipsec_enable_inbound(nba_ipsec_sa_table *t)
 {

@@ -113,6 +113,35 @@ struct InBatchArgs {
     uint32_t n;
 };
 
+// --- flow -> SA lookup (readings F1..F4) ---------
+// Open-addressing table, linear probing, capacity a power of two >= 2 x flows.
+// Entry = {src, dst, sport << 16 | dport, proto | FLOW_VALID | sa << 16}.
+constexpr uint32_t FLOW_VALID = 0x100u;
+#if defined(__CUDACC__)
+#define NBA_HD __host__ __device__
+#else
+#define NBA_HD
+#endif
+NBA_HD inline uint32_t flow_hash(uint32_t src, uint32_t dst, uint32_t ports, uint32_t proto)
+{
+    // murmur3-style finaliser over the folded key (host build and device probe)
+    uint32_t h = src * 0x9E3779B1u;
+    h ^= (dst << 13) | (dst >> 19);
+    h = h * 0x85EBCA6Bu ^ ports;
+    h = (h ^ (h >> 16)) * 0x7FEB352Du;
+    h ^= proto * 0xC2B2AE35u;
+    h = (h ^ (h >> 15)) * 0x846CA68Bu;
+    return h ^ (h >> 16);
+}
+
+struct FlowArgs {
+    const uint8_t *in_buf;
+    const uint32_t *in_off;
+    const uint16_t *in_len;
+    uint32_t *sa_idx;
+    uint32_t n;
+};
+
 #ifdef __CUDACC__
 // --- launchers (one per kernel file) ----------------------------------------
 cudaError_t launch_prologue(const DevTable &T, const DevWork &W, const BatchArgs &B,
@@ -140,6 +169,7 @@ cudaError_t launch_in_replay(const DevTable &T, const InState &S, const InBatchA
 cudaError_t launch_in_decide(const DevTable &T, const InState &S, const InBatchArgs &B,
                              uint32_t n_tiles, uint32_t hmask, cudaStream_t st);
 cudaError_t setup_inbound_attributes(uint32_t n_sa, uint32_t max_tiles, int num_sms, bool *gridsync);
+cudaError_t launch_flow_lookup(const uint4 *table, uint32_t mask, const FlowArgs &A, cudaStream_t st);
 
 // --- small device helpers ---------------------------------------------------
 __device__ __forceinline__ uint32_t bswap32(uint32_t x) { return __byte_perm(x, 0, 0x0123); }

@@ -55,6 +55,15 @@ class Counters(ctypes.Structure):
         return {k: int(getattr(self, k)) for k, _ in self._fields_}
 
 
+NO_SA = 0xFFFFFFFF
+
+
+class Flow(ctypes.Structure):
+    _fields_ = [("src", ctypes.c_uint32), ("dst", ctypes.c_uint32), ("sport", ctypes.c_uint16),
+                ("dport", ctypes.c_uint16), ("proto", ctypes.c_uint8), ("pad_", ctypes.c_uint8 * 3),
+                ("sa", ctypes.c_uint32)]
+
+
 class InBatch(ctypes.Structure):
     _fields_ = [("in_buf", ctypes.c_void_p), ("in_off", ctypes.c_void_p),
                 ("in_len", ctypes.c_void_p), ("sa_idx", ctypes.c_void_p),
@@ -98,6 +107,8 @@ def _load():
                                          P(i32), P(u32)]),
         "nba_ipsec_debug_trace": (i32, [vp, P(u64), u32]),
         "nba_ipsec_enable_inbound": (i32, [vp]),
+        "nba_ipsec_set_flow_table": (i32, [vp, P(Flow), u32]),
+        "nba_ipsec_lookup_sa": (i32, [vp, vp, vp, vp, u32, vp, vp]),
         "nba_ipsec_process_inbound": (i32, [vp, P(InBatch), vp]),
         "nba_ipsec_read_in_counters": (i32, [vp, P(InCounters), vp]),
         "nba_ipsec_reset_inbound": (i32, [vp, vp]),
@@ -237,6 +248,23 @@ class SATable:
         _check(lib.nba_ipsec_profile_read(self._h, ms, names, 8, ctypes.byref(nk),
                                           ctypes.byref(nb)), "nba_ipsec_profile_read")
         return {names[k].decode(): ms[k] for k in range(nk.value)}, int(nb.value)
+
+    # -- flow -> SA lookup ------------------------------------
+    def set_flow_table(self, flows):
+        """nba_ipsec_set_flow_table from a gen.Flows (numpy SoA)."""
+        n = len(flows.sa)
+        arr = (Flow * max(n, 1))()
+        for k in range(n):
+            f = arr[k]
+            f.src, f.dst = int(flows.src[k]), int(flows.dst[k])
+            f.sport, f.dport, f.proto = int(flows.sport[k]), int(flows.dport[k]), int(flows.proto[k])
+            f.sa = int(flows.sa[k])
+        _check(lib.nba_ipsec_set_flow_table(self._h, arr, n), "nba_ipsec_set_flow_table")
+
+    def lookup_sa(self, in_buf, in_off, in_len, sa_idx, n=None, stream=None):
+        n = int(in_len.numel() if n is None else n)
+        _check(lib.nba_ipsec_lookup_sa(self._h, _ptr(in_buf), _ptr(in_off), _ptr(in_len), n,
+                                       _ptr(sa_idx), _stream_handle(stream)), "nba_ipsec_lookup_sa")
 
     # -- ESP inbound (SURVEY §8(f) f2) ------------------------------------------
     def enable_inbound(self):

@@ -48,7 +48,7 @@ def _py_key(P):
 
 
 def _flows(rows):
-    a = np.array(rows, np.int64).reshape(-1, 6)
+    a = np.array(rows, np.int64).reshape(-1, 6) if rows else np.zeros((0, 6), np.int64)
     return gen.Flows(src=a[:, 0].astype(np.uint32), dst=a[:, 1].astype(np.uint32),
                      sport=a[:, 2].astype(np.uint16), dport=a[:, 3].astype(np.uint16),
                      proto=a[:, 4].astype(np.uint8), sa=a[:, 5].astype(np.uint32))
