@@ -349,6 +349,52 @@ def run_ours(args):
                 "all_accepted": bool(ok_all), "lengths_match_outbound_input": same,
                 "gpu_launches": 3 * steps}
 
+    def measure_flows(cfg_id, steps, warmup, n_flows=65536):
+        """Flow -> SA lookup on the config's traffic rewritten to
+        n_flows registered 5-tuples (5% unknown): the lookup kernel alone, and
+        the whole path taking its SAs from the flow table (sa_idx = NULL)."""
+        size = CFG_SIZE[cfg_id]
+        p, b = shard.rank_workload(cfg_id, PKTS_PER_GPU, size, N_SA_TOTAL, rank, world)
+        f = gen.make_flows(n_flows, len(p.spi), cfg_id=cfg_id, rank=rank)
+        gen.apply_flows(b, f, cfg_id=cfg_id, miss=0.05)
+        t = nba_ipsec.SATable(p, device=local, max_batch=PKTS_PER_GPU)
+        t.set_flow_table(f)
+        db = device.to_device(b, dev)
+        sa_out = torch.empty(b.n, dtype=torch.int32, device=dev)
+        look = lambda: t.lookup_sa(db.in_buf, db.in_off, db.in_len, sa_out, n=b.n)  # noqa: E731
+        path = lambda: t.process(db.in_buf, db.in_off, db.in_len, None, db.out_buf, db.out_off,  # noqa: E731
+                                 db.out_len, n=b.n)
+        out = {}
+        for name, fn in (("lookup", look), ("path_with_lookup", path)):
+            for _ in range(warmup):
+                flush.zero_()
+                fn()
+            torch.cuda.synchronize()
+            barrier()
+            ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                  for _ in range(steps)]
+            for k in range(steps):
+                flush.zero_()
+                ev[k][0].record()
+                fn()
+                ev[k][1].record()
+            torch.cuda.synchronize()
+            ms = shard.max_over_ranks(sum(a.elapsed_time(c) for a, c in ev) / steps, device=dev)
+            red = shard.reduce_counters({"pkts_ok": frame_bits(b) / 8.0, "pkts_dropped": 0,
+                                         "bytes_in": b.n, "bytes_out": 0, "batches": 0}, device=dev)
+            out[name] = {"ms_per_step": ms, "mpps": red["bytes_in"] / (ms * 1e-3) / 1e6,
+                         "gbps": 8.0 * red["pkts_ok"] / (ms * 1e-3) / 1e9}
+        # lookup roofline: HBM bytes of the headers read + SA indices written
+        # (table probes are L2 hits: 65,536 flows x 16 B x 2 = 2 MiB)
+        byts = b.n * (32 + 4 + 4 + 2)
+        out["lookup"]["roofline"] = {"bound": "hbm", "unit": "GB/s", "peak": peaks["hbm_gbs"],
+                                     "achieved": byts / (out["lookup"]["ms_per_step"] * 1e-3) / 1e9}
+        out["lookup"]["roofline"]["frac"] = out["lookup"]["roofline"]["achieved"] / peaks["hbm_gbs"]
+        out["n_flows"] = n_flows
+        out["miss_fraction"] = 0.05
+        t.close()
+        return out
+
     main_cfg = args.config
     res = measure(main_cfg, args.steps, args.warmup)
     agg = aggregate(res, args.steps)
@@ -403,6 +449,12 @@ def run_ours(args):
             inbound[str(CFG_SIZE[cfg_id])] = measure_inbound(cfg_id, max(10, args.steps // 4),
                                                             max(3, args.warmup // 2))
 
+    # ---- flow -> SA lookup -----------------------------------------
+    flows = None
+    if not args.no_inbound:
+        flows = {str(CFG_SIZE[main_cfg]): measure_flows(main_cfg, max(10, args.steps // 4),
+                                                        max(3, args.warmup // 2))}
+
     # ---- CPU baseline: the oracle on host cores (rank 0, N = 1 only) ----------
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
@@ -439,6 +491,7 @@ def run_ours(args):
             "work_per_step_per_gpu": w,
             "per_size": per_size,
             "inbound": inbound or None,
+            "flow_lookup": flows,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": res["launches"],

@@ -341,14 +341,17 @@ int nba_ipsec_process_batch(nba_ipsec_sa_table *t, const nba_ipsec_batch *b, voi
     DeviceGuard g(t->device);
     cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
     const uint32_t *sa_idx = b->sa_idx;
-    if (!sa_idx) {   // the SAs come from the flow table
+    const bool merged = t->pipeline == NBA_IPSEC_PIPE_FUSED && t->allow_merged &&
+                        fused_merged_ok(b->n_pkts, t->grid_fused);
+    if (!sa_idx && !merged) {   // the SAs come from the flow table
         FlowArgs A{b->in_buf, b->in_off, b->in_len, t->flow_sa, b->n_pkts};
         if (launch_flow_lookup(t->flow_table, t->flow_mask, A, st) != cudaSuccess)
             return NBA_IPSEC_ECUDA;
         sa_idx = t->flow_sa;
     }
+    // (the one-kernel path looks the SAs up itself, in its prologue)
     BatchArgs B{b->in_buf, b->in_off, b->in_len, sa_idx, b->out_buf, b->out_off, b->out_len,
-                b->n_pkts};
+                b->n_pkts, t->flow_table, t->flow_mask};
     return enqueue(t, B, st);
 }
 

@@ -391,4 +391,38 @@ __device__ __forceinline__ void extract16(const Raw5 &r, uint32_t (&o)[16])
 #undef NBA_PT_CASE
 }
 
+// Flow -> SA lookup of one inner datagram P (D bytes), readings F1..F4: one
+// unaligned 24-byte header load (two with IP options), then linear probing in
+// the L2-resident open-addressing table.  INVALID_SA: no key or no match.
+__device__ __forceinline__ uint32_t flow_lookup_one(const uint4 *__restrict__ table, uint32_t mask,
+                                                    const uint8_t *P, uint32_t D)
+{
+    if (D < 20u) return INVALID_SA;
+    const uintptr_t pa = reinterpret_cast<uintptr_t>(P);
+    uint32_t w[6];
+    load_words<6>(pa, pa + D, w);
+    const uint32_t vihl = w[0] & 0xffu, ihl = vihl & 15u;
+    if ((vihl >> 4) != 4u || ihl < 5u || D < 4u * ihl) return INVALID_SA;
+    const uint32_t src = bswap32(w[3]), dst = bswap32(w[4]);
+    const uint32_t proto = (w[2] >> 8) & 0xffu;
+    const uint32_t frag = ((w[1] >> 8) & 0x1f00u) | (w[1] >> 24);   // bytes 6..7, 13 bits
+    uint32_t ports = 0;
+    if ((proto == 6u || proto == 17u) && frag == 0u && D >= 4u * ihl + 4u) {
+        if (ihl == 5u) {
+            ports = bswap32(w[5]);
+        } else {
+            uint32_t x[1];
+            load_words<1>(pa + 4u * ihl, pa + D, x);
+            ports = bswap32(x[0]);
+        }
+    }
+    uint32_t h = flow_hash(src, dst, ports, proto) & mask;
+    while (true) {
+        const uint4 e = __ldg(&table[h]);
+        if (!(e.w & FLOW_VALID)) return INVALID_SA;
+        if (e.x == src && e.y == dst && e.z == ports && (e.w & 0xffu) == proto) return e.w >> 16;
+        h = (h + 1u) & mask;
+    }
+}
+
 }  // namespace nba

@@ -68,11 +68,13 @@ struct BatchArgs {
     const uint8_t *in_buf;
     const uint32_t *in_off;
     const uint16_t *in_len;
-    const uint32_t *sa_idx;
+    const uint32_t *sa_idx;       // null: the fused kernel looks the SAs up (flow table)
     uint8_t *out_buf;
     const uint32_t *out_off;
     uint16_t *out_len;
     uint32_t n;
+    const uint4 *flow_table = nullptr;
+    uint32_t flow_mask = 0;
 };
 
 // --- ESP inbound (readings B1..B9) ---------------

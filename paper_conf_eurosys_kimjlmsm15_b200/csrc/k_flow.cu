@@ -10,8 +10,8 @@
 // 4 bytes are there, else 0.  sa_idx[i] = the matching flow's SA, or
 // 0xffffffff (no key / no match: the path then drops the packet).
 //
-// One thread per packet: one unaligned 24-byte header load (two if the header
-// has options), then linear probing in the L2-resident table (16 B entries).
+// One thread per packet (flow_lookup_one, fused_common.cuh; the fused kernel
+// runs the same function in its prologue when the caller passes no sa_idx).
 #include "fused_common.cuh"
 
 namespace nba {
@@ -21,41 +21,7 @@ k_flow_lookup(const uint4 *__restrict__ table, uint32_t mask, FlowArgs A)
 {
     const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= A.n) return;
-    uint32_t sa = INVALID_SA;
-    const uint32_t D = A.in_len[i];
-    if (D >= 20u) {
-        const uint8_t *P = A.in_buf + A.in_off[i];
-        const uintptr_t pa = reinterpret_cast<uintptr_t>(P);
-        uint32_t w[6];
-        load_words<6>(pa, pa + D, w);
-        const uint32_t vihl = w[0] & 0xffu, ihl = vihl & 15u;
-        if ((vihl >> 4) == 4u && ihl >= 5u && D >= 4u * ihl) {
-            const uint32_t src = bswap32(w[3]), dst = bswap32(w[4]);
-            const uint32_t proto = (w[2] >> 8) & 0xffu;
-            const uint32_t frag = ((w[1] >> 8) & 0x1f00u) | (w[1] >> 24);   // bytes 6..7, 13 bits
-            uint32_t ports = 0;
-            if ((proto == 6u || proto == 17u) && frag == 0u && D >= 4u * ihl + 4u) {
-                if (ihl == 5u) {
-                    ports = bswap32(w[5]);
-                } else {
-                    uint32_t x[1];
-                    load_words<1>(pa + 4u * ihl, pa + D, x);
-                    ports = bswap32(x[0]);
-                }
-            }
-            uint32_t h = flow_hash(src, dst, ports, proto) & mask;
-            while (true) {
-                const uint4 e = __ldg(&table[h]);
-                if (!(e.w & FLOW_VALID)) break;
-                if (e.x == src && e.y == dst && e.z == ports && (e.w & 0xffu) == proto) {
-                    sa = e.w >> 16;
-                    break;
-                }
-                h = (h + 1u) & mask;
-            }
-        }
-    }
-    A.sa_idx[i] = sa;
+    A.sa_idx[i] = flow_lookup_one(table, mask, A.in_buf + A.in_off[i], A.in_len[i]);
 }
 
 cudaError_t launch_flow_lookup(const uint4 *table, uint32_t mask, const FlowArgs &A, cudaStream_t st)

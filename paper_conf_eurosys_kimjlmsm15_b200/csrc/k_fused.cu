@@ -304,10 +304,11 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
     // staging so their DRAM latency overlaps it
     uint32_t pre_sa = INVALID_SA, pre_D = 0, pre_inoff = 0, pre_outoff = 0;
     if (MERGED && p_begin + tid < p_end) {
-        pre_sa = B.sa_idx[p_begin + tid];
         pre_D = B.in_len[p_begin + tid];
         pre_inoff = B.in_off[p_begin + tid];
         pre_outoff = B.out_off[p_begin + tid];
+        pre_sa = B.sa_idx ? B.sa_idx[p_begin + tid]
+                          : flow_lookup_one(B.flow_table, B.flow_mask, B.in_buf + pre_inoff, pre_D);
     }
     aes_tables_to_smem(tabs, T.te0);
     if (tr && tid == 0) tr[2] = gtimer();
