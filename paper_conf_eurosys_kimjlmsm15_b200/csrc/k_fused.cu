@@ -181,7 +181,7 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
             const uint4 g2 = __ldg(&T.hmid[(size_t)sa * 3 + 2]);
             st[0] = g1.y; st[1] = g1.z; st[2] = g1.w; st[3] = g2.x; st[4] = g2.y;
         }
-        sha1_compress(st, W);
+        sha1_compress_fma(st, W, T.n_sa != 0u ? 1u : 0u);   // (n_sa >= 1: an opaque 1)
         if (it == 0) ck_sha = clock64();
     }
     // ICV = first 96 bits of the outer digest (RFC 2404)

@@ -111,7 +111,7 @@ __device__ __forceinline__ uint32_t esp_in_packet(const DevTable &T, const InBat
             const uint4 h2 = __ldg(&T.hmid[(size_t)sa * 3 + 2]);
             st[0] = h1.y; st[1] = h1.z; st[2] = h1.w; st[3] = h2.x; st[4] = h2.y;
         }
-        sha1_compress(st, W);
+        sha1_compress_fma(st, W, T.n_sa != 0u ? 1u : 0u);   // (n_sa >= 1: an opaque 1)
     }
     os.finish(B.out_buf + outoff + C);
 
