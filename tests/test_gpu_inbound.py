@@ -168,3 +168,44 @@ def test_reset_inbound_replays_same_traffic():
     assert c["pkts_ok"] == 2 * ib.n and c["drop_replay"] == ib.n and c["batches"] == 3
     t.close()
     torch.cuda.synchronize()
+
+
+def test_long_padding_and_bad_trailers():
+    """RFC 4303 §2.4 padding of up to 255 bytes (the kernel checks pad bytes
+    beyond its last two words by reading back its own output), wrong pad
+    bytes at every distance from the end, wrong next header, D < 20, and a
+    non-counter IV -- built with the independent pyca composition."""
+    import pyca_esp
+    from test_oracle_inbound import _packets_batch
+    p = gen.make_sas(1, cfg_id=99)
+    kw = dict(spi=int(p.spi[0]), key=p.aes_key[0], nonce=p.ctr_nonce[0], hkey=p.hmac_key[0],
+              src=int(p.tunnel_src[0]), dst=int(p.tunnel_dst[0]))
+    r = np.random.default_rng(99)
+    pk, q = [], 0
+    for plen in (0, 1, 2, 3, 5, 6, 7, 8, 13, 14, 15, 16, 17, 63, 64, 100, 200, 254, 255):
+        for bad in (None, "pad", "nh"):
+            D = int(r.integers(20, 300))
+            D -= (D + plen + 2) % 4                       # C = 0 mod 4
+            if D < 20:
+                D += 4
+            P = bytes([0x45, 0]) + bytes(r.integers(0, 256, D - 2, dtype=np.uint8))
+            pad = bytearray(range(1, plen + 1))
+            nh = 4
+            if bad == "pad" and plen:
+                pad[int(r.integers(0, plen))] ^= 0x40
+            if bad == "nh":
+                nh = 41
+            q += 1
+            T = P + bytes(pad) + bytes([plen, nh])
+            iv = bytes(r.integers(0, 256, 8, dtype=np.uint8)) if q % 3 == 0 else None
+            pk.append(pyca_esp.encap_raw(kw["spi"], kw["key"], kw["nonce"], kw["hkey"], kw["src"],
+                                         kw["dst"], q, T=T, iv=iv))
+    # D < 20 once the long padding is stripped
+    pk.append(pyca_esp.encap_raw(kw["spi"], kw["key"], kw["nonce"], kw["hkey"], kw["src"], kw["dst"],
+                                 q + 1, T=bytes([0x45, 0]) + bytes(14) + bytes(range(1, 7)) + bytes([6, 4])))
+    ib = _packets_batch([x for x in pk if len(x) <= 1552], [0] * len([x for x in pk if len(x) <= 1552]))
+    g = gpu_inbound_run(p, [ib])
+    o = oracle_inbound_run(p, [ib])
+    assert_same_inbound(g, o, [ib])
+    st = o[0][0][2]
+    assert (st == 0).sum() >= 15 and (st == 5).sum() >= 30
