@@ -395,6 +395,29 @@ def run_ours(args):
         out["n_flows"] = n_flows
         out["miss_fraction"] = 0.05
         t.close()
+        # single-ingress routing (f3): pack the batch for 8 owners (the
+        # all-to-all itself needs >1 GPU); HBM roofline on the bytes moved
+        from paper_conf_eurosys_kimjlmsm15_b200 import redistribute
+        for _ in range(warmup):
+            flush.zero_()
+            redistribute.pack(db, b.n, len(p.spi), 8)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        tot = 0.0
+        for k in range(steps):
+            flush.zero_()
+            e0.record()
+            pk = redistribute.pack(db, b.n, len(p.spi), 8)     # (includes a 2-value D2H for the splits)
+            e1.record()
+            torch.cuda.synchronize()
+            tot += e0.elapsed_time(e1)
+        ms = tot / steps
+        moved = 2 * int(b.in_len.astype(np.int64).sum()) + b.n * (4 + 2 + 4 + 2 + 4 + 12)
+        out["route_pack_8_owners"] = {"ms_per_step": ms, "mpps": b.n / (ms * 1e-3) / 1e6,
+                                      "roofline": {"bound": "hbm", "unit": "GB/s", "peak": peaks["hbm_gbs"],
+                                                   "achieved": moved / (ms * 1e-3) / 1e9,
+                                                   "frac": moved / (ms * 1e-3) / 1e9 / peaks["hbm_gbs"]},
+                                      "packets_per_owner": pk.counts}
         return out
 
     main_cfg = args.config

@@ -217,6 +217,29 @@ int nba_ipsec_lookup_sa(nba_ipsec_sa_table *t, const uint8_t *in_buf, const uint
                         const uint16_t *in_len, uint32_t n_pkts, uint32_t *sa_idx,
                         void *cuda_stream);
 
+/* ---- single-ingress redistribution ---------------
+ *
+ * With SA-hash sharding GPU g owns the SAs s with s mod world = g (local index
+ * s / world).  When all traffic enters at one GPU, route_pack sorts a batch by
+ * owner -- stable, so each owner receives its packets in batch order and the
+ * per-SA sequence numbers are those of one sequential gateway -- and packs it
+ * into destination-major send arrays for one all-to-all per array (NCCL over
+ * NVLink; paper_conf_eurosys_kimjlmsm15_b200/redistribute.py):
+ *   send_buf : packet bytes, destination 0's packets first, back to back
+ *   send_len : their lengths; send_sa: their LOCAL SA indices (s / world)
+ *   dest_counts[d], dest_bytes[d] (DEVICE, world + 1 entries): packets and
+ *   bytes per destination; entry `world` counts packets with s >= n_sa_total,
+ *   which are not sent.
+ * All pointers are DEVICE pointers; sizes: send_buf >= the batch's bytes,
+ * send_len / send_sa >= n_pkts entries, workspace >= route_workspace_bytes.
+ * world must be 1..8.  Enqueued on `cuda_stream` (3 kernel launches). */
+int nba_ipsec_route_workspace_bytes(uint32_t max_pkts, uint32_t world, uint64_t *bytes);
+int nba_ipsec_route_pack(const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
+                         const uint32_t *sa_global, uint32_t n_pkts, uint32_t n_sa_total,
+                         uint32_t world, void *workspace, uint8_t *send_buf, uint16_t *send_len,
+                         uint32_t *send_sa, uint64_t *dest_counts, uint64_t *dest_bytes,
+                         void *cuda_stream);
+
 /* ---- ESP inbound: the mirror of the path ------------------
  *
  * RFC 4303 §3.4 receive processing in tunnel mode on the same SA table (the

@@ -659,6 +659,41 @@ int nba_ipsec_lookup_sa(nba_ipsec_sa_table *t, const uint8_t *in_buf, const uint
                : NBA_IPSEC_ECUDA;
 }
 
+// ---- single-ingress redistribution ----------------------
+
+int nba_ipsec_route_workspace_bytes(uint32_t max_pkts, uint32_t world, uint64_t *bytes)
+{
+    if (!bytes || world == 0 || world > 8 || max_pkts > NBA_IPSEC_MAX_BATCH) return NBA_IPSEC_EINVAL;
+    *bytes = route_workspace_bytes(max_pkts, world);
+    return NBA_IPSEC_OK;
+}
+
+int nba_ipsec_route_pack(const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
+                         const uint32_t *sa_global, uint32_t n_pkts, uint32_t n_sa_total,
+                         uint32_t world, void *workspace, uint8_t *send_buf, uint16_t *send_len,
+                         uint32_t *send_sa, uint64_t *dest_counts, uint64_t *dest_bytes,
+                         void *cuda_stream)
+{
+    if (world == 0 || world > 8 || n_pkts > NBA_IPSEC_MAX_BATCH) return NBA_IPSEC_EINVAL;
+    if (!dest_counts || !dest_bytes) return NBA_IPSEC_EINVAL;
+    cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    if (n_pkts == 0) {
+        return cudaMemsetAsync(dest_counts, 0, (world + 1) * 8ull, st) == cudaSuccess &&
+                       cudaMemsetAsync(dest_bytes, 0, (world + 1) * 8ull, st) == cudaSuccess
+                   ? NBA_IPSEC_OK
+                   : NBA_IPSEC_ECUDA;
+    }
+    if (!in_buf || !in_off || !in_len || !sa_global || !workspace || !send_buf || !send_len ||
+        !send_sa)
+        return NBA_IPSEC_EINVAL;
+    return launch_route(in_buf, in_off, in_len, sa_global, n_pkts, n_sa_total, world, workspace,
+                        send_buf, send_len, send_sa,
+                        reinterpret_cast<unsigned long long *>(dest_counts),
+                        reinterpret_cast<unsigned long long *>(dest_bytes), st) == cudaSuccess
+               ? NBA_IPSEC_OK
+               : NBA_IPSEC_ECUDA;
+}
+
 int nba_ipsec_enable_inbound(nba_ipsec_sa_table *t)
 {
     if (!t) return NBA_IPSEC_EINVAL;

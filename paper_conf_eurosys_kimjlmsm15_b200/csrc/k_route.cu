@@ -1,0 +1,195 @@
+// k_route.cu -- single-ingress redistribution (second half):
+// when all traffic enters at one GPU, every packet must reach the GPU that owns
+// its SA (SA-hash shard, owner = sa mod world, S§8(e)) before the path runs
+// there.  These kernels route and pack a batch by destination so one NCCL
+// all-to-all per array moves it (paper_conf_eurosys_kimjlmsm15_b200/redistribute.py):
+//   k_route_tiles : per 256-packet tile, each packet's destination, its rank
+//                   and byte offset among the tile's packets for that
+//                   destination (warp ballots / segmented scans, warp order),
+//                   and the tile's per-destination counts and bytes;
+//   k_route_scan  : exclusive scans of those over tiles, and the destination
+//                   regions of the send buffers (destination-major);
+//   k_route_pack  : one warp per packet copies its bytes to its place and
+//                   writes its length and LOCAL SA index (sa / world).
+// Stable: a destination receives its packets in batch-index order, so the
+// per-SA sequence numbers at the owner are those of the sequential oracle.
+// Packets without a valid SA (sa >= n_sa_total) are not sent (counted in slot
+// `world`).
+#include "internal.cuh"
+
+namespace nba {
+
+constexpr uint32_t RT_MAX_WORLD = 8;
+constexpr uint32_t RT_TILE = 256;
+
+struct RouteWork {
+    uint32_t *dest;        // [n]   destination (world = dropped)
+    uint32_t *rank;        // [n]   rank among the tile's packets of that destination
+    uint32_t *brank;       // [n]   byte offset among them
+    uint32_t *tcnt;        // [tiles][world+1] counts -> exclusive prefix over tiles
+    unsigned long long *tbyt;   // [tiles][world+1] bytes  -> exclusive prefix over tiles
+    unsigned long long *base;   // [2][world+1] region starts: packets, bytes
+};
+
+__global__ void __launch_bounds__(RT_TILE)
+k_route_tiles(RouteWork R, const uint16_t *in_len, const uint32_t *sa, uint32_t n,
+              uint32_t n_sa_total, uint32_t world)
+{
+    __shared__ uint32_t s_wc[RT_TILE / 32][RT_MAX_WORLD + 1];
+    __shared__ uint32_t s_wb[RT_TILE / 32][RT_MAX_WORLD + 1];
+    const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
+    const uint32_t i = blockIdx.x * RT_TILE + tid;
+    const uint32_t len = i < n ? in_len[i] : 0u;
+    const uint32_t s = i < n ? sa[i] : INVALID_SA;
+    const uint32_t d = i < n ? (s < n_sa_total ? s % world : world) : RT_MAX_WORLD + 1u;
+    uint32_t my_rank = 0, my_brank = 0;
+    for (uint32_t k = 0; k <= world; k++) {
+        const uint32_t m = __ballot_sync(0xffffffffu, d == k);
+        uint32_t x = d == k ? len : 0u;          // inclusive scan of lengths over the warp
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+            if (lane >= (uint32_t)o) x += y;
+        }
+        if (d == k) {
+            my_rank = __popc(m & lanemask_lt());
+            my_brank = x - len;
+        }
+        if (lane == 31) {
+            s_wc[warp][k] = __popc(m);
+            s_wb[warp][k] = x;
+        }
+    }
+    __syncthreads();
+    if (i < n) {
+        uint32_t pc = 0, pb = 0;                // earlier warps of the tile, same destination
+        for (uint32_t w = 0; w < warp; w++) {
+            pc += s_wc[w][d];
+            pb += s_wb[w][d];
+        }
+        R.dest[i] = d;
+        R.rank[i] = pc + my_rank;
+        R.brank[i] = pb + my_brank;
+    }
+    if (tid <= world) {
+        uint32_t c = 0, b = 0;
+        for (uint32_t w = 0; w < RT_TILE / 32; w++) {
+            c += s_wc[w][tid];
+            b += s_wb[w][tid];
+        }
+        R.tcnt[blockIdx.x * (world + 1u) + tid] = c;
+        R.tbyt[blockIdx.x * (world + 1u) + tid] = b;
+    }
+}
+
+// One CTA: exclusive scans over tiles per destination, then region bases.
+__global__ void __launch_bounds__(256)
+k_route_scan(RouteWork R, uint32_t n_tiles, uint32_t world, unsigned long long *dest_counts,
+             unsigned long long *dest_bytes)
+{
+    __shared__ unsigned long long s_tc[RT_MAX_WORLD + 1], s_tb[RT_MAX_WORLD + 1];
+    const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
+    // warp k scans destination k's column (world + 1 <= 9 columns, 8 warps:
+    // warp 0 also takes column 8)
+    for (uint32_t k = warp; k <= world; k += 8u) {
+        unsigned long long cc = 0, cb = 0;
+        for (uint32_t t0 = 0; t0 < n_tiles; t0 += 32u) {
+            const uint32_t t = t0 + lane;
+            const unsigned long long c = t < n_tiles ? R.tcnt[t * (world + 1u) + k] : 0ull;
+            const unsigned long long b = t < n_tiles ? R.tbyt[t * (world + 1u) + k] : 0ull;
+            unsigned long long xc = c, xb = b;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const unsigned long long yc = __shfl_up_sync(0xffffffffu, xc, o);
+                const unsigned long long yb = __shfl_up_sync(0xffffffffu, xb, o);
+                if (lane >= (uint32_t)o) {
+                    xc += yc;
+                    xb += yb;
+                }
+            }
+            if (t < n_tiles) {
+                R.tcnt[t * (world + 1u) + k] = (uint32_t)(cc + xc - c);
+                R.tbyt[t * (world + 1u) + k] = cb + xb - b;
+            }
+            cc += __shfl_sync(0xffffffffu, xc, 31);
+            cb += __shfl_sync(0xffffffffu, xb, 31);
+        }
+        if (lane == 0) {
+            s_tc[k] = cc;
+            s_tb[k] = cb;
+        }
+    }
+    __syncthreads();
+    if (tid == 0) {
+        unsigned long long bc = 0, bb = 0;
+        for (uint32_t k = 0; k <= world; k++) {
+            R.base[k] = bc;
+            R.base[(world + 1u) + k] = bb;
+            dest_counts[k] = s_tc[k];
+            dest_bytes[k] = s_tb[k];
+            bc += s_tc[k];
+            bb += s_tb[k];
+        }
+    }
+}
+
+// One warp per packet: bytes to the send buffer (destination-major, batch
+// order inside a destination), length and local SA index to the send arrays.
+__global__ void __launch_bounds__(256)
+k_route_pack(RouteWork R, const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
+             const uint32_t *sa, uint32_t n, uint32_t world, uint8_t *send_buf, uint16_t *send_len,
+             uint32_t *send_sa)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (i >= n) return;
+    const uint32_t d = R.dest[i];
+    if (d >= world) return;                           // dropped: not sent
+    const uint32_t tile = i / RT_TILE;
+    const unsigned long long pos = R.base[d] + R.tcnt[tile * (world + 1u) + d] + R.rank[i];
+    const unsigned long long boff = R.base[(world + 1u) + d] + R.tbyt[tile * (world + 1u) + d] +
+                                    R.brank[i];
+    const uint32_t len = in_len[i];
+    const uint8_t *src = in_buf + in_off[i];
+    uint8_t *dst = send_buf + boff;
+    for (uint32_t b = lane; b < len; b += 32u) dst[b] = src[b];
+    if (lane == 0) {
+        send_len[pos] = (uint16_t)len;
+        send_sa[pos] = sa[i] / world;
+    }
+}
+
+size_t route_workspace_bytes(uint32_t max_pkts, uint32_t world)
+{
+    const size_t tiles = (max_pkts + RT_TILE - 1) / RT_TILE;
+    return 3ull * max_pkts * 4 + tiles * (world + 1) * (4 + 8) + 2ull * (world + 1) * 8 + 256;
+}
+
+cudaError_t launch_route(const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
+                         const uint32_t *sa, uint32_t n, uint32_t n_sa_total, uint32_t world,
+                         void *ws, uint8_t *send_buf, uint16_t *send_len, uint32_t *send_sa,
+                         unsigned long long *dest_counts, unsigned long long *dest_bytes,
+                         cudaStream_t st)
+{
+    const uint32_t tiles = (n + RT_TILE - 1) / RT_TILE;
+    uint8_t *p = static_cast<uint8_t *>(ws);
+    auto take = [&](size_t b) {
+        uint8_t *r = p;
+        p += (b + 15) & ~(size_t)15;
+        return r;
+    };
+    RouteWork R;
+    R.dest = reinterpret_cast<uint32_t *>(take((size_t)n * 4));
+    R.rank = reinterpret_cast<uint32_t *>(take((size_t)n * 4));
+    R.brank = reinterpret_cast<uint32_t *>(take((size_t)n * 4));
+    R.tcnt = reinterpret_cast<uint32_t *>(take((size_t)tiles * (world + 1) * 4));
+    R.tbyt = reinterpret_cast<unsigned long long *>(take((size_t)tiles * (world + 1) * 8));
+    R.base = reinterpret_cast<unsigned long long *>(take(2ull * (world + 1) * 8));
+    k_route_tiles<<<tiles, RT_TILE, 0, st>>>(R, in_len, sa, n, n_sa_total, world);
+    k_route_scan<<<1, 256, 0, st>>>(R, tiles, world, dest_counts, dest_bytes);
+    k_route_pack<<<(n * 32u + 255u) / 256u, 256, 0, st>>>(R, in_buf, in_off, in_len, sa, n, world,
+                                                         send_buf, send_len, send_sa);
+    return cudaGetLastError();
+}
+
+}  // namespace nba

@@ -108,6 +108,8 @@ def _load():
         "nba_ipsec_debug_trace": (i32, [vp, P(u64), u32]),
         "nba_ipsec_enable_inbound": (i32, [vp]),
         "nba_ipsec_set_flow_table": (i32, [vp, P(Flow), u32]),
+        "nba_ipsec_route_workspace_bytes": (i32, [u32, u32, P(u64)]),
+        "nba_ipsec_route_pack": (i32, [vp, vp, vp, vp, u32, u32, u32, vp, vp, vp, vp, vp, vp, vp]),
         "nba_ipsec_lookup_sa": (i32, [vp, vp, vp, vp, u32, vp, vp]),
         "nba_ipsec_process_inbound": (i32, [vp, P(InBatch), vp]),
         "nba_ipsec_read_in_counters": (i32, [vp, P(InCounters), vp]),
@@ -348,3 +350,21 @@ def host_hmac_sha1_midstates(key: bytes):
     lib.nba_ipsec_host_hmac_sha1_midstates(k.ctypes.data_as(ctypes.POINTER(ctypes.c_uint8)),
                                            hin.ctypes.data_as(u32p), hout.ctypes.data_as(u32p))
     return hin, hout
+
+
+# -- single-ingress redistribution ----------------------------
+def route_workspace_bytes(max_pkts: int, world: int) -> int:
+    b = ctypes.c_uint64(0)
+    _check(lib.nba_ipsec_route_workspace_bytes(max_pkts, world, ctypes.byref(b)),
+           "nba_ipsec_route_workspace_bytes")
+    return int(b.value)
+
+
+def route_pack(in_buf, in_off, in_len, sa_global, n, n_sa_total, world, workspace, send_buf,
+               send_len, send_sa, dest_counts, dest_bytes, stream=None):
+    """nba_ipsec_route_pack on device tensors (see include/nba_ipsec.h)."""
+    _check(lib.nba_ipsec_route_pack(_ptr(in_buf), _ptr(in_off), _ptr(in_len), _ptr(sa_global), int(n),
+                                    int(n_sa_total), int(world), _ptr(workspace), _ptr(send_buf),
+                                    _ptr(send_len), _ptr(send_sa), _ptr(dest_counts),
+                                    _ptr(dest_bytes), _stream_handle(stream)),
+           "nba_ipsec_route_pack")

@@ -1,0 +1,88 @@
+"""Single-ingress redistribution: when all traffic
+enters at one GPU, each packet must reach the GPU that owns its SA (SA-hash
+shard: owner = s mod world) before the ESP path runs there.
+
+  1. nba_ipsec_route_pack (CUDA kernels, libnba_ipsec.so) sorts the ingress
+     batch by owner -- stable -- into destination-major send arrays;
+  2. exchange() moves them with one all-to-all per array (NCCL over NVLink on
+     GPUs; any torch.distributed backend works, tests use gloo on CPU);
+  3. each owner runs nba_ipsec_process_batch on what it received (local SA
+     indices, packets back to back).
+
+This module is plumbing only (sizes, splits, offsets); the routing and packing
+arithmetic is in the kernels.
+"""
+from __future__ import annotations
+
+import dataclasses
+
+import torch
+import torch.distributed as dist
+
+
+@dataclasses.dataclass
+class Packed:
+    """One rank's destination-major send arrays (output of route_pack)."""
+    buf: torch.Tensor        # uint8 [>= total bytes]
+    length: torch.Tensor     # int16 [>= total packets] (uint16 values)
+    sa: torch.Tensor         # int32 [>= total packets] local SA indices
+    counts: list             # packets per destination (world entries)
+    nbytes: list             # bytes per destination
+
+
+@dataclasses.dataclass
+class Received:
+    """What a rank received: a packed batch for its own SA table."""
+    n: int
+    in_buf: torch.Tensor     # uint8
+    in_off: torch.Tensor     # int32 (uint32 values)
+    in_len: torch.Tensor     # int16 (uint16 values)
+    sa_idx: torch.Tensor     # int32 local SA indices
+
+
+def pack(db, n: int, n_sa_total: int, world: int, stream=None) -> Packed:
+    """Route and pack a device batch (gen/device.DeviceBatch with GLOBAL SA
+    indices) on the GPU with nba_ipsec_route_pack."""
+    from . import nba_ipsec
+    dev = db.in_buf.device
+    ws = torch.empty(nba_ipsec.route_workspace_bytes(max(n, 1), world), dtype=torch.uint8, device=dev)
+    send_buf = torch.empty(max(int(db.in_buf.numel()), 1), dtype=torch.uint8, device=dev)
+    send_len = torch.empty(max(n, 1), dtype=torch.int16, device=dev)
+    send_sa = torch.empty(max(n, 1), dtype=torch.int32, device=dev)
+    dc = torch.zeros(world + 1, dtype=torch.int64, device=dev)
+    dbytes = torch.zeros(world + 1, dtype=torch.int64, device=dev)
+    nba_ipsec.route_pack(db.in_buf, db.in_off, db.in_len, db.sa_idx, n, n_sa_total, world, ws,
+                         send_buf, send_len, send_sa, dc, dbytes, stream=stream)
+    c = dc.cpu().tolist()
+    b = dbytes.cpu().tolist()
+    return Packed(buf=send_buf, length=send_len, sa=send_sa, counts=c[:world], nbytes=b[:world])
+
+
+def exchange(p: Packed, group=None) -> Received:
+    """All-to-all of the packed arrays; returns this rank's received batch.
+    Every rank calls it (ranks without ingress traffic pass empty arrays)."""
+    world = dist.get_world_size(group)
+    dev = p.buf.device
+    sizes = torch.tensor([p.counts, p.nbytes], dtype=torch.int64).t().contiguous().to(dev)
+    got = torch.empty_like(sizes)
+    dist.all_to_all_single(got, sizes, group=group)
+    got = got.cpu()
+    r_cnt = got[:, 0].tolist()
+    r_byt = got[:, 1].tolist()
+    n_in, b_in = sum(p.counts), sum(p.nbytes)
+    n_out, b_out = sum(r_cnt), sum(r_byt)
+    # lengths travel as bytes (16-bit integers are not an NCCL type)
+    len_bytes = torch.empty(max(2 * n_out, 1), dtype=torch.uint8, device=dev)
+    dist.all_to_all_single(len_bytes[:2 * n_out], p.length[:n_in].view(torch.uint8)[:2 * n_in],
+                           [2 * c for c in r_cnt], [2 * c for c in p.counts], group=group)
+    sa = torch.empty(max(n_out, 1), dtype=torch.int32, device=dev)
+    dist.all_to_all_single(sa[:n_out], p.sa[:n_in], r_cnt, p.counts, group=group)
+    buf = torch.empty(max(b_out, 1) + 16, dtype=torch.uint8, device=dev)
+    dist.all_to_all_single(buf[:b_out], p.buf[:b_in], r_byt, p.nbytes, group=group)
+    length = len_bytes[:2 * n_out].view(torch.int16) if n_out else torch.zeros(1, dtype=torch.int16,
+                                                                                 device=dev)
+    lens = length[:n_out].to(torch.int64) & 0xFFFF
+    off = torch.zeros(max(n_out, 1), dtype=torch.int64, device=dev)
+    if n_out > 1:
+        off[1:n_out] = torch.cumsum(lens[:-1], 0)
+    return Received(n=n_out, in_buf=buf, in_off=off.to(torch.int32), in_len=length, sa_idx=sa)
