@@ -509,7 +509,8 @@ def run_ours(args):
                        "parallelism": f"sa-hash shard x{world} (no data-path collective)",
                        "l2": "flushed before every timed step (256 MiB device write, untimed)",
                        "timing": "CUDA events per step on the launching stream, sum over steps, max over ranks",
-                       "pipeline": "fused" if args.pipeline in (None, 0) and res["launches"] // args.steps == 2 else "unfused"},
+                       "pipeline": ("fused" if args.pipeline in (None, 0) else "unfused") +
+                                   f" ({res['launches'] // args.steps} launch(es) per step)"},
             "roofline": roof,
             "kernels": {k: {"ms_per_launch": v["ms_per_launch"], "frac": v["frac"], "unit": v["unit"],
                             "achieved": v["achieved"]} for k, v in kern_roofs.items()},
