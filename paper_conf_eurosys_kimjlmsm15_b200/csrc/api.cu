@@ -190,6 +190,7 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
     // ---- a0: host-side key schedules, midstates, header words -------------
     std::vector<uint4> rk((size_t)n_sa * 11), hm((size_t)n_sa * 3), hdr(n_sa);
     std::vector<uint32_t> seq(n_sa);
+    std::vector<uint4> sal((size_t)n_sa * SAL_U4, make_uint4(0, 0, 0, 0));
     for (uint32_t s = 0; s < n_sa; s++) {
         const nba_ipsec_sa_params &p = sas[s];
         uint8_t bytes[176];
@@ -208,10 +209,16 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
         std::memcpy(&nonce, p.ctr_nonce, 4);
         hdr[s] = make_uint4(be_img(p.spi), nonce, be_img(p.tunnel_src), be_img(p.tunnel_dst));
         seq[s] = p.seq;
+        uint4 *line = &sal[(size_t)s * SAL_U4];
+        line[0] = rk[(size_t)s * 11];
+        line[1] = hdr[s];
+        line[2] = hm[(size_t)s * 3 + 0];
+        line[3] = hm[(size_t)s * 3 + 1];
+        line[4] = hm[(size_t)s * 3 + 2];
     }
     t->seq0 = seq;
 
-    uint4 *d_rk = nullptr, *d_hm = nullptr, *d_hdr = nullptr;
+    uint4 *d_rk = nullptr, *d_hm = nullptr, *d_hdr = nullptr, *d_sal = nullptr;
     uint32_t *d_seq = nullptr, *d_seq_prev = nullptr, *d_te0 = nullptr;
     const uint32_t M = max_batch_pkts;
     cudaError_t e = cudaSuccess;
@@ -221,6 +228,7 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
     chk(dalloc(t, &d_rk, rk.size()));
     chk(dalloc(t, &d_hm, hm.size()));
     chk(dalloc(t, &d_hdr, hdr.size()));
+    chk(dalloc(t, &d_sal, sal.size()));
     chk(dalloc(t, &d_seq, n_sa));
     chk(dalloc(t, &d_seq_prev, n_sa));
     chk(dalloc(t, &d_te0, 256));
@@ -249,6 +257,7 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
         chk(cudaMemcpy(d_rk, rk.data(), rk.size() * sizeof(uint4), cudaMemcpyHostToDevice));
         chk(cudaMemcpy(d_hm, hm.data(), hm.size() * sizeof(uint4), cudaMemcpyHostToDevice));
         chk(cudaMemcpy(d_hdr, hdr.data(), hdr.size() * sizeof(uint4), cudaMemcpyHostToDevice));
+        chk(cudaMemcpy(d_sal, sal.data(), sal.size() * sizeof(uint4), cudaMemcpyHostToDevice));
         chk(cudaMemcpy(d_seq, seq.data(), n_sa * sizeof(uint32_t), cudaMemcpyHostToDevice));
         chk(cudaMemcpy(d_te0, host_te0(), 256 * sizeof(uint32_t), cudaMemcpyHostToDevice));
     }
@@ -266,7 +275,7 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
         delete t;
         return e == cudaErrorMemoryAllocation ? NBA_IPSEC_ENOMEM : NBA_IPSEC_ECUDA;
     }
-    t->T = DevTable{d_rk, d_hm, d_hdr, d_seq, d_seq_prev, d_te0, n_sa};
+    t->T = DevTable{d_rk, d_hm, d_hdr, d_seq, d_seq_prev, d_te0, n_sa, d_sal};
     *out = t;
     return NBA_IPSEC_OK;
 }

@@ -283,6 +283,35 @@ __device__ __forceinline__ void aes4_keystream(uint32_t lane4r, const CtrPre &c,
 #undef NBA_FINAL
 }
 
+// FIPS-197 §5.2 KeyExpansion of the lane's AES-128 key (round key 0 = r0) in
+// registers, SubWord through the S-box bytes of the T-tables (the S-box value
+// is byte 0 of T2[x], byte 1 of T3[x], byte 2 of T0[x], byte 3 of T1[x]);
+// RotWord on a little-endian word image is a rotation by 8 bits, folded into
+// which state byte indexes which table.  Round keys 1 and 2 are returned (the
+// CTR precompute uses them), 3..10 go to L.rkA / H.rkB[.][tid].  40 lookups and
+// ~100 ALU ops per packet replace 160 bytes of round-key loads per packet.
+__device__ __forceinline__ void expand_key_lane(uint32_t lane4r, const uint4 &r0, uint4 &r1, uint4 &r2,
+                                                FusedLo &L, FusedHi &H, uint32_t tid)
+{
+    uint32_t w0 = r0.x, w1 = r0.y, w2 = r0.z, w3 = r0.w;
+    uint32_t rc = 1u;
+#pragma unroll
+    for (int r = 1; r <= 10; r++) {
+        const uint32_t t = (TL(w3, 1, 2) & 0x000000ffu) | (TL(w3, 2, 3) & 0x0000ff00u) |
+                           (TL(w3, 3, 0) & 0x00ff0000u) | (TL(w3, 0, 1) & 0xff000000u);
+        w0 ^= t ^ rc;                              // Rcon[r] = {rc, 0, 0, 0}
+        w1 ^= w0;
+        w2 ^= w1;
+        w3 ^= w2;
+        rc = ((rc << 1) ^ ((rc >> 7) * 0x11bu)) & 0xffu;   // xtime (constant per r)
+        const uint4 k = make_uint4(w0, w1, w2, w3);
+        if (r == 1) r1 = k;
+        else if (r == 2) r2 = k;
+        else if (r <= 6) L.rkA[r - 3][tid] = k;
+        else H.rkB[r - 7][tid] = k;
+    }
+}
+
 // Warp-cooperative, coalesced staging of round keys 3..10 of each lane's SA
 // (sa_me; INVALID_SA = none) into L.rkA / H.rkB: load m of the warp covers 128
 // contiguous bytes of 4 lanes' SAs.  Followed by __syncwarp in the caller.
@@ -371,6 +400,15 @@ __device__ __forceinline__ void load_raw5(uintptr_t a, uintptr_t end, Raw5 &r)
         const uintptr_t qa = abase + 16u * i;
         r.c[i] = qa < end ? ldg_nc_v4(reinterpret_cast<const void *>(qa)) : z4;
     }
+}
+
+// load_raw5 when all five 16-byte loads are known to be inside the stream
+__device__ __forceinline__ void load_raw5_inb(uintptr_t a, Raw5 &r)
+{
+    const uintptr_t abase = a & ~(uintptr_t)15;
+    r.sh = (uint32_t)(a & 15u);
+#pragma unroll
+    for (int i = 0; i < 5; i++) r.c[i] = ldg_nc_v4(reinterpret_cast<const void *>(abase + 16u * i));
 }
 
 __device__ __forceinline__ void extract16(const Raw5 &r, uint32_t (&o)[16])

@@ -35,7 +35,11 @@ struct DevTable {
     uint32_t *seq_prev;     // [n_sa] value of seq before the current batch
     const uint32_t *te0;    // [256] T-table, row-0 byte in bits 0..7
     uint32_t n_sa;
+    const uint4 *sal;       // [n_sa * SAL_U4] one 128-byte line per SA: AES key (round
+                            //   key 0), sahdr, hmid[0..2] -- what an outbound lane
+                            //   loads (it expands round keys 1..10 itself)
 };
+constexpr uint32_t SAL_U4 = 8;   // uint4s per SA line (5 used)
 
 // --- per-batch workspace ----------------------------------------------------
 struct DevWork {
@@ -318,6 +322,29 @@ __device__ __forceinline__ void grid_sync_mono(uint32_t *count, uint32_t target)
     __syncthreads();
 }
 
+// The same barrier in two halves, so a CTA can issue independent loads between
+// its arrival and the wait: grid_arrive after a __syncthreads that orders the
+// CTA's prior global writes; grid_wait ends with a __syncthreads.
+__device__ __forceinline__ void grid_arrive(uint32_t *count)
+{
+    if (threadIdx.x == 0) {
+        __threadfence();
+        atomicAdd(count, 1u);
+    }
+}
+
+__device__ __forceinline__ void grid_wait(const uint32_t *count, uint32_t target)
+{
+    if (threadIdx.x == 0) {
+        uint32_t v;
+        do {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(count) : "memory");
+        } while ((int)(v - target) < 0);
+        __threadfence();
+    }
+    __syncthreads();
+}
+
 // Exclusive prefix of the tile counts down SA column `sa` by one warp, then the
 // SA counter advance (only the first (2^32-1 - seq) packets get numbers).
 __device__ __forceinline__ void st_relaxed_u64(unsigned long long *p, unsigned long long v)
@@ -351,11 +378,12 @@ __device__ __forceinline__ void put_prefix(const DevWork &W, size_t idx, uint32_
 // (2^32-1 - seq) packets get numbers).
 template <bool BASE>
 __device__ __forceinline__ void scan_sa_column(const DevTable &T, const DevWork &W, uint32_t sa,
-                                               uint32_t n_tiles, uint32_t lane, uint32_t epoch)
+                                               uint32_t n_tiles, uint32_t lane, uint32_t epoch,
+                                               bool have_pre = false, uint32_t old_pre = 0)
 {
     constexpr int U = 8;                       // 8 x 32 = 256 tiles per pass
     uint16_t *col = W.hist16 + (size_t)sa * n_tiles;
-    const uint32_t old = __shfl_sync(0xffffffffu, lane == 0 ? T.seq[sa] : 0u, 0);
+    const uint32_t old = have_pre ? old_pre : __shfl_sync(0xffffffffu, lane == 0 ? T.seq[sa] : 0u, 0);
     uint32_t carry = 0;
     for (uint32_t t0 = 0; t0 < n_tiles; t0 += 32u * U) {
         uint32_t h[U];
@@ -388,17 +416,29 @@ __device__ __forceinline__ void scan_sa_column(const DevTable &T, const DevWork 
     }
 }
 
+// The SA counter this warp's first row scan starts from (scan_all_columns with
+// have_pre): T.seq of row `slot` (warp-per-row) or of row slot + lane * nslots
+// (lane-per-row).  Only that scan writes T.seq of the row, so the value may be
+// loaded early -- the merged kernel loads it before it waits at its barrier.
+__device__ __forceinline__ uint32_t scan_first_old(const DevTable &T, uint32_t slot, uint32_t nslots,
+                                                   uint32_t n_tiles, uint32_t lane)
+{
+    const size_t sa = n_tiles > 32u ? (size_t)slot : slot + (size_t)lane * nslots;
+    return sa < T.n_sa ? T.seq[sa] : 0u;
+}
+
 // All SA rows, by `nslots` warps (this one is `slot`).  Long rows: one warp per
 // SA (scan_sa_column).  Short rows (small batches, n_tiles <= 32): one LANE per
 // SA, so a few warps still cover thousands of SAs in one memory round trip.
 template <bool BASE = false>
 __device__ __forceinline__ void scan_all_columns(const DevTable &T, const DevWork &W, uint32_t slot,
                                                  uint32_t nslots, uint32_t n_tiles, uint32_t lane,
-                                                 uint32_t epoch = 0)
+                                                 uint32_t epoch = 0, bool have_pre = false,
+                                                 uint32_t old_pre = 0)
 {
     if (n_tiles > 32u) {
         for (uint32_t col = slot; col < T.n_sa; col += nslots)
-            scan_sa_column<BASE>(T, W, col, n_tiles, lane, epoch);
+            scan_sa_column<BASE>(T, W, col, n_tiles, lane, epoch, have_pre && col == slot, old_pre);
         return;
     }
     for (uint32_t k0 = 0; (size_t)k0 * nslots < T.n_sa; k0 += 32u) {
@@ -407,7 +447,7 @@ __device__ __forceinline__ void scan_all_columns(const DevTable &T, const DevWor
         if (sa_l >= T.n_sa) continue;
         const uint32_t sa = (uint32_t)sa_l;
         uint16_t *col = W.hist16 + (size_t)sa * n_tiles;
-        const uint32_t old = T.seq[sa];
+        const uint32_t old = (have_pre && k0 == 0) ? old_pre : T.seq[sa];
         uint32_t h[32];
 #pragma unroll
         for (uint32_t t = 0; t < 32u; t++) h[t] = t < n_tiles ? __ldcg(&col[t]) : 0u;

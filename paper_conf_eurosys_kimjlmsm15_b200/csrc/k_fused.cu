@@ -37,29 +37,49 @@ namespace nba {
 #ifndef NBA_LONG_HIGH         // 1: longest packets in the highest warps (A/B: lowest is faster)
 #define NBA_LONG_HIGH 0
 #endif
+#ifndef NBA_INTERIOR          // 1: select-free fast path for interior 64-byte steps / SHA blocks
+#define NBA_INTERIOR 1
+#endif
 #ifndef NBA_SA_PREFETCH       // L2 prefetch of the SA table at kernel start
 #define NBA_SA_PREFETCH 1
 #endif
 
-constexpr uint32_t INFO_TOSLOAD = 0x40000000u;   // esp_packet loads the TOS byte itself
 
 // ---------------------------------------------- one packet, one lane
+// The packet's SA-table words (round keys 0..2, header words, inner HMAC
+// midstate) and the inner TOS byte: loaded together so their latencies
+// overlap; the merged kernel issues them before it waits at its grid barrier.
+struct PktPre {
+    uint4 r0, r1, r2, hd, h0, h1;
+    uint32_t tos;
+};
+
+// Loads the SA line (one 128-byte line per SA) and the TOS byte; r1 / r2 are
+// filled in by expand_key_lane.
+__device__ __forceinline__ PktPre load_pkt_pre(const DevTable &T, const uint8_t *in_buf, uint32_t sa,
+                                               uint32_t inoff, bool load_tos, uint32_t tos)
+{
+    PktPre p;
+    const uint4 *line = T.sal + (size_t)sa * SAL_U4;
+    p.r0 = __ldg(&line[0]);
+    p.hd = __ldg(&line[1]);
+    p.h0 = __ldg(&line[2]);
+    p.h1 = __ldg(&line[3]);
+    p.r1 = p.r2 = make_uint4(0, 0, 0, 0);
+    // TOS of the inner header (the outer header copies it, reading A13)
+    p.tos = load_tos ? (uint32_t)__ldg(in_buf + inoff + 1) : tos;
+    return p;
+}
+
 __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B, FusedLo &L,
                                            FusedHi &H, uint32_t lane4r, uint32_t tid, uint32_t sa,
                                            uint32_t info, uint32_t q32, uint32_t inoff,
-                                           uint32_t outoff, unsigned long long *dbg)
+                                           uint32_t outoff, const PktPre &pp, unsigned long long *dbg)
 {
     long long ck_start = clock64(), ck_setup = 0, ck_aes = 0, ck_sha = 0, ck_emit = 0;
-    // every global load of the setup first, so their latencies overlap
-    const uint4 *rks = T.rk + (size_t)sa * 11u;
-    const uint4 r0 = __ldg(&rks[0]), r1 = __ldg(&rks[1]), r2 = __ldg(&rks[2]);
-    const uint4 hd = __ldg(&T.sahdr[sa]);
-    const uint4 h0 = __ldg(&T.hmid[(size_t)sa * 3 + 0]);
-    const uint4 h1 = __ldg(&T.hmid[(size_t)sa * 3 + 1]);
+    const uint4 r0 = pp.r0, r1 = pp.r1, r2 = pp.r2, hd = pp.hd, h0 = pp.h0, h1 = pp.h1;
     const uint32_t D = info & 0x7ffu;
-    // TOS of the inner header (outer header copies it, reading A13): from the
-    // metadata phase, or loaded here (merged prologue: off its critical path)
-    const uint32_t tos = (info & INFO_TOSLOAD) ? (uint32_t)__ldg(B.in_buf + inoff + 1) : (info >> 16) & 0xffu;
+    const uint32_t tos = pp.tos;
     const uint32_t pad = esp_pad(D);
     const uint32_t C = D + pad + 2u;
     const uint32_t Lb = 48u + C;
@@ -73,7 +93,7 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
     // nonce || 0 || BE32(q) || BE32(k+1), k+1 < 256: only byte 3 of column 3
     // varies, so round 1 is t0 = T3[r3 ^ (k+1)] ^ X0 and round 2 is
     // u_c = T[row(t0)] ^ Z_c), header words, HMAC inner midstate
-    // round keys 3..10 were staged into L.rkA / H.rkB by the warp (coalesced)
+    // round keys 3..10 were expanded into L.rkA / H.rkB[.][tid] by expand_key_lane
     const uint32_t qbe = bswap32(q32);
     const CtrPre cp = ctr_precompute(lane4r, r0, r1, r2, hd.y, 0u, qbe);   // IV = BE64(q), A6
 
@@ -118,8 +138,13 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
         if (it < nsteps) {
             // payload words of T bytes [64 it, 64 it + 64), realigned
             if (64u * (it + NBA_PF_AHEAD) < D) prefetch_l2(src + 64u * (it + NBA_PF_AHEAD));
+            // interior step: all 16 words are payload, the trailer (last word and,
+            // when p = 3, the one before) lies beyond it, and the five 16-byte
+            // loads are inside the datagram -- no per-word selects, one bounds test
+            const bool interior = NBA_INTERIOR && 16u * it + 18u <= Cw;
             Raw5 raw;
-            load_raw5(reinterpret_cast<uintptr_t>(src) + 64u * it, src_end, raw);
+            if (interior) load_raw5_inb(reinterpret_cast<uintptr_t>(src) + 64u * it, raw);
+            else load_raw5(reinterpret_cast<uintptr_t>(src) + 64u * it, src_end, raw);
             // AES-128 of counter blocks 4 it + 1 .. 4 it + 4
             uint32_t ks[16];
             aes4_keystream(lane4r, cp, it, L, H, tid, ks);
@@ -129,7 +154,7 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
                 // trailer: T ends on a word boundary (C = 0 mod 4), so it touches only
                 // the last word (and the one before when p = 3):
                 //   p=0 [P P 0 4]  p=1 [P 1 1 4]  p=2 [1 2 2 4]  p=3 [.. 1][2 3 3 4]
-                {
+                if (!interior) {
                     const uint32_t lw = Cw - 1u - 16u * it;          // last T word in this step?
                     const uint32_t keep = pad == 0 ? 0x0000ffffu : pad == 1 ? 0x000000ffu : 0u;
                     const uint32_t trl = pad == 0 ? 0x04000000u : pad == 1 ? 0x04010100u
@@ -161,13 +186,18 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
         uint32_t W[16];
         if (it < nb_in) {
             const uint32_t m0 = 16u * it;
+            if (NBA_INTERIOR && m0 + 16u <= Mw && it + 1u < nb_in) {   // a block of message words only
 #pragma unroll
-            for (int i = 0; i < 16; i++) {
-                const uint32_t m = m0 + i;
-                const uint32_t msg = i < 4 ? carry[i] : bswap32(ct[i - 4]);
-                W[i] = m < Mw ? msg : (m == Mw ? 0x80000000u : 0u);
+                for (int i = 0; i < 16; i++) W[i] = i < 4 ? carry[i] : bswap32(ct[i - 4]);
+            } else {                                  // FIPS 180-4 §5.1.1 padding
+#pragma unroll
+                for (int i = 0; i < 16; i++) {
+                    const uint32_t m = m0 + i;
+                    const uint32_t msg = i < 4 ? carry[i] : bswap32(ct[i - 4]);
+                    W[i] = m < Mw ? msg : (m == Mw ? 0x80000000u : 0u);
+                }
+                if (it == nb_in - 1u) W[15] = bitlen;
             }
-            if (it == nb_in - 1u) W[15] = bitlen;
 #pragma unroll
             for (int i = 0; i < 4; i++) carry[i] = bswap32(ct[12 + i]);
         } else {
@@ -177,8 +207,8 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
 #pragma unroll
             for (int i = 6; i < 15; i++) W[i] = 0u;
             W[15] = (64u + 20u) * 8u;
-            const uint4 g1 = __ldg(&T.hmid[(size_t)sa * 3 + 1]);
-            const uint4 g2 = __ldg(&T.hmid[(size_t)sa * 3 + 2]);
+            const uint4 g1 = __ldg(&T.sal[(size_t)sa * SAL_U4 + 3]);
+            const uint4 g2 = __ldg(&T.sal[(size_t)sa * SAL_U4 + 4]);
             st[0] = g1.y; st[1] = g1.z; st[2] = g1.w; st[3] = g2.x; st[4] = g2.y;
         }
         sha1_compress_fma(st, W, T.n_sa != 0u ? 1u : 0u);   // (n_sa >= 1: an opaque 1)
@@ -206,12 +236,11 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
 // the CTA come from __match_any_sync groups merged across the 16 warps through
 // a small shared hash (slot per SA; per-warp group sizes); the CTA's per-SA
 // counts go to the SA-major matrix; after a grid barrier one warp per SA scans
-// its row (exclusive prefix over CTAs, SA counter advance); after a second
-// barrier every packet's sequence number is known.  Deterministic: no atomic
-// decides a rank.  Returns the packet's rank among the CTA's packets of its SA.
-__device__ __forceinline__ uint32_t merged_prologue(const DevTable &T, const DevWork &W, FusedLo &L,
-                                                    uint32_t s, uint32_t bar_base, uint32_t epoch,
-                                                    unsigned long long *tr)
+// its row (exclusive prefix over CTAs, SA counter advance) and publishes
+// epoch-tagged bases, which each packet polls.  Deterministic: no atomic
+// decides a rank.  This part returns the packet's rank among the CTA's packets
+// of its SA (INVALID_SA: not counted).
+__device__ __forceinline__ uint32_t merged_local_rank(const DevWork &W, FusedLo &L, uint32_t s)
 {
     constexpr uint32_t HS = 2u * F_SUPER, NW = F_THREADS / 32u;
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
@@ -248,14 +277,28 @@ __device__ __forceinline__ uint32_t merged_prologue(const DevTable &T, const Dev
         if ((m >> (warp + 1u)) == 0u && lane == hi_lane)
             W.hist16[(size_t)s * G + cta] = (uint16_t)(base + wcnt_me);
     }
-    if (tr && tid == 0) tr[4] = gtimer();
-    grid_sync_mono(&W.ctl[CTL_BAR_MONO], bar_base + G);
-    if (tr && tid == 0) tr[5] = gtimer();
-    // row scans publish epoch-tagged bases; no second barrier: each packet
-    // polls its own (SA, CTA) entry
-    scan_all_columns<true>(T, W, cta * NW + warp, G * NW, G, lane, epoch);
-    if (tr && tid == 0) tr[6] = gtimer();
     return rank;
+}
+
+// Counting sort of the super-round's packets by SHA-1 length (L.bins holds the
+// counts; `bin` is thread j's packet's bin): L.perm[position] = packet.
+__device__ __forceinline__ void length_sort(FusedLo &L, uint32_t j, uint32_t cnt_pk, uint32_t bin)
+{
+    const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
+    __syncthreads();
+    if (warp == 0) {   // exclusive scan of the 32 bin counts -> bin cursors
+        uint32_t cb = L.bins[lane], x = cb;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+            if (lane >= (uint32_t)o) x += y;
+        }
+        L.bins[lane] = x - cb;
+    }
+    __syncthreads();
+    if (j < cnt_pk) L.perm[atomicAdd(&L.bins[bin], 1u)] = (uint16_t)j;
+    __syncthreads();
+    if (tid < NBINS) L.bins[tid] = 0;   // next round's counts (after its barrier)
 }
 
 // ---------------------------------------------------------------- the kernel
@@ -313,7 +356,7 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
     aes_tables_to_smem(tabs, T.te0);
     if (tr && tid == 0) tr[2] = gtimer();
     if (tid < 4) L.cnt[tid] = 0ull;
-    if (tid < NBINS) L.bins[tid] = 0;   // re-zeroed after each use (below)
+    if (tid < NBINS) L.bins[tid] = 0;   // re-zeroed after each use (length_sort)
     if (MERGED) {
         for (uint32_t k = tid; k < 2u * F_SUPER; k += F_THREADS) {
             L.hkey[k] = INVALID_SA;
@@ -325,6 +368,88 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
     static_assert(F_SUPER <= F_THREADS, "one packet per thread in the metadata phase");
     uint32_t c_ok = 0, c_drop = 0, c_in = 0, c_out = 0;
 
+    if constexpr (MERGED) {
+        // ---- one super-round; thread j <-> packet p_begin + j ----------------
+        constexpr uint32_t NW = F_THREADS / 32u;
+        const uint32_t G = gridDim.x, cta = blockIdx.x;
+        const uint32_t cnt_pk = p_end > p_begin ? p_end - p_begin : 0u;
+        const uint32_t j = tid;
+        const bool cand = j < cnt_pk && pre_sa < n_sa && pre_D >= MIN_D && pre_D <= MAX_D;
+        const uint32_t bin = hmac_bin(cand, esp_C(pre_D));
+        if (j < cnt_pk) {
+            L.sa[j] = pre_sa;
+            L.info[j] = cand ? (pre_D | INFO_OK) : 0u;
+            L.inoff[j] = pre_inoff;
+            L.outoff[j] = pre_outoff;
+            atomicAdd(&L.bins[bin], 1u);
+            // the lane reads the payload after the barrier: DRAM -> L2 now
+            if (cand) prefetch_l2(B.in_buf + pre_inoff);
+        }
+        // 1. CTA-local ranks and per-SA counts (the prologue's tile part)
+        const uint32_t rank = merged_local_rank(W, L, cand ? pre_sa : INVALID_SA);
+        if (j < cnt_pk) L.seq[j] = rank;
+        if (tr && tid == 0) tr[4] = gtimer();
+        // 2. lane order: longest packets first (seq-overflow drops keep their bin)
+        length_sort(L, j, cnt_pk, bin);   // ends with __syncthreads: counts written
+        grid_arrive(&W.ctl[CTL_BAR_MONO]);
+        // 3. between arrival and wait: everything of the lane's packet that does
+        //    not depend on its sequence number -- round keys 3..10 to shared
+        //    memory, the SA words and TOS to registers; and the SA counter this
+        //    warp's row scan starts from
+        const bool have = tid < cnt_pk;
+        const uint32_t pk = have ? L.perm[tid] : 0u;
+        const uint32_t info = have ? L.info[pk] : 0u;
+        const uint32_t sa_me = (info & INFO_OK) ? L.sa[pk] : INVALID_SA;
+        const uint32_t inoff = have ? L.inoff[pk] : 0u;
+        PktPre pp = {};
+        if (sa_me != INVALID_SA) {
+            pp = load_pkt_pre(T, B.in_buf, sa_me, inoff, true, 0u);
+            expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
+        }
+        const uint32_t old0 = scan_first_old(T, cta * NW + warp, G * NW, G, lane);
+        grid_wait(&W.ctl[CTL_BAR_MONO], bar_base + G);
+        if (tr && tid == 0) tr[5] = gtimer();
+        // 4. row scans publish epoch-tagged bases; each packet polls its own
+        //    (SA, CTA) entry
+        scan_all_columns<true>(T, W, cta * NW + warp, G * NW, G, lane, epoch, true, old0);
+        if (tr && tid == 0) tr[6] = gtimer();
+        __syncwarp();
+        if (tr && tid == 0) tr[1] = gtimer();
+        // 5. sequence numbers: thread j polls the published base of its packet's
+        //    (SA, CTA) entry; all polls end before any lane starts its packet
+        //    (measured: letting each warp start after its own polls leaves
+        //    stragglers whose polls end only with other CTAs' lane phases)
+        if (cand) {
+            const unsigned long long *pb = &W.hbase[(size_t)pre_sa * G + cta];
+            unsigned long long v = ld_relaxed_u64(pb);
+            while ((uint32_t)(v >> 33) != epoch) v = ld_relaxed_u64(pb);
+            const unsigned long long q = (v & ((1ull << 33) - 1ull)) + 1ull + rank;
+            L.seq[j] = q <= 0xffffffffull ? (uint32_t)q : 0u;   // RFC 4303 §3.3.3: never cycle
+        }
+        __syncthreads();
+        if (tr && lane == 0) atomicMax(&tr[7], gtimer());
+        const uint32_t q32 = (sa_me != INVALID_SA) ? L.seq[pk] : 0u;
+        const bool ok = q32 != 0u;   // a valid sequence number is never 0
+        // 6. the lane's packet
+        if (have) {
+            const uint32_t pkt = p_begin + pk;
+            if (ok) {
+                esp_packet(T, B, L, H, lane4r, tid, sa_me, info, q32, inoff, L.outoff[pk], pp,
+                           (tr && blockIdx.x == 0 && (tid == 0 || tid == cnt_pk - 1u))
+                               ? W.trace + 148 * 8 + 8 + (tid == 0 ? 0 : 8) : nullptr);
+                const uint32_t Dp = info & 0x7ffu;
+                const uint32_t Lp = 48u + esp_C(Dp);
+                B.out_len[pkt] = (uint16_t)Lp;
+                c_ok++;
+                c_in += Dp;
+                c_out += Lp;
+            } else {
+                B.out_len[pkt] = 0;
+                c_drop++;
+            }
+        }
+        if (tr && lane == 0) atomicMax(&tr[3], gtimer());
+    } else {
     for (uint32_t base = p_begin; base < p_end; base += F_SUPER) {
         const uint32_t cnt_pk = min((uint32_t)F_SUPER, p_end - base);
         // ---- 1. metadata (thread j <-> packet base + j) ---------------------
@@ -335,49 +460,29 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
         uint32_t sa = INVALID_SA, D = 0, inoff = 0, tos = 0;
         bool cand = false;
         if (j < cnt_pk) {
-            if (MERGED) {
-                sa = pre_sa;
-                D = pre_D;
-                inoff = pre_inoff;
-                L.outoff[j] = pre_outoff;
-            } else {
-                sa = B.sa_idx[i];
-                D = B.in_len[i];
-                inoff = B.in_off[i];
-                L.outoff[j] = B.out_off[i];
-            }
+            sa = B.sa_idx[i];
+            D = B.in_len[i];
+            inoff = B.in_off[i];
+            L.outoff[j] = B.out_off[i];
             cand = sa < n_sa && D >= MIN_D && D <= MAX_D;
-            if (cand && !MERGED) tos = B.in_buf[inoff + 1];
-            // merged: the lane reads the payload after the prologue; start the
-            // DRAM -> L2 transfer of its first line now
-            if (cand && MERGED) prefetch_l2(B.in_buf + inoff);
+            if (cand) tos = B.in_buf[inoff + 1];
         }
-        uint32_t rank = 0;
-        if (MERGED) {
-            // the prologue, in this kernel (single super-round per CTA)
-            rank = merged_prologue(T, W, L, cand ? sa : INVALID_SA, bar_base, epoch, tr);
-        } else if (base == p_begin) {
+        if (base == p_begin) {
             // Programmatic dependent launch: the prologue kernel's outputs (ranks,
             // per-SA prefixes, seq_prev) are complete and visible after this.
             asm volatile("griddepcontrol.wait;" ::: "memory");
         }
         // 1b. sequence number, drop decision, length bin
+        uint32_t bin = NBINS - 1;
         if (j < cnt_pk) {
-            uint32_t info = 0, bin = NBINS - 1, q32 = 0;
+            uint32_t info = 0, q32 = 0;
             if (cand) {
-                unsigned long long q;
-                if (MERGED) {
-                    const unsigned long long *pb = &W.hbase[(size_t)sa * gridDim.x + blockIdx.x];
-                    unsigned long long v = ld_relaxed_u64(pb);
-                    while ((uint32_t)(v >> 33) != epoch) v = ld_relaxed_u64(pb);
-                    q = (v & ((1ull << 33) - 1ull)) + 1ull + rank;
-                } else {
-                    q = (unsigned long long)T.seq_prev[sa] + 1ull +
-                        W.hpfx[(size_t)sa * ((B.n + PTILE - 1) / PTILE) + i / PTILE] + W.lrank[i];
-                }
+                const unsigned long long q =
+                    (unsigned long long)T.seq_prev[sa] + 1ull +
+                    W.hpfx[(size_t)sa * ((B.n + PTILE - 1) / PTILE) + i / PTILE] + W.lrank[i];
                 if (q <= 0xffffffffull) {   // RFC 4303 §3.3.3: never cycle
                     q32 = (uint32_t)q;
-                    info = D | (tos << 16) | INFO_OK | (MERGED ? INFO_TOSLOAD : 0u);
+                    info = D | (tos << 16) | INFO_OK;
                     bin = hmac_bin(true, esp_C(D));
                 }
             }
@@ -387,24 +492,7 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
             L.inoff[j] = inoff;
             atomicAdd(&L.bins[bin], 1u);
         }
-        __syncthreads();   // also publishes the T-tables on the first round
-        if (warp == 0) {   // exclusive scan of the 32 bin counts -> bin cursors
-            uint32_t cb = L.bins[lane], x = cb;
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-                if (lane >= (uint32_t)o) x += y;
-            }
-            L.bins[lane] = x - cb;
-        }
-        __syncthreads();
-        if (j < cnt_pk) {
-            const uint32_t info = L.info[j];
-            const uint32_t bin = (info & INFO_OK) ? hmac_bin(true, esp_C(info & 0x7ffu)) : NBINS - 1;
-            L.perm[atomicAdd(&L.bins[bin], 1u)] = (uint16_t)j;
-        }
-        __syncthreads();
-        if (tid < NBINS) L.bins[tid] = 0;   // next round's counts (after its barrier)
+        length_sort(L, j, cnt_pk, bin);   // also publishes the T-tables on the first round
         if (tr && tid == 0 && base == p_begin) tr[1] = gtimer();
 
         // ---- 2. one lane per packet, length-sorted so a warp's lanes do equal
@@ -416,14 +504,13 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
             const uint32_t info = have ? L.info[pk] : 0u;
             const uint32_t pkt = base + pk;
             const uint32_t sa_me = (info & INFO_OK) ? L.sa[pk] : INVALID_SA;
-            // warp-cooperative, coalesced staging of round keys 3..10
-            stage_round_keys(T.rk, L, H, sa_me, warp, lane);
-            __syncwarp();
             if (tr && tid == 0) tr[7] = gtimer();
             if (!have) {
             } else if (info & INFO_OK) {
-                esp_packet(T, B, L, H, lane4r, tid, L.sa[pk], info, L.seq[pk], L.inoff[pk],
-                           L.outoff[pk],
+                PktPre pp = load_pkt_pre(T, B.in_buf, sa_me, L.inoff[pk], false, (info >> 16) & 0xffu);
+                expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
+                esp_packet(T, B, L, H, lane4r, tid, sa_me, info, L.seq[pk], L.inoff[pk],
+                           L.outoff[pk], pp,
                            (tr && blockIdx.x == 0 && (tid == 0 || tid == cnt_pk - 1u))
                                ? W.trace + 148 * 8 + 8 + (tid == 0 ? 0 : 8) : nullptr);
                 const uint32_t Dp = info & 0x7ffu;
@@ -439,6 +526,7 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
         }
         if (tr && lane == 0) atomicMax(&tr[3], gtimer());
         __syncthreads();   // shared metadata is reused by the next super-round
+    }
     }
     // counters: warp sums, then one 64-bit atomic per CTA and counter
     const uint32_t s0 = __reduce_add_sync(0xffffffffu, c_ok);

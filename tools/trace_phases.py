@@ -32,12 +32,18 @@ for cfg in [int(x) for x in sys.argv[1:] if x.isdigit()] or (2, 3, 4):
           ((pro[1] - t0) / 1e3, (pro[2] - t0) / 1e3, (pro[3] - t0) / 1e3))
     rel = (tr - t0) / 1000.0
     names = ["start", "meta_done", "tables_done", "lanes_done", "m_tiles_done", "m_bar1_done",
-             "m_scans_done", "keys_staged(tid0)"]
+             "m_scans_done", "keys_staged(tid0) / polls done (merged)"]
     print(f"config {cfg} ({c['name']}), {live.sum()} CTAs, times in us from the prologue's first "
           f"CTA start{' (L2 flushed before the batch)' if FLUSH else ''}")
     for k, nm in enumerate(names):
         col = rel[:, k]
         print(f"  {nm:12s} min {col.min():8.2f}  med {np.median(col):8.2f}  max {col.max():8.2f}")
+    ld = rel[:, 3]
+    print("  lanes_done percentiles:", np.percentile(ld, [10, 25, 50, 75, 90, 95, 99]).round(1))
+    idx = np.nonzero(live)[0]
+    order = np.argsort(-ld)[:8]
+    print("  slowest CTAs (index: lanes_done / meta_done us):",
+          ", ".join(f"{idx[k]}: {ld[k]:.1f}/{rel[k, 1]:.1f}/polls {rel[k, 7]:.1f}" for k in order))
     from paper_conf_eurosys_kimjlmsm15_b200 import nba_ipsec as nbm
     import ctypes
     raw = np.zeros(148 * 8 + 64, np.uint64)
