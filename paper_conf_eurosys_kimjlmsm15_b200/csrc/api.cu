@@ -215,6 +215,7 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
         line[2] = hm[(size_t)s * 3 + 0];
         line[3] = hm[(size_t)s * 3 + 1];
         line[4] = hm[(size_t)s * 3 + 2];
+        line[5] = make_uint4(hout[0], hout[1], hout[2], 0u);   // words 4..5 = hout[3,4,-,-,0,1,2]
     }
     t->seq0 = seq;
 

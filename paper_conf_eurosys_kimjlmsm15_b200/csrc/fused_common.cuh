@@ -43,6 +43,7 @@ static_assert(sizeof(FusedLo) <= F_TOFF_MAX, "FusedLo must fit below the tables"
 static_assert(F_SMEM <= 232448, "exceeds 227 KB of shared memory per block");
 
 // -------------------------------------------------------------------- helpers
+
 __device__ __forceinline__ uint32_t smem_u32(const void *p)
 {
     return (uint32_t)__cvta_generic_to_shared(p);
@@ -54,6 +55,24 @@ __device__ __forceinline__ uint32_t lds_abs(uint32_t a)
     uint32_t v;
     asm volatile("ld.shared.u32 %0, [%1+%2];" : "=r"(v) : "r"(a), "n"(OFF));
     return v;
+}
+
+// Warp-aggregated shared-memory counter increment: the lanes of a warp with
+// the same key add together (one atomic per distinct key; 448 same-bin packets
+// of a CTA otherwise serialise on one shared address), returning each lane's
+// slot = old value + its rank among its peers.  All 32 lanes call it; lanes
+// with active == false take no part.
+__device__ __forceinline__ uint32_t warp_agg_add(uint32_t *ctr, uint32_t key, bool active)
+{
+    const uint32_t k = active ? key : 0xffffffffu;
+    const uint32_t peers = __match_any_sync(0xffffffffu, k);
+    const uint32_t leader = __ffs(peers) - 1;
+    uint32_t lt;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(lt));
+    uint32_t base = 0;
+    if (active && (threadIdx.x & 31u) == leader) base = atomicAdd(&ctr[key], (uint32_t)__popc(peers));
+    base = __shfl_sync(0xffffffffu, base, leader);
+    return base + __popc(peers & lt);
 }
 
 // T-table lookup: table `tbl`, row `row` of state word `reg`; lane4r holds

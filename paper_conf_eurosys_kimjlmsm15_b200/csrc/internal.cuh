@@ -36,8 +36,9 @@ struct DevTable {
     const uint32_t *te0;    // [256] T-table, row-0 byte in bits 0..7
     uint32_t n_sa;
     const uint4 *sal;       // [n_sa * SAL_U4] one 128-byte line per SA: AES key (round
-                            //   key 0), sahdr, hmid[0..2] -- what an outbound lane
-                            //   loads (it expands round keys 1..10 itself)
+                            //   key 0), sahdr, hmid[0..2], {hout[0..2], 0} -- what an
+                            //   outbound lane loads, as three 256-bit loads (it
+                            //   expands round keys 1..10 itself)
 };
 constexpr uint32_t SAL_U4 = 8;   // uint4s per SA line (5 used)
 
@@ -235,6 +236,15 @@ __device__ __forceinline__ uint4 extract16(uint4 lo, uint4 hi, uint32_t sh)
     return o;
 }
 
+// 32 bytes (32-B aligned) in one 256-bit load (sm_100: LDG.E.ENL2.256)
+__device__ __forceinline__ void ldg_nc_v8(const void *p, uint4 &a, uint4 &b)
+{
+    asm volatile("ld.global.nc.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(a.x), "=r"(a.y), "=r"(a.z), "=r"(a.w), "=r"(b.x), "=r"(b.y), "=r"(b.z),
+                   "=r"(b.w)
+                 : "l"(p));
+}
+
 __device__ __forceinline__ uint4 ldg_nc_v4(const void *p)
 {
     uint4 v;
@@ -325,14 +335,27 @@ __device__ __forceinline__ void grid_sync_mono(uint32_t *count, uint32_t target)
 // The same barrier in two halves, so a CTA can issue independent loads between
 // its arrival and the wait: grid_arrive after a __syncthreads that orders the
 // CTA's prior global writes; grid_wait ends with a __syncthreads.
+#ifndef NBA_ARRIVE_RELEASE
+#define NBA_ARRIVE_RELEASE 1
+#endif
 __device__ __forceinline__ void grid_arrive(uint32_t *count)
 {
     if (threadIdx.x == 0) {
-        __threadfence();
-        atomicAdd(count, 1u);
+        if (NBA_ARRIVE_RELEASE) {
+            // release RMW: orders the CTA's prior writes (made visible to this
+            // thread by the preceding __syncthreads) before the arrival, without
+            // the full fence's wait for everything in flight
+            asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(count) : "memory");
+        } else {
+            __threadfence();
+            atomicAdd(count, 1u);
+        }
     }
 }
 
+#ifndef NBA_WAIT_FENCE
+#define NBA_WAIT_FENCE 0
+#endif
 __device__ __forceinline__ void grid_wait(const uint32_t *count, uint32_t target)
 {
     if (threadIdx.x == 0) {
@@ -340,7 +363,9 @@ __device__ __forceinline__ void grid_wait(const uint32_t *count, uint32_t target
         do {
             asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(count) : "memory");
         } while ((int)(v - target) < 0);
-        __threadfence();
+        // the acquire load orders what follows; no trailing fence, which would
+        // also wait for every load this thread still has in flight
+        if (NBA_WAIT_FENCE) __threadfence();
     }
     __syncthreads();
 }

@@ -40,6 +40,12 @@ namespace nba {
 #ifndef NBA_INTERIOR          // 1: select-free fast path for interior 64-byte steps / SHA blocks
 #define NBA_INTERIOR 1
 #endif
+#ifndef NBA_EXPAND_MID        // merged: expand round keys after the row scans (1) or before the barrier wait (0)
+#define NBA_EXPAND_MID 0
+#endif
+#ifndef NBA_POLL_NS           // back-off between polls of a sequence-number base (ns)
+#define NBA_POLL_NS 0
+#endif
 #ifndef NBA_SA_PREFETCH       // L2 prefetch of the SA table at kernel start
 #define NBA_SA_PREFETCH 1
 #endif
@@ -61,10 +67,8 @@ __device__ __forceinline__ PktPre load_pkt_pre(const DevTable &T, const uint8_t 
 {
     PktPre p;
     const uint4 *line = T.sal + (size_t)sa * SAL_U4;
-    p.r0 = __ldg(&line[0]);
-    p.hd = __ldg(&line[1]);
-    p.h0 = __ldg(&line[2]);
-    p.h1 = __ldg(&line[3]);
+    ldg_nc_v8(&line[0], p.r0, p.hd);
+    ldg_nc_v8(&line[2], p.h0, p.h1);
     p.r1 = p.r2 = make_uint4(0, 0, 0, 0);
     // TOS of the inner header (the outer header copies it, reading A13)
     p.tos = load_tos ? (uint32_t)__ldg(in_buf + inoff + 1) : tos;
@@ -207,9 +211,9 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
 #pragma unroll
             for (int i = 6; i < 15; i++) W[i] = 0u;
             W[15] = (64u + 20u) * 8u;
-            const uint4 g1 = __ldg(&T.sal[(size_t)sa * SAL_U4 + 3]);
-            const uint4 g2 = __ldg(&T.sal[(size_t)sa * SAL_U4 + 4]);
-            st[0] = g1.y; st[1] = g1.z; st[2] = g1.w; st[3] = g2.x; st[4] = g2.y;
+            uint4 g4, g5;   // {hout[3], hout[4], -, -}, {hout[0], hout[1], hout[2], 0}
+            ldg_nc_v8(&T.sal[(size_t)sa * SAL_U4 + 4], g4, g5);
+            st[0] = g5.x; st[1] = g5.y; st[2] = g5.z; st[3] = g4.x; st[4] = g4.y;
         }
         sha1_compress_fma(st, W, T.n_sa != 0u ? 1u : 0u);   // (n_sa >= 1: an opaque 1)
         if (it == 0) ck_sha = clock64();
@@ -296,7 +300,8 @@ __device__ __forceinline__ void length_sort(FusedLo &L, uint32_t j, uint32_t cnt
         L.bins[lane] = x - cb;
     }
     __syncthreads();
-    if (j < cnt_pk) L.perm[atomicAdd(&L.bins[bin], 1u)] = (uint16_t)j;
+    const uint32_t pos = warp_agg_add(L.bins, bin, j < cnt_pk);
+    if (j < cnt_pk) L.perm[pos] = (uint16_t)j;
     __syncthreads();
     if (tid < NBINS) L.bins[tid] = 0;   // next round's counts (after its barrier)
 }
@@ -326,19 +331,14 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
     const uint32_t lane4r = (lane * 4u) | (smem_u32(tabs) & 0xffff0000u);
 
 #if NBA_SA_PREFETCH
-    // warm L2 with the SA table (round keys, midstates, header words) while the
-    // prologue runs: each CTA prefetches a slice of the 128-byte lines
+    // warm L2 with the SA table (SA lines and counters) while the prologue
+    // runs: each CTA prefetches a slice of the 128-byte lines
     {
-        const uint32_t nl_rk = (T.n_sa * 176u + 127u) >> 7;
-        const uint32_t nl_hm = (T.n_sa * 48u + 127u) >> 7;
-        const uint32_t nl_hd = (T.n_sa * 16u + 127u) >> 7;
-        const uint32_t nl = nl_rk + nl_hm + nl_hd;
-        for (uint32_t l = blockIdx.x * blockDim.x + tid; l < nl; l += gridDim.x * blockDim.x) {
-            const uint8_t *a = l < nl_rk ? reinterpret_cast<const uint8_t *>(T.rk) + 128u * l
-                             : l < nl_rk + nl_hm ? reinterpret_cast<const uint8_t *>(T.hmid) + 128u * (l - nl_rk)
-                                                 : reinterpret_cast<const uint8_t *>(T.sahdr) + 128u * (l - nl_rk - nl_hm);
-            prefetch_l2(a);
-        }
+        const uint32_t nl_sal = T.n_sa;                        // one line per SA
+        const uint32_t nl = nl_sal + ((T.n_sa * 4u + 127u) >> 7);
+        for (uint32_t l = blockIdx.x * blockDim.x + tid; l < nl; l += gridDim.x * blockDim.x)
+            prefetch_l2(l < nl_sal ? reinterpret_cast<const uint8_t *>(T.sal + (size_t)l * SAL_U4)
+                                   : reinterpret_cast<const uint8_t *>(T.seq) + 128u * (l - nl_sal));
     }
 #endif
     const uint32_t p_begin = blockIdx.x * ppc;
@@ -353,6 +353,11 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
         pre_sa = B.sa_idx ? B.sa_idx[p_begin + tid]
                           : flow_lookup_one(B.flow_table, B.flow_mask, B.in_buf + pre_inoff, pre_D);
     }
+    // the SA counter this warp's row scan will start from (only that scan
+    // writes it, after the grid barrier)
+    uint32_t old0 = 0;
+    if (MERGED) old0 = scan_first_old(T, blockIdx.x * (F_THREADS / 32u) + warp,
+                                      gridDim.x * (F_THREADS / 32u), gridDim.x, lane);
     aes_tables_to_smem(tabs, T.te0);
     if (tr && tid == 0) tr[2] = gtimer();
     if (tid < 4) L.cnt[tid] = 0ull;
@@ -381,10 +386,10 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
             L.info[j] = cand ? (pre_D | INFO_OK) : 0u;
             L.inoff[j] = pre_inoff;
             L.outoff[j] = pre_outoff;
-            atomicAdd(&L.bins[bin], 1u);
             // the lane reads the payload after the barrier: DRAM -> L2 now
             if (cand) prefetch_l2(B.in_buf + pre_inoff);
         }
+        warp_agg_add(L.bins, bin, j < cnt_pk);
         // 1. CTA-local ranks and per-SA counts (the prologue's tile part)
         const uint32_t rank = merged_local_rank(W, L, cand ? pre_sa : INVALID_SA);
         if (j < cnt_pk) L.seq[j] = rank;
@@ -392,10 +397,9 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
         // 2. lane order: longest packets first (seq-overflow drops keep their bin)
         length_sort(L, j, cnt_pk, bin);   // ends with __syncthreads: counts written
         grid_arrive(&W.ctl[CTL_BAR_MONO]);
-        // 3. between arrival and wait: everything of the lane's packet that does
-        //    not depend on its sequence number -- round keys 3..10 to shared
-        //    memory, the SA words and TOS to registers; and the SA counter this
-        //    warp's row scan starts from
+        if (tr && tid == 0) tr[1] = gtimer();
+        // 3. between arrival and wait: issue the loads of the lane's SA line and
+        //    TOS byte (used after the barrier)
         const bool have = tid < cnt_pk;
         const uint32_t pk = have ? L.perm[tid] : 0u;
         const uint32_t info = have ? L.info[pk] : 0u;
@@ -404,17 +408,18 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
         PktPre pp = {};
         if (sa_me != INVALID_SA) {
             pp = load_pkt_pre(T, B.in_buf, sa_me, inoff, true, 0u);
-            expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
+            if (!NBA_EXPAND_MID) expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
         }
-        const uint32_t old0 = scan_first_old(T, cta * NW + warp, G * NW, G, lane);
         grid_wait(&W.ctl[CTL_BAR_MONO], bar_base + G);
         if (tr && tid == 0) tr[5] = gtimer();
         // 4. row scans publish epoch-tagged bases; each packet polls its own
         //    (SA, CTA) entry
         scan_all_columns<true>(T, W, cta * NW + warp, G * NW, G, lane, epoch, true, old0);
         if (tr && tid == 0) tr[6] = gtimer();
+        // round keys into shared memory: after the scans (nothing before the
+        // barrier waits for the SA line) and while the bases propagate
+        if (NBA_EXPAND_MID && sa_me != INVALID_SA) expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
         __syncwarp();
-        if (tr && tid == 0) tr[1] = gtimer();
         // 5. sequence numbers: thread j polls the published base of its packet's
         //    (SA, CTA) entry; all polls end before any lane starts its packet
         //    (measured: letting each warp start after its own polls leaves
@@ -422,7 +427,10 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
         if (cand) {
             const unsigned long long *pb = &W.hbase[(size_t)pre_sa * G + cta];
             unsigned long long v = ld_relaxed_u64(pb);
-            while ((uint32_t)(v >> 33) != epoch) v = ld_relaxed_u64(pb);
+            while ((uint32_t)(v >> 33) != epoch) {
+                if (NBA_POLL_NS) __nanosleep(NBA_POLL_NS);
+                v = ld_relaxed_u64(pb);
+            }
             const unsigned long long q = (v & ((1ull << 33) - 1ull)) + 1ull + rank;
             L.seq[j] = q <= 0xffffffffull ? (uint32_t)q : 0u;   // RFC 4303 §3.3.3: never cycle
         }
@@ -490,8 +498,8 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
             L.seq[j] = q32;
             L.info[j] = info;
             L.inoff[j] = inoff;
-            atomicAdd(&L.bins[bin], 1u);
         }
+        warp_agg_add(L.bins, bin, j < cnt_pk);
         length_sort(L, j, cnt_pk, bin);   // also publishes the T-tables on the first round
         if (tr && tid == 0 && base == p_begin) tr[1] = gtimer();
 

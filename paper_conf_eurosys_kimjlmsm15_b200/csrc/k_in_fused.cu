@@ -211,7 +211,10 @@ k_in_fused(DevTable T, InState S, InBatchArgs B, uint32_t ppc, uint32_t hmask)
             L.outoff[j] = B.out_off[i];
             L.aux0[j] = iv0;
             L.aux1[j] = iv1;
-            atomicAdd(&L.bins[info ? hmac_bin(true, info & 0xffffu) : NBINS - 1], 1u);
+        }
+        {
+            const uint32_t info = j < cnt_pk ? L.info[j] : 0u;
+            warp_agg_add(L.bins, info ? hmac_bin(true, info & 0xffffu) : NBINS - 1, j < cnt_pk);
         }
         __syncthreads();
         if (warp == 0) {
@@ -224,9 +227,11 @@ k_in_fused(DevTable T, InState S, InBatchArgs B, uint32_t ppc, uint32_t hmask)
             L.bins[lane] = x - cb;
         }
         __syncthreads();
-        if (j < cnt_pk) {
-            const uint32_t info = L.info[j];
-            L.perm[atomicAdd(&L.bins[info ? hmac_bin(true, info & 0xffffu) : NBINS - 1], 1u)] = (uint16_t)j;
+        {
+            const uint32_t info = j < cnt_pk ? L.info[j] : 0u;
+            const uint32_t pos = warp_agg_add(L.bins, info ? hmac_bin(true, info & 0xffffu) : NBINS - 1,
+                                              j < cnt_pk);
+            if (j < cnt_pk) L.perm[pos] = (uint16_t)j;
         }
         __syncthreads();
         if (tid < NBINS) L.bins[tid] = 0;

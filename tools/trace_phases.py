@@ -31,7 +31,7 @@ for cfg in [int(x) for x in sys.argv[1:] if x.isdigit()] or (2, 3, 4):
     print("prologue: first start 0, tiles done %.2f, last-CTA start %.2f, end %.2f us" %
           ((pro[1] - t0) / 1e3, (pro[2] - t0) / 1e3, (pro[3] - t0) / 1e3))
     rel = (tr - t0) / 1000.0
-    names = ["start", "meta_done", "tables_done", "lanes_done", "m_tiles_done", "m_bar1_done",
+    names = ["start", "meta_done/arrived(merged)", "tables_done", "lanes_done", "m_tiles_done", "m_bar1_done",
              "m_scans_done", "keys_staged(tid0) / polls done (merged)"]
     print(f"config {cfg} ({c['name']}), {live.sum()} CTAs, times in us from the prologue's first "
           f"CTA start{' (L2 flushed before the batch)' if FLUSH else ''}")
