@@ -550,6 +550,7 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
     __syncthreads();
     if (tid < 4 && L.cnt[tid]) atomicAdd(&W.counters[tid], L.cnt[tid]);
     if (tid == 4 && blockIdx.x == 0) atomicAdd(&W.counters[4], 1ull);
+    if (tr && tid == 0) atomicMax(W.trace + W.trace_pro + 48u, gtimer());   // CTA end
 }
 
 int fused_grid(int num_sms) { return num_sms; }

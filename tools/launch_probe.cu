@@ -52,5 +52,52 @@ int main()
                 printf("coop=%d flush=%d smem=%zu: %.2f us per empty launch\n", coop, flush, smem,
                        tot / 200 * 1000);
             }
+    // the same empty cooperative kernel as a one-node CUDA graph
+    for (int flush = 0; flush < 2; flush++) {
+        cudaStream_t st;
+        cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking);
+        cudaGraph_t g;
+        cudaGraphExec_t ge;
+        cudaStreamBeginCapture(st, cudaStreamCaptureModeGlobal);
+        {
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = dim3(148);
+            cfg.blockDim = dim3(512);
+            cfg.dynamicSmemBytes = SM;
+            cfg.stream = st;
+            cudaLaunchAttribute a[1];
+            a[0].id = cudaLaunchAttributeCooperative;
+            a[0].val.cooperative = 1;
+            cfg.attrs = a;
+            cfg.numAttrs = 1;
+            cudaLaunchKernelEx(&cfg, k_empty, (int *)nullptr);
+        }
+        cudaStreamEndCapture(st, &g);
+        cudaGraphInstantiate(&ge, g, 0);
+        float tot = 0;
+        for (int it = 0; it < 220; it++) {
+            if (flush) k_fill<<<592, 1024, 0, st>>>(buf, n);
+            cudaEventRecord(e0, st);
+            cudaGraphLaunch(ge, st);
+            cudaEventRecord(e1, st);
+            cudaEventSynchronize(e1);
+            float ms;
+            cudaEventElapsedTime(&ms, e0, e1);
+            if (it >= 20) tot += ms;
+        }
+        printf("graph coop=1 flush=%d smem=%zu: %.2f us per empty launch\n", flush, SM, tot / 200 * 1000);
+        // back-to-back events only (no kernel): the timing floor
+        tot = 0;
+        for (int it = 0; it < 220; it++) {
+            if (flush) k_fill<<<592, 1024, 0, st>>>(buf, n);
+            cudaEventRecord(e0, st);
+            cudaEventRecord(e1, st);
+            cudaEventSynchronize(e1);
+            float ms;
+            cudaEventElapsedTime(&ms, e0, e1);
+            if (it >= 20) tot += ms;
+        }
+        printf("events only flush=%d: %.2f us\n", flush, tot / 200 * 1000);
+    }
     return 0;
 }

@@ -54,7 +54,10 @@ for cfg in [int(x) for x in sys.argv[1:] if x.isdigit()] or (2, 3, 4):
     raw2 = np.zeros(148 * 8 + 64, np.uint64)
     nbm.lib.nba_ipsec_debug_trace(t._h, raw2.ctypes.data_as(ctypes.POINTER(ctypes.c_uint64)), raw2.size)
     G = int(live.sum()) if pro[0] == 0 else 148
-    wend = raw2[G * 8 + 32:G * 8 + 48].astype(np.int64)
+    kend = int(raw2[148 * 8 + 48])
+    if kend:
+        print("  kernel: last CTA end %.2f us after the first CTA start" % ((kend - t0) / 1e3))
+    wend = raw2[G * 8 + 32:G * 8 + 40].astype(np.int64)
     st0 = int(full[0, 0])
     print("  CTA 0 warp finish (us from its start):", " ".join(f"{(x - st0) / 1e3:.1f}" if x else "-" for x in wend))
     t.close()
