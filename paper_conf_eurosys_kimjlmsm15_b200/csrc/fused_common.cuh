@@ -29,6 +29,7 @@ struct FusedLo {
     unsigned long long cnt[4];
     uint32_t hkey[2 * F_SUPER];    // merged prologue: SA of each slot of the CTA's SA hash
     uint32_t hmask[2 * F_SUPER];   //   warps holding a group of that SA
+    uint8_t wrun[F_THREADS / 32];  // warp -> run of 32 sorted positions (0xff: none)
 };
 
 struct FusedHi {
@@ -230,6 +231,111 @@ struct OutStream {
     }
 };
 
+
+__device__ __forceinline__ void stg_v8(void *p, const uint32_t (&w)[8])
+{
+    asm volatile("st.global.v8.u32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "r"(w[0]), "r"(w[1]),
+                 "r"(w[2]), "r"(w[3]), "r"(w[4]), "r"(w[5]), "r"(w[6]), "r"(w[7])
+                 : "memory");
+}
+
+// Bytes [lo, hi) of the 32-byte image w[0..7] to chunk + [lo, hi); chunk 32-B aligned.
+__device__ __forceinline__ void store_chunk32_range(uint8_t *chunk, const uint32_t (&w)[8], uint32_t lo,
+                                                    uint32_t hi)
+{
+    if (lo == 0 && hi == 32) {
+        stg_v8(chunk, w);
+        return;
+    }
+    if (lo < 16) store_chunk_range(chunk, w[0], w[1], w[2], w[3], lo, hi < 16 ? hi : 16);
+    if (hi > 16) store_chunk_range(chunk + 16, w[4], w[5], w[6], w[7], lo > 16 ? lo - 16 : 0, hi - 16);
+}
+
+// OutStream with 32-byte destination chunks (256-bit stores): a 64-byte step
+// of ciphertext costs two store wavefronts per lane instead of four.
+struct OutStream32 {
+    uint8_t *cp;           // current 32-B aligned destination chunk
+    uint32_t a[8];
+    uint32_t p;            // next word position in the chunk (0..7)
+    uint32_t prev;         // previous output word (for the funnel shift)
+    uint32_t r;            // 8 * (e & 3)
+    uint32_t lo;           // first byte of the current chunk that is ours
+
+    __device__ __forceinline__ void init(uint8_t *dst)
+    {
+        const uintptr_t ad = reinterpret_cast<uintptr_t>(dst);
+        const uint32_t e = (uint32_t)(ad & 31u);
+        cp = reinterpret_cast<uint8_t *>(ad - e);
+#pragma unroll
+        for (int i = 0; i < 8; i++) a[i] = 0;
+        p = e >> 2;
+        prev = 0;
+        r = (e & 3u) * 8u;
+        lo = e;
+    }
+    __device__ __forceinline__ void place(uint32_t d)
+    {
+#pragma unroll
+        for (int i = 0; i < 8; i++) a[i] = p == (uint32_t)i ? d : a[i];
+    }
+    __device__ __forceinline__ void put(uint32_t v)
+    {
+        const uint32_t d = __funnelshift_l(prev, v, r);
+        prev = v;
+        place(d);
+        if (++p == 8) {
+            store_chunk32_range(cp, a, lo, 32);
+            cp += 32;
+            p = 0;
+            lo = 0;
+        }
+    }
+    // 16 words whose dest words start at chunk position p (any)
+    __device__ __forceinline__ void put16(const uint32_t (&v)[16])
+    {
+        uint32_t d[16];
+#pragma unroll
+        for (int i = 0; i < 16; i++) d[i] = __funnelshift_l(i ? v[i - 1] : prev, v[i], r);
+        prev = v[15];
+#define NBA_PUT16_32(P)                                                                        \
+    {                                                                                          \
+        uint32_t c[8];                                                                         \
+        _Pragma("unroll") for (int i = 0; i < 8; i++) c[i] = i < (P) ? a[i] : d[i - (P)];      \
+        store_chunk32_range(cp, c, lo, 32);                                                    \
+        uint32_t c2[8];                                                                        \
+        _Pragma("unroll") for (int i = 0; i < 8; i++) c2[i] = d[8 - (P) + i];                  \
+        stg_v8(cp + 32, c2);                                                                   \
+        cp += 64;                                                                              \
+        _Pragma("unroll") for (int i = 0; i < (P); i++) a[i] = d[16 - (P) + i];               \
+    }
+        switch (p) {
+        case 0: NBA_PUT16_32(0) break;
+        case 1: NBA_PUT16_32(1) break;
+        case 2: NBA_PUT16_32(2) break;
+        case 3: NBA_PUT16_32(3) break;
+        case 4: NBA_PUT16_32(4) break;
+        case 5: NBA_PUT16_32(5) break;
+        case 6: NBA_PUT16_32(6) break;
+        default: NBA_PUT16_32(7) break;
+        }
+#undef NBA_PUT16_32
+        lo = 0;
+    }
+    // after the last word: the spill-over dest word (if r) and the final partial chunk
+    __device__ __forceinline__ void finish(const uint8_t *end)
+    {
+        if (r) {
+            place(__funnelshift_l(prev, 0u, r));
+            if (++p == 8) {
+                const uint32_t hi = (uint32_t)(end - cp);
+                store_chunk32_range(cp, a, lo, hi < 32u ? hi : 32u);
+                return;
+            }
+        }
+        const intptr_t hi = end - cp;
+        if (hi > 0) store_chunk32_range(cp, a, lo, (uint32_t)hi);
+    }
+};
 
 // ---- AES-128-CTR for one lane's packet (FIPS-197 §5.1 with T-tables) -------
 // Counter block = n0 || iv0 || iv1 || BE32(k+1) (RFC 3686 §4; words are the
@@ -446,6 +552,66 @@ __device__ __forceinline__ void extract16(const Raw5 &r, uint32_t (&o)[16])
     default: NBA_PT_CASE(3) break;
     }
 #undef NBA_PT_CASE
+}
+
+// The same with three 256-bit loads of the 32-byte aligned blocks covering
+// [a, a + 64): fewer L1 data-pipe wavefronts per step (each lane's load touches
+// its own line, so a warp-wide load costs one wavefront per lane whatever its
+// width: 3 x 32 instead of 5 x 32).  Blocks starting at or past `end` are not
+// read; a block that is read never crosses a 4 KB page, so it cannot fault
+// where the datagram's own bytes do not.
+struct Raw6 {
+    uint4 c[6];
+    uint32_t sh;
+};
+
+__device__ __forceinline__ void load_raw6(uintptr_t a, uintptr_t end, Raw6 &r)
+{
+    const uintptr_t abase = a & ~(uintptr_t)31;
+    r.sh = (uint32_t)(a & 31u);
+    const uint4 z4 = make_uint4(0, 0, 0, 0);
+#pragma unroll
+    for (int i = 0; i < 3; i++) {
+        const uintptr_t qa = abase + 32u * i;
+        if (qa < end) ldg_nc_v8(reinterpret_cast<const void *>(qa), r.c[2 * i], r.c[2 * i + 1]);
+        else r.c[2 * i] = r.c[2 * i + 1] = z4;
+    }
+}
+
+__device__ __forceinline__ void load_raw6_inb(uintptr_t a, Raw6 &r)
+{
+    const uintptr_t abase = a & ~(uintptr_t)31;
+    r.sh = (uint32_t)(a & 31u);
+#pragma unroll
+    for (int i = 0; i < 3; i++)
+        ldg_nc_v8(reinterpret_cast<const void *>(abase + 32u * i), r.c[2 * i], r.c[2 * i + 1]);
+}
+
+__device__ __forceinline__ void extract16(const Raw6 &r, uint32_t (&o)[16])
+{
+    uint32_t v[24];
+#pragma unroll
+    for (int i = 0; i < 6; i++) {
+        v[4 * i] = r.c[i].x;
+        v[4 * i + 1] = r.c[i].y;
+        v[4 * i + 2] = r.c[i].z;
+        v[4 * i + 3] = r.c[i].w;
+    }
+    const uint32_t rr = (r.sh & 3u) * 8u;
+#define NBA_PT6_CASE(Q)                                                                   \
+    _Pragma("unroll") for (int w = 0; w < 16; w++) o[w] =                                 \
+        __funnelshift_r(v[(Q) + w], v[(Q) + w + 1], rr);
+    switch (r.sh >> 2) {
+    case 0: NBA_PT6_CASE(0) break;
+    case 1: NBA_PT6_CASE(1) break;
+    case 2: NBA_PT6_CASE(2) break;
+    case 3: NBA_PT6_CASE(3) break;
+    case 4: NBA_PT6_CASE(4) break;
+    case 5: NBA_PT6_CASE(5) break;
+    case 6: NBA_PT6_CASE(6) break;
+    default: NBA_PT6_CASE(7) break;
+    }
+#undef NBA_PT6_CASE
 }
 
 // Flow -> SA lookup of one inner datagram P (D bytes), readings F1..F4: one

@@ -46,6 +46,21 @@ namespace nba {
 #ifndef NBA_POLL_NS           // back-off between polls of a sequence-number base (ns)
 #define NBA_POLL_NS 0
 #endif
+#ifndef NBA_LDG256            // 1: payload steps as three 256-bit loads (else five 128-bit)
+#define NBA_LDG256 1
+#endif
+#ifndef NBA_CARRY             // 1: reuse the previous step's last 32-byte payload block
+#define NBA_CARRY 0
+#endif
+#ifndef NBA_STG256            // 1: output through 32-byte chunks (256-bit stores)
+#define NBA_STG256 0
+#endif
+#ifndef NBA_LPT               // 1: runs of 32 sorted packets to warps by LPT over sub-partitions
+#define NBA_LPT 1
+#endif
+#ifndef NBA_SMSP_BALANCE      // 1: spread a super-round's packets over all 16 warps
+#define NBA_SMSP_BALANCE 0
+#endif
 #ifndef NBA_SA_PREFETCH       // L2 prefetch of the SA table at kernel start
 #define NBA_SA_PREFETCH 1
 #endif
@@ -102,7 +117,11 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
     const CtrPre cp = ctr_precompute(lane4r, r0, r1, r2, hd.y, 0u, qbe);   // IV = BE64(q), A6
 
     // outer IPv4 header (reading A13) + ESP header + IV: output words 0..8
+#if NBA_STG256
+    OutStream32 os;
+#else
     OutStream os;
+#endif
     os.init(B.out_buf + outoff);
     {
         const uint32_t src = bswap32(hd.z), dst = bswap32(hd.w);
@@ -135,6 +154,7 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
 
     // ---- one SHA-1 compression per iteration; AES steps feed the first nsteps
 #pragma unroll 1
+    uint4 pcarry0 = make_uint4(0, 0, 0, 0), pcarry1 = pcarry0;   // NBA_CARRY: last payload block
     for (uint32_t it = 0; it <= nb_in; it++) {
         uint32_t ct[16];
 #pragma unroll
@@ -146,9 +166,39 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
             // when p = 3, the one before) lies beyond it, and the five 16-byte
             // loads are inside the datagram -- no per-word selects, one bounds test
             const bool interior = NBA_INTERIOR && 16u * it + 18u <= Cw;
+#if NBA_LDG256 && NBA_CARRY
+            // block 0 of this step is block 2 of the previous one (the stream
+            // advances 64 bytes = two 32-byte blocks per step): two new loads
+            Raw6 raw;
+            {
+                const uintptr_t a = reinterpret_cast<uintptr_t>(src) + 64u * it;
+                const uintptr_t abase = a & ~(uintptr_t)31;
+                raw.sh = (uint32_t)(a & 31u);
+                if (it == 0) {
+                    if (abase < src_end) ldg_nc_v8(reinterpret_cast<const void *>(abase), raw.c[0], raw.c[1]);
+                    else raw.c[0] = raw.c[1] = make_uint4(0, 0, 0, 0);
+                } else {
+                    raw.c[0] = pcarry0;
+                    raw.c[1] = pcarry1;
+                }
+#pragma unroll
+                for (int i = 1; i < 3; i++) {
+                    const uintptr_t qa = abase + 32u * i;
+                    if (interior || qa < src_end) ldg_nc_v8(reinterpret_cast<const void *>(qa), raw.c[2 * i], raw.c[2 * i + 1]);
+                    else raw.c[2 * i] = raw.c[2 * i + 1] = make_uint4(0, 0, 0, 0);
+                }
+                pcarry0 = raw.c[4];
+                pcarry1 = raw.c[5];
+            }
+#elif NBA_LDG256
+            Raw6 raw;
+            if (interior) load_raw6_inb(reinterpret_cast<uintptr_t>(src) + 64u * it, raw);
+            else load_raw6(reinterpret_cast<uintptr_t>(src) + 64u * it, src_end, raw);
+#else
             Raw5 raw;
             if (interior) load_raw5_inb(reinterpret_cast<uintptr_t>(src) + 64u * it, raw);
             else load_raw5(reinterpret_cast<uintptr_t>(src) + 64u * it, src_end, raw);
+#endif
             // AES-128 of counter blocks 4 it + 1 .. 4 it + 4
             uint32_t ks[16];
             aes4_keystream(lane4r, cp, it, L, H, tid, ks);
@@ -304,6 +354,62 @@ __device__ __forceinline__ void length_sort(FusedLo &L, uint32_t j, uint32_t cnt
     if (j < cnt_pk) L.perm[pos] = (uint16_t)j;
     __syncthreads();
     if (tid < NBINS) L.bins[tid] = 0;   // next round's counts (after its barrier)
+    if (NBA_LPT && warp == 0) {
+        // Runs of 32 sorted positions (one warp each) to warps: a warp costs
+        // about its longest lane (all lanes step together), and warp w issues
+        // on SM sub-partition w mod 4, so the runs go longest first to the
+        // least loaded sub-partition (LPT).  Equal costs: run r -> warp r.
+        constexpr uint32_t NW = F_THREADS / 32u;
+        const uint32_t nruns = (cnt_pk + 31u) / 32u;
+        uint32_t cost = 0;
+        if (lane < nruns) {
+            const uint32_t info = L.info[L.perm[32u * lane]];
+            const uint32_t C = esp_C(info & 0x7ffu);
+            cost = (info & INFO_OK) ? 8u * (esp_nsha_inner(C) + 1u) + 3u * ((C + 15u) >> 4) : 1u;
+        }
+        const uint32_t c0 = __shfl_sync(0xffffffffu, cost, 0);
+        if (__all_sync(0xffffffffu, lane >= nruns || cost == c0)) {
+            if (lane < NW) L.wrun[lane] = lane < nruns ? (uint8_t)lane : 0xffu;
+        } else {
+            uint32_t load[4] = {0u, 0u, 0u, 0u}, used[4] = {0u, 0u, 0u, 0u}, mine = 0xffu;
+            for (uint32_t r = 0; r < nruns; r++) {
+                const uint32_t cr = __shfl_sync(0xffffffffu, cost, r);
+                uint32_t best = 4u;
+#pragma unroll
+                for (uint32_t q = 0; q < 4u; q++)
+                    if (used[q] < NW / 4u && (best == 4u || load[q] < load[best])) best = q;
+                if (lane == best + 4u * used[best]) mine = r;
+                used[best]++;
+                load[best] += cr;
+            }
+            if (lane < NW) L.wrun[lane] = (uint8_t)mine;
+        }
+    }
+    if (NBA_LPT) __syncthreads();
+}
+
+// Lane -> position in the length-sorted order.  Default (NBA_LPT): warp w
+// takes run L.wrun[w] (32 positions) as placed by length_sort.  Measured and
+// kept off: NBA_SMSP_BALANCE, contiguous runs of ceil(cnt / 16) positions per
+// warp so all 16 warps get packets (its warps finish together, yet 1514 B is
+// 2% and 64 B 5% slower: the shared-memory / L1 data pipe is per SM, so the
+// sub-partition imbalance it removes was not the bound).
+__device__ __forceinline__ bool lane_position(const FusedLo &L, uint32_t cnt, uint32_t &pos)
+{
+    constexpr uint32_t NW = F_THREADS / 32u;
+    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+    if (NBA_LPT) {
+        const uint32_t r = L.wrun[warp];
+        pos = 32u * r + lane;
+        return r != 0xffu && pos < cnt;
+    }
+    if (!NBA_SMSP_BALANCE) {
+        pos = threadIdx.x;
+        return pos < cnt;
+    }
+    const uint32_t lw = (cnt + NW - 1u) / NW;
+    pos = warp * lw + lane;
+    return lane < lw && pos < cnt;
 }
 
 // ---------------------------------------------------------------- the kernel
@@ -400,8 +506,9 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
         if (tr && tid == 0) tr[1] = gtimer();
         // 3. between arrival and wait: issue the loads of the lane's SA line and
         //    TOS byte (used after the barrier)
-        const bool have = tid < cnt_pk;
-        const uint32_t pk = have ? L.perm[tid] : 0u;
+        uint32_t pos;
+        const bool have = lane_position(L, cnt_pk, pos);
+        const uint32_t pk = have ? L.perm[pos] : 0u;
         const uint32_t info = have ? L.info[pk] : 0u;
         const uint32_t sa_me = (info & INFO_OK) ? L.sa[pk] : INVALID_SA;
         const uint32_t inoff = have ? L.inoff[pk] : 0u;
@@ -443,8 +550,8 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
             const uint32_t pkt = p_begin + pk;
             if (ok) {
                 esp_packet(T, B, L, H, lane4r, tid, sa_me, info, q32, inoff, L.outoff[pk], pp,
-                           (tr && blockIdx.x == 0 && (tid == 0 || tid == cnt_pk - 1u))
-                               ? W.trace + 148 * 8 + 8 + (tid == 0 ? 0 : 8) : nullptr);
+                           (tr && blockIdx.x == 0 && (pos == 0 || pos == cnt_pk - 1u))
+                               ? W.trace + 148 * 8 + 8 + (pos == 0 ? 0 : 8) : nullptr);
                 const uint32_t Dp = info & 0x7ffu;
                 const uint32_t Lp = 48u + esp_C(Dp);
                 B.out_len[pkt] = (uint16_t)Lp;
@@ -456,7 +563,11 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
                 c_drop++;
             }
         }
-        if (tr && lane == 0) atomicMax(&tr[3], gtimer());
+        if (tr && lane == 0) {
+            const unsigned long long now = gtimer();
+            atomicMax(&tr[3], now);
+            if (blockIdx.x == 0) W.trace[W.trace_pro + 24u + warp] = now;   // CTA 0, per warp
+        }
     } else {
     for (uint32_t base = p_begin; base < p_end; base += F_SUPER) {
         const uint32_t cnt_pk = min((uint32_t)F_SUPER, p_end - base);
@@ -507,8 +618,9 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
         // work; the longest packets go to the LOWEST warps (measured on B200:
         // -2% at IMIX vs the highest warps, tools/ab_variants.py)
         {
-            const bool have = tid < cnt_pk;
-            const uint32_t pk = have ? L.perm[NBA_LONG_HIGH ? cnt_pk - 1u - tid : tid] : 0u;
+            uint32_t pos;
+            const bool have = lane_position(L, cnt_pk, pos);
+            const uint32_t pk = have ? L.perm[NBA_LONG_HIGH ? cnt_pk - 1u - pos : pos] : 0u;
             const uint32_t info = have ? L.info[pk] : 0u;
             const uint32_t pkt = base + pk;
             const uint32_t sa_me = (info & INFO_OK) ? L.sa[pk] : INVALID_SA;
@@ -519,8 +631,8 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
                 expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
                 esp_packet(T, B, L, H, lane4r, tid, sa_me, info, L.seq[pk], L.inoff[pk],
                            L.outoff[pk], pp,
-                           (tr && blockIdx.x == 0 && (tid == 0 || tid == cnt_pk - 1u))
-                               ? W.trace + 148 * 8 + 8 + (tid == 0 ? 0 : 8) : nullptr);
+                           (tr && blockIdx.x == 0 && (pos == 0 || pos == cnt_pk - 1u))
+                               ? W.trace + 148 * 8 + 8 + (pos == 0 ? 0 : 8) : nullptr);
                 const uint32_t Dp = info & 0x7ffu;
                 const uint32_t Lp = 48u + esp_C(Dp);
                 B.out_len[pkt] = (uint16_t)Lp;

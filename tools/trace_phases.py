@@ -57,7 +57,7 @@ for cfg in [int(x) for x in sys.argv[1:] if x.isdigit()] or (2, 3, 4):
     kend = int(raw2[148 * 8 + 48])
     if kend:
         print("  kernel: last CTA end %.2f us after the first CTA start" % ((kend - t0) / 1e3))
-    wend = raw2[G * 8 + 32:G * 8 + 40].astype(np.int64)
+    wend = raw2[148 * 8 + 24:148 * 8 + 40].astype(np.int64)
     st0 = int(full[0, 0])
     print("  CTA 0 warp finish (us from its start):", " ".join(f"{(x - st0) / 1e3:.1f}" if x else "-" for x in wend))
     t.close()
