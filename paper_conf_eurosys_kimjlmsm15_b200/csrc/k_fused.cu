@@ -55,12 +55,6 @@ namespace nba {
 #ifndef NBA_STG256            // 1: output through 32-byte chunks (256-bit stores)
 #define NBA_STG256 0
 #endif
-#ifndef NBA_LPT               // 1: runs of 32 sorted packets to warps by LPT over sub-partitions
-#define NBA_LPT 1
-#endif
-#ifndef NBA_SMSP_BALANCE      // 1: spread a super-round's packets over all 16 warps
-#define NBA_SMSP_BALANCE 0
-#endif
 #ifndef NBA_SA_PREFETCH       // L2 prefetch of the SA table at kernel start
 #define NBA_SA_PREFETCH 1
 #endif
@@ -332,84 +326,6 @@ __device__ __forceinline__ uint32_t merged_local_rank(const DevWork &W, FusedLo 
             W.hist16[(size_t)s * G + cta] = (uint16_t)(base + wcnt_me);
     }
     return rank;
-}
-
-// Counting sort of the super-round's packets by SHA-1 length (L.bins holds the
-// counts; `bin` is thread j's packet's bin): L.perm[position] = packet.
-__device__ __forceinline__ void length_sort(FusedLo &L, uint32_t j, uint32_t cnt_pk, uint32_t bin)
-{
-    const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
-    __syncthreads();
-    if (warp == 0) {   // exclusive scan of the 32 bin counts -> bin cursors
-        uint32_t cb = L.bins[lane], x = cb;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-            if (lane >= (uint32_t)o) x += y;
-        }
-        L.bins[lane] = x - cb;
-    }
-    __syncthreads();
-    const uint32_t pos = warp_agg_add(L.bins, bin, j < cnt_pk);
-    if (j < cnt_pk) L.perm[pos] = (uint16_t)j;
-    __syncthreads();
-    if (tid < NBINS) L.bins[tid] = 0;   // next round's counts (after its barrier)
-    if (NBA_LPT && warp == 0) {
-        // Runs of 32 sorted positions (one warp each) to warps: a warp costs
-        // about its longest lane (all lanes step together), and warp w issues
-        // on SM sub-partition w mod 4, so the runs go longest first to the
-        // least loaded sub-partition (LPT).  Equal costs: run r -> warp r.
-        constexpr uint32_t NW = F_THREADS / 32u;
-        const uint32_t nruns = (cnt_pk + 31u) / 32u;
-        uint32_t cost = 0;
-        if (lane < nruns) {
-            const uint32_t info = L.info[L.perm[32u * lane]];
-            const uint32_t C = esp_C(info & 0x7ffu);
-            cost = (info & INFO_OK) ? 8u * (esp_nsha_inner(C) + 1u) + 3u * ((C + 15u) >> 4) : 1u;
-        }
-        const uint32_t c0 = __shfl_sync(0xffffffffu, cost, 0);
-        if (__all_sync(0xffffffffu, lane >= nruns || cost == c0)) {
-            if (lane < NW) L.wrun[lane] = lane < nruns ? (uint8_t)lane : 0xffu;
-        } else {
-            uint32_t load[4] = {0u, 0u, 0u, 0u}, used[4] = {0u, 0u, 0u, 0u}, mine = 0xffu;
-            for (uint32_t r = 0; r < nruns; r++) {
-                const uint32_t cr = __shfl_sync(0xffffffffu, cost, r);
-                uint32_t best = 4u;
-#pragma unroll
-                for (uint32_t q = 0; q < 4u; q++)
-                    if (used[q] < NW / 4u && (best == 4u || load[q] < load[best])) best = q;
-                if (lane == best + 4u * used[best]) mine = r;
-                used[best]++;
-                load[best] += cr;
-            }
-            if (lane < NW) L.wrun[lane] = (uint8_t)mine;
-        }
-    }
-    if (NBA_LPT) __syncthreads();
-}
-
-// Lane -> position in the length-sorted order.  Default (NBA_LPT): warp w
-// takes run L.wrun[w] (32 positions) as placed by length_sort.  Measured and
-// kept off: NBA_SMSP_BALANCE, contiguous runs of ceil(cnt / 16) positions per
-// warp so all 16 warps get packets (its warps finish together, yet 1514 B is
-// 2% and 64 B 5% slower: the shared-memory / L1 data pipe is per SM, so the
-// sub-partition imbalance it removes was not the bound).
-__device__ __forceinline__ bool lane_position(const FusedLo &L, uint32_t cnt, uint32_t &pos)
-{
-    constexpr uint32_t NW = F_THREADS / 32u;
-    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
-    if (NBA_LPT) {
-        const uint32_t r = L.wrun[warp];
-        pos = 32u * r + lane;
-        return r != 0xffu && pos < cnt;
-    }
-    if (!NBA_SMSP_BALANCE) {
-        pos = threadIdx.x;
-        return pos < cnt;
-    }
-    const uint32_t lw = (cnt + NW - 1u) / NW;
-    pos = warp * lw + lane;
-    return lane < lw && pos < cnt;
 }
 
 // ---------------------------------------------------------------- the kernel

@@ -28,7 +28,9 @@ __device__ __forceinline__ uint32_t esp_in_packet(const DevTable &T, const InBat
                                                   const FusedLo &L, const FusedHi &H,
                                                   uint32_t lane4r, uint32_t tid, uint32_t sa,
                                                   uint32_t C, uint32_t q32, uint32_t iv0,
-                                                  uint32_t iv1, uint32_t inoff, uint32_t outoff)
+                                                  uint32_t iv1, uint32_t inoff, uint32_t outoff,
+                                                  const uint4 &r0, const uint4 &r1, const uint4 &r2,
+                                                  const uint4 &hd, const uint4 &h0, const uint4 &h1)
 {
     const uint32_t Cw = C >> 2;                  // ciphertext words
     const uint32_t Mw = 4u + Cw;                 // MAC input words (ESP hdr + ciphertext)
@@ -36,21 +38,13 @@ __device__ __forceinline__ uint32_t esp_in_packet(const DevTable &T, const InBat
     const uint32_t nb_in = (4u * Mw + 8u) / 64u + 1u;   // inner SHA-1 blocks
     const uint32_t bitlen = (64u + 4u * Mw) * 8u;
 
-    const uint4 *rks = T.rk + (size_t)sa * 11u;
-    const uint4 r0 = __ldg(&rks[0]), r1 = __ldg(&rks[1]), r2 = __ldg(&rks[2]);
-    const uint4 hd = __ldg(&T.sahdr[sa]);
     const CtrPre cp = ctr_precompute(lane4r, r0, r1, r2, hd.y, iv0, iv1);
 
     OutStream os;
     os.init(B.out_buf + outoff);
     // SHA-1 message words 0..3 = SPI || seq || IV (big-endian words of the wire bytes)
     uint32_t carry[4] = {bswap32(hd.x), q32, bswap32(iv0), bswap32(iv1)};
-    uint32_t st[5];
-    {
-        const uint4 h0 = __ldg(&T.hmid[(size_t)sa * 3 + 0]);
-        const uint4 h1 = __ldg(&T.hmid[(size_t)sa * 3 + 1]);
-        st[0] = h0.x; st[1] = h0.y; st[2] = h0.z; st[3] = h0.w; st[4] = h1.x;
-    }
+    uint32_t st[5] = {h0.x, h0.y, h0.z, h0.w, h1.x};
     const uint8_t *src = B.in_buf + inoff + 36u;          // ciphertext E
     const uintptr_t src_end = reinterpret_cast<uintptr_t>(src) + C;
     if (C > 64u) prefetch_l2(src + 64);
@@ -64,19 +58,25 @@ __device__ __forceinline__ uint32_t esp_in_packet(const DevTable &T, const InBat
         for (int w = 0; w < 16; w++) ct[w] = 0u;
         if (it < nsteps) {
             if (64u * it + 192u < C) prefetch_l2(src + 64u * it + 192u);
-            Raw5 raw;
-            load_raw5(reinterpret_cast<uintptr_t>(src) + 64u * it, src_end, raw);
+            // interior step: the three 32-byte blocks lie inside E and the
+            // step holds neither of the last two plaintext words
+            const bool interior = 16u * it + 18u <= Cw;
+            Raw6 raw;
+            if (interior) load_raw6_inb(reinterpret_cast<uintptr_t>(src) + 64u * it, raw);
+            else load_raw6(reinterpret_cast<uintptr_t>(src) + 64u * it, src_end, raw);
             uint32_t ks[16];
             aes4_keystream(lane4r, cp, it, L, H, tid, ks);
             extract16(raw, ct);                  // ciphertext words (beyond C: ignored)
             uint32_t pt[16];
 #pragma unroll
             for (int w = 0; w < 16; w++) pt[w] = ct[w] ^ ks[w];
-            const uint32_t lw = Cw - 1u - 16u * it;
+            if (!interior) {
+                const uint32_t lw = Cw - 1u - 16u * it;
 #pragma unroll
-            for (int w = 0; w < 16; w++) {
-                if ((uint32_t)w == lw) lastw = pt[w];
-                if ((uint32_t)w + 1u == lw) prevw = pt[w];
+                for (int w = 0; w < 16; w++) {
+                    if ((uint32_t)w == lw) lastw = pt[w];
+                    if ((uint32_t)w + 1u == lw) prevw = pt[w];
+                }
             }
             if (16u * it + 16u <= Cw) {
                 os.put16(pt);
@@ -91,13 +91,18 @@ __device__ __forceinline__ uint32_t esp_in_packet(const DevTable &T, const InBat
         uint32_t W[16];
         if (it < nb_in) {
             const uint32_t m0 = 16u * it;
+            if (m0 + 16u <= Mw) {                     // a block of message words only
 #pragma unroll
-            for (int i = 0; i < 16; i++) {
-                const uint32_t m = m0 + i;
-                const uint32_t msg = i < 4 ? carry[i] : bswap32(ct[i - 4]);
-                W[i] = m < Mw ? msg : (m == Mw ? 0x80000000u : 0u);
+                for (int i = 0; i < 16; i++) W[i] = i < 4 ? carry[i] : bswap32(ct[i - 4]);
+            } else {                                  // FIPS 180-4 §5.1.1 padding
+#pragma unroll
+                for (int i = 0; i < 16; i++) {
+                    const uint32_t m = m0 + i;
+                    const uint32_t msg = i < 4 ? carry[i] : bswap32(ct[i - 4]);
+                    W[i] = m < Mw ? msg : (m == Mw ? 0x80000000u : 0u);
+                }
+                if (it == nb_in - 1u) W[15] = bitlen;
             }
-            if (it == nb_in - 1u) W[15] = bitlen;
 #pragma unroll
             for (int i = 0; i < 4; i++) carry[i] = bswap32(ct[12 + i]);
         } else {
@@ -107,9 +112,9 @@ __device__ __forceinline__ uint32_t esp_in_packet(const DevTable &T, const InBat
 #pragma unroll
             for (int i = 6; i < 15; i++) W[i] = 0u;
             W[15] = (64u + 20u) * 8u;
-            const uint4 h1 = __ldg(&T.hmid[(size_t)sa * 3 + 1]);
-            const uint4 h2 = __ldg(&T.hmid[(size_t)sa * 3 + 2]);
-            st[0] = h1.y; st[1] = h1.z; st[2] = h1.w; st[3] = h2.x; st[4] = h2.y;
+            uint4 g4, g5;   // {hout[3], hout[4], -, -}, {hout[0], hout[1], hout[2], 0}
+            ldg_nc_v8(&T.sal[(size_t)sa * SAL_U4 + 4], g4, g5);
+            st[0] = g5.x; st[1] = g5.y; st[2] = g5.z; st[3] = g4.x; st[4] = g4.y;
         }
         sha1_compress_fma(st, W, T.n_sa != 0u ? 1u : 0u);   // (n_sa >= 1: an opaque 1)
     }
@@ -212,44 +217,32 @@ k_in_fused(DevTable T, InState S, InBatchArgs B, uint32_t ppc, uint32_t hmask)
             L.aux0[j] = iv0;
             L.aux1[j] = iv1;
         }
-        {
-            const uint32_t info = j < cnt_pk ? L.info[j] : 0u;
-            warp_agg_add(L.bins, info ? hmac_bin(true, info & 0xffffu) : NBINS - 1, j < cnt_pk);
-        }
-        __syncthreads();
-        if (warp == 0) {
-            uint32_t cb = L.bins[lane], x = cb;
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-                if (lane >= (uint32_t)o) x += y;
-            }
-            L.bins[lane] = x - cb;
-        }
-        __syncthreads();
-        {
-            const uint32_t info = j < cnt_pk ? L.info[j] : 0u;
-            const uint32_t pos = warp_agg_add(L.bins, info ? hmac_bin(true, info & 0xffffu) : NBINS - 1,
-                                              j < cnt_pk);
-            if (j < cnt_pk) L.perm[pos] = (uint16_t)j;
-        }
-        __syncthreads();
-        if (tid < NBINS) L.bins[tid] = 0;
+        const uint32_t bin_j = (j < cnt_pk && L.info[j]) ? hmac_bin(true, L.info[j] & 0xffffu) : NBINS - 1;
+        warp_agg_add(L.bins, bin_j, j < cnt_pk);
+        length_sort(L, j, cnt_pk, bin_j);
 
-        // ---- 2. one lane per packet, longest packets in the highest warps ----
+        // ---- 2. one lane per packet, runs of length-sorted packets placed on
+        //         warps by length_sort (LPT over the SM sub-partitions) ----
         {
-            const bool have = tid < cnt_pk;
-            const uint32_t pk = have ? L.perm[cnt_pk - 1u - tid] : 0u;
+            uint32_t pos;
+            const bool have = lane_position(L, cnt_pk, pos);
+            const uint32_t pk = have ? L.perm[pos] : 0u;
             const uint32_t info = have ? L.info[pk] : 0u;
             const uint32_t sa_me = (info & INFO_OK) ? L.sa[pk] : INVALID_SA;
-            stage_round_keys(T.rk, L, H, sa_me, warp, lane);
-            __syncwarp();
             if (have) {
                 uint32_t flags = 0;
-                if (info & INFO_OK)
+                if (info & INFO_OK) {
+                    // the SA line (AES key, header words, inner midstate); round
+                    // keys 1..10 expanded in the lane
+                    uint4 r0, hd, h0, h1, r1, r2;
+                    const uint4 *line = T.sal + (size_t)sa_me * SAL_U4;
+                    ldg_nc_v8(&line[0], r0, hd);
+                    ldg_nc_v8(&line[2], h0, h1);
+                    expand_key_lane(lane4r, r0, r1, r2, L, H, tid);
                     flags = INF_FMT | esp_in_packet(T, B, L, H, lane4r, tid, sa_me, info & 0xffffu,
                                                     L.seq[pk], L.aux0[pk], L.aux1[pk], L.inoff[pk],
-                                                    L.outoff[pk]);
+                                                    L.outoff[pk], r0, r1, r2, hd, h0, h1);
+                }
                 S.flags[base + pk] = flags;
                 S.seq[base + pk] = L.seq[pk];
             }
