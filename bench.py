@@ -319,6 +319,7 @@ def run_ours(args):
         ctr = t.in_counters()
         ok_all = ctr["pkts_ok"] == ctr["batches"] * b.n
         same = bool(torch.equal(inner_len[:b.n].to(torch.int32), db.in_len[:b.n].to(torch.int32)))
+        in_launches = t.inbound_launches_per_batch()
         t.close()
         C = esp_len - 48
         w = {"packets": int(b.n), "aes_blocks": int(((C + 15) // 16).sum()),
@@ -332,7 +333,7 @@ def run_ours(args):
         kk = {k: v / max(nb, 1) for k, v in kern.items()}
         rr = {}
         for k, ms in kk.items():
-            if ms <= 0.0:            # in_decide runs inside in_replay (one-pass form)
+            if ms <= 0.0:            # one-kernel form: only in_fused (replay inside it)
                 continue
             if k == "in_fused":
                 x = kernel_roofline("fused", ms, w, peaks)
@@ -349,7 +350,7 @@ def run_ours(args):
                 "mpps": red["bytes_in"] * steps / sec / 1e6,
                 "ms_per_step": tot_max / steps, "steps": steps, "kernels": rr,
                 "all_accepted": bool(ok_all), "lengths_match_outbound_input": same,
-                "gpu_launches": 3 * steps}
+                "gpu_launches": in_launches * steps}
 
     def measure_flows(cfg_id, steps, warmup, n_flows=65536):
         """Flow -> SA lookup on the config's traffic rewritten to

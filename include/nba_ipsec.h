@@ -156,6 +156,11 @@ int nba_ipsec_set_pipeline(nba_ipsec_sa_table *t, int pipeline);
 /* Number of kernel launches the most recent process_batch call enqueued
  * (2 before the first call). */
 int nba_ipsec_launches_per_batch(nba_ipsec_sa_table *t);
+/* Number of kernel launches the most recent process_inbound call enqueued:
+ * 1 when n_pkts <= 512 x SM count (one cooperative kernel, the anti-replay
+ * decision behind two grid barriers inside it), else 3 (3 before the first
+ * call). */
+int nba_ipsec_inbound_launches_per_batch(nba_ipsec_sa_table *t);
 
 /* Per-kernel timing with CUDA events recorded on the caller's stream between
  * the kernels of each batch.  enable=1 starts (and resets) collection;

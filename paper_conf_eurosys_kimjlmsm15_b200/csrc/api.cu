@@ -74,6 +74,8 @@ struct nba_ipsec_sa_table {
     std::vector<uint32_t> seq0;     // the SAs' initial seq (window start, reading B6)
     bool in_enabled = false, in_gridsync = false;
     uint32_t in_hcap = 0;
+    uint32_t in_bar_base = 0;     // arrivals so far at the one-kernel inbound path's barriers
+    uint32_t in_last_launches = 3;
     InState S{};
     uint32_t *in_top0 = nullptr;              // the windows' initial state (reset)
     unsigned long long *in_bmp0 = nullptr;
@@ -569,6 +571,12 @@ int nba_ipsec_launches_per_batch(nba_ipsec_sa_table *t)
     return t->last_launches;
 }
 
+int nba_ipsec_inbound_launches_per_batch(nba_ipsec_sa_table *t)
+{
+    if (!t) return NBA_IPSEC_EINVAL;
+    return (int)t->in_last_launches;
+}
+
 int nba_ipsec_profile_enable(nba_ipsec_sa_table *t, int enable)
 {
     if (!t) return NBA_IPSEC_EINVAL;
@@ -724,8 +732,10 @@ int nba_ipsec_enable_inbound(nba_ipsec_sa_table *t)
     chk(dalloc(t, &S.flags, M));
     chk(dalloc(t, &S.seq, M));
     chk(dalloc(t, &S.lmax, M));
-    chk(dalloc(t, &S.hmax, (size_t)t->max_tiles * n_sa));
-    chk(dalloc(t, &S.pmx, (size_t)t->max_tiles * n_sa));
+    // columns: the three-kernel path's tiles, or the one-kernel path's CTAs
+    const size_t cols = std::max<size_t>(t->max_tiles, (size_t)t->grid_fused);
+    chk(dalloc(t, &S.hmax, cols * n_sa));
+    chk(dalloc(t, &S.pmx, cols * n_sa));
     chk(dalloc(t, &S.hkey, hcap));
     chk(dalloc(t, &S.hval, hcap));
     chk(dalloc(t, &S.counters, N_IN_COUNTERS));
@@ -783,8 +793,14 @@ int nba_ipsec_process_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batch *b
         if (ps) cudaEventRecord(ps->ev[ps->n_ev++], st);
     };
     mark();
-    if (launch_in_fused(t->T, t->S, B, t->grid_fused, hmask, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
+    // one kernel when the batch fits one super-round per CTA (the replay
+    // decision inside, behind two grid barriers); else three kernels
+    const bool merged = t->allow_merged && in_merged_ok(n, t->grid_fused);
+    t->in_last_launches = merged ? 1 : 3;
+    if (launch_in_fused(t->T, t->S, B, t->grid_fused, hmask, merged, &t->in_bar_base, st) != cudaSuccess)
+        return NBA_IPSEC_ECUDA;
     mark();
+    if (merged) return NBA_IPSEC_OK;
     if (launch_in_replay(t->T, t->S, B, n_tiles, hmask, t->in_gridsync, st) != cudaSuccess)
         return NBA_IPSEC_ECUDA;
     mark();
@@ -851,7 +867,7 @@ int nba_ipsec_profile_read_inbound(nba_ipsec_sa_table *t, double *ms, const char
         if (ms) ms[k] = t->prof_in_ms[k];
         if (names) names[k] = nm[k];
     }
-    if (n_kernels) *n_kernels = 3;
+    if (n_kernels) *n_kernels = (int)t->in_last_launches;
     if (n_batches) *n_batches = t->prof_in_batches;
     return NBA_IPSEC_OK;
 }

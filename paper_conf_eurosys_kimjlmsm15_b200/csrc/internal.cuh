@@ -170,7 +170,8 @@ cudaError_t setup_fused_attributes();
 int aes_grid(int num_sms);
 int fused_grid(int num_sms);
 cudaError_t launch_in_fused(const DevTable &T, const InState &S, const InBatchArgs &B, int grid,
-                            uint32_t hmask, cudaStream_t st);
+                            uint32_t hmask, bool merged, uint32_t *bar_base, cudaStream_t st);
+bool in_merged_ok(uint32_t n, int grid);
 cudaError_t launch_in_replay(const DevTable &T, const InState &S, const InBatchArgs &B,
                              uint32_t n_tiles, uint32_t hmask, bool gridsync, cudaStream_t st);
 cudaError_t launch_in_decide(const DevTable &T, const InState &S, const InBatchArgs &B,

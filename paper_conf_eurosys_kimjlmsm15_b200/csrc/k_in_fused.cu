@@ -21,6 +21,7 @@
 //   trailer: next header 4, pad length p with D = C - 2 - p >= 20, pad bytes 1..p.
 // Output: flags[i] = INF_FMT | INF_ICV | INF_TRL | D, seq[i].
 #include "fused_common.cuh"
+#include "in_replay.cuh"
 
 namespace nba {
 
@@ -145,8 +146,125 @@ __device__ __forceinline__ uint32_t esp_in_packet(const DevTable &T, const InBat
     return flags;
 }
 
+// ---- one-kernel inbound (n <= F_SUPER x grid): the anti-replay decision of
+// k_in_replay / k_in_decide inside this kernel, each CTA one tile of the
+// batch (its packets in batch order, thread j <-> packet p_begin + j):
+//   tile part: warp-segmented prefix max of the authenticated numbers by SA,
+//     merged across the 16 warps through a shared hash; per-SA tile maxima to
+//     the SA-major matrix;
+//   grid barrier; (sa, q) -> first-index hash inserts; one warp per SA scans
+//     its row (exclusive prefix max) and moves the window edge;
+//   grid barrier; per-packet decision, window bits, out_len, status, counters.
+// The same arithmetic as the three-kernel path (in_replay.cuh), so the same
+// result as the sequential receiver.
+constexpr uint32_t CTLI_BAR = 4;   // S.ctl word: monotonic barrier arrivals
+
+__device__ __forceinline__ void in_merged_tail(const DevTable &T, const InState &S, const InBatchArgs &B,
+                                               FusedLo &L, uint8_t *tabs, uint32_t p_begin,
+                                               uint32_t p_end, uint32_t hmask, uint32_t bar_base)
+{
+    constexpr uint32_t HS = 2u * F_SUPER, NW = F_THREADS / 32u;
+    __shared__ unsigned long long s_cnt[N_IN_COUNTERS - 1];
+    const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
+    const uint32_t G = gridDim.x, cta = blockIdx.x, n_sa = T.n_sa;
+    const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
+    const uint32_t j = tid, i = p_begin + j;
+    const bool live = j < cnt;
+    const uint32_t f = live ? L.aux1[j] : 0u;
+    const uint32_t sa = live ? L.sa[j] : INVALID_SA;
+    const uint32_t q = (f & INF_FMT) ? L.seq[j] : 0u;
+    const uint32_t key = (f & INF_FMT) ? sa : INVALID_SA;
+    const bool inA = (f & INF_ICV) != 0u;
+    const uint32_t qa = inA ? q : 0u;
+    for (uint32_t k = tid; k < HS; k += F_THREADS) {
+        L.hkey[k] = INVALID_SA;
+        L.hmask[k] = 0;
+    }
+    if (tid < N_IN_COUNTERS - 1) s_cnt[tid] = 0;
+    // per-warp group maxima, [HS][NW] u32 = 64 KB in the (now unused) T-tables
+    uint32_t(*gm)[NW] = reinterpret_cast<uint32_t(*)[NW]>(tabs);
+    const uint32_t peers = __match_any_sync(0xffffffffu, key);
+    const uint32_t lt = peers & lanemask_lt();
+    uint32_t mex = 0;                                // max over earlier lanes of the group
+#pragma unroll
+    for (int l = 0; l < 32; l++) {
+        const uint32_t v = __shfl_sync(0xffffffffu, qa, l);
+        if ((lt >> l) & 1u) mex = max(mex, v);
+    }
+    const uint32_t leader = __ffs(peers) - 1, hi_lane = 31u - __clz(peers);
+    const uint32_t gmax = __shfl_sync(0xffffffffu, max(mex, qa), hi_lane);
+    __syncthreads();   // CTA hash initialised, T-tables no longer read
+    uint32_t slot = 0;
+    if (key != INVALID_SA && lane == leader) {
+        slot = (key * 0x9E3779B1u) >> 22;           // 10 bits -> HS = 1024 slots
+        while (true) {
+            const uint32_t old = atomicCAS(&L.hkey[slot], INVALID_SA, key);
+            if (old == INVALID_SA || old == key) break;
+            slot = (slot + 1u) & (HS - 1u);
+        }
+        gm[slot][warp] = gmax;
+        atomicOr(&L.hmask[slot], 1u << warp);
+    }
+    slot = __shfl_sync(0xffffffffu, slot, leader);
+    __syncthreads();
+    uint32_t base = 0;
+    if (key != INVALID_SA) {
+        const uint32_t m = L.hmask[slot];
+#pragma unroll
+        for (uint32_t w = 0; w < NW; w++)
+            if (w < warp && ((m >> w) & 1u)) base = max(base, gm[slot][w]);
+        const uint32_t tmax = max(base, gmax);       // per-tile SA maximum, nonzero only
+        if ((m >> (warp + 1u)) == 0u && lane == hi_lane && tmax != 0u)
+            S.hmax[(size_t)key * G + cta] = tmax;
+    }
+    const uint32_t lmax = max(base, mex);
+    __syncthreads();
+    grid_arrive(&S.ctl[CTLI_BAR]);
+    grid_wait(&S.ctl[CTLI_BAR], bar_base + G);
+    // hash inserts (the hash was cleared before the barrier) and the row scans
+    if (inA) replay_hash_insert(S, key, q, i, hmask);
+    scan_all_rows(S, n_sa, cta * NW + warp, G * NW, G, lane);
+    __syncthreads();
+    grid_arrive(&S.ctl[CTLI_BAR]);
+    grid_wait(&S.ctl[CTLI_BAR], bar_base + 2u * G);
+    uint32_t st = 0xffu, D = 0, Lin = 0;
+    if (live) {
+        if (sa >= n_sa) {
+            st = ST_DROP_SA;
+        } else if (!(f & INF_FMT)) {
+            st = ST_DROP_FORMAT;
+        } else {
+            const uint32_t t0 = S.top_prev[sa];
+            const unsigned long long b0 = S.bmp_prev[sa];
+            const uint32_t tj = max(t0, max(S.pmx[(size_t)sa * G + cta], lmax));
+            st = replay_decide(S, sa, i, f, q, t0, b0, tj, S.top[sa], hmask);
+            if (st == ST_OK) {
+                D = f & 0xffffu;
+                Lin = B.in_len[i];
+            }
+        }
+        B.out_len[i] = (uint16_t)D;
+        if (B.status) B.status[i] = (uint8_t)st;
+    }
+    // counters: pkts_ok, drop_sa, drop_format, drop_replay, drop_auth,
+    // drop_trailer, bytes_in, bytes_out (+ batches by CTA 0)
+#pragma unroll
+    for (uint32_t k = 0; k < 6; k++) {
+        const uint32_t c = __reduce_add_sync(0xffffffffu, st == k ? 1u : 0u);
+        if (lane == 0 && c) atomicAdd(&s_cnt[k], (unsigned long long)c);
+    }
+    const uint32_t bi = __reduce_add_sync(0xffffffffu, Lin);
+    const uint32_t bo = __reduce_add_sync(0xffffffffu, D);
+    if (lane == 0 && bi) atomicAdd(&s_cnt[6], (unsigned long long)bi);
+    if (lane == 0 && bo) atomicAdd(&s_cnt[7], (unsigned long long)bo);
+    __syncthreads();
+    if (tid < N_IN_COUNTERS - 1 && s_cnt[tid]) atomicAdd(&S.counters[tid], s_cnt[tid]);
+    if (tid == 0 && cta == 0) atomicAdd(&S.counters[N_IN_COUNTERS - 1], 1ull);
+}
+
+template <bool MERGED>
 __global__ void __launch_bounds__(F_THREADS, 1)
-k_in_fused(DevTable T, InState S, InBatchArgs B, uint32_t ppc, uint32_t hmask)
+k_in_fused(DevTable T, InState S, InBatchArgs B, uint32_t ppc, uint32_t hmask, uint32_t bar_base)
 {
     extern __shared__ __align__(16) uint8_t smem[];
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
@@ -243,28 +361,57 @@ k_in_fused(DevTable T, InState S, InBatchArgs B, uint32_t ppc, uint32_t hmask)
                                                     L.seq[pk], L.aux0[pk], L.aux1[pk], L.inoff[pk],
                                                     L.outoff[pk], r0, r1, r2, hd, h0, h1);
                 }
-                S.flags[base + pk] = flags;
-                S.seq[base + pk] = L.seq[pk];
+                if (MERGED) {
+                    L.aux1[pk] = flags;                 // for the in-kernel replay decision
+                } else {
+                    S.flags[base + pk] = flags;
+                    S.seq[base + pk] = L.seq[pk];
+                }
             }
         }
         __syncthreads();
     }
+    if constexpr (MERGED) in_merged_tail(T, S, B, L, tabs, p_begin, p_end, hmask, bar_base);
 }
 
 cudaError_t launch_in_fused(const DevTable &T, const InState &S, const InBatchArgs &B, int grid,
-                            uint32_t hmask, cudaStream_t st)
+                            uint32_t hmask, bool merged, uint32_t *bar_base, cudaStream_t st)
 {
     uint32_t ppc = (B.n + grid - 1) / grid;
     ppc = (ppc + 31u) & ~31u;
     if (ppc < 32u) ppc = 32u;
     const uint32_t g = (B.n + ppc - 1) / ppc;
-    k_in_fused<<<g, F_THREADS, F_SMEM, st>>>(T, S, B, ppc, hmask);
-    return cudaGetLastError();
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(g);
+    cfg.blockDim = dim3(F_THREADS);
+    cfg.dynamicSmemBytes = F_SMEM;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeCooperative;   // grid barriers inside (merged)
+    attr[0].val.cooperative = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = merged ? 1 : 0;
+    const uint32_t bb = *bar_base;
+    cudaError_t e = merged ? cudaLaunchKernelEx(&cfg, k_in_fused<true>, T, S, B, ppc, hmask, bb)
+                           : cudaLaunchKernelEx(&cfg, k_in_fused<false>, T, S, B, ppc, hmask, bb);
+    if (e == cudaSuccess && merged) *bar_base = bb + 2u * g;
+    return e;
+}
+
+bool in_merged_ok(uint32_t n, int grid)
+{
+    uint32_t ppc = (n + grid - 1) / grid;
+    ppc = (ppc + 31u) & ~31u;
+    return ppc <= (uint32_t)F_SUPER;
 }
 
 cudaError_t setup_in_fused_attributes()
 {
-    return cudaFuncSetAttribute(k_in_fused, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)F_SMEM);
+    cudaError_t e = cudaFuncSetAttribute(k_in_fused<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)F_SMEM);
+    if (e != cudaSuccess) return e;
+    return cudaFuncSetAttribute(k_in_fused<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)F_SMEM);
 }
 
 }  // namespace nba

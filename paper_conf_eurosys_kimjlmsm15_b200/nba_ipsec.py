@@ -102,6 +102,7 @@ def _load():
         "nba_ipsec_strerror": (ctypes.c_char_p, [i32]),
         "nba_ipsec_set_pipeline": (i32, [vp, i32]),
         "nba_ipsec_launches_per_batch": (i32, [vp]),
+        "nba_ipsec_inbound_launches_per_batch": (i32, [vp]),
         "nba_ipsec_profile_enable": (i32, [vp, i32]),
         "nba_ipsec_profile_read": (i32, [vp, P(ctypes.c_double), P(ctypes.c_char_p), i32,
                                          P(i32), P(u32)]),
@@ -239,6 +240,9 @@ class SATable:
 
     def launches_per_batch(self) -> int:
         return int(lib.nba_ipsec_launches_per_batch(self._h))
+
+    def inbound_launches_per_batch(self) -> int:
+        return int(lib.nba_ipsec_inbound_launches_per_batch(self._h))
 
     def profile_enable(self, on: bool = True):
         _check(lib.nba_ipsec_profile_enable(self._h, 1 if on else 0), "nba_ipsec_profile_enable")
