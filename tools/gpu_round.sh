@@ -17,7 +17,7 @@ if [ "$2" == "full" ]; then
   done
   for C in 2 3 4; do
     timeout 900 ncu --set full --clock-control none --import-source on -k regex:'k_in_' \
-      -s 3 -c 3 -o gpurun_out/prof_${TAG}_in_c$C -f python tools/run_inbound.py --config $C --batches 3 > gpurun_out/ncu_${TAG}_in_c$C.log 2>&1
+      -s 2 -c 1 -o gpurun_out/prof_${TAG}_in_c$C -f python tools/run_inbound.py --config $C --batches 3 > gpurun_out/ncu_${TAG}_in_c$C.log 2>&1
   done
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:'k_(aes|hmac|gather|scatter)' \
       -s 4 -c 4 -o gpurun_out/prof_${TAG}_unfused_c3 -f python tools/run_batches.py --config 3 --batches 3 --pipeline 1 > /dev/null 2>&1

@@ -30,6 +30,7 @@ METRICS = [
     ("sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_active", "alu_pipe_pct"),
     ("sm__pipe_fma_cycles_active.avg.pct_of_peak_sustained_active", "fma_pipe_pct"),
     ("sm__inst_executed_pipe_lsu.avg.pct_of_peak_sustained_active", "lsu_inst_pct"),
+    ("l1tex__data_pipe_lsu_wavefronts.avg.pct_of_peak_sustained_elapsed", "l1_data_pipe_pct"),
     ("l1tex__data_pipe_lsu_wavefronts_mem_shared.sum", "shared_wavefronts"),
     ("l1tex__data_bank_conflicts_pipe_lsu_mem_shared.sum", "shared_bank_conflicts"),
     ("sm__warps_active.avg.pct_of_peak_sustained_active", "warps_active_pct"),
@@ -90,8 +91,8 @@ def main(tag):
         for d in rows:
             agg[d["kernel"]].append(d)
         lines += [f"## {name} (fused pipeline)", "",
-                  "| kernel | us | DRAM rd MB | DRAM wr MB | issue % | ALU % | FMA % | LSU % | smem wavefronts | bank conflicts | warp inst | regs |",
-                  "|---|---|---|---|---|---|---|---|---|---|---|---|"]
+                  "| kernel | us | DRAM rd MB | DRAM wr MB | issue % | ALU % | FMA % | LSU % | L1 data pipe % | smem wavefronts | bank conflicts | warp inst | regs |",
+                  "|---|---|---|---|---|---|---|---|---|---|---|---|---|"]
         for k, ds in agg.items():
             d = collections.defaultdict(lambda: float("nan"))
             d.update({m: (v if isinstance(v, float) else float("nan")) for m, v in ds[-1].items()
@@ -99,8 +100,8 @@ def main(tag):
             lines.append(
                 f"| {k} | {d['duration'] * 1e6:.1f} | {d['dram_read'] / 1e6:.2f} | {d['dram_write'] / 1e6:.2f} | "
                 f"{d['issue_active_pct']:.1f} | {d['alu_pipe_pct']:.1f} | {d['fma_pipe_pct']:.1f} | "
-                f"{d['lsu_inst_pct']:.1f} | {d['shared_wavefronts']:.3g} | {d['shared_bank_conflicts']:.3g} | "
-                f"{d['warp_instructions']:.3g} | {d['registers']:.0f} |")
+                f"{d['lsu_inst_pct']:.1f} | {d['l1_data_pipe_pct']:.1f} | {d['shared_wavefronts']:.3g} | "
+                f"{d['shared_bank_conflicts']:.3g} | {d['warp_instructions']:.3g} | {d['registers']:.0f} |")
             kj[f"{k}:{name}"] = {"dram_bytes_per_launch": d["dram_read"] + d["dram_write"],
                                  "ncu_duration_us": d["duration"] * 1e6,
                                  "source": os.path.basename(rep)}
@@ -109,15 +110,15 @@ def main(tag):
         rep = os.path.join(OUT, f"prof_{tag}_in_{c}.ncu-rep")
         if not os.path.exists(rep):
             continue
-        lines += [f"## {name} ESP inbound (k_in_fused -> k_in_replay -> k_in_decide)", "",
-                  "| kernel | us | DRAM rd MB | DRAM wr MB | issue % | ALU % | LSU % | warp inst | regs |",
-                  "|---|---|---|---|---|---|---|---|---|"]
+        lines += [f"## {name} ESP inbound (one kernel: k_in_fused<true>, replay decision inside)", "",
+                  "| kernel | us | DRAM rd MB | DRAM wr MB | issue % | ALU % | LSU % | L1 data pipe % | warp inst | regs |",
+                  "|---|---|---|---|---|---|---|---|---|---|"]
         for d0 in raw(rep):
             d = collections.defaultdict(lambda: float("nan"))
             d.update({m: (v if isinstance(v, float) else float("nan")) for m, v in d0.items()})
             lines.append(f"| {d0['kernel']} | {d['duration'] * 1e6:.1f} | {d['dram_read'] / 1e6:.2f} | "
                          f"{d['dram_write'] / 1e6:.2f} | {d['issue_active_pct']:.1f} | "
-                         f"{d['alu_pipe_pct']:.1f} | {d['lsu_inst_pct']:.1f} | "
+                         f"{d['alu_pipe_pct']:.1f} | {d['lsu_inst_pct']:.1f} | {d['l1_data_pipe_pct']:.1f} | "
                          f"{d['warp_instructions']:.3g} | {d['registers']:.0f} |")
             kj[f"{d0['kernel']}:{name}"] = {"dram_bytes_per_launch": d["dram_read"] + d["dram_write"],
                                             "ncu_duration_us": d["duration"] * 1e6,
