@@ -352,6 +352,93 @@ def run_ours(args):
                 "all_accepted": bool(ok_all), "lengths_match_outbound_input": same,
                 "gpu_launches": in_launches * steps}
 
+    def measure_alb(cfg_id, n_steps=1500, fixed_steps=20):
+        """Adaptive split on one GPU: two SA tables with all SAs
+        stand in for two devices -- device 0 runs the fused pipeline, device 1
+        the unfused one (a slower device, like NBA's CPU next to its GPU) --
+        on their own streams.  Every step routes one ingress batch of the
+        config by the owner map (route_pack_map), both devices process their
+        shares concurrently, the library's controller observes the step
+        (device time as its clock; paper parameters except a 1 ms update
+        interval and 64-sample history, so it converges within the bench)
+        and counters of moved SAs are handed over.  Reported: the trajectory
+        of w, the throughput of the last steps, fixed-split throughputs for
+        comparison, and the host cost of a hand-over and of one observation."""
+        from paper_conf_eurosys_kimjlmsm15_b200 import alb, redistribute
+        size = CFG_SIZE[cfg_id]
+        p, b = shard.rank_workload(cfg_id, PKTS_PER_GPU, size, N_SA_TOTAL, 0, 1, layout="packed")
+        n_sa = len(p.spi)
+        tabs = [nba_ipsec.SATable(p, device=local, max_batch=PKTS_PER_GPU) for _ in range(2)]
+        tabs[1].set_pipeline(nba_ipsec.PIPE_UNFUSED)
+        sts = [torch.cuda.Stream(device=dev) for _ in range(2)]
+        db = device.to_device(b, dev)
+        main = torch.cuda.current_stream()
+
+        def step(sa_map_t):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(main)
+            pk = redistribute.pack(db, b.n, n_sa, 2, sa_map=sa_map_t)
+            for d in range(2):
+                n, ioff, ilen, sa, ooff, olen, obuf = redistribute.local_views(pk, d)
+                sts[d].wait_stream(main)
+                with torch.cuda.stream(sts[d]):
+                    tabs[d].process(pk.buf, ioff, ilen, sa, obuf, ooff, olen, n=n, stream=sts[d])
+                main.wait_stream(sts[d])
+            e1.record(main)
+            e1.synchronize()
+            return e0.elapsed_time(e1), pk.counts
+
+        def map_tensor(sa_map):
+            return torch.from_numpy(sa_map.view(np.int32)).to(dev)
+
+        fixed = {}
+        for k in (0, 6, 12, 19, 25):
+            _, m = nba_ipsec.alb_assign(n_sa, 2, [k], 25)
+            mt = map_tensor(m)
+            for _ in range(3):
+                step(mt)
+            ms = sum(step(mt)[0] for _ in range(fixed_steps)) / fixed_steps
+            fixed[str(k)] = {"w": k / 25, "ms_per_step": ms, "mpps": b.n / (ms * 1e-3) / 1e6}
+        bal = alb.Balancer(n_sa, 2, history=64, update_ns=1_000_000)
+        owner, sa_map = bal.assignment()
+        mt = map_tensor(sa_map)
+        t_ns, traj, tail, ho_us, obs_ns = 0, [int(bal.node_step[0])], [], [], []
+        for j in range(n_steps):
+            ms, counts = step(mt)
+            t_ns += int(ms * 1e6)
+            if j >= n_steps - 200:
+                tail.append(ms)
+            h0 = time.perf_counter_ns()
+            ch = bal.observe(t_ns, [int(ms * 1e6)] * 2, counts)
+            obs_ns.append(time.perf_counter_ns() - h0)
+            if ch:
+                new_owner, new_map = bal.assignment()
+                h0 = time.perf_counter_ns()
+                alb.handover_tables(tabs, owner, new_owner)
+                ho_us.append((time.perf_counter_ns() - h0) / 1e3)
+                owner, sa_map = new_owner, new_map
+                mt = map_tensor(sa_map)
+                traj.append(int(bal.node_step[0]))
+        # the hand-over kept every SA's counter on its owner: packets per SA so far
+        live = np.where(owner == 0, tabs[0].sa_seq(), tabs[1].sa_seq())
+        for t in tabs:
+            t.close()
+        ms_tail = float(np.mean(tail))
+        best = max(fixed.values(), key=lambda v: v["mpps"])
+        return {"devices": "2 SA tables on one B200: device 0 fused pipeline, device 1 unfused "
+                           "(slower); shares run concurrently on two streams",
+                "workload": gen.CONFIGS[cfg_id]["name"] + " as one ingress batch per step",
+                "params": {"delta": 0.04, "history": 64, "update_ms": 1.0, "wait": [2, 32],
+                           "clock": "device time"},
+                "steps": n_steps, "updates": len(traj) - 1, "w_trajectory": [k / 25 for k in traj],
+                "w_final": traj[-1] / 25,
+                "last200": {"ms_per_step": ms_tail, "mpps": b.n / (ms_tail * 1e-3) / 1e6},
+                "fixed_split": fixed, "best_fixed_w": best["w"],
+                "alb_vs_best_fixed": (b.n / (ms_tail * 1e-3) / 1e6) / best["mpps"],
+                "handover_us_mean": float(np.mean(ho_us)) if ho_us else None,
+                "observe_ns_median": float(np.median(obs_ns)),
+                "packets_numbered": int(live.astype(np.int64).sum())}
+
     def measure_flows(cfg_id, steps, warmup, n_flows=65536):
         """Flow -> SA lookup on the config's traffic rewritten to
         n_flows registered 5-tuples (5% unknown): the lookup kernel alone, and
@@ -481,6 +568,11 @@ def run_ours(args):
         flows = {str(CFG_SIZE[main_cfg]): measure_flows(main_cfg, max(10, args.steps // 4),
                                                         max(3, args.warmup // 2))}
 
+    # ---- adaptive split across devices (one GPU: two tables) --------
+    alb_res = None
+    if world == 1 and not args.no_alb:
+        alb_res = measure_alb(main_cfg)
+
     # ---- CPU baseline: the oracle on host cores (rank 0, N = 1 only) ----------
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
@@ -519,6 +611,7 @@ def run_ours(args):
             "per_size": per_size,
             "inbound": inbound or None,
             "flow_lookup": flows,
+            "adaptive_split": alb_res,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": res["launches"],
@@ -669,6 +762,7 @@ def main():
     ap.add_argument("--no-sweep", action="store_true")
     ap.add_argument("--no-inbound", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-alb", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=3.0)
     args = ap.parse_args()
     if args.warmup < 3:

@@ -144,6 +144,12 @@ int nba_ipsec_read_counters(nba_ipsec_sa_table *t, nba_ipsec_counters *out, void
  * nba_ipsec_sa_params.seq for exact resume).  host_seq has n_sa entries.
  * Synchronises `cuda_stream`. */
 int nba_ipsec_read_sa_seq(nba_ipsec_sa_table *t, uint32_t *host_seq, void *cuda_stream);
+/* Overwrite the per-SA sequence numbers with host_seq[0..n_sa) (HOST memory):
+ * the hand-over of an SA's counter when another device takes it over
+ * (reading L7) or an exact resume.  Enqueued on `cuda_stream`
+ * after earlier work; synchronises it (host_seq may be reused on return).
+ * NBA_IPSEC_EINVAL for NULL arguments. */
+int nba_ipsec_write_sa_seq(nba_ipsec_sa_table *t, const uint32_t *host_seq, void *cuda_stream);
 const char *nba_ipsec_strerror(int code);
 
 /* Pipeline selection (both produce identical bytes):
@@ -244,6 +250,65 @@ int nba_ipsec_route_pack(const uint8_t *in_buf, const uint32_t *in_off, const ui
                          uint32_t world, void *workspace, uint8_t *send_buf, uint16_t *send_len,
                          uint32_t *send_sa, uint64_t *dest_counts, uint64_t *dest_bytes,
                          void *cuda_stream);
+/* As nba_ipsec_route_pack with an explicit ownership map instead of s mod world
+ * (the adaptive split below): sa_map (DEVICE, n_sa_total entries) holds
+ * owner << 24 | local index for every SA, owner < world, local < 2^24; send_sa
+ * receives the local index.  sa_map == NULL is route_pack.  A packet whose
+ * map entry names an owner >= world is counted in dest_counts[world] and not
+ * sent. */
+int nba_ipsec_route_pack_map(const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
+                             const uint32_t *sa_global, uint32_t n_pkts, uint32_t n_sa_total,
+                             const uint32_t *sa_map, uint32_t world, void *workspace,
+                             uint8_t *send_buf, uint16_t *send_len, uint32_t *send_sa,
+                             uint64_t *dest_counts, uint64_t *dest_bytes, void *cuda_stream);
+
+/* ---- adaptive split of the SAs across devices -------------
+ *
+ * PAPER.md:351-365 (§3.4): NBA's load balancer hill-climbs the offloading
+ * fraction w in [0%, 100%] by delta, choosing the direction "by observing if
+ * throughput increases or decreases" (moving average of packets out per unit
+ * time), waits for the workers to apply each update (2 .. 32 update intervals,
+ * growing with w) and keeps perturbing w by delta.  Defaults: delta = 4%
+ * (steps = 25), history 16384 samples, update interval 0.2 s.
+ * Here w splits the SAs of a node of devices between its two halves (readings
+ * L1..L7); host code only, no device work, no CUDA needed.
+ *   observe(t_ns, dt_ns, pkts): one sample per completed batch -- the clock
+ *   now, the batch's duration and the packets it transmitted; returns (in
+ *   *step, may be NULL) the step k to apply, w = k / steps.  Deterministic:
+ *   integer samples, exact comparisons.
+ *   assign: owner[s] for s < n_sa under a binary tree of splits over n_dev <= 8
+ *   devices: node i (heap order: root 0, children 2i+1, 2i+2) covering devices
+ *   [lo, hi) and SAs [a, b) gives the last floor((b-a) * node_step[i] / steps)
+ *   SAs to [lo + (hi-lo)/2, hi).  node_step has NBA_IPSEC_ALB_TREE_NODES
+ *   entries (only internal nodes are read; may be NULL for n_dev = 1).
+ *   sa_map (optional) receives owner << 24 | s: every device keeps all SAs, the
+ *   owner's counter is the live one (nba_ipsec_write_sa_seq moves it). */
+#define NBA_IPSEC_ALB_MAX_DEV 8u
+#define NBA_IPSEC_ALB_TREE_NODES 15u
+
+typedef struct {
+    uint32_t steps;       /* K: w moves by 1/K (paper: delta = 4% -> 25); 1..10^6 */
+    uint32_t init_step;   /* starting w = init_step / K; <= K */
+    uint32_t history;     /* moving-average window, samples (paper: 16384); 1..2^26 */
+    uint64_t update_ns;   /* observation interval (paper: 0.2 s); > 0 */
+    uint32_t wait_min;    /* waiting interval at w = 0, in update intervals (paper: 2) */
+    uint32_t wait_max;    /* ... at w = 100% (paper: 32); >= wait_min */
+} nba_ipsec_alb_params;
+
+typedef struct nba_ipsec_alb nba_ipsec_alb;   /* opaque controller */
+
+void nba_ipsec_alb_default_params(nba_ipsec_alb_params *p);
+/* NBA_IPSEC_EINVAL for NULL arguments or out-of-range parameters. */
+int nba_ipsec_alb_create(const nba_ipsec_alb_params *p, nba_ipsec_alb **out);
+int nba_ipsec_alb_observe(nba_ipsec_alb *a, uint64_t t_ns, uint64_t dt_ns, uint64_t pkts,
+                          uint32_t *step);
+/* Current step, direction (+1/-1) and number of updates so far (NULL: skip). */
+int nba_ipsec_alb_state(const nba_ipsec_alb *a, uint32_t *step, int *direction, uint64_t *updates);
+int nba_ipsec_alb_destroy(nba_ipsec_alb *a);   /* NULL -> OK */
+/* NBA_IPSEC_EINVAL for n_dev outside 1..8, steps == 0, a node step > steps,
+ * NULL owner (or NULL node_step with n_dev > 1), n_sa > 2^24. */
+int nba_ipsec_alb_assign(uint32_t n_sa, uint32_t n_dev, const uint32_t *node_step, uint32_t steps,
+                         uint32_t *owner, uint32_t *sa_map);
 
 /* ---- ESP inbound: the mirror of the path ------------------
  *

@@ -544,6 +544,19 @@ int nba_ipsec_read_sa_seq(nba_ipsec_sa_table *t, uint32_t *host_seq, void *cuda_
     return NBA_IPSEC_OK;
 }
 
+int nba_ipsec_write_sa_seq(nba_ipsec_sa_table *t, const uint32_t *host_seq, void *cuda_stream)
+{
+    // counter hand-over between devices (reading L7)
+    if (!t || !host_seq) return NBA_IPSEC_EINVAL;
+    DeviceGuard g(t->device);
+    cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    if (cudaMemcpyAsync(t->T.seq, host_seq, t->n_sa * sizeof(uint32_t), cudaMemcpyHostToDevice,
+                        st) != cudaSuccess ||
+        cudaStreamSynchronize(st) != cudaSuccess)
+        return NBA_IPSEC_ECUDA;
+    return NBA_IPSEC_OK;
+}
+
 int nba_ipsec_debug_trace(nba_ipsec_sa_table *t, uint64_t *host, uint32_t n_words)
 {
     if (!t || !host) return NBA_IPSEC_EINVAL;
@@ -686,11 +699,11 @@ int nba_ipsec_route_workspace_bytes(uint32_t max_pkts, uint32_t world, uint64_t 
     return NBA_IPSEC_OK;
 }
 
-int nba_ipsec_route_pack(const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
-                         const uint32_t *sa_global, uint32_t n_pkts, uint32_t n_sa_total,
-                         uint32_t world, void *workspace, uint8_t *send_buf, uint16_t *send_len,
-                         uint32_t *send_sa, uint64_t *dest_counts, uint64_t *dest_bytes,
-                         void *cuda_stream)
+int nba_ipsec_route_pack_map(const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
+                             const uint32_t *sa_global, uint32_t n_pkts, uint32_t n_sa_total,
+                             const uint32_t *sa_map, uint32_t world, void *workspace,
+                             uint8_t *send_buf, uint16_t *send_len, uint32_t *send_sa,
+                             uint64_t *dest_counts, uint64_t *dest_bytes, void *cuda_stream)
 {
     if (world == 0 || world > 8 || n_pkts > NBA_IPSEC_MAX_BATCH) return NBA_IPSEC_EINVAL;
     if (!dest_counts || !dest_bytes) return NBA_IPSEC_EINVAL;
@@ -704,12 +717,23 @@ int nba_ipsec_route_pack(const uint8_t *in_buf, const uint32_t *in_off, const ui
     if (!in_buf || !in_off || !in_len || !sa_global || !workspace || !send_buf || !send_len ||
         !send_sa)
         return NBA_IPSEC_EINVAL;
-    return launch_route(in_buf, in_off, in_len, sa_global, n_pkts, n_sa_total, world, workspace,
-                        send_buf, send_len, send_sa,
+    return launch_route(in_buf, in_off, in_len, sa_global, n_pkts, n_sa_total, sa_map, world,
+                        workspace, send_buf, send_len, send_sa,
                         reinterpret_cast<unsigned long long *>(dest_counts),
                         reinterpret_cast<unsigned long long *>(dest_bytes), st) == cudaSuccess
                ? NBA_IPSEC_OK
                : NBA_IPSEC_ECUDA;
+}
+
+int nba_ipsec_route_pack(const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
+                         const uint32_t *sa_global, uint32_t n_pkts, uint32_t n_sa_total,
+                         uint32_t world, void *workspace, uint8_t *send_buf, uint16_t *send_len,
+                         uint32_t *send_sa, uint64_t *dest_counts, uint64_t *dest_bytes,
+                         void *cuda_stream)
+{
+    return nba_ipsec_route_pack_map(in_buf, in_off, in_len, sa_global, n_pkts, n_sa_total, nullptr,
+                                    world, workspace, send_buf, send_len, send_sa, dest_counts,
+                                    dest_bytes, cuda_stream);
 }
 
 int nba_ipsec_enable_inbound(nba_ipsec_sa_table *t)

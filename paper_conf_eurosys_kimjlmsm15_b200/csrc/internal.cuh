@@ -180,8 +180,8 @@ cudaError_t setup_inbound_attributes(uint32_t n_sa, uint32_t max_tiles, int num_
 cudaError_t launch_flow_lookup(const uint4 *table, uint32_t mask, const FlowArgs &A, cudaStream_t st);
 size_t route_workspace_bytes(uint32_t max_pkts, uint32_t world);
 cudaError_t launch_route(const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
-                         const uint32_t *sa, uint32_t n, uint32_t n_sa_total, uint32_t world,
-                         void *ws, uint8_t *send_buf, uint16_t *send_len, uint32_t *send_sa,
+                         const uint32_t *sa, uint32_t n, uint32_t n_sa_total,
+                         const uint32_t *sa_map, uint32_t world, void *ws, uint8_t *send_buf, uint16_t *send_len, uint32_t *send_sa,
                          unsigned long long *dest_counts, unsigned long long *dest_bytes,
                          cudaStream_t st);
 

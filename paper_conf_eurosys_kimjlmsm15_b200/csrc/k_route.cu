@@ -1,6 +1,7 @@
 // k_route.cu -- single-ingress redistribution (second half):
 // when all traffic enters at one GPU, every packet must reach the GPU that owns
-// its SA (SA-hash shard, owner = sa mod world, S§8(e)) before the path runs
+// its SA (SA-hash shard, owner = sa mod world, S§8(e), or the owner the
+// adaptive split assigned, f4: sa_map[sa] = owner << 24 | local) before the path runs
 // there.  These kernels route and pack a batch by destination so one NCCL
 // all-to-all per array moves it (paper_conf_eurosys_kimjlmsm15_b200/redistribute.py):
 //   k_route_tiles : per 256-packet tile, each packet's destination, its rank
@@ -10,7 +11,8 @@
 //   k_route_scan  : exclusive scans of those over tiles, and the destination
 //                   regions of the send buffers (destination-major);
 //   k_route_pack  : one warp per packet copies its bytes to its place and
-//                   writes its length and LOCAL SA index (sa / world).
+//                   writes its length and LOCAL SA index (sa / world, or
+//                   the map's low 24 bits).
 // Stable: a destination receives its packets in batch-index order, so the
 // per-SA sequence numbers at the owner are those of the sequential oracle.
 // Packets without a valid SA (sa >= n_sa_total) are not sent (counted in slot
@@ -33,7 +35,7 @@ struct RouteWork {
 
 __global__ void __launch_bounds__(RT_TILE)
 k_route_tiles(RouteWork R, const uint16_t *in_len, const uint32_t *sa, uint32_t n,
-              uint32_t n_sa_total, uint32_t world)
+              uint32_t n_sa_total, const uint32_t *sa_map, uint32_t world)
 {
     __shared__ uint32_t s_wc[RT_TILE / 32][RT_MAX_WORLD + 1];
     __shared__ uint32_t s_wb[RT_TILE / 32][RT_MAX_WORLD + 1];
@@ -41,7 +43,9 @@ k_route_tiles(RouteWork R, const uint16_t *in_len, const uint32_t *sa, uint32_t 
     const uint32_t i = blockIdx.x * RT_TILE + tid;
     const uint32_t len = i < n ? in_len[i] : 0u;
     const uint32_t s = i < n ? sa[i] : INVALID_SA;
-    const uint32_t d = i < n ? (s < n_sa_total ? s % world : world) : RT_MAX_WORLD + 1u;
+    // owner: s mod world (SA-hash shard) or the adaptive split's map (f4)
+    uint32_t d = RT_MAX_WORLD + 1u;
+    if (i < n) d = s < n_sa_total ? (sa_map ? min(__ldg(sa_map + s) >> 24, world) : s % world) : world;
     uint32_t my_rank = 0, my_brank = 0;
     for (uint32_t k = 0; k <= world; k++) {
         const uint32_t m = __ballot_sync(0xffffffffu, d == k);
@@ -137,8 +141,8 @@ k_route_scan(RouteWork R, uint32_t n_tiles, uint32_t world, unsigned long long *
 // order inside a destination), length and local SA index to the send arrays.
 __global__ void __launch_bounds__(256)
 k_route_pack(RouteWork R, const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
-             const uint32_t *sa, uint32_t n, uint32_t world, uint8_t *send_buf, uint16_t *send_len,
-             uint32_t *send_sa)
+             const uint32_t *sa, const uint32_t *sa_map, uint32_t n, uint32_t world,
+             uint8_t *send_buf, uint16_t *send_len, uint32_t *send_sa)
 {
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -155,7 +159,7 @@ k_route_pack(RouteWork R, const uint8_t *in_buf, const uint32_t *in_off, const u
     for (uint32_t b = lane; b < len; b += 32u) dst[b] = src[b];
     if (lane == 0) {
         send_len[pos] = (uint16_t)len;
-        send_sa[pos] = sa[i] / world;
+        send_sa[pos] = sa_map ? (__ldg(sa_map + sa[i]) & 0xFFFFFFu) : sa[i] / world;
     }
 }
 
@@ -166,8 +170,8 @@ size_t route_workspace_bytes(uint32_t max_pkts, uint32_t world)
 }
 
 cudaError_t launch_route(const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
-                         const uint32_t *sa, uint32_t n, uint32_t n_sa_total, uint32_t world,
-                         void *ws, uint8_t *send_buf, uint16_t *send_len, uint32_t *send_sa,
+                         const uint32_t *sa, uint32_t n, uint32_t n_sa_total,
+                         const uint32_t *sa_map, uint32_t world, void *ws, uint8_t *send_buf, uint16_t *send_len, uint32_t *send_sa,
                          unsigned long long *dest_counts, unsigned long long *dest_bytes,
                          cudaStream_t st)
 {
@@ -185,9 +189,9 @@ cudaError_t launch_route(const uint8_t *in_buf, const uint32_t *in_off, const ui
     R.tcnt = reinterpret_cast<uint32_t *>(take((size_t)tiles * (world + 1) * 4));
     R.tbyt = reinterpret_cast<unsigned long long *>(take((size_t)tiles * (world + 1) * 8));
     R.base = reinterpret_cast<unsigned long long *>(take(2ull * (world + 1) * 8));
-    k_route_tiles<<<tiles, RT_TILE, 0, st>>>(R, in_len, sa, n, n_sa_total, world);
+    k_route_tiles<<<tiles, RT_TILE, 0, st>>>(R, in_len, sa, n, n_sa_total, sa_map, world);
     k_route_scan<<<1, 256, 0, st>>>(R, tiles, world, dest_counts, dest_bytes);
-    k_route_pack<<<(n * 32u + 255u) / 256u, 256, 0, st>>>(R, in_buf, in_off, in_len, sa, n, world,
+    k_route_pack<<<(n * 32u + 255u) / 256u, 256, 0, st>>>(R, in_buf, in_off, in_len, sa, sa_map, n, world,
                                                          send_buf, send_len, send_sa);
     return cudaGetLastError();
 }

@@ -64,6 +64,15 @@ class Flow(ctypes.Structure):
                 ("sa", ctypes.c_uint32)]
 
 
+class AlbParams(ctypes.Structure):
+    _fields_ = [("steps", ctypes.c_uint32), ("init_step", ctypes.c_uint32),
+                ("history", ctypes.c_uint32), ("update_ns", ctypes.c_uint64),
+                ("wait_min", ctypes.c_uint32), ("wait_max", ctypes.c_uint32)]
+
+
+ALB_MAX_DEV, ALB_TREE_NODES = 8, 15
+
+
 class InBatch(ctypes.Structure):
     _fields_ = [("in_buf", ctypes.c_void_p), ("in_off", ctypes.c_void_p),
                 ("in_len", ctypes.c_void_p), ("sa_idx", ctypes.c_void_p),
@@ -111,6 +120,15 @@ def _load():
         "nba_ipsec_set_flow_table": (i32, [vp, P(Flow), u32]),
         "nba_ipsec_route_workspace_bytes": (i32, [u32, u32, P(u64)]),
         "nba_ipsec_route_pack": (i32, [vp, vp, vp, vp, u32, u32, u32, vp, vp, vp, vp, vp, vp, vp]),
+        "nba_ipsec_route_pack_map": (i32, [vp, vp, vp, vp, u32, u32, vp, u32, vp, vp, vp, vp, vp, vp,
+                                           vp]),
+        "nba_ipsec_write_sa_seq": (i32, [vp, P(u32), vp]),
+        "nba_ipsec_alb_default_params": (None, [P(AlbParams)]),
+        "nba_ipsec_alb_create": (i32, [P(AlbParams), P(vp)]),
+        "nba_ipsec_alb_observe": (i32, [vp, u64, u64, u64, P(u32)]),
+        "nba_ipsec_alb_state": (i32, [vp, P(u32), P(i32), P(u64)]),
+        "nba_ipsec_alb_destroy": (i32, [vp]),
+        "nba_ipsec_alb_assign": (i32, [u32, u32, P(u32), u32, P(u32), P(u32)]),
         "nba_ipsec_lookup_sa": (i32, [vp, vp, vp, vp, u32, vp, vp]),
         "nba_ipsec_process_inbound": (i32, [vp, P(InBatch), vp]),
         "nba_ipsec_read_in_counters": (i32, [vp, P(InCounters), vp]),
@@ -234,6 +252,14 @@ class SATable:
         _check(lib.nba_ipsec_read_sa_seq(self._h, out.ctypes.data_as(ctypes.POINTER(ctypes.c_uint32)),
                                          _stream_handle(stream)), "nba_ipsec_read_sa_seq")
         return out
+
+    def write_sa_seq(self, seq, stream=None):
+        """nba_ipsec_write_sa_seq: replace every SA's counter (hand-over, L7)."""
+        a = np.ascontiguousarray(seq, dtype=np.uint32)
+        if a.shape != (self.n_sa,):
+            raise ValueError(f"need {self.n_sa} sequence numbers")
+        _check(lib.nba_ipsec_write_sa_seq(self._h, a.ctypes.data_as(ctypes.POINTER(ctypes.c_uint32)),
+                                          _stream_handle(stream)), "nba_ipsec_write_sa_seq")
 
     def set_pipeline(self, pipeline: int):
         _check(lib.nba_ipsec_set_pipeline(self._h, int(pipeline)), "nba_ipsec_set_pipeline")
@@ -372,3 +398,72 @@ def route_pack(in_buf, in_off, in_len, sa_global, n, n_sa_total, world, workspac
                                     _ptr(send_len), _ptr(send_sa), _ptr(dest_counts),
                                     _ptr(dest_bytes), _stream_handle(stream)),
            "nba_ipsec_route_pack")
+
+
+def route_pack_map(in_buf, in_off, in_len, sa_global, n, n_sa_total, sa_map, world, workspace,
+                   send_buf, send_len, send_sa, dest_counts, dest_bytes, stream=None):
+    """nba_ipsec_route_pack_map: routing by an explicit owner map (f4)."""
+    _check(lib.nba_ipsec_route_pack_map(_ptr(in_buf), _ptr(in_off), _ptr(in_len), _ptr(sa_global),
+                                        int(n), int(n_sa_total), _ptr(sa_map), int(world),
+                                        _ptr(workspace), _ptr(send_buf), _ptr(send_len),
+                                        _ptr(send_sa), _ptr(dest_counts), _ptr(dest_bytes),
+                                        _stream_handle(stream)),
+           "nba_ipsec_route_pack_map")
+
+
+# -- adaptive split of the SAs across devices (SURVEY §8(f) f4) -----------------
+def alb_default_params() -> AlbParams:
+    p = AlbParams()
+    lib.nba_ipsec_alb_default_params(ctypes.byref(p))
+    return p
+
+
+class Alb:
+    """nba_ipsec_alb_* controller (host code in the library)."""
+
+    def __init__(self, steps=None, init_step=None, history=None, update_ns=None, wait_min=None,
+                 wait_max=None):
+        p = alb_default_params()
+        for k, v in (("steps", steps), ("init_step", init_step), ("history", history),
+                     ("update_ns", update_ns), ("wait_min", wait_min), ("wait_max", wait_max)):
+            if v is not None:
+                setattr(p, k, int(v))
+        self.params = p
+        self._h = ctypes.c_void_p()
+        _check(lib.nba_ipsec_alb_create(ctypes.byref(p), ctypes.byref(self._h)), "nba_ipsec_alb_create")
+
+    def observe(self, t_ns: int, dt_ns: int, pkts: int) -> int:
+        k = ctypes.c_uint32(0)
+        _check(lib.nba_ipsec_alb_observe(self._h, int(t_ns), int(dt_ns), int(pkts), ctypes.byref(k)),
+               "nba_ipsec_alb_observe")
+        return int(k.value)
+
+    def state(self):
+        k, d, u = ctypes.c_uint32(0), ctypes.c_int(0), ctypes.c_uint64(0)
+        _check(lib.nba_ipsec_alb_state(self._h, ctypes.byref(k), ctypes.byref(d), ctypes.byref(u)),
+               "nba_ipsec_alb_state")
+        return int(k.value), int(d.value), int(u.value)
+
+    def close(self):
+        if self._h:
+            lib.nba_ipsec_alb_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def alb_assign(n_sa: int, n_dev: int, node_step, steps: int):
+    """nba_ipsec_alb_assign -> (owner[n_sa], sa_map[n_sa]) as uint32 arrays."""
+    u32p = ctypes.POINTER(ctypes.c_uint32)
+    ns = np.zeros(ALB_TREE_NODES, np.uint32)
+    ns[:len(node_step)] = node_step
+    owner = np.zeros(max(n_sa, 1), np.uint32)
+    sa_map = np.zeros(max(n_sa, 1), np.uint32)
+    _check(lib.nba_ipsec_alb_assign(int(n_sa), int(n_dev), ns.ctypes.data_as(u32p), int(steps),
+                                    owner.ctypes.data_as(u32p), sa_map.ctypes.data_as(u32p)),
+           "nba_ipsec_alb_assign")
+    return owner[:n_sa], sa_map[:n_sa]

@@ -40,9 +40,11 @@ class Received:
     sa_idx: torch.Tensor     # int32 local SA indices
 
 
-def pack(db, n: int, n_sa_total: int, world: int, stream=None) -> Packed:
+def pack(db, n: int, n_sa_total: int, world: int, stream=None, sa_map=None) -> Packed:
     """Route and pack a device batch (gen/device.DeviceBatch with GLOBAL SA
-    indices) on the GPU with nba_ipsec_route_pack."""
+    indices) on the GPU with nba_ipsec_route_pack, or with
+    nba_ipsec_route_pack_map when `sa_map` (device uint32 tensor, owner << 24 |
+    local, e.g. from the adaptive split, alb.py) is given."""
     from . import nba_ipsec
     dev = db.in_buf.device
     ws = torch.empty(nba_ipsec.route_workspace_bytes(max(n, 1), world), dtype=torch.uint8, device=dev)
@@ -51,8 +53,12 @@ def pack(db, n: int, n_sa_total: int, world: int, stream=None) -> Packed:
     send_sa = torch.empty(max(n, 1), dtype=torch.int32, device=dev)
     dc = torch.zeros(world + 1, dtype=torch.int64, device=dev)
     dbytes = torch.zeros(world + 1, dtype=torch.int64, device=dev)
-    nba_ipsec.route_pack(db.in_buf, db.in_off, db.in_len, db.sa_idx, n, n_sa_total, world, ws,
-                         send_buf, send_len, send_sa, dc, dbytes, stream=stream)
+    if sa_map is None:
+        nba_ipsec.route_pack(db.in_buf, db.in_off, db.in_len, db.sa_idx, n, n_sa_total, world, ws,
+                             send_buf, send_len, send_sa, dc, dbytes, stream=stream)
+    else:
+        nba_ipsec.route_pack_map(db.in_buf, db.in_off, db.in_len, db.sa_idx, n, n_sa_total, sa_map,
+                                 world, ws, send_buf, send_len, send_sa, dc, dbytes, stream=stream)
     c = dc.cpu().tolist()
     b = dbytes.cpu().tolist()
     return Packed(buf=send_buf, length=send_len, sa=send_sa, counts=c[:world], nbytes=b[:world])
@@ -86,3 +92,24 @@ def exchange(p: Packed, group=None) -> Received:
     if n_out > 1:
         off[1:n_out] = torch.cumsum(lens[:-1], 0)
     return Received(n=n_out, in_buf=buf, in_off=off.to(torch.int32), in_len=length, sa_idx=sa)
+
+
+def local_views(p: Packed, d: int, out_pad: int = 64):
+    """One destination's region of the packed arrays as a batch for that
+    owner's table on THIS device (the one-process stand-in for the exchange,
+    used by the adaptive split, alb.py): (n, in_off, in_len, sa_idx, out_off,
+    out_len, out_buf), offsets into p.buf / a fresh output pool."""
+    dev = p.buf.device
+    c0, b0 = sum(p.counts[:d]), sum(p.nbytes[:d])
+    n = p.counts[d]
+    lens = p.length[c0:c0 + n].to(torch.int64) & 0xFFFF
+    in_off = torch.full((max(n, 1),), b0, dtype=torch.int64, device=dev)
+    out_off = torch.zeros(max(n, 1), dtype=torch.int64, device=dev)
+    if n > 1:
+        in_off[1:n] += torch.cumsum(lens[:-1], 0)
+        out_off[1:n] = torch.cumsum(lens[:-1] + out_pad, 0)
+    pool = int(p.nbytes[d]) + out_pad * n + 16
+    out_buf = torch.empty(pool, dtype=torch.uint8, device=dev)
+    out_len = torch.empty(max(n, 1), dtype=torch.int16, device=dev)
+    return (n, in_off.to(torch.int32), p.length[c0:], p.sa[c0:], out_off.to(torch.int32), out_len,
+            out_buf)
