@@ -36,18 +36,7 @@ struct FusedLo {
     uint32_t hkey[2 * F_SUPER];    // merged prologue: SA of each slot of the CTA's SA hash
     uint32_t hmask[2 * F_SUPER];   //   warps holding a group of that SA
     uint8_t wrun[F_THREADS / 32];  // warp -> run of 32 sorted positions (0xff: none)
-    // split AES / work stealing (outbound one-kernel path, length-divergent
-    // CTAs): the AES steps of the CTA's longest packets
-    uint32_t dstat[3];             // sum and max of AES steps, count (valid packets)
-    uint32_t nlong;                // sorted positions [0, nlong) are "long"
-    uint16_t lp_tid[192];          // position -> thread holding its round keys
-    uint32_t lp_pre[193];          // exclusive prefix of the long packets' AES steps
-    uint32_t lp_cp[6][192];        // their RFC 3686 counter-block precompute (CtrPre)
-    uint32_t st_claim[192];        // work stealing: step bits claimed (owner or thief)
-    uint32_t st_done[192];         //   steps whose ciphertext a thief has written
-    uint32_t st_cursor;            //   next steal item (r-major: last steps first)
 };
-constexpr uint32_t LP_MAX = 192;
 
 struct FusedHi {
     uint4 rkB[4][F_THREADS];       // round keys 7..10
@@ -592,29 +581,6 @@ __device__ __forceinline__ void load_raw6(uintptr_t a, uintptr_t end, Raw6 &r)
         const uintptr_t qa = abase + 32u * i;
         if (qa < end) ldg_nc_v8(reinterpret_cast<const void *>(qa), r.c[2 * i], r.c[2 * i + 1]);
         else r.c[2 * i] = r.c[2 * i + 1] = z4;
-    }
-}
-
-// load_raw6 through L2 (coherent): for bytes written earlier in the same
-// kernel by other threads of the CTA (the split-AES ciphertext).
-__device__ __forceinline__ void load_raw6_cg(uintptr_t a, uintptr_t end, Raw6 &r)
-{
-    const uintptr_t abase = a & ~(uintptr_t)31;
-    r.sh = (uint32_t)(a & 31u);
-    const uint4 z4 = make_uint4(0, 0, 0, 0);
-#pragma unroll
-    for (int i = 0; i < 3; i++) {
-        const uintptr_t qa = abase + 32u * i;
-        if (qa < end) {
-            uint4 &x = r.c[2 * i], &y = r.c[2 * i + 1];
-            asm volatile("ld.global.cg.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-                         : "=r"(x.x), "=r"(x.y), "=r"(x.z), "=r"(x.w), "=r"(y.x), "=r"(y.y),
-                           "=r"(y.z), "=r"(y.w)
-                         : "l"(qa)
-                         : "memory");
-        } else {
-            r.c[2 * i] = r.c[2 * i + 1] = z4;
-        }
     }
 }
 

@@ -58,21 +58,6 @@ namespace nba {
 #ifndef NBA_SA_PREFETCH       // L2 prefetch of the SA table at kernel start
 #define NBA_SA_PREFETCH 1
 #endif
-#ifndef NBA_SPLIT             // split AES for the longest packets of length-divergent CTAs
-#define NBA_SPLIT 0           // (measured: IMIX 104.6 -> 105.3 us, 64 B +2 us; kept off)
-#endif
-#ifndef NBA_SPLIT_FACTOR      // a CTA is length-divergent if its longest packet needs more
-#define NBA_SPLIT_FACTOR 2    // AES steps than FACTOR x its mean; then packets with more
-#endif                        // than LONG_FACTOR x the mean are "long"
-#ifndef NBA_LONG_FACTOR
-#define NBA_LONG_FACTOR 1
-#endif
-#ifndef NBA_STEAL             // warps done with their packets steal AES steps of the longest
-#define NBA_STEAL 0           // packets from the back (measured: IMIX -1% or +14%, 1514 B +0.7%)
-#endif
-#ifndef NBA_PDL_MERGED        // one-kernel form launched as a programmatic dependent of the
-#define NBA_PDL_MERGED 0      // previous kernel on the stream (measured: no gain at 64 B, -1.3% at 1514 B)
-#endif
 
 
 // ---------------------------------------------- one packet, one lane
@@ -102,8 +87,7 @@ __device__ __forceinline__ PktPre load_pkt_pre(const DevTable &T, const uint8_t 
 __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B, FusedLo &L,
                                            FusedHi &H, uint32_t lane4r, uint32_t tid, uint32_t sa,
                                            uint32_t info, uint32_t q32, uint32_t inoff,
-                                           uint32_t outoff, const PktPre &pp, unsigned long long *dbg,
-                                           uint32_t spos = 0xffffffffu)
+                                           uint32_t outoff, const PktPre &pp, unsigned long long *dbg)
 {
     long long ck_start = clock64(), ck_setup = 0, ck_aes = 0, ck_sha = 0, ck_emit = 0;
     const uint4 r0 = pp.r0, r1 = pp.r1, r2 = pp.r2, hd = pp.hd, h0 = pp.h0, h1 = pp.h1;
@@ -165,34 +149,11 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
     // ---- one SHA-1 compression per iteration; AES steps feed the first nsteps
 #pragma unroll 1
     uint4 pcarry0 = make_uint4(0, 0, 0, 0), pcarry1 = pcarry0;   // NBA_CARRY: last payload block
-    bool os_open = true;          // false once a thief took a step (the rest is theirs)
     for (uint32_t it = 0; it <= nb_in; it++) {
         uint32_t ct[16];
 #pragma unroll
         for (int w = 0; w < 16; w++) ct[w] = 0u;
-        bool mine = it < nsteps;
-#if NBA_STEAL
-        if (mine && spos < LP_MAX) {
-            // claim step it; a thief that got there first writes its ciphertext
-            // (thieves take steps from the back, so the stolen steps are a suffix)
-            const uint32_t bit = 1u << it;
-            if (!os_open || (atomicOr(&L.st_claim[spos], bit) & bit)) {
-                mine = false;
-                if (os_open) {
-                    os.finish(B.out_buf + outoff + 36u + 64u * it);
-                    os_open = false;
-                }
-                while (!(*reinterpret_cast<volatile uint32_t *>(&L.st_done[spos]) & bit)) {
-                }
-                __threadfence_block();
-                const uintptr_t c0 = reinterpret_cast<uintptr_t>(B.out_buf + outoff + 36u);
-                Raw6 raw;
-                load_raw6_cg(c0 + 64u * it, c0 + 4u * Cw, raw);
-                extract16(raw, ct);
-            }
-        }
-#endif
-        if (mine) {
+        if (it < nsteps) {
             // payload words of T bytes [64 it, 64 it + 64), realigned
             if (64u * (it + NBA_PF_AHEAD) < D) prefetch_l2(src + 64u * (it + NBA_PF_AHEAD));
             // interior step: all 16 words are payload, the trailer (last word and,
@@ -302,7 +263,6 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
         if (it == 0) ck_sha = clock64();
     }
     // ICV = first 96 bits of the outer digest (RFC 2404)
-    if (!os_open) os.init(B.out_buf + outoff + 36u + 4u * Cw);
     os.put(bswap32(st[0]));
     os.put(bswap32(st[1]));
     os.put(bswap32(st[2]));
@@ -316,160 +276,6 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
         dbg[4] = ck_end - ck_sha;          // the rest
         dbg[5] = st[0];
     }
-}
-
-// ------------------------------------------------ split AES (IMIX-like CTAs)
-// With one lane per packet a CTA's longest packets serialise in one or two
-// warps: in an IMIX batch the warps holding the 1514-byte packets run ~3x
-// longer than the rest, alone at the end.  When a CTA's longest packets need
-// more than NBA_SPLIT_FACTOR x its mean number of 64-byte steps, the AES-CTR
-// steps of its LP_MAX (= 2 warps) longest packets are spread over all 512
-// threads first (same arithmetic as esp_packet's step, RFC 3686 counter
-// blocks, ciphertext written to its final place), and those lanes then run
-// only the HMAC over the ciphertext they read back (esp_packet_sha).
-
-// Ciphertext of 64-byte step `it` of the packet at sorted position `pos`.
-__device__ __forceinline__ void split_step(const BatchArgs &B, FusedLo &L, FusedHi &H,
-                                           uint32_t lane4r, uint32_t pos, uint32_t it)
-{
-    const uint32_t pk = L.perm[pos];
-    const uint32_t D = L.info[pk] & 0x7ffu;
-    const uint32_t pad = esp_pad(D);
-    const uint32_t Cw = (D + pad + 2u) >> 2;
-    const uint8_t *src = B.in_buf + L.inoff[pk];
-    const uintptr_t src_end = reinterpret_cast<uintptr_t>(src) + D;
-    CtrPre cp;
-    cp.X0 = L.lp_cp[0][pos];
-    cp.Z0 = L.lp_cp[1][pos];
-    cp.Z1 = L.lp_cp[2][pos];
-    cp.Z2 = L.lp_cp[3][pos];
-    cp.Z3 = L.lp_cp[4][pos];
-    cp.R3 = L.lp_cp[5][pos];
-    uint32_t ks[16];
-    aes4_keystream(lane4r, cp, it, L, H, L.lp_tid[pos], ks);
-    uint32_t ct[16];
-    const bool interior = 16u * it + 18u <= Cw;
-    Raw6 raw;
-    if (interior) load_raw6_inb(reinterpret_cast<uintptr_t>(src) + 64u * it, raw);
-    else load_raw6(reinterpret_cast<uintptr_t>(src) + 64u * it, src_end, raw);
-    extract16(raw, ct);
-    if (!interior) {   // trailer (see esp_packet)
-        const uint32_t lw = Cw - 1u - 16u * it;
-        const uint32_t keep = pad == 0 ? 0x0000ffffu : pad == 1 ? 0x000000ffu : 0u;
-        const uint32_t trl = pad == 0 ? 0x04000000u : pad == 1 ? 0x04010100u
-                           : pad == 2 ? 0x04020201u : 0x04030302u;
-#pragma unroll
-        for (int w = 0; w < 16; w++) {
-            if ((uint32_t)w == lw) ct[w] = (ct[w] & keep) | trl;
-            if (pad == 3u && (uint32_t)w + 1u == lw) ct[w] = (ct[w] & 0x00ffffffu) | 0x01000000u;
-        }
-        if (pad == 3u && lw == 16u) ct[15] = (ct[15] & 0x00ffffffu) | 0x01000000u;
-    }
-#pragma unroll
-    for (int w = 0; w < 16; w++) ct[w] ^= ks[w];
-    // ciphertext starts 36 bytes into the output packet (outer IPv4, SPI, seq, IV)
-    uint8_t *dst = B.out_buf + L.outoff[pk] + 36u + 64u * it;
-    const uint32_t nw = min(16u, Cw - 16u * it);
-    OutStream os;
-    os.init(dst);
-    // word by word: the first chunk is shared with the previous step's thread,
-    // so only put()'s byte-exact partial stores may touch it (put16 assumes a
-    // chunk the stream started itself)
-#pragma unroll
-    for (int w = 0; w < 16; w++)
-        if ((uint32_t)w < nw) os.put(ct[w]);
-    os.finish(dst + 4u * nw);
-}
-
-// esp_packet for a packet whose ciphertext split_step already wrote: outer
-// header + ESP header, HMAC-SHA1-96 over the ciphertext read back from the
-// output slot, ICV.
-__device__ __forceinline__ void esp_packet_sha(const DevTable &T, const BatchArgs &B, uint32_t sa,
-                                               uint32_t info, uint32_t q32, uint32_t outoff,
-                                               const PktPre &pp)
-{
-    const uint4 hd = pp.hd, h0 = pp.h0, h1 = pp.h1;
-    const uint32_t D = info & 0x7ffu;
-    const uint32_t tos = pp.tos;
-    const uint32_t pad = esp_pad(D);
-    const uint32_t C = D + pad + 2u;
-    const uint32_t Lb = 48u + C;
-    const uint32_t Cw = C >> 2;
-    const uint32_t Mw = 4u + Cw;
-    const uint32_t nsteps = (Cw + 15u) >> 4;
-    const uint32_t nb_in = (4u * Mw + 8u) / 64u + 1u;
-    const uint32_t bitlen = (64u + 4u * Mw) * 8u;
-    const uint32_t qbe = bswap32(q32);
-    uint8_t *out = B.out_buf + outoff;
-    {
-        OutStream os;
-        os.init(out);
-        const uint32_t src = bswap32(hd.z), dst = bswap32(hd.w);
-        uint32_t sum = (0x4500u | tos) + Lb + 0x4000u + ((64u << 8) | 50u) + (src >> 16) +
-                       (src & 0xffffu) + (dst >> 16) + (dst & 0xffffu);
-        sum = (sum & 0xffffu) + (sum >> 16);
-        sum = (sum & 0xffffu) + (sum >> 16);
-        const uint32_t cs = ~sum & 0xffffu;
-        os.put(0x45u | (tos << 8) | ((Lb >> 8) << 16) | ((Lb & 0xffu) << 24));
-        os.put(0x00400000u);
-        os.put(64u | (50u << 8) | ((cs >> 8) << 16) | ((cs & 0xffu) << 24));
-        os.put(hd.z);
-        os.put(hd.w);
-        os.put(hd.x);
-        os.put(qbe);
-        os.put(0u);
-        os.put(qbe);
-        os.finish(out + 36u);
-    }
-    uint32_t carry[4] = {bswap32(hd.x), q32, 0u, q32};
-    uint32_t st[5] = {h0.x, h0.y, h0.z, h0.w, h1.x};
-    const uintptr_t ct0 = reinterpret_cast<uintptr_t>(out + 36u), ct_end = ct0 + C;
-#pragma unroll 1
-    for (uint32_t it = 0; it <= nb_in; it++) {
-        uint32_t ct[16];
-#pragma unroll
-        for (int w = 0; w < 16; w++) ct[w] = 0u;
-        if (it < nsteps) {
-            Raw6 raw;
-            load_raw6_cg(ct0 + 64u * it, ct_end, raw);
-            extract16(raw, ct);
-        }
-        uint32_t W[16];
-        if (it < nb_in) {
-            const uint32_t m0 = 16u * it;
-            if (NBA_INTERIOR && m0 + 16u <= Mw && it + 1u < nb_in) {
-#pragma unroll
-                for (int i = 0; i < 16; i++) W[i] = i < 4 ? carry[i] : bswap32(ct[i - 4]);
-            } else {
-#pragma unroll
-                for (int i = 0; i < 16; i++) {
-                    const uint32_t m = m0 + i;
-                    const uint32_t msg = i < 4 ? carry[i] : bswap32(ct[i - 4]);
-                    W[i] = m < Mw ? msg : (m == Mw ? 0x80000000u : 0u);
-                }
-                if (it == nb_in - 1u) W[15] = bitlen;
-            }
-#pragma unroll
-            for (int i = 0; i < 4; i++) carry[i] = bswap32(ct[12 + i]);
-        } else {
-#pragma unroll
-            for (int i = 0; i < 5; i++) W[i] = st[i];
-            W[5] = 0x80000000u;
-#pragma unroll
-            for (int i = 6; i < 15; i++) W[i] = 0u;
-            W[15] = (64u + 20u) * 8u;
-            uint4 g4, g5;
-            ldg_nc_v8(&T.sal[(size_t)sa * SAL_U4 + 4], g4, g5);
-            st[0] = g5.x; st[1] = g5.y; st[2] = g5.z; st[3] = g4.x; st[4] = g4.y;
-        }
-        sha1_compress_fma(st, W, T.n_sa != 0u ? 1u : 0u);
-    }
-    OutStream oi;
-    oi.init(out + 36u + C);
-    oi.put(bswap32(st[0]));
-    oi.put(bswap32(st[1]));
-    oi.put(bswap32(st[2]));
-    oi.finish(out + Lb);
 }
 
 // ------------------------------------------- merged prologue (row a1 in-kernel)
@@ -559,17 +365,6 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
 #endif
     const uint32_t p_begin = blockIdx.x * ppc;
     const uint32_t p_end = min(B.n, p_begin + ppc);
-#if NBA_PDL_MERGED
-    // launched as a programmatic dependent: this CTA may start while the
-    // previous kernel on the stream is still finishing.  Only constant state
-    // (T-tables) is touched before the wait; batch inputs, SA counters and the
-    // shared matrices are read after it.
-    if (MERGED) {
-        aes_tables_to_smem(tabs, T.te0);
-        if (tr && tid == 0) tr[2] = gtimer();
-        asm volatile("griddepcontrol.wait;" ::: "memory");
-    }
-#endif
     // merged prologue: the packet metadata loads are issued before the table
     // staging so their DRAM latency overlaps it
     uint32_t pre_sa = INVALID_SA, pre_D = 0, pre_inoff = 0, pre_outoff = 0;
@@ -585,12 +380,9 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
     uint32_t old0 = 0;
     if (MERGED) old0 = scan_first_old(T, blockIdx.x * (F_THREADS / 32u) + warp,
                                       gridDim.x * (F_THREADS / 32u), gridDim.x, lane);
-    if (!(NBA_PDL_MERGED && MERGED)) {
-        aes_tables_to_smem(tabs, T.te0);
-        if (tr && tid == 0) tr[2] = gtimer();
-    }
+    aes_tables_to_smem(tabs, T.te0);
+    if (tr && tid == 0) tr[2] = gtimer();
     if (tid < 4) L.cnt[tid] = 0ull;
-    if (tid < 3) L.dstat[tid] = 0u;
     if (tid < NBINS) L.bins[tid] = 0;   // re-zeroed after each use (length_sort)
     if (MERGED) {
         for (uint32_t k = tid; k < 2u * F_SUPER; k += F_THREADS) {
@@ -620,19 +412,6 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
             if (cand) prefetch_l2(B.in_buf + pre_inoff);
         }
         warp_agg_add(L.bins, bin, j < cnt_pk);
-#if NBA_SPLIT || NBA_STEAL
-        {   // AES-step statistics of the CTA (length divergence test)
-            const uint32_t stp = cand ? (esp_C(pre_D) + 63u) >> 6 : 0u;
-            const uint32_t ssum = __reduce_add_sync(0xffffffffu, stp);
-            const uint32_t smax = __reduce_max_sync(0xffffffffu, stp);
-            const uint32_t scnt = __popc(__ballot_sync(0xffffffffu, cand));
-            if (lane == 0 && scnt) {
-                atomicAdd(&L.dstat[0], ssum);
-                atomicMax(&L.dstat[1], smax);
-                atomicAdd(&L.dstat[2], scnt);
-            }
-        }
-#endif
         // 1. CTA-local ranks and per-SA counts (the prologue's tile part)
         const uint32_t rank = merged_local_rank(W, L, cand ? pre_sa : INVALID_SA);
         if (j < cnt_pk) L.seq[j] = rank;
@@ -682,109 +461,13 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
         if (tr && lane == 0) atomicMax(&tr[7], gtimer());
         const uint32_t q32 = (sa_me != INVALID_SA) ? L.seq[pk] : 0u;
         const bool ok = q32 != 0u;   // a valid sequence number is never 0
-        uint32_t nlong = 0;
-#if NBA_SPLIT || NBA_STEAL
-        const uint32_t dsum = L.dstat[0], dmax = L.dstat[1], dcnt = L.dstat[2];
-        if (dcnt && dmax * dcnt > NBA_SPLIT_FACTOR * dsum) {   // CTA-uniform
-            if (warp == 0) {
-                // long = more AES steps than NBA_LONG_FACTOR x the mean, among
-                // the packets that get numbers; positions are sorted longest first
-                constexpr uint32_t NG = LP_MAX / 32u;
-                uint32_t stv[NG];
-                uint32_t nraw = 0;
-                bool run = true;
-#pragma unroll
-                for (uint32_t g = 0; g < NG; g++) {
-                    const uint32_t p0 = 32u * g + lane;
-                    const uint32_t k = p0 < cnt_pk ? L.perm[p0] : 0u;
-                    const bool okp = p0 < cnt_pk && (L.info[k] & INFO_OK) && L.seq[k];
-                    stv[g] = okp ? (esp_C(L.info[k] & 0x7ffu) + 63u) >> 6 : 0u;
-                    const uint32_t bl = __ballot_sync(0xffffffffu, okp && stv[g] * dcnt > NBA_LONG_FACTOR * dsum);
-                    if (run) {
-                        if (~bl) {
-                            nraw += __ffs(~bl) - 1u;
-                            run = false;
-                        } else {
-                            nraw += 32u;
-                        }
-                    }
-                }
-                const uint32_t nl = nraw ? min(((nraw + 31u) / 32u) * 32u, LP_MAX) : 0u;
-                uint32_t carry = 0;
-#pragma unroll
-                for (uint32_t g = 0; g < NG; g++) {
-                    const uint32_t a = 32u * g + lane < nl ? stv[g] : 0u;
-                    uint32_t x = a;
-#pragma unroll
-                    for (int o = 1; o < 32; o <<= 1) {
-                        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-                        if (lane >= (uint32_t)o) x += y;
-                    }
-                    L.lp_pre[32u * g + lane] = carry + x - a;
-                    carry += __shfl_sync(0xffffffffu, x, 31);
-                }
-                if (lane == 0) {
-                    L.lp_pre[LP_MAX] = carry;
-                    L.nlong = nl;
-                }
-            }
-            // the lanes holding the longest packets publish their round-key slot
-            // and CTR precompute
-            if (have && pos < LP_MAX) {
-                L.lp_tid[pos] = (uint16_t)tid;
-                if (ok) {
-                    const CtrPre c = ctr_precompute(lane4r, pp.r0, pp.r1, pp.r2, pp.hd.y, 0u, bswap32(q32));
-                    L.lp_cp[0][pos] = c.X0;
-                    L.lp_cp[1][pos] = c.Z0;
-                    L.lp_cp[2][pos] = c.Z1;
-                    L.lp_cp[3][pos] = c.Z2;
-                    L.lp_cp[4][pos] = c.Z3;
-                    L.lp_cp[5][pos] = c.R3;
-                }
-            }
-            if (NBA_STEAL && tid < LP_MAX) {
-                L.st_claim[tid] = 0u;
-                L.st_done[tid] = 0u;
-                if (tid == 0) L.st_cursor = 0u;
-            }
-            __syncthreads();
-            nlong = L.nlong;
-        }
-        if (!NBA_STEAL && nlong) {
-            const uint32_t items = L.lp_pre[nlong];
-            for (uint32_t k = tid; k < items; k += F_THREADS) {
-                uint32_t ps = 0;   // last position whose prefix <= k (steps > 0)
-#pragma unroll 1
-                for (uint32_t step = 128u; step; step >>= 1)   // LP_MAX <= 256
-                    if (ps + step < nlong && L.lp_pre[ps + step] <= k) ps += step;
-                split_step(B, L, H, lane4r, ps, k - L.lp_pre[ps]);
-            }
-            __syncthreads();   // ciphertext in place (read back through L2)
-            if (tr && tid == 0) atomicMax(&tr[7], gtimer());   // (trace: split pre-pass end)
-        }
-#endif
-#if NBA_PDL_MERGED
-        // the grid-wide part is over: the next kernel on the stream may start
-        // its CTAs as this one's exit (they wait for its completion before
-        // reading anything it writes)
-        asm volatile("griddepcontrol.launch_dependents;");
-#endif
         // 6. the lane's packet
         if (have) {
             const uint32_t pkt = p_begin + pk;
-            if (!NBA_STEAL && ok && pos < nlong) {
-                esp_packet_sha(T, B, sa_me, info, q32, L.outoff[pk], pp);
-                const uint32_t Dp = info & 0x7ffu;
-                const uint32_t Lp = 48u + esp_C(Dp);
-                B.out_len[pkt] = (uint16_t)Lp;
-                c_ok++;
-                c_in += Dp;
-                c_out += Lp;
-            } else if (ok) {
+            if (ok) {
                 esp_packet(T, B, L, H, lane4r, tid, sa_me, info, q32, inoff, L.outoff[pk], pp,
                            (tr && blockIdx.x == 0 && (pos == 0 || pos == cnt_pk - 1u))
-                               ? W.trace + 148 * 8 + 8 + (pos == 0 ? 0 : 8) : nullptr,
-                           (NBA_STEAL && pos < nlong) ? pos : 0xffffffffu);
+                               ? W.trace + 148 * 8 + 8 + (pos == 0 ? 0 : 8) : nullptr);
                 const uint32_t Dp = info & 0x7ffu;
                 const uint32_t Lp = 48u + esp_C(Dp);
                 B.out_len[pkt] = (uint16_t)Lp;
@@ -796,27 +479,6 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
                 c_drop++;
             }
         }
-#if NBA_STEAL
-        // done with its own packet: steal AES steps of the long packets, last
-        // steps first (item j -> r = j / nlong, position j mod nlong, step
-        // nsteps - 1 - r); the owner waits for a stolen step's ciphertext
-        if (nlong) {
-            const uint32_t total = nlong * 24u;   // <= 24 steps (D <= 1500)
-            for (;;) {
-                const uint32_t j = atomicAdd(&L.st_cursor, 1u);
-                if (j >= total) break;
-                const uint32_t r = j / nlong, ps = j - r * nlong;
-                const uint32_t n_p = L.lp_pre[ps + 1u] - L.lp_pre[ps];
-                if (r >= n_p) continue;
-                const uint32_t sstep = n_p - 1u - r;
-                const uint32_t bit = 1u << sstep;
-                if (atomicOr(&L.st_claim[ps], bit) & bit) continue;   // the owner has it
-                split_step(B, L, H, lane4r, ps, sstep);
-                __threadfence_block();
-                atomicOr(&L.st_done[ps], bit);
-            }
-        }
-#endif
         if (tr && lane == 0) {
             const unsigned long long now = gtimer();
             atomicMax(&tr[3], now);
@@ -933,12 +595,6 @@ bool fused_merged_ok(uint32_t n, int grid)
     return fused_ppc(n, grid) <= (uint32_t)F_SUPER;
 }
 
-static bool &pdl_rejected()
-{
-    static bool r = std::getenv("NBA_IPSEC_NO_PDL") != nullptr;
-    return r;
-}
-
 cudaError_t launch_fused(const DevTable &T, const DevWork &W, const BatchArgs &B, int grid,
                          bool merged, uint32_t *bar_base, uint32_t *epoch, cudaStream_t st)
 {
@@ -951,34 +607,21 @@ cudaError_t launch_fused(const DevTable &T, const DevWork &W, const BatchArgs &B
     cfg.stream = st;
     cudaLaunchAttribute attr[1];
     static const bool no_coop = std::getenv("NBA_IPSEC_NO_COOP") != nullptr;   // A/B only
-    cudaLaunchAttribute attr2[2];
     if (merged) {
         // grid barriers inside: the driver must make all CTAs co-resident
-        attr2[0].id = cudaLaunchAttributeCooperative;
-        attr2[0].val.cooperative = no_coop ? 0 : 1;
-        attr2[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-        attr2[1].val.programmaticStreamSerializationAllowed = 1;
-        cfg.attrs = attr2;
-        cfg.numAttrs = (NBA_PDL_MERGED && !pdl_rejected()) ? 2 : 1;
+        attr[0].id = cudaLaunchAttributeCooperative;
+        attr[0].val.cooperative = no_coop ? 0 : 1;
     } else {
         attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
         attr[0].val.programmaticStreamSerializationAllowed = 1;
-        cfg.attrs = attr;
-        cfg.numAttrs = 1;
     }
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
     const uint32_t bb = *bar_base;
     // epoch: 31-bit batch tag of the in-kernel prologue's published bases (never 0)
     const uint32_t ep = merged ? ((*epoch % 0x7fffffffu) + 1u) : 0u;
     cudaError_t e = merged ? cudaLaunchKernelEx(&cfg, k_fused<true>, T, W, B, ppc, bb, ep)
                            : cudaLaunchKernelEx(&cfg, k_fused<false>, T, W, B, ppc, bb, ep);
-    if (merged && e != cudaSuccess && cfg.numAttrs == 2) {
-        // the driver does not take cooperative + programmatic together:
-        // cooperative only from now on (griddepcontrol.wait is then a no-op)
-        (void)cudaGetLastError();
-        pdl_rejected() = true;
-        cfg.numAttrs = 1;
-        e = cudaLaunchKernelEx(&cfg, k_fused<true>, T, W, B, ppc, bb, ep);
-    }
     if (e == cudaSuccess && merged) {
         *bar_base = bb + g;
         *epoch = ep;
