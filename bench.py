@@ -252,22 +252,37 @@ def run_ours(args):
         # touched bytes exceed 2x the L2, so every batch's inputs and output
         # slots are L2-cold ("inputs larger than L2"); the SA table stays
         # resident, as in a running gateway.
+        # The slots are launched through a batch ring (nba_ipsec_ring_run: the
+        # R process_batch launches recorded once as a CUDA graph, no host launch
+        # per batch); steps % R batches go through process_batch directly.
         dbs = [db] + [clone_batch(db) for _ in range(n_rot(b) - 1)]
+        R = len(dbs)
+        ring = t.ring([(*d.args(), b.n) for d in dbs]) if not args.no_ring else None
         runs = [(lambda d=d: t.process(*d.args(), n=b.n)) for d in dbs]
-        for k in range(2 * len(runs)):
-            runs[k % len(runs)]()
+
+        def timed_batches(k_steps):
+            if ring is not None:
+                ring.run(k_steps // R)
+                for k in range(k_steps % R):
+                    runs[k]()
+            else:
+                for k in range(k_steps):
+                    runs[k % R]()
+
+        timed_batches(2 * R)
         torch.cuda.synchronize()
         barrier()
         e_all = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
         with ClockSampler(local) as clk:
             torch.cuda.synchronize()
             e_all[0].record()
-            for k in range(steps):
-                runs[k % len(runs)]()
+            timed_batches(steps)
             e_all[1].record()
             torch.cuda.synchronize()
         barrier()
         tot_ms = e_all[0].elapsed_time(e_all[1])
+        if ring is not None:
+            ring.close()
         # isolated batches (secondary): L2 flushed before each batch, one event
         # pair per batch (includes the launch and event-pair floor)
         iso_steps = min(steps, 50)
@@ -669,7 +684,9 @@ def run_ours(args):
                        "l2": f"inputs larger than L2: batches rotate over {res['n_rot']} device copies "
                              "(> 2x L2 touched per rotation), SA table resident",
                        "timing": "K back-to-back batches on the launching stream between one CUDA "
-                                 "event pair, max over ranks",
+                                 "event pair, max over ranks" + ("" if args.no_ring else
+                                 "; launched through the batch ring (nba_ipsec_ring_run, one CUDA "
+                                 "graph of the rotation's process_batch launches)"),
                        "pipeline": ("fused" if args.pipeline in (None, 0) else "unfused") +
                                    f" ({res['launches'] // args.steps} launch(es) per step)"},
             "roofline": roof,
@@ -836,6 +853,8 @@ def main():
     ap.add_argument("--no-inbound", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-alb", action="store_true")
+    ap.add_argument("--no-ring", action="store_true",
+                    help="launch every timed batch with process_batch instead of the ring graph")
     ap.add_argument("--cpu-seconds", type=float, default=3.0)
     args = ap.parse_args()
     if args.warmup < 3:

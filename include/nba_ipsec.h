@@ -144,6 +144,27 @@ int nba_ipsec_read_counters(nba_ipsec_sa_table *t, nba_ipsec_counters *out, void
  * nba_ipsec_sa_params.seq for exact resume).  host_seq has n_sa entries.
  * Synchronises `cuda_stream`. */
 int nba_ipsec_read_sa_seq(nba_ipsec_sa_table *t, uint32_t *host_seq, void *cuda_stream);
+/* ---- batch rings: a fixed set of batch slots as one CUDA graph --------------
+ *
+ * A gateway that recycles a fixed pool of packet-buffer slots (PAPER.md:
+ * 327-343: datablocks are byte ranges of the packets in their buffers) calls
+ * the path on the same n_slots batches over and over.  ring_create records
+ * nba_ipsec_process_batch for every slot, in slot order, into a CUDA graph
+ * (the path keeps all per-batch state -- SA counters, the one-kernel path's
+ * barrier base and batch epoch -- on the device, so the recorded launches stay
+ * valid); ring_run enqueues n_rounds passes over the slots on cuda_stream:
+ * the same results as n_rounds x n_slots process_batch calls, without a host
+ * launch per batch.  The slots' DEVICE pointers and sizes are fixed at
+ * creation (their contents may change between runs, in stream order).
+ * NBA_IPSEC_EINVAL for NULL arguments, n_slots == 0 or > 4096, a slot that
+ * process_batch would reject, or while profiling / tracing is enabled.  The
+ * ring must be destroyed before its table. */
+typedef struct nba_ipsec_ring nba_ipsec_ring;
+int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, uint32_t n_slots,
+                          nba_ipsec_ring **out);
+int nba_ipsec_ring_run(nba_ipsec_ring *r, uint32_t n_rounds, void *cuda_stream);
+int nba_ipsec_ring_destroy(nba_ipsec_ring *r);   /* NULL -> OK */
+
 /* Overwrite the per-SA sequence numbers with host_seq[0..n_sa) (HOST memory):
  * the hand-over of an SA's counter when another device takes it over
  * (reading L7) or an exact resume.  Enqueued on `cuda_stream`

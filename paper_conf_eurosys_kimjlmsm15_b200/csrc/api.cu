@@ -51,7 +51,10 @@ struct nba_ipsec_sa_table {
     // host-I/O pipeline (process_batch_host): IO_DEPTH staging slots, copy-in /
     // compute / copy-out on three internal streams so batch k+1's H2D and batch
     // k-1's D2H overlap batch k's kernels
-    static constexpr int IO_DEPTH = 2;
+#ifndef NBA_IO_DEPTH
+#define NBA_IO_DEPTH 2
+#endif
+    static constexpr int IO_DEPTH = NBA_IO_DEPTH;
     struct IoSlot {
         uint8_t *in = nullptr, *out = nullptr;
         uint32_t *meta = nullptr;   // in_off, sa_idx, out_off (u32) + in_len, out_len (u16)
@@ -365,6 +368,82 @@ int nba_ipsec_process_batch(nba_ipsec_sa_table *t, const nba_ipsec_batch *b, voi
     BatchArgs B{b->in_buf, b->in_off, b->in_len, sa_idx, b->out_buf, b->out_off, b->out_len,
                 b->n_pkts, t->flow_table, t->flow_mask};
     return enqueue(t, B, st);
+}
+
+// ---- batch rings: the path for a fixed set of batch slots as one CUDA graph ----
+
+struct nba_ipsec_ring {
+    nba_ipsec_sa_table *t = nullptr;
+    cudaGraph_t graph = nullptr;
+    cudaGraphExec_t exec = nullptr;
+    uint32_t n_slots = 0;
+};
+
+int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, uint32_t n_slots,
+                          nba_ipsec_ring **out)
+{
+    if (!t || !slots || !out || n_slots == 0 || n_slots > 4096) return NBA_IPSEC_EINVAL;
+    *out = nullptr;
+    if (t->prof || t->W.trace) return NBA_IPSEC_EINVAL;   // host-side per-batch state
+    for (uint32_t i = 0; i < n_slots; i++) {
+        const nba_ipsec_batch &b = slots[i];
+        if (b.n_pkts > t->max_batch || !b.in_buf || !b.in_off || !b.in_len || !b.out_buf ||
+            !b.out_off || !b.out_len || (!b.sa_idx && !t->flow_table))
+            return NBA_IPSEC_EINVAL;
+    }
+    DeviceGuard g(t->device);
+    nba_ipsec_ring *r = new (std::nothrow) nba_ipsec_ring();
+    if (!r) return NBA_IPSEC_ENOMEM;
+    r->t = t;
+    r->n_slots = n_slots;
+    cudaStream_t cs = nullptr;
+    cudaError_t e = cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
+    int rc = NBA_IPSEC_OK;
+    if (e == cudaSuccess) e = cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal);
+    if (e == cudaSuccess) {
+        // every launch of the path reads its per-batch state (SA counters, the
+        // one-kernel path's barrier base and epoch) from the device, so the
+        // captured kernels are valid for any number of replays
+        for (uint32_t i = 0; i < n_slots && rc == NBA_IPSEC_OK; i++)
+            if (slots[i].n_pkts) rc = nba_ipsec_process_batch(t, &slots[i], cs);
+        cudaGraph_t gr = nullptr;
+        const cudaError_t e2 = cudaStreamEndCapture(cs, &gr);
+        if (e2 != cudaSuccess && rc == NBA_IPSEC_OK) rc = NBA_IPSEC_ECUDA;
+        r->graph = gr;
+        if (rc == NBA_IPSEC_OK && cudaGraphInstantiate(&r->exec, r->graph, 0) != cudaSuccess)
+            rc = NBA_IPSEC_ECUDA;
+    } else {
+        rc = NBA_IPSEC_ECUDA;
+    }
+    if (cs) cudaStreamDestroy(cs);
+    if (rc != NBA_IPSEC_OK) {
+        nba_ipsec_ring_destroy(r);
+        return rc;
+    }
+    *out = r;
+    return NBA_IPSEC_OK;
+}
+
+int nba_ipsec_ring_run(nba_ipsec_ring *r, uint32_t n_rounds, void *cuda_stream)
+{
+    if (!r || !r->exec) return NBA_IPSEC_EINVAL;
+    DeviceGuard g(r->t->device);
+    cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    for (uint32_t k = 0; k < n_rounds; k++)
+        if (cudaGraphLaunch(r->exec, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
+    return NBA_IPSEC_OK;
+}
+
+int nba_ipsec_ring_destroy(nba_ipsec_ring *r)
+{
+    if (!r) return NBA_IPSEC_OK;
+    {
+        DeviceGuard g(r->t->device);
+        if (r->exec) cudaGraphExecDestroy(r->exec);
+        if (r->graph) cudaGraphDestroy(r->graph);
+    }
+    delete r;
+    return NBA_IPSEC_OK;
 }
 
 static void io_free(nba_ipsec_sa_table *t)

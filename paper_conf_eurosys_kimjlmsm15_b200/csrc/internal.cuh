@@ -66,7 +66,11 @@ struct DevWork {
 };
 
 constexpr int CTL_TICKET = 0, CTL_TOTAL_REC = 1, CTL_TOTAL_BLK = 2, CTL_WORK = 3,
-              CTL_BAR_COUNT = 4, CTL_BAR_GEN = 5, CTL_BAR_MONO = 6;
+              CTL_BAR_COUNT = 4, CTL_BAR_GEN = 5, CTL_BAR_MONO = 6,
+              // one-kernel fused path: arrivals before the current launch and the
+              // last batch epoch, kept on the device so launches need no host
+              // state (graph replay)
+              CTL_BAR_BASE = 7, CTL_EPOCH = 8;
 constexpr int NBINS = 32;   // HMAC bins by number of inner SHA-1 blocks (2..25)
 
 struct BatchArgs {

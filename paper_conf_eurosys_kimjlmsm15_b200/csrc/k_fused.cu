@@ -331,8 +331,16 @@ __device__ __forceinline__ uint32_t merged_local_rank(const DevWork &W, FusedLo 
 // ---------------------------------------------------------------- the kernel
 template <bool MERGED>
 __global__ void __launch_bounds__(F_THREADS, 1)
-k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uint32_t epoch)
+k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base_h, uint32_t epoch_h)
 {
+    // one-kernel path: barrier base and batch epoch from the device (read by
+    // every thread before its CTA arrives at the grid barrier; CTA 0 advances
+    // them after the barrier, when every CTA has read them)
+    uint32_t bar_base = bar_base_h, epoch = epoch_h;
+    if (MERGED) {
+        bar_base = *reinterpret_cast<volatile uint32_t *>(&W.ctl[CTL_BAR_BASE]);
+        epoch = (*reinterpret_cast<volatile uint32_t *>(&W.ctl[CTL_EPOCH]) % 0x7fffffffu) + 1u;
+    }
     extern __shared__ __align__(16) uint8_t smem[];
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
     const uint32_t n_sa = T.n_sa;
@@ -434,6 +442,10 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
             if (!NBA_EXPAND_MID) expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
         }
         grid_wait(&W.ctl[CTL_BAR_MONO], bar_base + G);
+        if (blockIdx.x == 0 && tid == 0) {
+            W.ctl[CTL_BAR_BASE] = bar_base + G;
+            W.ctl[CTL_EPOCH] = epoch;
+        }
         if (tr && tid == 0) tr[5] = gtimer();
         // 4. row scans publish epoch-tagged bases; each packet polls its own
         //    (SA, CTA) entry
@@ -462,7 +474,10 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base, uin
         const uint32_t q32 = (sa_me != INVALID_SA) ? L.seq[pk] : 0u;
         const bool ok = q32 != 0u;   // a valid sequence number is never 0
         // 6. the lane's packet
-        if (have) {
+#ifndef NBA_PROLOGUE_ONLY      // debug A/B: 1 skips the lane phase (timing of the prologue alone)
+#define NBA_PROLOGUE_ONLY 0
+#endif
+        if (have && !NBA_PROLOGUE_ONLY) {
             const uint32_t pkt = p_begin + pk;
             if (ok) {
                 esp_packet(T, B, L, H, lane4r, tid, sa_me, info, q32, inoff, L.outoff[pk], pp,
@@ -617,16 +632,13 @@ cudaError_t launch_fused(const DevTable &T, const DevWork &W, const BatchArgs &B
     }
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    const uint32_t bb = *bar_base;
-    // epoch: 31-bit batch tag of the in-kernel prologue's published bases (never 0)
-    const uint32_t ep = merged ? ((*epoch % 0x7fffffffu) + 1u) : 0u;
-    cudaError_t e = merged ? cudaLaunchKernelEx(&cfg, k_fused<true>, T, W, B, ppc, bb, ep)
-                           : cudaLaunchKernelEx(&cfg, k_fused<false>, T, W, B, ppc, bb, ep);
-    if (e == cudaSuccess && merged) {
-        *bar_base = bb + g;
-        *epoch = ep;
-    }
-    return e;
+    // the one-kernel path keeps its barrier base and 31-bit batch epoch on the
+    // device (W.ctl), so a launch carries no per-batch host state and can be
+    // replayed from a CUDA graph; the host copies only count launches
+    (void)bar_base;
+    (void)epoch;
+    return merged ? cudaLaunchKernelEx(&cfg, k_fused<true>, T, W, B, ppc, 0u, 0u)
+                  : cudaLaunchKernelEx(&cfg, k_fused<false>, T, W, B, ppc, 0u, 0u);
 }
 
 cudaError_t setup_fused_attributes()

@@ -123,6 +123,9 @@ def _load():
         "nba_ipsec_route_pack_map": (i32, [vp, vp, vp, vp, u32, u32, vp, u32, vp, vp, vp, vp, vp, vp,
                                            vp]),
         "nba_ipsec_write_sa_seq": (i32, [vp, P(u32), vp]),
+        "nba_ipsec_ring_create": (i32, [vp, P(Batch), u32, P(vp)]),
+        "nba_ipsec_ring_run": (i32, [vp, u32, vp]),
+        "nba_ipsec_ring_destroy": (i32, [vp]),
         "nba_ipsec_alb_default_params": (None, [P(AlbParams)]),
         "nba_ipsec_alb_create": (i32, [P(AlbParams), P(vp)]),
         "nba_ipsec_alb_observe": (i32, [vp, u64, u64, u64, P(u32)]),
@@ -260,6 +263,11 @@ class SATable:
             raise ValueError(f"need {self.n_sa} sequence numbers")
         _check(lib.nba_ipsec_write_sa_seq(self._h, a.ctypes.data_as(ctypes.POINTER(ctypes.c_uint32)),
                                           _stream_handle(stream)), "nba_ipsec_write_sa_seq")
+
+    def ring(self, slots):
+        """nba_ipsec_ring_create: `slots` = sequence of (in_buf, in_off, in_len,
+        sa_idx, out_buf, out_off, out_len, n) device-tensor tuples."""
+        return Ring(self, slots)
 
     def set_pipeline(self, pipeline: int):
         _check(lib.nba_ipsec_set_pipeline(self._h, int(pipeline)), "nba_ipsec_set_pipeline")
@@ -409,6 +417,37 @@ def route_pack_map(in_buf, in_off, in_len, sa_global, n, n_sa_total, sa_map, wor
                                         _ptr(send_sa), _ptr(dest_counts), _ptr(dest_bytes),
                                         _stream_handle(stream)),
            "nba_ipsec_route_pack_map")
+
+
+class Ring:
+    """A fixed set of batch slots recorded as one CUDA graph (nba_ipsec_ring_*)."""
+
+    def __init__(self, table, slots):
+        arr = (Batch * len(slots))()
+        self._keep = list(slots)            # the tensors must outlive the ring
+        for i, sl in enumerate(slots):
+            *bufs, n = sl
+            arr[i] = Batch(*(_ptr(x) for x in bufs), int(n))
+        self.table = table
+        self.n_slots = len(slots)
+        self._h = ctypes.c_void_p()
+        _check(lib.nba_ipsec_ring_create(table._h, arr, len(slots), ctypes.byref(self._h)),
+               "nba_ipsec_ring_create")
+
+    def run(self, n_rounds: int = 1, stream=None):
+        _check(lib.nba_ipsec_ring_run(self._h, int(n_rounds), _stream_handle(stream)),
+               "nba_ipsec_ring_run")
+
+    def close(self):
+        if self._h:
+            lib.nba_ipsec_ring_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 # -- adaptive split of the SAs across devices (SURVEY §8(f) f4) -----------------

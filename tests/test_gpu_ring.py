@@ -1,0 +1,89 @@
+"""GPU parity for batch rings (nba_ipsec_ring_*): a fixed set of batch slots
+recorded as one CUDA graph and replayed must give exactly what the same
+sequence of process_batch calls gives -- here against the oracle processing
+the slots' batches in ring order, round after round (the slots are refilled
+between runs, in stream order), including the final SA counters and the
+device counters; and replay equals stream launches on a second table."""
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_eurosys_kimjlmsm15_b200 import gen
+
+pytestmark = pytest.mark.gpu
+
+
+def _slot(db):
+    return (db.in_buf, db.in_off, db.in_len, db.sa_idx, db.out_buf, db.out_off, db.out_len, db.n)
+
+
+@pytest.mark.parametrize("sizes,n_sa", [((64, "imix", 1514), 1024), (("imix", "imix"), 7)])
+def test_ring_rounds_match_oracle(sizes, n_sa):
+    import torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    p = gen.make_sas(n_sa, cfg_id=51)
+    n = 20000
+    sas = oracle.make_sas(p)
+    ctr = oracle.Counters()
+    with nba_ipsec.SATable(p, device=0, max_batch=n) as t:
+        dbs = [device.to_device(gen.make_batch(n, s, n_sa, cfg_id=51, batch=i), "cuda")
+               for i, s in enumerate(sizes)]
+        ring = t.ring([_slot(d) for d in dbs])
+        for rnd in range(3):
+            # refill the slots with this round's traffic (stream order), run one pass
+            hb = [gen.make_batch(n, s, n_sa, cfg_id=51, batch=100 * rnd + i)
+                  for i, s in enumerate(sizes)]
+            hb[0].sa_idx[::97] = n_sa + 1                      # some invalid SAs
+            for d, b in zip(dbs, hb):
+                d.in_buf.copy_(torch.from_numpy(b.in_buf))
+                d.in_len.copy_(torch.from_numpy(b.in_len.view(np.int16)))
+                d.sa_idx.copy_(torch.from_numpy(b.sa_idx.view(np.int32)))
+            ring.run(1)
+            torch.cuda.synchronize()
+            for d, b in zip(dbs, hb):
+                o_out, o_len, _ = oracle.process_batch(sas, n_sa, b, n_threads=8, counters=ctr)
+                g_out, g_len = device.fetch(d)
+                assert np.array_equal(g_len, o_len)
+                for i in np.nonzero(o_len)[0][::7]:
+                    a, L = int(b.out_off[i]), int(o_len[i])
+                    assert np.array_equal(g_out[a:a + L], o_out[a:a + L])
+        assert np.array_equal(t.sa_seq(), oracle.sa_seq(sas, n_sa))
+        assert t.counters() == ctr.as_dict()
+        ring.close()
+
+
+def test_ring_replay_equals_stream_launches():
+    import torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    p = gen.make_sas(1024, cfg_id=52)
+    b = gen.make_batch(65536, 64, 1024, cfg_id=52)
+    da = [device.to_device(b, "cuda") for _ in range(3)]
+    db_ = [device.to_device(b, "cuda") for _ in range(3)]
+    with nba_ipsec.SATable(p, device=0, max_batch=b.n) as ta, \
+            nba_ipsec.SATable(p, device=0, max_batch=b.n) as tb:
+        ring = ta.ring([_slot(d) for d in da])
+        s = torch.cuda.Stream()
+        ring.run(4, stream=s)
+        s.synchronize()
+        for _ in range(4):
+            for d in db_:
+                tb.process(*d.args(), n=b.n)
+        torch.cuda.synchronize()
+        for x, y in zip(da, db_):
+            assert torch.equal(x.out_buf, y.out_buf) and torch.equal(x.out_len, y.out_len)
+        assert np.array_equal(ta.sa_seq(), tb.sa_seq())
+        assert ta.counters() == tb.counters()
+        ring.close()
+
+
+def test_ring_rejects_bad_slots():
+    import ctypes
+    from paper_conf_eurosys_kimjlmsm15_b200 import nba_ipsec
+    p = gen.make_sas(4, cfg_id=53)
+    with nba_ipsec.SATable(p, device=0, max_batch=100) as t:
+        h = ctypes.c_void_p()
+        bad = (nba_ipsec.Batch * 1)()
+        bad[0] = nba_ipsec.Batch(0, 0, 0, 0, 0, 0, 0, 50)     # NULL buffers
+        assert nba_ipsec.lib.nba_ipsec_ring_create(t._h, bad, 1, ctypes.byref(h)) == nba_ipsec.EINVAL
+        assert nba_ipsec.lib.nba_ipsec_ring_create(t._h, bad, 0, ctypes.byref(h)) == nba_ipsec.EINVAL
+        assert nba_ipsec.lib.nba_ipsec_ring_destroy(None) == nba_ipsec.OK
