@@ -582,6 +582,39 @@ def run_ours(args):
             tot += e0.elapsed_time(e1)
         ms = tot / steps
         moved = 2 * int(b.in_len.astype(np.int64).sum()) + b.n * (4 + 2 + 4 + 2 + 4 + 12)
+        # the same routing with the data written straight into 8 owners' receive
+        # buffers (nba_ipsec_route_dispatch; here all on this GPU, standing in for
+        # peer GPUs' memory over NVLink): no send buffer, no all-to-all
+        from paper_conf_eurosys_kimjlmsm15_b200 import nba_ipsec as _nb
+        cap_b = int(b.in_len.astype(np.int64).sum()) + 64
+        rxs = [redistribute.alloc_rx(b.n, cap_b, dev) for _ in range(8)]
+        table = redistribute.rx_table(rxs, dev)
+        ws = torch.empty(_nb.route_workspace_bytes(b.n, 8), dtype=torch.uint8, device=dev)
+        dcnt = torch.zeros(9, dtype=torch.int64, device=dev)
+        dbyt = torch.zeros(9, dtype=torch.int64, device=dev)
+        disp = lambda: _nb.route_dispatch(db.in_buf, db.in_off, db.in_len, db.sa_idx, b.n,  # noqa: E731
+                                          len(p.spi), None, 8, ws, table, b.n, cap_b, dcnt, dbyt)
+        for _ in range(warmup):
+            flush.zero_()
+            disp()
+        torch.cuda.synchronize()
+        tot_d = 0.0
+        for k in range(steps):
+            flush.zero_()
+            e0.record()
+            disp()
+            e1.record()
+            torch.cuda.synchronize()
+            tot_d += e0.elapsed_time(e1)
+        ms_d = tot_d / steps
+        moved_d = 2 * int(b.in_len.astype(np.int64).sum()) + b.n * (4 + 2 + 4 + 4 + 2 + 4 + 4)
+        out["dispatch_8_owners"] = {"ms_per_step": ms_d, "mpps": b.n / (ms_d * 1e-3) / 1e6,
+                                    "roofline": {"bound": "hbm", "unit": "GB/s", "peak": peaks["hbm_gbs"],
+                                                 "achieved": moved_d / (ms_d * 1e-3) / 1e9,
+                                                 "frac": moved_d / (ms_d * 1e-3) / 1e9 / peaks["hbm_gbs"]},
+                                    "note": "route + write into 8 owners' receive buffers in one "
+                                            "pass (single-GPU stand-in for NVLink peers)"}
+        del rxs
         out["route_pack_8_owners"] = {"ms_per_step": ms, "mpps": b.n / (ms * 1e-3) / 1e6,
                                       "roofline": {"bound": "hbm", "unit": "GB/s", "peak": peaks["hbm_gbs"],
                                                    "achieved": moved / (ms * 1e-3) / 1e9,

@@ -283,6 +283,35 @@ int nba_ipsec_route_pack_map(const uint8_t *in_buf, const uint32_t *in_off, cons
                              uint8_t *send_buf, uint16_t *send_len, uint32_t *send_sa,
                              uint64_t *dest_counts, uint64_t *dest_bytes, void *cuda_stream);
 
+/* Single-ingress dispatch straight into the owners' receive buffers: the
+ * routing of route_pack_map (same destinations, same owner-local order) and
+ * the data movement in one pass -- one warp per packet writes its bytes,
+ * offset, length and local SA index into rx[owner], which may be this
+ * device's memory or a peer GPU's mapped over NVLink (cudaIpcOpenMemHandle /
+ * peer access), so no send buffer and no collective sit between routing and
+ * the owners' process_batch.  rx: DEVICE array of `world` descriptors whose
+ * pointers are valid on the calling device; receiver d gets its packets at
+ * positions 0..count-1 (batch order), offsets into its buf, and
+ * count[0] = packets, count[1] = bytes (written by the dispatch).  Each
+ * receiver needs cap_pkts >= n_pkts entries and cap_bytes >= the batch's bytes
+ * (larger batches are not written past the capacity).  Single ingress: one
+ * dispatch per receive buffer at a time; the receivers may read them after the
+ * caller's stream work completed (e.g. stream sync + a process-group barrier).
+ * sa_map as in route_pack_map (NULL: owner = s mod world).  dest_counts /
+ * dest_bytes (DEVICE, world + 1) as in route_pack.  4 kernel launches. */
+typedef struct {
+    uint8_t  *buf;          /* received packet bytes */
+    uint32_t *off;          /* per packet: offset into buf */
+    uint16_t *len;          /* per packet: length */
+    uint32_t *sa;           /* per packet: local SA index */
+    uint64_t *count;        /* [2]: packets, bytes */
+} nba_ipsec_peer_rx;
+int nba_ipsec_route_dispatch(const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
+                             const uint32_t *sa_global, uint32_t n_pkts, uint32_t n_sa_total,
+                             const uint32_t *sa_map, uint32_t world, void *workspace,
+                             const nba_ipsec_peer_rx *rx, uint64_t cap_pkts, uint64_t cap_bytes,
+                             uint64_t *dest_counts, uint64_t *dest_bytes, void *cuda_stream);
+
 /* ---- adaptive split of the SAs across devices -------------
  *
  * PAPER.md:351-365 (§3.4): NBA's load balancer hill-climbs the offloading

@@ -804,6 +804,28 @@ int nba_ipsec_route_pack_map(const uint8_t *in_buf, const uint32_t *in_off, cons
                : NBA_IPSEC_ECUDA;
 }
 
+int nba_ipsec_route_dispatch(const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
+                             const uint32_t *sa_global, uint32_t n_pkts, uint32_t n_sa_total,
+                             const uint32_t *sa_map, uint32_t world, void *workspace,
+                             const nba_ipsec_peer_rx *rx, uint64_t cap_pkts, uint64_t cap_bytes,
+                             uint64_t *dest_counts, uint64_t *dest_bytes, void *cuda_stream)
+{
+    if (world == 0 || world > 8 || n_pkts > NBA_IPSEC_MAX_BATCH) return NBA_IPSEC_EINVAL;
+    if (!dest_counts || !dest_bytes || !rx || cap_pkts < n_pkts) return NBA_IPSEC_EINVAL;
+    if (n_pkts && (!in_buf || !in_off || !in_len || !sa_global || !workspace))
+        return NBA_IPSEC_EINVAL;
+    cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    // (an empty batch runs only the scan, which writes every receiver's zero counts)
+    if (!workspace) return NBA_IPSEC_EINVAL;
+    return launch_route(in_buf, in_off, in_len, sa_global, n_pkts, n_sa_total, sa_map, world,
+                        workspace, nullptr, nullptr, nullptr,
+                        reinterpret_cast<unsigned long long *>(dest_counts),
+                        reinterpret_cast<unsigned long long *>(dest_bytes), st, rx, cap_pkts,
+                        cap_bytes) == cudaSuccess
+               ? NBA_IPSEC_OK
+               : NBA_IPSEC_ECUDA;
+}
+
 int nba_ipsec_route_pack(const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
                          const uint32_t *sa_global, uint32_t n_pkts, uint32_t n_sa_total,
                          uint32_t world, void *workspace, uint8_t *send_buf, uint16_t *send_len,

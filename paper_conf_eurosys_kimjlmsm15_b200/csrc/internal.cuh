@@ -7,6 +7,8 @@
 
 #ifdef __CUDACC__
 #include <cuda_runtime.h>
+
+#include "nba_ipsec.h"
 #endif
 
 namespace nba {
@@ -187,7 +189,8 @@ cudaError_t launch_route(const uint8_t *in_buf, const uint32_t *in_off, const ui
                          const uint32_t *sa, uint32_t n, uint32_t n_sa_total,
                          const uint32_t *sa_map, uint32_t world, void *ws, uint8_t *send_buf, uint16_t *send_len, uint32_t *send_sa,
                          unsigned long long *dest_counts, unsigned long long *dest_bytes,
-                         cudaStream_t st);
+                         cudaStream_t st, const nba_ipsec_peer_rx *rx = nullptr,
+                         unsigned long long cap_pkts = 0, unsigned long long cap_bytes = 0);
 
 // --- small device helpers ---------------------------------------------------
 __device__ __forceinline__ uint32_t bswap32(uint32_t x) { return __byte_perm(x, 0, 0x0123); }

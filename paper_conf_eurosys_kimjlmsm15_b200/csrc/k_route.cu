@@ -89,7 +89,7 @@ k_route_tiles(RouteWork R, const uint16_t *in_len, const uint32_t *sa, uint32_t 
 // One CTA: exclusive scans over tiles per destination, then region bases.
 __global__ void __launch_bounds__(256)
 k_route_scan(RouteWork R, uint32_t n_tiles, uint32_t world, unsigned long long *dest_counts,
-             unsigned long long *dest_bytes)
+             unsigned long long *dest_bytes, const nba_ipsec_peer_rx *rx)
 {
     __shared__ unsigned long long s_tc[RT_MAX_WORLD + 1], s_tb[RT_MAX_WORLD + 1];
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
@@ -131,6 +131,10 @@ k_route_scan(RouteWork R, uint32_t n_tiles, uint32_t world, unsigned long long *
             R.base[(world + 1u) + k] = bb;
             dest_counts[k] = s_tc[k];
             dest_bytes[k] = s_tb[k];
+            if (rx && k < world) {   // the receiver's counts, in its own memory
+                rx[k].count[0] = s_tc[k];
+                rx[k].count[1] = s_tb[k];
+            }
             bc += s_tc[k];
             bb += s_tb[k];
         }
@@ -163,6 +167,49 @@ k_route_pack(RouteWork R, const uint8_t *in_buf, const uint32_t *in_off, const u
     }
 }
 
+// Single-ingress dispatch (nba_ipsec_route_dispatch): one warp per packet
+// writes it straight into its owner's receive buffers -- own memory or a
+// peer's, mapped over NVLink -- at the owner-local position (tile prefix +
+// rank within the tile, batch order), with its offset, length and local SA.
+// 16-byte stores where source and destination share alignment, bytes else.
+__global__ void __launch_bounds__(256)
+k_route_dispatch(RouteWork R, const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
+                 const uint32_t *sa, const uint32_t *sa_map, uint32_t n, uint32_t world,
+                 const nba_ipsec_peer_rx *rx, unsigned long long cap_pkts,
+                 unsigned long long cap_bytes)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (i >= n) return;
+    const uint32_t d = R.dest[i];
+    if (d >= world) return;                           // not routable: not sent
+    const uint32_t tile = i / RT_TILE;
+    const unsigned long long pos = R.tcnt[tile * (world + 1u) + d] + R.rank[i];
+    const unsigned long long boff = R.tbyt[tile * (world + 1u) + d] + R.brank[i];
+    const uint32_t len = in_len[i];
+    if (pos >= cap_pkts || boff + len > cap_bytes) return;   // contract violated: never write OOB
+    const nba_ipsec_peer_rx r = rx[d];
+    const uint8_t *src = in_buf + in_off[i];
+    uint8_t *dst = r.buf + boff;
+    const uintptr_t sa16 = reinterpret_cast<uintptr_t>(src) & 15u;
+    if (sa16 == (reinterpret_cast<uintptr_t>(dst) & 15u)) {
+        const uint32_t head = min(len, (16u - (uint32_t)sa16) & 15u);
+        const uint32_t nv = (len - head) >> 4;
+        if (lane < head) dst[lane] = src[lane];
+        const uint4 *s4 = reinterpret_cast<const uint4 *>(src + head);
+        uint4 *d4 = reinterpret_cast<uint4 *>(dst + head);
+        for (uint32_t v = lane; v < nv; v += 32u) d4[v] = s4[v];
+        for (uint32_t b = head + 16u * nv + lane; b < len; b += 32u) dst[b] = src[b];
+    } else {
+        for (uint32_t b = lane; b < len; b += 32u) dst[b] = src[b];
+    }
+    if (lane == 0) {
+        r.off[pos] = (uint32_t)boff;
+        r.len[pos] = (uint16_t)len;
+        r.sa[pos] = sa_map ? (__ldg(sa_map + sa[i]) & 0xFFFFFFu) : sa[i] / world;
+    }
+}
+
 size_t route_workspace_bytes(uint32_t max_pkts, uint32_t world)
 {
     const size_t tiles = (max_pkts + RT_TILE - 1) / RT_TILE;
@@ -173,7 +220,8 @@ cudaError_t launch_route(const uint8_t *in_buf, const uint32_t *in_off, const ui
                          const uint32_t *sa, uint32_t n, uint32_t n_sa_total,
                          const uint32_t *sa_map, uint32_t world, void *ws, uint8_t *send_buf, uint16_t *send_len, uint32_t *send_sa,
                          unsigned long long *dest_counts, unsigned long long *dest_bytes,
-                         cudaStream_t st)
+                         cudaStream_t st, const nba_ipsec_peer_rx *rx, unsigned long long cap_pkts,
+                         unsigned long long cap_bytes)
 {
     const uint32_t tiles = (n + RT_TILE - 1) / RT_TILE;
     uint8_t *p = static_cast<uint8_t *>(ws);
@@ -189,10 +237,16 @@ cudaError_t launch_route(const uint8_t *in_buf, const uint32_t *in_off, const ui
     R.tcnt = reinterpret_cast<uint32_t *>(take((size_t)tiles * (world + 1) * 4));
     R.tbyt = reinterpret_cast<unsigned long long *>(take((size_t)tiles * (world + 1) * 8));
     R.base = reinterpret_cast<unsigned long long *>(take(2ull * (world + 1) * 8));
-    k_route_tiles<<<tiles, RT_TILE, 0, st>>>(R, in_len, sa, n, n_sa_total, sa_map, world);
-    k_route_scan<<<1, 256, 0, st>>>(R, tiles, world, dest_counts, dest_bytes);
-    k_route_pack<<<(n * 32u + 255u) / 256u, 256, 0, st>>>(R, in_buf, in_off, in_len, sa, sa_map, n, world,
-                                                         send_buf, send_len, send_sa);
+    if (tiles) k_route_tiles<<<tiles, RT_TILE, 0, st>>>(R, in_len, sa, n, n_sa_total, sa_map, world);
+    k_route_scan<<<1, 256, 0, st>>>(R, tiles, world, dest_counts, dest_bytes, rx);
+    if (n == 0) return cudaGetLastError();
+    if (rx)
+        k_route_dispatch<<<(n * 32u + 255u) / 256u, 256, 0, st>>>(R, in_buf, in_off, in_len, sa,
+                                                                 sa_map, n, world, rx, cap_pkts,
+                                                                 cap_bytes);
+    else
+        k_route_pack<<<(n * 32u + 255u) / 256u, 256, 0, st>>>(R, in_buf, in_off, in_len, sa, sa_map,
+                                                             n, world, send_buf, send_len, send_sa);
     return cudaGetLastError();
 }
 

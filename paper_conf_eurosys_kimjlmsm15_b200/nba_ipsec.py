@@ -123,6 +123,8 @@ def _load():
         "nba_ipsec_route_pack_map": (i32, [vp, vp, vp, vp, u32, u32, vp, u32, vp, vp, vp, vp, vp, vp,
                                            vp]),
         "nba_ipsec_write_sa_seq": (i32, [vp, P(u32), vp]),
+        "nba_ipsec_route_dispatch": (i32, [vp, vp, vp, vp, u32, u32, vp, u32, vp, vp, u64, u64, vp,
+                                           vp, vp]),
         "nba_ipsec_ring_create": (i32, [vp, P(Batch), u32, P(vp)]),
         "nba_ipsec_ring_run": (i32, [vp, u32, vp]),
         "nba_ipsec_ring_destroy": (i32, [vp]),
@@ -448,6 +450,18 @@ class Ring:
             self.close()
         except Exception:
             pass
+
+
+def route_dispatch(in_buf, in_off, in_len, sa_global, n, n_sa_total, sa_map, world, workspace,
+                   rx_table, cap_pkts, cap_bytes, dest_counts, dest_bytes, stream=None):
+    """nba_ipsec_route_dispatch: route + write straight into the owners' receive
+    buffers (rx_table: device array of nba_ipsec_peer_rx descriptors)."""
+    _check(lib.nba_ipsec_route_dispatch(_ptr(in_buf), _ptr(in_off), _ptr(in_len), _ptr(sa_global),
+                                        int(n), int(n_sa_total), _ptr(sa_map), int(world),
+                                        _ptr(workspace), _ptr(rx_table), int(cap_pkts),
+                                        int(cap_bytes), _ptr(dest_counts), _ptr(dest_bytes),
+                                        _stream_handle(stream)),
+           "nba_ipsec_route_dispatch")
 
 
 # -- adaptive split of the SAs across devices (SURVEY §8(f) f4) -----------------

@@ -9,6 +9,11 @@ shard: owner = s mod world) before the ESP path runs there.
   3. each owner runs nba_ipsec_process_batch on what it received (local SA
      indices, packets back to back).
 
+Without the collective: nba_ipsec_route_dispatch routes AND writes every
+packet straight into its owner's receive buffers (PeerRx) -- on this GPU or a
+peer GPU's memory mapped over NVLink (CUDA IPC: torch shares CUDA tensors
+between processes) -- in one pass; see dispatch() below.
+
 This module is plumbing only (sizes, splits, offsets); the routing and packing
 arithmetic is in the kernels.
 """
@@ -113,3 +118,54 @@ def local_views(p: Packed, d: int, out_pad: int = 64):
     out_len = torch.empty(max(n, 1), dtype=torch.int16, device=dev)
     return (n, in_off.to(torch.int32), p.length[c0:], p.sa[c0:], out_off.to(torch.int32), out_len,
             out_buf)
+
+
+# ---- single-ingress dispatch over peer memory (no send buffer, no NCCL) --------
+
+@dataclasses.dataclass
+class PeerRx:
+    """One owner's receive buffers (device tensors on the owner's GPU; another
+    process may hold them through CUDA IPC)."""
+    buf: torch.Tensor        # uint8 [cap_bytes]
+    off: torch.Tensor        # int32 [cap_pkts]
+    length: torch.Tensor     # int16 [cap_pkts]
+    sa: torch.Tensor         # int32 [cap_pkts]
+    count: torch.Tensor      # int64 [2]: packets, bytes
+
+
+def alloc_rx(cap_pkts: int, cap_bytes: int, device) -> PeerRx:
+    return PeerRx(buf=torch.empty(max(cap_bytes, 16), dtype=torch.uint8, device=device),
+                  off=torch.empty(max(cap_pkts, 1), dtype=torch.int32, device=device),
+                  length=torch.empty(max(cap_pkts, 1), dtype=torch.int16, device=device),
+                  sa=torch.empty(max(cap_pkts, 1), dtype=torch.int32, device=device),
+                  count=torch.zeros(2, dtype=torch.int64, device=device))
+
+
+def rx_table(rxs, device) -> torch.Tensor:
+    """Device array of nba_ipsec_peer_rx descriptors (5 pointers each), with the
+    pointers as seen by THIS process (own or IPC-mapped tensors)."""
+    ptrs = [[r.buf.data_ptr(), r.off.data_ptr(), r.length.data_ptr(), r.sa.data_ptr(),
+             r.count.data_ptr()] for r in rxs]
+    return torch.tensor(ptrs, dtype=torch.int64).view(-1).to(device)
+
+
+def dispatch(db, n: int, n_sa_total: int, world: int, table: torch.Tensor, cap_pkts: int,
+             cap_bytes: int, sa_map=None, stream=None):
+    """Route a device batch with GLOBAL SA indices and write each packet into its
+    owner's receive buffers (nba_ipsec_route_dispatch).  Returns the per-owner
+    (packets, bytes) counts (read back; synchronises)."""
+    from . import nba_ipsec
+    dev = db.in_buf.device
+    ws = torch.empty(nba_ipsec.route_workspace_bytes(max(n, 1), world), dtype=torch.uint8, device=dev)
+    dc = torch.zeros(world + 1, dtype=torch.int64, device=dev)
+    dbytes = torch.zeros(world + 1, dtype=torch.int64, device=dev)
+    nba_ipsec.route_dispatch(db.in_buf, db.in_off, db.in_len, db.sa_idx, n, n_sa_total, sa_map,
+                             world, ws, table, cap_pkts, cap_bytes, dc, dbytes, stream=stream)
+    return dc.cpu().tolist()[:world], dbytes.cpu().tolist()[:world]
+
+
+def received_batch(rx: PeerRx):
+    """(n, in_buf, in_off, in_len, sa_idx) of what the dispatch wrote into rx, as
+    process_batch arguments (device tensors; n read back)."""
+    n = int(rx.count[0].item())
+    return n, rx.buf, rx.off, rx.length, rx.sa
