@@ -758,8 +758,10 @@ def run_e2e(args, rank, world, local, dev, barrier):
     import torch
     from paper_conf_eurosys_kimjlmsm15_b200 import nba_ipsec
     size = CFG_SIZE[args.config]
+    # packed datagrams in, output slots of D + 53 bytes (the largest ESP
+    # overhead, NBA_IPSEC_MAX_OVERHEAD) out: the fewest bytes over PCIe
     p, b = shard.rank_workload(args.config, PKTS_PER_GPU, size, N_SA_TOTAL, rank, world,
-                               layout="packed")
+                               layout="packed", out_pad=53)
     t = nba_ipsec.SATable(p, device=local, max_batch=PKTS_PER_GPU)
     if args.pipeline is not None:
         t.set_pipeline(args.pipeline)

@@ -110,12 +110,13 @@ def _csum16(words: np.ndarray) -> np.ndarray:
 
 def make_batch(n: int, size, n_sa: int, cfg_id: int = 0, rank: int = 0, batch: int = 0,
                locality: int = 1, layout: str = "slots", in_len_override=None,
-               sa_idx_override=None) -> Batch:
+               sa_idx_override=None, out_pad: int = 64) -> Batch:
     """Synthesise one batch of n packets.
 
     layout="slots": slot stride 2048, headroom 128 -> in_off = 2048 i + 142
     (≡ 14 mod 16, deliberately unaligned), same formula for out_off in a
-    separate pool.  layout="packed": datagrams back to back (for host I/O).
+    separate pool.  layout="packed": datagrams back to back (for host I/O),
+    output slots of D + out_pad bytes (out_pad >= 53, the largest ESP overhead).
     locality=k: SA chosen per run of k consecutive packets (flow locality)."""
     r = rng_for(cfg_id, rank, batch)
     L = frame_sizes(n, size, r)
@@ -136,7 +137,7 @@ def make_batch(n: int, size, n_sa: int, cfg_id: int = 0, rank: int = 0, batch: i
     elif layout == "packed":
         in_off = np.concatenate([[0], np.cumsum(Dc)[:-1]]) if n else np.zeros(0, np.int64)
         pool = int(Dc.sum()) + 16
-        cap = Dc + 64
+        cap = Dc + out_pad
         out_off = np.concatenate([[0], np.cumsum(cap)[:-1]]) if n else np.zeros(0, np.int64)
         out_pool = int(cap.sum()) + 16
     else:
