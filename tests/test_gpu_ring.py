@@ -87,3 +87,31 @@ def test_ring_rejects_bad_slots():
         assert nba_ipsec.lib.nba_ipsec_ring_create(t._h, bad, 1, ctypes.byref(h)) == nba_ipsec.EINVAL
         assert nba_ipsec.lib.nba_ipsec_ring_create(t._h, bad, 0, ctypes.byref(h)) == nba_ipsec.EINVAL
         assert nba_ipsec.lib.nba_ipsec_ring_destroy(None) == nba_ipsec.OK
+
+
+@pytest.mark.parametrize("n,pipeline", [(100_000, None), (30_000, 1)])
+def test_ring_two_kernel_and_unfused_paths(n, pipeline):
+    """Batches larger than one super-round per CTA take the two-kernel path
+    (prologue + fused, chained by programmatic dependent launch); the unfused
+    pipeline launches five kernels: both recorded in the ring's graph must still
+    equal the oracle over rounds."""
+    import torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    n_sa = 1024
+    p = gen.make_sas(n_sa, cfg_id=54)
+    b = gen.make_batch(n, "imix", n_sa, cfg_id=54)
+    sas = oracle.make_sas(p)
+    with nba_ipsec.SATable(p, device=0, max_batch=n) as t:
+        if pipeline is not None:
+            t.set_pipeline(pipeline)
+        d = device.to_device(b, "cuda")
+        ring = t.ring([_slot(d)])
+        ring.run(2)
+        torch.cuda.synchronize()
+        oracle.process_batch(sas, n_sa, b, n_threads=8)
+        o_out, o_len, _ = oracle.process_batch(sas, n_sa, b, n_threads=8)
+        g_out, g_len = device.fetch(d)
+        assert np.array_equal(g_len, o_len)
+        assert np.array_equal(g_out, o_out)
+        assert np.array_equal(t.sa_seq(), oracle.sa_seq(sas, n_sa))
+        ring.close()
