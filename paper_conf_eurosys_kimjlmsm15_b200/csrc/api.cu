@@ -424,6 +424,46 @@ int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, u
     return NBA_IPSEC_OK;
 }
 
+int nba_ipsec_ring_create_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batch *slots,
+                                  uint32_t n_slots, nba_ipsec_ring **out)
+{
+    if (!t || !slots || !out || n_slots == 0 || n_slots > 4096) return NBA_IPSEC_EINVAL;
+    *out = nullptr;
+    if (t->prof || t->W.trace || !t->in_enabled) return NBA_IPSEC_EINVAL;
+    for (uint32_t i = 0; i < n_slots; i++) {
+        const nba_ipsec_in_batch &b = slots[i];
+        if (b.n_pkts > t->max_batch || !b.in_buf || !b.in_off || !b.in_len || !b.sa_idx ||
+            !b.out_buf || !b.out_off || !b.out_len)
+            return NBA_IPSEC_EINVAL;
+    }
+    DeviceGuard g(t->device);
+    nba_ipsec_ring *r = new (std::nothrow) nba_ipsec_ring();
+    if (!r) return NBA_IPSEC_ENOMEM;
+    r->t = t;
+    r->n_slots = n_slots;
+    cudaStream_t cs = nullptr;
+    int rc = NBA_IPSEC_OK;
+    if (cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
+        rc = NBA_IPSEC_ECUDA;
+    } else {
+        for (uint32_t i = 0; i < n_slots && rc == NBA_IPSEC_OK; i++)
+            if (slots[i].n_pkts) rc = nba_ipsec_process_inbound(t, &slots[i], cs);
+        cudaGraph_t gr = nullptr;
+        if (cudaStreamEndCapture(cs, &gr) != cudaSuccess && rc == NBA_IPSEC_OK) rc = NBA_IPSEC_ECUDA;
+        r->graph = gr;
+        if (rc == NBA_IPSEC_OK && cudaGraphInstantiate(&r->exec, r->graph, 0) != cudaSuccess)
+            rc = NBA_IPSEC_ECUDA;
+    }
+    if (cs) cudaStreamDestroy(cs);
+    if (rc != NBA_IPSEC_OK) {
+        nba_ipsec_ring_destroy(r);
+        return rc;
+    }
+    *out = r;
+    return NBA_IPSEC_OK;
+}
+
 int nba_ipsec_ring_run(nba_ipsec_ring *r, uint32_t n_rounds, void *cuda_stream)
 {
     if (!r || !r->exec) return NBA_IPSEC_EINVAL;

@@ -158,6 +158,7 @@ __device__ __forceinline__ uint32_t esp_in_packet(const DevTable &T, const InBat
 // The same arithmetic as the three-kernel path (in_replay.cuh), so the same
 // result as the sequential receiver.
 constexpr uint32_t CTLI_BAR = 4;   // S.ctl word: monotonic barrier arrivals
+constexpr uint32_t CTLI_BASE = 5;  // S.ctl word: arrivals before the current one-kernel launch
 
 __device__ __forceinline__ void in_merged_tail(const DevTable &T, const InState &S, const InBatchArgs &B,
                                                FusedLo &L, uint8_t *tabs, uint32_t p_begin,
@@ -221,6 +222,8 @@ __device__ __forceinline__ void in_merged_tail(const DevTable &T, const InState 
     __syncthreads();
     grid_arrive(&S.ctl[CTLI_BAR]);
     grid_wait(&S.ctl[CTLI_BAR], bar_base + G);
+    // every CTA has read the base (before arriving): advance it for the next launch
+    if (cta == 0 && tid == 0) S.ctl[CTLI_BASE] = bar_base + 2u * G;
     // hash inserts (the hash was cleared before the barrier) and the row scans
     if (inA) replay_hash_insert(S, key, q, i, hmask);
     scan_all_rows(S, n_sa, cta * NW + warp, G * NW, G, lane);
@@ -264,9 +267,13 @@ __device__ __forceinline__ void in_merged_tail(const DevTable &T, const InState 
 
 template <bool MERGED>
 __global__ void __launch_bounds__(F_THREADS, 1)
-k_in_fused(DevTable T, InState S, InBatchArgs B, uint32_t ppc, uint32_t hmask, uint32_t bar_base)
+k_in_fused(DevTable T, InState S, InBatchArgs B, uint32_t ppc, uint32_t hmask, uint32_t bar_base_h)
 {
     extern __shared__ __align__(16) uint8_t smem[];
+    // one-kernel form: the barrier base lives on the device (launches carry no
+    // host state and can be recorded in a graph); read before arriving
+    const uint32_t bar_base =
+        MERGED ? *reinterpret_cast<volatile uint32_t *>(&S.ctl[CTLI_BASE]) : bar_base_h;
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
     const uint32_t n_sa = T.n_sa;
 
@@ -391,10 +398,9 @@ cudaError_t launch_in_fused(const DevTable &T, const InState &S, const InBatchAr
     attr[0].val.cooperative = 1;
     cfg.attrs = attr;
     cfg.numAttrs = merged ? 1 : 0;
-    const uint32_t bb = *bar_base;
-    cudaError_t e = merged ? cudaLaunchKernelEx(&cfg, k_in_fused<true>, T, S, B, ppc, hmask, bb)
-                           : cudaLaunchKernelEx(&cfg, k_in_fused<false>, T, S, B, ppc, hmask, bb);
-    if (e == cudaSuccess && merged) *bar_base = bb + 2u * g;
+    (void)bar_base;   // the one-kernel form keeps its barrier base on the device
+    cudaError_t e = merged ? cudaLaunchKernelEx(&cfg, k_in_fused<true>, T, S, B, ppc, hmask, 0u)
+                           : cudaLaunchKernelEx(&cfg, k_in_fused<false>, T, S, B, ppc, hmask, 0u);
     return e;
 }
 

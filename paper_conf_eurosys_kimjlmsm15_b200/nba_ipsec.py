@@ -127,6 +127,7 @@ def _load():
                                            vp, vp]),
         "nba_ipsec_ring_create": (i32, [vp, P(Batch), u32, P(vp)]),
         "nba_ipsec_ring_run": (i32, [vp, u32, vp]),
+        "nba_ipsec_ring_create_inbound": (i32, [vp, P(InBatch), u32, P(vp)]),
         "nba_ipsec_ring_destroy": (i32, [vp]),
         "nba_ipsec_alb_default_params": (None, [P(AlbParams)]),
         "nba_ipsec_alb_create": (i32, [P(AlbParams), P(vp)]),
@@ -270,6 +271,11 @@ class SATable:
         """nba_ipsec_ring_create: `slots` = sequence of (in_buf, in_off, in_len,
         sa_idx, out_buf, out_off, out_len, n) device-tensor tuples."""
         return Ring(self, slots)
+
+    def ring_inbound(self, slots):
+        """nba_ipsec_ring_create_inbound: `slots` = sequence of (in_buf, in_off,
+        in_len, sa_idx, out_buf, out_off, out_len, status-or-None, n)."""
+        return Ring(self, slots, inbound=True)
 
     def set_pipeline(self, pipeline: int):
         _check(lib.nba_ipsec_set_pipeline(self._h, int(pipeline)), "nba_ipsec_set_pipeline")
@@ -424,17 +430,18 @@ def route_pack_map(in_buf, in_off, in_len, sa_global, n, n_sa_total, sa_map, wor
 class Ring:
     """A fixed set of batch slots recorded as one CUDA graph (nba_ipsec_ring_*)."""
 
-    def __init__(self, table, slots):
-        arr = (Batch * len(slots))()
+    def __init__(self, table, slots, inbound=False):
+        kind = InBatch if inbound else Batch
+        arr = (kind * len(slots))()
         self._keep = list(slots)            # the tensors must outlive the ring
         for i, sl in enumerate(slots):
             *bufs, n = sl
-            arr[i] = Batch(*(_ptr(x) for x in bufs), int(n))
+            arr[i] = kind(*(_ptr(x) for x in bufs), int(n))
         self.table = table
         self.n_slots = len(slots)
         self._h = ctypes.c_void_p()
-        _check(lib.nba_ipsec_ring_create(table._h, arr, len(slots), ctypes.byref(self._h)),
-               "nba_ipsec_ring_create")
+        create = lib.nba_ipsec_ring_create_inbound if inbound else lib.nba_ipsec_ring_create
+        _check(create(table._h, arr, len(slots), ctypes.byref(self._h)), "nba_ipsec_ring_create")
 
     def run(self, n_rounds: int = 1, stream=None):
         _check(lib.nba_ipsec_ring_run(self._h, int(n_rounds), _stream_handle(stream)),

@@ -115,3 +115,48 @@ def test_ring_two_kernel_and_unfused_paths(n, pipeline):
         assert np.array_equal(g_out, o_out)
         assert np.array_equal(t.sa_seq(), oracle.sa_seq(sas, n_sa))
         ring.close()
+
+
+def test_inbound_ring_equals_stream_launches_and_oracle():
+    """ESP inbound slots in a ring: status, inner bytes, lengths, windows and
+    counters equal process_inbound from the stream and the oracle's receiver."""
+    import torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    n_sa, n = 64, 5000
+    p = gen.make_sas(n_sa, cfg_id=55)
+    sas = oracle.make_sas(p)
+    win = oracle.make_windows(sas, n_sa)
+    esp = []
+    for j in range(3):                                   # three consecutive outbound batches
+        b = gen.make_batch(n, "imix", n_sa, cfg_id=55, batch=j)
+        e_out, e_len, _ = oracle.process_batch(sas, n_sa, b)
+        ib = gen.esp_batch(e_out, b.out_off, e_len, b.sa_idx, np.arange(n))
+        esp.append(ib)
+    sas_in = oracle.make_sas(p)
+    ref = [oracle.process_inbound(sas_in, win, n_sa, ib) for ib in esp]
+    with nba_ipsec.SATable(p, device=0, max_batch=n) as ta, \
+            nba_ipsec.SATable(p, device=0, max_batch=n) as tb:
+        ta.enable_inbound()
+        tb.enable_inbound()
+        da = [device.to_device(ib, "cuda") for ib in esp]
+        db_ = [device.to_device(ib, "cuda") for ib in esp]
+        sa_ = [torch.zeros(ib.n, dtype=torch.uint8, device="cuda") for ib in esp]
+        sb_ = [torch.zeros(ib.n, dtype=torch.uint8, device="cuda") for ib in esp]
+        ring = ta.ring_inbound([(*d.args(), st, ib.n) for d, st, ib in zip(da, sa_, esp)])
+        ring.run(1)
+        for d, st, ib in zip(db_, sb_, esp):
+            tb.process_inbound(*d.args(), status=st, n=ib.n)
+        torch.cuda.synchronize()
+        for k, (ib, (o_out, o_len, o_st, _)) in enumerate(zip(esp, ref)):
+            ga, la = device.fetch(da[k])
+            gb, lb = device.fetch(db_[k])
+            assert np.array_equal(sa_[k].cpu().numpy(), o_st) and np.array_equal(sb_[k].cpu().numpy(), o_st)
+            assert np.array_equal(la, o_len) and np.array_equal(lb, o_len)
+            for i in np.nonzero(o_len)[0][::5]:
+                a, L = int(ib.out_off[i]), int(o_len[i])
+                assert np.array_equal(ga[a:a + L], o_out[a:a + L])
+        ta_top, ta_bmp = ta.replay_window()
+        o_top, o_bmp = oracle.window_state(win, n_sa)
+        assert np.array_equal(ta_top, o_top) and np.array_equal(ta_bmp, o_bmp)
+        assert ta.in_counters() == tb.in_counters()
+        ring.close()
