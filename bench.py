@@ -252,9 +252,9 @@ def run_ours(args):
         # touched bytes exceed 2x the L2, so every batch's inputs and output
         # slots are L2-cold ("inputs larger than L2"); the SA table stays
         # resident, as in a running gateway.
-        # The slots are launched through a batch ring (nba_ipsec_ring_run: the
-        # R process_batch launches recorded once as a CUDA graph, no host launch
-        # per batch); steps % R batches go through process_batch directly.
+        # The slots are launched through a batch ring (nba_ipsec_ring_run: one
+        # persistent cooperative launch walks all batches of a run; no host
+        # launch per batch); steps % R batches go through process_batch.
         dbs = [db] + [clone_batch(db) for _ in range(n_rot(b) - 1)]
         R = len(dbs)
         ring = t.ring([(*d.args(), b.n) for d in dbs]) if not args.no_ring else None
@@ -740,8 +740,8 @@ def run_ours(args):
                              "(> 2x L2 touched per rotation), SA table resident",
                        "timing": "K back-to-back batches on the launching stream between one CUDA "
                                  "event pair, max over ranks" + ("" if args.no_ring else
-                                 "; launched through the batch ring (nba_ipsec_ring_run, one CUDA "
-                                 "graph of the rotation's process_batch launches)"),
+                                 "; launched through the batch ring (nba_ipsec_ring_run over the "
+                                 "rotation's slots: one persistent cooperative launch per run)"),
                        "pipeline": ("fused" if args.pipeline in (None, 0) else "unfused") +
                                    f" ({res['launches'] // args.steps} launch(es) per step)"},
             "roofline": roof,

@@ -148,13 +148,17 @@ int nba_ipsec_read_sa_seq(nba_ipsec_sa_table *t, uint32_t *host_seq, void *cuda_
  *
  * A gateway that recycles a fixed pool of packet-buffer slots (PAPER.md:
  * 327-343: datablocks are byte ranges of the packets in their buffers) calls
- * the path on the same n_slots batches over and over.  ring_create records
- * nba_ipsec_process_batch for every slot, in slot order, into a CUDA graph
- * (the path keeps all per-batch state -- SA counters, the one-kernel path's
- * barrier base and batch epoch -- on the device, so the recorded launches stay
- * valid); ring_run enqueues n_rounds passes over the slots on cuda_stream:
- * the same results as n_rounds x n_slots process_batch calls, without a host
- * launch per batch.  The slots' DEVICE pointers and sizes are fixed at
+ * the path on the same n_slots batches over and over.  ring_run enqueues
+ * n_rounds passes over the slots, in slot order, on cuda_stream: the same
+ * results as n_rounds x n_slots process_batch calls, without a host launch
+ * per batch.  When every slot takes the one-kernel path (fused pipeline,
+ * n_pkts <= 512 x SMs) a run is ONE persistent cooperative launch that walks
+ * all its batches, keeping the AES tables in shared memory and letting a CTA
+ * start the next batch while others finish (set NBA_IPSEC_RING_GRAPH to force
+ * the other form); otherwise ring_create records process_batch for every slot
+ * into a CUDA graph (the path keeps all per-batch state -- SA counters, the
+ * one-kernel path's barrier base and batch epoch -- on the device, so the
+ * recorded launches stay valid) and a run replays it n_rounds times.  The slots' DEVICE pointers and sizes are fixed at
  * creation (their contents may change between runs, in stream order).
  * NBA_IPSEC_EINVAL for NULL arguments, n_slots == 0 or > 4096, a slot that
  * process_batch would reject, or while profiling / tracing is enabled.  The

@@ -377,6 +377,10 @@ struct nba_ipsec_ring {
     cudaGraph_t graph = nullptr;
     cudaGraphExec_t exec = nullptr;
     uint32_t n_slots = 0;
+    // persistent form (every slot takes the one-kernel path): the slots'
+    // arguments on the device and the second count-matrix buffer
+    BatchArgs *d_slots = nullptr;
+    uint16_t *hist_b = nullptr;
 };
 
 int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, uint32_t n_slots,
@@ -396,6 +400,30 @@ int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, u
     if (!r) return NBA_IPSEC_ENOMEM;
     r->t = t;
     r->n_slots = n_slots;
+    // persistent form: one cooperative launch walks all batches of a run
+    bool persist = !std::getenv("NBA_IPSEC_RING_GRAPH") && t->pipeline == NBA_IPSEC_PIPE_FUSED &&
+                   t->allow_merged;
+    for (uint32_t i = 0; i < n_slots && persist; i++)
+        persist = slots[i].n_pkts > 0 && fused_merged_ok(slots[i].n_pkts, t->grid_fused);
+    if (persist) {
+        std::vector<BatchArgs> hb(n_slots);
+        for (uint32_t i = 0; i < n_slots; i++) {
+            const nba_ipsec_batch &b = slots[i];
+            hb[i] = BatchArgs{b.in_buf, b.in_off, b.in_len, b.sa_idx, b.out_buf, b.out_off,
+                              b.out_len, b.n_pkts, t->flow_table, t->flow_mask};
+        }
+        const size_t hb_bytes = (size_t)t->grid_fused * t->n_sa * sizeof(uint16_t);
+        if (cudaMalloc(&r->d_slots, n_slots * sizeof(BatchArgs)) != cudaSuccess ||
+            cudaMalloc(&r->hist_b, hb_bytes) != cudaSuccess ||
+            cudaMemset(r->hist_b, 0, hb_bytes) != cudaSuccess ||
+            cudaMemcpy(r->d_slots, hb.data(), n_slots * sizeof(BatchArgs), cudaMemcpyHostToDevice) !=
+                cudaSuccess) {
+            nba_ipsec_ring_destroy(r);
+            return NBA_IPSEC_ENOMEM;
+        }
+        *out = r;
+        return NBA_IPSEC_OK;
+    }
     cudaStream_t cs = nullptr;
     cudaError_t e = cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking);
     int rc = NBA_IPSEC_OK;
@@ -466,9 +494,18 @@ int nba_ipsec_ring_create_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batc
 
 int nba_ipsec_ring_run(nba_ipsec_ring *r, uint32_t n_rounds, void *cuda_stream)
 {
-    if (!r || !r->exec) return NBA_IPSEC_EINVAL;
+    if (!r || (!r->exec && !r->d_slots)) return NBA_IPSEC_EINVAL;
     DeviceGuard g(r->t->device);
     cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
+    if (r->d_slots) {
+        if (n_rounds == 0) return NBA_IPSEC_OK;
+        if ((uint64_t)n_rounds * r->n_slots > 0xffffffffull) return NBA_IPSEC_EINVAL;
+        nba_ipsec_sa_table *t = r->t;
+        return launch_fused_ring(t->T, t->W, r->d_slots, r->n_slots, n_rounds * r->n_slots,
+                                 r->hist_b, t->grid_fused, st) == cudaSuccess
+                   ? NBA_IPSEC_OK
+                   : NBA_IPSEC_ECUDA;
+    }
     for (uint32_t k = 0; k < n_rounds; k++)
         if (cudaGraphLaunch(r->exec, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
     return NBA_IPSEC_OK;
@@ -481,6 +518,9 @@ int nba_ipsec_ring_destroy(nba_ipsec_ring *r)
         DeviceGuard g(r->t->device);
         if (r->exec) cudaGraphExecDestroy(r->exec);
         if (r->graph) cudaGraphDestroy(r->graph);
+        if (r->d_slots || r->hist_b) cudaDeviceSynchronize();   // a run may still be in flight
+        if (r->d_slots) cudaFree(r->d_slots);
+        if (r->hist_b) cudaFree(r->hist_b);
     }
     delete r;
     return NBA_IPSEC_OK;

@@ -329,18 +329,23 @@ __device__ __forceinline__ uint32_t merged_local_rank(const DevWork &W, FusedLo 
 }
 
 // ---------------------------------------------------------------- the kernel
-template <bool MERGED>
-__global__ void __launch_bounds__(F_THREADS, 1)
-k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base_h, uint32_t epoch_h)
+__host__ __device__ __forceinline__ uint32_t fused_ppc_hd(uint32_t n, uint32_t grid)
 {
-    // one-kernel path: barrier base and batch epoch from the device (read by
-    // every thread before its CTA arrives at the grid barrier; CTA 0 advances
-    // them after the barrier, when every CTA has read them)
-    uint32_t bar_base = bar_base_h, epoch = epoch_h;
-    if (MERGED) {
-        bar_base = *reinterpret_cast<volatile uint32_t *>(&W.ctl[CTL_BAR_BASE]);
-        epoch = (*reinterpret_cast<volatile uint32_t *>(&W.ctl[CTL_EPOCH]) % 0x7fffffffu) + 1u;
-    }
+    uint32_t ppc = (n + grid - 1) / grid;
+    ppc = (ppc + 31u) & ~31u;
+    return ppc < 32u ? 32u : ppc;
+}
+#define fused_ppc(n, g) fused_ppc_hd((uint32_t)(n), (uint32_t)(g))
+
+// One batch through the kernel (the body of k_fused; k_fused_ring runs it for
+// a sequence of batches).  bar_base / epoch: this batch's grid-barrier base and
+// epoch; stage_tables: copy the T-tables into shared memory first (a ring's
+// later batches find them there).
+template <bool MERGED>
+__device__ __forceinline__ void fused_body(const DevTable &T, const DevWork &W, const BatchArgs &B,
+                                           uint32_t ppc, uint32_t bar_base, uint32_t epoch,
+                                           bool stage_tables)
+{
     extern __shared__ __align__(16) uint8_t smem[];
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
     const uint32_t n_sa = T.n_sa;
@@ -388,7 +393,7 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base_h, u
     uint32_t old0 = 0;
     if (MERGED) old0 = scan_first_old(T, blockIdx.x * (F_THREADS / 32u) + warp,
                                       gridDim.x * (F_THREADS / 32u), gridDim.x, lane);
-    aes_tables_to_smem(tabs, T.te0);
+    if (stage_tables) aes_tables_to_smem(tabs, T.te0);
     if (tr && tid == 0) tr[2] = gtimer();
     if (tid < 4) L.cnt[tid] = 0ull;
     if (tid < NBINS) L.bins[tid] = 0;   // re-zeroed after each use (length_sort)
@@ -596,14 +601,48 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base_h, u
     if (tr && tid == 0) atomicMax(W.trace + W.trace_pro + 48u, gtimer());   // CTA end
 }
 
+template <bool MERGED>
+__global__ void __launch_bounds__(F_THREADS, 1)
+k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base_h, uint32_t epoch_h)
+{
+    // one-kernel path: barrier base and batch epoch from the device (read by
+    // every thread before its CTA arrives at the grid barrier; CTA 0 advances
+    // them after the barrier, when every CTA has read them)
+    uint32_t bar_base = bar_base_h, epoch = epoch_h;
+    if (MERGED) {
+        bar_base = *reinterpret_cast<volatile uint32_t *>(&W.ctl[CTL_BAR_BASE]);
+        epoch = (*reinterpret_cast<volatile uint32_t *>(&W.ctl[CTL_EPOCH]) % 0x7fffffffu) + 1u;
+    }
+    fused_body<MERGED>(T, W, B, ppc, bar_base, epoch, true);
+}
+
+// A batch ring as ONE persistent launch (nba_ipsec_ring_run): the grid (one
+// CTA per SM) walks n_batches batches, slot bi mod n_slots, keeping the
+// T-tables in shared memory; a CTA that finishes batch bi starts bi + 1's
+// metadata phase while the others finish, and waits at that batch's grid
+// barrier.  The per-(SA, CTA) count matrix alternates between two buffers by
+// batch parity: batch bi's row scans re-zero buffer bi & 1 after every CTA
+// passed barrier bi, and batch bi + 2 writes it only after barrier bi + 1.
+__global__ void __launch_bounds__(F_THREADS, 1)
+k_fused_ring(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slots, uint32_t n_batches,
+             uint16_t *hist_b)
+{
+    const uint32_t base0 = *reinterpret_cast<volatile uint32_t *>(&W.ctl[CTL_BAR_BASE]);
+    const uint32_t ep0 = *reinterpret_cast<volatile uint32_t *>(&W.ctl[CTL_EPOCH]);
+    const uint32_t G = gridDim.x;
+    for (uint32_t bi = 0; bi < n_batches; bi++) {
+        const BatchArgs B = slots[bi % n_slots];
+        DevWork Wb = W;
+        if (bi & 1u) Wb.hist16 = hist_b;
+        const uint32_t epoch = ((ep0 + bi) % 0x7fffffffu) + 1u;
+        fused_body<true>(T, Wb, B, fused_ppc(B.n, G), base0 + bi * G, epoch, bi == 0);
+        __syncthreads();   // shared memory is reused by the next batch
+    }
+}
+
 int fused_grid(int num_sms) { return num_sms; }
 
-uint32_t fused_ppc(uint32_t n, int grid)
-{
-    uint32_t ppc = (n + grid - 1) / grid;
-    ppc = (ppc + 31u) & ~31u;
-    return ppc < 32u ? 32u : ppc;
-}
+
 
 bool fused_merged_ok(uint32_t n, int grid)
 {
@@ -641,8 +680,28 @@ cudaError_t launch_fused(const DevTable &T, const DevWork &W, const BatchArgs &B
                   : cudaLaunchKernelEx(&cfg, k_fused<false>, T, W, B, ppc, 0u, 0u);
 }
 
+cudaError_t launch_fused_ring(const DevTable &T, const DevWork &W, const BatchArgs *slots,
+                              uint32_t n_slots, uint32_t n_batches, uint16_t *hist_b, int grid,
+                              cudaStream_t st)
+{
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(F_THREADS);
+    cfg.dynamicSmemBytes = F_SMEM;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeCooperative;   // grid barriers inside
+    attr[0].val.cooperative = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, k_fused_ring, T, W, slots, n_slots, n_batches, hist_b);
+}
+
 cudaError_t setup_fused_attributes()
 {
+    cudaError_t e0 = cudaFuncSetAttribute(k_fused_ring, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                          (int)F_SMEM);
+    if (e0 != cudaSuccess) return e0;
     cudaError_t e = cudaFuncSetAttribute(k_fused<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          (int)F_SMEM);
     if (e != cudaSuccess) return e;

@@ -160,3 +160,42 @@ def test_inbound_ring_equals_stream_launches_and_oracle():
         assert np.array_equal(ta_top, o_top) and np.array_equal(ta_bmp, o_bmp)
         assert ta.in_counters() == tb.in_counters()
         ring.close()
+
+
+@pytest.mark.parametrize("force_graph", [False, True])
+def test_ring_flow_table_slots_persistent_and_graph(force_graph, monkeypatch):
+    """Slots without SA indices (the one-kernel path looks each packet's SA up in
+    the flow table) in a ring -- the persistent form (one launch walks all
+    batches) and, forced, the graph form -- equal the oracle over 3 rounds."""
+    import torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    if force_graph:
+        monkeypatch.setenv("NBA_IPSEC_RING_GRAPH", "1")
+    else:
+        monkeypatch.delenv("NBA_IPSEC_RING_GRAPH", raising=False)
+    n_sa, n = 256, 30000
+    p = gen.make_sas(n_sa, cfg_id=56)
+    f = gen.make_flows(3000, n_sa, cfg_id=56)
+    bs = []
+    for k in range(2):
+        b = gen.make_batch(n, "imix", n_sa, cfg_id=56, batch=k)
+        gen.apply_flows(b, f, cfg_id=56, batch=k, miss=0.05)
+        b.sa_idx = oracle.flow_lookup(f, b)
+        bs.append(b)
+    sas = oracle.make_sas(p)
+    with nba_ipsec.SATable(p, device=0, max_batch=n) as t:
+        t.set_flow_table(f)
+        ds = [device.to_device(b, "cuda") for b in bs]
+        ring = t.ring([(d.in_buf, d.in_off, d.in_len, None, d.out_buf, d.out_off, d.out_len, n)
+                       for d in ds])
+        ring.run(3)
+        torch.cuda.synchronize()
+        for _ in range(2):
+            for b in bs:
+                oracle.process_batch(sas, n_sa, b, n_threads=8)
+        for d, b in zip(ds, bs):
+            o_out, o_len, _ = oracle.process_batch(sas, n_sa, b, n_threads=8)
+            g_out, g_len = device.fetch(d)
+            assert np.array_equal(g_len, o_len) and np.array_equal(g_out, o_out)
+        assert np.array_equal(t.sa_seq(), oracle.sa_seq(sas, n_sa))
+        ring.close()
