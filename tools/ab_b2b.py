@@ -29,16 +29,25 @@ for cfg, size in [c for c in ((2, 64), (3, 1514), (4, "imix")) if str(c[0]) in o
                                      out_len=torch.empty_like(db.out_len)) for _ in range(R - 1)]
     t = nba_ipsec.SATable(p, max_batch=b.n)
     K = 200
-    for k in range(2 * R):
-        t.process(*dbs[k %% R].args(), n=b.n)
+    ring = t.ring([(*d.args(), b.n) for d in dbs]) if os.environ.get("AB_RING") else None
+    def go(k_steps):
+        if ring is not None:
+            ring.run(k_steps // R)
+            for k in range(k_steps %% R):
+                t.process(*dbs[k].args(), n=b.n)
+        else:
+            for k in range(k_steps):
+                t.process(*dbs[k %% R].args(), n=b.n)
+    go(2 * R)
     torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record()
-    for k in range(K):
-        t.process(*dbs[k %% R].args(), n=b.n)
+    go(K)
     e1.record()
     torch.cuda.synchronize()
     print(f"  cfg {cfg}: {e0.elapsed_time(e1) / K * 1e3:.2f} us/step (R={R})", flush=True)
+    if ring is not None:
+        ring.close()
     t.close()
     del dbs
 '''
