@@ -157,14 +157,15 @@ def kernel_roofline(name, ms_per_launch, w, peaks):
     alu_peak = SM_COUNT * ALU_LANES_PER_CLK_SM * f / 1e9            # Gop/s
     aes_ops = w["aes_blocks"] * AES_ALU_OPS_PER_BLOCK
     sha_ops = w["sha1_compressions"] * SHA1_ALU_OPS_PER_COMPRESSION
-    if name in ("fused", "aes_ctr", "hmac_sha1"):
-        ops = {"fused": aes_ops + sha_ops, "aes_ctr": aes_ops, "hmac_sha1": sha_ops}[name]
+    if name in ("fused", "fused_ring", "aes_ctr", "hmac_sha1"):
+        ops = {"fused": aes_ops + sha_ops, "fused_ring": aes_ops + sha_ops, "aes_ctr": aes_ops,
+               "hmac_sha1": sha_ops}[name]
         r = {"bound": "alu", "unit": "Gop/s", "achieved": ops / s / 1e9, "peak": alu_peak,
              "peak_basis": f"integer ALU pipe: {ALU_LANES_PER_CLK_SM} lanes/clk/SM x {SM_COUNT} SMs x "
                            f"{peaks['sm_max_mhz']:.0f} MHz (microbenchmarked 63.9 lanes/clk/SM); "
                            f"work = {AES_ALU_OPS_PER_BLOCK} ops/AES block + "
                            f"{SHA1_ALU_OPS_PER_COMPRESSION} ops/SHA-1 compression"}
-        if name in ("fused", "aes_ctr"):
+        if name in ("fused", "fused_ring", "aes_ctr"):
             lds = w["aes_blocks"] * AES_LOOKUPS_PER_BLOCK / s / 1e9
             r["lds_lookups_gps"] = lds
             r["lds_frac"] = lds / (SM_COUNT * LDS_LANES_PER_CLK_SM * f / 1e9)
@@ -281,6 +282,7 @@ def run_ours(args):
             torch.cuda.synchronize()
         barrier()
         tot_ms = e_all[0].elapsed_time(e_all[1])
+        used_ring = ring is not None and steps >= R and not os.environ.get("NBA_IPSEC_RING_GRAPH")
         if ring is not None:
             ring.close()
         # isolated batches (secondary): L2 flushed before each batch, one event
@@ -308,13 +310,15 @@ def run_ours(args):
             kern, nb = t.profile_read()
             t.profile_enable(False)
         t_lpb = t.launches_per_batch()
-        launches = t_lpb * steps
+        # kernels launched in the timed region: one k_fused_ring per ring run
+        # (steps // R batches) plus the remaining batches' own launches
+        launches = (steps // R + (steps % R) * t_lpb) if used_ring else t_lpb * steps
         ctr = t.counters()
         t.close()
         del dbs, runs
         return dict(b=b, p=p, tot_ms=tot_ms, step_ms=step_ms, kern=kern, nb=nb, clk=clk,
                     launches=launches, ctr=ctr, n_rot=n_rot(b),
-                    iso_ms=float(np.mean(step_ms)), lpb=t_lpb)
+                    iso_ms=float(np.mean(step_ms)), lpb=t_lpb, ring=used_ring)
 
     def kernel_times(res, steps):
         """Average duration per launch of each kernel.  One launch per batch
@@ -322,7 +326,9 @@ def run_ours(args):
         pass (includes the inter-kernel gaps, so it is conservative).  Several
         launches: the library's per-kernel CUDA events (profiled pass)."""
         if res["lpb"] == 1 and len(res["kern"]) == 1:
-            return {k: res["tot_ms"] / steps for k in res["kern"]}
+            # through the persistent ring the timed batches ran in k_fused_ring
+            return {(k + "_ring" if res.get("ring") else k): res["tot_ms"] / steps
+                    for k in res["kern"]}
         return {k: v / max(res["nb"], 1) for k, v in res["kern"].items()}
 
     def aggregate(res, steps):

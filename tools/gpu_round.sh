@@ -9,11 +9,15 @@ nvcc -gencode arch=compute_100a,code=sm_100a -O3 -std=c++17 -I paper_conf_eurosy
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw --format=csv > gpurun_out/smi_$TAG.txt
 timeout 900 python bench.py > gpurun_out/bench_$TAG.json 2> gpurun_out/bench_$TAG.err
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv \
-   --log-file gpurun_out/launches_$TAG.csv python bench.py --steps 5 --warmup 3 --no-sweep --no-cpu --no-inbound > /dev/null 2>&1
+   --log-file gpurun_out/launches_$TAG.csv python bench.py --steps 22 --warmup 3 --no-sweep --no-cpu --no-inbound --no-alb > /dev/null 2>&1
 if [ "$2" == "full" ]; then
   for C in 2 3 4; do
     timeout 900 ncu --set full --clock-control none --import-source on -k regex:'k_(fused|prologue)' \
       -s 3 -c 1 -o gpurun_out/prof_${TAG}_c$C -f python tools/run_batches.py --config $C --batches 5 > gpurun_out/ncu_${TAG}_c$C.log 2>&1
+  done
+  for C in 2 3 4; do   # the persistent ring kernel: one run of 4 batch slots (4 batches)
+    timeout 900 ncu --set full --clock-control none --import-source on -k regex:'k_fused_ring' \
+      -c 1 -o gpurun_out/prof_${TAG}_ring_c$C -f python tools/run_batches.py --config $C --batches 1 --ring 4 > gpurun_out/ncu_${TAG}_ring_c$C.log 2>&1
   done
   for C in 2 3 4; do
     timeout 900 ncu --set full --clock-control none --import-source on -k regex:'k_in_' \

@@ -107,6 +107,26 @@ def main(tag):
                                  "source": os.path.basename(rep)}
         lines.append("")
     for c, name in CFG.items():
+        rep = os.path.join(OUT, f"prof_{tag}_ring_{c}.ncu-rep")
+        if not os.path.exists(rep):
+            continue
+        lines += [f"## {name} batch ring (k_fused_ring: ONE launch walks a run of 4 batches; "
+                  "per-batch figures = launch / 4)", "",
+                  "| kernel | us / batch | DRAM rd MB / batch | DRAM wr MB / batch | issue % | ALU % | FMA % | LSU % | L1 data pipe % | warp inst / batch | regs |",
+                  "|---|---|---|---|---|---|---|---|---|---|---|"]
+        for d0 in raw(rep):
+            d = collections.defaultdict(lambda: float("nan"))
+            d.update({m: (v if isinstance(v, float) else float("nan")) for m, v in d0.items()})
+            lines.append(f"| {d0['kernel']} | {d['duration'] * 1e6 / 4:.1f} | {d['dram_read'] / 4e6:.2f} | "
+                         f"{d['dram_write'] / 4e6:.2f} | {d['issue_active_pct']:.1f} | "
+                         f"{d['alu_pipe_pct']:.1f} | {d['fma_pipe_pct']:.1f} | {d['lsu_inst_pct']:.1f} | "
+                         f"{d['l1_data_pipe_pct']:.1f} | {d['warp_instructions'] / 4:.3g} | {d['registers']:.0f} |")
+            kj[f"fused_ring:{name}"] = {"dram_bytes_per_launch": (d["dram_read"] + d["dram_write"]) / 4,
+                                        "ncu_duration_us": d["duration"] * 1e6 / 4,
+                                        "note": "per batch of a 4-batch ring run",
+                                        "source": os.path.basename(rep)}
+        lines.append("")
+    for c, name in CFG.items():
         rep = os.path.join(OUT, f"prof_{tag}_in_{c}.ncu-rep")
         if not os.path.exists(rep):
             continue
