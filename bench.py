@@ -749,7 +749,10 @@ def run_ours(args):
                                  "; launched through the batch ring (nba_ipsec_ring_run over the "
                                  "rotation's slots: one persistent cooperative launch per run)"),
                        "pipeline": ("fused" if args.pipeline in (None, 0) else "unfused") +
-                                   f" ({res['launches'] // args.steps} launch(es) per step)"},
+                                   (f" (k_fused_ring: one launch per ring run of {res['n_rot']} "
+                                    f"batches; {res['launches']} launches for {args.steps} steps)"
+                                    if res.get("ring") else
+                                    f" ({res['launches'] // args.steps} launch(es) per step)")},
             "roofline": roof,
             "kernels": {k: {"ms_per_launch": v["ms_per_launch"], "frac": v["frac"], "unit": v["unit"],
                             "achieved": v["achieved"]} for k, v in kern_roofs.items()},
