@@ -160,9 +160,12 @@ int nba_ipsec_read_sa_seq(nba_ipsec_sa_table *t, uint32_t *host_seq, void *cuda_
  * one-kernel path's barrier base and batch epoch -- on the device, so the
  * recorded launches stay valid) and a run replays it n_rounds times.  The slots' DEVICE pointers and sizes are fixed at
  * creation (their contents may change between runs, in stream order).
+ * The form and the pipeline are fixed when the ring is created.
  * NBA_IPSEC_EINVAL for NULL arguments, n_slots == 0 or > 4096, a slot that
- * process_batch would reject, or while profiling / tracing is enabled.  The
- * ring must be destroyed before its table. */
+ * process_batch would reject, or while profiling / tracing is enabled;
+ * ring_run: NBA_IPSEC_EINVAL once the table's flow table was replaced
+ * (nba_ipsec_set_flow_table) -- re-create the ring.  The ring must be
+ * destroyed before its table. */
 typedef struct nba_ipsec_ring nba_ipsec_ring;
 int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, uint32_t n_slots,
                           nba_ipsec_ring **out);

@@ -199,3 +199,19 @@ def test_ring_flow_table_slots_persistent_and_graph(force_graph, monkeypatch):
             assert np.array_equal(g_len, o_len) and np.array_equal(g_out, o_out)
         assert np.array_equal(t.sa_seq(), oracle.sa_seq(sas, n_sa))
         ring.close()
+
+
+def test_ring_refuses_after_flow_table_replaced():
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    n_sa, n = 16, 1000
+    p = gen.make_sas(n_sa, cfg_id=57)
+    b = gen.make_batch(n, 64, n_sa, cfg_id=57)
+    with nba_ipsec.SATable(p, device=0, max_batch=n) as t:
+        t.set_flow_table(gen.make_flows(100, n_sa, cfg_id=57))
+        d = device.to_device(b, "cuda")
+        ring = t.ring([(*d.args(), n)])
+        ring.run(1)
+        t.set_flow_table(gen.make_flows(200, n_sa, cfg_id=58))
+        with pytest.raises(nba_ipsec.NbaIpsecError):
+            ring.run(1)
+        ring.close()
