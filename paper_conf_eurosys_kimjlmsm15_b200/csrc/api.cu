@@ -87,6 +87,7 @@ struct nba_ipsec_sa_table {
     // flow -> SA lookup (nba_ipsec_set_flow_table)
     uint4 *flow_table = nullptr;
     uint32_t flow_mask = 0;
+    uint64_t flow_gen = 0;         // bumped by every nba_ipsec_set_flow_table
     uint32_t *flow_sa = nullptr;   // [max_batch] SA indices looked up for process_batch
 };
 
@@ -381,7 +382,7 @@ struct nba_ipsec_ring {
     // arguments on the device and the second count-matrix buffer
     BatchArgs *d_slots = nullptr;
     uint16_t *hist_b = nullptr;
-    const uint4 *flow_table = nullptr;   // the table's flow table when recorded
+    uint64_t flow_gen = 0;               // the table's flow-table generation when recorded
 };
 
 int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, uint32_t n_slots,
@@ -401,7 +402,7 @@ int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, u
     if (!r) return NBA_IPSEC_ENOMEM;
     r->t = t;
     r->n_slots = n_slots;
-    r->flow_table = t->flow_table;
+    r->flow_gen = t->flow_gen;
     // persistent form: one cooperative launch walks all batches of a run
     bool persist = !std::getenv("NBA_IPSEC_RING_GRAPH") && t->pipeline == NBA_IPSEC_PIPE_FUSED &&
                    t->allow_merged;
@@ -471,7 +472,7 @@ int nba_ipsec_ring_create_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batc
     if (!r) return NBA_IPSEC_ENOMEM;
     r->t = t;
     r->n_slots = n_slots;
-    r->flow_table = t->flow_table;
+    r->flow_gen = t->flow_gen;
     cudaStream_t cs = nullptr;
     int rc = NBA_IPSEC_OK;
     if (cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking) != cudaSuccess ||
@@ -498,7 +499,7 @@ int nba_ipsec_ring_create_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batc
 int nba_ipsec_ring_run(nba_ipsec_ring *r, uint32_t n_rounds, void *cuda_stream)
 {
     if (!r || (!r->exec && !r->d_slots)) return NBA_IPSEC_EINVAL;
-    if (r->t->flow_table != r->flow_table) return NBA_IPSEC_EINVAL;   // replaced: re-create the ring
+    if (r->t->flow_gen != r->flow_gen) return NBA_IPSEC_EINVAL;   // replaced: re-create the ring
     DeviceGuard g(r->t->device);
     cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
     if (r->d_slots) {
@@ -792,6 +793,7 @@ int nba_ipsec_set_flow_table(nba_ipsec_sa_table *t, const nba_ipsec_flow *flows,
 {
     if (!t || (!flows && n_flows) || n_flows > (1u << 26)) return NBA_IPSEC_EINVAL;
     DeviceGuard g(t->device);
+    t->flow_gen++;
     if (n_flows == 0) {
         cudaDeviceSynchronize();
         if (t->flow_table) cudaFree(t->flow_table);
