@@ -155,7 +155,8 @@ int nba_ipsec_read_sa_seq(nba_ipsec_sa_table *t, uint32_t *host_seq, void *cuda_
  * n_pkts <= 512 x SMs) a run is ONE persistent cooperative launch that walks
  * all its batches, keeping the AES tables in shared memory and letting a CTA
  * start the next batch while others finish (set NBA_IPSEC_RING_GRAPH to force
- * the other form); otherwise ring_create records process_batch for every slot
+ * the other form; NBA_IPSEC_RING_PIPE selects a software-pipelined variant
+ * whose last two warps prepare the next batch while the others run this one); otherwise ring_create records process_batch for every slot
  * into a CUDA graph (the path keeps all per-batch state -- SA counters, the
  * one-kernel path's barrier base and batch epoch -- on the device, so the
  * recorded launches stay valid) and a run replays it n_rounds times.  The slots' DEVICE pointers and sizes are fixed at

@@ -382,6 +382,7 @@ struct nba_ipsec_ring {
     // arguments on the device and the second count-matrix buffer
     BatchArgs *d_slots = nullptr;
     uint16_t *hist_b = nullptr;
+    bool pipe = false;                   // software-pipelined form (k_fused_ring_pipe)
     uint64_t flow_gen = 0;               // the table's flow-table generation when recorded
 };
 
@@ -409,6 +410,12 @@ int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, u
     for (uint32_t i = 0; i < n_slots && persist; i++)
         persist = slots[i].n_pkts > 0 && fused_merged_ok(slots[i].n_pkts, t->grid_fused);
     if (persist) {
+        // the software-pipelined form is opt-in (measured: 1514 B 195.9 -> 190.7
+        // us, but 64 B 25.9 -> 33.9 us and IMIX 93 -> 107 us: the two prologue
+        // warps, starved of issue slots by the lanes, no longer keep up)
+        r->pipe = std::getenv("NBA_IPSEC_RING_PIPE") != nullptr;
+        for (uint32_t i = 0; i < n_slots && r->pipe; i++)
+            r->pipe = slots[i].sa_idx && fused_pipe_ok(slots[i].n_pkts, t->grid_fused);
         std::vector<BatchArgs> hb(n_slots);
         for (uint32_t i = 0; i < n_slots; i++) {
             const nba_ipsec_batch &b = slots[i];
@@ -506,10 +513,12 @@ int nba_ipsec_ring_run(nba_ipsec_ring *r, uint32_t n_rounds, void *cuda_stream)
         if (n_rounds == 0) return NBA_IPSEC_OK;
         if ((uint64_t)n_rounds * r->n_slots > 0xffffffffull) return NBA_IPSEC_EINVAL;
         nba_ipsec_sa_table *t = r->t;
-        return launch_fused_ring(t->T, t->W, r->d_slots, r->n_slots, n_rounds * r->n_slots,
-                                 r->hist_b, t->grid_fused, st) == cudaSuccess
-                   ? NBA_IPSEC_OK
-                   : NBA_IPSEC_ECUDA;
+        const cudaError_t e =
+            r->pipe ? launch_fused_ring_pipe(t->T, t->W, r->d_slots, r->n_slots, n_rounds * r->n_slots,
+                                             r->hist_b, t->grid_fused, st)
+                    : launch_fused_ring(t->T, t->W, r->d_slots, r->n_slots, n_rounds * r->n_slots,
+                                        r->hist_b, t->grid_fused, st);
+        return e == cudaSuccess ? NBA_IPSEC_OK : NBA_IPSEC_ECUDA;
     }
     for (uint32_t k = 0; k < n_rounds; k++)
         if (cudaGraphLaunch(r->exec, st) != cudaSuccess) return NBA_IPSEC_ECUDA;

@@ -173,6 +173,10 @@ bool fused_merged_ok(uint32_t n, int grid);
 cudaError_t setup_prologue_attributes(uint32_t n_sa, uint32_t max_tiles, int num_sms, bool *gridsync);
 cudaError_t setup_aes_attributes();
 cudaError_t setup_fused_attributes();
+cudaError_t launch_fused_ring_pipe(const DevTable &T, const DevWork &W, const BatchArgs *slots,
+                                   uint32_t n_slots, uint32_t n_batches, uint16_t *hist_b,
+                                   int grid, cudaStream_t st);
+bool fused_pipe_ok(uint32_t n, int grid);
 cudaError_t launch_fused_ring(const DevTable &T, const DevWork &W, const BatchArgs *slots,
                               uint32_t n_slots, uint32_t n_batches, uint16_t *hist_b, int grid,
                               cudaStream_t st);

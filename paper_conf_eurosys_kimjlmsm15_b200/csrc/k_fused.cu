@@ -640,6 +640,304 @@ k_fused_ring(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slots, ui
     }
 }
 
+// ------------------------------------------- software-pipelined batch ring
+// k_fused_ring_pipe: the ring with warp roles.  Warps 0..13 ("lanes") carry
+// batch k's packets, one per lane (ppc <= 448); warps 14..15 ("prologue")
+// meanwhile prepare batch k+1 for this CTA -- metadata, CTA-local stable
+// per-SA ranks (rounds of 64 packets in index order through a shared hash of
+// running counts), the per-(SA, CTA) counts, the length order -- arrive at
+// batch k+1's grid barrier, run their share of the row scans (two warps per
+// CTA) and poll the published bases into L.seq.  The lanes copy their
+// packet's fields into registers first (named barrier 2), so one set of
+// per-packet shared arrays serves both batches; each lane expands its own
+// round keys.  Same arithmetic and the same results as the other paths; the
+// count matrix alternates between two buffers by batch parity as in
+// k_fused_ring.
+constexpr uint32_t PIPE_LANE_WARPS = 14;
+constexpr uint32_t PIPE_MAX_PPC = PIPE_LANE_WARPS * 32u;          // 448 packets per CTA
+constexpr uint32_t PIPE_P = F_THREADS - PIPE_MAX_PPC;             // 64 prologue threads
+
+__device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long v)
+{
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xffffffffu, v, o);
+    return v;   // lane 0
+}
+
+__device__ __forceinline__ void bar_sync_n(uint32_t id, uint32_t n)
+{
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+__device__ __forceinline__ void bar_arrive_n(uint32_t id, uint32_t n)
+{
+    asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+
+// Prologue of one batch by the 64 prologue threads (pt = 0..63) of this CTA.
+__device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &W, const BatchArgs &B,
+                                              uint32_t ppc, uint32_t bar_target, uint32_t epoch,
+                                              FusedLo &L, uint32_t pt)
+{
+    const uint32_t G = gridDim.x, cta = blockIdx.x, n_sa = T.n_sa;
+    const uint32_t lane = pt & 31u, pw = pt >> 5;
+    const uint32_t p_begin = cta * ppc;
+    const uint32_t p_end = min(B.n, p_begin + ppc);
+    const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
+    const uint32_t rounds = (cnt + PIPE_P - 1u) / PIPE_P;
+    // 1. metadata (all loads issued together: one memory latency), validity,
+    //    length bins (counts)
+    constexpr uint32_t PR = PIPE_MAX_PPC / PIPE_P;                  // 7 rounds
+    uint32_t mD[PR], mS[PR], mI[PR], mO[PR];
+#pragma unroll
+    for (uint32_t r = 0; r < PR; r++) {
+        const uint32_t j = r * PIPE_P + pt;
+        const uint32_t i = p_begin + j;
+        mD[r] = j < cnt ? B.in_len[i] : 0u;
+        mS[r] = j < cnt ? B.sa_idx[i] : INVALID_SA;
+        mI[r] = j < cnt ? B.in_off[i] : 0u;
+        mO[r] = j < cnt ? B.out_off[i] : 0u;
+    }
+#pragma unroll
+    for (uint32_t r = 0; r < PR; r++) {
+        const uint32_t j = r * PIPE_P + pt;
+        uint32_t bin = NBINS - 1;
+        if (j < cnt) {
+            const bool cand = mS[r] < n_sa && mD[r] >= MIN_D && mD[r] <= MAX_D;
+            L.sa[j] = mS[r];
+            L.info[j] = cand ? (mD[r] | INFO_OK) : 0u;
+            L.inoff[j] = mI[r];
+            L.outoff[j] = mO[r];
+            bin = hmac_bin(cand, esp_C(mD[r]));
+            if (cand) prefetch_l2(B.in_buf + mI[r]);   // the lane reads it next round
+        }
+        if (r < rounds) warp_agg_add(L.bins, bin, j < cnt);
+    }
+    bar_sync_n(1, PIPE_P);
+    // 2. stable CTA-local ranks: rounds of 64 packets in index order, within a
+    //    round prologue warp 0 (the lower 32 packets) before warp 1
+    for (uint32_t r = 0; r < rounds; r++) {
+#pragma unroll 1
+        for (uint32_t w = 0; w < 2u; w++) {
+            if (pw == w) {
+                const uint32_t j = r * PIPE_P + 32u * w + lane;
+                const bool act = j < cnt && (L.info[j] & INFO_OK);
+                const uint32_t s = act ? L.sa[j] : INVALID_SA;
+                const uint32_t peers = __match_any_sync(0xffffffffu, s);
+                const uint32_t leader = __ffs(peers) - 1;
+                uint32_t base = 0;
+                if (act && lane == leader) {
+                    uint32_t slot = (s * 0x9E3779B1u) >> 22;      // 1024 slots
+                    while (true) {
+                        const uint32_t old = atomicCAS(&L.hkey[slot], INVALID_SA, s);
+                        if (old == INVALID_SA || old == s) break;
+                        slot = (slot + 1u) & (2u * F_SUPER - 1u);
+                    }
+                    base = L.hmask[slot];                      // running count of the SA
+                    L.hmask[slot] = base + (uint32_t)__popc(peers);
+                }
+                base = __shfl_sync(0xffffffffu, base, leader);
+                if (j < cnt) L.seq[j] = act ? base + (uint32_t)__popc(peers & lanemask_lt()) : 0u;
+            }
+            bar_sync_n(1, PIPE_P);
+        }
+    }
+    // 3. this CTA's per-SA counts -> count matrix (nonzero only); clear the hash.
+    //    Length order: exclusive scan of the bins, positions, bins re-zeroed.
+    for (uint32_t k = pt; k < 2u * F_SUPER; k += PIPE_P) {
+        const uint32_t s = L.hkey[k];
+        if (s != INVALID_SA) {
+            W.hist16[(size_t)s * G + cta] = (uint16_t)L.hmask[k];
+            L.hkey[k] = INVALID_SA;
+            L.hmask[k] = 0u;
+        }
+    }
+    if (pw == 0) {
+        const uint32_t cb = L.bins[lane];
+        uint32_t x = cb;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+            if (lane >= (uint32_t)o) x += y;
+        }
+        L.bins[lane] = x - cb;
+    }
+    bar_sync_n(1, PIPE_P);
+    for (uint32_t r = 0; r < rounds; r++) {
+        const uint32_t j = r * PIPE_P + pt;
+        const uint32_t info = j < cnt ? L.info[j] : 0u;
+        const uint32_t bin = hmac_bin((info & INFO_OK) != 0u, esp_C(info & 0x7ffu));
+        const uint32_t pos = warp_agg_add(L.bins, bin, j < cnt);
+        if (j < cnt) L.perm[pos] = (uint16_t)j;
+    }
+    bar_sync_n(1, PIPE_P);                      // count-matrix writes done, bins read
+    if (pt < NBINS) L.bins[pt] = 0u;
+    // 4. grid barrier of this batch (prologue threads of every CTA)
+    if (pt == 0) {
+        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&W.ctl[CTL_BAR_MONO]) : "memory");
+        uint32_t v;
+        while (true) {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(&W.ctl[CTL_BAR_MONO]) : "memory");
+            if ((int)(v - bar_target) >= 0) break;
+            __nanosleep(64);
+        }
+    }
+    bar_sync_n(1, PIPE_P);
+    // 5. row scans (two warps per CTA), then each packet's published base
+    scan_all_columns<true>(T, W, cta * 2u + pw, G * 2u, G, lane, epoch, false, 0u);
+    // (all first polls issued together)
+    unsigned long long pv[PR];
+#pragma unroll
+    for (uint32_t r = 0; r < PR; r++) {
+        const uint32_t j = r * PIPE_P + pt;
+        pv[r] = (j < cnt && (L.info[j] & INFO_OK)) ? ld_relaxed_u64(&W.hbase[(size_t)L.sa[j] * G + cta])
+                                                   : 0ull;
+    }
+#pragma unroll
+    for (uint32_t r = 0; r < PR; r++) {
+        const uint32_t j = r * PIPE_P + pt;
+        if (j >= cnt) continue;
+        uint32_t q32 = 0;
+        if (L.info[j] & INFO_OK) {
+            const unsigned long long *pb = &W.hbase[(size_t)L.sa[j] * G + cta];
+            unsigned long long v = pv[r];
+            while ((uint32_t)(v >> 33) != epoch) {
+                __nanosleep(32);
+                v = ld_relaxed_u64(pb);
+            }
+            const unsigned long long q = (v & ((1ull << 33) - 1ull)) + 1ull + L.seq[j];
+            q32 = q <= 0xffffffffull ? (uint32_t)q : 0u;   // RFC 4303 §3.3.3: never cycle
+        }
+        L.seq[j] = q32;
+    }
+}
+
+__global__ void __launch_bounds__(F_THREADS, 1)
+k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slots,
+                  uint32_t n_batches, uint16_t *hist_b)
+{
+    extern __shared__ __align__(16) uint8_t smem[];
+    const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
+    const uint32_t G = gridDim.x, cta = blockIdx.x;
+    if (n_batches == 0) return;
+    const uint32_t base0 = *reinterpret_cast<volatile uint32_t *>(&W.ctl[CTL_BAR_BASE]);
+    const uint32_t ep0 = *reinterpret_cast<volatile uint32_t *>(&W.ctl[CTL_EPOCH]);
+    const uint32_t sb = smem_u32(smem);
+    const uint32_t toff = (0x10000u - (sb & 0xffffu)) & 0xffffu;
+    uint32_t lo_off = 0;
+    if (toff < sizeof(FusedLo)) {
+        if (toff + AES_TABLE_BYTES + sizeof(FusedHi) + sizeof(FusedLo) > F_SMEM) __trap();
+        lo_off = toff + AES_TABLE_BYTES + (uint32_t)sizeof(FusedHi);
+    }
+    uint8_t *tabs = smem + toff;
+    FusedLo &L = *reinterpret_cast<FusedLo *>(smem + lo_off);
+    FusedHi &H = *reinterpret_cast<FusedHi *>(smem + toff + AES_TABLE_BYTES);
+    const uint32_t lane4r = (lane * 4u) | (smem_u32(tabs) & 0xffff0000u);
+    aes_tables_to_smem(tabs, T.te0);
+    if (tid < NBINS) L.bins[tid] = 0u;
+    for (uint32_t k = tid; k < 2u * F_SUPER; k += F_THREADS) {
+        L.hkey[k] = INVALID_SA;
+        L.hmask[k] = 0u;
+    }
+    __syncthreads();
+    const bool isP = tid >= PIPE_MAX_PPC;
+    const uint32_t pt = tid - PIPE_MAX_PPC;
+    auto epoch_of = [&](uint32_t bi) { return ((ep0 + bi) % 0x7fffffffu) + 1u; };
+    auto work_of = [&](uint32_t bi) {
+        DevWork Wb = W;
+        if (bi & 1u) Wb.hist16 = hist_b;
+        return Wb;
+    };
+    if (isP) {
+        const BatchArgs B0 = slots[0];
+        pipe_prologue(T, work_of(0), B0, fused_ppc(B0.n, G), base0 + G, epoch_of(0), L, pt);
+    }
+    __syncthreads();
+    unsigned long long c_ok = 0, c_drop = 0, c_in = 0, c_out = 0;
+    for (uint32_t bi = 0; bi < n_batches; bi++) {
+        const BatchArgs B = slots[bi % n_slots];
+        if (!isP) {
+            const uint32_t ppc = fused_ppc(B.n, G);
+            const uint32_t p_begin = cta * ppc;
+            const uint32_t p_end = min(B.n, p_begin + ppc);
+            const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
+            const uint32_t pos = tid;                     // run r -> warp r, longest first
+            const bool have = pos < cnt;
+            const uint32_t pk = have ? L.perm[pos] : 0u;
+            const uint32_t info = have ? L.info[pk] : 0u;
+            const uint32_t q32 = have ? L.seq[pk] : 0u;
+            const uint32_t sa = (info & INFO_OK) ? L.sa[pk] : INVALID_SA;
+            const uint32_t inoff = have ? L.inoff[pk] : 0u;
+            const uint32_t outoff = have ? L.outoff[pk] : 0u;
+            bar_arrive_n(2, F_THREADS);                  // fields taken: the arrays are free
+            if (have) {
+                const uint32_t pkt = p_begin + pk;
+                if ((info & INFO_OK) && q32 != 0u) {
+                    PktPre pp = load_pkt_pre(T, B.in_buf, sa, inoff, true, 0u);
+                    expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
+                    esp_packet(T, B, L, H, lane4r, tid, sa, info, q32, inoff, outoff, pp, nullptr);
+                    const uint32_t Dp = info & 0x7ffu;
+                    const uint32_t Lp = 48u + esp_C(Dp);
+                    B.out_len[pkt] = (uint16_t)Lp;
+                    c_ok++;
+                    c_in += Dp;
+                    c_out += Lp;
+                } else {
+                    B.out_len[pkt] = 0;
+                    c_drop++;
+                }
+            }
+        } else {
+            bar_sync_n(2, F_THREADS);                    // every lane took its fields
+            if (bi + 1 < n_batches) {
+                const BatchArgs Bn = slots[(bi + 1) % n_slots];
+                pipe_prologue(T, work_of(bi + 1), Bn, fused_ppc(Bn.n, G), base0 + (bi + 2) * G,
+                              epoch_of(bi + 1), L, pt);
+            }
+        }
+        __syncthreads();                                  // batch bi done, bi + 1 prepared
+    }
+    // counters (as fused_body), device state for the next launch
+    if (tid < 4) L.cnt[tid] = 0ull;
+    __syncthreads();
+    const unsigned long long s0 = warp_sum_u64(c_ok), s1 = warp_sum_u64(c_drop);
+    const unsigned long long s2 = warp_sum_u64(c_in), s3 = warp_sum_u64(c_out);
+    if (lane == 0) {
+        if (s0) atomicAdd(&L.cnt[0], s0);
+        if (s1) atomicAdd(&L.cnt[1], s1);
+        if (s2) atomicAdd(&L.cnt[2], s2);
+        if (s3) atomicAdd(&L.cnt[3], s3);
+    }
+    __syncthreads();
+    if (tid < 4 && L.cnt[tid]) atomicAdd(&W.counters[tid], L.cnt[tid]);
+    if (tid == 4 && cta == 0) {
+        atomicAdd(&W.counters[4], (unsigned long long)n_batches);
+        W.ctl[CTL_BAR_BASE] = base0 + n_batches * G;   // one barrier per batch
+        W.ctl[CTL_EPOCH] = epoch_of(n_batches - 1u);      // the last batch's epoch
+    }
+}
+
+cudaError_t launch_fused_ring_pipe(const DevTable &T, const DevWork &W, const BatchArgs *slots,
+                                   uint32_t n_slots, uint32_t n_batches, uint16_t *hist_b,
+                                   int grid, cudaStream_t st)
+{
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(F_THREADS);
+    cfg.dynamicSmemBytes = F_SMEM;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeCooperative;   // grid barriers inside
+    attr[0].val.cooperative = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, k_fused_ring_pipe, T, W, slots, n_slots, n_batches, hist_b);
+}
+
+bool fused_pipe_ok(uint32_t n, int grid)
+{
+    return n > 0 && fused_ppc(n, grid) <= PIPE_MAX_PPC;
+}
+
 int fused_grid(int num_sms) { return num_sms; }
 
 
@@ -701,6 +999,9 @@ cudaError_t setup_fused_attributes()
 {
     cudaError_t e0 = cudaFuncSetAttribute(k_fused_ring, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                           (int)F_SMEM);
+    if (e0 != cudaSuccess) return e0;
+    e0 = cudaFuncSetAttribute(k_fused_ring_pipe, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              (int)F_SMEM);
     if (e0 != cudaSuccess) return e0;
     cudaError_t e = cudaFuncSetAttribute(k_fused<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          (int)F_SMEM);

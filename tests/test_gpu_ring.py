@@ -17,10 +17,13 @@ def _slot(db):
     return (db.in_buf, db.in_off, db.in_len, db.sa_idx, db.out_buf, db.out_off, db.out_len, db.n)
 
 
+@pytest.mark.parametrize("pipe", [False, True])
 @pytest.mark.parametrize("sizes,n_sa", [((64, "imix", 1514), 1024), (("imix", "imix"), 7)])
-def test_ring_rounds_match_oracle(sizes, n_sa):
+def test_ring_rounds_match_oracle(sizes, n_sa, pipe, monkeypatch):
     import torch
     from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    if pipe:     # the software-pipelined persistent form (k_fused_ring_pipe)
+        monkeypatch.setenv("NBA_IPSEC_RING_PIPE", "1")
     p = gen.make_sas(n_sa, cfg_id=51)
     n = 20000
     sas = oracle.make_sas(p)
@@ -52,8 +55,11 @@ def test_ring_rounds_match_oracle(sizes, n_sa):
         ring.close()
 
 
-def test_ring_replay_equals_stream_launches():
+@pytest.mark.parametrize("pipe", [False, True])
+def test_ring_replay_equals_stream_launches(pipe, monkeypatch):
     import torch
+    if pipe:
+        monkeypatch.setenv("NBA_IPSEC_RING_PIPE", "1")
     from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
     p = gen.make_sas(1024, cfg_id=52)
     b = gen.make_batch(65536, 64, 1024, cfg_id=52)
