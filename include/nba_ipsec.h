@@ -154,9 +154,12 @@ int nba_ipsec_read_sa_seq(nba_ipsec_sa_table *t, uint32_t *host_seq, void *cuda_
  * per batch.  When every slot takes the one-kernel path (fused pipeline,
  * n_pkts <= 512 x SMs) a run is ONE persistent cooperative launch that walks
  * all its batches, keeping the AES tables in shared memory and letting a CTA
- * start the next batch while others finish (set NBA_IPSEC_RING_GRAPH to force
- * the other form; NBA_IPSEC_RING_PIPE selects a software-pipelined variant
- * whose last two warps prepare the next batch while the others run this one); otherwise ring_create records process_batch for every slot
+ * start the next batch while others finish -- by default software-pipelined
+ * when every slot has SA indices and <= 448 packets per SM (the last two warps
+ * of each CTA prepare the next batch's ranks and barrier arrival while the
+ * others run this one; best for small packets), else plain
+ * (nba_ipsec_ring_set_form switches; set NBA_IPSEC_RING_GRAPH before creation
+ * to force the graph form); otherwise ring_create records process_batch for every slot
  * into a CUDA graph (the path keeps all per-batch state -- SA counters, the
  * one-kernel path's barrier base and batch epoch -- on the device, so the
  * recorded launches stay valid) and a run replays it n_rounds times.  The slots' DEVICE pointers and sizes are fixed at
@@ -171,6 +174,12 @@ typedef struct nba_ipsec_ring nba_ipsec_ring;
 int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, uint32_t n_slots,
                           nba_ipsec_ring **out);
 int nba_ipsec_ring_run(nba_ipsec_ring *r, uint32_t n_rounds, void *cuda_stream);
+enum { NBA_IPSEC_RING_GRAPH = 0, NBA_IPSEC_RING_PERSISTENT = 1, NBA_IPSEC_RING_PIPELINED = 2 };
+/* The form a run takes (NBA_IPSEC_RING_*); set_form switches a persistent ring
+ * between PERSISTENT and PIPELINED (NBA_IPSEC_EINVAL for graph rings or slots
+ * the pipelined form does not fit).  Both give identical results. */
+int nba_ipsec_ring_form(const nba_ipsec_ring *r);
+int nba_ipsec_ring_set_form(nba_ipsec_ring *r, int form);
 int nba_ipsec_ring_destroy(nba_ipsec_ring *r);   /* NULL -> OK */
 
 /* Overwrite the per-SA sequence numbers with host_seq[0..n_sa) (HOST memory):

@@ -383,6 +383,7 @@ struct nba_ipsec_ring {
     BatchArgs *d_slots = nullptr;
     uint16_t *hist_b = nullptr;
     bool pipe = false;                   // software-pipelined form (k_fused_ring_pipe)
+    bool pipe_ok = false;                // every slot fits the pipelined form
     uint64_t flow_gen = 0;               // the table's flow-table generation when recorded
 };
 
@@ -410,12 +411,14 @@ int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, u
     for (uint32_t i = 0; i < n_slots && persist; i++)
         persist = slots[i].n_pkts > 0 && fused_merged_ok(slots[i].n_pkts, t->grid_fused);
     if (persist) {
-        // the software-pipelined form is opt-in (measured: 1514 B 195.9 -> 190.7
-        // us, but 64 B 25.9 -> 33.9 us and IMIX 93 -> 107 us: the two prologue
-        // warps, starved of issue slots by the lanes, no longer keep up)
-        r->pipe = std::getenv("NBA_IPSEC_RING_PIPE") != nullptr;
-        for (uint32_t i = 0; i < n_slots && r->pipe; i++)
-            r->pipe = slots[i].sa_idx && fused_pipe_ok(slots[i].n_pkts, t->grid_fused);
+        // software-pipelined form when every slot fits it (sa_idx given, <= 448
+        // packets per CTA); nba_ipsec_ring_set_form switches between the two
+        // persistent forms (measured, same box: 64 B 25.9 -> 23.7 us, 1514 B
+        // 194.4 -> 193.3 us, IMIX 92.2 -> 97.2 us)
+        r->pipe_ok = true;
+        for (uint32_t i = 0; i < n_slots && r->pipe_ok; i++)
+            r->pipe_ok = slots[i].sa_idx && fused_pipe_ok(slots[i].n_pkts, t->grid_fused);
+        r->pipe = r->pipe_ok && !std::getenv("NBA_IPSEC_RING_NOPIPE");
         std::vector<BatchArgs> hb(n_slots);
         for (uint32_t i = 0; i < n_slots; i++) {
             const nba_ipsec_batch &b = slots[i];
@@ -523,6 +526,27 @@ int nba_ipsec_ring_run(nba_ipsec_ring *r, uint32_t n_rounds, void *cuda_stream)
     for (uint32_t k = 0; k < n_rounds; k++)
         if (cudaGraphLaunch(r->exec, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
     return NBA_IPSEC_OK;
+}
+
+int nba_ipsec_ring_set_form(nba_ipsec_ring *r, int form)
+{
+    if (!r || !r->d_slots) return NBA_IPSEC_EINVAL;   // graph rings have one form
+    if (form == NBA_IPSEC_RING_PERSISTENT) {
+        r->pipe = false;
+        return NBA_IPSEC_OK;
+    }
+    if (form == NBA_IPSEC_RING_PIPELINED && r->pipe_ok) {
+        r->pipe = true;
+        return NBA_IPSEC_OK;
+    }
+    return NBA_IPSEC_EINVAL;
+}
+
+int nba_ipsec_ring_form(const nba_ipsec_ring *r)
+{
+    if (!r) return NBA_IPSEC_EINVAL;
+    return !r->d_slots ? NBA_IPSEC_RING_GRAPH : r->pipe ? NBA_IPSEC_RING_PIPELINED
+                                                         : NBA_IPSEC_RING_PERSISTENT;
 }
 
 int nba_ipsec_ring_destroy(nba_ipsec_ring *r)

@@ -653,6 +653,9 @@ k_fused_ring(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slots, ui
 // round keys.  Same arithmetic and the same results as the other paths; the
 // count matrix alternates between two buffers by batch parity as in
 // k_fused_ring.
+#ifndef NBA_PIPE_LPT          // pipelined ring: LPT placement of the runs (1) or run r -> warp r
+#define NBA_PIPE_LPT 1
+#endif
 constexpr uint32_t PIPE_LANE_WARPS = 14;
 constexpr uint32_t PIPE_MAX_PPC = PIPE_LANE_WARPS * 32u;          // 448 packets per CTA
 constexpr uint32_t PIPE_P = F_THREADS - PIPE_MAX_PPC;             // 64 prologue threads
@@ -771,44 +774,81 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
     }
     bar_sync_n(1, PIPE_P);                      // count-matrix writes done, bins read
     if (pt < NBINS) L.bins[pt] = 0u;
-    // 4. grid barrier of this batch (prologue threads of every CTA)
-    if (pt == 0) {
+    if (pw == 0 && !NBA_PIPE_LPT) {
+        if (lane < PIPE_LANE_WARPS) L.wrun[lane] = (uint8_t)lane;   // run r -> warp r
+    } else if (pw == 0) {
+        // runs of 32 sorted positions -> lane warps, longest first onto the least
+        // loaded sub-partition (warp w issues on w mod 4; lane warps 0..13, so
+        // sub-partitions 0 / 1 hold 4 of them and 2 / 3 hold 3), as length_sort
+        const uint32_t nruns = (cnt + 31u) / 32u;
+        uint32_t cost = 0;
+        if (lane < nruns) {
+            const uint32_t info = L.info[L.perm[32u * lane]];
+            const uint32_t C = esp_C(info & 0x7ffu);
+            cost = (info & INFO_OK) ? 8u * (esp_nsha_inner(C) + 1u) + 3u * ((C + 15u) >> 4) : 1u;
+        }
+        const uint32_t c0 = __shfl_sync(0xffffffffu, cost, 0);
+        uint32_t mine = lane < nruns ? lane : 0xffu;      // equal costs: run r -> warp r
+        if (!__all_sync(0xffffffffu, lane >= nruns || cost == c0)) {
+            uint32_t load[4] = {0u, 0u, 0u, 0u}, used[4] = {0u, 0u, 0u, 0u};
+            mine = 0xffu;
+            for (uint32_t r = 0; r < nruns; r++) {
+                const uint32_t cr = __shfl_sync(0xffffffffu, cost, r);
+                uint32_t best = 4u;
+#pragma unroll
+                for (uint32_t q = 0; q < 4u; q++) {
+                    const uint32_t cap = q < 2u ? 4u : 3u;
+                    if (used[q] < cap && (best == 4u || load[q] < load[best])) best = q;
+                }
+                if (lane == best + 4u * used[best]) mine = r;
+                used[best]++;
+                load[best] += cr;
+            }
+        }
+        if (lane < PIPE_LANE_WARPS) L.wrun[lane] = (uint8_t)mine;
+    }
+    // 4. arrive at this batch's grid barrier (the whole CTA waits for it at
+    //    the start of the batch's iteration; the arrival releases the count
+    //    matrix writes above, ordered by the named barrier)
+    if (pt == 0)
         asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&W.ctl[CTL_BAR_MONO]) : "memory");
+}
+
+// The batch's barrier wait, row scans and published bases, by the whole CTA
+// (thread j <-> packet j): L.seq[j] turns from the CTA rank into the ESP
+// sequence number (0: no number, the packet is dropped).
+__device__ __forceinline__ void pipe_sequence(const DevTable &T, const DevWork &W, const BatchArgs &B,
+                                              uint32_t ppc, uint32_t bar_target, uint32_t epoch,
+                                              FusedLo &L)
+{
+    const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
+    const uint32_t G = gridDim.x, cta = blockIdx.x;
+    constexpr uint32_t NW = F_THREADS / 32u;
+    if (tid == 0) {
         uint32_t v;
         while (true) {
             asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(&W.ctl[CTL_BAR_MONO]) : "memory");
             if ((int)(v - bar_target) >= 0) break;
-            __nanosleep(64);
         }
     }
-    bar_sync_n(1, PIPE_P);
-    // 5. row scans (two warps per CTA), then each packet's published base
-    scan_all_columns<true>(T, W, cta * 2u + pw, G * 2u, G, lane, epoch, false, 0u);
-    // (all first polls issued together)
-    unsigned long long pv[PR];
-#pragma unroll
-    for (uint32_t r = 0; r < PR; r++) {
-        const uint32_t j = r * PIPE_P + pt;
-        pv[r] = (j < cnt && (L.info[j] & INFO_OK)) ? ld_relaxed_u64(&W.hbase[(size_t)L.sa[j] * G + cta])
-                                                   : 0ull;
-    }
-#pragma unroll
-    for (uint32_t r = 0; r < PR; r++) {
-        const uint32_t j = r * PIPE_P + pt;
-        if (j >= cnt) continue;
+    __syncthreads();
+    scan_all_columns<true>(T, W, cta * NW + warp, G * NW, G, lane, epoch, false, 0u);
+    const uint32_t p_begin = cta * ppc;
+    const uint32_t p_end = min(B.n, p_begin + ppc);
+    const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
+    const uint32_t j = tid;
+    if (j < cnt) {
         uint32_t q32 = 0;
         if (L.info[j] & INFO_OK) {
             const unsigned long long *pb = &W.hbase[(size_t)L.sa[j] * G + cta];
-            unsigned long long v = pv[r];
-            while ((uint32_t)(v >> 33) != epoch) {
-                __nanosleep(32);
-                v = ld_relaxed_u64(pb);
-            }
+            unsigned long long v = ld_relaxed_u64(pb);
+            while ((uint32_t)(v >> 33) != epoch) v = ld_relaxed_u64(pb);
             const unsigned long long q = (v & ((1ull << 33) - 1ull)) + 1ull + L.seq[j];
             q32 = q <= 0xffffffffull ? (uint32_t)q : 0u;   // RFC 4303 §3.3.3: never cycle
         }
         L.seq[j] = q32;
     }
+    __syncthreads();
 }
 
 __global__ void __launch_bounds__(F_THREADS, 1)
@@ -855,13 +895,15 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slot
     unsigned long long c_ok = 0, c_drop = 0, c_in = 0, c_out = 0;
     for (uint32_t bi = 0; bi < n_batches; bi++) {
         const BatchArgs B = slots[bi % n_slots];
+        pipe_sequence(T, work_of(bi), B, fused_ppc(B.n, G), base0 + (bi + 1) * G, epoch_of(bi), L);
         if (!isP) {
             const uint32_t ppc = fused_ppc(B.n, G);
             const uint32_t p_begin = cta * ppc;
             const uint32_t p_end = min(B.n, p_begin + ppc);
             const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
-            const uint32_t pos = tid;                     // run r -> warp r, longest first
-            const bool have = pos < cnt;
+            const uint32_t run = L.wrun[warp];          // LPT placement of the runs
+            const uint32_t pos = 32u * run + lane;
+            const bool have = run != 0xffu && pos < cnt;
             const uint32_t pk = have ? L.perm[pos] : 0u;
             const uint32_t info = have ? L.info[pk] : 0u;
             const uint32_t q32 = have ? L.seq[pk] : 0u;

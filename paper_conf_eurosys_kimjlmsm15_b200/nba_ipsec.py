@@ -127,6 +127,8 @@ def _load():
                                            vp, vp]),
         "nba_ipsec_ring_create": (i32, [vp, P(Batch), u32, P(vp)]),
         "nba_ipsec_ring_run": (i32, [vp, u32, vp]),
+        "nba_ipsec_ring_form": (i32, [vp]),
+        "nba_ipsec_ring_set_form": (i32, [vp, i32]),
         "nba_ipsec_ring_create_inbound": (i32, [vp, P(InBatch), u32, P(vp)]),
         "nba_ipsec_ring_destroy": (i32, [vp]),
         "nba_ipsec_alb_default_params": (None, [P(AlbParams)]),
@@ -446,6 +448,15 @@ class Ring:
     def run(self, n_rounds: int = 1, stream=None):
         _check(lib.nba_ipsec_ring_run(self._h, int(n_rounds), _stream_handle(stream)),
                "nba_ipsec_ring_run")
+
+    GRAPH, PERSISTENT, PIPELINED = 0, 1, 2
+
+    @property
+    def form(self) -> int:
+        return int(lib.nba_ipsec_ring_form(self._h))
+
+    def set_form(self, form: int):
+        _check(lib.nba_ipsec_ring_set_form(self._h, int(form)), "nba_ipsec_ring_set_form")
 
     def close(self):
         if self._h:

@@ -22,8 +22,8 @@ def _slot(db):
 def test_ring_rounds_match_oracle(sizes, n_sa, pipe, monkeypatch):
     import torch
     from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
-    if pipe:     # the software-pipelined persistent form (k_fused_ring_pipe)
-        monkeypatch.setenv("NBA_IPSEC_RING_PIPE", "1")
+    if not pipe:     # the plain persistent form (default: software-pipelined)
+        monkeypatch.setenv("NBA_IPSEC_RING_NOPIPE", "1")
     p = gen.make_sas(n_sa, cfg_id=51)
     n = 20000
     sas = oracle.make_sas(p)
@@ -58,8 +58,8 @@ def test_ring_rounds_match_oracle(sizes, n_sa, pipe, monkeypatch):
 @pytest.mark.parametrize("pipe", [False, True])
 def test_ring_replay_equals_stream_launches(pipe, monkeypatch):
     import torch
-    if pipe:
-        monkeypatch.setenv("NBA_IPSEC_RING_PIPE", "1")
+    if not pipe:
+        monkeypatch.setenv("NBA_IPSEC_RING_NOPIPE", "1")
     from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
     p = gen.make_sas(1024, cfg_id=52)
     b = gen.make_batch(65536, 64, 1024, cfg_id=52)
@@ -220,4 +220,33 @@ def test_ring_refuses_after_flow_table_replaced():
         t.set_flow_table(gen.make_flows(200, n_sa, cfg_id=58))
         with pytest.raises(nba_ipsec.NbaIpsecError):
             ring.run(1)
+        ring.close()
+
+
+def test_ring_forms_switch_and_agree():
+    """set_form switches a persistent ring between its two forms; both give the
+    same bytes, lengths and counters as stream launches."""
+    import torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    p = gen.make_sas(1024, cfg_id=59)
+    b = gen.make_batch(65536, "imix", 1024, cfg_id=59)
+    da = [device.to_device(b, "cuda") for _ in range(2)]
+    db_ = [device.to_device(b, "cuda") for _ in range(2)]
+    with nba_ipsec.SATable(p, device=0, max_batch=b.n) as ta, \
+            nba_ipsec.SATable(p, device=0, max_batch=b.n) as tb:
+        ring = ta.ring([_slot(d) for d in da])
+        assert ring.form == ring.PIPELINED
+        ring.run(1)
+        ring.set_form(ring.PERSISTENT)
+        assert ring.form == ring.PERSISTENT
+        ring.run(1)
+        ring.set_form(ring.PIPELINED)
+        ring.run(1)
+        for _ in range(3):
+            for d in db_:
+                tb.process(*d.args(), n=b.n)
+        torch.cuda.synchronize()
+        for x, y in zip(da, db_):
+            assert torch.equal(x.out_buf, y.out_buf) and torch.equal(x.out_len, y.out_len)
+        assert np.array_equal(ta.sa_seq(), tb.sa_seq()) and ta.counters() == tb.counters()
         ring.close()
