@@ -653,6 +653,9 @@ k_fused_ring(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slots, ui
 // round keys.  Same arithmetic and the same results as the other paths; the
 // count matrix alternates between two buffers by batch parity as in
 // k_fused_ring.
+#ifndef NBA_PIPE_PSCAN        // pipelined ring: the prologue warps also run the row scans
+#define NBA_PIPE_PSCAN 0
+#endif
 #ifndef NBA_PIPE_LPT          // pipelined ring: LPT placement of the runs (1) or run r -> warp r
 #define NBA_PIPE_LPT 1
 #endif
@@ -812,6 +815,19 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
     //    matrix writes above, ordered by the named barrier)
     if (pt == 0)
         asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&W.ctl[CTL_BAR_MONO]) : "memory");
+#if NBA_PIPE_PSCAN
+    // and, once every CTA arrived, this CTA's share of the row scans (two warps)
+    if (pt == 0) {
+        uint32_t v;
+        while (true) {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(&W.ctl[CTL_BAR_MONO]) : "memory");
+            if ((int)(v - bar_target) >= 0) break;
+            __nanosleep(128);
+        }
+    }
+    bar_sync_n(1, PIPE_P);
+    scan_all_columns<true>(T, W, cta * 2u + pw, G * 2u, G, lane, epoch, false, 0u);
+#endif
 }
 
 // The batch's barrier wait, row scans and published bases, by the whole CTA
@@ -832,7 +848,7 @@ __device__ __forceinline__ void pipe_sequence(const DevTable &T, const DevWork &
         }
     }
     __syncthreads();
-    scan_all_columns<true>(T, W, cta * NW + warp, G * NW, G, lane, epoch, false, 0u);
+    if (!NBA_PIPE_PSCAN) scan_all_columns<true>(T, W, cta * NW + warp, G * NW, G, lane, epoch, false, 0u);
     const uint32_t p_begin = cta * ppc;
     const uint32_t p_end = min(B.n, p_begin + ppc);
     const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
