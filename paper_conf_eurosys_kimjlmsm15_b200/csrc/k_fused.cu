@@ -653,6 +653,9 @@ k_fused_ring(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slots, ui
 // round keys.  Same arithmetic and the same results as the other paths; the
 // count matrix alternates between two buffers by batch parity as in
 // k_fused_ring.
+#ifndef NBA_PIPE_EARLY_KEYS   // pipelined ring: SA line + round keys before the scans / polls
+#define NBA_PIPE_EARLY_KEYS 1
+#endif
 #ifndef NBA_PIPE_PSCAN        // pipelined ring: the prologue warps also run the row scans
 #define NBA_PIPE_PSCAN 0
 #endif
@@ -911,6 +914,51 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slot
     unsigned long long c_ok = 0, c_drop = 0, c_in = 0, c_out = 0;
     for (uint32_t bi = 0; bi < n_batches; bi++) {
         const BatchArgs B = slots[bi % n_slots];
+#if NBA_PIPE_EARLY_KEYS
+        // lanes: the packet (known since the previous batch) and its SA line and
+        // round keys before the barrier wait / scans / polls, whose latency
+        // these loads and lookups then overlap
+        const uint32_t ppc = fused_ppc(B.n, G);
+        const uint32_t p_begin = cta * ppc;
+        const uint32_t p_end = min(B.n, p_begin + ppc);
+        const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
+        uint32_t pk = 0, info = 0, sa = INVALID_SA, inoff = 0, outoff = 0;
+        bool have = false;
+        PktPre pp = {};
+        if (!isP) {
+            const uint32_t run = L.wrun[warp];          // LPT placement of the runs
+            const uint32_t pos = 32u * run + lane;
+            have = run != 0xffu && pos < cnt;
+            pk = have ? L.perm[pos] : 0u;
+            info = have ? L.info[pk] : 0u;
+            sa = (info & INFO_OK) ? L.sa[pk] : INVALID_SA;
+            inoff = have ? L.inoff[pk] : 0u;
+            outoff = have ? L.outoff[pk] : 0u;
+            if (info & INFO_OK) {
+                pp = load_pkt_pre(T, B.in_buf, sa, inoff, true, 0u);
+                expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
+            }
+        }
+        pipe_sequence(T, work_of(bi), B, ppc, base0 + (bi + 1) * G, epoch_of(bi), L);
+        if (!isP) {
+            const uint32_t q32 = have ? L.seq[pk] : 0u;
+            bar_arrive_n(2, F_THREADS);                  // fields taken: the arrays are free
+            if (have) {
+                const uint32_t pkt = p_begin + pk;
+                if ((info & INFO_OK) && q32 != 0u) {
+                    esp_packet(T, B, L, H, lane4r, tid, sa, info, q32, inoff, outoff, pp, nullptr);
+                    const uint32_t Dp = info & 0x7ffu;
+                    const uint32_t Lp = 48u + esp_C(Dp);
+                    B.out_len[pkt] = (uint16_t)Lp;
+                    c_ok++;
+                    c_in += Dp;
+                    c_out += Lp;
+                } else {
+                    B.out_len[pkt] = 0;
+                    c_drop++;
+                }
+            }
+#else
         pipe_sequence(T, work_of(bi), B, fused_ppc(B.n, G), base0 + (bi + 1) * G, epoch_of(bi), L);
         if (!isP) {
             const uint32_t ppc = fused_ppc(B.n, G);
@@ -944,6 +992,7 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slot
                     c_drop++;
                 }
             }
+#endif
         } else {
             bar_sync_n(2, F_THREADS);                    // every lane took its fields
             if (bi + 1 < n_batches) {
