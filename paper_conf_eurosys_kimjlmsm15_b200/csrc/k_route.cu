@@ -87,7 +87,7 @@ k_route_tiles(RouteWork R, const uint16_t *in_len, const uint32_t *sa, uint32_t 
 }
 
 // One CTA: exclusive scans over tiles per destination, then region bases.
-__global__ void __launch_bounds__(256)
+__global__ void __launch_bounds__(32 * (RT_MAX_WORLD + 1))
 k_route_scan(RouteWork R, uint32_t n_tiles, uint32_t world, unsigned long long *dest_counts,
              unsigned long long *dest_bytes, const nba_ipsec_peer_rx *rx)
 {
@@ -95,28 +95,49 @@ k_route_scan(RouteWork R, uint32_t n_tiles, uint32_t world, unsigned long long *
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
     // warp k scans destination k's column (world + 1 <= 9 columns, 8 warps:
     // warp 0 also takes column 8)
-    for (uint32_t k = warp; k <= world; k += 8u) {
+    constexpr uint32_t U = 8;                  // 8 x 32 tiles per pass, loads issued together
+    for (uint32_t k = warp; k <= world; k += blockDim.x >> 5) {   // one warp per column
         unsigned long long cc = 0, cb = 0;
-        for (uint32_t t0 = 0; t0 < n_tiles; t0 += 32u) {
-            const uint32_t t = t0 + lane;
-            const unsigned long long c = t < n_tiles ? R.tcnt[t * (world + 1u) + k] : 0ull;
-            const unsigned long long b = t < n_tiles ? R.tbyt[t * (world + 1u) + k] : 0ull;
-            unsigned long long xc = c, xb = b;
+        for (uint32_t t0 = 0; t0 < n_tiles; t0 += 32u * U) {
+            uint32_t cu[U];
+            unsigned long long bu[U];
+#pragma unroll
+            for (uint32_t u = 0; u < U; u++) {
+                const uint32_t t = t0 + 32u * u + lane;
+                cu[u] = t < n_tiles ? R.tcnt[t * (world + 1u) + k] : 0u;
+                bu[u] = t < n_tiles ? R.tbyt[t * (world + 1u) + k] : 0ull;
+            }
+            // the U inclusive scans are independent (their shuffle chains
+            // interleave); the carries are applied afterwards
+            uint32_t xc[U];
+            unsigned long long xb[U];
+#pragma unroll
+            for (uint32_t u = 0; u < U; u++) {
+                xc[u] = cu[u];
+                xb[u] = bu[u];
+            }
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
-                const unsigned long long yc = __shfl_up_sync(0xffffffffu, xc, o);
-                const unsigned long long yb = __shfl_up_sync(0xffffffffu, xb, o);
-                if (lane >= (uint32_t)o) {
-                    xc += yc;
-                    xb += yb;
+#pragma unroll
+                for (uint32_t u = 0; u < U; u++) {
+                    const uint32_t yc = __shfl_up_sync(0xffffffffu, xc[u], o);
+                    const unsigned long long yb = __shfl_up_sync(0xffffffffu, xb[u], o);
+                    if (lane >= (uint32_t)o) {
+                        xc[u] += yc;
+                        xb[u] += yb;
+                    }
                 }
             }
-            if (t < n_tiles) {
-                R.tcnt[t * (world + 1u) + k] = (uint32_t)(cc + xc - c);
-                R.tbyt[t * (world + 1u) + k] = cb + xb - b;
+#pragma unroll
+            for (uint32_t u = 0; u < U; u++) {
+                const uint32_t t = t0 + 32u * u + lane;
+                if (t < n_tiles) {
+                    R.tcnt[t * (world + 1u) + k] = (uint32_t)(cc + xc[u] - cu[u]);
+                    R.tbyt[t * (world + 1u) + k] = cb + xb[u] - bu[u];
+                }
+                cc += __shfl_sync(0xffffffffu, xc[u], 31);
+                cb += __shfl_sync(0xffffffffu, xb[u], 31);
             }
-            cc += __shfl_sync(0xffffffffu, xc, 31);
-            cb += __shfl_sync(0xffffffffu, xb, 31);
         }
         if (lane == 0) {
             s_tc[k] = cc;
@@ -141,73 +162,130 @@ k_route_scan(RouteWork R, uint32_t n_tiles, uint32_t world, unsigned long long *
     }
 }
 
-// One warp per packet: bytes to the send buffer (destination-major, batch
-// order inside a destination), length and local SA index to the send arrays.
+// Copy kernels: a warp moves RT_PPW consecutive packets.  Lanes 0..RT_PPW-1
+// first gather those packets' metadata and destinations together (two memory
+// rounds for all of them instead of two per packet), then the warp copies the
+// packets; for each, the first 64 bytes of all RT_PPW packets are loaded before
+// any is stored, so short packets need one load round for the whole group.
+constexpr uint32_t RT_PPW = 4;
+
+struct RtPkt {
+    const uint8_t *src;
+    uint8_t *dst;
+    uint32_t len;
+};
+
+template <bool DISPATCH>
+__device__ __forceinline__ void route_copy_group(const RouteWork &R, const uint8_t *in_buf,
+                                                 const uint32_t *in_off, const uint16_t *in_len,
+                                                 const uint32_t *sa, const uint32_t *sa_map,
+                                                 uint32_t n, uint32_t world, uint8_t *send_buf,
+                                                 uint16_t *send_len, uint32_t *send_sa,
+                                                 const nba_ipsec_peer_rx *rx,
+                                                 unsigned long long cap_pkts,
+                                                 unsigned long long cap_bytes)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const uint32_t i0 = w * RT_PPW;
+    if (i0 >= n) return;
+    // lane q < RT_PPW: packet i0 + q's place
+    RtPkt me = {nullptr, nullptr, 0u};
+    if (lane < RT_PPW && i0 + lane < n) {
+        const uint32_t i = i0 + lane;
+        const uint32_t d = R.dest[i];
+        const uint32_t len = in_len[i];
+        const uint32_t off = in_off[i];
+        const uint32_t s = sa[i];
+        const uint32_t rk = R.rank[i], brk = R.brank[i];
+        if (d < world) {
+            const uint32_t tile = i / RT_TILE;
+            const unsigned long long pos = R.tcnt[tile * (world + 1u) + d] + rk;
+            const unsigned long long boff = R.tbyt[tile * (world + 1u) + d] + brk;
+            const uint32_t local = sa_map ? (__ldg(sa_map + s) & 0xFFFFFFu) : s / world;
+            if (DISPATCH) {
+                if (pos < cap_pkts && boff + len <= cap_bytes) {   // never write out of bounds
+                    const nba_ipsec_peer_rx r = rx[d];
+                    me = {in_buf + off, r.buf + boff, len};
+                    r.off[pos] = (uint32_t)boff;
+                    r.len[pos] = (uint16_t)len;
+                    r.sa[pos] = local;
+                }
+            } else {
+                const unsigned long long gpos = R.base[d] + pos;
+                me = {in_buf + off, send_buf + R.base[(world + 1u) + d] + boff, len};
+                send_len[gpos] = (uint16_t)len;
+                send_sa[gpos] = local;
+            }
+        }
+    }
+    RtPkt g[RT_PPW];
+#pragma unroll
+    for (uint32_t q = 0; q < RT_PPW; q++) {
+        g[q].src = reinterpret_cast<const uint8_t *>(
+            __shfl_sync(0xffffffffu, reinterpret_cast<unsigned long long>(me.src), q));
+        g[q].dst = reinterpret_cast<uint8_t *>(
+            __shfl_sync(0xffffffffu, reinterpret_cast<unsigned long long>(me.dst), q));
+        g[q].len = __shfl_sync(0xffffffffu, me.len, q);
+    }
+    // first 64 bytes of every packet: all loads, then all stores
+    uint8_t v[RT_PPW][2];
+#pragma unroll
+    for (uint32_t q = 0; q < RT_PPW; q++) {
+        v[q][0] = (g[q].dst && lane < g[q].len) ? g[q].src[lane] : 0;
+        v[q][1] = (g[q].dst && lane + 32u < g[q].len) ? g[q].src[lane + 32u] : 0;
+    }
+#pragma unroll
+    for (uint32_t q = 0; q < RT_PPW; q++) {
+        if (g[q].dst && lane < g[q].len) g[q].dst[lane] = v[q][0];
+        if (g[q].dst && lane + 32u < g[q].len) g[q].dst[lane + 32u] = v[q][1];
+    }
+    // the rest of longer packets, 16 bytes per lane where source and
+    // destination share their alignment, bytes otherwise
+#pragma unroll 1
+    for (uint32_t q = 0; q < RT_PPW; q++) {
+        const uint32_t len = g[q].len;
+        if (!g[q].dst || len <= 64u) continue;
+        const uint8_t *src = g[q].src;
+        uint8_t *dst = g[q].dst;
+        const uintptr_t a16 = reinterpret_cast<uintptr_t>(src + 64u) & 15u;
+        if (a16 == (reinterpret_cast<uintptr_t>(dst + 64u) & 15u)) {
+            const uint32_t head = min(len - 64u, (16u - (uint32_t)a16) & 15u);
+            const uint32_t nv = (len - 64u - head) >> 4;
+            if (lane < head) dst[64u + lane] = src[64u + lane];
+            const uint4 *s4 = reinterpret_cast<const uint4 *>(src + 64u + head);
+            uint4 *d4 = reinterpret_cast<uint4 *>(dst + 64u + head);
+            for (uint32_t k = lane; k < nv; k += 32u) d4[k] = s4[k];
+            for (uint32_t b = 64u + head + 16u * nv + lane; b < len; b += 32u) dst[b] = src[b];
+        } else {
+            for (uint32_t b = 64u + lane; b < len; b += 32u) dst[b] = src[b];
+        }
+    }
+}
+
+// Bytes to the send buffer (destination-major, batch order inside a
+// destination), lengths and local SA indices to the send arrays.
 __global__ void __launch_bounds__(256)
 k_route_pack(RouteWork R, const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
              const uint32_t *sa, const uint32_t *sa_map, uint32_t n, uint32_t world,
              uint8_t *send_buf, uint16_t *send_len, uint32_t *send_sa)
 {
-    const uint32_t lane = threadIdx.x & 31u;
-    const uint32_t i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    if (i >= n) return;
-    const uint32_t d = R.dest[i];
-    if (d >= world) return;                           // dropped: not sent
-    const uint32_t tile = i / RT_TILE;
-    const unsigned long long pos = R.base[d] + R.tcnt[tile * (world + 1u) + d] + R.rank[i];
-    const unsigned long long boff = R.base[(world + 1u) + d] + R.tbyt[tile * (world + 1u) + d] +
-                                    R.brank[i];
-    const uint32_t len = in_len[i];
-    const uint8_t *src = in_buf + in_off[i];
-    uint8_t *dst = send_buf + boff;
-    for (uint32_t b = lane; b < len; b += 32u) dst[b] = src[b];
-    if (lane == 0) {
-        send_len[pos] = (uint16_t)len;
-        send_sa[pos] = sa_map ? (__ldg(sa_map + sa[i]) & 0xFFFFFFu) : sa[i] / world;
-    }
+    route_copy_group<false>(R, in_buf, in_off, in_len, sa, sa_map, n, world, send_buf, send_len,
+                            send_sa, nullptr, 0ull, 0ull);
 }
 
-// Single-ingress dispatch (nba_ipsec_route_dispatch): one warp per packet
-// writes it straight into its owner's receive buffers -- own memory or a
-// peer's, mapped over NVLink -- at the owner-local position (tile prefix +
-// rank within the tile, batch order), with its offset, length and local SA.
-// 16-byte stores where source and destination share alignment, bytes else.
+// Single-ingress dispatch (nba_ipsec_route_dispatch): every packet straight
+// into its owner's receive buffers -- own memory or a peer GPU's mapped over
+// NVLink -- at the owner-local position (tile prefix + rank within the tile,
+// batch order), with its offset, length and local SA index.
 __global__ void __launch_bounds__(256)
 k_route_dispatch(RouteWork R, const uint8_t *in_buf, const uint32_t *in_off, const uint16_t *in_len,
                  const uint32_t *sa, const uint32_t *sa_map, uint32_t n, uint32_t world,
                  const nba_ipsec_peer_rx *rx, unsigned long long cap_pkts,
                  unsigned long long cap_bytes)
 {
-    const uint32_t lane = threadIdx.x & 31u;
-    const uint32_t i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    if (i >= n) return;
-    const uint32_t d = R.dest[i];
-    if (d >= world) return;                           // not routable: not sent
-    const uint32_t tile = i / RT_TILE;
-    const unsigned long long pos = R.tcnt[tile * (world + 1u) + d] + R.rank[i];
-    const unsigned long long boff = R.tbyt[tile * (world + 1u) + d] + R.brank[i];
-    const uint32_t len = in_len[i];
-    if (pos >= cap_pkts || boff + len > cap_bytes) return;   // contract violated: never write OOB
-    const nba_ipsec_peer_rx r = rx[d];
-    const uint8_t *src = in_buf + in_off[i];
-    uint8_t *dst = r.buf + boff;
-    const uintptr_t sa16 = reinterpret_cast<uintptr_t>(src) & 15u;
-    if (sa16 == (reinterpret_cast<uintptr_t>(dst) & 15u)) {
-        const uint32_t head = min(len, (16u - (uint32_t)sa16) & 15u);
-        const uint32_t nv = (len - head) >> 4;
-        if (lane < head) dst[lane] = src[lane];
-        const uint4 *s4 = reinterpret_cast<const uint4 *>(src + head);
-        uint4 *d4 = reinterpret_cast<uint4 *>(dst + head);
-        for (uint32_t v = lane; v < nv; v += 32u) d4[v] = s4[v];
-        for (uint32_t b = head + 16u * nv + lane; b < len; b += 32u) dst[b] = src[b];
-    } else {
-        for (uint32_t b = lane; b < len; b += 32u) dst[b] = src[b];
-    }
-    if (lane == 0) {
-        r.off[pos] = (uint32_t)boff;
-        r.len[pos] = (uint16_t)len;
-        r.sa[pos] = sa_map ? (__ldg(sa_map + sa[i]) & 0xFFFFFFu) : sa[i] / world;
-    }
+    route_copy_group<true>(R, in_buf, in_off, in_len, sa, sa_map, n, world, nullptr, nullptr,
+                           nullptr, rx, cap_pkts, cap_bytes);
 }
 
 size_t route_workspace_bytes(uint32_t max_pkts, uint32_t world)
@@ -238,14 +316,15 @@ cudaError_t launch_route(const uint8_t *in_buf, const uint32_t *in_off, const ui
     R.tbyt = reinterpret_cast<unsigned long long *>(take((size_t)tiles * (world + 1) * 8));
     R.base = reinterpret_cast<unsigned long long *>(take(2ull * (world + 1) * 8));
     if (tiles) k_route_tiles<<<tiles, RT_TILE, 0, st>>>(R, in_len, sa, n, n_sa_total, sa_map, world);
-    k_route_scan<<<1, 256, 0, st>>>(R, tiles, world, dest_counts, dest_bytes, rx);
+    k_route_scan<<<1, 32 * (world + 1), 0, st>>>(R, tiles, world, dest_counts, dest_bytes, rx);
     if (n == 0) return cudaGetLastError();
+    const uint32_t copy_blocks = ((n + RT_PPW - 1u) / RT_PPW * 32u + 255u) / 256u;   // warp per RT_PPW packets
     if (rx)
-        k_route_dispatch<<<(n * 32u + 255u) / 256u, 256, 0, st>>>(R, in_buf, in_off, in_len, sa,
+        k_route_dispatch<<<copy_blocks, 256, 0, st>>>(R, in_buf, in_off, in_len, sa,
                                                                  sa_map, n, world, rx, cap_pkts,
                                                                  cap_bytes);
     else
-        k_route_pack<<<(n * 32u + 255u) / 256u, 256, 0, st>>>(R, in_buf, in_off, in_len, sa, sa_map,
+        k_route_pack<<<copy_blocks, 256, 0, st>>>(R, in_buf, in_off, in_len, sa, sa_map,
                                                              n, world, send_buf, send_len, send_sa);
     return cudaGetLastError();
 }
