@@ -442,9 +442,10 @@ int nba_ipsec_enable_inbound(nba_ipsec_sa_table *t);
 int nba_ipsec_process_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batch *b, void *cuda_stream);
 /* A batch ring (nba_ipsec_ring_create) of ESP inbound slots: process_inbound
  * per slot recorded once as a CUDA graph (the one-kernel inbound path keeps
- * its barrier base on the device too); run / destroy with nba_ipsec_ring_run
- * / nba_ipsec_ring_destroy.  Additionally NBA_IPSEC_EINVAL if inbound is not
- * enabled. */
+ * its barrier base on the device too), or -- opt-in, NBA_IPSEC_RING_IN_PERSIST
+ * set at creation -- one persistent launch per run; run / destroy with
+ * nba_ipsec_ring_run / nba_ipsec_ring_destroy.  Additionally NBA_IPSEC_EINVAL
+ * if inbound is not enabled. */
 int nba_ipsec_ring_create_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batch *slots,
                                   uint32_t n_slots, nba_ipsec_ring **out);
 /* Enqueue (on `cuda_stream`) a reset of every receive window to its initial

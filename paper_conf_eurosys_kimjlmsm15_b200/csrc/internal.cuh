@@ -185,6 +185,10 @@ int fused_grid(int num_sms);
 cudaError_t launch_in_fused(const DevTable &T, const InState &S, const InBatchArgs &B, int grid,
                             uint32_t hmask, bool merged, uint32_t *bar_base, cudaStream_t st);
 bool in_merged_ok(uint32_t n, int grid);
+cudaError_t launch_in_fused_ring(const DevTable &T, const InState &S, const InBatchArgs *slots,
+                                 uint32_t n_slots, uint32_t n_batches, uint32_t hmask,
+                                 unsigned long long *hkey_b, uint32_t *hval_b, int grid,
+                                 cudaStream_t st);
 cudaError_t launch_in_replay(const DevTable &T, const InState &S, const InBatchArgs &B,
                              uint32_t n_tiles, uint32_t hmask, bool gridsync, cudaStream_t st);
 cudaError_t launch_in_decide(const DevTable &T, const InState &S, const InBatchArgs &B,

@@ -265,15 +265,14 @@ __device__ __forceinline__ void in_merged_tail(const DevTable &T, const InState 
     if (tid == 0 && cta == 0) atomicAdd(&S.counters[N_IN_COUNTERS - 1], 1ull);
 }
 
+// One batch (the body of k_in_fused; k_in_fused_ring runs it for a sequence
+// of batches).  bar_base: the batch's grid-barrier base (one-kernel form).
 template <bool MERGED>
-__global__ void __launch_bounds__(F_THREADS, 1)
-k_in_fused(DevTable T, InState S, InBatchArgs B, uint32_t ppc, uint32_t hmask, uint32_t bar_base_h)
+__device__ __forceinline__ void in_fused_body(const DevTable &T, const InState &S,
+                                              const InBatchArgs &B, uint32_t ppc, uint32_t hmask,
+                                              uint32_t bar_base)
 {
     extern __shared__ __align__(16) uint8_t smem[];
-    // one-kernel form: the barrier base lives on the device (launches carry no
-    // host state and can be recorded in a graph); read before arriving
-    const uint32_t bar_base =
-        MERGED ? *reinterpret_cast<volatile uint32_t *>(&S.ctl[CTLI_BASE]) : bar_base_h;
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
     const uint32_t n_sa = T.n_sa;
 
@@ -381,6 +380,63 @@ k_in_fused(DevTable T, InState S, InBatchArgs B, uint32_t ppc, uint32_t hmask, u
     if constexpr (MERGED) in_merged_tail(T, S, B, L, tabs, p_begin, p_end, hmask, bar_base);
 }
 
+template <bool MERGED>
+__global__ void __launch_bounds__(F_THREADS, 1)
+k_in_fused(DevTable T, InState S, InBatchArgs B, uint32_t ppc, uint32_t hmask, uint32_t bar_base_h)
+{
+    // one-kernel form: the barrier base lives on the device (launches carry no
+    // host state and can be recorded in a graph); read before arriving
+    const uint32_t bar_base =
+        MERGED ? *reinterpret_cast<volatile uint32_t *>(&S.ctl[CTLI_BASE]) : bar_base_h;
+    in_fused_body<MERGED>(T, S, B, ppc, hmask, bar_base);
+}
+
+// An inbound batch ring as ONE persistent launch: the grid walks the run's
+// batches (two grid barriers each).  The duplicate-detection hash alternates
+// between two buffers by batch parity: batch bi + 1 clears its buffer while
+// slower CTAs may still read batch bi's, and batch bi - 1 (the buffer's last
+// user) finished everywhere before batch bi's first barrier.  The T-tables are
+// re-staged per batch (the replay merge uses their shared memory as scratch).
+__global__ void __launch_bounds__(F_THREADS, 1)
+k_in_fused_ring(DevTable T, InState S, const InBatchArgs *slots, uint32_t n_slots,
+                uint32_t n_batches, uint32_t hmask, unsigned long long *hkey_b, uint32_t *hval_b)
+{
+    const uint32_t base0 = *reinterpret_cast<volatile uint32_t *>(&S.ctl[CTLI_BASE]);
+    const uint32_t G = gridDim.x;
+    for (uint32_t bi = 0; bi < n_batches; bi++) {
+        const InBatchArgs B = slots[bi % n_slots];
+        InState Sb = S;
+        if (bi & 1u) {
+            Sb.hkey = hkey_b;
+            Sb.hval = hval_b;
+        }
+        uint32_t ppc = (B.n + G - 1) / G;
+        ppc = (ppc + 31u) & ~31u;
+        if (ppc < 32u) ppc = 32u;
+        in_fused_body<true>(T, Sb, B, ppc, hmask, base0 + 2u * bi * G);
+        __syncthreads();   // shared memory is reused by the next batch
+    }
+}
+
+cudaError_t launch_in_fused_ring(const DevTable &T, const InState &S, const InBatchArgs *slots,
+                                 uint32_t n_slots, uint32_t n_batches, uint32_t hmask,
+                                 unsigned long long *hkey_b, uint32_t *hval_b, int grid,
+                                 cudaStream_t st)
+{
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(F_THREADS);
+    cfg.dynamicSmemBytes = F_SMEM;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeCooperative;   // grid barriers inside
+    attr[0].val.cooperative = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, k_in_fused_ring, T, S, slots, n_slots, n_batches, hmask, hkey_b,
+                              hval_b);
+}
+
 cudaError_t launch_in_fused(const DevTable &T, const InState &S, const InBatchArgs &B, int grid,
                             uint32_t hmask, bool merged, uint32_t *bar_base, cudaStream_t st)
 {
@@ -413,8 +469,11 @@ bool in_merged_ok(uint32_t n, int grid)
 
 cudaError_t setup_in_fused_attributes()
 {
-    cudaError_t e = cudaFuncSetAttribute(k_in_fused<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaError_t e = cudaFuncSetAttribute(k_in_fused_ring, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          (int)F_SMEM);
+    if (e != cudaSuccess) return e;
+    e = cudaFuncSetAttribute(k_in_fused<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)F_SMEM);
     if (e != cudaSuccess) return e;
     return cudaFuncSetAttribute(k_in_fused<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 (int)F_SMEM);

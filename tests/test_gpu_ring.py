@@ -123,10 +123,14 @@ def test_ring_two_kernel_and_unfused_paths(n, pipeline):
         ring.close()
 
 
-def test_inbound_ring_equals_stream_launches_and_oracle():
-    """ESP inbound slots in a ring: status, inner bytes, lengths, windows and
-    counters equal process_inbound from the stream and the oracle's receiver."""
+@pytest.mark.parametrize("persist", [False, True])
+def test_inbound_ring_equals_stream_launches_and_oracle(persist, monkeypatch):
+    """ESP inbound slots in a ring (graph form, and the opt-in persistent form):
+    status, inner bytes, lengths, windows and counters equal process_inbound
+    from the stream and the oracle's receiver."""
     import torch
+    if persist:
+        monkeypatch.setenv("NBA_IPSEC_RING_IN_PERSIST", "1")
     from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
     n_sa, n = 64, 5000
     p = gen.make_sas(n_sa, cfg_id=55)
@@ -149,6 +153,7 @@ def test_inbound_ring_equals_stream_launches_and_oracle():
         sa_ = [torch.zeros(ib.n, dtype=torch.uint8, device="cuda") for ib in esp]
         sb_ = [torch.zeros(ib.n, dtype=torch.uint8, device="cuda") for ib in esp]
         ring = ta.ring_inbound([(*d.args(), st, ib.n) for d, st, ib in zip(da, sa_, esp)])
+        assert ring.form == (ring.PERSISTENT if persist else ring.GRAPH)
         ring.run(1)
         for d, st, ib in zip(db_, sb_, esp):
             tb.process_inbound(*d.args(), status=st, n=ib.n)
