@@ -36,6 +36,8 @@ struct FusedLo {
     uint32_t hkey[2 * F_SUPER];    // merged prologue: SA of each slot of the CTA's SA hash
     uint32_t hmask[2 * F_SUPER];   //   warps holding a group of that SA
     uint8_t wrun[F_THREADS / 32];  // warp -> run of 32 sorted positions (0xff: none)
+    uint32_t pstat[3];             // pipelined ring: the next batch's AES steps (sum, max) and
+                                   //   its "early round keys" decision
 };
 
 struct FusedHi {

@@ -653,8 +653,8 @@ k_fused_ring(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slots, ui
 // round keys.  Same arithmetic and the same results as the other paths; the
 // count matrix alternates between two buffers by batch parity as in
 // k_fused_ring.
-#ifndef NBA_PIPE_EARLY_KEYS   // pipelined ring: SA line + round keys before the scans / polls
-#define NBA_PIPE_EARLY_KEYS 1
+#ifndef NBA_PIPE_EARLY_KEYS   // pipelined ring: SA line + round keys before the scans / polls:
+#define NBA_PIPE_EARLY_KEYS 2 // 1 always, 0 never, 2 per batch (long or length-divergent)
 #endif
 #ifndef NBA_PIPE_PSCAN        // pipelined ring: the prologue warps also run the row scans
 #define NBA_PIPE_PSCAN 0
@@ -706,12 +706,18 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
         mI[r] = j < cnt ? B.in_off[i] : 0u;
         mO[r] = j < cnt ? B.out_off[i] : 0u;
     }
+    uint32_t st_sum = 0, st_max = 0;   // AES steps of the valid packets
 #pragma unroll
     for (uint32_t r = 0; r < PR; r++) {
         const uint32_t j = r * PIPE_P + pt;
         uint32_t bin = NBINS - 1;
         if (j < cnt) {
             const bool cand = mS[r] < n_sa && mD[r] >= MIN_D && mD[r] <= MAX_D;
+            if (cand) {
+                const uint32_t stp = (esp_C(mD[r]) + 63u) >> 6;
+                st_sum += stp;
+                st_max = max(st_max, stp);
+            }
             L.sa[j] = mS[r];
             L.info[j] = cand ? (mD[r] | INFO_OK) : 0u;
             L.inoff[j] = mI[r];
@@ -721,7 +727,17 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
         }
         if (r < rounds) warp_agg_add(L.bins, bin, j < cnt);
     }
+    st_sum = __reduce_add_sync(0xffffffffu, st_sum);
+    st_max = __reduce_max_sync(0xffffffffu, st_max);
+    if (pt == 0) {
+        L.pstat[0] = st_sum;
+        L.pstat[1] = st_max;
+    }
     bar_sync_n(1, PIPE_P);
+    if (pt == 32) {     // the second prologue warp adds its share
+        L.pstat[0] += st_sum;
+        L.pstat[1] = max(L.pstat[1], st_max);
+    }
     // 2. stable CTA-local ranks: rounds of 64 packets in index order, within a
     //    round prologue warp 0 (the lower 32 packets) before warp 1
     for (uint32_t r = 0; r < rounds; r++) {
@@ -780,6 +796,13 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
     }
     bar_sync_n(1, PIPE_P);                      // count-matrix writes done, bins read
     if (pt < NBINS) L.bins[pt] = 0u;
+    if (pt == 0) {
+        // round keys before the scans / polls (their latency overlaps) pays for
+        // long or length-divergent batches; for uniform short ones after
+        // (measured: 64 B 23.5 vs 24.1 us, IMIX 96.8 vs 90.4, 1514 B 193.7 vs 192.3)
+        const uint32_t sum = L.pstat[0], mx = L.pstat[1], nv = cnt ? cnt : 1u;
+        L.pstat[2] = (mx * nv > 2u * sum || sum >= 8u * nv) ? 1u : 0u;
+    }
     if (pw == 0 && !NBA_PIPE_LPT) {
         if (lane < PIPE_LANE_WARPS) L.wrun[lane] = (uint8_t)lane;   // run r -> warp r
     } else if (pw == 0) {
@@ -914,16 +937,18 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slot
     unsigned long long c_ok = 0, c_drop = 0, c_in = 0, c_out = 0;
     for (uint32_t bi = 0; bi < n_batches; bi++) {
         const BatchArgs B = slots[bi % n_slots];
-#if NBA_PIPE_EARLY_KEYS
-        // lanes: the packet (known since the previous batch) and its SA line and
-        // round keys before the barrier wait / scans / polls, whose latency
-        // these loads and lookups then overlap
+        // lanes: the packet (known since the previous batch); its SA line and
+        // round keys either before the barrier wait / scans / polls, whose
+        // latency they then overlap (long or length-divergent batches, as
+        // decided by the prologue warps), or after them (uniform short ones)
         const uint32_t ppc = fused_ppc(B.n, G);
         const uint32_t p_begin = cta * ppc;
         const uint32_t p_end = min(B.n, p_begin + ppc);
         const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
         uint32_t pk = 0, info = 0, sa = INVALID_SA, inoff = 0, outoff = 0;
         bool have = false;
+        const bool early = NBA_PIPE_EARLY_KEYS == 1 ? true
+                         : NBA_PIPE_EARLY_KEYS == 0 ? false : L.pstat[2] != 0u;
         PktPre pp = {};
         if (!isP) {
             const uint32_t run = L.wrun[warp];          // LPT placement of the runs
@@ -934,7 +959,7 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slot
             sa = (info & INFO_OK) ? L.sa[pk] : INVALID_SA;
             inoff = have ? L.inoff[pk] : 0u;
             outoff = have ? L.outoff[pk] : 0u;
-            if (info & INFO_OK) {
+            if (early && (info & INFO_OK)) {
                 pp = load_pkt_pre(T, B.in_buf, sa, inoff, true, 0u);
                 expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
             }
@@ -946,6 +971,10 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slot
             if (have) {
                 const uint32_t pkt = p_begin + pk;
                 if ((info & INFO_OK) && q32 != 0u) {
+                    if (!early) {
+                        pp = load_pkt_pre(T, B.in_buf, sa, inoff, true, 0u);
+                        expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
+                    }
                     esp_packet(T, B, L, H, lane4r, tid, sa, info, q32, inoff, outoff, pp, nullptr);
                     const uint32_t Dp = info & 0x7ffu;
                     const uint32_t Lp = 48u + esp_C(Dp);
@@ -958,41 +987,6 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slot
                     c_drop++;
                 }
             }
-#else
-        pipe_sequence(T, work_of(bi), B, fused_ppc(B.n, G), base0 + (bi + 1) * G, epoch_of(bi), L);
-        if (!isP) {
-            const uint32_t ppc = fused_ppc(B.n, G);
-            const uint32_t p_begin = cta * ppc;
-            const uint32_t p_end = min(B.n, p_begin + ppc);
-            const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
-            const uint32_t run = L.wrun[warp];          // LPT placement of the runs
-            const uint32_t pos = 32u * run + lane;
-            const bool have = run != 0xffu && pos < cnt;
-            const uint32_t pk = have ? L.perm[pos] : 0u;
-            const uint32_t info = have ? L.info[pk] : 0u;
-            const uint32_t q32 = have ? L.seq[pk] : 0u;
-            const uint32_t sa = (info & INFO_OK) ? L.sa[pk] : INVALID_SA;
-            const uint32_t inoff = have ? L.inoff[pk] : 0u;
-            const uint32_t outoff = have ? L.outoff[pk] : 0u;
-            bar_arrive_n(2, F_THREADS);                  // fields taken: the arrays are free
-            if (have) {
-                const uint32_t pkt = p_begin + pk;
-                if ((info & INFO_OK) && q32 != 0u) {
-                    PktPre pp = load_pkt_pre(T, B.in_buf, sa, inoff, true, 0u);
-                    expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
-                    esp_packet(T, B, L, H, lane4r, tid, sa, info, q32, inoff, outoff, pp, nullptr);
-                    const uint32_t Dp = info & 0x7ffu;
-                    const uint32_t Lp = 48u + esp_C(Dp);
-                    B.out_len[pkt] = (uint16_t)Lp;
-                    c_ok++;
-                    c_in += Dp;
-                    c_out += Lp;
-                } else {
-                    B.out_len[pkt] = 0;
-                    c_drop++;
-                }
-            }
-#endif
         } else {
             bar_sync_n(2, F_THREADS);                    // every lane took its fields
             if (bi + 1 < n_batches) {
