@@ -975,7 +975,8 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slot
                         pp = load_pkt_pre(T, B.in_buf, sa, inoff, true, 0u);
                         expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
                     }
-                    esp_packet(T, B, L, H, lane4r, tid, sa, info, q32, inoff, outoff, pp, nullptr);
+                    if (!NBA_PROLOGUE_ONLY)   // (debug A/B: the ring without the lane work)
+                        esp_packet(T, B, L, H, lane4r, tid, sa, info, q32, inoff, outoff, pp, nullptr);
                     const uint32_t Dp = info & 0x7ffu;
                     const uint32_t Lp = 48u + esp_C(Dp);
                     B.out_len[pkt] = (uint16_t)Lp;
