@@ -294,3 +294,30 @@ def test_ring_sequence_overflow_matches_oracle(form):
         assert (g_len == 0).sum() > 0                          # drops happened
         assert np.array_equal(t.sa_seq(), oracle.sa_seq(sas, n_sa))
         ring.close()
+
+
+@pytest.mark.parametrize("n", [1, 31, 100, 4737])
+def test_pipelined_ring_small_batches(n):
+    """Batches that leave most CTAs without packets (ppc = 32): the pipelined
+    ring still equals the oracle over three rounds."""
+    import torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    n_sa = 8
+    p = gen.make_sas(n_sa, cfg_id=61)
+    bs = [gen.make_batch(n, "imix", n_sa, cfg_id=61, batch=k) for k in range(2)]
+    sas = oracle.make_sas(p)
+    with nba_ipsec.SATable(p, device=0, max_batch=n) as t:
+        ds = [device.to_device(b, "cuda") for b in bs]
+        ring = t.ring([_slot(d) for d in ds])
+        assert ring.form == ring.PIPELINED
+        ring.run(3)
+        torch.cuda.synchronize()
+        for _ in range(2):
+            for b in bs:
+                oracle.process_batch(sas, n_sa, b)
+        for d, b in zip(ds, bs):
+            o_out, o_len, _ = oracle.process_batch(sas, n_sa, b)
+            g_out, g_len = device.fetch(d)
+            assert np.array_equal(g_len, o_len) and np.array_equal(g_out, o_out)
+        assert np.array_equal(t.sa_seq(), oracle.sa_seq(sas, n_sa))
+        ring.close()
