@@ -659,6 +659,9 @@ k_fused_ring(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slots, ui
 #ifndef NBA_PIPE_PSCAN        // pipelined ring: the prologue warps also run the row scans
 #define NBA_PIPE_PSCAN 0
 #endif
+#ifndef NBA_PIPE_HALVES       // pipelined ring: the two prologue warps rank halves concurrently
+#define NBA_PIPE_HALVES 1
+#endif
 #ifndef NBA_PIPE_LPT          // pipelined ring: LPT placement of the runs (1) or run r -> warp r
 #define NBA_PIPE_LPT 1
 #endif
@@ -738,6 +741,48 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
         L.pstat[0] += st_sum;
         L.pstat[1] = max(L.pstat[1], st_max);
     }
+#if NBA_PIPE_HALVES
+    // 2. stable CTA-local ranks: prologue warp w ranks its half of the packets
+    //    (rounds of 32 in index order) with its own running count per SA slot
+    //    (warp 0: L.hmask, warp 1: cnt1), concurrently; warp 1's ranks then
+    //    add warp 0's final count of the SA
+    uint32_t *cnt1 = &L.aux0[0];                 // aux0 | aux1: 1024 slot counts (outbound only)
+    {
+        const uint32_t half = ((cnt + 1u) / 2u + 31u) & ~31u;
+        const uint32_t j0 = pw ? half : 0u, j1 = pw ? cnt : min(cnt, half);
+        uint32_t *cw = pw ? cnt1 : L.hmask;
+        for (uint32_t jb = j0; jb < j1; jb += 32u) {
+            const uint32_t j = jb + lane;
+            const bool act = j < j1 && (L.info[j] & INFO_OK);
+            const uint32_t s = act ? L.sa[j] : INVALID_SA;
+            const uint32_t peers = __match_any_sync(0xffffffffu, s);
+            const uint32_t leader = __ffs(peers) - 1;
+            uint32_t base = 0, slot = 0;
+            if (act && lane == leader) {
+                slot = (s * 0x9E3779B1u) >> 22;          // 1024 slots
+                while (true) {
+                    const uint32_t old = atomicCAS(&L.hkey[slot], INVALID_SA, s);
+                    if (old == INVALID_SA || old == s) break;
+                    slot = (slot + 1u) & (2u * F_SUPER - 1u);
+                }
+                base = cw[slot];
+                cw[slot] = base + (uint32_t)__popc(peers);
+            }
+            base = __shfl_sync(0xffffffffu, base, leader);
+            slot = __shfl_sync(0xffffffffu, slot, leader);
+            if (j < j1) {
+                L.seq[j] = act ? base + (uint32_t)__popc(peers & lanemask_lt()) : 0u;
+                if (pw) L.perm[j] = (uint16_t)slot;     // (perm is rebuilt in step 3)
+            }
+        }
+        bar_sync_n(1, PIPE_P);
+        if (pw) {
+            for (uint32_t j = j0 + lane; j < j1; j += 32u)
+                if (L.info[j] & INFO_OK) L.seq[j] += L.hmask[L.perm[j]];
+        }
+        bar_sync_n(1, PIPE_P);
+    }
+#else
     // 2. stable CTA-local ranks: rounds of 64 packets in index order, within a
     //    round prologue warp 0 (the lower 32 packets) before warp 1
     for (uint32_t r = 0; r < rounds; r++) {
@@ -766,12 +811,18 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
             bar_sync_n(1, PIPE_P);
         }
     }
+#endif
     // 3. this CTA's per-SA counts -> count matrix (nonzero only); clear the hash.
     //    Length order: exclusive scan of the bins, positions, bins re-zeroed.
     for (uint32_t k = pt; k < 2u * F_SUPER; k += PIPE_P) {
         const uint32_t s = L.hkey[k];
         if (s != INVALID_SA) {
+#if NBA_PIPE_HALVES
+            W.hist16[(size_t)s * G + cta] = (uint16_t)(L.hmask[k] + cnt1[k]);
+            cnt1[k] = 0u;
+#else
             W.hist16[(size_t)s * G + cta] = (uint16_t)L.hmask[k];
+#endif
             L.hkey[k] = INVALID_SA;
             L.hmask[k] = 0u;
         }
@@ -919,6 +970,7 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slot
     for (uint32_t k = tid; k < 2u * F_SUPER; k += F_THREADS) {
         L.hkey[k] = INVALID_SA;
         L.hmask[k] = 0u;
+        (&L.aux0[0])[k] = 0u;                     // the prologue's second count array
     }
     __syncthreads();
     const bool isP = tid >= PIPE_MAX_PPC;
