@@ -685,6 +685,61 @@ __device__ __forceinline__ void bar_arrive_n(uint32_t id, uint32_t n)
     asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory");
 }
 
+// The prologue warps' share of the row scans (rows slot, slot + nslots, ...;
+// G <= 160 CTAs, so a row is at most 5 x 32 counts): every row's counts are
+// loaded before any is scanned, so the rows cost one memory round trip
+// instead of one each.  Same results as scan_all_columns (warp per row).
+__device__ __forceinline__ void pipe_scan_rows(const DevTable &T, const DevWork &W, uint32_t slot,
+                                               uint32_t nslots, uint32_t G, uint32_t lane,
+                                               uint32_t epoch)
+{
+    constexpr uint32_t MR = 4, U = 5;           // up to 4 rows per warp, 160 counts per row
+    uint32_t h[MR][U], old[MR];
+#pragma unroll
+    for (uint32_t r = 0; r < MR; r++) {
+        const uint32_t sa = slot + r * nslots;
+        const bool ok = sa < T.n_sa;
+        old[r] = ok ? T.seq[sa] : 0u;
+#pragma unroll
+        for (uint32_t u = 0; u < U; u++) {
+            const uint32_t t = 32u * u + lane;
+            h[r][u] = (ok && t < G) ? (uint32_t)__ldcg(&W.hist16[(size_t)sa * G + t]) : 0u;
+        }
+    }
+#pragma unroll
+    for (uint32_t r = 0; r < MR; r++) {
+        const uint32_t sa = slot + r * nslots;
+        if (sa >= T.n_sa) break;
+        uint16_t *col = W.hist16 + (size_t)sa * G;
+        uint32_t carry = 0;
+#pragma unroll
+        for (uint32_t u = 0; u < U; u++) {
+            uint32_t x = h[r][u];
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+                if (lane >= (uint32_t)o) x += y;
+            }
+            const uint32_t t = 32u * u + lane;
+            if (t < G) {
+                st_relaxed_u64(&W.hbase[(size_t)sa * G + t],
+                               ((unsigned long long)epoch << 33) |
+                                   ((unsigned long long)old[r] + carry + x - h[r][u]));
+                if (h[r][u]) col[t] = 0;           // re-arm for the next batch of this parity
+            }
+            carry += __shfl_sync(0xffffffffu, x, 31);
+        }
+        if (lane == 0) {
+            T.seq_prev[sa] = old[r];
+            const uint32_t room = 0xffffffffu - old[r];
+            T.seq[sa] = old[r] + (carry < room ? carry : room);
+        }
+    }
+    // rows beyond MR per warp (more SAs than 4 x 2 x CTAs): the generic scan
+    for (uint32_t sa = slot + MR * nslots; sa < T.n_sa; sa += nslots)
+        scan_sa_column<true>(T, W, sa, G, lane, epoch);
+}
+
 // Prologue of one batch by the 64 prologue threads (pt = 0..63) of this CTA.
 __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &W, const BatchArgs &B,
                                               uint32_t ppc, uint32_t bar_target, uint32_t epoch,
@@ -903,7 +958,7 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
         }
     }
     bar_sync_n(1, PIPE_P);
-    scan_all_columns<true>(T, W, cta * 2u + pw, G * 2u, G, lane, epoch, false, 0u);
+    pipe_scan_rows(T, W, cta * 2u + pw, G * 2u, G, lane, epoch);
 #endif
 }
 
