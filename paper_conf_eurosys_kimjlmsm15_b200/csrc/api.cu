@@ -251,6 +251,7 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
     chk(dalloc(t, &W.hist16, cols * n_sa));
     chk(dalloc(t, &W.hpfx, cols * n_sa));
     chk(dalloc(t, &W.hbase, (size_t)t->grid_fused * n_sa));
+    chk(dalloc(t, &W.pvote, 2ull * t->grid_fused));
     chk(dalloc(t, &W.tile_rec, t->max_tiles));
     chk(dalloc(t, &W.tile_blk, t->max_tiles));
     chk(dalloc(t, &W.tile_bin, (size_t)t->max_tiles * NBINS));

@@ -56,6 +56,7 @@ struct DevWork {
                             //   all-zero between batches)
     uint32_t *hpfx;         // [n_sa][n_tiles] exclusive prefix of hist16 along each SA row
     unsigned long long *hbase;   // [n_sa][G] in-kernel prologue: epoch << 33 | (seq_prev + prefix)
+    unsigned long long *pvote;   // [2][G] pipelined ring: epoch << 1 | "long batch" per CTA
     uint32_t *tile_rec;     // [max_tiles] record chunks per tile -> exclusive prefix
     uint32_t *tile_blk;     // [max_tiles] AES blocks per tile -> exclusive prefix
     uint32_t *tile_bin;     // [max_tiles * NBINS] HMAC length bins per tile -> prefix

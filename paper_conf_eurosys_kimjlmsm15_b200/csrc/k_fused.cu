@@ -656,8 +656,8 @@ k_fused_ring(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slots, ui
 #ifndef NBA_PIPE_EARLY_KEYS   // pipelined ring: SA line + round keys before the scans / polls:
 #define NBA_PIPE_EARLY_KEYS 2 // 1 always, 0 never, 2 per batch (long or length-divergent)
 #endif
-#ifndef NBA_PIPE_PSCAN        // pipelined ring: the prologue warps also run the row scans
-#define NBA_PIPE_PSCAN 0
+#ifndef NBA_PIPE_PSCAN        // pipelined ring: the prologue warps also run the row scans:
+#define NBA_PIPE_PSCAN 0      // 0 never, 1 always, 2 when most CTAs vote the batch long
 #endif
 #ifndef NBA_PIPE_HALVES       // pipelined ring: the two prologue warps rank halves concurrently
 #define NBA_PIPE_HALVES 1
@@ -743,7 +743,7 @@ __device__ __forceinline__ void pipe_scan_rows(const DevTable &T, const DevWork 
 // Prologue of one batch by the 64 prologue threads (pt = 0..63) of this CTA.
 __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &W, const BatchArgs &B,
                                               uint32_t ppc, uint32_t bar_target, uint32_t epoch,
-                                              FusedLo &L, uint32_t pt)
+                                              FusedLo &L, uint32_t pt, uint32_t parity)
 {
     const uint32_t G = gridDim.x, cta = blockIdx.x, n_sa = T.n_sa;
     const uint32_t lane = pt & 31u, pw = pt >> 5;
@@ -945,10 +945,21 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
     // 4. arrive at this batch's grid barrier (the whole CTA waits for it at
     //    the start of the batch's iteration; the arrival releases the count
     //    matrix writes above, ordered by the named barrier)
+#if NBA_PIPE_PSCAN == 2
+    // this CTA's vote: a long batch (mean >= 8 AES steps) lets the prologue
+    // warps run the row scans too (published before the arrival releases it)
+    if (pt == 0) {
+        const uint32_t nv = cnt ? cnt : 1u;
+        const unsigned long long vote = L.pstat[0] >= 8u * nv ? 1ull : 0ull;
+        W.pvote[(size_t)parity * G + cta] = ((unsigned long long)epoch << 1) | vote;
+    }
+#endif
     if (pt == 0)
         asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&W.ctl[CTL_BAR_MONO]) : "memory");
 #if NBA_PIPE_PSCAN
-    // and, once every CTA arrived, this CTA's share of the row scans (two warps)
+    // and, once every CTA arrived, this CTA's share of the row scans (two
+    // warps) -- always (PSCAN 1), or when most CTAs voted "long" (PSCAN 2: the
+    // same count of the same complete votes in every CTA, so all agree)
     if (pt == 0) {
         uint32_t v;
         while (true) {
@@ -958,7 +969,21 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
         }
     }
     bar_sync_n(1, PIPE_P);
-    pipe_scan_rows(T, W, cta * 2u + pw, G * 2u, G, lane, epoch);
+    bool pscan = true;
+#if NBA_PIPE_PSCAN == 2
+    {
+        uint32_t longs = 0;
+#pragma unroll
+        for (uint32_t u = 0; u < 5u; u++) {
+            const uint32_t c = 32u * u + lane;
+            const unsigned long long e = c < G ? ld_relaxed_u64(&W.pvote[(size_t)parity * G + c]) : 0ull;
+            longs += __popc(__ballot_sync(0xffffffffu, c < G && (uint32_t)(e >> 1) == epoch && (e & 1ull)));
+        }
+        pscan = 2u * longs > G;
+        if (pt == 0) L.pstat[2] |= pscan ? 2u : 0u;    // bit 1: the CTA skips its scans
+    }
+#endif
+    if (pscan) pipe_scan_rows(T, W, cta * 2u + pw, G * 2u, G, lane, epoch);
 #endif
 }
 
@@ -980,7 +1005,8 @@ __device__ __forceinline__ void pipe_sequence(const DevTable &T, const DevWork &
         }
     }
     __syncthreads();
-    if (!NBA_PIPE_PSCAN) scan_all_columns<true>(T, W, cta * NW + warp, G * NW, G, lane, epoch, false, 0u);
+    const bool p_scanned = NBA_PIPE_PSCAN == 1 || (NBA_PIPE_PSCAN == 2 && (L.pstat[2] & 2u));
+    if (!p_scanned) scan_all_columns<true>(T, W, cta * NW + warp, G * NW, G, lane, epoch, false, 0u);
     const uint32_t p_begin = cta * ppc;
     const uint32_t p_end = min(B.n, p_begin + ppc);
     const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
@@ -1038,7 +1064,7 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slot
     };
     if (isP) {
         const BatchArgs B0 = slots[0];
-        pipe_prologue(T, work_of(0), B0, fused_ppc(B0.n, G), base0 + G, epoch_of(0), L, pt);
+        pipe_prologue(T, work_of(0), B0, fused_ppc(B0.n, G), base0 + G, epoch_of(0), L, pt, 0u);
     }
     __syncthreads();
     unsigned long long c_ok = 0, c_drop = 0, c_in = 0, c_out = 0;
@@ -1055,7 +1081,7 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slot
         uint32_t pk = 0, info = 0, sa = INVALID_SA, inoff = 0, outoff = 0;
         bool have = false;
         const bool early = NBA_PIPE_EARLY_KEYS == 1 ? true
-                         : NBA_PIPE_EARLY_KEYS == 0 ? false : L.pstat[2] != 0u;
+                         : NBA_PIPE_EARLY_KEYS == 0 ? false : (L.pstat[2] & 1u) != 0u;
         PktPre pp = {};
         if (!isP) {
             const uint32_t run = L.wrun[warp];          // LPT placement of the runs
@@ -1100,7 +1126,7 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slot
             if (bi + 1 < n_batches) {
                 const BatchArgs Bn = slots[(bi + 1) % n_slots];
                 pipe_prologue(T, work_of(bi + 1), Bn, fused_ppc(Bn.n, G), base0 + (bi + 2) * G,
-                              epoch_of(bi + 1), L, pt);
+                              epoch_of(bi + 1), L, pt, (bi + 1) & 1u);
             }
         }
         __syncthreads();                                  // batch bi done, bi + 1 prepared
