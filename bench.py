@@ -270,7 +270,7 @@ def run_ours(args):
                 for k in range(k_steps):
                     runs[k % R]()
 
-        timed_batches(2 * R)
+        timed_batches(max(warmup, 2 * R))      # >= W untimed warm-up batches
         torch.cuda.synchronize()
         barrier()
         e_all = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
