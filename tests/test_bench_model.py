@@ -1,0 +1,58 @@
+"""The bench's algorithmic work model (the roofline numerators)
+against SURVEY.md Appendix B's per-size table (computed there from the RFC
+formulas), and the IMIX composition of the generator (PAPER.md:603 sizes,
+7:4:1 mix) -- no GPU needed."""
+import os
+import sys
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import bench  # noqa: E402
+from paper_conf_eurosys_kimjlmsm15_b200 import gen  # noqa: E402
+
+# L -> (AES blocks, SHA-1 compressions inner + outer, out IP length)
+APPENDIX_B = {64: (4, 3, 100), 128: (8, 4, 164), 256: (16, 6, 292), 512: (32, 10, 548),
+              594: (37, 11, 632), 1024: (64, 18, 1060), 1514: (94, 25, 1552)}
+
+
+def test_work_model_per_packet_matches_appendix_b():
+    for L, (blocks, comps, out_len) in APPENDIX_B.items():
+        b = gen.make_batch(10, L, 4, cfg_id=1)
+        w = bench.work_model(b)
+        assert w["packets"] == 10
+        assert w["aes_blocks"] == 10 * blocks, L
+        assert w["sha1_compressions"] == 10 * comps, L
+        assert w["bytes_out"] == 10 * out_len, L
+
+
+def test_work_model_batch_totals_match_appendix_b():
+    # per 64K batch: AES threads and SHA-1 compressions
+    expect = {64: (262144, 196608), 1514: (6160384, 1638400), "imix": (1474609, 491532)}
+    for size, (blocks, comps) in expect.items():
+        b = gen.make_batch(65536, size, 1024, cfg_id=2)
+        w = bench.work_model(b)
+        assert (w["aes_blocks"], w["sha1_compressions"]) == (blocks, comps), size
+
+
+def test_imix_composition_and_invalid_packets_excluded():
+    b = gen.make_batch(65536, "imix", 1024, cfg_id=4)
+    L = np.asarray(b.frame_len)
+    assert sorted(np.unique(L).tolist()) == [64, 594, 1514]
+    assert [int((L == x).sum()) for x in (64, 594, 1514)] == [38229, 21845, 5462]
+    b.in_len[:3] = [19, 1501, 0]                      # dropped by the path: no work
+    w = bench.work_model(b)
+    assert w["packets"] == 65536 - 3
+
+
+def test_roofline_arithmetic():
+    w = {"aes_blocks": 1000, "sha1_compressions": 100}
+    peaks = {"sm_max_mhz": 1965.0, "hbm_gbs": 6500.0}
+    r = bench.kernel_roofline("fused", 0.001, w, peaks)
+    ops = 1000 * bench.AES_ALU_OPS_PER_BLOCK + 100 * bench.SHA1_ALU_OPS_PER_COMPRESSION
+    assert abs(r["achieved"] - ops / 1e-6 / 1e9) < 1e-6
+    assert abs(r["peak"] - 148 * 64 * 1965e6 / 1e9) < 1e-6
+    assert r["bound"] == "alu"
+    assert bench.kernel_roofline("fused_ring", 0.001, w, peaks)["achieved"] == r["achieved"]
