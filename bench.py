@@ -1,22 +1,31 @@
 #!/usr/bin/env python
-"""Benchmark: IPsec ESP outbound throughput (Gbps, Mpps) on B200.
+"""Benchmark: IPsec ESP outbound throughput (Gbps, Mpps) per packet size on B200.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--config 2|3|4] [--impl ours|reference]
     python -m torch.distributed.run --nproc-per-node N --master-addr 127.0.0.1 bench.py --gpus N
 
 One step = one batch of 65,536 packets per GPU through the whole hot path
-(prologue, gather+ESP encapsulation, AES-128-CTR, HMAC-SHA1-96, scatter) via
-the C ABI (nba_ipsec_process_batch), inputs resident in HBM.  Default workload
-is BASELINE.json configs[1] (64 B frames, 1024 SAs); configs[2] (1514 B) and
-configs[3] (IMIX) are measured too and reported under "per_size".  Multi-GPU:
-SA-hash sharding (GPU g owns SAs s = g mod N), weak scaling, no data-path
+(prologue, gather + ESP encapsulation, AES-128-CTR, HMAC-SHA1-96,
+scatter) with inputs resident in HBM.  The headline (`value`) is BASELINE.json
+configs[1] (64-B frames, 1024 SAs); configs[2] (1514 B), configs[3] (IMIX) and
+the configs[4] sweep (64 / 128 / 256 / 512 / 1024 / 1514 B + IMIX) are measured
+in the same run (`gbps_by_size`).  Multi-GPU (configs[4] at 2/4/8 GPUs): SA-hash
+sharding (GPU g owns SAs s = g mod N), weak scaling, no data-path
 collective; NCCL only reduces counters and takes the max elapsed time.
+`--gpus N` without a torchrun environment re-launches itself under torchrun
+(one process per GPU).
 
-Gbps = 8 * sum(frame bytes L) / t (reading A18, frames excluding FCS);
-Mpps = packets / t.  The K timed batches run back to back on the launching
-stream between one CUDA event pair, rotating over device copies of the batch
-whose touched bytes exceed 2x the L2 (every batch starts L2-cold); the
-isolated-batch time (L2 flushed, one event pair per batch) is reported beside it.
+Timing: the K timed batches run back to back on the launching
+stream between one CUDA event pair (barrier + synchronize on both sides, max
+over ranks), rotating over R device copies of the batch whose touched bytes
+exceed 2x the L2 (every batch starts L2-cold); EVERY timed batch goes through
+the library's batch ring (nba_ipsec_ring_run_batches: one persistent launch for
+all K).  A second pass records per-batch device timestamps (median / p10 / p90).
+Beside it: the same K batches as plain process_batch launches, as CUDA-graph
+replay, and one batch at a time with L2 flushed.
+
+Gbps = 8 * sum(frame bytes L) / t (reading A18, frames excluding FCS); Mpps =
+packets / t; ESP-payload Gbps = 8 * sum(D) / t.
 """
 from __future__ import annotations
 
@@ -40,6 +49,7 @@ METRIC = "IPsec ESP throughput Gbps & Mpps per packet size at 1/2/4/8 B200; % ro
 N_SA_TOTAL = 1024
 PKTS_PER_GPU = 65536
 CFG_SIZE = {2: 64, 3: 1514, 4: "imix"}
+SWEEP = [(2, 64), (5, 128), (5, 256), (5, 512), (5, 1024), (3, 1514), (4, "imix")]   # configs[4]
 SM_COUNT = 148
 
 
@@ -51,8 +61,7 @@ def load_peaks():
         return {"hbm_gbs": float(d["hbm_gbs"]), "sm_max_mhz": float(d.get("sm_max_mhz", 1965.0)),
                 "source": "measured (MEASURED_PEAKS.json)"}
     except Exception:
-        return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0,
-                "source": "fallback (B200_PROFILING.md)"}
+        return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0, "source": "fallback (B200_PROFILING.md)"}
 
 
 class ClockSampler:
@@ -113,9 +122,10 @@ def frame_bits(b):
 
 
 def work_model(b):
-    """Algorithmic work of one batch: per valid packet
-    AES blocks ceil(C/16), SHA-1 compressions (inner ceil((C+25)/64) + outer 1,
-    the ipad/opad blocks are precomputed), bytes read D and written 48+C."""
+    """Algorithmic work of one batch: per
+    valid packet AES blocks ceil(C/16), SHA-1 compressions (inner
+    ceil((C+25)/64) + outer 1; the ipad/opad blocks are precomputed at SA
+    setup), bytes read D and written 48 + C, 16 B of metadata."""
     D = b.in_len.astype(np.int64)
     ok = (D >= 20) & (D <= 1500) & (b.sa_idx < 2**31)
     D = D[ok]
@@ -126,670 +136,427 @@ def work_model(b):
         "sha1_compressions": int(((16 + C + 8) // 64 + 1 + 1).sum()),
         "bytes_in": int(D.sum()),
         "bytes_out": int((48 + C).sum()),
-        "rec_bytes": int((((28 + C + 15) // 16) * 16).sum()),
+        "hbm_bytes": int(D.sum() + (48 + C).sum() + 16 * ok.sum()),
     }
 
 
-# Per-kernel roofline model.
-#
-# The path is integer work: AES-128 T-table rounds (shared-memory lookups plus
-# ALU byte-permutes / XORs) and SHA-1 compressions (ALU rotates / logic / adds).
-# Its roofline is the SM's integer ALU pipe: 64 int32 lanes/clk/SM (4 SMSPs x 16;
-# B300_MICROARCH.md "Pipe rates", re-measured on B200 by tools/microbench.cu:
-# 63.9 lanes/clk/SM for LOP3 / PRMT / SHF / IADD3) x 148 SMs x the max SM clock.
-# Algorithmic ALU work:
-#   AES-128-CTR block (T-table method with the per-packet round-1/2 CTR
-#   precompute): 133 table lookups, each one byte-select/address op, plus the
-#   XOR merges -> AES_ALU_OPS_PER_BLOCK = 220
-#   SHA-1 compression (FIPS 180-4 §6.1.2): 80 rounds x 5 (f, rotl5, rotl30,
-#   two 3-input adds) + 64 x 3 schedule ops -> SHA1_ALU_OPS_PER_COMPRESSION = 592
-# The shared-memory LSU (32 lookups/clk/SM) is reported alongside for AES.
-AES_ALU_OPS_PER_BLOCK = 220
-AES_LOOKUPS_PER_BLOCK = 133
-SHA1_ALU_OPS_PER_COMPRESSION = 592
-ALU_LANES_PER_CLK_SM = 64
-LDS_LANES_PER_CLK_SM = 32
+# Per-unit work, SASS-derived (tools/sass_hist.py over the shipped
+# k_fused_ring_pipe, committed as profiles/r02_sass_hist.txt): instructions per
+# AES-128 block (a quarter of the 4-block step, round loop x 7) and per SHA-1
+# compression, by issuing pipe.  Fallbacks = the r02 counts.
+SASS_HIST = os.path.join(ROOT, "profiles", "r02_sass_hist.txt")
+SASS_FALLBACK = {"aes_block": {"alu": 217.75, "fma": 19.5, "smem": 136.75},
+                 "sha1_compression": {"alu": 434, "fma": 244, "smem": 0}}
+ALU_LANES_PER_CLK_SM = 64          # B300_MICROARCH "Pipe rates"; microbenchmarked 63.9 on B200
+LDS_LANES_PER_CLK_SM = 32          # 128 B/clk/SM shared crossbar (B300_MICROARCH LDS/STS)
 
 
-def kernel_roofline(name, ms_per_launch, w, peaks):
+def sass_units():
+    try:
+        for line in open(SASS_HIST):
+            if line.startswith("JSON "):
+                d = json.loads(line[5:])
+                return {"aes_block": d["aes_block"], "sha1_compression": d["sha1_compression"],
+                        "source": "profiles/r02_sass_hist.txt"}
+    except Exception:
+        pass
+    return dict(SASS_FALLBACK, source="fallback constants (r02 SASS counts)")
+
+
+def roofline(ms_per_batch, w, peaks, units):
+    """ALU, LDS and HBM fractions of the fused kernel side by side; `bound` is
+    the resource the kernel is closest to (the largest fraction)."""
     f = peaks["sm_max_mhz"] * 1e6
-    s = ms_per_launch * 1e-3
-    alu_peak = SM_COUNT * ALU_LANES_PER_CLK_SM * f / 1e9            # Gop/s
-    aes_ops = w["aes_blocks"] * AES_ALU_OPS_PER_BLOCK
-    sha_ops = w["sha1_compressions"] * SHA1_ALU_OPS_PER_COMPRESSION
-    if name in ("fused", "fused_ring", "aes_ctr", "hmac_sha1"):
-        ops = {"fused": aes_ops + sha_ops, "fused_ring": aes_ops + sha_ops, "aes_ctr": aes_ops,
-               "hmac_sha1": sha_ops}[name]
-        r = {"bound": "alu", "unit": "Gop/s", "achieved": ops / s / 1e9, "peak": alu_peak,
-             "peak_basis": f"integer ALU pipe: {ALU_LANES_PER_CLK_SM} lanes/clk/SM x {SM_COUNT} SMs x "
-                           f"{peaks['sm_max_mhz']:.0f} MHz (microbenchmarked 63.9 lanes/clk/SM); "
-                           f"work = {AES_ALU_OPS_PER_BLOCK} ops/AES block + "
-                           f"{SHA1_ALU_OPS_PER_COMPRESSION} ops/SHA-1 compression"}
-        if name in ("fused", "fused_ring", "aes_ctr"):
-            lds = w["aes_blocks"] * AES_LOOKUPS_PER_BLOCK / s / 1e9
-            r["lds_lookups_gps"] = lds
-            r["lds_frac"] = lds / (SM_COUNT * LDS_LANES_PER_CLK_SM * f / 1e9)
-        return r
-    # memory-bound kernels: algorithmic bytes
-    if name == "gather":
-        byts = w["bytes_in"] + w["rec_bytes"]
-    elif name == "scatter":
-        byts = (w["rec_bytes"]) + w["bytes_out"]
-    else:  # prologue: read sa_idx + in_len, write rank
-        byts = w["packets"] * 10
-    return {"bound": "hbm", "unit": "GB/s", "achieved": byts / s / 1e9, "peak": peaks["hbm_gbs"],
-            "peak_basis": "measured HBM copy bandwidth"}
+    s = ms_per_batch * 1e-3
+    a, h = units["aes_block"], units["sha1_compression"]
+    alu_ops = w["aes_blocks"] * a["alu"] + w["sha1_compressions"] * h["alu"]
+    lds_ops = w["aes_blocks"] * a["smem"]
+    alu_peak = SM_COUNT * ALU_LANES_PER_CLK_SM * f / 1e12       # T lane-ops/s
+    lds_peak = SM_COUNT * LDS_LANES_PER_CLK_SM * f / 1e12
+    alu = {"achieved": alu_ops / s / 1e12, "peak": alu_peak, "unit": "Tops/s"}
+    lds = {"achieved": lds_ops / s / 1e12, "peak": lds_peak, "unit": "Tlookups/s"}
+    hbm = {"achieved": w["hbm_bytes"] / s / 1e9, "peak": peaks["hbm_gbs"], "unit": "GB/s"}
+    for x in (alu, lds, hbm):
+        x["frac"] = x["achieved"] / x["peak"]
+    return {"alu": alu, "lds": lds, "hbm": hbm,
+            "basis": (f"ALU pipe {ALU_LANES_PER_CLK_SM} lanes/clk/SM, LDS {LDS_LANES_PER_CLK_SM} "
+                      f"lanes/clk/SM, x {SM_COUNT} SMs x {peaks['sm_max_mhz']:.0f} MHz; per unit "
+                      f"(SASS, {units['source']}): AES block {a['alu']} ALU + {a['smem']} LDS, "
+                      f"SHA-1 compression {h['alu']} ALU ({h['fma']} more on the FMA pipe); HBM "
+                      f"D + 48 + C + 16 B per packet vs {peaks['source']} copy bandwidth")}
 
 
-def load_traffic(kernel, cfg_name=None):
-    """dram bytes per launch of `kernel` from the committed ncu summary, if any."""
+def load_traffic(kernel, cfg_name):
+    """DRAM bytes per batch of `kernel` from the committed ncu summary, if any."""
     p = os.path.join(ROOT, "profiles", "ncu_kernels.json")
     try:
         with open(p) as f:
             d = json.load(f)
-        key = f"{kernel}:{cfg_name}" if cfg_name else kernel
-        return d.get(key, d.get(kernel, {})).get("dram_bytes_per_launch")
+        return d.get(f"{kernel}:{cfg_name}", {}).get("dram_bytes_per_launch")
     except Exception:
         return None
 
 
+def pct(v, q):
+    return float(np.percentile(np.asarray(v, np.float64), q)) if len(v) else None
+
+
+def size_key(size):
+    return str(size)
+
+
 # --------------------------------------------------------------------------- ours
-def run_ours(args):
-    import torch
-    import torch.distributed as dist
+class Ctx:
+    """Process-group / device plumbing of one rank."""
+
+    def __init__(self, args):
+        import torch
+        import torch.distributed as dist
+        self.torch, self.dist = torch, dist
+        self.world = int(os.environ.get("WORLD_SIZE", "1"))
+        self.rank = int(os.environ.get("RANK", "0"))
+        self.local = int(os.environ.get("LOCAL_RANK", "0"))
+        if self.world != args.gpus:
+            raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={self.world}: launch one "
+                             f"process per GPU (bench.py re-launches itself under torchrun when "
+                             f"WORLD_SIZE is unset)")
+        torch.cuda.set_device(self.local)
+        self.dev = torch.device("cuda", self.local)
+        if self.world > 1:
+            dist.init_process_group("nccl", device_id=self.dev)
+        self.peaks = load_peaks()
+        self.l2 = int(getattr(torch.cuda.get_device_properties(self.dev), "L2_cache_size", 126 << 20))
+        self.flush_buf = torch.empty(256 << 20, dtype=torch.uint8, device=self.dev)
+
+    def barrier(self):
+        if self.world > 1:
+            self.dist.barrier(device_ids=[self.local])
+
+    def flush(self):
+        self.flush_buf.zero_()
+
+    def max_ms(self, ms):
+        return shard.max_over_ranks(ms, device=self.dev)
+
+    def sum_all(self, d):
+        return shard.reduce_counters(d, device=self.dev)
+
+
+def measure_outbound(ctx, args, cfg_id, size, steps, warmup, full):
+    """One workload (cfg_id / size) on this rank: the ring-timed headline pass,
+    per-batch timestamps, and (full) the process_batch / graph / isolated
+    comparisons and the profiled per-kernel pass."""
+    torch = ctx.torch
     from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
-
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
-    if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
-    peaks = load_peaks()
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
-
-    def barrier():
-        if world > 1:
-            dist.barrier(device_ids=[local])
-
-    l2_bytes = int(getattr(torch.cuda.get_device_properties(dev), "L2_cache_size", 126 << 20))
-
-    def n_rot(b):
-        """Device copies of a batch so that the rotation touches > 2x L2:
-        bytes touched per batch ~ input + output bytes at 128-byte line
-        granularity plus the metadata arrays."""
-        touched = int(b.in_len.astype(np.int64).sum()) + int(b.n) * (128 + 53 + 128 + 14)
-        return int(os.environ.get("BENCH_NROT", 0)) or max(2, -(-2 * l2_bytes // touched))
-
-    def clone_batch(d):
-        return device.DeviceBatch(n=d.n, in_buf=d.in_buf.clone(), in_off=d.in_off.clone(),
-                                  in_len=d.in_len.clone(), sa_idx=d.sa_idx.clone(),
-                                  out_buf=torch.empty_like(d.out_buf), out_off=d.out_off.clone(),
-                                  out_len=torch.empty_like(d.out_len))
-
-    def measure(cfg_id, steps, warmup, profile=True):
-        size = CFG_SIZE[cfg_id]
-        p, b = shard.rank_workload(cfg_id, PKTS_PER_GPU, size, N_SA_TOTAL, rank, world)
-        t = nba_ipsec.SATable(p, device=local, max_batch=PKTS_PER_GPU)
-        if args.pipeline is not None:
-            t.set_pipeline(args.pipeline)
-        db = device.to_device(b, dev)
-        run = lambda: t.process(*db.args(), n=b.n)  # noqa: E731
-        for _ in range(warmup):
-            flush.zero_()
-            run()
-        torch.cuda.synchronize()
-        t_end = time.time() + 0.3          # settle clocks: >= 0.3 s of back-to-back work
-        while time.time() < t_end:
-            for _ in range(20):
-                run()
-            torch.cuda.synchronize()
-        torch.cuda.synchronize()
-        barrier()
-        # timed pass (headline): K back-to-back batches on the launching
-        # stream, one CUDA event pair around all of them -- steady-state
-        # gateway throughput.  The batches rotate over R device copies whose
-        # touched bytes exceed 2x the L2, so every batch's inputs and output
-        # slots are L2-cold ("inputs larger than L2"); the SA table stays
-        # resident, as in a running gateway.
-        # The slots are launched through a batch ring (nba_ipsec_ring_run: one
-        # persistent cooperative launch walks all batches of a run; no host
-        # launch per batch); steps % R batches go through process_batch.
-        dbs = [db] + [clone_batch(db) for _ in range(n_rot(b) - 1)]
-        R = len(dbs)
-        ring = t.ring([(*d.args(), b.n) for d in dbs]) if not args.no_ring else None
-        runs = [(lambda d=d: t.process(*d.args(), n=b.n)) for d in dbs]
-
-        def timed_batches(k_steps):
-            if ring is not None:
-                ring.run(k_steps // R)
-                for k in range(k_steps % R):
-                    runs[k]()
-            else:
-                for k in range(k_steps):
-                    runs[k % R]()
-
-        timed_batches(max(warmup, 2 * R))      # >= W untimed warm-up batches
-        torch.cuda.synchronize()
-        barrier()
-        e_all = (torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-        with ClockSampler(local) as clk:
-            torch.cuda.synchronize()
-            e_all[0].record()
-            timed_batches(steps)
-            e_all[1].record()
-            torch.cuda.synchronize()
-        barrier()
-        tot_ms = e_all[0].elapsed_time(e_all[1])
-        used_ring = ring is not None and steps >= R and not os.environ.get("NBA_IPSEC_RING_GRAPH")
-        if ring is not None:
-            ring.close()
-        # isolated batches (secondary): L2 flushed before each batch, one event
-        # pair per batch (includes the launch and event-pair floor)
-        iso_steps = min(steps, 50)
-        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-              for _ in range(iso_steps)]
-        torch.cuda.synchronize()
-        for k in range(iso_steps):
-            flush.zero_()
-            ev[k][0].record()
-            run()
-            ev[k][1].record()
-        torch.cuda.synchronize()
-        step_ms = [a.elapsed_time(c) for a, c in ev]
-        # profiled pass (same protocol, per-kernel CUDA events on the stream):
-        # per-kernel durations and shares for the roofline
-        kern, nb = {}, 0
-        if profile:
-            t.profile_enable(True)
-            for k in range(max(10, steps // 4)):
-                flush.zero_()
-                run()
-            torch.cuda.synchronize()
-            kern, nb = t.profile_read()
-            t.profile_enable(False)
-        t_lpb = t.launches_per_batch()
-        # kernels launched in the timed region: one k_fused_ring per ring run
-        # (steps // R batches) plus the remaining batches' own launches
-        launches = (steps // R + (steps % R) * t_lpb) if used_ring else t_lpb * steps
-        ctr = t.counters()
-        t.close()
-        del dbs, runs
-        return dict(b=b, p=p, tot_ms=tot_ms, step_ms=step_ms, kern=kern, nb=nb, clk=clk,
-                    launches=launches, ctr=ctr, n_rot=n_rot(b),
-                    iso_ms=float(np.mean(step_ms)), lpb=t_lpb, ring=used_ring)
-
-    def kernel_times(res, steps):
-        """Average duration per launch of each kernel.  One launch per batch
-        (the fused default): the back-to-back stream time / K of the timed
-        pass (includes the inter-kernel gaps, so it is conservative).  Several
-        launches: the library's per-kernel CUDA events (profiled pass)."""
-        if res["lpb"] == 1 and len(res["kern"]) == 1:
-            # through the persistent ring the timed batches ran in k_fused_ring
-            return {(k + "_ring" if res.get("ring") else k): res["tot_ms"] / steps
-                    for k in res["kern"]}
-        return {k: v / max(res["nb"], 1) for k, v in res["kern"].items()}
-
-    def aggregate(res, steps):
-        tot_ms_max = shard.max_over_ranks(res["tot_ms"], device=dev)
-        bits = shard.reduce_counters({"pkts_ok": frame_bits(res["b"]) / 8.0, "pkts_dropped": 0,
-                                      "bytes_in": res["b"].n, "bytes_out": 0, "batches": 0},
-                                     device=dev)
-        frame_bytes_all, pkts_all = bits["pkts_ok"], bits["bytes_in"]
-        s = tot_ms_max * 1e-3
-        return {"gbps": 8.0 * frame_bytes_all * steps / s / 1e9,
-                "mpps": pkts_all * steps / s / 1e6,
-                "ms_per_step": tot_ms_max / steps}
-
-    def measure_inbound(cfg_id, steps, warmup):
-        """ESP inbound on the same traffic: the library's own
-        outbound output of R consecutive batches of the config (R as for the
-        outbound rotation: > 2x L2 touched, every batch starts L2-cold), each
-        in its own device buffers, is decapsulated back to back, K batches
-        between one CUDA event pair.  Sequence numbers grow along the rotation,
-        so every packet is fresh and accepted; when the rotation wraps, the
-        receive windows are reset (one small kernel, inside the timed region)."""
-        size = CFG_SIZE[cfg_id]
-        p, b = shard.rank_workload(cfg_id, PKTS_PER_GPU, size, N_SA_TOTAL, rank, world)
-        t_out = nba_ipsec.SATable(p, device=local, max_batch=PKTS_PER_GPU)
-        db = device.to_device(b, dev)
-        n_esp = n_rot(b)
-        esp = []
-        for _ in range(n_esp):
-            ob, ol = torch.empty_like(db.out_buf), torch.zeros_like(db.out_len)
-            t_out.process(db.in_buf, db.in_off, db.in_len, db.sa_idx, ob, db.out_off, ol, n=b.n)
-            esp.append((ob, ol, torch.empty_like(db.out_buf), torch.zeros_like(db.out_len)))
-        torch.cuda.synchronize()
-        esp_len = esp[0][1][:b.n].cpu().numpy().view(np.uint16).astype(np.int64)
-        t_out.close()
-        t = nba_ipsec.SATable(p, device=local, max_batch=PKTS_PER_GPU)
-        t.enable_inbound()
-
-        def run_k(k):
-            if k % n_esp == 0:
-                t.reset_inbound()
-            ob, ol, inner, inner_len = esp[k % n_esp]
-            t.process_inbound(ob, db.out_off, ol, db.sa_idx, inner, db.out_off, inner_len, n=b.n)
-
-        # launched through an inbound batch ring (one CUDA graph per pass over
-        # the R slots), the windows reset before each pass
-        ring = None if args.no_ring else t.ring_inbound(
-            [(e[0], db.out_off, e[1], db.sa_idx, e[2], db.out_off, e[3], None, b.n) for e in esp])
-
-        def timed_batches(k_steps):
-            if ring is None:
-                for k in range(k_steps):
-                    run_k(k)
-                return
-            for _ in range(k_steps // n_esp):
-                t.reset_inbound()
-                ring.run(1)
-            for k in range(k_steps % n_esp):
-                run_k(k)
-
-        timed_batches(max(warmup, n_esp))
-        torch.cuda.synchronize()
-        barrier()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record()
-        timed_batches(steps)
-        e1.record()
-        torch.cuda.synchronize()
-        barrier()
-        tot_ms = e0.elapsed_time(e1)
-        ctr = t.in_counters()
-        ok_all = ctr["pkts_ok"] == ctr["batches"] * b.n
-        inner_len = esp[-1][3]
-        same = bool(torch.equal(inner_len[:b.n].to(torch.int32), db.in_len[:b.n].to(torch.int32)))
-        # profiled pass (windows reset, L2 flushed per batch): kernel shares
-        t.profile_enable(True)
-        for k in range(max(10, steps // 4)):
-            flush.zero_()
-            run_k(k % n_esp)
-        torch.cuda.synchronize()
-        kern, nb = t.profile_read_inbound()
-        t.profile_enable(False)
-        if ring is not None:
-            ring.close()
-        in_launches = t.inbound_launches_per_batch()
-        if in_launches == 1:
-            kern = {k: (tot_ms / steps if v > 0 else 0.0) for k, v in kern.items()}
-            nb = 1
-        del esp
-        t.close()
-        C = esp_len - 48
-        w = {"packets": int(b.n), "aes_blocks": int(((C + 15) // 16).sum()),
-             "sha1_compressions": int(((16 + C + 8) // 64 + 1 + 1).sum()),
-             "bytes_in": int(esp_len.sum()), "bytes_out": int(b.in_len.astype(np.int64).sum())}
-        tot_max = shard.max_over_ranks(tot_ms, device=dev)
-        red = shard.reduce_counters({"pkts_ok": frame_bits(b) / 8.0, "pkts_dropped": 0,
-                                     "bytes_in": b.n, "bytes_out": float((esp_len + 14).sum()),
-                                     "batches": 0}, device=dev)
-        sec = tot_max * 1e-3
-        kk = {k: v / max(nb, 1) for k, v in kern.items()}
-        rr = {}
-        for k, ms in kk.items():
-            if ms <= 0.0:            # one-kernel form: only in_fused (replay inside it)
-                continue
-            if k == "in_fused":
-                x = kernel_roofline("fused", ms, w, peaks)
-            else:
-                x = {"bound": "hbm", "unit": "GB/s", "peak": peaks["hbm_gbs"],
-                     "achieved": w["packets"] * (38 if k == "in_replay" else 22) / (ms * 1e-3) / 1e9}
-            rr[k] = {"ms": ms, "frac": x["achieved"] / x["peak"], "unit": x["unit"],
-                     "achieved": x["achieved"], "bound": x["bound"],
-                     "traffic": load_traffic(k, gen.CONFIGS[cfg_id]["name"])}
-            if "lds_frac" in x:
-                rr[k]["lds_frac"] = x["lds_frac"]
-        return {"gbps": 8.0 * red["pkts_ok"] * steps / sec / 1e9,
-                "gbps_esp_wire": 8.0 * red["bytes_out"] * steps / sec / 1e9,
-                "mpps": red["bytes_in"] * steps / sec / 1e6,
-                "ms_per_step": tot_max / steps, "steps": steps, "kernels": rr,
-                "all_accepted": bool(ok_all), "lengths_match_outbound_input": same,
-                "gpu_launches": in_launches * steps}
-
-    def measure_alb(cfg_id, n_steps=1500, fixed_steps=20):
-        """Adaptive split with two devices emulated on one GPU:
-        device 0 runs the fused path once per packet, device 1 twice (a device
-        with half the throughput; the second pass goes to a scratch table and
-        buffer), each with its own SA table holding every SA.  Every step
-        routes one ingress batch of the config by the owner map
-        (route_pack_map), then each device processes its share, timed alone
-        with CUDA events on its own stream; as two GPUs would run their shares
-        in parallel, the step time the controller observes is the max of the
-        two (device time as its clock; paper parameters except a 1 ms update
-        interval and a 64-sample history, so it converges within the bench).
-        Run on configs[2] (1514 B), where a batch's per-packet work dominates
-        its fixed cost (on 64-byte batches splitting one batch in two never
-        pays: each device would carry the ~15 us per-batch prologue).  Counters of SAs that change owner are handed over.  Reported:
-        the trajectory of w, the last steps' throughput, fixed-split
-        throughputs for comparison, and the host cost of a hand-over and of
-        one observation."""
-        from paper_conf_eurosys_kimjlmsm15_b200 import alb, redistribute
-        size = CFG_SIZE[cfg_id]
-        p, b = shard.rank_workload(cfg_id, PKTS_PER_GPU, size, N_SA_TOTAL, 0, 1, layout="packed")
-        n_sa = len(p.spi)
-        tabs = [nba_ipsec.SATable(p, device=local, max_batch=PKTS_PER_GPU) for _ in range(2)]
-        scratch = nba_ipsec.SATable(p, device=local, max_batch=PKTS_PER_GPU)
-        sts = [torch.cuda.Stream(device=dev) for _ in range(2)]
-        db = device.to_device(b, dev)
-        main = torch.cuda.current_stream()
-
-        def step(sa_map_t):
-            pk = redistribute.pack(db, b.n, n_sa, 2, sa_map=sa_map_t)
-            dts = []
-            for d in range(2):
-                n, ioff, ilen, sa, ooff, olen, obuf = redistribute.local_views(pk, d)
-                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                sts[d].wait_stream(main)
-                with torch.cuda.stream(sts[d]):
-                    e0.record(sts[d])
-                    tabs[d].process(pk.buf, ioff, ilen, sa, obuf, ooff, olen, n=n, stream=sts[d])
-                    if d == 1:   # the slower device: the same work again (scratch state)
-                        scratch.process(pk.buf, ioff, ilen, sa, torch.empty_like(obuf), ooff,
-                                        torch.empty_like(olen), n=n, stream=sts[d])
-                    e1.record(sts[d])
-                e1.synchronize()
-                dts.append(int(e0.elapsed_time(e1) * 1e6))
-            main.wait_stream(sts[0])
-            main.wait_stream(sts[1])
-            return dts, pk.counts
-
-        def map_tensor(sa_map):
-            return torch.from_numpy(sa_map.view(np.int32)).to(dev)
-
-        fixed = {}
-        for k in (0, 4, 6, 7, 8, 9, 10, 12, 16, 25):
-            _, m = nba_ipsec.alb_assign(n_sa, 2, [k], 25)
-            mt = map_tensor(m)
-            for _ in range(3):
-                step(mt)
-            ms = sum(max(step(mt)[0]) for _ in range(fixed_steps)) / fixed_steps / 1e6
-            fixed[str(k)] = {"w": k / 25, "ms_per_step": ms, "mpps": b.n / (ms * 1e-3) / 1e6}
-        bal = alb.Balancer(n_sa, 2, history=64, update_ns=1_000_000)
-        owner, sa_map = bal.assignment()
-        mt = map_tensor(sa_map)
-        t_ns, traj, tail, ho_us, obs_ns = 0, [int(bal.node_step[0])], [], [], []
-        for j in range(n_steps):
-            dts, counts = step(mt)
-            t_ns += max(dts)
-            if j >= n_steps - 200:
-                tail.append(max(dts) / 1e6)
-            h0 = time.perf_counter_ns()
-            ch = bal.observe(t_ns, dts, counts)
-            obs_ns.append(time.perf_counter_ns() - h0)
-            if ch:
-                new_owner, new_map = bal.assignment()
-                h0 = time.perf_counter_ns()
-                alb.handover_tables(tabs, owner, new_owner)
-                ho_us.append((time.perf_counter_ns() - h0) / 1e3)
-                owner, sa_map = new_owner, new_map
-                mt = map_tensor(sa_map)
-                traj.append(int(bal.node_step[0]))
-        live = np.where(owner == 0, tabs[0].sa_seq(), tabs[1].sa_seq())
-        for t in tabs + [scratch]:
-            t.close()
-        ms_tail = float(np.mean(tail))
-        best = max(fixed.values(), key=lambda v: v["mpps"])
-        return {"devices": "2 emulated devices on one B200 (device 0: the path once per "
-                           "packet, device 1: twice = half the throughput); each share timed alone, "
-                           "step time = max of the two (parallel devices)",
-                "workload": gen.CONFIGS[cfg_id]["name"] + " as one ingress batch per step",
-                "params": {"delta": 0.04, "history": 64, "update_ms": 1.0, "wait": [2, 32],
-                           "clock": "device time"},
-                "steps": n_steps, "updates": len(traj) - 1, "w_trajectory": [k / 25 for k in traj],
-                "w_final": traj[-1] / 25,
-                "w_last10_mean": float(np.mean(traj[-10:])) / 25,
-                "last200": {"ms_per_step": ms_tail, "mpps": b.n / (ms_tail * 1e-3) / 1e6},
-                "fixed_split": fixed, "best_fixed_w": best["w"],
-                "alb_vs_best_fixed": (b.n / (ms_tail * 1e-3) / 1e6) / best["mpps"],
-                "handover_us_mean": float(np.mean(ho_us)) if ho_us else None,
-                "observe_ns_median": float(np.median(obs_ns)),
-                "packets_numbered": int(live.astype(np.int64).sum())}
-
-    def measure_flows(cfg_id, steps, warmup, n_flows=65536):
-        """Flow -> SA lookup on the config's traffic rewritten to
-        n_flows registered 5-tuples (5% unknown): the lookup kernel alone, and
-        the whole path taking its SAs from the flow table (sa_idx = NULL)."""
-        size = CFG_SIZE[cfg_id]
-        p, b = shard.rank_workload(cfg_id, PKTS_PER_GPU, size, N_SA_TOTAL, rank, world)
-        f = gen.make_flows(n_flows, len(p.spi), cfg_id=cfg_id, rank=rank)
-        gen.apply_flows(b, f, cfg_id=cfg_id, miss=0.05)
-        t = nba_ipsec.SATable(p, device=local, max_batch=PKTS_PER_GPU)
-        t.set_flow_table(f)
-        db = device.to_device(b, dev)
-        sa_out = torch.empty(b.n, dtype=torch.int32, device=dev)
-        look = lambda: t.lookup_sa(db.in_buf, db.in_off, db.in_len, sa_out, n=b.n)  # noqa: E731
-        path = lambda: t.process(db.in_buf, db.in_off, db.in_len, None, db.out_buf, db.out_off,  # noqa: E731
-                                 db.out_len, n=b.n)
-        out = {}
-        for name, fn in (("lookup", look), ("path_with_lookup", path)):
-            for _ in range(warmup):
-                flush.zero_()
-                fn()
-            torch.cuda.synchronize()
-            barrier()
-            ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-                  for _ in range(steps)]
-            for k in range(steps):
-                flush.zero_()
-                ev[k][0].record()
-                fn()
-                ev[k][1].record()
-            torch.cuda.synchronize()
-            ms = shard.max_over_ranks(sum(a.elapsed_time(c) for a, c in ev) / steps, device=dev)
-            red = shard.reduce_counters({"pkts_ok": frame_bits(b) / 8.0, "pkts_dropped": 0,
-                                         "bytes_in": b.n, "bytes_out": 0, "batches": 0}, device=dev)
-            out[name] = {"ms_per_step": ms, "mpps": red["bytes_in"] / (ms * 1e-3) / 1e6,
-                         "gbps": 8.0 * red["pkts_ok"] / (ms * 1e-3) / 1e9}
-        # lookup roofline: HBM bytes of the headers read + SA indices written
-        # (table probes are L2 hits: 65,536 flows x 16 B x 2 = 2 MiB)
-        byts = b.n * (32 + 4 + 4 + 2)
-        out["lookup"]["roofline"] = {"bound": "hbm", "unit": "GB/s", "peak": peaks["hbm_gbs"],
-                                     "achieved": byts / (out["lookup"]["ms_per_step"] * 1e-3) / 1e9}
-        out["lookup"]["roofline"]["frac"] = out["lookup"]["roofline"]["achieved"] / peaks["hbm_gbs"]
-        out["n_flows"] = n_flows
-        out["miss_fraction"] = 0.05
-        t.close()
-        # single-ingress routing (f3): pack the batch for 8 owners (the
-        # all-to-all itself needs >1 GPU); HBM roofline on the bytes moved
-        from paper_conf_eurosys_kimjlmsm15_b200 import redistribute
-        for _ in range(warmup):
-            flush.zero_()
-            redistribute.pack(db, b.n, len(p.spi), 8)
-        torch.cuda.synchronize()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        tot = 0.0
-        for k in range(steps):
-            flush.zero_()
-            e0.record()
-            pk = redistribute.pack(db, b.n, len(p.spi), 8)     # (includes a 2-value D2H for the splits)
-            e1.record()
-            torch.cuda.synchronize()
-            tot += e0.elapsed_time(e1)
-        ms = tot / steps
-        moved = 2 * int(b.in_len.astype(np.int64).sum()) + b.n * (4 + 2 + 4 + 2 + 4 + 12)
-        # the same routing with the data written straight into 8 owners' receive
-        # buffers (nba_ipsec_route_dispatch; here all on this GPU, standing in for
-        # peer GPUs' memory over NVLink): no send buffer, no all-to-all
-        from paper_conf_eurosys_kimjlmsm15_b200 import nba_ipsec as _nb
-        cap_b = int(b.in_len.astype(np.int64).sum()) + 64
-        rxs = [redistribute.alloc_rx(b.n, cap_b, dev) for _ in range(8)]
-        table = redistribute.rx_table(rxs, dev)
-        ws = torch.empty(_nb.route_workspace_bytes(b.n, 8), dtype=torch.uint8, device=dev)
-        dcnt = torch.zeros(9, dtype=torch.int64, device=dev)
-        dbyt = torch.zeros(9, dtype=torch.int64, device=dev)
-        disp = lambda: _nb.route_dispatch(db.in_buf, db.in_off, db.in_len, db.sa_idx, b.n,  # noqa: E731
-                                          len(p.spi), None, 8, ws, table, b.n, cap_b, dcnt, dbyt)
-        for _ in range(warmup):
-            flush.zero_()
-            disp()
-        torch.cuda.synchronize()
-        tot_d = 0.0
-        for k in range(steps):
-            flush.zero_()
-            e0.record()
-            disp()
-            e1.record()
-            torch.cuda.synchronize()
-            tot_d += e0.elapsed_time(e1)
-        ms_d = tot_d / steps
-        moved_d = 2 * int(b.in_len.astype(np.int64).sum()) + b.n * (4 + 2 + 4 + 4 + 2 + 4 + 4)
-        out["dispatch_8_owners"] = {"ms_per_step": ms_d, "mpps": b.n / (ms_d * 1e-3) / 1e6,
-                                    "roofline": {"bound": "hbm", "unit": "GB/s", "peak": peaks["hbm_gbs"],
-                                                 "achieved": moved_d / (ms_d * 1e-3) / 1e9,
-                                                 "frac": moved_d / (ms_d * 1e-3) / 1e9 / peaks["hbm_gbs"]},
-                                    "note": "route + write into 8 owners' receive buffers in one "
-                                            "pass (single-GPU stand-in for NVLink peers)"}
-        del rxs
-        out["route_pack_8_owners"] = {"ms_per_step": ms, "mpps": b.n / (ms * 1e-3) / 1e6,
-                                      "roofline": {"bound": "hbm", "unit": "GB/s", "peak": peaks["hbm_gbs"],
-                                                   "achieved": moved / (ms * 1e-3) / 1e9,
-                                                   "frac": moved / (ms * 1e-3) / 1e9 / peaks["hbm_gbs"]},
-                                      "packets_per_owner": pk.counts}
-        return out
-
-    main_cfg = args.config
-    res = measure(main_cfg, args.steps, args.warmup)
-    agg = aggregate(res, args.steps)
-
-    # per-kernel breakdown and roofline of the dominant kernel (this rank)
-    w = work_model(res["b"])
-    kern_avg = kernel_times(res, args.steps)
-    dom = max(kern_avg, key=kern_avg.get) if kern_avg else None
-    roof = None
-    kern_roofs = {}
-    for k, ms in kern_avg.items():
-        r = kernel_roofline(k, ms, w, peaks)
-        r["frac"] = r["achieved"] / r["peak"]
-        r["ms_per_launch"] = ms
-        kern_roofs[k] = r
-    if dom:
-        r = kern_roofs[dom]
-        roof = {"kernel": dom, "bound": r["bound"], "achieved": r["achieved"], "peak": r["peak"],
-                "unit": r["unit"], "frac": r["frac"],
-                "traffic": load_traffic(dom, gen.CONFIGS[main_cfg]["name"]),
-                "traffic_unit": "bytes per launch (ncu dram__bytes_read.sum + dram__bytes_write.sum)",
-                "peak_basis": r["peak_basis"], "peak_source": peaks["source"],
-                "share_of_step": kern_avg[dom] / max(sum(kern_avg.values()), 1e-12)}
-
-    # ---- e2e: host buffers through nba_ipsec_process_batch_host ---------------
-    e2e = run_e2e(args, rank, world, local, dev, barrier)
-
-    # ---- other packet sizes (same protocol, fewer steps) ------------------------
-    per_size = {}
-    if not args.no_sweep:
-        for cfg_id in (2, 3, 4):
-            if cfg_id == main_cfg:
-                per_size[str(CFG_SIZE[cfg_id])] = {"gbps": agg["gbps"], "mpps": agg["mpps"],
-                                                   "ms_per_step": agg["ms_per_step"]}
-                continue
-            r2 = measure(cfg_id, max(10, args.steps // 4), max(3, args.warmup // 2))
-            a2 = aggregate(r2, max(10, args.steps // 4))
-            kk = kernel_times(r2, max(10, args.steps // 4))
-            w2 = work_model(r2["b"])
-            rr = {}
-            for k, ms in kk.items():
-                x = kernel_roofline(k, ms, w2, peaks)
-                rr[k] = {"ms": ms, "frac": x["achieved"] / x["peak"], "unit": x["unit"],
-                         "achieved": x["achieved"], "bound": x["bound"]}
-            per_size[str(CFG_SIZE[cfg_id])] = {"gbps": a2["gbps"], "mpps": a2["mpps"],
-                                               "ms_per_step": a2["ms_per_step"], "kernels": rr}
-
-    # ---- ESP inbound on the same traffic (SURVEY f2) ----------------------------
-    inbound = {}
-    if not args.no_inbound:
-        for cfg_id in (2, 3, 4):
-            inbound[str(CFG_SIZE[cfg_id])] = measure_inbound(cfg_id, max(10, args.steps // 4),
-                                                            max(3, args.warmup // 2))
-
-    # ---- flow -> SA lookup (SURVEY f3) -----------------------------------------
-    flows = None
-    if not args.no_inbound:
-        flows = {str(CFG_SIZE[main_cfg]): measure_flows(main_cfg, max(10, args.steps // 4),
-                                                        max(3, args.warmup // 2))}
-
-    # ---- adaptive split across devices (SURVEY f4; one GPU: two tables) --------
-    alb_res = None
-    if world == 1 and not args.no_alb:
-        alb_res = measure_alb(3)    # 1514 B: per-packet work dominates the batch's fixed cost
-
-    # ---- CPU baseline: the oracle on host cores (rank 0, N = 1 only) ----------
-    cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu:
-        cpu = cpu_baseline(res["p"], res["b"], budget_s=args.cpu_seconds,
-                           label=gen.CONFIGS[main_cfg]["name"])
-
-    ctr_all = shard.reduce_counters(res["ctr"], device=dev)
-    if rank == 0:
-        clk = res["clk"].summary()
-        out = {
-            "metric": METRIC,
-            "value": agg["gbps"],
-            "unit": "Gbps",
-            "mpps": agg["mpps"],
-            "n_gpus": world,
-            "steps": args.steps,
-            "warmup": args.warmup,
-            "ms_per_step": agg["ms_per_step"],
-            "higher_is_better": True,
-            "scaling": "weak",
-            "vs_baseline": None,
-            "dtype": "u8",
-            "data": "synthetic (seeded random IPv4/UDP, random SA keys; PAPER.md:395 workload shape)",
-            "config": {"workload": f"configs[{main_cfg - 1}]: {gen.CONFIGS[main_cfg]['name']}",
-                       "frame_bytes": CFG_SIZE[main_cfg], "packets_per_gpu": PKTS_PER_GPU,
-                       "n_sa_total": N_SA_TOTAL, "global_batch": PKTS_PER_GPU * world,
-                       "parallelism": f"sa-hash shard x{world} (no data-path collective)",
-                       "l2": f"inputs larger than L2: batches rotate over {res['n_rot']} device copies "
-                             "(> 2x L2 touched per rotation), SA table resident",
-                       "timing": "K back-to-back batches on the launching stream between one CUDA "
-                                 "event pair, max over ranks" + ("" if args.no_ring else
-                                 "; launched through the batch ring (nba_ipsec_ring_run over the "
-                                 "rotation's slots: one persistent cooperative launch per run)"),
-                       "pipeline": ("fused" if args.pipeline in (None, 0) else "unfused") +
-                                   (f" (k_fused_ring: one launch per ring run of {res['n_rot']} "
-                                    f"batches; {res['launches']} launches for {args.steps} steps)"
-                                    if res.get("ring") else
-                                    f" ({res['launches'] // args.steps} launch(es) per step)")},
-            "roofline": roof,
-            "kernels": {k: {"ms_per_launch": v["ms_per_launch"], "frac": v["frac"], "unit": v["unit"],
-                            "achieved": v["achieved"]} for k, v in kern_roofs.items()},
-            "work_per_step_per_gpu": w,
-            "isolated_batch": {"ms_per_step": res["iso_ms"],
-                               "gbps_per_gpu": frame_bits(res["b"]) / (res["iso_ms"] * 1e-3) / 1e9,
-                               "note": "one batch at a time: L2 flushed (256 MiB write) before each, "
-                                       "one CUDA event pair per batch (adds the launch and the "
-                                       "~2.6 us event-pair floor)"},
-            "per_size": per_size,
-            "inbound": inbound or None,
-            "flow_lookup": flows,
-            "adaptive_split": alb_res,
-            "cpu_baseline": cpu,
-            "e2e": e2e,
-            "gpu_launches": res["launches"],
-            "counters": ctr_all,
-            "clocks": clk,
-        }
-        print(json.dumps(out), flush=True)
-    if world > 1:
-        dist.destroy_process_group()
-
-
-def run_e2e(args, rank, world, local, dev, barrier):
-    """Same metric through nba_ipsec_process_batch_host: every step copies the
-    step's inputs from pinned host memory and reads back the results."""
-    import torch
-    from paper_conf_eurosys_kimjlmsm15_b200 import nba_ipsec
-    size = CFG_SIZE[args.config]
-    # packed datagrams in, output slots of D + 53 bytes (the largest ESP
-    # overhead, NBA_IPSEC_MAX_OVERHEAD) out: the fewest bytes over PCIe
-    p, b = shard.rank_workload(args.config, PKTS_PER_GPU, size, N_SA_TOTAL, rank, world,
-                               layout="packed", out_pad=53)
-    t = nba_ipsec.SATable(p, device=local, max_batch=PKTS_PER_GPU)
+    p, b = shard.rank_workload(cfg_id, PKTS_PER_GPU, size, N_SA_TOTAL, ctx.rank, ctx.world)
+    t = nba_ipsec.SATable(p, device=ctx.local, max_batch=PKTS_PER_GPU)
     if args.pipeline is not None:
         t.set_pipeline(args.pipeline)
+    db = device.to_device(b, ctx.dev)
+    R = int(os.environ.get("BENCH_NROT", 0)) or device.ring_slot_count(b.in_len, b.n, ctx.l2)
+    dbs = [db] + [device.clone(db) for _ in range(R - 1)]
+    slots = [(*d.args(), b.n) for d in dbs]
+    ring = t.ring(slots)
+    form = {0: "graph", 1: "persistent", 2: "pipelined"}[ring.form]
+    # settle clocks (>= 0.3 s of back-to-back batches), then >= W warm-up batches
+    t_end = time.time() + 0.3
+    while time.time() < t_end:
+        ring.run_batches(4 * R)
+        torch.cuda.synchronize()
+    ring.run_batches(max(warmup, 2 * R))
+    torch.cuda.synchronize()
+    ctx.barrier()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(ctx.local) as clk:
+        torch.cuda.synchronize()
+        e0.record()
+        ring.run_batches(steps)            # ALL K timed batches: ONE persistent launch
+        e1.record()
+        torch.cuda.synchronize()
+    ctx.barrier()
+    tot_ms = e0.elapsed_time(e1)
+    res = {"b": b, "p": p, "R": R, "form": form, "tot_ms": tot_ms, "clk": clk, "launches": 1}
+    # per-batch device timestamps (a second, identical pass)
+    per_batch = None
+    if ring.form != 0:
+        ts = torch.zeros(steps + 1, dtype=torch.int64, device=ctx.dev)
+        ring.set_timestamps(ts)
+        ring.run_batches(steps)
+        torch.cuda.synchronize()
+        ring.set_timestamps(None)
+        v = ts.cpu().numpy().astype(np.int64)
+        d_us = np.diff(v)[1:] / 1e3         # batch 0 includes the ring's start-up
+        per_batch = {"median_us": pct(d_us, 50), "p10_us": pct(d_us, 10), "p90_us": pct(d_us, 90),
+                     "mean_us": float((v[-1] - v[1]) / 1e3 / max(steps - 1, 1)),
+                     "first_us": float((v[1] - v[0]) / 1e3), "n": int(d_us.size)}
+    res["per_batch"] = per_batch
+    ring.close()
+    if full:
+        runs = [(lambda d=d: t.process(*d.args(), n=b.n)) for d in dbs]
+        # (a) the same K batches as process_batch launches, back to back
+        for k in range(2 * R):
+            runs[k % R]()
+        torch.cuda.synchronize()
+        e0.record()
+        for k in range(steps):
+            runs[k % R]()
+        e1.record()
+        torch.cuda.synchronize()
+        res["launch_loop_ms"] = e0.elapsed_time(e1)
+        res["lpb"] = t.launches_per_batch()
+        # (b) CUDA-graph replay of the slots' launches (the ring's graph form)
+        os.environ["NBA_IPSEC_RING_GRAPH"] = "1"
+        try:
+            g = t.ring(slots)
+        finally:
+            del os.environ["NBA_IPSEC_RING_GRAPH"]
+        g.run_batches(2 * R)
+        torch.cuda.synchronize()
+        e0.record()
+        g.run_batches(steps)
+        e1.record()
+        torch.cuda.synchronize()
+        res["graph_ms"] = e0.elapsed_time(e1)
+        g.close()
+        # (c) isolated batches: L2 flushed before each, one event pair per batch
+        iso = min(steps, 50)
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+              for _ in range(iso)]
+        for k in range(iso):
+            ctx.flush()
+            ev[k][0].record()
+            runs[0]()
+            ev[k][1].record()
+        torch.cuda.synchronize()
+        res["iso_ms"] = [a.elapsed_time(c) for a, c in ev]
+    res["ctr"] = t.counters()
+    t.close()
+    del dbs
+    return res
+
+
+def rates(ctx, res, steps, ms=None):
+    """Whole-job Gbps / Mpps / ESP-payload Gbps over all ranks for `steps`
+    batches per rank in `ms` (default: the ring-timed pass), max over ranks."""
+    b = res["b"]
+    ms_max = ctx.max_ms(res["tot_ms"] if ms is None else ms)
+    s = ms_max * 1e-3
+    tot = ctx.sum_all({"pkts_ok": frame_bits(b) / 8.0, "pkts_dropped": 0, "bytes_in": b.n,
+                       "bytes_out": int(b.in_len.astype(np.int64).sum()), "batches": 0})
+    return {"gbps": 8.0 * tot["pkts_ok"] * steps / s / 1e9, "mpps": tot["bytes_in"] * steps / s / 1e6,
+            "esp_payload_gbps": 8.0 * tot["bytes_out"] * steps / s / 1e9,
+            "ms_per_step": ms_max / steps}
+
+
+def measure_inbound(ctx, args, cfg_id, steps, warmup):
+    """ESP inbound on the same traffic: the library's own outbound
+    output of R consecutive batches of the config (> 2x L2 touched per
+    rotation, every batch L2-cold), each in its own device buffers,
+    decapsulated back to back, K batches between one CUDA event pair.  Sequence
+    numbers grow along the rotation, so every packet is fresh and accepted;
+    when the rotation wraps the receive windows are reset (one small kernel,
+    inside the timed region).  The rotation runs through the inbound batch ring
+    (nba_ipsec_ring_run_batches, one call per rotation)."""
+    torch = ctx.torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    size = CFG_SIZE[cfg_id]
+    p, b = shard.rank_workload(cfg_id, PKTS_PER_GPU, size, N_SA_TOTAL, ctx.rank, ctx.world)
+    t_out = nba_ipsec.SATable(p, device=ctx.local, max_batch=PKTS_PER_GPU)
+    db = device.to_device(b, ctx.dev)
+    R = device.ring_slot_count(b.in_len, b.n, ctx.l2)
+    esp = []
+    for _ in range(R):
+        ob, ol = torch.empty_like(db.out_buf), torch.zeros_like(db.out_len)
+        t_out.process(db.in_buf, db.in_off, db.in_len, db.sa_idx, ob, db.out_off, ol, n=b.n)
+        esp.append((ob, ol, torch.empty_like(db.out_buf), torch.zeros_like(db.out_len)))
+    torch.cuda.synchronize()
+    esp_len = esp[0][1][:b.n].cpu().numpy().view(np.uint16).astype(np.int64)
+    t_out.close()
+    t = nba_ipsec.SATable(p, device=ctx.local, max_batch=PKTS_PER_GPU)
+    t.enable_inbound()
+    ring = t.ring_inbound([(e[0], db.out_off, e[1], db.sa_idx, e[2], db.out_off, e[3], None, b.n)
+                           for e in esp])
+
+    def timed_batches(k_steps):
+        left = k_steps
+        while left:
+            if ring.cursor == 0:
+                t.reset_inbound()
+            nb = min(left, R - ring.cursor)
+            ring.run_batches(nb)
+            left -= nb
+
+    timed_batches(max(warmup, R))
+    torch.cuda.synchronize()
+    ctx.barrier()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    timed_batches(steps)
+    e1.record()
+    torch.cuda.synchronize()
+    ctx.barrier()
+    tot_ms = e0.elapsed_time(e1)
+    ctr = t.in_counters()
+    ok_all = ctr["pkts_ok"] == ctr["batches"] * b.n
+    same = bool(torch.equal(esp[-1][3][:b.n].to(torch.int32), db.in_len[:b.n].to(torch.int32)))
+    form = {0: "graph", 1: "persistent", 2: "pipelined"}[ring.form]
+    ring.close()
+    del esp
+    t.close()
+    tot_max = ctx.max_ms(tot_ms)
+    red = ctx.sum_all({"pkts_ok": frame_bits(b) / 8.0, "pkts_dropped": 0, "bytes_in": b.n,
+                       "bytes_out": float((esp_len + 14).sum()), "batches": 0})
+    sec = tot_max * 1e-3
+    return {"gbps": 8.0 * red["pkts_ok"] * steps / sec / 1e9,
+            "gbps_esp_wire": 8.0 * red["bytes_out"] * steps / sec / 1e9,
+            "mpps": red["bytes_in"] * steps / sec / 1e6, "us_per_step": 1e3 * tot_max / steps,
+            "all_accepted": bool(ok_all), "lengths_match_outbound_input": same, "ring_form": form}
+
+
+def measure_flows(ctx, args, cfg_id, steps, warmup, n_flows=65536):
+    """Flow -> SA lookup on the config's traffic rewritten to
+    n_flows registered 5-tuples (5% unknown): the lookup kernel alone and the
+    whole path taking its SAs from the flow table (sa_idx = NULL); and
+    single-ingress dispatch into 8 owners' receive buffers (one GPU standing in
+    for NVLink peers)."""
+    torch = ctx.torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec, redistribute
+    size = CFG_SIZE[cfg_id]
+    p, b = shard.rank_workload(cfg_id, PKTS_PER_GPU, size, N_SA_TOTAL, ctx.rank, ctx.world)
+    f = gen.make_flows(n_flows, len(p.spi), cfg_id=cfg_id, rank=ctx.rank)
+    gen.apply_flows(b, f, cfg_id=cfg_id, miss=0.05)
+    t = nba_ipsec.SATable(p, device=ctx.local, max_batch=PKTS_PER_GPU)
+    t.set_flow_table(f)
+    db = device.to_device(b, ctx.dev)
+    sa_out = torch.empty(b.n, dtype=torch.int32, device=ctx.dev)
+    cap_b = int(b.in_len.astype(np.int64).sum()) + 64
+    rxs = [redistribute.alloc_rx(b.n, cap_b, ctx.dev) for _ in range(8)]
+    table = redistribute.rx_table(rxs, ctx.dev)
+    ws = torch.empty(nba_ipsec.route_workspace_bytes(b.n, 8), dtype=torch.uint8, device=ctx.dev)
+    dcnt = torch.zeros(9, dtype=torch.int64, device=ctx.dev)
+    dbyt = torch.zeros(9, dtype=torch.int64, device=ctx.dev)
+    fns = {
+        "lookup": lambda: t.lookup_sa(db.in_buf, db.in_off, db.in_len, sa_out, n=b.n),
+        "path_with_lookup": lambda: t.process(db.in_buf, db.in_off, db.in_len, None, db.out_buf,
+                                              db.out_off, db.out_len, n=b.n),
+        "dispatch_8_owners": lambda: nba_ipsec.route_dispatch(
+            db.in_buf, db.in_off, db.in_len, db.sa_idx, b.n, len(p.spi), None, 8, ws, table, b.n,
+            cap_b, dcnt, dbyt),
+    }
+    out = {}
+    for name, fn in fns.items():
+        for _ in range(warmup):
+            ctx.flush()
+            fn()
+        torch.cuda.synchronize()
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+              for _ in range(steps)]
+        for k in range(steps):
+            ctx.flush()
+            ev[k][0].record()
+            fn()
+            ev[k][1].record()
+        torch.cuda.synchronize()
+        ms = ctx.max_ms(sum(a.elapsed_time(c) for a, c in ev) / steps)
+        out[name] = {"us": 1e3 * ms, "mpps": b.n / (ms * 1e-3) / 1e6}
+    moved = 2 * int(b.in_len.astype(np.int64).sum()) + b.n * 28
+    out["dispatch_8_owners"]["hbm_frac"] = moved / (out["dispatch_8_owners"]["us"] * 1e-6) / 1e9 / \
+        ctx.peaks["hbm_gbs"]
+    out["n_flows"], out["miss_fraction"] = n_flows, 0.05
+    t.close()
+    del rxs
+    return out
+
+
+def measure_alb(ctx, args, cfg_id, n_steps=1500, fixed_steps=20):
+    """Adaptive split with two devices emulated on one GPU: device 0
+    runs the fused path once per packet, device 1 twice (half the throughput),
+    each with its own SA table holding every SA.  Every step routes one ingress
+    batch of the config by the owner map (route_pack_map), then each device
+    processes its share, timed alone with CUDA events on its own stream; the
+    controller observes the max of the two (parallel devices).  Counters of SAs
+    that change owner are handed over."""
+    torch = ctx.torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import alb, device, nba_ipsec, redistribute
+    size = CFG_SIZE[cfg_id]
+    p, b = shard.rank_workload(cfg_id, PKTS_PER_GPU, size, N_SA_TOTAL, 0, 1, layout="packed")
+    n_sa = len(p.spi)
+    tabs = [nba_ipsec.SATable(p, device=ctx.local, max_batch=PKTS_PER_GPU) for _ in range(2)]
+    scratch = nba_ipsec.SATable(p, device=ctx.local, max_batch=PKTS_PER_GPU)
+    sts = [torch.cuda.Stream(device=ctx.dev) for _ in range(2)]
+    db = device.to_device(b, ctx.dev)
+    main = torch.cuda.current_stream()
+
+    def step(sa_map_t):
+        pk = redistribute.pack(db, b.n, n_sa, 2, sa_map=sa_map_t)
+        dts = []
+        for d in range(2):
+            n, ioff, ilen, sa, ooff, olen, obuf = redistribute.local_views(pk, d)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            sts[d].wait_stream(main)
+            with torch.cuda.stream(sts[d]):
+                e0.record(sts[d])
+                tabs[d].process(pk.buf, ioff, ilen, sa, obuf, ooff, olen, n=n, stream=sts[d])
+                if d == 1:
+                    scratch.process(pk.buf, ioff, ilen, sa, torch.empty_like(obuf), ooff,
+                                    torch.empty_like(olen), n=n, stream=sts[d])
+                e1.record(sts[d])
+            e1.synchronize()
+            dts.append(int(e0.elapsed_time(e1) * 1e6))
+        main.wait_stream(sts[0])
+        main.wait_stream(sts[1])
+        return dts, pk.counts
+
+    def map_tensor(sa_map):
+        return torch.from_numpy(sa_map.view(np.int32)).to(ctx.dev)
+
+    fixed = {}
+    for k in (0, 4, 8, 12, 16, 25):
+        _, m = nba_ipsec.alb_assign(n_sa, 2, [k], 25)
+        mt = map_tensor(m)
+        for _ in range(3):
+            step(mt)
+        ms = sum(max(step(mt)[0]) for _ in range(fixed_steps)) / fixed_steps / 1e6
+        fixed[str(k / 25)] = round(b.n / (ms * 1e-3) / 1e6, 1)
+    bal = alb.Balancer(n_sa, 2, history=64, update_ns=1_000_000)
+    owner, sa_map = bal.assignment()
+    mt = map_tensor(sa_map)
+    t_ns, traj, tail, ho_us = 0, [int(bal.node_step[0])], [], []
+    for j in range(n_steps):
+        dts, counts = step(mt)
+        t_ns += max(dts)
+        if j >= n_steps - 200:
+            tail.append(max(dts) / 1e6)
+        if bal.observe(t_ns, dts, counts):
+            new_owner, new_map = bal.assignment()
+            h0 = time.perf_counter_ns()
+            alb.handover_tables(tabs, owner, new_owner)
+            ho_us.append((time.perf_counter_ns() - h0) / 1e3)
+            owner, sa_map = new_owner, new_map
+            mt = map_tensor(sa_map)
+            traj.append(int(bal.node_step[0]))
+    for t in tabs + [scratch]:
+        t.close()
+    ms_tail = float(np.mean(tail))
+    best_w = max(fixed, key=fixed.get)
+    mpps = b.n / (ms_tail * 1e-3) / 1e6
+    return {"devices": "2 emulated on one B200 (device 1 does the work twice); step = max of the two",
+            "workload": gen.CONFIGS[cfg_id]["name"], "updates": len(traj) - 1,
+            "w_final": traj[-1] / 25, "w_last10_mean": float(np.mean(traj[-10:])) / 25,
+            "mpps_last200": mpps, "mpps_fixed_w": fixed, "best_fixed_w": float(best_w),
+            "alb_vs_best_fixed": mpps / fixed[best_w],
+            "handover_us_mean": float(np.mean(ho_us)) if ho_us else None}
+
+
+def run_e2e(ctx, args):
+    """Same metric through nba_ipsec_process_batch_host: every step copies the
+    step's inputs from pinned host memory and reads back the results."""
+    torch = ctx.torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import nba_ipsec
+    size = CFG_SIZE[args.config]
+    p, b = shard.rank_workload(args.config, PKTS_PER_GPU, size, N_SA_TOTAL, ctx.rank, ctx.world,
+                               layout="packed", out_pad=53)
+    t = nba_ipsec.SATable(p, device=ctx.local, max_batch=PKTS_PER_GPU)
     in_bytes = int(b.in_off[-1]) + int(b.in_len[-1])
     out_bytes = int(b.out_pool_bytes)
     t.reserve_host_io(in_bytes, out_bytes)
@@ -799,7 +566,7 @@ def run_e2e(args, rank, world, local, dev, barrier):
     h_ooff = pin(b.out_off.view(np.int32))
     h_out = torch.empty(out_bytes, dtype=torch.uint8).pin_memory()
     h_olen = torch.empty(b.n, dtype=torch.int16).pin_memory()
-    st = torch.cuda.current_stream(dev)
+    st = torch.cuda.current_stream(ctx.dev)
 
     def step():
         t.process_host(h_in, h_off, h_len, h_sa, h_out, h_ooff, h_olen, in_bytes, out_bytes,
@@ -809,7 +576,7 @@ def run_e2e(args, rank, world, local, dev, barrier):
         step()
     t.host_wait(st)
     torch.cuda.synchronize()
-    barrier()
+    ctx.barrier()
     steps = max(5, args.steps // 2)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record()
@@ -818,10 +585,10 @@ def run_e2e(args, rank, world, local, dev, barrier):
     t.host_wait(st)            # the last step's outputs are in host memory
     e1.record()
     torch.cuda.synchronize()
-    barrier()
-    ms = shard.max_over_ranks(e0.elapsed_time(e1), device=dev)
-    tot = shard.reduce_counters({"pkts_ok": frame_bits(b) / 8.0, "pkts_dropped": 0, "bytes_in": b.n,
-                                 "bytes_out": 0, "batches": 0}, device=dev)
+    ctx.barrier()
+    ms = ctx.max_ms(e0.elapsed_time(e1))
+    tot = ctx.sum_all({"pkts_ok": frame_bits(b) / 8.0, "pkts_dropped": 0, "bytes_in": b.n,
+                       "bytes_out": 0, "batches": 0})
     t.close()
     h2d = in_bytes + b.n * (4 + 2 + 4 + 4)
     d2h = out_bytes + b.n * 2
@@ -829,33 +596,213 @@ def run_e2e(args, rank, world, local, dev, barrier):
             "mpps": tot["bytes_in"] * steps / (ms * 1e-3) / 1e6,
             "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
             "steps": steps, "ms_per_step": ms / steps,
-            "note": "nba_ipsec_process_batch_host: pinned H2D of packed datagrams + metadata, "
-                    "kernels, D2H of output pool + out_len every step; copy-in / kernels / "
-                    "copy-out pipelined over consecutive steps (2 staging slots); timed from the "
-                    "first copy-in to the last copy-out"}
+            "api": "nba_ipsec_process_batch_host (pinned H2D of packed datagrams + metadata, "
+                   "kernels, D2H of output pool + out_len every step, 2 staging slots pipelined)"}
 
 
-def cpu_baseline(p, b, budget_s=3.0, threads=None, label=""):
-    """The oracle as it stands (plain C, -O2) on the host's cores: full batches
-    repeated until `budget_s` of wall time, SAs partitioned s mod T over T threads."""
+def cpu_model():
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            if line.startswith("Model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return None
+
+
+def oracle_leg(p, b, threads, budget_s):
+    """The oracle as it stands (plain C -O2, SAs partitioned s mod T over T
+    threads) on a bounded sample of batch b: the first m packets, m sized from a
+    probe so one call takes ~budget_s / 3, repeated until budget_s."""
     import oracle
-    T = threads or len(os.sched_getaffinity(0))
     sas = oracle.make_sas(p)
     n_sa = len(p.spi)
     out = np.zeros(b.out_pool_bytes, np.uint8)
+
+    def sub(m):
+        return gen.Batch(n=m, in_buf=b.in_buf, in_off=b.in_off[:m], in_len=b.in_len[:m],
+                         sa_idx=b.sa_idx[:m], out_off=b.out_off[:m], out_pool_bytes=b.out_pool_bytes,
+                         frame_len=b.frame_len[:m])
+    probe = sub(min(b.n, 2048))
     t0 = time.perf_counter()
-    reps = 0
+    oracle.process_batch(sas, n_sa, probe, n_threads=threads, out_buf=out)
+    per_pkt = (time.perf_counter() - t0) / probe.n
+    m = int(max(256, min(b.n, budget_s / 3.0 / max(per_pkt, 1e-9))))
+    sb = sub(m)
+    reps, t0 = 0, time.perf_counter()
     while True:
-        oracle.process_batch(sas, n_sa, b, n_threads=T, out_buf=out)
+        oracle.process_batch(sas, n_sa, sb, n_threads=threads, out_buf=out)
         reps += 1
         el = time.perf_counter() - t0
         if el >= budget_s:
             break
-    gbps = frame_bits(b) * reps / el / 1e9
-    return {"value": gbps, "unit": "Gbps", "mpps": b.n * reps / el / 1e6, "cores": T,
-            "kind": "oracle",
-            "sample": f"{reps} full batch(es) of {b.n} packets ({label}, the benchmarked batch), "
-                      f"{el:.2f} s wall on {T} threads (~{el * T:.0f} CPU-s)"}
+    return {"gbps": frame_bits(sb) * reps / el / 1e9, "mpps": m * reps / el / 1e6, "threads": threads,
+            "sample": f"first {m} of {b.n} packets x {reps} ({el:.1f} s)"}
+
+
+def cpu_baselines(budget_s):
+    """SURVEY §8(d) oracle timing: configs[0] in ms (1 thread), and configs[1..3]
+    on 1 thread and on all host threads (bounded samples)."""
+    import oracle
+    T = len(os.sched_getaffinity(0))
+    c = gen.CONFIGS[1]
+    p1 = gen.make_sas(c["n_sa"], cfg_id=1)
+    b1 = gen.make_batch(c["n"], c["size"], c["n_sa"], cfg_id=1)
+    ms = []
+    t_end = time.perf_counter() + 0.5
+    while time.perf_counter() < t_end or len(ms) < 5:
+        sas = oracle.make_sas(p1)
+        t0 = time.perf_counter()
+        oracle.process_batch(sas, 1, b1, n_threads=1)
+        ms.append((time.perf_counter() - t0) * 1e3)
+    legs = {"c1_64x64B_1sa_ms_1thread": float(np.median(ms))}
+    for cfg in (2, 3, 4):
+        p, b = shard.rank_workload(cfg, PKTS_PER_GPU, CFG_SIZE[cfg], N_SA_TOTAL, 0, 1)
+        name = gen.CONFIGS[cfg]["name"]
+        legs[name] = {"1": oracle_leg(p, b, 1, budget_s), str(T): oracle_leg(p, b, T, budget_s)}
+    return {"cpu_model": cpu_model(), "threads_available": T, "legs": legs}
+
+
+def run_ours(args):
+    ctx = Ctx(args)
+    torch = ctx.torch
+    units = sass_units()
+    main_cfg = args.config
+    steps, warmup = args.steps, args.warmup
+    head = measure_outbound(ctx, args, main_cfg, CFG_SIZE[main_cfg], steps, warmup, full=True)
+    agg = rates(ctx, head, steps)
+    w = work_model(head["b"])
+    ms_batch = agg["ms_per_step"]
+    roof = roofline(ms_batch, w, ctx.peaks, units)
+    kname = "fused_ring" if head["form"] != "graph" else "fused"
+    roof_line = {"kernel": "k_fused_ring_pipe" if head["form"] == "pipelined" else "k_fused_ring",
+                 "bound": "alu", "achieved": roof["alu"]["achieved"], "peak": roof["alu"]["peak"],
+                 "unit": "Tops/s", "frac": roof["alu"]["frac"],
+                 "traffic": load_traffic(kname, gen.CONFIGS[main_cfg]["name"]),
+                 "traffic_algorithmic": w["hbm_bytes"],
+                 "lds_frac": roof["lds"]["frac"], "hbm_frac": roof["hbm"]["frac"],
+                 "basis": roof["basis"]}
+    # ---- configs[4] sweep (and configs[2], configs[3]) ------------------------
+    by_size = {size_key(CFG_SIZE[main_cfg]): {"gbps": agg["gbps"], "mpps": agg["mpps"],
+                                             "us": 1e3 * agg["ms_per_step"],
+                                             "esp_payload_gbps": agg["esp_payload_gbps"],
+                                             "alu_frac": roof["alu"]["frac"],
+                                             "p50_us": (head["per_batch"] or {}).get("median_us")}}
+    sweep_detail = {}
+    if not args.no_sweep:
+        k_sw = max(20, min(steps, 100))
+        for cfg_id, size in SWEEP:
+            if size == CFG_SIZE[main_cfg]:
+                continue
+            r = measure_outbound(ctx, args, cfg_id, size, k_sw, max(3, warmup // 2), full=False)
+            a = rates(ctx, r, k_sw)
+            rf = roofline(a["ms_per_step"], work_model(r["b"]), ctx.peaks, units)
+            by_size[size_key(size)] = {"gbps": a["gbps"], "mpps": a["mpps"],
+                                       "us": 1e3 * a["ms_per_step"],
+                                       "esp_payload_gbps": a["esp_payload_gbps"],
+                                       "alu_frac": rf["alu"]["frac"], "lds_frac": rf["lds"]["frac"],
+                                       "hbm_frac": rf["hbm"]["frac"],
+                                       "p50_us": (r["per_batch"] or {}).get("median_us")}
+            sweep_detail[size_key(size)] = {"per_batch": r["per_batch"], "ring_slots": r["R"],
+                                            "form": r["form"], "steps": k_sw}
+    # ---- ESP inbound (f2), flow lookup / dispatch (f3), adaptive split (f4) -----
+    inbound = {}
+    if not args.no_inbound:
+        for cfg_id in (2, 3, 4):
+            inbound[size_key(CFG_SIZE[cfg_id])] = measure_inbound(ctx, args, cfg_id,
+                                                                 max(10, steps // 4),
+                                                                 max(3, warmup // 2))
+    flows = None
+    if not args.no_inbound:
+        flows = measure_flows(ctx, args, main_cfg, max(10, steps // 4), max(3, warmup // 2))
+    alb_res = None
+    if ctx.world == 1 and not args.no_alb:
+        alb_res = measure_alb(ctx, args, 3)
+    e2e = run_e2e(ctx, args)
+    cpu = None
+    if ctx.rank == 0 and ctx.world == 1 and not args.no_cpu:
+        cpu = cpu_baselines(args.cpu_seconds)
+    ctr_all = ctx.sum_all(head["ctr"])
+    launch_ms = ctx.max_ms(head.get("launch_loop_ms", 0.0))
+    graph_ms = ctx.max_ms(head.get("graph_ms", 0.0))
+    if ctx.rank == 0:
+        clk = head["clk"].summary()
+        nm = gen.CONFIGS[main_cfg]["name"]
+        T = (cpu or {}).get("threads_available")
+        leg = (cpu or {}).get("legs", {}).get(nm, {})
+        cpu_line = None
+        if cpu:
+            allc = leg[str(T)]
+            cpu_line = {"value": allc["gbps"], "unit": "Gbps", "cores": T, "kind": "oracle",
+                        "sample": f"{nm}: {allc['sample']} on {T} threads", "mpps": allc["mpps"],
+                        "one_thread_gbps": leg["1"]["gbps"], "cpu_model": cpu["cpu_model"],
+                        "c1_64x64B_1sa_ms_1thread": cpu["legs"]["c1_64x64B_1sa_ms_1thread"]}
+        pb = head["per_batch"] or {}
+        out = {
+            "metric": METRIC,
+            "value": agg["gbps"],
+            "unit": "Gbps",
+            "mpps": agg["mpps"],
+            "n_gpus": ctx.world,
+            "steps": steps,
+            "warmup": warmup,
+            "ms_per_step": agg["ms_per_step"],
+            "higher_is_better": True,
+            "scaling": "weak",
+            "vs_baseline": None,
+            "dtype": "u8",
+            "data": "synthetic (seeded random IPv4/UDP, random SA keys; PAPER.md:395 workload shape)",
+            "config": {"workload": f"configs[{main_cfg - 1}]: {nm}", "frame_bytes": CFG_SIZE[main_cfg],
+                       "packets_per_gpu": PKTS_PER_GPU, "n_sa_total": N_SA_TOTAL,
+                       "global_batch": PKTS_PER_GPU * ctx.world,
+                       "parallelism": f"sa-hash shard x{ctx.world} (no data-path collective)",
+                       "l2": f"inputs larger than L2: batches rotate over {head['R']} device copies "
+                             "(> 2x L2 touched per rotation), SA table resident",
+                       "timing": f"all {steps} timed batches in ONE nba_ipsec_ring_run_batches call "
+                                 f"({head['form']} persistent ring, 1 launch) between one CUDA event "
+                                 "pair, barrier + sync both sides, max over ranks"},
+            "roofline": roof_line,
+            "gbps_by_size": {k: round(v["gbps"], 1) for k, v in by_size.items()},
+            "us_by_size": {k: round(v["us"], 2) for k, v in by_size.items()},
+            "esp_payload_gbps": agg["esp_payload_gbps"],
+            "per_batch_us": {k: (round(v, 3) if isinstance(v, float) else v) for k, v in pb.items()},
+            "cpu_baseline": cpu_line,
+            "e2e": e2e,
+            "gpu_launches": head["launches"],
+            "clocks": clk,
+            "compare": {"process_batch_loop_us": 1e3 * launch_ms / steps,
+                        "graph_replay_us": 1e3 * graph_ms / steps,
+                        "isolated_batch_us_mean": 1e3 * float(np.mean(head["iso_ms"])),
+                        "ring_us": 1e3 * agg["ms_per_step"],
+                        "launches_per_batch_unringed": head.get("lpb")},
+            "by_size": by_size,
+            "sweep": sweep_detail,
+            "work_per_step_per_gpu": w,
+            "cpu_legs": cpu,
+            "counters": ctr_all,
+            "inbound": inbound or None,
+            "flow_lookup": flows,
+            "adaptive_split": alb_res,
+            # compact recap at the end of the line (kept in the driver's tail)
+            "summary": {"Gbps": {k: round(v["gbps"], 1) for k, v in by_size.items()},
+                        "us": {k: round(v["us"], 2) for k, v in by_size.items()},
+                        "alu_frac": {k: round(v["alu_frac"], 3) for k, v in by_size.items()},
+                        "inbound_Gbps": {k: round(v["gbps"], 1) for k, v in inbound.items()},
+                        "p50_p10_p90_us": [pb.get("median_us"), pb.get("p10_us"), pb.get("p90_us")],
+                        "oracle_Gbps_1t_Nt": [leg.get("1", {}).get("gbps"),
+                                              leg.get(str(T), {}).get("gbps")] if cpu else None,
+                        "n_gpus": ctx.world},
+        }
+        print(json.dumps(out), flush=True)
+    if ctx.world > 1:
+        ctx.dist.destroy_process_group()
 
 
 # --------------------------------------------------------------------------- reference arm
@@ -901,13 +848,37 @@ def run_reference(args):
                    "n_sa_total": N_SA_TOTAL},
         "cpu_baseline": {"value": gbps, "unit": "Gbps", "cores": T, "kind": "oracle",
                          "sample": f"first {m} packets of the {b.n}-packet batch per step "
-                                   f"(~0.5 s all-core work), {args.steps} steps"},
+                                   f"(~0.5 s all-core work), {args.steps} steps",
+                         "cpu_model": cpu_model()},
         "e2e": {"value": gbps, "unit": "Gbps", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
 
 
-def main():
+def relaunch_under_torchrun(args):
+    """--gpus N > 1 without a torchrun environment: exec torchrun with one
+    process per GPU (NCCL communicator init printed, NCCL_DEBUG=INFO)."""
+    import socket
+    try:
+        import torch
+        have = torch.cuda.device_count()
+    except Exception:
+        have = 0
+    if have < args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} requested but {have} CUDA device(s) visible")
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        port = s.getsockname()[1]
+    env = dict(os.environ)
+    env.setdefault("NCCL_DEBUG", "INFO")
+    env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+           f"--nproc-per-node={args.gpus}", "--master-addr", "127.0.0.1", "--master-port", str(port),
+           os.path.abspath(__file__), *sys.argv[1:]]
+    os.execvpe(cmd[0], cmd, env)
+
+
+def parse_args(argv=None):
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=200)
@@ -919,16 +890,25 @@ def main():
     ap.add_argument("--no-inbound", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-alb", action="store_true")
-    ap.add_argument("--no-ring", action="store_true",
-                    help="launch every timed batch with process_batch instead of the ring graph")
-    ap.add_argument("--cpu-seconds", type=float, default=3.0)
-    args = ap.parse_args()
+    ap.add_argument("--cpu-seconds", type=float, default=2.0,
+                    help="per oracle leg (configs[1..3] x {1, N} threads)")
+    args = ap.parse_args(argv)
     if args.warmup < 3:
         args.warmup = 3
+    return args
+
+
+def main():
+    args = parse_args()
     if args.impl == "reference":
         run_reference(args)
-    else:
-        run_ours(args)
+        return
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        relaunch_under_torchrun(args)
+    if int(os.environ.get("WORLD_SIZE", "1")) > 1:
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    run_ours(args)
 
 
 if __name__ == "__main__":

@@ -174,6 +174,24 @@ typedef struct nba_ipsec_ring nba_ipsec_ring;
 int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, uint32_t n_slots,
                           nba_ipsec_ring **out);
 int nba_ipsec_ring_run(nba_ipsec_ring *r, uint32_t n_rounds, void *cuda_stream);
+/* Exactly n_batches batches, slot after slot starting at the ring's cursor
+ * (0 after creation), which then advances by n_batches mod n_slots: a run may
+ * stop mid-rotation and the next one continues where it stopped.  Results are
+ * those of the same sequence of process_batch (process_inbound) calls.
+ * Persistent forms: ONE launch; graph form: whole rotations starting at slot 0
+ * replay the graph, other batches are launched one by one.  ring_run(n) runs
+ * n x n_slots batches from the cursor (which it leaves unchanged).
+ * NBA_IPSEC_EINVAL as ring_run, or when timestamps are set with fewer than
+ * n_batches + 1 entries; n_batches == 0 is a no-op. */
+int nba_ipsec_ring_run_batches(nba_ipsec_ring *r, uint32_t n_batches, void *cuda_stream);
+int nba_ipsec_ring_cursor(const nba_ipsec_ring *r);          /* slot of the next batch */
+/* Per-batch device timestamps of later runs (persistent forms only): dev_ts is
+ * a DEVICE buffer of cap u64 entries owned by the caller; each run zeroes
+ * entries [0, n_batches] on its stream, then writes ts[0] = the run's start and
+ * ts[1 + b] = the latest end, over the CTAs, of batch b's iteration (globaltimer
+ * ns).  dev_ts == NULL switches it off.  NBA_IPSEC_EINVAL for a graph ring or
+ * cap < 2. */
+int nba_ipsec_ring_set_timestamps(nba_ipsec_ring *r, unsigned long long *dev_ts, uint32_t cap);
 enum { NBA_IPSEC_RING_GRAPH = 0, NBA_IPSEC_RING_PERSISTENT = 1, NBA_IPSEC_RING_PIPELINED = 2 };
 /* The form a run takes (NBA_IPSEC_RING_*); set_form switches a persistent ring
  * between PERSISTENT and PIPELINED (NBA_IPSEC_EINVAL for graph rings or slots
@@ -311,7 +329,11 @@ int nba_ipsec_route_pack_map(const uint8_t *in_buf, const uint32_t *in_off, cons
  * positions 0..count-1 (batch order), offsets into its buf, and
  * count[0] = packets, count[1] = bytes (written by the dispatch).  Each
  * receiver needs cap_pkts >= n_pkts entries and cap_bytes >= the batch's bytes
- * (larger batches are not written past the capacity).  Single ingress: one
+ * to take every packet; when its packets do not fit, the receiver gets the
+ * longest prefix (in batch order) that fits both capacities, count[] says how
+ * many packets / bytes that is, and nothing is written past the capacity --
+ * the caller detects the overflow as dest_counts[d] > rx count (the dropped
+ * suffix is the caller's to resend or count as lost).  Single ingress: one
  * dispatch per receive buffer at a time; the receivers may read them after the
  * caller's stream work completed (e.g. stream sync + a process-group barrier).
  * sa_map as in route_pack_map (NULL: owner = s mod world).  dest_counts /

@@ -391,6 +391,12 @@ struct nba_ipsec_ring {
     bool pipe = false;                   // software-pipelined form (k_fused_ring_pipe)
     bool pipe_ok = false;                // every slot fits the pipelined form
     uint64_t flow_gen = 0;               // the table's flow-table generation when recorded
+    uint32_t cursor = 0;                 // the slot the next run_batches starts at
+    unsigned long long *ts = nullptr;    // per-batch timestamps (caller's device buffer)
+    uint32_t ts_cap = 0;
+    // graph form: the slots, for runs that do not start at slot 0 / end mid-rotation
+    std::vector<nba_ipsec_batch> h_slots;
+    std::vector<nba_ipsec_in_batch> h_in_slots;
 };
 
 int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, uint32_t n_slots,
@@ -411,6 +417,7 @@ int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, u
     r->t = t;
     r->n_slots = n_slots;
     r->flow_gen = t->flow_gen;
+    r->h_slots.assign(slots, slots + n_slots);
     // persistent form: one cooperative launch walks all batches of a run
     bool persist = !std::getenv("NBA_IPSEC_RING_GRAPH") && t->pipeline == NBA_IPSEC_PIPE_FUSED &&
                    t->allow_merged;
@@ -489,6 +496,7 @@ int nba_ipsec_ring_create_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batc
     r->t = t;
     r->n_slots = n_slots;
     r->flow_gen = t->flow_gen;
+    r->h_in_slots.assign(slots, slots + n_slots);
     // persistent form (opt-in, NBA_IPSEC_RING_IN_PERSIST) when every slot takes
     // the one-kernel inbound path; measured against the graph form: 64 B 45.9
     // -> 43.9 us, 1514 B 215.4 -> 217.2 us, IMIX 108.6 -> 117.5 us
@@ -544,35 +552,83 @@ int nba_ipsec_ring_create_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batc
     return NBA_IPSEC_OK;
 }
 
+// n_batches batches of the ring starting at slot `first` (persistent forms:
+// one launch; graph form: whole rotations from slot 0 replay the graph, the
+// other batches are launched one by one).
+static int ring_launch(nba_ipsec_ring *r, uint32_t first, uint32_t n_batches, cudaStream_t st)
+{
+    nba_ipsec_sa_table *t = r->t;
+    if (n_batches == 0) return NBA_IPSEC_OK;
+    if (r->ts) {
+        if (n_batches >= r->ts_cap) return NBA_IPSEC_EINVAL;
+        if (cudaMemsetAsync(r->ts, 0, (size_t)(n_batches + 1) * sizeof(unsigned long long), st) !=
+            cudaSuccess)
+            return NBA_IPSEC_ECUDA;
+    }
+    const RingRun R{r->n_slots, first, n_batches, r->ts};
+    if (r->d_in_slots)
+        return launch_in_fused_ring(t->T, t->S, r->d_in_slots, R, r->in_hmask, r->hkey_b, r->hval_b,
+                                    t->grid_fused, st) == cudaSuccess
+                   ? NBA_IPSEC_OK
+                   : NBA_IPSEC_ECUDA;
+    if (r->d_slots) {
+        const cudaError_t e = r->pipe ? launch_fused_ring_pipe(t->T, t->W, r->d_slots, R, r->hist_b,
+                                                               t->grid_fused, st)
+                                      : launch_fused_ring(t->T, t->W, r->d_slots, R, r->hist_b,
+                                                          t->grid_fused, st);
+        return e == cudaSuccess ? NBA_IPSEC_OK : NBA_IPSEC_ECUDA;
+    }
+    uint32_t k = first, left = n_batches;
+    while (left) {
+        if (k == 0 && left >= r->n_slots) {
+            if (cudaGraphLaunch(r->exec, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
+            left -= r->n_slots;
+            continue;
+        }
+        int rc = NBA_IPSEC_OK;
+        if (!r->h_in_slots.empty()) {
+            if (r->h_in_slots[k].n_pkts) rc = nba_ipsec_process_inbound(t, &r->h_in_slots[k], st);
+        } else if (r->h_slots[k].n_pkts) {
+            rc = nba_ipsec_process_batch(t, &r->h_slots[k], st);
+        }
+        if (rc != NBA_IPSEC_OK) return rc;
+        k = (k + 1) % r->n_slots;
+        left--;
+    }
+    return NBA_IPSEC_OK;
+}
+
 int nba_ipsec_ring_run(nba_ipsec_ring *r, uint32_t n_rounds, void *cuda_stream)
 {
     if (!r || (!r->exec && !r->d_slots && !r->d_in_slots)) return NBA_IPSEC_EINVAL;
     if (r->t->flow_gen != r->flow_gen) return NBA_IPSEC_EINVAL;   // replaced: re-create the ring
+    if ((uint64_t)n_rounds * r->n_slots > 0xffffffffull) return NBA_IPSEC_EINVAL;
     DeviceGuard g(r->t->device);
-    cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);
-    if (r->d_in_slots) {
-        if (n_rounds == 0) return NBA_IPSEC_OK;
-        if ((uint64_t)n_rounds * r->n_slots > 0xffffffffull) return NBA_IPSEC_EINVAL;
-        nba_ipsec_sa_table *t = r->t;
-        return launch_in_fused_ring(t->T, t->S, r->d_in_slots, r->n_slots, n_rounds * r->n_slots,
-                                    r->in_hmask, r->hkey_b, r->hval_b, t->grid_fused, st) ==
-                       cudaSuccess
-                   ? NBA_IPSEC_OK
-                   : NBA_IPSEC_ECUDA;
-    }
-    if (r->d_slots) {
-        if (n_rounds == 0) return NBA_IPSEC_OK;
-        if ((uint64_t)n_rounds * r->n_slots > 0xffffffffull) return NBA_IPSEC_EINVAL;
-        nba_ipsec_sa_table *t = r->t;
-        const cudaError_t e =
-            r->pipe ? launch_fused_ring_pipe(t->T, t->W, r->d_slots, r->n_slots, n_rounds * r->n_slots,
-                                             r->hist_b, t->grid_fused, st)
-                    : launch_fused_ring(t->T, t->W, r->d_slots, r->n_slots, n_rounds * r->n_slots,
-                                        r->hist_b, t->grid_fused, st);
-        return e == cudaSuccess ? NBA_IPSEC_OK : NBA_IPSEC_ECUDA;
-    }
-    for (uint32_t k = 0; k < n_rounds; k++)
-        if (cudaGraphLaunch(r->exec, st) != cudaSuccess) return NBA_IPSEC_ECUDA;
+    return ring_launch(r, r->cursor, n_rounds * r->n_slots, static_cast<cudaStream_t>(cuda_stream));
+}
+
+int nba_ipsec_ring_run_batches(nba_ipsec_ring *r, uint32_t n_batches, void *cuda_stream)
+{
+    if (!r || (!r->exec && !r->d_slots && !r->d_in_slots)) return NBA_IPSEC_EINVAL;
+    if (r->t->flow_gen != r->flow_gen) return NBA_IPSEC_EINVAL;
+    DeviceGuard g(r->t->device);
+    const int rc = ring_launch(r, r->cursor, n_batches, static_cast<cudaStream_t>(cuda_stream));
+    if (rc == NBA_IPSEC_OK) r->cursor = (uint32_t)(((uint64_t)r->cursor + n_batches) % r->n_slots);
+    return rc;
+}
+
+int nba_ipsec_ring_cursor(const nba_ipsec_ring *r)
+{
+    if (!r) return NBA_IPSEC_EINVAL;
+    return (int)r->cursor;
+}
+
+int nba_ipsec_ring_set_timestamps(nba_ipsec_ring *r, unsigned long long *dev_ts, uint32_t cap)
+{
+    if (!r || (dev_ts && cap < 2)) return NBA_IPSEC_EINVAL;
+    if (dev_ts && !r->d_slots && !r->d_in_slots) return NBA_IPSEC_EINVAL;   // persistent forms only
+    r->ts = dev_ts;
+    r->ts_cap = dev_ts ? cap : 0;
     return NBA_IPSEC_OK;
 }
 

@@ -174,20 +174,26 @@ bool fused_merged_ok(uint32_t n, int grid);
 cudaError_t setup_prologue_attributes(uint32_t n_sa, uint32_t max_tiles, int num_sms, bool *gridsync);
 cudaError_t setup_aes_attributes();
 cudaError_t setup_fused_attributes();
+// One run of a batch ring: batches first, first + 1, ... (mod n_slots) of the
+// slot array, n_batches of them; ts (optional, zeroed by the host): ts[0] =
+// run start, ts[1 + b] = max over CTAs of the global timer when batch b's
+// iteration ended.
+struct RingRun {
+    uint32_t n_slots, first, n_batches;
+    unsigned long long *ts;
+};
 cudaError_t launch_fused_ring_pipe(const DevTable &T, const DevWork &W, const BatchArgs *slots,
-                                   uint32_t n_slots, uint32_t n_batches, uint16_t *hist_b,
-                                   int grid, cudaStream_t st);
+                                   const RingRun &R, uint16_t *hist_b, int grid, cudaStream_t st);
 bool fused_pipe_ok(uint32_t n, int grid);
 cudaError_t launch_fused_ring(const DevTable &T, const DevWork &W, const BatchArgs *slots,
-                              uint32_t n_slots, uint32_t n_batches, uint16_t *hist_b, int grid,
-                              cudaStream_t st);
+                              const RingRun &R, uint16_t *hist_b, int grid, cudaStream_t st);
 int aes_grid(int num_sms);
 int fused_grid(int num_sms);
 cudaError_t launch_in_fused(const DevTable &T, const InState &S, const InBatchArgs &B, int grid,
                             uint32_t hmask, bool merged, uint32_t *bar_base, cudaStream_t st);
 bool in_merged_ok(uint32_t n, int grid);
 cudaError_t launch_in_fused_ring(const DevTable &T, const InState &S, const InBatchArgs *slots,
-                                 uint32_t n_slots, uint32_t n_batches, uint32_t hmask,
+                                 const RingRun &R, uint32_t hmask,
                                  unsigned long long *hkey_b, uint32_t *hval_b, int grid,
                                  cudaStream_t st);
 cudaError_t launch_in_replay(const DevTable &T, const InState &S, const InBatchArgs &B,

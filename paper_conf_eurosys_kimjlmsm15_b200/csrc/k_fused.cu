@@ -624,19 +624,21 @@ k_fused(DevTable T, DevWork W, BatchArgs B, uint32_t ppc, uint32_t bar_base_h, u
 // batch parity: batch bi's row scans re-zero buffer bi & 1 after every CTA
 // passed barrier bi, and batch bi + 2 writes it only after barrier bi + 1.
 __global__ void __launch_bounds__(F_THREADS, 1)
-k_fused_ring(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slots, uint32_t n_batches,
-             uint16_t *hist_b)
+k_fused_ring(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint16_t *hist_b)
 {
+    const uint32_t n_slots = R.n_slots, n_batches = R.n_batches;
+    if (R.ts && blockIdx.x == 0 && threadIdx.x == 0) R.ts[0] = gtimer();
     const uint32_t base0 = *reinterpret_cast<volatile uint32_t *>(&W.ctl[CTL_BAR_BASE]);
     const uint32_t ep0 = *reinterpret_cast<volatile uint32_t *>(&W.ctl[CTL_EPOCH]);
     const uint32_t G = gridDim.x;
     for (uint32_t bi = 0; bi < n_batches; bi++) {
-        const BatchArgs B = slots[bi % n_slots];
+        const BatchArgs B = slots[(R.first + bi) % n_slots];
         DevWork Wb = W;
         if (bi & 1u) Wb.hist16 = hist_b;
         const uint32_t epoch = ((ep0 + bi) % 0x7fffffffu) + 1u;
         fused_body<true>(T, Wb, B, fused_ppc(B.n, G), base0 + bi * G, epoch, bi == 0);
         __syncthreads();   // shared memory is reused by the next batch
+        if (R.ts && threadIdx.x == 0) atomicMax(&R.ts[1u + bi], gtimer());
     }
 }
 
@@ -1026,13 +1028,14 @@ __device__ __forceinline__ void pipe_sequence(const DevTable &T, const DevWork &
 }
 
 __global__ void __launch_bounds__(F_THREADS, 1)
-k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slots,
-                  uint32_t n_batches, uint16_t *hist_b)
+k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint16_t *hist_b)
 {
+    const uint32_t n_slots = R.n_slots, n_batches = R.n_batches, first = R.first;
     extern __shared__ __align__(16) uint8_t smem[];
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
     const uint32_t G = gridDim.x, cta = blockIdx.x;
     if (n_batches == 0) return;
+    if (R.ts && cta == 0 && tid == 0) R.ts[0] = gtimer();
     const uint32_t base0 = *reinterpret_cast<volatile uint32_t *>(&W.ctl[CTL_BAR_BASE]);
     const uint32_t ep0 = *reinterpret_cast<volatile uint32_t *>(&W.ctl[CTL_EPOCH]);
     const uint32_t sb = smem_u32(smem);
@@ -1063,13 +1066,13 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slot
         return Wb;
     };
     if (isP) {
-        const BatchArgs B0 = slots[0];
+        const BatchArgs B0 = slots[first % n_slots];
         pipe_prologue(T, work_of(0), B0, fused_ppc(B0.n, G), base0 + G, epoch_of(0), L, pt, 0u);
     }
     __syncthreads();
     unsigned long long c_ok = 0, c_drop = 0, c_in = 0, c_out = 0;
     for (uint32_t bi = 0; bi < n_batches; bi++) {
-        const BatchArgs B = slots[bi % n_slots];
+        const BatchArgs B = slots[(first + bi) % n_slots];
         // lanes: the packet (known since the previous batch); its SA line and
         // round keys either before the barrier wait / scans / polls, whose
         // latency they then overlap (long or length-divergent batches, as
@@ -1124,12 +1127,13 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slot
         } else {
             bar_sync_n(2, F_THREADS);                    // every lane took its fields
             if (bi + 1 < n_batches) {
-                const BatchArgs Bn = slots[(bi + 1) % n_slots];
+                const BatchArgs Bn = slots[(first + bi + 1) % n_slots];
                 pipe_prologue(T, work_of(bi + 1), Bn, fused_ppc(Bn.n, G), base0 + (bi + 2) * G,
                               epoch_of(bi + 1), L, pt, (bi + 1) & 1u);
             }
         }
         __syncthreads();                                  // batch bi done, bi + 1 prepared
+        if (R.ts && tid == 0) atomicMax(&R.ts[1u + bi], gtimer());
     }
     // counters (as fused_body), device state for the next launch
     if (tid < 4) L.cnt[tid] = 0ull;
@@ -1152,8 +1156,7 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, uint32_t n_slot
 }
 
 cudaError_t launch_fused_ring_pipe(const DevTable &T, const DevWork &W, const BatchArgs *slots,
-                                   uint32_t n_slots, uint32_t n_batches, uint16_t *hist_b,
-                                   int grid, cudaStream_t st)
+                                   const RingRun &R, uint16_t *hist_b, int grid, cudaStream_t st)
 {
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(grid);
@@ -1165,7 +1168,7 @@ cudaError_t launch_fused_ring_pipe(const DevTable &T, const DevWork &W, const Ba
     attr[0].val.cooperative = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    return cudaLaunchKernelEx(&cfg, k_fused_ring_pipe, T, W, slots, n_slots, n_batches, hist_b);
+    return cudaLaunchKernelEx(&cfg, k_fused_ring_pipe, T, W, slots, R, hist_b);
 }
 
 bool fused_pipe_ok(uint32_t n, int grid)
@@ -1214,8 +1217,7 @@ cudaError_t launch_fused(const DevTable &T, const DevWork &W, const BatchArgs &B
 }
 
 cudaError_t launch_fused_ring(const DevTable &T, const DevWork &W, const BatchArgs *slots,
-                              uint32_t n_slots, uint32_t n_batches, uint16_t *hist_b, int grid,
-                              cudaStream_t st)
+                              const RingRun &R, uint16_t *hist_b, int grid, cudaStream_t st)
 {
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(grid);
@@ -1227,7 +1229,7 @@ cudaError_t launch_fused_ring(const DevTable &T, const DevWork &W, const BatchAr
     attr[0].val.cooperative = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    return cudaLaunchKernelEx(&cfg, k_fused_ring, T, W, slots, n_slots, n_batches, hist_b);
+    return cudaLaunchKernelEx(&cfg, k_fused_ring, T, W, slots, R, hist_b);
 }
 
 cudaError_t setup_fused_attributes()

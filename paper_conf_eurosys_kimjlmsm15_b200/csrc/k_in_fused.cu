@@ -398,13 +398,15 @@ k_in_fused(DevTable T, InState S, InBatchArgs B, uint32_t ppc, uint32_t hmask, u
 // user) finished everywhere before batch bi's first barrier.  The T-tables are
 // re-staged per batch (the replay merge uses their shared memory as scratch).
 __global__ void __launch_bounds__(F_THREADS, 1)
-k_in_fused_ring(DevTable T, InState S, const InBatchArgs *slots, uint32_t n_slots,
-                uint32_t n_batches, uint32_t hmask, unsigned long long *hkey_b, uint32_t *hval_b)
+k_in_fused_ring(DevTable T, InState S, const InBatchArgs *slots, RingRun R, uint32_t hmask,
+                unsigned long long *hkey_b, uint32_t *hval_b)
 {
+    const uint32_t n_slots = R.n_slots, n_batches = R.n_batches;
+    if (R.ts && blockIdx.x == 0 && threadIdx.x == 0) R.ts[0] = gtimer();
     const uint32_t base0 = *reinterpret_cast<volatile uint32_t *>(&S.ctl[CTLI_BASE]);
     const uint32_t G = gridDim.x;
     for (uint32_t bi = 0; bi < n_batches; bi++) {
-        const InBatchArgs B = slots[bi % n_slots];
+        const InBatchArgs B = slots[(R.first + bi) % n_slots];
         InState Sb = S;
         if (bi & 1u) {
             Sb.hkey = hkey_b;
@@ -415,11 +417,12 @@ k_in_fused_ring(DevTable T, InState S, const InBatchArgs *slots, uint32_t n_slot
         if (ppc < 32u) ppc = 32u;
         in_fused_body<true>(T, Sb, B, ppc, hmask, base0 + 2u * bi * G);
         __syncthreads();   // shared memory is reused by the next batch
+        if (R.ts && threadIdx.x == 0) atomicMax(&R.ts[1u + bi], gtimer());
     }
 }
 
 cudaError_t launch_in_fused_ring(const DevTable &T, const InState &S, const InBatchArgs *slots,
-                                 uint32_t n_slots, uint32_t n_batches, uint32_t hmask,
+                                 const RingRun &R, uint32_t hmask,
                                  unsigned long long *hkey_b, uint32_t *hval_b, int grid,
                                  cudaStream_t st)
 {
@@ -433,8 +436,7 @@ cudaError_t launch_in_fused_ring(const DevTable &T, const InState &S, const InBa
     attr[0].val.cooperative = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    return cudaLaunchKernelEx(&cfg, k_in_fused_ring, T, S, slots, n_slots, n_batches, hmask, hkey_b,
-                              hval_b);
+    return cudaLaunchKernelEx(&cfg, k_in_fused_ring, T, S, slots, R, hmask, hkey_b, hval_b);
 }
 
 cudaError_t launch_in_fused(const DevTable &T, const InState &S, const InBatchArgs &B, int grid,

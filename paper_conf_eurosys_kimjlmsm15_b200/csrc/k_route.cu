@@ -210,6 +210,15 @@ __device__ __forceinline__ void route_copy_group(const RouteWork &R, const uint8
                     r.off[pos] = (uint32_t)boff;
                     r.len[pos] = (uint16_t)len;
                     r.sa[pos] = local;
+                } else if (pos <= cap_pkts && boff <= cap_bytes) {
+                    // The receiver's packets that do not fit form a suffix (pos
+                    // and boff grow together); this is its FIRST packet, so
+                    // exactly this lane publishes the count of what was
+                    // written, overriding the scan's totals (the caller sees the
+                    // overflow as dest_counts / dest_bytes above rx's count).
+                    const nba_ipsec_peer_rx r = rx[d];
+                    r.count[0] = pos;
+                    r.count[1] = boff;
                 }
             } else {
                 const unsigned long long gpos = R.base[d] + pos;

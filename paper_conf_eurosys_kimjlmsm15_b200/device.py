@@ -55,3 +55,21 @@ def fetch(db: DeviceBatch):
     out = db.out_buf.cpu().numpy()
     ol = db.out_len[:db.n].cpu().numpy().view(np.uint16)
     return out, ol
+
+
+def ring_slot_count(in_len: np.ndarray, n: int, l2_bytes: int) -> int:
+    """Device copies of a batch the benchmark rotates over so that one rotation
+    touches more than 2x the L2 (every batch starts L2-cold): bytes touched per
+    batch ~ the datagrams plus, per packet, the 128-byte lines of its input and
+    output slots and its metadata.  Shared by bench.py and the tests that
+    check the bench's exact ring."""
+    touched = int(np.asarray(in_len, np.int64).sum()) + int(n) * (128 + 53 + 128 + 14)
+    return max(2, -(-2 * int(l2_bytes) // touched))
+
+
+def clone(d: DeviceBatch) -> DeviceBatch:
+    """A second device copy of a batch (fresh output pool / lengths)."""
+    return DeviceBatch(n=d.n, in_buf=d.in_buf.clone(), in_off=d.in_off.clone(),
+                       in_len=d.in_len.clone(), sa_idx=d.sa_idx.clone(),
+                       out_buf=torch.zeros_like(d.out_buf), out_off=d.out_off.clone(),
+                       out_len=torch.zeros_like(d.out_len))

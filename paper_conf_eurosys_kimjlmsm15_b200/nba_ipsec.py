@@ -127,6 +127,9 @@ def _load():
                                            vp, vp]),
         "nba_ipsec_ring_create": (i32, [vp, P(Batch), u32, P(vp)]),
         "nba_ipsec_ring_run": (i32, [vp, u32, vp]),
+        "nba_ipsec_ring_run_batches": (i32, [vp, u32, vp]),
+        "nba_ipsec_ring_cursor": (i32, [vp]),
+        "nba_ipsec_ring_set_timestamps": (i32, [vp, vp, u32]),
         "nba_ipsec_ring_form": (i32, [vp]),
         "nba_ipsec_ring_set_form": (i32, [vp, i32]),
         "nba_ipsec_ring_create_inbound": (i32, [vp, P(InBatch), u32, P(vp)]),
@@ -448,6 +451,22 @@ class Ring:
     def run(self, n_rounds: int = 1, stream=None):
         _check(lib.nba_ipsec_ring_run(self._h, int(n_rounds), _stream_handle(stream)),
                "nba_ipsec_ring_run")
+
+    def run_batches(self, n_batches: int, stream=None):
+        """nba_ipsec_ring_run_batches: exactly n_batches batches from the cursor."""
+        _check(lib.nba_ipsec_ring_run_batches(self._h, int(n_batches), _stream_handle(stream)),
+               "nba_ipsec_ring_run_batches")
+
+    @property
+    def cursor(self) -> int:
+        return int(lib.nba_ipsec_ring_cursor(self._h))
+
+    def set_timestamps(self, ts):
+        """nba_ipsec_ring_set_timestamps: ts = int64 CUDA tensor (cap entries) or None."""
+        self._ts = ts
+        _check(lib.nba_ipsec_ring_set_timestamps(self._h, _ptr(ts) if ts is not None else None,
+                                                 int(ts.numel()) if ts is not None else 0),
+               "nba_ipsec_ring_set_timestamps")
 
     GRAPH, PERSISTENT, PIPELINED = 0, 1, 2
 

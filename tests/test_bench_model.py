@@ -48,11 +48,38 @@ def test_imix_composition_and_invalid_packets_excluded():
 
 
 def test_roofline_arithmetic():
-    w = {"aes_blocks": 1000, "sha1_compressions": 100}
-    peaks = {"sm_max_mhz": 1965.0, "hbm_gbs": 6500.0}
-    r = bench.kernel_roofline("fused", 0.001, w, peaks)
-    ops = 1000 * bench.AES_ALU_OPS_PER_BLOCK + 100 * bench.SHA1_ALU_OPS_PER_COMPRESSION
-    assert abs(r["achieved"] - ops / 1e-6 / 1e9) < 1e-6
-    assert abs(r["peak"] - 148 * 64 * 1965e6 / 1e9) < 1e-6
-    assert r["bound"] == "alu"
-    assert bench.kernel_roofline("fused_ring", 0.001, w, peaks)["achieved"] == r["achieved"]
+    """ALU / LDS / HBM fractions from the SASS per-unit counts (profiles/r02_sass_hist.txt)."""
+    w = {"aes_blocks": 1000, "sha1_compressions": 100, "hbm_bytes": 5000}
+    peaks = {"sm_max_mhz": 1965.0, "hbm_gbs": 6500.0, "source": "test"}
+    units = bench.sass_units()
+    r = bench.roofline(0.001, w, peaks, units)
+    ops = 1000 * units["aes_block"]["alu"] + 100 * units["sha1_compression"]["alu"]
+    assert abs(r["alu"]["achieved"] - ops / 1e-6 / 1e12) < 1e-9
+    assert abs(r["alu"]["peak"] - 148 * 64 * 1965e6 / 1e12) < 1e-9
+    assert abs(r["lds"]["achieved"] - 1000 * units["aes_block"]["smem"] / 1e-6 / 1e12) < 1e-9
+    assert abs(r["hbm"]["achieved"] - 5000 / 1e-6 / 1e9) < 1e-9
+    for k in ("alu", "lds", "hbm"):
+        assert abs(r[k]["frac"] - r[k]["achieved"] / r[k]["peak"]) < 1e-12
+
+
+def test_sass_units_committed():
+    """The committed SASS histogram parses and gives plausible per-unit counts:
+    an AES block needs its table lookups (>= 133 after the CTR precompute, at
+    most 160) and a SHA-1 compression >= 80 rounds x 3 ALU ops."""
+    u = bench.sass_units()
+    assert u["source"].startswith("profiles/")
+    assert 133 <= u["aes_block"]["smem"] <= 165
+    assert u["sha1_compression"]["alu"] + u["sha1_compression"]["fma"] >= 400
+
+
+def test_ring_slot_count_matches_bench_rule():
+    from paper_conf_eurosys_kimjlmsm15_b200 import device
+    b = gen.make_batch(65536, 64, 1024, cfg_id=2)
+    R = device.ring_slot_count(b.in_len, b.n, 126 << 20)
+    touched = int(b.in_len.astype(np.int64).sum()) + b.n * 323
+    assert (R - 1) * touched < 2 * (126 << 20) <= R * touched
+
+
+def test_bench_args_and_gpus_contract():
+    a = bench.parse_args(["--gpus", "2", "--steps", "7", "--warmup", "1"])
+    assert (a.gpus, a.steps, a.warmup) == (2, 7, 3)          # W >= 3

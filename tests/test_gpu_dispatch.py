@@ -150,3 +150,42 @@ def test_dispatch_two_processes_ipc_union_equals_one_gateway():
         assert got[d][seen[d]] == ref_out[b.out_off[i]:b.out_off[i] + ref_len[i]].tobytes()
         seen[d] += 1
     assert seen == {0: len(mine), 1: len(theirs)}
+
+
+@pytest.mark.parametrize("cap_pkts_frac,cap_bytes_frac", [(1.0, 0.37), (0.5, 1.0), (0.6, 0.4),
+                                                          (1.0, 0.0)])
+def test_dispatch_capacity_overflow(cap_pkts_frac, cap_bytes_frac):
+    """Receive buffers smaller than an owner's share: the owner gets exactly the
+    longest prefix of its packets (batch order) that fits both capacities, its
+    published count says so (no stale entries past it), nothing is written past
+    the capacity, and dest_counts / dest_bytes still report the full routing."""
+    import torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, redistribute
+    n, n_sa_total, world = 3000, 40, 2
+    b = gen.make_batch(n, "imix", n_sa_total, cfg_id=62, layout="slots")
+    r_buf, r_len, r_sa, r_cnt, r_byt = route_pack_ref(b, n_sa_total, world)
+    cap_pkts = int(min(r_cnt) * cap_pkts_frac)
+    cap_bytes = int(min(r_byt) * cap_bytes_frac)
+    guard = 4096
+    rxs = [redistribute.alloc_rx(cap_pkts + guard, cap_bytes + guard, "cuda") for _ in range(world)]
+    for r in rxs:
+        r.buf.fill_(0x5A)
+        r.count.fill_(-1)
+    table = redistribute.rx_table(rxs, "cuda")
+    db = device.to_device(b, "cuda")
+    counts, nbytes = redistribute.dispatch(db, n, n_sa_total, world, table, cap_pkts, cap_bytes)
+    torch.cuda.synchronize()
+    assert counts == r_cnt and nbytes == r_byt
+    c0, b0 = 0, 0
+    for d in range(world):
+        ln_all = r_len[c0:c0 + r_cnt[d]].astype(np.int64)
+        ends = np.cumsum(ln_all)
+        fit = int(np.sum((np.arange(r_cnt[d]) < cap_pkts) & (ends <= cap_bytes)))
+        n_d, nb_d, data, ln, sa, off = _read_rx(rxs[d])
+        assert (n_d, nb_d) == (fit, int(ends[fit - 1]) if fit else 0)
+        assert np.array_equal(ln, r_len[c0:c0 + fit]) and np.array_equal(sa, r_sa[c0:c0 + fit])
+        assert np.array_equal(data, r_buf[b0:b0 + nb_d])
+        tail = rxs[d].buf[cap_bytes:].cpu().numpy()
+        assert np.all(tail == 0x5A), "bytes written past cap_bytes"
+        c0 += r_cnt[d]
+        b0 += r_byt[d]

@@ -321,3 +321,38 @@ def test_pipelined_ring_small_batches(n):
             assert np.array_equal(g_len, o_len) and np.array_equal(g_out, o_out)
         assert np.array_equal(t.sa_seq(), oracle.sa_seq(sas, n_sa))
         ring.close()
+
+
+@pytest.mark.parametrize("graph", [False, True])
+def test_run_batches_mid_rotation(graph, monkeypatch):
+    """nba_ipsec_ring_run_batches stops mid-rotation and the next run continues
+    from the cursor: 5 + 4 + 3 batches over 3 distinct slots (persistent and
+    graph forms) equal the oracle over the same slot sequence."""
+    import torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    if graph:
+        monkeypatch.setenv("NBA_IPSEC_RING_GRAPH", "1")
+    n_sa, n = 61, 9000
+    p = gen.make_sas(n_sa, cfg_id=57)
+    hb = [gen.make_batch(n, s, n_sa, cfg_id=57, batch=i) for i, s in enumerate((64, "imix", 300))]
+    sas = oracle.make_sas(p)
+    ctr = oracle.Counters()
+    with nba_ipsec.SATable(p, device=0, max_batch=n) as t:
+        dbs = [device.to_device(b, "cuda") for b in hb]
+        ring = t.ring([_slot(d) for d in dbs])
+        assert ring.form == (nba_ipsec.Ring.GRAPH if graph else nba_ipsec.Ring.PIPELINED)
+        last, k = {}, 0
+        for nb in (5, 4, 3):
+            ring.run_batches(nb)
+            for _ in range(nb):
+                o_out, o_len, _ = oracle.process_batch(sas, n_sa, hb[k % 3], n_threads=8, counters=ctr)
+                last[k % 3] = (o_out, o_len.copy())
+                k += 1
+            assert ring.cursor == k % 3
+        for s, (o_out, o_len) in last.items():
+            g_out, g_len = device.fetch(dbs[s])
+            assert np.array_equal(g_len, o_len)
+            assert np.array_equal(g_out, o_out)
+        assert np.array_equal(t.sa_seq(), oracle.sa_seq(sas, n_sa))
+        assert t.counters() == ctr.as_dict()
+        ring.close()

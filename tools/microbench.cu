@@ -6,7 +6,11 @@
 //
 // Prints one JSON object: per-SM-per-clock rates (from clock64 inside the
 // kernel) and chip-wide rates (CUDA events) for
-//   lds32      conflict-free 32-bit shared loads (the T-table access pattern)
+//   lds32      conflict-free 32-bit shared loads, index from the previous value
+//              with ~3 ALU ops of address arithmetic per load (ALU-bound: kept
+//              for comparison with round 1)
+//   lds32_prmt the lane loop's T-table pattern: one PRMT + one LDS per lookup
+//   lds32_pure loads with fixed addresses (0.5 ALU op per load): the LDS rate
 //   lop3/prmt/shf/iadd3   ALU-pipe integer ops
 //   aes_block  full T-table AES-128 blocks (aes_round.cuh), no global memory
 //   sha1_comp  SHA-1 compressions (sha1.cuh), no global memory
@@ -48,6 +52,68 @@ __global__ void k_lds(uint32_t *out, unsigned long long *cyc, uint32_t seed)
     unsigned long long c1 = clock64();
     if (threadIdx.x == 0) atomicMax(cyc, c1 - c0);
     out[blockIdx.x * blockDim.x + threadIdx.x] = a0 ^ a1 ^ a2 ^ a3;
+}
+
+// The T-table access pattern of the lane loop (fused_common.cuh TL): a 64 KB
+// table image at a 64 KB-aligned shared address, one PRMT forms the whole
+// address (byte 0 of the state word -> bits 8..15, lane*4 -> bits 0..7, the
+// base -> bits 16..31): 1 ALU op per LDS, 8 independent chains per thread.
+__global__ void __launch_bounds__(512, 1) k_lds_prmt(uint32_t *out, unsigned long long *cyc, uint32_t seed)
+{
+    extern __shared__ __align__(16) uint8_t smem[];
+    const uint32_t sb = (uint32_t)__cvta_generic_to_shared(smem);
+    const uint32_t toff = (0x10000u - (sb & 0xffffu)) & 0xffffu;
+    uint32_t *tw = reinterpret_cast<uint32_t *>(smem + toff);
+    for (uint32_t i = threadIdx.x; i < 16384u; i += blockDim.x) tw[i] = (i * 2654435761u) ^ seed;
+    __syncthreads();
+    const uint32_t lane4r = ((threadIdx.x & 31u) * 4u) | ((sb + toff) & 0xffff0000u);
+    uint32_t a[8];
+#pragma unroll
+    for (int k = 0; k < 8; k++) a[k] = seed * (threadIdx.x + 1u) + 977u * k;
+    unsigned long long c0 = clock64();
+#pragma unroll 2
+    for (int i = 0; i < ITERS; i++) {
+#pragma unroll
+        for (int k = 0; k < 8; k++) {
+            const uint32_t ad = __byte_perm(a[k], lane4r, 0x7604u | ((k & 3) << 4));
+            asm volatile("ld.shared.u32 %0, [%1];" : "=r"(a[k]) : "r"(ad));
+        }
+    }
+    unsigned long long c1 = clock64();
+    if (threadIdx.x == 0) atomicMax(cyc, c1 - c0);
+    uint32_t x = 0;
+#pragma unroll
+    for (int k = 0; k < 8; k++) x ^= a[k];
+    out[blockIdx.x * blockDim.x + threadIdx.x] = x;
+}
+
+// Shared-memory loads with no address arithmetic (fixed per-lane addresses,
+// conflict-free, volatile so they are not hoisted): 16 loads and 8 three-input
+// XORs per iteration -- the LDS rate with the ALU pipe nearly idle.
+__global__ void __launch_bounds__(512, 1) k_lds_pure(uint32_t *out, unsigned long long *cyc, uint32_t seed)
+{
+    __shared__ uint32_t t[16 * 32 * 8];
+    for (uint32_t i = threadIdx.x; i < 16u * 32u * 8u; i += blockDim.x) t[i] = i * 2654435761u ^ seed;
+    __syncthreads();
+    const uint32_t base = (uint32_t)__cvta_generic_to_shared(&t[(threadIdx.x & 31u) + 512u * ((threadIdx.x >> 5) & 7u)]);
+    uint32_t acc0 = 0, acc1 = 0;
+    unsigned long long c0 = clock64();
+#pragma unroll 1
+    for (int i = 0; i < ITERS; i++) {
+        uint32_t v[16];
+#define LDK(k) asm volatile("ld.shared.u32 %0, [%1+" #k "];" : "=r"(v[(k) / 128]) : "r"(base))
+        LDK(0); LDK(128); LDK(256); LDK(384); LDK(512); LDK(640); LDK(768); LDK(896);
+        LDK(1024); LDK(1152); LDK(1280); LDK(1408); LDK(1536); LDK(1664); LDK(1792); LDK(1920);
+#undef LDK
+#pragma unroll
+        for (int k = 0; k < 16; k += 4) {
+            acc0 ^= v[k] ^ v[k + 1];
+            acc1 ^= v[k + 2] ^ v[k + 3];
+        }
+    }
+    unsigned long long c1 = clock64();
+    if (threadIdx.x == 0) atomicMax(cyc, c1 - c0);
+    out[blockIdx.x * blockDim.x + threadIdx.x] = acc0 ^ acc1;
 }
 
 template <int OP>
@@ -154,6 +220,13 @@ int main()
     printf("{\n  \"sms\": %d, \"clock_khz_attr\": %d,\n", nsm, clk_khz);
     const int B = nsm * 2, TH = 1024;
     run([&] { k_lds<<<B, TH>>>(out, cyc, 1); }, 4.0 * ITERS, B, TH, "lds32_lanes", false);
+    CK(cudaFuncSetAttribute(k_lds_prmt, cudaFuncAttributeMaxDynamicSharedMemorySize, 131072));
+    run([&] { k_lds_prmt<<<nsm, 512, 131072>>>(out, cyc, 1); }, 8.0 * ITERS, nsm, 512,
+        "lds32_prmt_lanes", false);
+    run([&] { k_lds_pure<<<nsm, 512>>>(out, cyc, 1); }, 16.0 * ITERS, nsm, 512, "lds32_pure_lanes",
+        false);
+    run([&] { k_lds_pure<<<nsm * 2, 512>>>(out, cyc, 1); }, 16.0 * ITERS, nsm * 2, 512,
+        "lds32_pure_lanes_2cta", false);
     run([&] { k_alu<0><<<B, TH>>>(out, cyc, 1); }, 8.0 * ITERS, B, TH, "lop3_lanes", false);
     run([&] { k_alu<1><<<B, TH>>>(out, cyc, 1); }, 8.0 * ITERS, B, TH, "prmt_lanes", false);
     run([&] { k_alu<2><<<B, TH>>>(out, cyc, 1); }, 8.0 * ITERS, B, TH, "shf_lanes", false);
