@@ -328,8 +328,9 @@ int nba_ipsec_route_pack_map(const uint8_t *in_buf, const uint32_t *in_off, cons
  * pointers are valid on the calling device; receiver d gets its packets at
  * positions 0..count-1 (batch order), offsets into its buf, and
  * count[0] = packets, count[1] = bytes (written by the dispatch).  Each
- * receiver needs cap_pkts >= n_pkts entries and cap_bytes >= the batch's bytes
- * to take every packet; when its packets do not fit, the receiver gets the
+ * receiver needs cap_pkts >= its packets and cap_bytes >= their bytes to take
+ * all of them (cap_pkts = n_pkts and cap_bytes = the batch's bytes always do);
+ * when its packets do not fit, the receiver gets the
  * longest prefix (in batch order) that fits both capacities, count[] says how
  * many packets / bytes that is, and nothing is written past the capacity --
  * the caller detects the overflow as dest_counts[d] > rx count (the dropped

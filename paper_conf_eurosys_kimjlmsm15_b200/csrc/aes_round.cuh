@@ -15,7 +15,6 @@
 
 namespace nba {
 
-constexpr uint32_t AES_TABLE_BYTES = 2u * 65536u;
 
 // Build the replicated tables from the 1-KB base T0 (global).  All threads of
 // the block participate; caller synchronises afterwards.

@@ -227,6 +227,7 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
 
     uint4 *d_rk = nullptr, *d_hm = nullptr, *d_hdr = nullptr, *d_sal = nullptr;
     uint32_t *d_seq = nullptr, *d_seq_prev = nullptr, *d_te0 = nullptr;
+    uint4 *d_timg = nullptr;
     const uint32_t M = max_batch_pkts;
     cudaError_t e = cudaSuccess;
     auto chk = [&](cudaError_t x) {
@@ -239,6 +240,7 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
     chk(dalloc(t, &d_seq, n_sa));
     chk(dalloc(t, &d_seq_prev, n_sa));
     chk(dalloc(t, &d_te0, 256));
+    chk(dalloc(t, &d_timg, AES_TABLE_BYTES / sizeof(uint4)));
     DevWork &W = t->W;
     chk(dalloc(t, &W.lrank, M));
     chk(dalloc(t, &W.m_rec, M));
@@ -268,6 +270,18 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
         chk(cudaMemcpy(d_sal, sal.data(), sal.size() * sizeof(uint4), cudaMemcpyHostToDevice));
         chk(cudaMemcpy(d_seq, seq.data(), n_sa * sizeof(uint32_t), cudaMemcpyHostToDevice));
         chk(cudaMemcpy(d_te0, host_te0(), 256 * sizeof(uint32_t), cudaMemcpyHostToDevice));
+        // the kernels' shared-memory table image (bulk-copied per CTA): entry x
+        // of table j (Tj = rotl(T0, 8j)) at byte (j >> 1) * 64 KB + 256 x +
+        // 128 (j & 1) + 4 lane, replicated over the 32 lanes (fused_common.cuh TL)
+        std::vector<uint32_t> img(AES_TABLE_BYTES / 4);
+        const uint32_t *te0 = host_te0();
+        for (uint32_t j = 0; j < 4; j++)
+            for (uint32_t x = 0; x < 256; x++) {
+                const uint32_t v = j ? (te0[x] << (8 * j)) | (te0[x] >> (32 - 8 * j)) : te0[x];
+                for (uint32_t l = 0; l < 32; l++)
+                    img[(j >> 1) * 16384u + x * 64u + (j & 1u) * 32u + l] = v;
+            }
+        chk(cudaMemcpy(d_timg, img.data(), AES_TABLE_BYTES, cudaMemcpyHostToDevice));
     }
     if (e == cudaSuccess) chk(setup_prologue_attributes(n_sa, t->max_tiles, t->num_sms, &t->gridsync));
     // testing: force the last-CTA (non co-resident) fallback of the per-SA scans
@@ -283,7 +297,7 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
         delete t;
         return e == cudaErrorMemoryAllocation ? NBA_IPSEC_ENOMEM : NBA_IPSEC_ECUDA;
     }
-    t->T = DevTable{d_rk, d_hm, d_hdr, d_seq, d_seq_prev, d_te0, n_sa, d_sal};
+    t->T = DevTable{d_rk, d_hm, d_hdr, d_seq, d_seq_prev, d_te0, n_sa, d_sal, d_timg};
     *out = t;
     return NBA_IPSEC_OK;
 }
@@ -560,9 +574,13 @@ static int ring_launch(nba_ipsec_ring *r, uint32_t first, uint32_t n_batches, cu
     nba_ipsec_sa_table *t = r->t;
     if (n_batches == 0) return NBA_IPSEC_OK;
     if (r->ts) {
-        if (n_batches >= r->ts_cap) return NBA_IPSEC_EINVAL;
-        if (cudaMemsetAsync(r->ts, 0, (size_t)(n_batches + 1) * sizeof(unsigned long long), st) !=
-            cudaSuccess)
+#ifdef NBA_RING_TRACE   // debug variant: [n_batches][grid][8] phase stamps
+        const size_t need = (size_t)n_batches * t->grid_fused * 8u;
+#else
+        const size_t need = (size_t)n_batches + 1u;
+#endif
+        if (need > r->ts_cap) return NBA_IPSEC_EINVAL;
+        if (cudaMemsetAsync(r->ts, 0, need * sizeof(unsigned long long), st) != cudaSuccess)
             return NBA_IPSEC_ECUDA;
     }
     const RingRun R{r->n_slots, first, n_batches, r->ts};
@@ -1039,7 +1057,7 @@ int nba_ipsec_route_dispatch(const uint8_t *in_buf, const uint32_t *in_off, cons
                              uint64_t *dest_counts, uint64_t *dest_bytes, void *cuda_stream)
 {
     if (world == 0 || world > 8 || n_pkts > NBA_IPSEC_MAX_BATCH) return NBA_IPSEC_EINVAL;
-    if (!dest_counts || !dest_bytes || !rx || cap_pkts < n_pkts) return NBA_IPSEC_EINVAL;
+    if (!dest_counts || !dest_bytes || !rx) return NBA_IPSEC_EINVAL;   // any capacity: prefix kept
     if (n_pkts && (!in_buf || !in_off || !in_len || !sa_global || !workspace))
         return NBA_IPSEC_EINVAL;
     cudaStream_t st = static_cast<cudaStream_t>(cuda_stream);

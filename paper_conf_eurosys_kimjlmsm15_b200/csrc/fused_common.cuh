@@ -38,6 +38,7 @@ struct FusedLo {
     uint8_t wrun[F_THREADS / 32];  // warp -> run of 32 sorted positions (0xff: none)
     uint32_t pstat[3];             // pipelined ring: the next batch's AES steps (sum, max) and
                                    //   its "early round keys" decision
+    unsigned long long tbar;       // mbarrier: the bulk copy of the T-table image landed
 };
 
 struct FusedHi {
@@ -56,6 +57,69 @@ static_assert(F_SMEM <= 232448, "exceeds 227 KB of shared memory per block");
 __device__ __forceinline__ uint32_t smem_u32(const void *p)
 {
     return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+// ---- T-table staging by bulk-async copy (TMA engine, cp.async.bulk) ---------
+// The 128 KB bank-replicated table image is built once per SA table in global
+// memory (DevTable::timg, exactly the shared-memory layout), and one thread
+// per CTA copies it into shared memory with eight 16 KB cp.async.bulk
+// operations that complete on an mbarrier (transaction count = 128 KB); the
+// other threads go on with the batch's metadata / ranking and wait on the
+// mbarrier only before their first table lookup.
+#ifndef NBA_TMA_TABLES        // 0: the A/B baseline -- every thread copies the 1 KB T0 and
+#define NBA_TMA_TABLES 1      //   stores the replicated / rotated image (aes_tables_to_smem)
+#endif
+
+__device__ __forceinline__ void tbar_init(unsigned long long *bar)
+{
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(bar)) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+
+// One thread: arm the mbarrier for 128 KB and issue the copies.  Earlier
+// generic-proxy accesses of the region (scratch use) are ordered before the
+// async-proxy writes by the proxy fence (the caller has synchronised the CTA).
+__device__ __forceinline__ void tables_bulk_issue(uint8_t *tabs, const uint4 *timg, unsigned long long *bar)
+{
+    const uint32_t b = smem_u32(bar), d = smem_u32(tabs);
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(b), "n"(AES_TABLE_BYTES)
+                 : "memory");
+#pragma unroll
+    for (uint32_t i = 0; i < AES_TABLE_BYTES / 16384u; i++)
+        asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], 16384, [%2];"
+                     ::"r"(d + 16384u * i), "l"(timg + 1024u * i), "r"(b)
+                     : "memory");
+}
+
+// Start staging the tables (all threads call it; a CTA barrier must follow
+// before the mbarrier is waited on).  init: first staging of this launch.
+__device__ __forceinline__ void tables_stage(uint8_t *tabs, const DevTable &T, unsigned long long *bar,
+                                             bool init)
+{
+    if (!NBA_TMA_TABLES) {
+        aes_tables_to_smem(tabs, T.te0);
+        return;
+    }
+    if (threadIdx.x == 0) {
+        if (init) tbar_init(bar);
+        tables_bulk_issue(tabs, T.timg, bar);
+    }
+}
+
+// Wait until the phase with parity `phase` of the table mbarrier completed.
+__device__ __forceinline__ void tables_bulk_wait(unsigned long long *bar, uint32_t phase)
+{
+    if (!NBA_TMA_TABLES) return;   // staged by plain stores before a CTA barrier
+    const uint32_t b = smem_u32(bar);
+    uint32_t ok;
+    do {
+        asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+                     "selp.u32 %0, 1, 0, p;\n\t}"
+                     : "=r"(ok)
+                     : "r"(b), "r"(phase)
+                     : "memory");
+    } while (!ok);
 }
 
 template <uint32_t OFF>
@@ -659,16 +723,20 @@ __device__ __forceinline__ void length_sort(FusedLo &L, uint32_t j, uint32_t cnt
         if (__all_sync(0xffffffffu, lane >= nruns || cost == c0)) {
             if (lane < NW) L.wrun[lane] = lane < nruns ? (uint8_t)lane : 0xffu;
         } else {
-            uint32_t load[4] = {0u, 0u, 0u, 0u}, used[4] = {0u, 0u, 0u, 0u}, mine = 0xffu;
+            // least-loaded sub-partition first, in registers (no local memory)
+            uint32_t l0 = 0, l1 = 0, l2 = 0, l3 = 0, u0 = 0, u1 = 0, u2 = 0, u3 = 0, mine = 0xffu;
+            constexpr uint32_t CAP = NW / 4u;
             for (uint32_t r = 0; r < nruns; r++) {
                 const uint32_t cr = __shfl_sync(0xffffffffu, cost, r);
-                uint32_t best = 4u;
-#pragma unroll
-                for (uint32_t q = 0; q < 4u; q++)
-                    if (used[q] < NW / 4u && (best == 4u || load[q] < load[best])) best = q;
-                if (lane == best + 4u * used[best]) mine = r;
-                used[best]++;
-                load[best] += cr;
+                uint32_t best = 0, bl = 0xffffffffu, bu = 0;
+                if (u0 < CAP && l0 < bl) { best = 0; bl = l0; bu = u0; }
+                if (u1 < CAP && l1 < bl) { best = 1; bl = l1; bu = u1; }
+                if (u2 < CAP && l2 < bl) { best = 2; bl = l2; bu = u2; }
+                if (u3 < CAP && l3 < bl) { best = 3; bl = l3; bu = u3; }
+                if (lane == best + 4u * bu) mine = r;
+                u0 += best == 0; u1 += best == 1; u2 += best == 2; u3 += best == 3;
+                l0 += best == 0 ? cr : 0u; l1 += best == 1 ? cr : 0u;
+                l2 += best == 2 ? cr : 0u; l3 += best == 3 ? cr : 0u;
             }
             if (lane < NW) L.wrun[lane] = (uint8_t)mine;
         }

@@ -41,8 +41,11 @@ struct DevTable {
                             //   key 0), sahdr, hmid[0..2], {hout[0..2], 0} -- what an
                             //   outbound lane loads, as three 256-bit loads (it
                             //   expands round keys 1..10 itself)
+    const uint4 *timg;      // [8192] the 128 KB bank-replicated T-table image, laid out
+                            //   exactly as in shared memory (bulk-copied per CTA)
 };
 constexpr uint32_t SAL_U4 = 8;   // uint4s per SA line (5 used)
+constexpr uint32_t AES_TABLE_BYTES = 2u * 65536u;   // four 32x bank-replicated T-tables
 
 // --- per-batch workspace ----------------------------------------------------
 struct DevWork {

@@ -393,7 +393,7 @@ __device__ __forceinline__ void fused_body(const DevTable &T, const DevWork &W, 
     uint32_t old0 = 0;
     if (MERGED) old0 = scan_first_old(T, blockIdx.x * (F_THREADS / 32u) + warp,
                                       gridDim.x * (F_THREADS / 32u), gridDim.x, lane);
-    if (stage_tables) aes_tables_to_smem(tabs, T.te0);
+    if (stage_tables) tables_stage(tabs, T, &L.tbar, true);   // waited for before the first lookup
     if (tr && tid == 0) tr[2] = gtimer();
     if (tid < 4) L.cnt[tid] = 0ull;
     if (tid < NBINS) L.bins[tid] = 0;   // re-zeroed after each use (length_sort)
@@ -444,6 +444,7 @@ __device__ __forceinline__ void fused_body(const DevTable &T, const DevWork &W, 
         PktPre pp = {};
         if (sa_me != INVALID_SA) {
             pp = load_pkt_pre(T, B.in_buf, sa_me, inoff, true, 0u);
+            tables_bulk_wait(&L.tbar, 0u);
             if (!NBA_EXPAND_MID) expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
         }
         grid_wait(&W.ctl[CTL_BAR_MONO], bar_base + G);
@@ -564,6 +565,7 @@ __device__ __forceinline__ void fused_body(const DevTable &T, const DevWork &W, 
             if (!have) {
             } else if (info & INFO_OK) {
                 PktPre pp = load_pkt_pre(T, B.in_buf, sa_me, L.inoff[pk], false, (info >> 16) & 0xffu);
+                tables_bulk_wait(&L.tbar, 0u);
                 expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
                 esp_packet(T, B, L, H, lane4r, tid, sa_me, info, L.seq[pk], L.inoff[pk],
                            L.outoff[pk], pp,
@@ -584,6 +586,7 @@ __device__ __forceinline__ void fused_body(const DevTable &T, const DevWork &W, 
         __syncthreads();   // shared metadata is reused by the next super-round
     }
     }
+    tables_bulk_wait(&L.tbar, 0u);   // no bulk copy in flight past here (threads without packets)
     // counters: warp sums, then one 64-bit atomic per CTA and counter
     const uint32_t s0 = __reduce_add_sync(0xffffffffu, c_ok);
     const uint32_t s1 = __reduce_add_sync(0xffffffffu, c_drop);
@@ -667,6 +670,12 @@ k_fused_ring(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint16_t 
 #ifndef NBA_PIPE_LPT          // pipelined ring: LPT placement of the runs (1) or run r -> warp r
 #define NBA_PIPE_LPT 1
 #endif
+#ifndef NBA_RING_TRACE        // debug variant: per-(batch, CTA) phase stamps into RingRun::ts
+#define NBA_RING_TRACE 0      //   (tools/ring_trace.py; [n_batches][G][8] globaltimer ns)
+#endif
+#if NBA_RING_TRACE
+#define RTR(bi, k) (R.ts + ((size_t)(bi) * gridDim.x + blockIdx.x) * 8u + (k))
+#endif
 constexpr uint32_t PIPE_LANE_WARPS = 14;
 constexpr uint32_t PIPE_MAX_PPC = PIPE_LANE_WARPS * 32u;          // 448 packets per CTA
 constexpr uint32_t PIPE_P = F_THREADS - PIPE_MAX_PPC;             // 64 prologue threads
@@ -742,10 +751,38 @@ __device__ __forceinline__ void pipe_scan_rows(const DevTable &T, const DevWork 
         scan_sa_column<true>(T, W, sa, G, lane, epoch);
 }
 
+// LPT placement of nruns runs (costs in lanes 0..nruns-1) onto the four SM
+// sub-partitions (warp w issues on w mod 4; capq = lane warps on partition q):
+// longest-first is the caller's order, each run goes to the least loaded
+// partition with room (first minimum on ties), taking its next warp
+// q + 4 * used_q.  Returns the run this lane's warp gets (0xff: none).  All
+// state in registers (compare-select over the four partitions), so the
+// prologue warps spill nothing.
+__device__ __forceinline__ uint32_t lpt_place(uint32_t cost, uint32_t nruns, uint32_t lane,
+                                              uint32_t cap0, uint32_t cap1, uint32_t cap2,
+                                              uint32_t cap3)
+{
+    uint32_t l0 = 0, l1 = 0, l2 = 0, l3 = 0, u0 = 0, u1 = 0, u2 = 0, u3 = 0, mine = 0xffu;
+    for (uint32_t r = 0; r < nruns; r++) {
+        const uint32_t cr = __shfl_sync(0xffffffffu, cost, r);
+        uint32_t best = 0, bl = 0xffffffffu, bu = 0;
+        if (u0 < cap0 && l0 < bl) { best = 0; bl = l0; bu = u0; }
+        if (u1 < cap1 && l1 < bl) { best = 1; bl = l1; bu = u1; }
+        if (u2 < cap2 && l2 < bl) { best = 2; bl = l2; bu = u2; }
+        if (u3 < cap3 && l3 < bl) { best = 3; bl = l3; bu = u3; }
+        if (lane == best + 4u * bu) mine = r;
+        u0 += best == 0; u1 += best == 1; u2 += best == 2; u3 += best == 3;
+        l0 += best == 0 ? cr : 0u; l1 += best == 1 ? cr : 0u;
+        l2 += best == 2 ? cr : 0u; l3 += best == 3 ? cr : 0u;
+    }
+    return mine;
+}
+
 // Prologue of one batch by the 64 prologue threads (pt = 0..63) of this CTA.
 __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &W, const BatchArgs &B,
                                               uint32_t ppc, uint32_t bar_target, uint32_t epoch,
-                                              FusedLo &L, uint32_t pt, uint32_t parity)
+                                              FusedLo &L, uint32_t pt, uint32_t parity,
+                                              unsigned long long *tr_arrive = nullptr)
 {
     const uint32_t G = gridDim.x, cta = blockIdx.x, n_sa = T.n_sa;
     const uint32_t lane = pt & 31u, pw = pt >> 5;
@@ -926,22 +963,8 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
         }
         const uint32_t c0 = __shfl_sync(0xffffffffu, cost, 0);
         uint32_t mine = lane < nruns ? lane : 0xffu;      // equal costs: run r -> warp r
-        if (!__all_sync(0xffffffffu, lane >= nruns || cost == c0)) {
-            uint32_t load[4] = {0u, 0u, 0u, 0u}, used[4] = {0u, 0u, 0u, 0u};
-            mine = 0xffu;
-            for (uint32_t r = 0; r < nruns; r++) {
-                const uint32_t cr = __shfl_sync(0xffffffffu, cost, r);
-                uint32_t best = 4u;
-#pragma unroll
-                for (uint32_t q = 0; q < 4u; q++) {
-                    const uint32_t cap = q < 2u ? 4u : 3u;
-                    if (used[q] < cap && (best == 4u || load[q] < load[best])) best = q;
-                }
-                if (lane == best + 4u * used[best]) mine = r;
-                used[best]++;
-                load[best] += cr;
-            }
-        }
+        if (!__all_sync(0xffffffffu, lane >= nruns || cost == c0))
+            mine = lpt_place(cost, nruns, lane, 4u, 4u, 3u, 3u);
         if (lane < PIPE_LANE_WARPS) L.wrun[lane] = (uint8_t)mine;
     }
     // 4. arrive at this batch's grid barrier (the whole CTA waits for it at
@@ -958,6 +981,7 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
 #endif
     if (pt == 0)
         asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&W.ctl[CTL_BAR_MONO]) : "memory");
+    if (tr_arrive && pt == 0) *tr_arrive = gtimer();
 #if NBA_PIPE_PSCAN
     // and, once every CTA arrived, this CTA's share of the row scans (two
     // warps) -- always (PSCAN 1), or when most CTAs voted "long" (PSCAN 2: the
@@ -994,7 +1018,7 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
 // sequence number (0: no number, the packet is dropped).
 __device__ __forceinline__ void pipe_sequence(const DevTable &T, const DevWork &W, const BatchArgs &B,
                                               uint32_t ppc, uint32_t bar_target, uint32_t epoch,
-                                              FusedLo &L)
+                                              FusedLo &L, unsigned long long *tr = nullptr)
 {
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
     const uint32_t G = gridDim.x, cta = blockIdx.x;
@@ -1005,6 +1029,7 @@ __device__ __forceinline__ void pipe_sequence(const DevTable &T, const DevWork &
             asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(&W.ctl[CTL_BAR_MONO]) : "memory");
             if ((int)(v - bar_target) >= 0) break;
         }
+        if (tr) tr[1] = gtimer();
     }
     __syncthreads();
     const bool p_scanned = NBA_PIPE_PSCAN == 1 || (NBA_PIPE_PSCAN == 2 && (L.pstat[2] & 2u));
@@ -1025,6 +1050,7 @@ __device__ __forceinline__ void pipe_sequence(const DevTable &T, const DevWork &
         L.seq[j] = q32;
     }
     __syncthreads();
+    if (tr && tid == 0) tr[2] = gtimer();
 }
 
 __global__ void __launch_bounds__(F_THREADS, 1)
@@ -1035,7 +1061,7 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
     const uint32_t G = gridDim.x, cta = blockIdx.x;
     if (n_batches == 0) return;
-    if (R.ts && cta == 0 && tid == 0) R.ts[0] = gtimer();
+    if (!NBA_RING_TRACE && R.ts && cta == 0 && tid == 0) R.ts[0] = gtimer();
     const uint32_t base0 = *reinterpret_cast<volatile uint32_t *>(&W.ctl[CTL_BAR_BASE]);
     const uint32_t ep0 = *reinterpret_cast<volatile uint32_t *>(&W.ctl[CTL_EPOCH]);
     const uint32_t sb = smem_u32(smem);
@@ -1049,7 +1075,7 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
     FusedLo &L = *reinterpret_cast<FusedLo *>(smem + lo_off);
     FusedHi &H = *reinterpret_cast<FusedHi *>(smem + toff + AES_TABLE_BYTES);
     const uint32_t lane4r = (lane * 4u) | (smem_u32(tabs) & 0xffff0000u);
-    aes_tables_to_smem(tabs, T.te0);
+    tables_stage(tabs, T, &L.tbar, true);   // bulk copy, waited for before the first lookup
     if (tid < NBINS) L.bins[tid] = 0u;
     for (uint32_t k = tid; k < 2u * F_SUPER; k += F_THREADS) {
         L.hkey[k] = INVALID_SA;
@@ -1073,6 +1099,9 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
     unsigned long long c_ok = 0, c_drop = 0, c_in = 0, c_out = 0;
     for (uint32_t bi = 0; bi < n_batches; bi++) {
         const BatchArgs B = slots[(first + bi) % n_slots];
+#if NBA_RING_TRACE
+        if (tid == 0) *RTR(bi, 0) = gtimer();
+#endif
         // lanes: the packet (known since the previous batch); its SA line and
         // round keys either before the barrier wait / scans / polls, whose
         // latency they then overlap (long or length-divergent batches, as
@@ -1097,10 +1126,18 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
             outoff = have ? L.outoff[pk] : 0u;
             if (early && (info & INFO_OK)) {
                 pp = load_pkt_pre(T, B.in_buf, sa, inoff, true, 0u);
+                tables_bulk_wait(&L.tbar, 0u);
                 expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
             }
+#if NBA_RING_TRACE
+            if (lane == 0) atomicMax(RTR(bi, 6), gtimer());
+#endif
         }
+#if NBA_RING_TRACE
+        pipe_sequence(T, work_of(bi), B, ppc, base0 + (bi + 1) * G, epoch_of(bi), L, RTR(bi, 0));
+#else
         pipe_sequence(T, work_of(bi), B, ppc, base0 + (bi + 1) * G, epoch_of(bi), L);
+#endif
         if (!isP) {
             const uint32_t q32 = have ? L.seq[pk] : 0u;
             bar_arrive_n(2, F_THREADS);                  // fields taken: the arrays are free
@@ -1109,6 +1146,7 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
                 if ((info & INFO_OK) && q32 != 0u) {
                     if (!early) {
                         pp = load_pkt_pre(T, B.in_buf, sa, inoff, true, 0u);
+                        tables_bulk_wait(&L.tbar, 0u);
                         expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
                     }
                     if (!NBA_PROLOGUE_ONLY)   // (debug A/B: the ring without the lane work)
@@ -1124,17 +1162,30 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
                     c_drop++;
                 }
             }
+#if NBA_RING_TRACE
+            if (lane == 0) atomicMax(RTR(bi, 3), gtimer());
+#endif
         } else {
             bar_sync_n(2, F_THREADS);                    // every lane took its fields
             if (bi + 1 < n_batches) {
                 const BatchArgs Bn = slots[(first + bi + 1) % n_slots];
+#if NBA_RING_TRACE
+                pipe_prologue(T, work_of(bi + 1), Bn, fused_ppc(Bn.n, G), base0 + (bi + 2) * G,
+                              epoch_of(bi + 1), L, pt, (bi + 1) & 1u, RTR(bi, 4));
+#else
                 pipe_prologue(T, work_of(bi + 1), Bn, fused_ppc(Bn.n, G), base0 + (bi + 2) * G,
                               epoch_of(bi + 1), L, pt, (bi + 1) & 1u);
+#endif
             }
         }
         __syncthreads();                                  // batch bi done, bi + 1 prepared
+#if NBA_RING_TRACE
+        if (tid == 0) *RTR(bi, 5) = gtimer();
+#else
         if (R.ts && tid == 0) atomicMax(&R.ts[1u + bi], gtimer());
+#endif
     }
+    tables_bulk_wait(&L.tbar, 0u);   // no bulk copy in flight at exit
     // counters (as fused_body), device state for the next launch
     if (tid < 4) L.cnt[tid] = 0ull;
     __syncthreads();

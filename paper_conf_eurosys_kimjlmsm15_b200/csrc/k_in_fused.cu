@@ -270,7 +270,7 @@ __device__ __forceinline__ void in_merged_tail(const DevTable &T, const InState 
 template <bool MERGED>
 __device__ __forceinline__ void in_fused_body(const DevTable &T, const InState &S,
                                               const InBatchArgs &B, uint32_t ppc, uint32_t hmask,
-                                              uint32_t bar_base)
+                                              uint32_t bar_base, bool tinit, uint32_t tphase)
 {
     extern __shared__ __align__(16) uint8_t smem[];
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
@@ -294,7 +294,10 @@ __device__ __forceinline__ void in_fused_body(const DevTable &T, const InState &
         S.hkey[k] = ~0ull;
         S.hval[k] = ~0u;
     }
-    aes_tables_to_smem(tabs, T.te0);
+    // T-tables by bulk copy (re-staged per batch: the replay merge of the
+    // previous batch used their shared memory as scratch); waited for (phase
+    // tphase of the mbarrier) before the first lookup
+    tables_stage(tabs, T, &L.tbar, tinit);
     if (tid < NBINS) L.bins[tid] = 0;
     __syncthreads();
 
@@ -362,6 +365,7 @@ __device__ __forceinline__ void in_fused_body(const DevTable &T, const InState &
                     const uint4 *line = T.sal + (size_t)sa_me * SAL_U4;
                     ldg_nc_v8(&line[0], r0, hd);
                     ldg_nc_v8(&line[2], h0, h1);
+                    tables_bulk_wait(&L.tbar, tphase);
                     expand_key_lane(lane4r, r0, r1, r2, L, H, tid);
                     flags = INF_FMT | esp_in_packet(T, B, L, H, lane4r, tid, sa_me, info & 0xffffu,
                                                     L.seq[pk], L.aux0[pk], L.aux1[pk], L.inoff[pk],
@@ -377,6 +381,10 @@ __device__ __forceinline__ void in_fused_body(const DevTable &T, const InState &
         }
         __syncthreads();
     }
+    // every thread has seen the bulk copy land (also those without packets):
+    // the tail uses the table region as scratch, and no copy may be in flight
+    // when the CTA exits
+    tables_bulk_wait(&L.tbar, tphase);
     if constexpr (MERGED) in_merged_tail(T, S, B, L, tabs, p_begin, p_end, hmask, bar_base);
 }
 
@@ -388,7 +396,7 @@ k_in_fused(DevTable T, InState S, InBatchArgs B, uint32_t ppc, uint32_t hmask, u
     // host state and can be recorded in a graph); read before arriving
     const uint32_t bar_base =
         MERGED ? *reinterpret_cast<volatile uint32_t *>(&S.ctl[CTLI_BASE]) : bar_base_h;
-    in_fused_body<MERGED>(T, S, B, ppc, hmask, bar_base);
+    in_fused_body<MERGED>(T, S, B, ppc, hmask, bar_base, true, 0u);
 }
 
 // An inbound batch ring as ONE persistent launch: the grid walks the run's
@@ -415,7 +423,7 @@ k_in_fused_ring(DevTable T, InState S, const InBatchArgs *slots, RingRun R, uint
         uint32_t ppc = (B.n + G - 1) / G;
         ppc = (ppc + 31u) & ~31u;
         if (ppc < 32u) ppc = 32u;
-        in_fused_body<true>(T, Sb, B, ppc, hmask, base0 + 2u * bi * G);
+        in_fused_body<true>(T, Sb, B, ppc, hmask, base0 + 2u * bi * G, bi == 0, bi & 1u);
         __syncthreads();   // shared memory is reused by the next batch
         if (R.ts && threadIdx.x == 0) atomicMax(&R.ts[1u + bi], gtimer());
     }

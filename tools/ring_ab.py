@@ -1,0 +1,101 @@
+#!/usr/bin/env python
+"""Same-box A/B of compile-time variants of the batch ring, and a phase trace.
+
+    python tools/ring_ab.py build NAME=DEF1,DEF2 ...      (CPU: nvcc only -> build/variants/NAME.so)
+    python tools/ring_ab.py run [sizes...]                (GPU: bench protocol per variant, 2 passes)
+    python tools/ring_ab.py trace [sizes...]              (GPU: needs build/variants/trace.so,
+                                                           built with NBA_RING_TRACE=1)
+
+`run` times every variant (and the default library as `base`) in a fresh
+process through the NBA_IPSEC_LIB override with the bench's protocol: R device
+copies of a full-size 65,536-packet batch (1024 SAs), >= 2R warm-up batches,
+then K = 200 batches in ONE nba_ipsec_ring_run_batches call between one CUDA
+event pair.  Passes are interleaved to expose drift.
+
+`trace` prints, per size, the median over batches and CTAs of each phase of
+the software-pipelined ring (k_fused_ring_pipe): barrier seen, scans + polls
+done, lanes done, prologue warps' arrival for the next batch, iteration end,
+relative to the iteration start -- what sits on the per-batch critical path."""
+import os
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+VDIR = os.path.join(ROOT, "build", "variants")
+sys.path.insert(0, ROOT)
+
+TIMER = r'''
+import os, sys, json
+sys.path.insert(0, %(root)r)
+import numpy as np, torch
+from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec, shard
+K = %(k)d
+out = {}
+for size in %(sizes)r:
+    cfg = {64: 2, 1514: 3, "imix": 4}.get(size, 5)
+    p, b = shard.rank_workload(cfg, 65536, size, 1024, 0, 1)
+    t = nba_ipsec.SATable(p, max_batch=65536)
+    d0 = device.to_device(b, "cuda")
+    R = device.ring_slot_count(b.in_len, b.n, torch.cuda.get_device_properties(0).L2_cache_size)
+    dbs = [d0] + [device.clone(d0) for _ in range(R - 1)]
+    ring = t.ring([(*d.args(), b.n) for d in dbs])
+    ring.run_batches(max(40, 4 * R)); torch.cuda.synchronize()
+    if %(trace)r:
+        G = 148
+        ts = torch.zeros(K * G * 8, dtype=torch.int64, device="cuda")
+        ring.set_timestamps(ts)
+        ring.run_batches(K); torch.cuda.synchronize()
+        v = ts.cpu().numpy().reshape(K, G, 8).astype(np.int64)[2:]     # skip start-up
+        rel = (v - v[:, :, :1]) / 1e3
+        names = ["start", "barrier_seen", "polls_done", "lanes_done", "prologue_arrived",
+                 "iter_end", "early_keys_done"]
+        med = {n: float(np.median(rel[:, :, i])) for i, n in enumerate(names) if i}
+        p90 = {n: float(np.percentile(rel[:, :, i], 90)) for i, n in enumerate(names) if i}
+        it = np.diff(v[:, 0, 0]) / 1e3
+        out[str(size)] = {"median_us": med, "p90_us": p90, "iter_us": float(np.median(it))}
+    else:
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(); ring.run_batches(K); e1.record(); torch.cuda.synchronize()
+        out[str(size)] = round(e0.elapsed_time(e1) * 1e3 / K, 2)
+    ring.close(); t.close(); del dbs
+print(json.dumps(out), flush=True)
+'''
+
+
+def run_one(lib, sizes, k, trace):
+    env = dict(os.environ)
+    if lib:
+        env["NBA_IPSEC_LIB"] = lib
+    code = TIMER % {"root": ROOT, "sizes": sizes, "k": k, "trace": trace}
+    r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True)
+    if r.returncode:
+        return "FAILED: " + r.stderr[-600:]
+    return r.stdout.strip()
+
+
+def main():
+    cmd = sys.argv[1]
+    args = sys.argv[2:]
+    if cmd == "build":
+        from paper_conf_eurosys_kimjlmsm15_b200 import build
+        os.makedirs(VDIR, exist_ok=True)
+        for spec in args:
+            name, _, defs = spec.partition("=")
+            d = [x for x in defs.split(",") if x]
+            print(name, build.build(out=os.path.join(VDIR, name + ".so"), defines=d), flush=True)
+        return
+    sizes = [x if x == "imix" else int(x) for x in args] or [64, 1514, "imix"]
+    if cmd == "trace":
+        print("trace", run_one(os.path.join(VDIR, "trace.so"), sizes, 50, True), flush=True)
+        return
+    names = sorted(f[:-3] for f in os.listdir(VDIR) if f.endswith(".so") and f != "trace.so") \
+        if os.path.isdir(VDIR) else []
+    for rep in range(2):
+        print(f"pass {rep} base", run_one(None, sizes, 200, False), flush=True)
+        for n in names:
+            print(f"pass {rep} {n}", run_one(os.path.join(VDIR, n + ".so"), sizes, 200, False),
+                  flush=True)
+
+
+if __name__ == "__main__":
+    main()
