@@ -167,6 +167,24 @@ __device__ __forceinline__ void prefetch_l2(const void *p)
     asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
 }
 
+#ifndef NBA_BULK_PF            // 1: packet prefetches as bulk L2 prefetches of exactly the
+#define NBA_BULK_PF 0         //   16-byte-aligned cover of the bytes used (else whole lines)
+#endif
+
+// L2 prefetch of bytes [p, p + n) of a packet (n > 0): one line prefetch at p,
+// or (NBA_BULK_PF) a bulk prefetch of the 16-B aligned cover of the range
+// (sectors only, no whole-line over-fetch of short packets).
+__device__ __forceinline__ void prefetch_bytes(const uint8_t *p, uint32_t n)
+{
+    if (!NBA_BULK_PF) {
+        prefetch_l2(p);
+        return;
+    }
+    const uintptr_t a = reinterpret_cast<uintptr_t>(p), lo = a & ~(uintptr_t)15;
+    const uint32_t sz = (uint32_t)(((a + n + 15u) & ~(uintptr_t)15) - lo);
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(lo), "r"(sz) : "memory");
+}
+
 __device__ __forceinline__ void stg_v4(void *p, uint32_t a, uint32_t b, uint32_t c, uint32_t d)
 {
     asm volatile("st.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(a), "r"(b), "r"(c), "r"(d)

@@ -144,7 +144,7 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
     // metadata phase); each step prefetches two steps ahead
 #pragma unroll
     for (uint32_t k = 1; k < NBA_PF_AHEAD; k++)
-        if (D > 64u * k) prefetch_l2(src + 64u * k);
+        if (D > 64u * k) prefetch_bytes(src + 64u * k, min(64u, D - 64u * k));
 
     // ---- one SHA-1 compression per iteration; AES steps feed the first nsteps
 #pragma unroll 1
@@ -155,7 +155,8 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
         for (int w = 0; w < 16; w++) ct[w] = 0u;
         if (it < nsteps) {
             // payload words of T bytes [64 it, 64 it + 64), realigned
-            if (64u * (it + NBA_PF_AHEAD) < D) prefetch_l2(src + 64u * (it + NBA_PF_AHEAD));
+            if (64u * (it + NBA_PF_AHEAD) < D)
+                prefetch_bytes(src + 64u * (it + NBA_PF_AHEAD), min(64u, D - 64u * (it + NBA_PF_AHEAD)));
             // interior step: all 16 words are payload, the trailer (last word and,
             // when p = 3, the one before) lies beyond it, and the five 16-byte
             // loads are inside the datagram -- no per-word selects, one bounds test
@@ -422,7 +423,7 @@ __device__ __forceinline__ void fused_body(const DevTable &T, const DevWork &W, 
             L.inoff[j] = pre_inoff;
             L.outoff[j] = pre_outoff;
             // the lane reads the payload after the barrier: DRAM -> L2 now
-            if (cand) prefetch_l2(B.in_buf + pre_inoff);
+            if (cand) prefetch_bytes(B.in_buf + pre_inoff, min(64u, pre_D));
         }
         warp_agg_add(L.bins, bin, j < cnt_pk);
         // 1. CTA-local ranks and per-SA counts (the prologue's tile part)
@@ -662,8 +663,9 @@ k_fused_ring(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint16_t 
 #define NBA_PIPE_EARLY_KEYS 2 // 1 always, 0 never, 2 per batch (long or length-divergent)
 #endif
 #ifndef NBA_PIPE_PSCAN        // pipelined ring: the prologue warps also run the row scans:
-#define NBA_PIPE_PSCAN 0      // 0 never, 1 always, 2 when most CTAs vote the batch long
-#endif
+#define NBA_PIPE_PSCAN 0      // 0 never, 1 always, 2 when most CTAs vote the batch long,
+#endif                        // 3 always + the prologue warps poll the bases too (the next
+                              //   batch's sequence numbers are ready when it starts)
 #ifndef NBA_PIPE_HALVES       // pipelined ring: the two prologue warps rank halves concurrently
 #define NBA_PIPE_HALVES 1
 #endif
@@ -674,7 +676,7 @@ k_fused_ring(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint16_t 
 #define NBA_RING_TRACE 0      //   (tools/ring_trace.py; [n_batches][G][8] globaltimer ns)
 #endif
 #if NBA_RING_TRACE
-#define RTR(bi, k) (R.ts + ((size_t)(bi) * gridDim.x + blockIdx.x) * 8u + (k))
+#define RTR(bi, k) (R.ts ? R.ts + ((size_t)(bi) * gridDim.x + blockIdx.x) * 8u + (k) : nullptr)
 #endif
 constexpr uint32_t PIPE_LANE_WARPS = 14;
 constexpr uint32_t PIPE_MAX_PPC = PIPE_LANE_WARPS * 32u;          // 448 packets per CTA
@@ -820,7 +822,7 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
             L.inoff[j] = mI[r];
             L.outoff[j] = mO[r];
             bin = hmac_bin(cand, esp_C(mD[r]));
-            if (cand) prefetch_l2(B.in_buf + mI[r]);   // the lane reads it next round
+            if (cand) prefetch_bytes(B.in_buf + mI[r], min(64u, mD[r]));   // the lane reads it next round
         }
         if (r < rounds) warp_agg_add(L.bins, bin, j < cnt);
     }
@@ -1010,6 +1012,34 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
     }
 #endif
     if (pscan) pipe_scan_rows(T, W, cta * 2u + pw, G * 2u, G, lane, epoch);
+#if NBA_PIPE_PSCAN == 3
+    // the sequence numbers of this CTA's packets: every poll issued before any
+    // is re-tried (one memory round trip when the bases are already published)
+    {
+        unsigned long long v[PR];
+        uint32_t sa_r[PR];
+#pragma unroll
+        for (uint32_t r = 0; r < PR; r++) {
+            const uint32_t j = r * PIPE_P + pt;
+            const bool ok = j < cnt && (L.info[j] & INFO_OK);
+            sa_r[r] = ok ? L.sa[j] : INVALID_SA;
+            v[r] = ok ? ld_relaxed_u64(&W.hbase[(size_t)sa_r[r] * G + cta]) : 0ull;
+        }
+#pragma unroll
+        for (uint32_t r = 0; r < PR; r++) {
+            const uint32_t j = r * PIPE_P + pt;
+            if (j >= cnt) continue;
+            uint32_t q32 = 0;
+            if (sa_r[r] != INVALID_SA) {
+                const unsigned long long *pb = &W.hbase[(size_t)sa_r[r] * G + cta];
+                while ((uint32_t)(v[r] >> 33) != epoch) v[r] = ld_relaxed_u64(pb);
+                const unsigned long long q = (v[r] & ((1ull << 33) - 1ull)) + 1ull + L.seq[j];
+                q32 = q <= 0xffffffffull ? (uint32_t)q : 0u;   // RFC 4303 §3.3.3: never cycle
+            }
+            L.seq[j] = q32;
+        }
+    }
+#endif
 #endif
 }
 
@@ -1023,6 +1053,7 @@ __device__ __forceinline__ void pipe_sequence(const DevTable &T, const DevWork &
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
     const uint32_t G = gridDim.x, cta = blockIdx.x;
     constexpr uint32_t NW = F_THREADS / 32u;
+    if (NBA_PIPE_PSCAN == 3) return;   // the prologue warps numbered the packets already
     if (tid == 0) {
         uint32_t v;
         while (true) {
@@ -1096,11 +1127,14 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
         pipe_prologue(T, work_of(0), B0, fused_ppc(B0.n, G), base0 + G, epoch_of(0), L, pt, 0u);
     }
     __syncthreads();
+    // the T-table image landed (the bulk copy overlapped the first prologue);
+    // every later lookup of the run finds it in place
+    tables_bulk_wait(&L.tbar, 0u);
     unsigned long long c_ok = 0, c_drop = 0, c_in = 0, c_out = 0;
     for (uint32_t bi = 0; bi < n_batches; bi++) {
         const BatchArgs B = slots[(first + bi) % n_slots];
 #if NBA_RING_TRACE
-        if (tid == 0) *RTR(bi, 0) = gtimer();
+        if (tid == 0 && R.ts) *RTR(bi, 0) = gtimer();
 #endif
         // lanes: the packet (known since the previous batch); its SA line and
         // round keys either before the barrier wait / scans / polls, whose
@@ -1126,11 +1160,10 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
             outoff = have ? L.outoff[pk] : 0u;
             if (early && (info & INFO_OK)) {
                 pp = load_pkt_pre(T, B.in_buf, sa, inoff, true, 0u);
-                tables_bulk_wait(&L.tbar, 0u);
                 expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
             }
 #if NBA_RING_TRACE
-            if (lane == 0) atomicMax(RTR(bi, 6), gtimer());
+            if (lane == 0 && R.ts) atomicMax(RTR(bi, 6), gtimer());
 #endif
         }
 #if NBA_RING_TRACE
@@ -1146,7 +1179,6 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
                 if ((info & INFO_OK) && q32 != 0u) {
                     if (!early) {
                         pp = load_pkt_pre(T, B.in_buf, sa, inoff, true, 0u);
-                        tables_bulk_wait(&L.tbar, 0u);
                         expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
                     }
                     if (!NBA_PROLOGUE_ONLY)   // (debug A/B: the ring without the lane work)
@@ -1163,7 +1195,7 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
                 }
             }
 #if NBA_RING_TRACE
-            if (lane == 0) atomicMax(RTR(bi, 3), gtimer());
+            if (lane == 0 && R.ts) atomicMax(RTR(bi, 3), gtimer());
 #endif
         } else {
             bar_sync_n(2, F_THREADS);                    // every lane took its fields
@@ -1180,12 +1212,11 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
         }
         __syncthreads();                                  // batch bi done, bi + 1 prepared
 #if NBA_RING_TRACE
-        if (tid == 0) *RTR(bi, 5) = gtimer();
+        if (tid == 0 && R.ts) *RTR(bi, 5) = gtimer();
 #else
         if (R.ts && tid == 0) atomicMax(&R.ts[1u + bi], gtimer());
 #endif
     }
-    tables_bulk_wait(&L.tbar, 0u);   // no bulk copy in flight at exit
     // counters (as fused_body), device state for the next launch
     if (tid < 4) L.cnt[tid] = 0ull;
     __syncthreads();

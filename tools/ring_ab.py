@@ -86,9 +86,11 @@ def main():
         return
     sizes = [x if x == "imix" else int(x) for x in args] or [64, 1514, "imix"]
     if cmd == "trace":
-        print("trace", run_one(os.path.join(VDIR, "trace.so"), sizes, 50, True), flush=True)
+        for f in sorted(os.listdir(VDIR)):
+            if f.endswith("trace.so"):
+                print(f[:-3], run_one(os.path.join(VDIR, f), sizes, 50, True), flush=True)
         return
-    names = sorted(f[:-3] for f in os.listdir(VDIR) if f.endswith(".so") and f != "trace.so") \
+    names = sorted(f[:-3] for f in os.listdir(VDIR) if f.endswith(".so") and not f.endswith("trace.so")) \
         if os.path.isdir(VDIR) else []
     for rep in range(2):
         print(f"pass {rep} base", run_one(None, sizes, 200, False), flush=True)
