@@ -784,7 +784,7 @@ __device__ __forceinline__ uint32_t lpt_place(uint32_t cost, uint32_t nruns, uin
 __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &W, const BatchArgs &B,
                                               uint32_t ppc, uint32_t bar_target, uint32_t epoch,
                                               FusedLo &L, uint32_t pt, uint32_t parity,
-                                              unsigned long long *tr_arrive = nullptr)
+                                              unsigned long long *tr = nullptr)
 {
     const uint32_t G = gridDim.x, cta = blockIdx.x, n_sa = T.n_sa;
     const uint32_t lane = pt & 31u, pw = pt >> 5;
@@ -983,7 +983,7 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
 #endif
     if (pt == 0)
         asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&W.ctl[CTL_BAR_MONO]) : "memory");
-    if (tr_arrive && pt == 0) *tr_arrive = gtimer();
+    if (tr && pt == 0) tr[4] = gtimer();   // (trace variant: tr = this iteration's stamps)
 #if NBA_PIPE_PSCAN
     // and, once every CTA arrived, this CTA's share of the row scans (two
     // warps) -- always (PSCAN 1), or when most CTAs voted "long" (PSCAN 2: the
@@ -997,6 +997,7 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
         }
     }
     bar_sync_n(1, PIPE_P);
+    if (tr && pt == 0) tr[1] = gtimer();
     bool pscan = true;
 #if NBA_PIPE_PSCAN == 2
     {
@@ -1012,6 +1013,7 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
     }
 #endif
     if (pscan) pipe_scan_rows(T, W, cta * 2u + pw, G * 2u, G, lane, epoch);
+    if (tr && pt == 0) tr[2] = gtimer();
 #if NBA_PIPE_PSCAN == 3
     // the sequence numbers of this CTA's packets: every poll issued before any
     // is re-tried (one memory round trip when the bases are already published)
@@ -1038,6 +1040,7 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
             }
             L.seq[j] = q32;
         }
+        if (tr && (pt & 31u) == 0) atomicMax(&tr[7], gtimer());
     }
 #endif
 #endif
@@ -1203,7 +1206,7 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
                 const BatchArgs Bn = slots[(first + bi + 1) % n_slots];
 #if NBA_RING_TRACE
                 pipe_prologue(T, work_of(bi + 1), Bn, fused_ppc(Bn.n, G), base0 + (bi + 2) * G,
-                              epoch_of(bi + 1), L, pt, (bi + 1) & 1u, RTR(bi, 4));
+                              epoch_of(bi + 1), L, pt, (bi + 1) & 1u, RTR(bi, 0));
 #else
                 pipe_prologue(T, work_of(bi + 1), Bn, fused_ppc(Bn.n, G), base0 + (bi + 2) * G,
                               epoch_of(bi + 1), L, pt, (bi + 1) & 1u);

@@ -48,7 +48,7 @@ for size in %(sizes)r:
         v = ts.cpu().numpy().reshape(K, G, 8).astype(np.int64)[2:]     # skip start-up
         rel = (v - v[:, :, :1]) / 1e3
         names = ["start", "barrier_seen", "polls_done", "lanes_done", "prologue_arrived",
-                 "iter_end", "early_keys_done"]
+                 "iter_end", "early_keys_done", "pseq_polls_done"]
         med = {n: float(np.median(rel[:, :, i])) for i, n in enumerate(names) if i}
         p90 = {n: float(np.percentile(rel[:, :, i], 90)) for i, n in enumerate(names) if i}
         it = np.diff(v[:, 0, 0]) / 1e3
