@@ -58,7 +58,7 @@ def _compile(src: str, verbose: bool, obj_dir: str = OBJ, defines=()) -> str:
 
 def build(force: bool = False, verbose: bool = False, out: str | None = None, defines=()) -> str:
     """Build the library (in-tree).  `out` + `defines`: an A/B variant with extra
-    -D flags, written elsewhere (tools/ab_variants.py); the product is the default."""
+    -D flags, written elsewhere (tools/ring_ab.py); the product is the default."""
     so = out or SO
     if out is None and not defines and not force and up_to_date():
         return SO

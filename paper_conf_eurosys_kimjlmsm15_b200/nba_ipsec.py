@@ -15,7 +15,7 @@ import re
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-# NBA_IPSEC_LIB: an A/B build variant of the same library (tools/ab_variants.py)
+# NBA_IPSEC_LIB: an A/B build variant of the same library (tools/ring_ab.py)
 LIB_PATH = os.environ.get("NBA_IPSEC_LIB") or os.path.join(_HERE, "libnba_ipsec.so")
 HEADER = os.path.join(os.path.dirname(_HERE), "include", "nba_ipsec.h")
 

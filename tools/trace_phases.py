@@ -28,8 +28,11 @@ for cfg in [int(x) for x in sys.argv[1:] if x.isdigit()] or (2, 3, 4):
     live = tr[:, 0] > 0
     tr = tr[live]
     t0 = pro[0] if pro[0] > 0 else tr[:, 0].min()
-    print("prologue: first start 0, tiles done %.2f, last-CTA start %.2f, end %.2f us" %
-          ((pro[1] - t0) / 1e3, (pro[2] - t0) / 1e3, (pro[3] - t0) / 1e3))
+    if pro[0] > 0 and pro[1] > 0:      # two-kernel path: the prologue kernel's own stamps
+        print("prologue kernel: first start 0, tiles done %.2f, last-CTA start %.2f, end %.2f us" %
+              ((pro[1] - t0) / 1e3, (pro[2] - t0) / 1e3, (pro[3] - t0) / 1e3))
+    else:                              # one-kernel path: the prologue runs inside k_fused
+        print("prologue: inside the fused kernel (one launch); phases below")
     rel = (tr - t0) / 1000.0
     names = ["start", "meta_done/arrived(merged)", "tables_done", "lanes_done", "m_tiles_done", "m_bar1_done",
              "m_scans_done", "keys_staged(tid0) / polls done (merged)"]
