@@ -575,7 +575,7 @@ static int ring_launch(nba_ipsec_ring *r, uint32_t first, uint32_t n_batches, cu
     if (n_batches == 0) return NBA_IPSEC_OK;
     if (r->ts) {
 #ifdef NBA_RING_TRACE   // debug variant: [n_batches][grid][8] phase stamps
-        const size_t need = (size_t)n_batches * t->grid_fused * 8u;
+        const size_t need = (size_t)n_batches * t->grid_fused * 16u;
 #else
         const size_t need = (size_t)n_batches + 1u;
 #endif

@@ -676,7 +676,7 @@ k_fused_ring(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint16_t 
 #define NBA_RING_TRACE 0      //   (tools/ring_trace.py; [n_batches][G][8] globaltimer ns)
 #endif
 #if NBA_RING_TRACE
-#define RTR(bi, k) (R.ts ? R.ts + ((size_t)(bi) * gridDim.x + blockIdx.x) * 8u + (k) : nullptr)
+#define RTR(bi, k) (R.ts ? R.ts + ((size_t)(bi) * gridDim.x + blockIdx.x) * 16u + (k) : nullptr)
 #endif
 constexpr uint32_t PIPE_LANE_WARPS = 14;
 constexpr uint32_t PIPE_MAX_PPC = PIPE_LANE_WARPS * 32u;          // 448 packets per CTA
@@ -698,59 +698,55 @@ __device__ __forceinline__ void bar_arrive_n(uint32_t id, uint32_t n)
     asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory");
 }
 
-// The prologue warps' share of the row scans (rows slot, slot + nslots, ...;
-// G <= 160 CTAs, so a row is at most 5 x 32 counts): every row's counts are
-// loaded before any is scanned, so the rows cost one memory round trip
-// instead of one each.  Same results as scan_all_columns (warp per row).
+// The prologue warps' share of the row scans (rows slot, slot + nslots, ...),
+// four rows at a time: 8 lanes per row, each lane owning CPL consecutive
+// columns (G <= 8 x CPL = 160 CTAs).  A lane loads its columns' counts (all
+// loads in flight together), sums them in registers, and one 3-step shuffle
+// scan across the row's 8 lanes gives each lane its starting prefix: ONE
+// memory round trip and a short shuffle chain per four rows, instead of a
+// 5 x 5-step shuffle chain per row.  Same results as scan_all_columns.
 __device__ __forceinline__ void pipe_scan_rows(const DevTable &T, const DevWork &W, uint32_t slot,
                                                uint32_t nslots, uint32_t G, uint32_t lane,
                                                uint32_t epoch)
 {
-    constexpr uint32_t MR = 4, U = 5;           // up to 4 rows per warp, 160 counts per row
-    uint32_t h[MR][U], old[MR];
-#pragma unroll
-    for (uint32_t r = 0; r < MR; r++) {
-        const uint32_t sa = slot + r * nslots;
+    constexpr uint32_t CPL = 20;                 // columns per lane (8 lanes per row)
+    const uint32_t r = lane >> 3, q = lane & 7u, c0 = q * CPL;
+    for (uint32_t g = 0; slot + g * 4u * nslots < T.n_sa; g++) {
+        const uint32_t sa = slot + (4u * g + r) * nslots;
         const bool ok = sa < T.n_sa;
-        old[r] = ok ? T.seq[sa] : 0u;
+        uint16_t *col = W.hist16 + (size_t)(ok ? sa : 0u) * G;
+        const uint32_t old = (ok && q == 0) ? T.seq[sa] : 0u;
+        uint32_t h[CPL];
 #pragma unroll
-        for (uint32_t u = 0; u < U; u++) {
-            const uint32_t t = 32u * u + lane;
-            h[r][u] = (ok && t < G) ? (uint32_t)__ldcg(&W.hist16[(size_t)sa * G + t]) : 0u;
+        for (uint32_t k = 0; k < CPL; k++) h[k] = (ok && c0 + k < G) ? (uint32_t)__ldcg(&col[c0 + k]) : 0u;
+        uint32_t sum = 0;
+#pragma unroll
+        for (uint32_t k = 0; k < CPL; k++) sum += h[k];
+        uint32_t x = sum;                        // inclusive scan over the row's 8 lanes
+#pragma unroll
+        for (uint32_t o = 1; o < 8u; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, x, o, 8);
+            if (q >= o) x += y;
+        }
+        const uint32_t tot = __shfl_sync(0xffffffffu, x, 7, 8);
+        const uint32_t old_r = __shfl_sync(0xffffffffu, old, 0, 8);
+        if (ok) {
+            unsigned long long run = (unsigned long long)old_r + (x - sum);
+#pragma unroll
+            for (uint32_t k = 0; k < CPL; k++) {
+                if (c0 + k < G) {
+                    st_relaxed_u64(&W.hbase[(size_t)sa * G + c0 + k], ((unsigned long long)epoch << 33) | run);
+                    if (h[k]) col[c0 + k] = 0;   // re-arm for the next batch of this parity
+                }
+                run += h[k];
+            }
+            if (q == 0) {
+                T.seq_prev[sa] = old_r;
+                const uint32_t room = 0xffffffffu - old_r;
+                T.seq[sa] = old_r + (tot < room ? tot : room);
+            }
         }
     }
-#pragma unroll
-    for (uint32_t r = 0; r < MR; r++) {
-        const uint32_t sa = slot + r * nslots;
-        if (sa >= T.n_sa) break;
-        uint16_t *col = W.hist16 + (size_t)sa * G;
-        uint32_t carry = 0;
-#pragma unroll
-        for (uint32_t u = 0; u < U; u++) {
-            uint32_t x = h[r][u];
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-                if (lane >= (uint32_t)o) x += y;
-            }
-            const uint32_t t = 32u * u + lane;
-            if (t < G) {
-                st_relaxed_u64(&W.hbase[(size_t)sa * G + t],
-                               ((unsigned long long)epoch << 33) |
-                                   ((unsigned long long)old[r] + carry + x - h[r][u]));
-                if (h[r][u]) col[t] = 0;           // re-arm for the next batch of this parity
-            }
-            carry += __shfl_sync(0xffffffffu, x, 31);
-        }
-        if (lane == 0) {
-            T.seq_prev[sa] = old[r];
-            const uint32_t room = 0xffffffffu - old[r];
-            T.seq[sa] = old[r] + (carry < room ? carry : room);
-        }
-    }
-    // rows beyond MR per warp (more SAs than 4 x 2 x CTAs): the generic scan
-    for (uint32_t sa = slot + MR * nslots; sa < T.n_sa; sa += nslots)
-        scan_sa_column<true>(T, W, sa, G, lane, epoch);
 }
 
 // LPT placement of nruns runs (costs in lanes 0..nruns-1) onto the four SM
@@ -833,6 +829,7 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
         L.pstat[1] = st_max;
     }
     bar_sync_n(1, PIPE_P);
+    if (tr && pt == 0) tr[8] = gtimer();
     if (pt == 32) {     // the second prologue warp adds its share
         L.pstat[0] += st_sum;
         L.pstat[1] = max(L.pstat[1], st_max);
@@ -877,6 +874,7 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
                 if (L.info[j] & INFO_OK) L.seq[j] += L.hmask[L.perm[j]];
         }
         bar_sync_n(1, PIPE_P);
+        if (tr && pt == 0) tr[9] = gtimer();
     }
 #else
     // 2. stable CTA-local ranks: rounds of 64 packets in index order, within a
@@ -934,6 +932,7 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
         L.bins[lane] = x - cb;
     }
     bar_sync_n(1, PIPE_P);
+    if (tr && pt == 0) tr[10] = gtimer();
     for (uint32_t r = 0; r < rounds; r++) {
         const uint32_t j = r * PIPE_P + pt;
         const uint32_t info = j < cnt ? L.info[j] : 0u;
@@ -942,6 +941,7 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
         if (j < cnt) L.perm[pos] = (uint16_t)j;
     }
     bar_sync_n(1, PIPE_P);                      // count-matrix writes done, bins read
+    if (tr && pt == 0) tr[11] = gtimer();
     if (pt < NBINS) L.bins[pt] = 0u;
     if (pt == 0) {
         // round keys before the scans / polls (their latency overlaps) pays for
@@ -981,6 +981,7 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
         W.pvote[(size_t)parity * G + cta] = ((unsigned long long)epoch << 1) | vote;
     }
 #endif
+    if (tr && pt == 0) tr[12] = gtimer();
     if (pt == 0)
         asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&W.ctl[CTL_BAR_MONO]) : "memory");
     if (tr && pt == 0) tr[4] = gtimer();   // (trace variant: tr = this iteration's stamps)
@@ -1258,7 +1259,8 @@ cudaError_t launch_fused_ring_pipe(const DevTable &T, const DevWork &W, const Ba
 
 bool fused_pipe_ok(uint32_t n, int grid)
 {
-    return n > 0 && fused_ppc(n, grid) <= PIPE_MAX_PPC;
+    // pipe_scan_rows covers rows of up to 8 x 20 = 160 CTAs
+    return n > 0 && grid <= 160 && fused_ppc(n, grid) <= PIPE_MAX_PPC;
 }
 
 int fused_grid(int num_sms) { return num_sms; }

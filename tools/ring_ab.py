@@ -42,15 +42,17 @@ for size in %(sizes)r:
     ring.run_batches(max(40, 4 * R)); torch.cuda.synchronize()
     if %(trace)r:
         G = 148
-        ts = torch.zeros(K * G * 8, dtype=torch.int64, device="cuda")
+        ts = torch.zeros(K * G * 16, dtype=torch.int64, device="cuda")
         ring.set_timestamps(ts)
         ring.run_batches(K); torch.cuda.synchronize()
-        v = ts.cpu().numpy().reshape(K, G, 8).astype(np.int64)[2:]     # skip start-up
+        v = ts.cpu().numpy().reshape(K, G, 16).astype(np.int64)[2:]    # skip start-up
         rel = (v - v[:, :, :1]) / 1e3
         names = ["start", "barrier_seen", "polls_done", "lanes_done", "prologue_arrived",
-                 "iter_end", "early_keys_done", "pseq_polls_done"]
-        med = {n: float(np.median(rel[:, :, i])) for i, n in enumerate(names) if i}
-        p90 = {n: float(np.percentile(rel[:, :, i], 90)) for i, n in enumerate(names) if i}
+                 "iter_end", "early_keys_done", "pseq_polls_done", "pro_meta", "pro_ranked",
+                 "pro_counts", "pro_perm", "pro_lpt"]
+        ok = lambda i: bool(np.all(v[:, :, i] > 0))
+        med = {n: round(float(np.median(rel[:, :, i])), 2) for i, n in enumerate(names) if i and ok(i)}
+        p90 = {n: round(float(np.percentile(rel[:, :, i], 90)), 2) for i, n in enumerate(names) if i and ok(i)}
         it = np.diff(v[:, 0, 0]) / 1e3
         out[str(size)] = {"median_us": med, "p90_us": p90, "iter_us": float(np.median(it))}
     else:
