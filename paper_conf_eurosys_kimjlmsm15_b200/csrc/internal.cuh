@@ -470,49 +470,6 @@ __device__ __forceinline__ void scan_sa_column(const DevTable &T, const DevWork 
     }
 }
 
-// One SA row of at most 160 tiles by one warp, lane-parallel: lane l owns
-// tiles 5 l .. 5 l + 4, sums them in registers, and one 5-step shuffle scan
-// gives its starting prefix (one memory round trip, one shuffle chain -- the
-// warp-per-32-tiles loop above chains a 5-step scan per 32 tiles).  Same
-// results as scan_sa_column.
-template <bool BASE>
-__device__ __forceinline__ void scan_sa_row_lanes(const DevTable &T, const DevWork &W, uint32_t sa,
-                                                  uint32_t n_tiles, uint32_t lane, uint32_t epoch,
-                                                  bool have_pre = false, uint32_t old_pre = 0)
-{
-    constexpr uint32_t CPL = 5;
-    uint16_t *col = W.hist16 + (size_t)sa * n_tiles;
-    const uint32_t c0 = lane * CPL;
-    const uint32_t old = have_pre ? old_pre : __shfl_sync(0xffffffffu, lane == 0 ? T.seq[sa] : 0u, 0);
-    uint32_t h[CPL], sum = 0;
-#pragma unroll
-    for (uint32_t k = 0; k < CPL; k++) {
-        h[k] = c0 + k < n_tiles ? (uint32_t)__ldcg(&col[c0 + k]) : 0u;
-        sum += h[k];
-    }
-    uint32_t x = sum;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
-        if (lane >= (uint32_t)o) x += y;
-    }
-    const uint32_t tot = __shfl_sync(0xffffffffu, x, 31);
-    uint32_t run = x - sum;
-#pragma unroll
-    for (uint32_t k = 0; k < CPL; k++) {
-        if (c0 + k < n_tiles) {
-            put_prefix<BASE>(W, (size_t)sa * n_tiles + c0 + k, run, old, epoch);
-            if (h[k]) col[c0 + k] = 0;           // re-arm for the next batch
-        }
-        run += h[k];
-    }
-    if (lane == 0) {
-        T.seq_prev[sa] = old;
-        const uint32_t room = 0xffffffffu - old;
-        T.seq[sa] = old + (tot < room ? tot : room);
-    }
-}
-
 // The SA counter this warp's first row scan starts from (scan_all_columns with
 // have_pre): T.seq of row `slot` (warp-per-row) or of row slot + lane * nslots
 // (lane-per-row).  Only that scan writes T.seq of the row, so the value may be
@@ -533,11 +490,6 @@ __device__ __forceinline__ void scan_all_columns(const DevTable &T, const DevWor
                                                  uint32_t epoch = 0, bool have_pre = false,
                                                  uint32_t old_pre = 0)
 {
-    if (n_tiles > 32u && n_tiles <= 160u) {
-        for (uint32_t col = slot; col < T.n_sa; col += nslots)
-            scan_sa_row_lanes<BASE>(T, W, col, n_tiles, lane, epoch, have_pre && col == slot, old_pre);
-        return;
-    }
     if (n_tiles > 32u) {
         for (uint32_t col = slot; col < T.n_sa; col += nslots)
             scan_sa_column<BASE>(T, W, col, n_tiles, lane, epoch, have_pre && col == slot, old_pre);

@@ -45,7 +45,7 @@ for size in %(sizes)r:
         ts = torch.zeros(K * G * 16, dtype=torch.int64, device="cuda")
         ring.set_timestamps(ts)
         ring.run_batches(K); torch.cuda.synchronize()
-        v = ts.cpu().numpy().reshape(K, G, 16).astype(np.int64)[2:]    # skip start-up
+        v = ts.cpu().numpy().reshape(K, G, 16).astype(np.int64)[2:-1]  # skip start-up, last
         rel = (v - v[:, :, :1]) / 1e3
         names = ["start", "barrier_seen", "polls_done", "lanes_done", "prologue_arrived",
                  "iter_end", "early_keys_done", "pseq_polls_done", "pro_meta", "pro_ranked",
