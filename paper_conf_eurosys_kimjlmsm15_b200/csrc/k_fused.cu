@@ -666,9 +666,6 @@ k_fused_ring(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint16_t 
 #define NBA_PIPE_PSCAN 0      // 0 never, 1 always, 2 when most CTAs vote the batch long,
 #endif                        // 3 always + the prologue warps poll the bases too (the next
                               //   batch's sequence numbers are ready when it starts)
-#ifndef NBA_PIPE_HALVES       // pipelined ring: the two prologue warps rank halves concurrently
-#define NBA_PIPE_HALVES 1
-#endif
 #ifndef NBA_PIPE_LPT          // pipelined ring: LPT placement of the runs (1) or run r -> warp r
 #define NBA_PIPE_LPT 1
 #endif
@@ -776,11 +773,67 @@ __device__ __forceinline__ uint32_t lpt_place(uint32_t cost, uint32_t nruns, uin
     return mine;
 }
 
+// The packet metadata of this prologue thread (packets j = r * 64 + pt of the
+// CTA's range, r < 7), all loads issued together.
+constexpr uint32_t PR = PIPE_MAX_PPC / PIPE_P;                      // 7 rounds
+struct PipeMeta {
+    uint32_t D[PR], S[PR], I[PR], O[PR];
+};
+
+__device__ __forceinline__ void pipe_load_meta(const BatchArgs &B, uint32_t ppc, uint32_t pt, PipeMeta &m)
+{
+    const uint32_t p_begin = blockIdx.x * ppc;
+    const uint32_t p_end = min(B.n, p_begin + ppc);
+    const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
+#pragma unroll
+    for (uint32_t r = 0; r < PR; r++) {
+        const uint32_t j = r * PIPE_P + pt;
+        const uint32_t i = p_begin + j;
+        m.D[r] = j < cnt ? B.in_len[i] : 0u;
+        m.S[r] = j < cnt ? B.sa_idx[i] : INVALID_SA;
+        m.I[r] = j < cnt ? B.in_off[i] : 0u;
+        m.O[r] = j < cnt ? B.out_off[i] : 0u;
+    }
+}
+
+// L2 prefetch of a batch's metadata lines for this CTA (in_len, sa_idx,
+// in_off, out_off of its packet range) by the 64 prologue threads: issued two
+// batches ahead, so the prologue's metadata loads hit L2 (the ring's slots
+// rotate through more than the L2, the arrays are DRAM-cold otherwise).
+__device__ __forceinline__ void pipe_prefetch_meta(const BatchArgs &B, uint32_t ppc, uint32_t pt)
+{
+    const uint32_t p_begin = blockIdx.x * ppc;
+    const uint32_t p_end = min(B.n, p_begin + ppc);
+    if (p_end <= p_begin) return;
+    const uint32_t cnt = p_end - p_begin;
+    // lines of the four arrays: 2-byte and 4-byte elements, <= 448 packets
+    const uint32_t l16 = (2u * cnt + 127u) / 128u + 1u, l32 = (4u * cnt + 127u) / 128u + 1u;
+    const uint32_t tot = l16 + 3u * l32;
+    for (uint32_t k = pt; k < tot; k += PIPE_P) {
+        const uint8_t *a;
+        if (k < l16) {
+            a = reinterpret_cast<const uint8_t *>(B.in_len + p_begin) + 128u * k;
+            if (a >= reinterpret_cast<const uint8_t *>(B.in_len + p_end)) continue;
+        } else {
+            const uint32_t q = (k - l16) / l32, m = (k - l16) % l32;
+            const uint32_t *base = q == 0 ? B.sa_idx : q == 1 ? B.in_off : B.out_off;
+            a = reinterpret_cast<const uint8_t *>(base + p_begin) + 128u * m;
+            if (a >= reinterpret_cast<const uint8_t *>(base + p_end)) continue;
+        }
+        prefetch_l2(a);
+    }
+}
+
+#ifndef NBA_PIPE_DIRECT       // pipelined ring: per-SA counts in arrays indexed by the SA
+#define NBA_PIPE_DIRECT 1     //   (n_sa <= 1024: no hash probing, no atomics) instead of the hash
+#endif
+constexpr uint32_t PIPE_DIRECT_MAX_SA = 2u * F_SUPER;              // 1024 (the hash arrays' size)
+
 // Prologue of one batch by the 64 prologue threads (pt = 0..63) of this CTA.
 __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &W, const BatchArgs &B,
                                               uint32_t ppc, uint32_t bar_target, uint32_t epoch,
                                               FusedLo &L, uint32_t pt, uint32_t parity,
-                                              unsigned long long *tr = nullptr)
+                                              const PipeMeta &m, unsigned long long *tr = nullptr)
 {
     const uint32_t G = gridDim.x, cta = blockIdx.x, n_sa = T.n_sa;
     const uint32_t lane = pt & 31u, pw = pt >> 5;
@@ -788,37 +841,24 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
     const uint32_t p_end = min(B.n, p_begin + ppc);
     const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
     const uint32_t rounds = (cnt + PIPE_P - 1u) / PIPE_P;
-    // 1. metadata (all loads issued together: one memory latency), validity,
-    //    length bins (counts)
-    constexpr uint32_t PR = PIPE_MAX_PPC / PIPE_P;                  // 7 rounds
-    uint32_t mD[PR], mS[PR], mI[PR], mO[PR];
-#pragma unroll
-    for (uint32_t r = 0; r < PR; r++) {
-        const uint32_t j = r * PIPE_P + pt;
-        const uint32_t i = p_begin + j;
-        mD[r] = j < cnt ? B.in_len[i] : 0u;
-        mS[r] = j < cnt ? B.sa_idx[i] : INVALID_SA;
-        mI[r] = j < cnt ? B.in_off[i] : 0u;
-        mO[r] = j < cnt ? B.out_off[i] : 0u;
-    }
+    const bool direct = NBA_PIPE_DIRECT && n_sa <= PIPE_DIRECT_MAX_SA;
+    // 1. metadata (loaded by pipe_load_meta), validity, length bins (counts)
     uint32_t st_sum = 0, st_max = 0;   // AES steps of the valid packets
 #pragma unroll
     for (uint32_t r = 0; r < PR; r++) {
         const uint32_t j = r * PIPE_P + pt;
         uint32_t bin = NBINS - 1;
         if (j < cnt) {
-            const bool cand = mS[r] < n_sa && mD[r] >= MIN_D && mD[r] <= MAX_D;
-            if (cand) {
-                const uint32_t stp = (esp_C(mD[r]) + 63u) >> 6;
-                st_sum += stp;
-                st_max = max(st_max, stp);
-            }
-            L.sa[j] = mS[r];
-            L.info[j] = cand ? (mD[r] | INFO_OK) : 0u;
-            L.inoff[j] = mI[r];
-            L.outoff[j] = mO[r];
-            bin = hmac_bin(cand, esp_C(mD[r]));
-            if (cand) prefetch_bytes(B.in_buf + mI[r], min(64u, mD[r]));   // the lane reads it next round
+            const bool cand = m.S[r] < n_sa && m.D[r] >= MIN_D && m.D[r] <= MAX_D;
+            const uint32_t stp = cand ? (esp_C(m.D[r]) + 63u) >> 6 : 0u;
+            st_sum += stp;
+            st_max = max(st_max, stp);
+            L.sa[j] = m.S[r];
+            L.info[j] = cand ? (m.D[r] | INFO_OK) : 0u;
+            L.inoff[j] = m.I[r];
+            L.outoff[j] = m.O[r];
+            bin = hmac_bin(cand, esp_C(m.D[r]));
+            if (cand) prefetch_bytes(B.in_buf + m.I[r], min(64u, m.D[r]));   // the lane reads it next round
         }
         if (r < rounds) warp_agg_add(L.bins, bin, j < cnt);
     }
@@ -834,15 +874,15 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
         L.pstat[0] += st_sum;
         L.pstat[1] = max(L.pstat[1], st_max);
     }
-#if NBA_PIPE_HALVES
     // 2. stable CTA-local ranks: prologue warp w ranks its half of the packets
-    //    (rounds of 32 in index order) with its own running count per SA slot
-    //    (warp 0: L.hmask, warp 1: cnt1), concurrently; warp 1's ranks then
+    //    (rounds of 32 in index order) with its own running count per SA
+    //    (direct: arrays indexed by the SA -- warp 0 L.hmask, warp 1 cnt1 --;
+    //    else per slot of the CTA's SA hash), concurrently; warp 1's ranks then
     //    add warp 0's final count of the SA
-    uint32_t *cnt1 = &L.aux0[0];                 // aux0 | aux1: 1024 slot counts (outbound only)
+    uint32_t *cnt1 = &L.aux0[0];                 // aux0 | aux1: 1024 counts (outbound only)
+    const uint32_t half = ((cnt + 1u) / 2u + 31u) & ~31u;
+    const uint32_t j0 = pw ? half : 0u, j1 = pw ? cnt : min(cnt, half);
     {
-        const uint32_t half = ((cnt + 1u) / 2u + 31u) & ~31u;
-        const uint32_t j0 = pw ? half : 0u, j1 = pw ? cnt : min(cnt, half);
         uint32_t *cw = pw ? cnt1 : L.hmask;
         for (uint32_t jb = j0; jb < j1; jb += 32u) {
             const uint32_t j = jb + lane;
@@ -850,79 +890,68 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
             const uint32_t s = act ? L.sa[j] : INVALID_SA;
             const uint32_t peers = __match_any_sync(0xffffffffu, s);
             const uint32_t leader = __ffs(peers) - 1;
-            uint32_t base = 0, slot = 0;
+            uint32_t base = 0, slot = s;
             if (act && lane == leader) {
-                slot = (s * 0x9E3779B1u) >> 22;          // 1024 slots
-                while (true) {
-                    const uint32_t old = atomicCAS(&L.hkey[slot], INVALID_SA, s);
-                    if (old == INVALID_SA || old == s) break;
-                    slot = (slot + 1u) & (2u * F_SUPER - 1u);
-                }
-                base = cw[slot];
-                cw[slot] = base + (uint32_t)__popc(peers);
-            }
-            base = __shfl_sync(0xffffffffu, base, leader);
-            slot = __shfl_sync(0xffffffffu, slot, leader);
-            if (j < j1) {
-                L.seq[j] = act ? base + (uint32_t)__popc(peers & lanemask_lt()) : 0u;
-                if (pw) L.perm[j] = (uint16_t)slot;     // (perm is rebuilt in step 3)
-            }
-        }
-        bar_sync_n(1, PIPE_P);
-        if (pw) {
-            for (uint32_t j = j0 + lane; j < j1; j += 32u)
-                if (L.info[j] & INFO_OK) L.seq[j] += L.hmask[L.perm[j]];
-        }
-        bar_sync_n(1, PIPE_P);
-        if (tr && pt == 0) tr[9] = gtimer();
-    }
-#else
-    // 2. stable CTA-local ranks: rounds of 64 packets in index order, within a
-    //    round prologue warp 0 (the lower 32 packets) before warp 1
-    for (uint32_t r = 0; r < rounds; r++) {
-#pragma unroll 1
-        for (uint32_t w = 0; w < 2u; w++) {
-            if (pw == w) {
-                const uint32_t j = r * PIPE_P + 32u * w + lane;
-                const bool act = j < cnt && (L.info[j] & INFO_OK);
-                const uint32_t s = act ? L.sa[j] : INVALID_SA;
-                const uint32_t peers = __match_any_sync(0xffffffffu, s);
-                const uint32_t leader = __ffs(peers) - 1;
-                uint32_t base = 0;
-                if (act && lane == leader) {
-                    uint32_t slot = (s * 0x9E3779B1u) >> 22;      // 1024 slots
+                if (!direct) {
+                    slot = (s * 0x9E3779B1u) >> 22;          // 1024 slots
                     while (true) {
                         const uint32_t old = atomicCAS(&L.hkey[slot], INVALID_SA, s);
                         if (old == INVALID_SA || old == s) break;
                         slot = (slot + 1u) & (2u * F_SUPER - 1u);
                     }
-                    base = L.hmask[slot];                      // running count of the SA
-                    L.hmask[slot] = base + (uint32_t)__popc(peers);
                 }
-                base = __shfl_sync(0xffffffffu, base, leader);
-                if (j < cnt) L.seq[j] = act ? base + (uint32_t)__popc(peers & lanemask_lt()) : 0u;
+                base = cw[slot];
+                cw[slot] = base + (uint32_t)__popc(peers);
             }
-            bar_sync_n(1, PIPE_P);
+            base = __shfl_sync(0xffffffffu, base, leader);
+            if (!direct) slot = __shfl_sync(0xffffffffu, slot, leader);
+            if (j < j1) {
+                L.seq[j] = act ? base + (uint32_t)__popc(peers & lanemask_lt()) : 0u;
+                if (pw && !direct) L.perm[j] = (uint16_t)slot;     // (perm is rebuilt in step 3)
+            }
+        }
+        bar_sync_n(1, PIPE_P);
+        if (pw) {
+            for (uint32_t j = j0 + lane; j < j1; j += 32u)
+                if (L.info[j] & INFO_OK) L.seq[j] += L.hmask[direct ? L.sa[j] : L.perm[j]];
+        }
+        bar_sync_n(1, PIPE_P);
+        if (tr && pt == 0) tr[9] = gtimer();
+    }
+    // 3. this CTA's per-SA counts -> count matrix (nonzero only) and the
+    //    counters cleared for the next batch: direct -- the SA's last packet in
+    //    the CTA (rank = count - 1) writes it; hash -- a sweep over the slots.
+    //    Length order: exclusive scan of the bins, positions, bins re-zeroed;
+    //    a batch whose packets all share one bin keeps index order.
+    uint32_t owner = 0;                          // direct: rounds whose packet is its SA's last
+    if (direct) {
+#pragma unroll
+        for (uint32_t r = 0; r < PR; r++) {
+            const uint32_t j = r * PIPE_P + pt;
+            if (j < cnt && (L.info[j] & INFO_OK)) {
+                const uint32_t s = L.sa[j];
+                const uint32_t tot = L.hmask[s] + cnt1[s];
+                if (L.seq[j] + 1u == tot) {
+                    W.hist16[(size_t)s * G + cta] = (uint16_t)tot;
+                    owner |= 1u << r;            // clears the counters after the barrier
+                }
+            }
+        }
+    } else {
+        for (uint32_t k = pt; k < 2u * F_SUPER; k += PIPE_P) {
+            const uint32_t s = L.hkey[k];
+            if (s != INVALID_SA) {
+                W.hist16[(size_t)s * G + cta] = (uint16_t)(L.hmask[k] + cnt1[k]);
+                cnt1[k] = 0u;
+                L.hkey[k] = INVALID_SA;
+                L.hmask[k] = 0u;
+            }
         }
     }
-#endif
-    // 3. this CTA's per-SA counts -> count matrix (nonzero only); clear the hash.
-    //    Length order: exclusive scan of the bins, positions, bins re-zeroed.
-    for (uint32_t k = pt; k < 2u * F_SUPER; k += PIPE_P) {
-        const uint32_t s = L.hkey[k];
-        if (s != INVALID_SA) {
-#if NBA_PIPE_HALVES
-            W.hist16[(size_t)s * G + cta] = (uint16_t)(L.hmask[k] + cnt1[k]);
-            cnt1[k] = 0u;
-#else
-            W.hist16[(size_t)s * G + cta] = (uint16_t)L.hmask[k];
-#endif
-            L.hkey[k] = INVALID_SA;
-            L.hmask[k] = 0u;
-        }
-    }
+    bool one_bin = false;
     if (pw == 0) {
         const uint32_t cb = L.bins[lane];
+        one_bin = __any_sync(0xffffffffu, cb == cnt);
         uint32_t x = cb;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
@@ -930,11 +959,25 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
             if (lane >= (uint32_t)o) x += y;
         }
         L.bins[lane] = x - cb;
+        if (lane == 0) L.pstat[2] = one_bin ? 4u : 0u;     // bit 2: one length bin
     }
     bar_sync_n(1, PIPE_P);
     if (tr && pt == 0) tr[10] = gtimer();
+#pragma unroll
+    for (uint32_t r = 0; r < PR; r++) {          // every total was read: clear for the next batch
+        if ((owner >> r) & 1u) {
+            const uint32_t s = L.sa[r * PIPE_P + pt];
+            L.hmask[s] = 0u;
+            cnt1[s] = 0u;
+        }
+    }
+    one_bin = (L.pstat[2] & 4u) != 0u;
     for (uint32_t r = 0; r < rounds; r++) {
         const uint32_t j = r * PIPE_P + pt;
+        if (one_bin) {                           // counting sort of one bin = index order
+            if (j < cnt) L.perm[j] = (uint16_t)j;
+            continue;
+        }
         const uint32_t info = j < cnt ? L.info[j] : 0u;
         const uint32_t bin = hmac_bin((info & INFO_OK) != 0u, esp_C(info & 0x7ffu));
         const uint32_t pos = warp_agg_add(L.bins, bin, j < cnt);
@@ -948,7 +991,7 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
         // long or length-divergent batches; for uniform short ones after
         // (measured: 64 B 23.5 vs 24.1 us, IMIX 96.8 vs 90.4, 1514 B 193.7 vs 192.3)
         const uint32_t sum = L.pstat[0], mx = L.pstat[1], nv = cnt ? cnt : 1u;
-        L.pstat[2] = (mx * nv > 2u * sum || sum >= 8u * nv) ? 1u : 0u;
+        L.pstat[2] = (mx * nv > 2u * sum || sum >= 8u * nv) ? 1u : 0u;   // (clears bit 2)
     }
     if (pw == 0 && !NBA_PIPE_LPT) {
         if (lane < PIPE_LANE_WARPS) L.wrun[lane] = (uint8_t)lane;   // run r -> warp r
@@ -1127,8 +1170,14 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
         return Wb;
     };
     if (isP) {
+        if (n_batches > 1) {
+            const BatchArgs B1 = slots[(first + 1) % n_slots];
+            pipe_prefetch_meta(B1, fused_ppc(B1.n, G), pt);
+        }
         const BatchArgs B0 = slots[first % n_slots];
-        pipe_prologue(T, work_of(0), B0, fused_ppc(B0.n, G), base0 + G, epoch_of(0), L, pt, 0u);
+        PipeMeta meta;
+        pipe_load_meta(B0, fused_ppc(B0.n, G), pt, meta);
+        pipe_prologue(T, work_of(0), B0, fused_ppc(B0.n, G), base0 + G, epoch_of(0), L, pt, 0u, meta);
     }
     __syncthreads();
     // the T-table image landed (the bulk copy overlapped the first prologue);
@@ -1169,6 +1218,9 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
 #if NBA_RING_TRACE
             if (lane == 0 && R.ts) atomicMax(RTR(bi, 6), gtimer());
 #endif
+        } else if (bi + 2 < n_batches) {
+            const BatchArgs B2 = slots[(first + bi + 2) % n_slots];
+            pipe_prefetch_meta(B2, fused_ppc(B2.n, G), pt);      // two batches ahead, into L2
         }
 #if NBA_RING_TRACE
         pipe_sequence(T, work_of(bi), B, ppc, base0 + (bi + 1) * G, epoch_of(bi), L, RTR(bi, 0));
@@ -1205,12 +1257,14 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
             bar_sync_n(2, F_THREADS);                    // every lane took its fields
             if (bi + 1 < n_batches) {
                 const BatchArgs Bn = slots[(first + bi + 1) % n_slots];
+                PipeMeta meta;
+                pipe_load_meta(Bn, fused_ppc(Bn.n, G), pt, meta);
 #if NBA_RING_TRACE
                 pipe_prologue(T, work_of(bi + 1), Bn, fused_ppc(Bn.n, G), base0 + (bi + 2) * G,
-                              epoch_of(bi + 1), L, pt, (bi + 1) & 1u, RTR(bi, 0));
+                              epoch_of(bi + 1), L, pt, (bi + 1) & 1u, meta, RTR(bi, 0));
 #else
                 pipe_prologue(T, work_of(bi + 1), Bn, fused_ppc(Bn.n, G), base0 + (bi + 2) * G,
-                              epoch_of(bi + 1), L, pt, (bi + 1) & 1u);
+                              epoch_of(bi + 1), L, pt, (bi + 1) & 1u, meta);
 #endif
             }
         }
