@@ -222,6 +222,8 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
         line[3] = hm[(size_t)s * 3 + 1];
         line[4] = hm[(size_t)s * 3 + 2];
         line[5] = make_uint4(hout[0], hout[1], hout[2], 0u);   // words 4..5 = hout[3,4,-,-,0,1,2]
+        line[6] = rk[(size_t)s * 11 + 1];                        // round keys 1, 2 (CTR precompute)
+        line[7] = rk[(size_t)s * 11 + 2];
     }
     t->seq0 = seq;
 

@@ -527,6 +527,29 @@ __device__ __forceinline__ void expand_key_lane(uint32_t lane4r, const uint4 &r0
     }
 }
 
+// Round keys 3..10 of the lane's SA (FIPS-197 §5.2 schedule, built once per
+// SA at setup, DevTable::rk) copied global -> the lane's own shared-memory
+// slots L.rkA / H.rkB[.][tid] by cp.async (LDGSTS, 8 x 16 bytes, one commit
+// group): issued before the batch's barrier wait / scans / polls, whose
+// latency hides the copy; rk_async_wait() before the first AES round.  The
+// lane's own copies only, so no CTA barrier is involved.
+__device__ __forceinline__ void rk_async_issue(const uint4 *rk, uint32_t sa, FusedLo &L, FusedHi &H,
+                                               uint32_t tid)
+{
+    const uint4 *src = rk + (size_t)sa * 11u + 3u;
+#pragma unroll
+    for (uint32_t r = 0; r < 8u; r++) {
+        const uint32_t dst = r < 4u ? smem_u32(&L.rkA[r][tid]) : smem_u32(&H.rkB[r - 4u][tid]);
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src + r) : "memory");
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+}
+
+__device__ __forceinline__ void rk_async_wait()
+{
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
+}
+
 // Warp-cooperative, coalesced staging of round keys 3..10 of each lane's SA
 // (sa_me; INVALID_SA = none) into L.rkA / H.rkB: load m of the warp covers 128
 // contiguous bytes of 4 lanes' SAs.  Followed by __syncwarp in the caller.

@@ -55,6 +55,9 @@ namespace nba {
 #ifndef NBA_STG256            // 1: output through 32-byte chunks (256-bit stores)
 #define NBA_STG256 0
 #endif
+#ifndef NBA_RK_ASYNC          // pipelined ring: round keys 3..10 by cp.async from the SA's
+#define NBA_RK_ASYNC 1        //   schedule (1) instead of expanded in the lane (0)
+#endif
 #ifndef NBA_SA_PREFETCH       // L2 prefetch of the SA table at kernel start
 #define NBA_SA_PREFETCH 1
 #endif
@@ -825,7 +828,7 @@ __device__ __forceinline__ void pipe_prefetch_meta(const BatchArgs &B, uint32_t 
 }
 
 #ifndef NBA_PIPE_DIRECT       // pipelined ring: per-SA counts in arrays indexed by the SA
-#define NBA_PIPE_DIRECT 1     //   (n_sa <= 1024: no hash probing, no atomics) instead of the hash
+#define NBA_PIPE_DIRECT 0     //   (n_sa <= 1024: no hash probing; measured slower under the lanes' load) instead of the hash
 #endif
 constexpr uint32_t PIPE_DIRECT_MAX_SA = 2u * F_SUPER;              // 1024 (the hash arrays' size)
 
@@ -1211,7 +1214,13 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
             sa = (info & INFO_OK) ? L.sa[pk] : INVALID_SA;
             inoff = have ? L.inoff[pk] : 0u;
             outoff = have ? L.outoff[pk] : 0u;
-            if (early && (info & INFO_OK)) {
+            if (NBA_RK_ASYNC && (info & INFO_OK)) {
+                // round keys by cp.async and the SA line (with round keys 1, 2):
+                // in flight during the barrier wait / scans / polls
+                rk_async_issue(T.rk, sa, L, H, tid);
+                pp = load_pkt_pre(T, B.in_buf, sa, inoff, true, 0u);
+                ldg_nc_v8(&T.sal[(size_t)sa * SAL_U4 + 6], pp.r1, pp.r2);
+            } else if (early && (info & INFO_OK)) {
                 pp = load_pkt_pre(T, B.in_buf, sa, inoff, true, 0u);
                 expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
             }
@@ -1232,8 +1241,9 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
             bar_arrive_n(2, F_THREADS);                  // fields taken: the arrays are free
             if (have) {
                 const uint32_t pkt = p_begin + pk;
+                if (NBA_RK_ASYNC && (info & INFO_OK)) rk_async_wait();   // (dropped ones too)
                 if ((info & INFO_OK) && q32 != 0u) {
-                    if (!early) {
+                    if (!NBA_RK_ASYNC && !early) {
                         pp = load_pkt_pre(T, B.in_buf, sa, inoff, true, 0u);
                         expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
                     }

@@ -356,3 +356,38 @@ def test_run_batches_mid_rotation(graph, monkeypatch):
         assert np.array_equal(t.sa_seq(), oracle.sa_seq(sas, n_sa))
         assert t.counters() == ctr.as_dict()
         ring.close()
+
+
+@pytest.mark.parametrize("n_sa,sizes", [(2500, (64, "imix")), (1024, (300, 300)), (1, (64, 1514))])
+def test_pipelined_prologue_modes(n_sa, sizes):
+    """The pipelined ring's prologue with the SA hash (n_sa > 1024), with
+    per-SA counters indexed by the SA (one SA; 1024 SAs), one-length-bin
+    batches (all packets one size: index order kept) and mixed ones; some
+    invalid SAs and lengths; 4 runs of 2-3 batches against the oracle."""
+    import torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    n = 30000
+    p = gen.make_sas(n_sa, cfg_id=58)
+    hb = [gen.make_batch(n, s, n_sa, cfg_id=58, batch=i) for i, s in enumerate(sizes)]
+    hb[1].sa_idx[::101] = n_sa + 3
+    hb[1].in_len[5::203] = 19
+    sas = oracle.make_sas(p)
+    ctr = oracle.Counters()
+    with nba_ipsec.SATable(p, device=0, max_batch=n) as t:
+        dbs = [device.to_device(b, "cuda") for b in hb]
+        ring = t.ring([_slot(d) for d in dbs])
+        assert ring.form == nba_ipsec.Ring.PIPELINED
+        last, k = {}, 0
+        for nb in (3, 2, 3, 2):
+            ring.run_batches(nb)
+            for _ in range(nb):
+                o_out, o_len, _ = oracle.process_batch(sas, n_sa, hb[k % 2], n_threads=8, counters=ctr)
+                last[k % 2] = (o_out, o_len.copy())
+                k += 1
+        for s, (o_out, o_len) in last.items():
+            g_out, g_len = device.fetch(dbs[s])
+            assert np.array_equal(g_len, o_len)
+            assert np.array_equal(g_out, o_out)
+        assert np.array_equal(t.sa_seq(), oracle.sa_seq(sas, n_sa))
+        assert t.counters() == ctr.as_dict()
+        ring.close()
