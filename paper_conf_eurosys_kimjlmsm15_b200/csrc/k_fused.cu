@@ -56,7 +56,13 @@ namespace nba {
 #define NBA_STG256 0
 #endif
 #ifndef NBA_RK_ASYNC          // pipelined ring: round keys 3..10 by cp.async from the SA's
-#define NBA_RK_ASYNC 1        //   schedule (1) instead of expanded in the lane (0)
+#define NBA_RK_ASYNC 0        //   schedule (1) instead of expanded in the lane (0); measured
+#endif                        //   slower (64 B 24.4 -> 27.5 us: the LDGSTS issue delays the scans)
+#ifndef NBA_PIPE_ONEBIN       // pipelined ring: one-length-bin batches keep index order (no sort)
+#define NBA_PIPE_ONEBIN 1
+#endif
+#ifndef NBA_PIPE_META_PF      // pipelined ring: L2 prefetch of the metadata two batches ahead
+#define NBA_PIPE_META_PF 1
 #endif
 #ifndef NBA_SA_PREFETCH       // L2 prefetch of the SA table at kernel start
 #define NBA_SA_PREFETCH 1
@@ -974,7 +980,7 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
             cnt1[s] = 0u;
         }
     }
-    one_bin = (L.pstat[2] & 4u) != 0u;
+    one_bin = NBA_PIPE_ONEBIN && (L.pstat[2] & 4u) != 0u;
     for (uint32_t r = 0; r < rounds; r++) {
         const uint32_t j = r * PIPE_P + pt;
         if (one_bin) {                           // counting sort of one bin = index order
@@ -1173,7 +1179,7 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
         return Wb;
     };
     if (isP) {
-        if (n_batches > 1) {
+        if (NBA_PIPE_META_PF && n_batches > 1) {
             const BatchArgs B1 = slots[(first + 1) % n_slots];
             pipe_prefetch_meta(B1, fused_ppc(B1.n, G), pt);
         }
@@ -1227,7 +1233,7 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
 #if NBA_RING_TRACE
             if (lane == 0 && R.ts) atomicMax(RTR(bi, 6), gtimer());
 #endif
-        } else if (bi + 2 < n_batches) {
+        } else if (NBA_PIPE_META_PF && bi + 2 < n_batches) {
             const BatchArgs B2 = slots[(first + bi + 2) % n_slots];
             pipe_prefetch_meta(B2, fused_ppc(B2.n, G), pt);      // two batches ahead, into L2
         }

@@ -1,0 +1,6 @@
+#!/bin/bash
+TAG=${1:-r02i}
+mkdir -p gpurun_out
+python -m paper_conf_eurosys_kimjlmsm15_b200.build >/dev/null
+timeout 900 python tools/ring_ab.py run > gpurun_out/${TAG}_ring_ab.txt 2>&1; cat gpurun_out/${TAG}_ring_ab.txt
+timeout 900 python tools/inbound_ab.py > gpurun_out/${TAG}_inbound_ab.txt 2>&1; cat gpurun_out/${TAG}_inbound_ab.txt
