@@ -83,3 +83,34 @@ def test_ring_slot_count_matches_bench_rule():
 def test_bench_args_and_gpus_contract():
     a = bench.parse_args(["--gpus", "2", "--steps", "7", "--warmup", "1"])
     assert (a.gpus, a.steps, a.warmup) == (2, 7, 3)          # W >= 3
+
+
+def test_gpus_n_relaunches_under_torchrun(monkeypatch):
+    """`bench.py --gpus N` without a torchrun environment re-executes itself
+    under torch.distributed.run with one process per GPU on 127.0.0.1 (the
+    driver's form), NCCL init logging on; fewer visible GPUs fail loudly."""
+    import pytest
+    calls = []
+    monkeypatch.delenv("WORLD_SIZE", raising=False)
+    monkeypatch.setattr(bench.os, "execvpe", lambda f, argv, env: calls.append((argv, env)))
+    import torch
+    monkeypatch.setattr(torch.cuda, "device_count", lambda: 8)
+    monkeypatch.setattr(bench.sys, "argv", ["bench.py", "--gpus", "4", "--steps", "5"])
+    bench.relaunch_under_torchrun(bench.parse_args(["--gpus", "4", "--steps", "5"]))
+    argv, env = calls[0]
+    assert argv[1:3] == ["-m", "torch.distributed.run"]
+    assert "--nproc-per-node=4" in argv and "127.0.0.1" in argv
+    assert argv[-4:] == ["--gpus", "4", "--steps", "5"] and argv[-5].endswith("bench.py")
+    assert env["NCCL_DEBUG"] == "INFO"
+    monkeypatch.setattr(torch.cuda, "device_count", lambda: 1)
+    with pytest.raises(SystemExit):
+        bench.relaunch_under_torchrun(bench.parse_args(["--gpus", "4"]))
+
+
+def test_ctx_rejects_world_mismatch(monkeypatch):
+    """A rank whose WORLD_SIZE differs from --gpus refuses to run (no silent
+    single-GPU number reported as N GPUs)."""
+    import pytest
+    monkeypatch.setenv("WORLD_SIZE", "2")
+    with pytest.raises(SystemExit):
+        bench.Ctx(bench.parse_args(["--gpus", "4"]))

@@ -90,3 +90,54 @@ def test_virtual_shard_union_equals_single_oracle_cpu():
         # packets with an invalid SA belong to no shard: the rest matches
         assert tot["pkts_ok"] == ref_ctr.pkts_ok
         assert tot["bytes_out"] == ref_ctr.bytes_out
+
+
+class _GlooCtx:
+    """bench.Ctx's reduction surface on a gloo process group (CPU)."""
+
+    def max_ms(self, ms):
+        return shard.max_over_ranks(ms)
+
+    def sum_all(self, d):
+        return shard.reduce_counters(d)
+
+
+def _bench_rates_worker(rank, world, port, out_q):
+    import sys
+    import torch.distributed as dist
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import bench
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    # each rank: its own SA shard and batch (weak scaling), a different elapsed time
+    p, b = shard.rank_workload(2, 2000, 64 if rank == 0 else "imix", 64, rank, world)
+    res = {"b": b, "tot_ms": 10.0 + rank}
+    r = bench.rates(_GlooCtx(), res, steps=5)
+    out_q.put((rank, r, float(np.asarray(b.frame_len, np.float64).sum()), int(b.in_len.astype(np.int64).sum())))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_bench_rates_whole_job_over_ranks():
+    """bench.rates over 2 gloo ranks: value = all ranks' frame bits x steps /
+    the MAX elapsed time over ranks (the contract's whole-job aggregate), the
+    same on every rank; ESP-payload Gbps from the datagram bytes."""
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_bench_rates_worker, args=(r, world, port, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    res = sorted(q.get(timeout=120) for _ in range(world))
+    for pr in procs:
+        pr.join(timeout=60)
+    frames = sum(x[2] for x in res)
+    payload = sum(x[3] for x in res)
+    t = 11.0e-3                                         # max over ranks
+    for _, r, _, _ in res:
+        assert abs(r["gbps"] - 8 * frames * 5 / t / 1e9) < 1e-9
+        assert abs(r["esp_payload_gbps"] - 8 * payload * 5 / t / 1e9) < 1e-9
+        assert abs(r["mpps"] - 4000 * 5 / t / 1e6) < 1e-9
+        assert abs(r["ms_per_step"] - 11.0 / 5) < 1e-12
