@@ -1253,6 +1253,9 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
                         pp = load_pkt_pre(T, B.in_buf, sa, inoff, true, 0u);
                         expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
                     }
+#ifdef NBA_STAGGER_NS   // experiment: delay the upper lane warps (phase-locking of AES / SHA-1)
+                    if (warp >= 7u) __nanosleep(NBA_STAGGER_NS);
+#endif
                     if (!NBA_PROLOGUE_ONLY)   // (debug A/B: the ring without the lane work)
                         esp_packet(T, B, L, H, lane4r, tid, sa, info, q32, inoff, outoff, pp, nullptr);
                     const uint32_t Dp = info & 0x7ffu;
