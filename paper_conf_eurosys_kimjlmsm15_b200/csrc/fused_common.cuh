@@ -39,6 +39,8 @@ struct FusedLo {
     uint32_t pstat[3];             // pipelined ring: the next batch's AES steps (sum, max) and
                                    //   its "early round keys" decision
     unsigned long long tbar;       // mbarrier: the bulk copy of the T-table image landed
+    uint32_t stag_ns;              // pipelined ring: start delay of the upper lane warps
+    uint32_t stag_acc;             //   (AES step 0 of the lower ones, measured per batch)
 };
 
 struct FusedHi {

@@ -58,6 +58,9 @@ namespace nba {
 #ifndef NBA_RK_ASYNC          // pipelined ring: round keys 3..10 by cp.async from the SA's
 #define NBA_RK_ASYNC 0        //   schedule (1) instead of expanded in the lane (0); measured
 #endif                        //   slower (64 B 24.4 -> 27.5 us: the LDGSTS issue delays the scans)
+#ifndef NBA_PIPE_STAGGER      // pipelined ring: lane warps 7..13 start their packets later by
+#define NBA_PIPE_STAGGER 0    //   STAGGER/256 x the time the lower warps took to their first AES
+#endif                        //   step (previous batch), so AES (LDS) and SHA-1 (ALU) overlap
 #ifndef NBA_PIPE_ONEBIN       // pipelined ring: one-length-bin batches keep index order (no sort)
 #define NBA_PIPE_ONEBIN 1
 #endif
@@ -96,7 +99,8 @@ __device__ __forceinline__ PktPre load_pkt_pre(const DevTable &T, const uint8_t 
 __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B, FusedLo &L,
                                            FusedHi &H, uint32_t lane4r, uint32_t tid, uint32_t sa,
                                            uint32_t info, uint32_t q32, uint32_t inoff,
-                                           uint32_t outoff, const PktPre &pp, unsigned long long *dbg)
+                                           uint32_t outoff, const PktPre &pp, unsigned long long *dbg,
+                                           uint32_t *aes0_mark = nullptr, uint32_t t_start = 0)
 {
     long long ck_start = clock64(), ck_setup = 0, ck_aes = 0, ck_sha = 0, ck_emit = 0;
     const uint4 r0 = pp.r0, r1 = pp.r1, r2 = pp.r2, hd = pp.hd, h0 = pp.h0, h1 = pp.h1;
@@ -229,6 +233,9 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
             }
             long long ck_a1 = clock64();
             ck_aes += 0;
+            // pipelined ring: how long the lower lane warps take to their first
+            // AES step (the upper ones start that much later next batch)
+            if (aes0_mark && it == 0) atomicMax(aes0_mark, (uint32_t)gtimer() - t_start);
             // stream the ciphertext words of this step to the output slot
             if (16u * it + 16u <= Cw) {
                 os.put16(ct);
@@ -1164,6 +1171,10 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
     const uint32_t lane4r = (lane * 4u) | (smem_u32(tabs) & 0xffff0000u);
     tables_stage(tabs, T, &L.tbar, true);   // bulk copy, waited for before the first lookup
     if (tid < NBINS) L.bins[tid] = 0u;
+    if (tid == 0) {
+        L.stag_ns = 0u;
+        L.stag_acc = 0u;
+    }
     for (uint32_t k = tid; k < 2u * F_SUPER; k += F_THREADS) {
         L.hkey[k] = INVALID_SA;
         L.hmask[k] = 0u;
@@ -1256,8 +1267,19 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
 #ifdef NBA_STAGGER_NS   // experiment: delay the upper lane warps (phase-locking of AES / SHA-1)
                     if (warp >= 7u) __nanosleep(NBA_STAGGER_NS);
 #endif
+                    uint32_t t_start = 0;
+                    if (NBA_PIPE_STAGGER) {
+                        t_start = (uint32_t)gtimer();
+                        if (warp >= PIPE_LANE_WARPS / 2u) {   // the upper half waits
+                            const uint32_t d = L.stag_ns;
+                            while ((uint32_t)gtimer() - t_start < d) __nanosleep(256);
+                        }
+                    }
                     if (!NBA_PROLOGUE_ONLY)   // (debug A/B: the ring without the lane work)
-                        esp_packet(T, B, L, H, lane4r, tid, sa, info, q32, inoff, outoff, pp, nullptr);
+                        esp_packet(T, B, L, H, lane4r, tid, sa, info, q32, inoff, outoff, pp, nullptr,
+                                   (NBA_PIPE_STAGGER && warp < PIPE_LANE_WARPS / 2u) ? &L.stag_acc
+                                                                                     : nullptr,
+                                   t_start);
                     const uint32_t Dp = info & 0x7ffu;
                     const uint32_t Lp = 48u + esp_C(Dp);
                     B.out_len[pkt] = (uint16_t)Lp;
@@ -1288,6 +1310,10 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
             }
         }
         __syncthreads();                                  // batch bi done, bi + 1 prepared
+        if (NBA_PIPE_STAGGER && tid == 0) {               // next batch's delay of the upper warps
+            L.stag_ns = (uint32_t)(((unsigned long long)L.stag_acc * NBA_PIPE_STAGGER) >> 8);
+            L.stag_acc = 0u;
+        }
 #if NBA_RING_TRACE
         if (tid == 0 && R.ts) *RTR(bi, 5) = gtimer();
 #else
