@@ -1007,7 +1007,7 @@ __device__ __forceinline__ void pipe_prologue(const DevTable &T, const DevWork &
         // long or length-divergent batches; for uniform short ones after
         // (measured: 64 B 23.5 vs 24.1 us, IMIX 96.8 vs 90.4, 1514 B 193.7 vs 192.3)
         const uint32_t sum = L.pstat[0], mx = L.pstat[1], nv = cnt ? cnt : 1u;
-        L.pstat[2] = (mx * nv > 2u * sum || sum >= 8u * nv) ? 1u : 0u;   // (clears bit 2)
+        L.pstat[2] = (L.pstat[2] & 4u) | ((mx * nv > 2u * sum || sum >= 8u * nv) ? 1u : 0u);
     }
     if (pw == 0 && !NBA_PIPE_LPT) {
         if (lane < PIPE_LANE_WARPS) L.wrun[lane] = (uint8_t)lane;   // run r -> warp r
@@ -1221,6 +1221,7 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
         bool have = false;
         const bool early = NBA_PIPE_EARLY_KEYS == 1 ? true
                          : NBA_PIPE_EARLY_KEYS == 0 ? false : (L.pstat[2] & 1u) != 0u;
+        const bool uniform = (L.pstat[2] & 4u) != 0u;    // the batch's packets share one length bin
         PktPre pp = {};
         if (!isP) {
             const uint32_t run = L.wrun[warp];          // LPT placement of the runs
@@ -1268,7 +1269,7 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
                     if (warp >= 7u) __nanosleep(NBA_STAGGER_NS);
 #endif
                     uint32_t t_start = 0;
-                    if (NBA_PIPE_STAGGER) {
+                    if (NBA_PIPE_STAGGER && uniform) {       // one-length batches only
                         t_start = (uint32_t)gtimer();
                         if (warp >= PIPE_LANE_WARPS / 2u) {   // the upper half waits
                             const uint32_t d = L.stag_ns;
@@ -1277,8 +1278,8 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
                     }
                     if (!NBA_PROLOGUE_ONLY)   // (debug A/B: the ring without the lane work)
                         esp_packet(T, B, L, H, lane4r, tid, sa, info, q32, inoff, outoff, pp, nullptr,
-                                   (NBA_PIPE_STAGGER && warp < PIPE_LANE_WARPS / 2u) ? &L.stag_acc
-                                                                                     : nullptr,
+                                   (NBA_PIPE_STAGGER && uniform && warp < PIPE_LANE_WARPS / 2u)
+                                       ? &L.stag_acc : nullptr,
                                    t_start);
                     const uint32_t Dp = info & 0x7ffu;
                     const uint32_t Lp = 48u + esp_C(Dp);

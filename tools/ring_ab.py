@@ -94,7 +94,7 @@ def main():
         return
     names = sorted(f[:-3] for f in os.listdir(VDIR) if f.endswith(".so") and not f.endswith("trace.so")) \
         if os.path.isdir(VDIR) else []
-    for rep in range(2):
+    for rep in range(int(os.environ.get("AB_PASSES", "2"))):
         print(f"pass {rep} base", run_one(None, sizes, 200, False), flush=True)
         for n in names:
             print(f"pass {rep} {n}", run_one(os.path.join(VDIR, n + ".so"), sizes, 200, False),
