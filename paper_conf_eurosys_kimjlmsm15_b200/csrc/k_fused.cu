@@ -59,7 +59,7 @@ namespace nba {
 #define NBA_RK_ASYNC 0        //   schedule (1) instead of expanded in the lane (0); measured
 #endif                        //   slower (64 B 24.4 -> 27.5 us: the LDGSTS issue delays the scans)
 #ifndef NBA_PIPE_STAGGER      // pipelined ring: lane warps 7..13 start their packets later by
-#define NBA_PIPE_STAGGER 0    //   STAGGER/256 x the time the lower warps took to their first AES
+#define NBA_PIPE_STAGGER 128  //   STAGGER/256 x the time the lower warps took to their first AES
 #endif                        //   step (previous batch), so AES (LDS) and SHA-1 (ALU) overlap
 #ifndef NBA_PIPE_ONEBIN       // pipelined ring: one-length-bin batches keep index order (no sort)
 #define NBA_PIPE_ONEBIN 1
