@@ -405,6 +405,7 @@ struct nba_ipsec_ring {
     uint32_t *hval_b = nullptr;
     uint32_t in_hmask = 0;
     bool pipe = false;                   // software-pipelined form (k_fused_ring_pipe)
+    bool in_pipe = false;                // inbound: software-pipelined form (k_in_fused_ring_pipe)
     bool pipe_ok = false;                // every slot fits the pipelined form
     uint64_t flow_gen = 0;               // the table's flow-table generation when recorded
     uint32_t cursor = 0;                 // the slot the next run_batches starts at
@@ -513,17 +514,23 @@ int nba_ipsec_ring_create_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batc
     r->n_slots = n_slots;
     r->flow_gen = t->flow_gen;
     r->h_in_slots.assign(slots, slots + n_slots);
-    // persistent form (opt-in, NBA_IPSEC_RING_IN_PERSIST) when every slot takes
-    // the one-kernel inbound path; measured against the graph form: 64 B 45.9
-    // -> 43.9 us, 1514 B 215.4 -> 217.2 us, IMIX 108.6 -> 117.5 us
+    // persistent forms: the software-pipelined ring (k_in_fused_ring_pipe) when
+    // every slot fits it (<= 448 packets per SM) -- the default --, else the
+    // plain persistent ring (opt-in, NBA_IPSEC_RING_IN_PERSIST; measured
+    // against the graph form: 64 B 45.0 -> 43.3 us, 1514 B 213.9 -> 214.9 us,
+    // IMIX 107.3 -> 112.6 us), else a CUDA graph of one-kernel launches
+    bool pipe = !std::getenv("NBA_IPSEC_RING_GRAPH") && !std::getenv("NBA_IPSEC_RING_NOPIPE") &&
+                t->allow_merged;
     bool persist = std::getenv("NBA_IPSEC_RING_IN_PERSIST") && !std::getenv("NBA_IPSEC_RING_GRAPH") &&
                    t->allow_merged;
     uint32_t nmax = 0;
-    for (uint32_t i = 0; i < n_slots && persist; i++) {
-        persist = slots[i].n_pkts > 0 && in_merged_ok(slots[i].n_pkts, t->grid_fused);
+    for (uint32_t i = 0; i < n_slots; i++) {
+        pipe = pipe && in_pipe_ok(slots[i].n_pkts, t->grid_fused);
+        persist = persist && slots[i].n_pkts > 0 && in_merged_ok(slots[i].n_pkts, t->grid_fused);
         nmax = std::max(nmax, slots[i].n_pkts);
     }
-    if (persist) {
+    r->in_pipe = pipe;
+    if (pipe || persist) {
         uint32_t hmask = 1023;   // one hash size for every slot: the largest batch's
         while (hmask + 1ull < 2ull * nmax) hmask = hmask * 2 + 1;
         r->in_hmask = hmask;
@@ -587,8 +594,11 @@ static int ring_launch(nba_ipsec_ring *r, uint32_t first, uint32_t n_batches, cu
     }
     const RingRun R{r->n_slots, first, n_batches, r->ts};
     if (r->d_in_slots)
-        return launch_in_fused_ring(t->T, t->S, r->d_in_slots, R, r->in_hmask, r->hkey_b, r->hval_b,
-                                    t->grid_fused, st) == cudaSuccess
+        return (r->in_pipe ? launch_in_fused_ring_pipe(t->T, t->S, r->d_in_slots, R, r->in_hmask,
+                                                       r->hkey_b, r->hval_b, t->grid_fused, st)
+                           : launch_in_fused_ring(t->T, t->S, r->d_in_slots, R, r->in_hmask,
+                                                  r->hkey_b, r->hval_b, t->grid_fused, st)) ==
+                       cudaSuccess
                    ? NBA_IPSEC_OK
                    : NBA_IPSEC_ECUDA;
     if (r->d_slots) {
@@ -669,7 +679,7 @@ int nba_ipsec_ring_set_form(nba_ipsec_ring *r, int form)
 int nba_ipsec_ring_form(const nba_ipsec_ring *r)
 {
     if (!r) return NBA_IPSEC_EINVAL;
-    if (r->d_in_slots) return NBA_IPSEC_RING_PERSISTENT;
+    if (r->d_in_slots) return r->in_pipe ? NBA_IPSEC_RING_PIPELINED : NBA_IPSEC_RING_PERSISTENT;
     return !r->d_slots ? NBA_IPSEC_RING_GRAPH : r->pipe ? NBA_IPSEC_RING_PIPELINED
                                                          : NBA_IPSEC_RING_PERSISTENT;
 }

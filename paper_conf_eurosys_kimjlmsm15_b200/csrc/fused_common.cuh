@@ -39,6 +39,8 @@ struct FusedLo {
     uint32_t pstat[3];             // pipelined ring: the next batch's AES steps (sum, max) and
                                    //   its "early round keys" decision
     unsigned long long tbar;       // mbarrier: the bulk copy of the T-table image landed
+    uint32_t tailf[448];           // inbound pipelined ring: a batch's per-packet flags and
+    uint32_t tailq[448];           //   sequence numbers (by packet index) for its replay tail
     uint32_t stag_ns;              // pipelined ring: start delay of the upper lane warps
     uint32_t stag_acc;             //   (AES step 0 of the lower ones, measured per batch)
 };
@@ -809,6 +811,49 @@ __device__ __forceinline__ bool lane_position(const FusedLo &L, uint32_t cnt, ui
     const uint32_t lw = (cnt + NW - 1u) / NW;
     pos = warp * lw + lane;
     return lane < lw && pos < cnt;
+}
+
+// ---- warp-specialised (software-pipelined) batch rings ---------------------
+// Warps 0..13 ("lanes") carry a batch's packets, one per lane; warps 14..15
+// ("prologue" / side warps) prepare the next batch meanwhile.
+constexpr uint32_t PIPE_LANE_WARPS = 14;
+constexpr uint32_t PIPE_MAX_PPC = PIPE_LANE_WARPS * 32u;          // 448 packets per CTA
+constexpr uint32_t PIPE_P = F_THREADS - PIPE_MAX_PPC;             // 64 prologue threads
+
+__device__ __forceinline__ void bar_sync_n(uint32_t id, uint32_t n)
+{
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+__device__ __forceinline__ void bar_arrive_n(uint32_t id, uint32_t n)
+{
+    asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+
+// LPT placement of nruns runs (costs in lanes 0..nruns-1) onto the four SM
+// sub-partitions (warp w issues on w mod 4; capq = lane warps on partition q):
+// longest-first is the caller's order, each run goes to the least loaded
+// partition with room (first minimum on ties), taking its next warp
+// q + 4 * used_q.  Returns the run this lane's warp gets (0xff: none).  All
+// state in registers (compare-select over the four partitions), so the
+// prologue warps spill nothing.
+__device__ __forceinline__ uint32_t lpt_place(uint32_t cost, uint32_t nruns, uint32_t lane,
+                                              uint32_t cap0, uint32_t cap1, uint32_t cap2,
+                                              uint32_t cap3)
+{
+    uint32_t l0 = 0, l1 = 0, l2 = 0, l3 = 0, u0 = 0, u1 = 0, u2 = 0, u3 = 0, mine = 0xffu;
+    for (uint32_t r = 0; r < nruns; r++) {
+        const uint32_t cr = __shfl_sync(0xffffffffu, cost, r);
+        uint32_t best = 0, bl = 0xffffffffu, bu = 0;
+        if (u0 < cap0 && l0 < bl) { best = 0; bl = l0; bu = u0; }
+        if (u1 < cap1 && l1 < bl) { best = 1; bl = l1; bu = u1; }
+        if (u2 < cap2 && l2 < bl) { best = 2; bl = l2; bu = u2; }
+        if (u3 < cap3 && l3 < bl) { best = 3; bl = l3; bu = u3; }
+        if (lane == best + 4u * bu) mine = r;
+        u0 += best == 0; u1 += best == 1; u2 += best == 2; u3 += best == 3;
+        l0 += best == 0 ? cr : 0u; l1 += best == 1 ? cr : 0u;
+        l2 += best == 2 ? cr : 0u; l3 += best == 3 ? cr : 0u;
+    }
+    return mine;
 }
 
 // Flow -> SA lookup of one inner datagram P (D bytes), readings F1..F4: one

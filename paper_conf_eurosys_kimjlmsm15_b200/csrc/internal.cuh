@@ -199,6 +199,10 @@ cudaError_t launch_in_fused_ring(const DevTable &T, const InState &S, const InBa
                                  const RingRun &R, uint32_t hmask,
                                  unsigned long long *hkey_b, uint32_t *hval_b, int grid,
                                  cudaStream_t st);
+cudaError_t launch_in_fused_ring_pipe(const DevTable &T, const InState &S, const InBatchArgs *slots,
+                                      const RingRun &R, uint32_t hmask, unsigned long long *hkey_b,
+                                      uint32_t *hval_b, int grid, cudaStream_t st);
+bool in_pipe_ok(uint32_t n, int grid);
 cudaError_t launch_in_replay(const DevTable &T, const InState &S, const InBatchArgs &B,
                              uint32_t n_tiles, uint32_t hmask, bool gridsync, cudaStream_t st);
 cudaError_t launch_in_decide(const DevTable &T, const InState &S, const InBatchArgs &B,

@@ -691,24 +691,12 @@ k_fused_ring(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint16_t 
 #if NBA_RING_TRACE
 #define RTR(bi, k) (R.ts ? R.ts + ((size_t)(bi) * gridDim.x + blockIdx.x) * 16u + (k) : nullptr)
 #endif
-constexpr uint32_t PIPE_LANE_WARPS = 14;
-constexpr uint32_t PIPE_MAX_PPC = PIPE_LANE_WARPS * 32u;          // 448 packets per CTA
-constexpr uint32_t PIPE_P = F_THREADS - PIPE_MAX_PPC;             // 64 prologue threads
 
 __device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long v)
 {
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v += __shfl_down_sync(0xffffffffu, v, o);
     return v;   // lane 0
-}
-
-__device__ __forceinline__ void bar_sync_n(uint32_t id, uint32_t n)
-{
-    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
-}
-__device__ __forceinline__ void bar_arrive_n(uint32_t id, uint32_t n)
-{
-    asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(n) : "memory");
 }
 
 // The prologue warps' share of the row scans (rows slot, slot + nslots, ...),
@@ -760,33 +748,6 @@ __device__ __forceinline__ void pipe_scan_rows(const DevTable &T, const DevWork 
             }
         }
     }
-}
-
-// LPT placement of nruns runs (costs in lanes 0..nruns-1) onto the four SM
-// sub-partitions (warp w issues on w mod 4; capq = lane warps on partition q):
-// longest-first is the caller's order, each run goes to the least loaded
-// partition with room (first minimum on ties), taking its next warp
-// q + 4 * used_q.  Returns the run this lane's warp gets (0xff: none).  All
-// state in registers (compare-select over the four partitions), so the
-// prologue warps spill nothing.
-__device__ __forceinline__ uint32_t lpt_place(uint32_t cost, uint32_t nruns, uint32_t lane,
-                                              uint32_t cap0, uint32_t cap1, uint32_t cap2,
-                                              uint32_t cap3)
-{
-    uint32_t l0 = 0, l1 = 0, l2 = 0, l3 = 0, u0 = 0, u1 = 0, u2 = 0, u3 = 0, mine = 0xffu;
-    for (uint32_t r = 0; r < nruns; r++) {
-        const uint32_t cr = __shfl_sync(0xffffffffu, cost, r);
-        uint32_t best = 0, bl = 0xffffffffu, bu = 0;
-        if (u0 < cap0 && l0 < bl) { best = 0; bl = l0; bu = u0; }
-        if (u1 < cap1 && l1 < bl) { best = 1; bl = l1; bu = u1; }
-        if (u2 < cap2 && l2 < bl) { best = 2; bl = l2; bu = u2; }
-        if (u3 < cap3 && l3 < bl) { best = 3; bl = l3; bu = u3; }
-        if (lane == best + 4u * bu) mine = r;
-        u0 += best == 0; u1 += best == 1; u2 += best == 2; u3 += best == 3;
-        l0 += best == 0 ? cr : 0u; l1 += best == 1 ? cr : 0u;
-        l2 += best == 2 ? cr : 0u; l3 += best == 3 ? cr : 0u;
-    }
-    return mine;
 }
 
 // The packet metadata of this prologue thread (packets j = r * 64 + pt of the

@@ -146,6 +146,40 @@ __device__ __forceinline__ uint32_t esp_in_packet(const DevTable &T, const InBat
     return flags;
 }
 
+// Format checks of one received packet (reading B2): outer IPv4 header without
+// options, total length = L, not a fragment, protocol 50, valid checksum, the
+// SA's SPI.  info = C | INFO_OK (0: DROP_FORMAT / DROP_SA), q = the sequence
+// number field, iv0 / iv1 = the IV words.
+__device__ __forceinline__ void in_format(const DevTable &T, const InBatchArgs &B, uint32_t sa,
+                                          uint32_t Lin, uint32_t inoff, uint32_t &info, uint32_t &q,
+                                          uint32_t &iv0, uint32_t &iv1)
+{
+    info = q = iv0 = iv1 = 0;
+    if (sa < T.n_sa && Lin >= IN_MIN_LEN && Lin <= IN_MAX_LEN && ((Lin - 48u) & 3u) == 0) {
+        const uint8_t *pk = B.in_buf + inoff;
+        uint32_t w[9];
+        load_words<9>(reinterpret_cast<uintptr_t>(pk), reinterpret_cast<uintptr_t>(pk) + Lin, w);
+        // RFC 1071: the one's complement sum over the header (checksum
+        // included) is 0xffff; byte order does not matter (§2(B))
+        uint32_t sum = 0;
+#pragma unroll
+        for (int k = 0; k < 5; k++) sum += (w[k] & 0xffffu) + (w[k] >> 16);
+        sum = (sum & 0xffffu) + (sum >> 16);
+        sum = (sum & 0xffffu) + (sum >> 16);
+        const uint32_t tot = ((w[0] >> 8) & 0xff00u) | (w[0] >> 24);
+        const bool ok = (w[0] & 0xffu) == 0x45u && tot == Lin &&
+                        (w[1] & 0xff3f0000u) == 0u &&         // MF = 0, offset 0
+                        ((w[2] >> 8) & 0xffu) == 50u && sum == 0xffffu &&
+                        w[5] == __ldg(&T.sahdr[sa]).x;        // SPI (RFC 4303 §3.4.2)
+        if (ok) {
+            info = (Lin - 48u) | INFO_OK;
+            q = bswap32(w[6]);
+            iv0 = w[7];
+            iv1 = w[8];
+        }
+    }
+}
+
 // ---- one-kernel inbound (n <= F_SUPER x grid): the anti-replay decision of
 // k_in_replay / k_in_decide inside this kernel, each CTA one tile of the
 // batch (its packets in batch order, thread j <-> packet p_begin + j):
@@ -313,29 +347,7 @@ __device__ __forceinline__ void in_fused_body(const DevTable &T, const InState &
             const uint32_t Lin = B.in_len[i];
             const uint32_t inoff = B.in_off[i];
             uint32_t info = 0, q = 0, iv0 = 0, iv1 = 0;
-            if (sa < n_sa && Lin >= IN_MIN_LEN && Lin <= IN_MAX_LEN && ((Lin - 48u) & 3u) == 0) {
-                const uint8_t *pk = B.in_buf + inoff;
-                uint32_t w[9];
-                load_words<9>(reinterpret_cast<uintptr_t>(pk), reinterpret_cast<uintptr_t>(pk) + Lin, w);
-                // RFC 1071: the one's complement sum over the header (checksum
-                // included) is 0xffff; byte order does not matter (§2(B))
-                uint32_t sum = 0;
-#pragma unroll
-                for (int k = 0; k < 5; k++) sum += (w[k] & 0xffffu) + (w[k] >> 16);
-                sum = (sum & 0xffffu) + (sum >> 16);
-                sum = (sum & 0xffffu) + (sum >> 16);
-                const uint32_t tot = ((w[0] >> 8) & 0xff00u) | (w[0] >> 24);
-                const bool ok = (w[0] & 0xffu) == 0x45u && tot == Lin &&
-                                (w[1] & 0xff3f0000u) == 0u &&         // MF = 0, offset 0
-                                ((w[2] >> 8) & 0xffu) == 50u && sum == 0xffffu &&
-                                w[5] == __ldg(&T.sahdr[sa]).x;        // SPI (RFC 4303 §3.4.2)
-                if (ok) {
-                    info = (Lin - 48u) | INFO_OK;
-                    q = bswap32(w[6]);
-                    iv0 = w[7];
-                    iv1 = w[8];
-                }
-            }
+            in_format(T, B, sa, Lin, inoff, info, q, iv0, iv1);
             L.sa[j] = sa;
             L.info[j] = info;
             L.seq[j] = q;
@@ -429,6 +441,343 @@ k_in_fused_ring(DevTable T, InState S, const InBatchArgs *slots, RingRun R, uint
     }
 }
 
+// ------------------------------------------ software-pipelined inbound ring
+// k_in_fused_ring_pipe: the inbound ring with warp roles, as the outbound
+// k_fused_ring_pipe.  Per batch k: warps 0..13 ("lanes") take their packet's
+// fields (named barrier 2) and run the ICV check + decryption, leaving each
+// packet's flags and sequence number in L.tailf / L.tailq (by packet index);
+// warps 14..15 meanwhile prepare batch k + 1 -- metadata, format checks (the
+// outer header of every packet), length order and LPT run placement -- so
+// neither the metadata's DRAM latency nor the header loads sit on the
+// critical path; then the whole CTA runs batch k's anti-replay tail (the
+// same arithmetic as in_merged_tail: warp-segmented prefix maxima, the CTA's
+// SA hash, the (SA, CTA) tile maxima, grid barrier, first-index hash inserts
+// and row scans, grid barrier, decisions).  The per-warp group maxima of the
+// tail live in the lanes' round-key slots (L.rkA / H.rkB, free once the lanes
+// are done), so the T-tables stay in shared memory for the whole run (staged
+// once).  The duplicate hash alternates between two buffers by batch parity;
+// batch k clears its buffer before its first barrier, and that buffer's last
+// user (batch k - 2) finished everywhere before batch k - 1's second barrier.
+
+// Metadata + format checks + length order of one inbound batch by the 64
+// prologue threads (pt = 0..63) of this CTA.
+__device__ __forceinline__ void in_pipe_prologue(const DevTable &T, const InBatchArgs &B, uint32_t ppc,
+                                                 FusedLo &L, uint32_t pt)
+{
+    constexpr uint32_t PR = PIPE_MAX_PPC / PIPE_P;                  // 7 rounds
+    const uint32_t lane = pt & 31u, pw = pt >> 5;
+    const uint32_t p_begin = blockIdx.x * ppc;
+    const uint32_t p_end = min(B.n, p_begin + ppc);
+    const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
+    const uint32_t rounds = (cnt + PIPE_P - 1u) / PIPE_P;
+    uint32_t mS[PR], mL[PR], mI[PR];
+#pragma unroll
+    for (uint32_t r = 0; r < PR; r++) {                             // all loads issued together
+        const uint32_t j = r * PIPE_P + pt, i = p_begin + j;
+        mS[r] = j < cnt ? B.sa_idx[i] : INVALID_SA;
+        mL[r] = j < cnt ? B.in_len[i] : 0u;
+        mI[r] = j < cnt ? B.in_off[i] : 0u;
+    }
+#pragma unroll
+    for (uint32_t r = 0; r < PR; r++)                               // outer headers -> L2 / L1
+        if (r * PIPE_P + pt < cnt) prefetch_l2(B.in_buf + mI[r]);
+    for (uint32_t r = 0; r < rounds; r++) {
+        const uint32_t j = r * PIPE_P + pt, i = p_begin + j;
+        uint32_t bin = NBINS - 1;
+        if (j < cnt) {
+            uint32_t info, q, iv0, iv1;
+            in_format(T, B, mS[r], mL[r], mI[r], info, q, iv0, iv1);
+            L.sa[j] = mS[r];
+            L.info[j] = info;
+            L.seq[j] = q;
+            L.inoff[j] = mI[r];
+            L.outoff[j] = B.out_off[i];
+            L.aux0[j] = iv0;
+            L.aux1[j] = iv1;
+            if (info) bin = hmac_bin(true, info & 0xffffu);
+        }
+        warp_agg_add(L.bins, bin, j < cnt);
+    }
+    bar_sync_n(1, PIPE_P);
+    bool one_bin = false;
+    if (pw == 0) {                                                  // bins -> cursors
+        const uint32_t cb = L.bins[lane];
+        one_bin = __any_sync(0xffffffffu, cb == cnt);
+        uint32_t x = cb;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+            if (lane >= (uint32_t)o) x += y;
+        }
+        L.bins[lane] = x - cb;
+        if (lane == 0) L.pstat[2] = one_bin ? 4u : 0u;
+    }
+    bar_sync_n(1, PIPE_P);
+    one_bin = (L.pstat[2] & 4u) != 0u;
+    for (uint32_t r = 0; r < rounds; r++) {
+        const uint32_t j = r * PIPE_P + pt;
+        if (one_bin) {                           // counting sort of one bin = index order
+            if (j < cnt) L.perm[j] = (uint16_t)j;
+            continue;
+        }
+        const uint32_t info = j < cnt ? L.info[j] : 0u;
+        const uint32_t bin = info ? hmac_bin(true, info & 0xffffu) : NBINS - 1;
+        const uint32_t pos = warp_agg_add(L.bins, bin, j < cnt);
+        if (j < cnt) L.perm[pos] = (uint16_t)j;
+    }
+    bar_sync_n(1, PIPE_P);
+    if (pt < NBINS) L.bins[pt] = 0u;
+    if (pw == 0) {
+        // runs of 32 sorted positions -> lane warps, longest first onto the
+        // least loaded sub-partition (as the outbound pipelined ring)
+        const uint32_t nruns = (cnt + 31u) / 32u;
+        uint32_t cost = 0;
+        if (lane < nruns) {
+            const uint32_t info = L.info[L.perm[32u * lane]];
+            const uint32_t C = info & 0xffffu;
+            cost = info ? 8u * (esp_nsha_inner(C) + 1u) + 3u * ((C + 15u) >> 4) : 1u;
+        }
+        const uint32_t c0 = __shfl_sync(0xffffffffu, cost, 0);
+        uint32_t mine = lane < nruns ? lane : 0xffu;
+        if (!__all_sync(0xffffffffu, lane >= nruns || cost == c0))
+            mine = lpt_place(cost, nruns, lane, 4u, 4u, 3u, 3u);
+        if (lane < PIPE_LANE_WARPS) L.wrun[lane] = (uint8_t)mine;
+    }
+}
+
+// Batch k's anti-replay tail by the whole CTA (thread j <-> packet p_begin + j):
+// in_merged_tail with the flags / sequence numbers from L.tailf / L.tailq, the
+// group maxima in the round-key slots, and the duplicate hash cleared here.
+__device__ __forceinline__ void in_pipe_tail(const DevTable &T, const InState &S, const InBatchArgs &B,
+                                             FusedLo &L, FusedHi &H, uint32_t p_begin, uint32_t p_end,
+                                             uint32_t hmask, uint32_t bar_base,
+                                             unsigned long long (&ctr)[N_IN_COUNTERS - 1])
+{
+    constexpr uint32_t HS = 2u * F_SUPER, NW = F_THREADS / 32u;
+    const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
+    const uint32_t G = gridDim.x, cta = blockIdx.x, n_sa = T.n_sa;
+    const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
+    const uint32_t j = tid, i = p_begin + j;
+    const bool live = j < cnt;
+    // this batch's duplicate hash (its previous user finished everywhere)
+    for (uint32_t k = cta * F_THREADS + tid; k <= hmask; k += G * F_THREADS) {
+        S.hkey[k] = ~0ull;
+        S.hval[k] = ~0u;
+    }
+    const uint32_t f = live ? L.tailf[j] : 0u;
+    const uint32_t sa = live ? B.sa_idx[i] : INVALID_SA;
+    const uint32_t q = (f & INF_FMT) ? L.tailq[j] : 0u;
+    const uint32_t key = (f & INF_FMT) ? sa : INVALID_SA;
+    const bool inA = (f & INF_ICV) != 0u;
+    const uint32_t qa = inA ? q : 0u;
+    for (uint32_t k = tid; k < HS; k += F_THREADS) {
+        L.hkey[k] = INVALID_SA;
+        L.hmask[k] = 0;
+    }
+    // per-warp group maxima [HS][NW] u32: slots < 512 in L.rkA, the rest in H.rkB
+    auto gm = [&](uint32_t slot) -> uint32_t * {
+        uint32_t *b = slot < 512u ? reinterpret_cast<uint32_t *>(&L.rkA[0][0])
+                                  : reinterpret_cast<uint32_t *>(&H.rkB[0][0]);
+        return b + (slot & 511u) * NW;
+    };
+    const uint32_t peers = __match_any_sync(0xffffffffu, key);
+    const uint32_t lt = peers & lanemask_lt();
+    uint32_t mex = 0;                                // max over earlier lanes of the group
+#pragma unroll
+    for (int l = 0; l < 32; l++) {
+        const uint32_t v = __shfl_sync(0xffffffffu, qa, l);
+        if ((lt >> l) & 1u) mex = max(mex, v);
+    }
+    const uint32_t leader = __ffs(peers) - 1, hi_lane = 31u - __clz(peers);
+    const uint32_t gmax = __shfl_sync(0xffffffffu, max(mex, qa), hi_lane);
+    __syncthreads();   // CTA hash initialised, round-key slots no longer read
+    uint32_t slot = 0;
+    if (key != INVALID_SA && lane == leader) {
+        slot = (key * 0x9E3779B1u) >> 22;           // 10 bits -> HS = 1024 slots
+        while (true) {
+            const uint32_t old = atomicCAS(&L.hkey[slot], INVALID_SA, key);
+            if (old == INVALID_SA || old == key) break;
+            slot = (slot + 1u) & (HS - 1u);
+        }
+        gm(slot)[warp] = gmax;
+        atomicOr(&L.hmask[slot], 1u << warp);
+    }
+    slot = __shfl_sync(0xffffffffu, slot, leader);
+    __syncthreads();
+    uint32_t base = 0;
+    if (key != INVALID_SA) {
+        const uint32_t m = L.hmask[slot];
+        const uint32_t *g = gm(slot);
+#pragma unroll
+        for (uint32_t w = 0; w < NW; w++)
+            if (w < warp && ((m >> w) & 1u)) base = max(base, g[w]);
+        const uint32_t tmax = max(base, gmax);       // per-tile SA maximum, nonzero only
+        if ((m >> (warp + 1u)) == 0u && lane == hi_lane && tmax != 0u)
+            S.hmax[(size_t)key * G + cta] = tmax;
+    }
+    const uint32_t lmax = max(base, mex);
+    __syncthreads();
+    grid_arrive(&S.ctl[CTLI_BAR]);
+    grid_wait(&S.ctl[CTLI_BAR], bar_base + G);
+    if (inA) replay_hash_insert(S, key, q, i, hmask);
+    scan_all_rows(S, n_sa, cta * NW + warp, G * NW, G, lane);
+    __syncthreads();
+    grid_arrive(&S.ctl[CTLI_BAR]);
+    grid_wait(&S.ctl[CTLI_BAR], bar_base + 2u * G);
+    uint32_t st = 0xffu, D = 0, Lin = 0;
+    if (live) {
+        if (sa >= n_sa) {
+            st = ST_DROP_SA;
+        } else if (!(f & INF_FMT)) {
+            st = ST_DROP_FORMAT;
+        } else {
+            const uint32_t t0 = S.top_prev[sa];
+            const unsigned long long b0 = S.bmp_prev[sa];
+            const uint32_t tj = max(t0, max(S.pmx[(size_t)sa * G + cta], lmax));
+            st = replay_decide(S, sa, i, f, q, t0, b0, tj, S.top[sa], hmask);
+            if (st == ST_OK) {
+                D = f & 0xffffu;
+                Lin = B.in_len[i];
+            }
+        }
+        B.out_len[i] = (uint16_t)D;
+        if (B.status) B.status[i] = (uint8_t)st;
+    }
+    // counters in registers (lane 0 of each warp), reduced once per run
+#pragma unroll
+    for (uint32_t k = 0; k < 6; k++) ctr[k] += __reduce_add_sync(0xffffffffu, st == k ? 1u : 0u);
+    ctr[6] += __reduce_add_sync(0xffffffffu, Lin);
+    ctr[7] += __reduce_add_sync(0xffffffffu, D);
+}
+
+__global__ void __launch_bounds__(F_THREADS, 1)
+k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R, uint32_t hmask,
+                     unsigned long long *hkey_b, uint32_t *hval_b)
+{
+    extern __shared__ __align__(16) uint8_t smem[];
+    const uint32_t n_slots = R.n_slots, n_batches = R.n_batches, first = R.first;
+    const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
+    const uint32_t G = gridDim.x, cta = blockIdx.x;
+    if (n_batches == 0) return;
+    if (R.ts && cta == 0 && tid == 0) R.ts[0] = gtimer();
+    const uint32_t base0 = *reinterpret_cast<volatile uint32_t *>(&S.ctl[CTLI_BASE]);
+    const uint32_t sb = smem_u32(smem);
+    const uint32_t toff = (0x10000u - (sb & 0xffffu)) & 0xffffu;
+    uint32_t lo_off = 0;
+    if (toff < sizeof(FusedLo)) {
+        if (toff + AES_TABLE_BYTES + sizeof(FusedHi) + sizeof(FusedLo) > F_SMEM) __trap();
+        lo_off = toff + AES_TABLE_BYTES + (uint32_t)sizeof(FusedHi);
+    }
+    uint8_t *tabs = smem + toff;
+    FusedLo &L = *reinterpret_cast<FusedLo *>(smem + lo_off);
+    FusedHi &H = *reinterpret_cast<FusedHi *>(smem + toff + AES_TABLE_BYTES);
+    const uint32_t lane4r = (lane * 4u) | (smem_u32(tabs) & 0xffff0000u);
+    tables_stage(tabs, T, &L.tbar, true);   // bulk copy, waited for before the first lookup
+    if (tid < NBINS) L.bins[tid] = 0u;
+    __syncthreads();
+    const bool isP = tid >= PIPE_MAX_PPC;
+    const uint32_t pt = tid - PIPE_MAX_PPC;
+    auto ppc_of = [&](const InBatchArgs &B) {
+        uint32_t ppc = (B.n + G - 1) / G;
+        ppc = (ppc + 31u) & ~31u;
+        return ppc < 32u ? 32u : ppc;
+    };
+    if (isP) {
+        const InBatchArgs B0 = slots[first % n_slots];
+        in_pipe_prologue(T, B0, ppc_of(B0), L, pt);
+    }
+    __syncthreads();
+    tables_bulk_wait(&L.tbar, 0u);
+    unsigned long long ctr[N_IN_COUNTERS - 1] = {};
+    for (uint32_t bi = 0; bi < n_batches; bi++) {
+        const InBatchArgs B = slots[(first + bi) % n_slots];
+        const uint32_t ppc = ppc_of(B);
+        const uint32_t p_begin = cta * ppc;
+        const uint32_t p_end = min(B.n, p_begin + ppc);
+        const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
+        if (!isP) {
+            const uint32_t run = L.wrun[warp];
+            const uint32_t pos = 32u * run + lane;
+            const bool have = run != 0xffu && pos < cnt;
+            const uint32_t pk = have ? L.perm[pos] : 0u;
+            const uint32_t info = have ? L.info[pk] : 0u;
+            const uint32_t sa = (info & INFO_OK) ? L.sa[pk] : INVALID_SA;
+            const uint32_t q = have ? L.seq[pk] : 0u;
+            const uint32_t iv0 = have ? L.aux0[pk] : 0u, iv1 = have ? L.aux1[pk] : 0u;
+            const uint32_t inoff = have ? L.inoff[pk] : 0u, outoff = have ? L.outoff[pk] : 0u;
+            bar_arrive_n(2, F_THREADS);                  // fields taken: the arrays are free
+            if (have) {
+                uint32_t flags = 0;
+                if (info & INFO_OK) {
+                    uint4 r0, hd, h0, h1, r1, r2;
+                    const uint4 *line = T.sal + (size_t)sa * SAL_U4;
+                    ldg_nc_v8(&line[0], r0, hd);
+                    ldg_nc_v8(&line[2], h0, h1);
+                    expand_key_lane(lane4r, r0, r1, r2, L, H, tid);
+                    flags = INF_FMT | esp_in_packet(T, B, L, H, lane4r, tid, sa, info & 0xffffu, q, iv0,
+                                                    iv1, inoff, outoff, r0, r1, r2, hd, h0, h1);
+                }
+                L.tailf[pk] = flags;
+                L.tailq[pk] = q;
+            }
+        } else {
+            bar_sync_n(2, F_THREADS);                    // every lane took its fields
+            if (bi + 1 < n_batches) {
+                const InBatchArgs Bn = slots[(first + bi + 1) % n_slots];
+                in_pipe_prologue(T, Bn, ppc_of(Bn), L, pt);
+            }
+        }
+        __syncthreads();                                  // lanes done, bi + 1 prepared
+        InState Sb = S;
+        if (bi & 1u) {
+            Sb.hkey = hkey_b;
+            Sb.hval = hval_b;
+        }
+        in_pipe_tail(T, Sb, B, L, H, p_begin, p_end, hmask, base0 + 2u * bi * G, ctr);
+        __syncthreads();                                  // the tail's scratch is free again
+        if (R.ts && tid == 0) atomicMax(&R.ts[1u + bi], gtimer());
+    }
+    // counters: warp sums (lane 0 holds them) -> one atomic per CTA and counter
+    __shared__ unsigned long long s_cnt[N_IN_COUNTERS - 1];
+    if (tid < N_IN_COUNTERS - 1) s_cnt[tid] = 0ull;
+    __syncthreads();
+    if (lane == 0) {
+#pragma unroll
+        for (uint32_t k = 0; k < N_IN_COUNTERS - 1; k++)
+            if (ctr[k]) atomicAdd(&s_cnt[k], ctr[k]);
+    }
+    __syncthreads();
+    if (tid < N_IN_COUNTERS - 1 && s_cnt[tid]) atomicAdd(&S.counters[tid], s_cnt[tid]);
+    if (tid == 0 && cta == 0) {
+        atomicAdd(&S.counters[N_IN_COUNTERS - 1], (unsigned long long)n_batches);
+        S.ctl[CTLI_BASE] = base0 + 2u * n_batches * G;   // two barriers per batch
+    }
+}
+
+cudaError_t launch_in_fused_ring_pipe(const DevTable &T, const InState &S, const InBatchArgs *slots,
+                                      const RingRun &R, uint32_t hmask, unsigned long long *hkey_b,
+                                      uint32_t *hval_b, int grid, cudaStream_t st)
+{
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(F_THREADS);
+    cfg.dynamicSmemBytes = F_SMEM;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeCooperative;   // grid barriers inside
+    attr[0].val.cooperative = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, k_in_fused_ring_pipe, T, S, slots, R, hmask, hkey_b, hval_b);
+}
+
+bool in_pipe_ok(uint32_t n, int grid)
+{
+    uint32_t ppc = (n + grid - 1) / grid;
+    ppc = (ppc + 31u) & ~31u;
+    return n > 0 && grid <= 160 && ppc <= PIPE_MAX_PPC;
+}
+
 cudaError_t launch_in_fused_ring(const DevTable &T, const InState &S, const InBatchArgs *slots,
                                  const RingRun &R, uint32_t hmask,
                                  unsigned long long *hkey_b, uint32_t *hval_b, int grid,
@@ -481,6 +830,9 @@ cudaError_t setup_in_fused_attributes()
 {
     cudaError_t e = cudaFuncSetAttribute(k_in_fused_ring, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          (int)F_SMEM);
+    if (e != cudaSuccess) return e;
+    e = cudaFuncSetAttribute(k_in_fused_ring_pipe, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)F_SMEM);
     if (e != cudaSuccess) return e;
     e = cudaFuncSetAttribute(k_in_fused<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)F_SMEM);

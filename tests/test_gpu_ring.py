@@ -123,14 +123,18 @@ def test_ring_two_kernel_and_unfused_paths(n, pipeline):
         ring.close()
 
 
-@pytest.mark.parametrize("persist", [False, True])
-def test_inbound_ring_equals_stream_launches_and_oracle(persist, monkeypatch):
-    """ESP inbound slots in a ring (graph form, and the opt-in persistent form):
-    status, inner bytes, lengths, windows and counters equal process_inbound
-    from the stream and the oracle's receiver."""
+@pytest.mark.parametrize("form", ["graph", "persistent", "pipelined"])
+def test_inbound_ring_equals_stream_launches_and_oracle(form, monkeypatch):
+    """ESP inbound slots in a ring (graph form, the opt-in plain persistent form
+    and the default software-pipelined form): status, inner bytes, lengths,
+    windows and counters equal process_inbound from the stream and the
+    oracle's receiver."""
     import torch
-    if persist:
+    if form == "graph":
+        monkeypatch.setenv("NBA_IPSEC_RING_GRAPH", "1")
+    if form == "persistent":
         monkeypatch.setenv("NBA_IPSEC_RING_IN_PERSIST", "1")
+        monkeypatch.setenv("NBA_IPSEC_RING_NOPIPE", "1")
     from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
     n_sa, n = 64, 5000
     p = gen.make_sas(n_sa, cfg_id=55)
@@ -153,7 +157,8 @@ def test_inbound_ring_equals_stream_launches_and_oracle(persist, monkeypatch):
         sa_ = [torch.zeros(ib.n, dtype=torch.uint8, device="cuda") for ib in esp]
         sb_ = [torch.zeros(ib.n, dtype=torch.uint8, device="cuda") for ib in esp]
         ring = ta.ring_inbound([(*d.args(), st, ib.n) for d, st, ib in zip(da, sa_, esp)])
-        assert ring.form == (ring.PERSISTENT if persist else ring.GRAPH)
+        assert ring.form == {"graph": ring.GRAPH, "persistent": ring.PERSISTENT,
+                             "pipelined": ring.PIPELINED}[form]
         ring.run(1)
         for d, st, ib in zip(db_, sb_, esp):
             tb.process_inbound(*d.args(), status=st, n=ib.n)
@@ -390,4 +395,62 @@ def test_pipelined_prologue_modes(n_sa, sizes):
             assert np.array_equal(g_out, o_out)
         assert np.array_equal(t.sa_seq(), oracle.sa_seq(sas, n_sa))
         assert t.counters() == ctr.as_dict()
+        ring.close()
+
+
+@pytest.mark.parametrize("n_sa,sizes", [(16, [3000, 2500, 4000]), (1024, [20000, 20000, 9000])])
+def test_inbound_pipelined_ring_mixed_stream(n_sa, sizes):
+    """The software-pipelined inbound ring (k_in_fused_ring_pipe) on traffic
+    with reordering, duplicates, stale replays, single-byte corruption,
+    invalid SA indices and SPI mismatches: one rotation over the slots, then a
+    partial rotation that replays the first two slots (every earlier packet
+    now a replay), each run against the oracle's sequential receiver
+    continuing from the same state: statuses, lengths, inner bytes, windows
+    and counters."""
+    import torch
+    from harness import esp_source
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    p = gen.make_sas(n_sa, cfg_id=70 + n_sa)
+    b, out, ol = esp_source(p, sum(sizes), "imix", 70 + n_sa)
+    r = gen.rng_for(6, salt=n_sa)
+    bs, start = [], 0
+    for k, n in enumerate(sizes):
+        order = start + gen.arrival_order(n, n, r, reorder=9, dup=0.05, old=0.05, old_span=3000)
+        order = np.clip(order, 0, sum(sizes) - 1)
+        ib = gen.esp_batch(out, b.out_off, ol, b.sa_idx, order)
+        kk = r.random(ib.n)
+        ib.sa_idx[kk < 0.01] = n_sa + 7
+        m = (kk >= 0.01) & (kk < 0.02)
+        ib.sa_idx[m] = (ib.sa_idx[m] + 1) % n_sa
+        for j in np.nonzero(r.random(ib.n) < 0.03)[0]:
+            ib.in_buf[ib.in_off[j] + int(r.integers(0, ib.in_len[j]))] ^= np.uint8(r.integers(1, 256))
+        bs.append(ib)
+        start += n
+    sas = oracle.make_sas(p)
+    win = oracle.make_windows(sas, n_sa)
+    ctr = oracle.InCounters()
+    with nba_ipsec.SATable(p, device=0, max_batch=max(x.n for x in bs)) as t:
+        t.enable_inbound()
+        ds = [device.to_device(ib, "cuda", out_fill=0xA5) for ib in bs]
+        sts = [torch.zeros(ib.n, dtype=torch.uint8, device="cuda") for ib in bs]
+        ring = t.ring_inbound([(*d.args(), st, ib.n) for d, st, ib in zip(ds, sts, bs)])
+        assert ring.form == ring.PIPELINED
+        k = 0
+        for nb in (len(bs), 2):
+            ring.run_batches(nb)
+            torch.cuda.synchronize()
+            for _ in range(nb):
+                ib = bs[k % len(bs)]
+                o_out, o_len, o_st, _ = oracle.process_inbound(sas, win, n_sa, ib, counters=ctr)
+                g_out, g_len = device.fetch(ds[k % len(bs)])
+                assert np.array_equal(sts[k % len(bs)].cpu().numpy(), o_st), f"batch {k}: status"
+                assert np.array_equal(g_len, o_len), f"batch {k}: out_len"
+                for i in np.nonzero(o_len)[0]:
+                    a, L = int(ib.out_off[i]), int(o_len[i])
+                    assert np.array_equal(g_out[a:a + L], o_out[a:a + L]), f"batch {k}: packet {i}"
+                k += 1
+            top, bmp = t.replay_window()
+            o_top, o_bmp = oracle.window_state(win, n_sa)
+            assert np.array_equal(top, o_top) and np.array_equal(bmp, o_bmp)
+            assert t.in_counters() == ctr.as_dict()
         ring.close()

@@ -57,10 +57,13 @@ print(json.dumps(out), flush=True)
 def main():
     sizes = [x if x == "imix" else int(x) for x in sys.argv[1:]] or [64, 1514, "imix"]
     for rep in range(2):
-        for form in ("graph", "persistent"):
+        for form in ("graph", "persistent", "pipelined"):
             env = dict(os.environ)
+            if form == "graph":
+                env["NBA_IPSEC_RING_GRAPH"] = "1"
             if form == "persistent":
                 env["NBA_IPSEC_RING_IN_PERSIST"] = "1"
+                env["NBA_IPSEC_RING_NOPIPE"] = "1"
             r = subprocess.run([sys.executable, "-c", CODE % {"root": ROOT, "sizes": sizes}], env=env,
                                capture_output=True, text=True)
             print(f"pass {rep} {form}", r.stdout.strip() if r.returncode == 0 else "FAILED " + r.stderr[-500:],

@@ -9,6 +9,7 @@ ring64     the bench's ring: 2 full-size 64-B slots (65,536 packets, 1024 SAs),
            3 batches in one run_batches (k_fused_ring_pipe)
 ring_small a 3,000-packet 64 B / IMIX ring in both persistent forms
 inbound    ESP inbound of an IMIX batch (k_in_fused<1>) with replays and a forgery
+inring     the software-pipelined inbound ring (k_in_fused_ring_pipe), 3 slots, 5 batches
 Each case checks its result against the oracle and prints one line."""
 import os
 import sys
@@ -87,6 +88,32 @@ def main():
             t.process_inbound(*db.args(), status=st, n=ib.n)
             g_out, g_len = device.fetch(db)
             ok = bool(np.array_equal(st.cpu().numpy(), o_st) and np.array_equal(g_len, o_len))
+    elif case == "inring":          # the software-pipelined inbound ring, 3 slots x 2 runs
+        n_sa = 33
+        p = gen.make_sas(n_sa, cfg_id=8)
+        sas0 = oracle.make_sas(p)
+        bs = []
+        for k in range(3):
+            b = gen.make_batch(3000, "imix", n_sa, cfg_id=8, batch=k)
+            e_out, e_len, _ = oracle.process_batch(sas0, n_sa, b)
+            bs.append(gen.esp_batch(e_out, b.out_off, e_len, b.sa_idx, np.arange(b.n)))
+        sas = oracle.make_sas(p)
+        win = oracle.make_windows(sas, n_sa)
+        with nba_ipsec.SATable(p, device=0, max_batch=3000) as t:
+            t.enable_inbound()
+            ds = [device.to_device(ib, "cuda") for ib in bs]
+            sts = [torch.zeros(ib.n, dtype=torch.uint8, device="cuda") for ib in bs]
+            ring = t.ring_inbound([(*d.args(), st, ib.n) for d, st, ib in zip(ds, sts, bs)])
+            ok = ring.form == ring.PIPELINED
+            ring.run_batches(3)
+            ring.run_batches(2)
+            torch.cuda.synchronize()
+            for k in list(range(3)) + [0, 1]:
+                o_st = oracle.process_inbound(sas, win, n_sa, bs[k])[2]
+            for k in (0, 1):
+                ok &= bool(np.all(sts[k].cpu().numpy() == 3))     # the replayed slots: DROP_REPLAY
+            ok &= bool(np.array_equal(sts[2].cpu().numpy(), np.zeros(bs[2].n, np.uint8)))
+            ring.close()
     else:
         raise SystemExit(f"unknown case {case}")
     print(f"{case}: result == oracle: {ok}", flush=True)
