@@ -459,6 +459,13 @@ k_in_fused_ring(DevTable T, InState S, const InBatchArgs *slots, RingRun R, uint
 // batch k clears its buffer before its first barrier, and that buffer's last
 // user (batch k - 2) finished everywhere before batch k - 1's second barrier.
 
+#ifndef NBA_RING_TRACE        // debug variant: per-(batch, CTA) phase stamps into RingRun::ts
+#define NBA_RING_TRACE 0
+#endif
+#if NBA_RING_TRACE
+#define IRTR(bi, k) (R.ts ? R.ts + ((size_t)(bi) * gridDim.x + blockIdx.x) * 16u + (k) : nullptr)
+#endif
+
 // Metadata + format checks + length order of one inbound batch by the 64
 // prologue threads (pt = 0..63) of this CTA.
 __device__ __forceinline__ void in_pipe_prologue(const DevTable &T, const InBatchArgs &B, uint32_t ppc,
@@ -481,7 +488,9 @@ __device__ __forceinline__ void in_pipe_prologue(const DevTable &T, const InBatc
 #pragma unroll
     for (uint32_t r = 0; r < PR; r++)                               // outer headers -> L2 / L1
         if (r * PIPE_P + pt < cnt) prefetch_l2(B.in_buf + mI[r]);
-    for (uint32_t r = 0; r < rounds; r++) {
+#pragma unroll
+    for (uint32_t r = 0; r < PR; r++) {                             // (unrolled: mS[r] in registers)
+        if (r >= rounds) break;
         const uint32_t j = r * PIPE_P + pt, i = p_begin + j;
         uint32_t bin = NBINS - 1;
         if (j < cnt) {
@@ -551,8 +560,9 @@ __device__ __forceinline__ void in_pipe_prologue(const DevTable &T, const InBatc
 __device__ __forceinline__ void in_pipe_tail(const DevTable &T, const InState &S, const InBatchArgs &B,
                                              FusedLo &L, FusedHi &H, uint32_t p_begin, uint32_t p_end,
                                              uint32_t hmask, uint32_t bar_base,
-                                             unsigned long long (&ctr)[N_IN_COUNTERS - 1])
+                                             unsigned long long *tr = nullptr)
 {
+    __shared__ unsigned long long s_cnt[N_IN_COUNTERS - 1];
     constexpr uint32_t HS = 2u * F_SUPER, NW = F_THREADS / 32u;
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
     const uint32_t G = gridDim.x, cta = blockIdx.x, n_sa = T.n_sa;
@@ -574,6 +584,7 @@ __device__ __forceinline__ void in_pipe_tail(const DevTable &T, const InState &S
         L.hkey[k] = INVALID_SA;
         L.hmask[k] = 0;
     }
+    if (tid < N_IN_COUNTERS - 1) s_cnt[tid] = 0;
     // per-warp group maxima [HS][NW] u32: slots < 512 in L.rkA, the rest in H.rkB
     auto gm = [&](uint32_t slot) -> uint32_t * {
         uint32_t *b = slot < 512u ? reinterpret_cast<uint32_t *>(&L.rkA[0][0])
@@ -617,13 +628,16 @@ __device__ __forceinline__ void in_pipe_tail(const DevTable &T, const InState &S
     }
     const uint32_t lmax = max(base, mex);
     __syncthreads();
+    if (tr && tid == 0) tr[6] = gtimer();
     grid_arrive(&S.ctl[CTLI_BAR]);
     grid_wait(&S.ctl[CTLI_BAR], bar_base + G);
+    if (tr && tid == 0) tr[1] = gtimer();
     if (inA) replay_hash_insert(S, key, q, i, hmask);
     scan_all_rows(S, n_sa, cta * NW + warp, G * NW, G, lane);
     __syncthreads();
     grid_arrive(&S.ctl[CTLI_BAR]);
     grid_wait(&S.ctl[CTLI_BAR], bar_base + 2u * G);
+    if (tr && tid == 0) tr[2] = gtimer();
     uint32_t st = 0xffu, D = 0, Lin = 0;
     if (live) {
         if (sa >= n_sa) {
@@ -643,11 +657,19 @@ __device__ __forceinline__ void in_pipe_tail(const DevTable &T, const InState &S
         B.out_len[i] = (uint16_t)D;
         if (B.status) B.status[i] = (uint8_t)st;
     }
-    // counters in registers (lane 0 of each warp), reduced once per run
+    // counters: pkts_ok, drop_sa, drop_format, drop_replay, drop_auth,
+    // drop_trailer, bytes_in, bytes_out (warp sums -> shared -> one atomic per CTA)
 #pragma unroll
-    for (uint32_t k = 0; k < 6; k++) ctr[k] += __reduce_add_sync(0xffffffffu, st == k ? 1u : 0u);
-    ctr[6] += __reduce_add_sync(0xffffffffu, Lin);
-    ctr[7] += __reduce_add_sync(0xffffffffu, D);
+    for (uint32_t k = 0; k < 6; k++) {
+        const uint32_t c = __reduce_add_sync(0xffffffffu, st == k ? 1u : 0u);
+        if (lane == 0 && c) atomicAdd(&s_cnt[k], (unsigned long long)c);
+    }
+    const uint32_t bi_ = __reduce_add_sync(0xffffffffu, Lin);
+    const uint32_t bo_ = __reduce_add_sync(0xffffffffu, D);
+    if (lane == 0 && bi_) atomicAdd(&s_cnt[6], (unsigned long long)bi_);
+    if (lane == 0 && bo_) atomicAdd(&s_cnt[7], (unsigned long long)bo_);
+    __syncthreads();
+    if (tid < N_IN_COUNTERS - 1 && s_cnt[tid]) atomicAdd(&S.counters[tid], s_cnt[tid]);
 }
 
 __global__ void __launch_bounds__(F_THREADS, 1)
@@ -659,7 +681,7 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
     const uint32_t G = gridDim.x, cta = blockIdx.x;
     if (n_batches == 0) return;
-    if (R.ts && cta == 0 && tid == 0) R.ts[0] = gtimer();
+    if (!NBA_RING_TRACE && R.ts && cta == 0 && tid == 0) R.ts[0] = gtimer();
     const uint32_t base0 = *reinterpret_cast<volatile uint32_t *>(&S.ctl[CTLI_BASE]);
     const uint32_t sb = smem_u32(smem);
     const uint32_t toff = (0x10000u - (sb & 0xffffu)) & 0xffffu;
@@ -688,13 +710,18 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
     }
     __syncthreads();
     tables_bulk_wait(&L.tbar, 0u);
-    unsigned long long ctr[N_IN_COUNTERS - 1] = {};
     for (uint32_t bi = 0; bi < n_batches; bi++) {
         const InBatchArgs B = slots[(first + bi) % n_slots];
         const uint32_t ppc = ppc_of(B);
         const uint32_t p_begin = cta * ppc;
         const uint32_t p_end = min(B.n, p_begin + ppc);
         const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
+#if NBA_RING_TRACE
+        unsigned long long *tr = IRTR(bi, 0);
+        if (tr && tid == 0) tr[0] = gtimer();
+#else
+        unsigned long long *tr = nullptr;
+#endif
         if (!isP) {
             const uint32_t run = L.wrun[warp];
             const uint32_t pos = 32u * run + lane;
@@ -720,12 +747,14 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
                 L.tailf[pk] = flags;
                 L.tailq[pk] = q;
             }
+            if (tr && lane == 0) atomicMax(&tr[3], gtimer());
         } else {
             bar_sync_n(2, F_THREADS);                    // every lane took its fields
             if (bi + 1 < n_batches) {
                 const InBatchArgs Bn = slots[(first + bi + 1) % n_slots];
                 in_pipe_prologue(T, Bn, ppc_of(Bn), L, pt);
             }
+            if (tr && pt == 0) tr[4] = gtimer();
         }
         __syncthreads();                                  // lanes done, bi + 1 prepared
         InState Sb = S;
@@ -733,21 +762,14 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
             Sb.hkey = hkey_b;
             Sb.hval = hval_b;
         }
-        in_pipe_tail(T, Sb, B, L, H, p_begin, p_end, hmask, base0 + 2u * bi * G, ctr);
+        in_pipe_tail(T, Sb, B, L, H, p_begin, p_end, hmask, base0 + 2u * bi * G, tr);
         __syncthreads();                                  // the tail's scratch is free again
+#if NBA_RING_TRACE
+        if (tr && tid == 0) tr[5] = gtimer();
+#else
         if (R.ts && tid == 0) atomicMax(&R.ts[1u + bi], gtimer());
+#endif
     }
-    // counters: warp sums (lane 0 holds them) -> one atomic per CTA and counter
-    __shared__ unsigned long long s_cnt[N_IN_COUNTERS - 1];
-    if (tid < N_IN_COUNTERS - 1) s_cnt[tid] = 0ull;
-    __syncthreads();
-    if (lane == 0) {
-#pragma unroll
-        for (uint32_t k = 0; k < N_IN_COUNTERS - 1; k++)
-            if (ctr[k]) atomicAdd(&s_cnt[k], ctr[k]);
-    }
-    __syncthreads();
-    if (tid < N_IN_COUNTERS - 1 && s_cnt[tid]) atomicAdd(&S.counters[tid], s_cnt[tid]);
     if (tid == 0 && cta == 0) {
         atomicAdd(&S.counters[N_IN_COUNTERS - 1], (unsigned long long)n_batches);
         S.ctl[CTLI_BASE] = base0 + 2u * n_batches * G;   // two barriers per batch

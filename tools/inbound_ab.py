@@ -44,6 +44,18 @@ for size in %(sizes)r:
             ring.run_batches(nb)
             left -= nb
     run(2 * R); torch.cuda.synchronize()
+    if %(trace)r:
+        G = 148
+        ts = torch.zeros(R * G * 16, dtype=torch.int64, device="cuda")
+        ring.set_timestamps(ts)
+        t.reset_inbound(); ring.run_batches(R); torch.cuda.synchronize()
+        v = ts.cpu().numpy().reshape(R, G, 16).astype(np.int64)[1:-1]
+        rel = (v - v[:, :, :1]) / 1e3
+        names = {1: "bar1_passed", 2: "bar2_passed", 3: "lanes_done", 4: "side_done", 5: "iter_end",
+                 6: "tail_tile_done"}
+        out[str(size)] = {n: round(float(np.median(rel[:, :, i])), 2) for i, n in names.items()}
+        ring.close(); t.close(); del esp
+        continue
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(); run(K); e1.record(); torch.cuda.synchronize()
     c = t.in_counters()
@@ -55,6 +67,13 @@ print(json.dumps(out), flush=True)
 
 
 def main():
+    if sys.argv[1:2] == ["trace"]:
+        sizes = [x if x == "imix" else int(x) for x in sys.argv[2:]] or [64, 1514, "imix"]
+        env = dict(os.environ, NBA_IPSEC_LIB=os.path.join(ROOT, "build", "variants", "trace.so"))
+        r = subprocess.run([sys.executable, "-c", CODE % {"root": ROOT, "sizes": sizes, "trace": True}],
+                           env=env, capture_output=True, text=True)
+        print("trace", r.stdout.strip() if r.returncode == 0 else "FAILED " + r.stderr[-800:])
+        return
     sizes = [x if x == "imix" else int(x) for x in sys.argv[1:]] or [64, 1514, "imix"]
     for rep in range(2):
         for form in ("graph", "persistent", "pipelined"):
@@ -64,7 +83,7 @@ def main():
             if form == "persistent":
                 env["NBA_IPSEC_RING_IN_PERSIST"] = "1"
                 env["NBA_IPSEC_RING_NOPIPE"] = "1"
-            r = subprocess.run([sys.executable, "-c", CODE % {"root": ROOT, "sizes": sizes}], env=env,
+            r = subprocess.run([sys.executable, "-c", CODE % {"root": ROOT, "sizes": sizes, "trace": False}], env=env,
                                capture_output=True, text=True)
             print(f"pass {rep} {form}", r.stdout.strip() if r.returncode == 0 else "FAILED " + r.stderr[-500:],
                   flush=True)
