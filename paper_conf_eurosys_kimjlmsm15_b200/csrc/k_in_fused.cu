@@ -633,8 +633,14 @@ __device__ __forceinline__ void in_pipe_tail(const DevTable &T, const InState &S
     grid_wait(&S.ctl[CTLI_BAR], bar_base + G);
     if (tr && tid == 0) tr[1] = gtimer();
     if (inA) replay_hash_insert(S, key, q, i, hmask);
+    if (tr) {
+        __syncwarp();
+        if (lane == 0) atomicMax(&tr[7], gtimer());
+    }
     scan_all_rows(S, n_sa, cta * NW + warp, G * NW, G, lane);
+    if (tr && lane == 0) atomicMax(&tr[8], gtimer());
     __syncthreads();
+    if (tr && tid == 0) tr[9] = gtimer();
     grid_arrive(&S.ctl[CTLI_BAR]);
     grid_wait(&S.ctl[CTLI_BAR], bar_base + 2u * G);
     if (tr && tid == 0) tr[2] = gtimer();

@@ -52,7 +52,7 @@ for size in %(sizes)r:
         v = ts.cpu().numpy().reshape(R, G, 16).astype(np.int64)[1:-1]
         rel = (v - v[:, :, :1]) / 1e3
         names = {1: "bar1_passed", 2: "bar2_passed", 3: "lanes_done", 4: "side_done", 5: "iter_end",
-                 6: "tail_tile_done"}
+                 6: "tail_tile_done", 7: "inserts_done", 8: "row_scans_done", 9: "cta_done_mid"}
         out[str(size)] = {n: round(float(np.median(rel[:, :, i])), 2) for i, n in names.items()}
         ring.close(); t.close(); del esp
         continue
