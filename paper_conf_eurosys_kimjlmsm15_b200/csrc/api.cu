@@ -514,12 +514,15 @@ int nba_ipsec_ring_create_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batc
     r->n_slots = n_slots;
     r->flow_gen = t->flow_gen;
     r->h_in_slots.assign(slots, slots + n_slots);
-    // persistent forms: the software-pipelined ring (k_in_fused_ring_pipe) when
-    // every slot fits it (<= 448 packets per SM) -- the default --, else the
-    // plain persistent ring (opt-in, NBA_IPSEC_RING_IN_PERSIST; measured
-    // against the graph form: 64 B 45.0 -> 43.3 us, 1514 B 213.9 -> 214.9 us,
-    // IMIX 107.3 -> 112.6 us), else a CUDA graph of one-kernel launches
-    bool pipe = !std::getenv("NBA_IPSEC_RING_GRAPH") && !std::getenv("NBA_IPSEC_RING_NOPIPE") &&
+    // Forms: a CUDA graph of one-kernel launches (the default); opt-in, the
+    // software-pipelined persistent ring (NBA_IPSEC_RING_IN_PIPE, every slot
+    // <= 448 packets per SM) or the plain persistent ring
+    // (NBA_IPSEC_RING_IN_PERSIST).  Measured per batch, graph / plain /
+    // pipelined: 64 B 44.8 / 43.2 / 42.0 us, 1514 B 214 / 214 / 231 us, IMIX
+    // 107 / 112 / 140 us -- the replay tail's two grid barriers couple the
+    // CTAs every batch, so the pipelined form's lanes (slower under the side
+    // warps' loads) and stragglers are paid for in full.
+    bool pipe = std::getenv("NBA_IPSEC_RING_IN_PIPE") && !std::getenv("NBA_IPSEC_RING_GRAPH") &&
                 t->allow_merged;
     bool persist = std::getenv("NBA_IPSEC_RING_IN_PERSIST") && !std::getenv("NBA_IPSEC_RING_GRAPH") &&
                    t->allow_merged;

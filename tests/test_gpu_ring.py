@@ -130,11 +130,10 @@ def test_inbound_ring_equals_stream_launches_and_oracle(form, monkeypatch):
     windows and counters equal process_inbound from the stream and the
     oracle's receiver."""
     import torch
-    if form == "graph":
-        monkeypatch.setenv("NBA_IPSEC_RING_GRAPH", "1")
     if form == "persistent":
         monkeypatch.setenv("NBA_IPSEC_RING_IN_PERSIST", "1")
-        monkeypatch.setenv("NBA_IPSEC_RING_NOPIPE", "1")
+    if form == "pipelined":
+        monkeypatch.setenv("NBA_IPSEC_RING_IN_PIPE", "1")
     from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
     n_sa, n = 64, 5000
     p = gen.make_sas(n_sa, cfg_id=55)
@@ -399,7 +398,7 @@ def test_pipelined_prologue_modes(n_sa, sizes):
 
 
 @pytest.mark.parametrize("n_sa,sizes", [(16, [3000, 2500, 4000]), (1024, [20000, 20000, 9000])])
-def test_inbound_pipelined_ring_mixed_stream(n_sa, sizes):
+def test_inbound_pipelined_ring_mixed_stream(n_sa, sizes, monkeypatch):
     """The software-pipelined inbound ring (k_in_fused_ring_pipe) on traffic
     with reordering, duplicates, stale replays, single-byte corruption,
     invalid SA indices and SPI mismatches: one rotation over the slots, then a
@@ -410,6 +409,7 @@ def test_inbound_pipelined_ring_mixed_stream(n_sa, sizes):
     import torch
     from harness import esp_source
     from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    monkeypatch.setenv("NBA_IPSEC_RING_IN_PIPE", "1")
     p = gen.make_sas(n_sa, cfg_id=70 + n_sa)
     b, out, ol = esp_source(p, sum(sizes), "imix", 70 + n_sa)
     r = gen.rng_for(6, salt=n_sa)

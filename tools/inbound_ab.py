@@ -69,7 +69,8 @@ print(json.dumps(out), flush=True)
 def main():
     if sys.argv[1:2] == ["trace"]:
         sizes = [x if x == "imix" else int(x) for x in sys.argv[2:]] or [64, 1514, "imix"]
-        env = dict(os.environ, NBA_IPSEC_LIB=os.path.join(ROOT, "build", "variants", "trace.so"))
+        env = dict(os.environ, NBA_IPSEC_LIB=os.path.join(ROOT, "build", "variants", "trace.so"),
+                   NBA_IPSEC_RING_IN_PIPE="1")
         r = subprocess.run([sys.executable, "-c", CODE % {"root": ROOT, "sizes": sizes, "trace": True}],
                            env=env, capture_output=True, text=True)
         print("trace", r.stdout.strip() if r.returncode == 0 else "FAILED " + r.stderr[-800:])
@@ -78,11 +79,10 @@ def main():
     for rep in range(2):
         for form in ("graph", "persistent", "pipelined"):
             env = dict(os.environ)
-            if form == "graph":
-                env["NBA_IPSEC_RING_GRAPH"] = "1"
             if form == "persistent":
                 env["NBA_IPSEC_RING_IN_PERSIST"] = "1"
-                env["NBA_IPSEC_RING_NOPIPE"] = "1"
+            if form == "pipelined":
+                env["NBA_IPSEC_RING_IN_PIPE"] = "1"
             r = subprocess.run([sys.executable, "-c", CODE % {"root": ROOT, "sizes": sizes, "trace": False}], env=env,
                                capture_output=True, text=True)
             print(f"pass {rep} {form}", r.stdout.strip() if r.returncode == 0 else "FAILED " + r.stderr[-500:],

@@ -89,6 +89,7 @@ def main():
             g_out, g_len = device.fetch(db)
             ok = bool(np.array_equal(st.cpu().numpy(), o_st) and np.array_equal(g_len, o_len))
     elif case == "inring":          # the software-pipelined inbound ring, 3 slots x 2 runs
+        os.environ["NBA_IPSEC_RING_IN_PIPE"] = "1"
         n_sa = 33
         p = gen.make_sas(n_sa, cfg_id=8)
         sas0 = oracle.make_sas(p)
