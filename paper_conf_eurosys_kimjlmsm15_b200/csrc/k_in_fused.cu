@@ -560,6 +560,7 @@ __device__ __forceinline__ void in_pipe_prologue(const DevTable &T, const InBatc
 __device__ __forceinline__ void in_pipe_tail(const DevTable &T, const InState &S, const InBatchArgs &B,
                                              FusedLo &L, FusedHi &H, uint32_t p_begin, uint32_t p_end,
                                              uint32_t hmask, uint32_t bar_base,
+                                             unsigned long long *next_hkey, uint32_t *next_hval,
                                              unsigned long long *tr = nullptr)
 {
     __shared__ unsigned long long s_cnt[N_IN_COUNTERS - 1];
@@ -569,11 +570,6 @@ __device__ __forceinline__ void in_pipe_tail(const DevTable &T, const InState &S
     const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
     const uint32_t j = tid, i = p_begin + j;
     const bool live = j < cnt;
-    // this batch's duplicate hash (its previous user finished everywhere)
-    for (uint32_t k = cta * F_THREADS + tid; k <= hmask; k += G * F_THREADS) {
-        S.hkey[k] = ~0ull;
-        S.hval[k] = ~0u;
-    }
     const uint32_t f = live ? L.tailf[j] : 0u;
     const uint32_t sa = live ? B.sa_idx[i] : INVALID_SA;
     const uint32_t q = (f & INF_FMT) ? L.tailq[j] : 0u;
@@ -627,12 +623,24 @@ __device__ __forceinline__ void in_pipe_tail(const DevTable &T, const InState &S
             S.hmax[(size_t)key * G + cta] = tmax;
     }
     const uint32_t lmax = max(base, mex);
+    // (sa, q) -> first index of the authenticated packets, into this batch's
+    // hash (cleared during the previous batch, before its second barrier):
+    // before the first barrier, so the atomics overlap the wait for the
+    // slowest CTA
+    if (inA) replay_hash_insert(S, key, q, i, hmask);
     __syncthreads();
     if (tr && tid == 0) tr[6] = gtimer();
     grid_arrive(&S.ctl[CTLI_BAR]);
     grid_wait(&S.ctl[CTLI_BAR], bar_base + G);
     if (tr && tid == 0) tr[1] = gtimer();
-    if (inA) replay_hash_insert(S, key, q, i, hmask);
+    // the next batch's hash: its last user (the batch before this one) made
+    // its lookups before this batch's first barrier; every CTA clears its
+    // slice before arriving at the second barrier, which the next batch's
+    // inserts follow
+    for (uint32_t k = cta * F_THREADS + tid; k <= hmask; k += G * F_THREADS) {
+        next_hkey[k] = ~0ull;
+        next_hval[k] = ~0u;
+    }
     if (tr) {
         __syncwarp();
         if (lane == 0) atomicMax(&tr[7], gtimer());
@@ -702,7 +710,14 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
     const uint32_t lane4r = (lane * 4u) | (smem_u32(tabs) & 0xffff0000u);
     tables_stage(tabs, T, &L.tbar, true);   // bulk copy, waited for before the first lookup
     if (tid < NBINS) L.bins[tid] = 0u;
+    // the first batch's duplicate hash, cleared by every CTA before a start
+    // barrier that the first inserts (after the first batch's lanes) follow
+    for (uint32_t k = cta * F_THREADS + tid; k <= hmask; k += G * F_THREADS) {
+        S.hkey[k] = ~0ull;
+        S.hval[k] = ~0u;
+    }
     __syncthreads();
+    grid_arrive(&S.ctl[CTLI_BAR]);
     const bool isP = tid >= PIPE_MAX_PPC;
     const uint32_t pt = tid - PIPE_MAX_PPC;
     auto ppc_of = [&](const InBatchArgs &B) {
@@ -716,6 +731,8 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
     }
     __syncthreads();
     tables_bulk_wait(&L.tbar, 0u);
+    grid_wait(&S.ctl[CTLI_BAR], base0 + G);          // the start barrier (long since complete)
+    const uint32_t bbase = base0 + G;                 // batch bi: barriers bbase + 2 bi G + {G, 2G}
     for (uint32_t bi = 0; bi < n_batches; bi++) {
         const InBatchArgs B = slots[(first + bi) % n_slots];
         const uint32_t ppc = ppc_of(B);
@@ -768,7 +785,8 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
             Sb.hkey = hkey_b;
             Sb.hval = hval_b;
         }
-        in_pipe_tail(T, Sb, B, L, H, p_begin, p_end, hmask, base0 + 2u * bi * G, tr);
+        in_pipe_tail(T, Sb, B, L, H, p_begin, p_end, hmask, bbase + 2u * bi * G,
+                     (bi & 1u) ? S.hkey : hkey_b, (bi & 1u) ? S.hval : hval_b, tr);
         __syncthreads();                                  // the tail's scratch is free again
 #if NBA_RING_TRACE
         if (tr && tid == 0) tr[5] = gtimer();
@@ -778,7 +796,7 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
     }
     if (tid == 0 && cta == 0) {
         atomicAdd(&S.counters[N_IN_COUNTERS - 1], (unsigned long long)n_batches);
-        S.ctl[CTLI_BASE] = base0 + 2u * n_batches * G;   // two barriers per batch
+        S.ctl[CTLI_BASE] = bbase + 2u * n_batches * G;   // a start barrier, two per batch
     }
 }
 
