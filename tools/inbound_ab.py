@@ -53,7 +53,13 @@ for size in %(sizes)r:
         rel = (v - v[:, :, :1]) / 1e3
         names = {1: "bar1_passed", 2: "bar2_passed", 3: "lanes_done", 4: "side_done", 5: "iter_end",
                  6: "tail_tile_done", 7: "inserts_done", 8: "row_scans_done", 9: "cta_done_mid"}
-        out[str(size)] = {n: round(float(np.median(rel[:, :, i])), 2) for i, n in names.items()}
+        out[str(size)] = {n: [round(float(np.median(rel[:, :, i])), 2),
+                              round(float(np.median(np.max(rel[:, :, i], axis=1))), 2)]
+                          for i, n in names.items()}
+        lanes = rel[:, :, 3]
+        order = np.argsort(-np.median(lanes, axis=0))[:6]
+        out[str(size)]["slowest_ctas_lanes_us"] = [(int(c), round(float(np.median(lanes[:, c])), 2))
+                                                  for c in order]
         ring.close(); t.close(); del esp
         continue
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)

@@ -53,6 +53,10 @@ for size in %(sizes)r:
         ok = lambda i: bool(np.all(v[:, :, i] > 0))
         med = {n: round(float(np.median(rel[:, :, i])), 2) for i, n in enumerate(names) if i and ok(i)}
         p90 = {n: round(float(np.percentile(rel[:, :, i], 90)), 2) for i, n in enumerate(names) if i and ok(i)}
+        lanes = rel[:, :, 3]
+        order = np.argsort(-np.median(lanes, axis=0))[:6]
+        p90["slowest_ctas_lanes_us"] = [(int(c), round(float(np.median(lanes[:, c])), 2)) for c in order]
+        p90["lanes_done_max_over_ctas"] = round(float(np.median(np.max(lanes, axis=1))), 2)
         it = np.diff(v[:, 0, 0]) / 1e3
         out[str(size)] = {"median_us": med, "p90_us": p90, "iter_us": float(np.median(it))}
     else:
