@@ -130,19 +130,25 @@ __device__ __forceinline__ uint32_t replay_decide(const InState &S, uint32_t s, 
 }
 
 // (s, q) -> smallest packet index i among the authenticated packets
-__device__ __forceinline__ void replay_hash_insert(const InState &S, uint32_t s, uint32_t q, uint32_t i,
-                                                   uint32_t hmask)
+__device__ __forceinline__ void replay_hash_insert(unsigned long long *hkey, uint32_t *hval, uint32_t s,
+                                                   uint32_t q, uint32_t i, uint32_t hmask)
 {
     const unsigned long long k64 = ((unsigned long long)s << 32) | q;
     uint32_t h = hash_slot(k64, hmask);
     while (true) {
-        const unsigned long long old = atomicCAS(&S.hkey[h], ~0ull, k64);
+        const unsigned long long old = atomicCAS(&hkey[h], ~0ull, k64);
         if (old == ~0ull || old == k64) {
-            atomicMin(&S.hval[h], i);
+            atomicMin(&hval[h], i);
             break;
         }
         h = (h + 1u) & hmask;
     }
+}
+
+__device__ __forceinline__ void replay_hash_insert(const InState &S, uint32_t s, uint32_t q, uint32_t i,
+                                                   uint32_t hmask)
+{
+    replay_hash_insert(S.hkey, S.hval, s, q, i, hmask);
 }
 
 }  // namespace nba

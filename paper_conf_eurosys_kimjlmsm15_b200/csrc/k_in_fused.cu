@@ -623,11 +623,8 @@ __device__ __forceinline__ void in_pipe_tail(const DevTable &T, const InState &S
             S.hmax[(size_t)key * G + cta] = tmax;
     }
     const uint32_t lmax = max(base, mex);
-    // (sa, q) -> first index of the authenticated packets, into this batch's
-    // hash (cleared during the previous batch, before its second barrier):
-    // before the first barrier, so the atomics overlap the wait for the
-    // slowest CTA
-    if (inA) replay_hash_insert(S, key, q, i, hmask);
+    // ((sa, q) -> first index of the authenticated packets went into this
+    // batch's hash from the lanes, right after each packet's ICV check)
     __syncthreads();
     if (tr && tid == 0) tr[6] = gtimer();
     grid_arrive(&S.ctl[CTLI_BAR]);
@@ -766,6 +763,13 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
                     expand_key_lane(lane4r, r0, r1, r2, L, H, tid);
                     flags = INF_FMT | esp_in_packet(T, B, L, H, lane4r, tid, sa, info & 0xffffu, q, iv0,
                                                     iv1, inoff, outoff, r0, r1, r2, hd, h0, h1);
+                    // (sa, q) -> first index into this batch's duplicate hash
+                    // (cleared during the previous batch, before its second
+                    // barrier; read after this batch's first): the atomics'
+                    // latency overlaps the other lanes' crypto
+                    if (flags & INF_ICV)
+                        replay_hash_insert((bi & 1u) ? hkey_b : S.hkey, (bi & 1u) ? hval_b : S.hval, sa,
+                                           q, p_begin + pk, hmask);
                 }
                 L.tailf[pk] = flags;
                 L.tailq[pk] = q;
