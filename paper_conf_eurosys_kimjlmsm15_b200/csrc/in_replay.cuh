@@ -12,6 +12,24 @@ __device__ __forceinline__ uint32_t hash_slot(unsigned long long key, uint32_t h
     return (uint32_t)((key * 0x9E3779B97F4A7C15ull) >> 32) & hmask;
 }
 
+// Max of v over the earlier lanes of this lane's group (lt = the group's lanes
+// below this one; 0 when none): one shuffle per earlier group member, the
+// loop warp-uniform over the largest such count (a group's lanes share a
+// key, so with many SAs a group has one or two lanes per warp) instead of 32
+// shuffles.  All 32 lanes call it.
+__device__ __forceinline__ uint32_t group_prefix_max(uint32_t lt, uint32_t v)
+{
+    uint32_t m = lt, mex = 0;
+    const uint32_t rounds = __reduce_max_sync(0xffffffffu, (uint32_t)__popc(lt));
+    for (uint32_t k = 0; k < rounds; k++) {
+        const uint32_t l = m ? (uint32_t)(__ffs(m) - 1) : (threadIdx.x & 31u);
+        const uint32_t x = __shfl_sync(0xffffffffu, v, l);
+        if (m) mex = max(mex, x);
+        m &= m - 1u;
+    }
+    return mex;
+}
+
 __device__ __forceinline__ void window_advance(const InState &S, uint32_t sa, uint32_t batch_max)
 {
     const uint32_t t0 = S.top[sa];

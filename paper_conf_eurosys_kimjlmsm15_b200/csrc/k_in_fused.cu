@@ -220,12 +220,7 @@ __device__ __forceinline__ void in_merged_tail(const DevTable &T, const InState 
     uint32_t(*gm)[NW] = reinterpret_cast<uint32_t(*)[NW]>(tabs);
     const uint32_t peers = __match_any_sync(0xffffffffu, key);
     const uint32_t lt = peers & lanemask_lt();
-    uint32_t mex = 0;                                // max over earlier lanes of the group
-#pragma unroll
-    for (int l = 0; l < 32; l++) {
-        const uint32_t v = __shfl_sync(0xffffffffu, qa, l);
-        if ((lt >> l) & 1u) mex = max(mex, v);
-    }
+    const uint32_t mex = group_prefix_max(lt, qa);   // max over earlier lanes of the group
     const uint32_t leader = __ffs(peers) - 1, hi_lane = 31u - __clz(peers);
     const uint32_t gmax = __shfl_sync(0xffffffffu, max(mex, qa), hi_lane);
     __syncthreads();   // CTA hash initialised, T-tables no longer read
@@ -589,12 +584,7 @@ __device__ __forceinline__ void in_pipe_tail(const DevTable &T, const InState &S
     };
     const uint32_t peers = __match_any_sync(0xffffffffu, key);
     const uint32_t lt = peers & lanemask_lt();
-    uint32_t mex = 0;                                // max over earlier lanes of the group
-#pragma unroll
-    for (int l = 0; l < 32; l++) {
-        const uint32_t v = __shfl_sync(0xffffffffu, qa, l);
-        if ((lt >> l) & 1u) mex = max(mex, v);
-    }
+    const uint32_t mex = group_prefix_max(lt, qa);   // max over earlier lanes of the group
     const uint32_t leader = __ffs(peers) - 1, hi_lane = 31u - __clz(peers);
     const uint32_t gmax = __shfl_sync(0xffffffffu, max(mex, qa), hi_lane);
     __syncthreads();   // CTA hash initialised, round-key slots no longer read

@@ -79,12 +79,7 @@ k_in_replay(DevTable T, InState S, InBatchArgs B, uint32_t n_tiles, uint32_t hma
     }
     const uint32_t peers = __match_any_sync(0xffffffffu, key);
     const uint32_t lt = peers & lanemask_lt();
-    uint32_t mex = 0;                                // max over earlier lanes of the group
-#pragma unroll
-    for (int l = 0; l < 32; l++) {
-        const uint32_t v = __shfl_sync(0xffffffffu, q, l);
-        if ((lt >> l) & 1u) mex = max(mex, v);
-    }
+    const uint32_t mex = group_prefix_max(lt, q);   // max over earlier lanes of the group
     const uint32_t leader = __ffs(peers) - 1;
     const uint32_t hi_lane = 31u - __clz(peers);
     const uint32_t gmax = __shfl_sync(0xffffffffu, max(mex, q), hi_lane);
