@@ -40,7 +40,8 @@ struct FusedLo {
                                    //   its "early round keys" decision
     unsigned long long tbar;       // mbarrier: the bulk copy of the T-table image landed
     uint32_t tailf[448];           // inbound pipelined ring: a batch's per-packet flags and
-    uint32_t tailq[448];           //   sequence numbers (by packet index) for its replay tail
+    uint32_t tailq[448];           //   sequence numbers and SA indices (by packet index) for
+    uint32_t tails[448];           //   its replay tail
     uint32_t stag_ns;              // pipelined ring: start delay of the upper lane warps
     uint32_t stag_acc;             //   (AES step 0 of the lower ones, measured per batch)
 };

@@ -566,7 +566,7 @@ __device__ __forceinline__ void in_pipe_tail(const DevTable &T, const InState &S
     const uint32_t j = tid, i = p_begin + j;
     const bool live = j < cnt;
     const uint32_t f = live ? L.tailf[j] : 0u;
-    const uint32_t sa = live ? B.sa_idx[i] : INVALID_SA;
+    const uint32_t sa = live ? L.tails[j] : INVALID_SA;
     const uint32_t q = (f & INF_FMT) ? L.tailq[j] : 0u;
     const uint32_t key = (f & INF_FMT) ? sa : INVALID_SA;
     const bool inA = (f & INF_ICV) != 0u;
@@ -738,7 +738,8 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
             const bool have = run != 0xffu && pos < cnt;
             const uint32_t pk = have ? L.perm[pos] : 0u;
             const uint32_t info = have ? L.info[pk] : 0u;
-            const uint32_t sa = (info & INFO_OK) ? L.sa[pk] : INVALID_SA;
+            const uint32_t sa_raw = have ? L.sa[pk] : INVALID_SA;   // (the tail tells DROP_SA apart)
+            const uint32_t sa = (info & INFO_OK) ? sa_raw : INVALID_SA;
             const uint32_t q = have ? L.seq[pk] : 0u;
             const uint32_t iv0 = have ? L.aux0[pk] : 0u, iv1 = have ? L.aux1[pk] : 0u;
             const uint32_t inoff = have ? L.inoff[pk] : 0u, outoff = have ? L.outoff[pk] : 0u;
@@ -763,6 +764,7 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
                 }
                 L.tailf[pk] = flags;
                 L.tailq[pk] = q;
+                L.tails[pk] = sa_raw;
             }
             if (tr && lane == 0) atomicMax(&tr[3], gtimer());
         } else {
