@@ -348,7 +348,7 @@ def rates(ctx, res, steps, ms=None):
             "ms_per_step": ms_max / steps}
 
 
-def measure_inbound(ctx, args, cfg_id, steps, warmup):
+def measure_inbound(ctx, args, cfg_id, steps, warmup, form=None):
     """ESP inbound on the same traffic: the library's own outbound
     output of R consecutive batches of the config (> 2x L2 touched per
     rotation, every batch L2-cold), each in its own device buffers,
@@ -374,8 +374,13 @@ def measure_inbound(ctx, args, cfg_id, steps, warmup):
     t_out.close()
     t = nba_ipsec.SATable(p, device=ctx.local, max_batch=PKTS_PER_GPU)
     t.enable_inbound()
-    ring = t.ring_inbound([(e[0], db.out_off, e[1], db.sa_idx, e[2], db.out_off, e[3], None, b.n)
-                           for e in esp])
+    if form == "pipelined":          # the opt-in software-pipelined inbound ring
+        os.environ["NBA_IPSEC_RING_IN_PIPE"] = "1"
+    try:
+        ring = t.ring_inbound([(e[0], db.out_off, e[1], db.sa_idx, e[2], db.out_off, e[3], None, b.n)
+                               for e in esp])
+    finally:
+        os.environ.pop("NBA_IPSEC_RING_IN_PIPE", None)
 
     def timed_batches(k_steps):
         left = k_steps
@@ -719,6 +724,10 @@ def run_ours(args):
             inbound[size_key(CFG_SIZE[cfg_id])] = measure_inbound(ctx, args, cfg_id,
                                                                  max(10, steps // 4),
                                                                  max(3, warmup // 2))
+        # the opt-in software-pipelined inbound ring (faster for small packets,
+        # slower for large ones), on the same traffic
+        inbound["64_pipelined_ring"] = measure_inbound(ctx, args, 2, max(10, steps // 4),
+                                                       max(3, warmup // 2), form="pipelined")
     flows = None
     if not args.no_inbound:
         flows = measure_flows(ctx, args, main_cfg, max(10, steps // 4), max(3, warmup // 2))
