@@ -461,8 +461,11 @@ __device__ __forceinline__ CtrPre ctr_precompute(uint32_t lane4r, const uint4 &r
 
 // Keystream of counter blocks 4 it + 1 .. 4 it + 4 (rounds 3..10; round keys
 // 3..10 of this thread's packet staged in L.rkA / H.rkB), as 16 LE words.
+// rkl / rkh: round keys 3..6 at rkl[(r - 3) * F_THREADS + slot], 7..10 at
+// rkh[(r - 7) * F_THREADS + slot] (the thread's own slots in L.rkA / H.rkB, or
+// other slots of the same arrays).
 __device__ __forceinline__ void aes4_keystream(uint32_t lane4r, const CtrPre &c, uint32_t it,
-                                               const FusedLo &L, const FusedHi &H, uint32_t tid,
+                                               const uint4 *rkl, const uint4 *rkh, uint32_t slot,
                                                uint32_t (&ks)[16])
 {
     uint32_t x[4][4];
@@ -476,7 +479,7 @@ __device__ __forceinline__ void aes4_keystream(uint32_t lane4r, const CtrPre &c,
     }
 #pragma unroll 1
     for (int r = 0; r < 7; r++) {
-        const uint4 rk = r < 4 ? L.rkA[r][tid] : H.rkB[r - 4][tid];
+        const uint4 rk = r < 4 ? rkl[r * F_THREADS + slot] : rkh[(r - 4) * F_THREADS + slot];
 #pragma unroll
         for (int b = 0; b < 4; b++) {
             const uint32_t u0 = TL(x[b][0], 0, 0) ^ TL(x[b][1], 1, 1) ^ TL(x[b][2], 2, 2) ^ TL(x[b][3], 3, 3) ^ rk.x;
@@ -489,7 +492,7 @@ __device__ __forceinline__ void aes4_keystream(uint32_t lane4r, const CtrPre &c,
             x[b][3] = u3;
         }
     }
-    const uint4 rk = H.rkB[3][tid];
+    const uint4 rk = rkh[3 * F_THREADS + slot];
 #define NBA_FINAL(s0, s1, s2, s3)                                                               \
     ((TL(s0, 0, 2) & 0x000000ffu) | (TL(s1, 1, 3) & 0x0000ff00u) | (TL(s2, 2, 0) & 0x00ff0000u) | \
      (TL(s3, 3, 1) & 0xff000000u))
@@ -503,6 +506,13 @@ __device__ __forceinline__ void aes4_keystream(uint32_t lane4r, const CtrPre &c,
 #undef NBA_FINAL
 }
 
+__device__ __forceinline__ void aes4_keystream(uint32_t lane4r, const CtrPre &c, uint32_t it,
+                                               const FusedLo &L, const FusedHi &H, uint32_t tid,
+                                               uint32_t (&ks)[16])
+{
+    aes4_keystream(lane4r, c, it, &L.rkA[0][0], &H.rkB[0][0], tid, ks);
+}
+
 // FIPS-197 §5.2 KeyExpansion of the lane's AES-128 key (round key 0 = r0) in
 // registers, SubWord through the S-box bytes of the T-tables (the S-box value
 // is byte 0 of T2[x], byte 1 of T3[x], byte 2 of T0[x], byte 3 of T1[x]);
@@ -510,8 +520,8 @@ __device__ __forceinline__ void aes4_keystream(uint32_t lane4r, const CtrPre &c,
 // which state byte indexes which table.  Round keys 1 and 2 are returned (the
 // CTR precompute uses them), 3..10 go to L.rkA / H.rkB[.][tid].  40 lookups and
 // ~100 ALU ops per packet replace 160 bytes of round-key loads per packet.
-__device__ __forceinline__ void expand_key_lane(uint32_t lane4r, const uint4 &r0, uint4 &r1, uint4 &r2,
-                                                FusedLo &L, FusedHi &H, uint32_t tid)
+__device__ __forceinline__ void expand_key_slots(uint32_t lane4r, const uint4 &r0, uint4 &r1, uint4 &r2,
+                                                 uint4 *rkl, uint4 *rkh, uint32_t slot)
 {
     uint32_t w0 = r0.x, w1 = r0.y, w2 = r0.z, w3 = r0.w;
     uint32_t rc = 1u;
@@ -527,9 +537,15 @@ __device__ __forceinline__ void expand_key_lane(uint32_t lane4r, const uint4 &r0
         const uint4 k = make_uint4(w0, w1, w2, w3);
         if (r == 1) r1 = k;
         else if (r == 2) r2 = k;
-        else if (r <= 6) L.rkA[r - 3][tid] = k;
-        else H.rkB[r - 7][tid] = k;
+        else if (r <= 6) rkl[(r - 3) * F_THREADS + slot] = k;
+        else rkh[(r - 7) * F_THREADS + slot] = k;
     }
+}
+
+__device__ __forceinline__ void expand_key_lane(uint32_t lane4r, const uint4 &r0, uint4 &r1, uint4 &r2,
+                                                FusedLo &L, FusedHi &H, uint32_t tid)
+{
+    expand_key_slots(lane4r, r0, r1, r2, &L.rkA[0][0], &H.rkB[0][0], tid);
 }
 
 // Round keys 3..10 of the lane's SA (FIPS-197 §5.2 schedule, built once per

@@ -61,6 +61,9 @@ namespace nba {
 #ifndef NBA_PIPE_STAGGER      // pipelined ring: lane warps 7..13 start their packets later by
 #define NBA_PIPE_STAGGER 128  //   STAGGER/256 x the time the lower warps took to their first AES
 #endif                        //   step (previous batch), so AES (LDS) and SHA-1 (ALU) overlap
+#ifndef NBA_PIPE_SPLIT        // pipelined ring: batches of one-AES-step packets run on producer
+#define NBA_PIPE_SPLIT 1      //   (AES) and consumer (SHA-1) warps (split_produce / _consume)
+#endif
 #ifndef NBA_PIPE_ONEBIN       // pipelined ring: one-length-bin batches keep index order (no sort)
 #define NBA_PIPE_ONEBIN 1
 #endif
@@ -293,6 +296,154 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
         dbg[4] = ck_end - ck_sha;          // the rest
         dbg[5] = st[0];
     }
+}
+
+// ---------------------------------- one-step packets, producer / consumer warps
+// For a batch whose packets all fit one 64-byte AES step (C <= 64: frames up to
+// 76 bytes), the pipelined ring can split each packet's work between two
+// kinds of warps instead of one lane doing AES then SHA-1: PRODUCER threads
+// (warps 0..5) run the AES-CTR step and write the ciphertext into a shared
+// staging slot, CONSUMER threads (warps 6..13) wait for it and run the three
+// SHA-1 compressions and the output stream.  With every lane doing AES first
+// and SHA-1 second, the SM's shared-memory pipe and ALU pipe take turns;
+// split, the shared-memory-bound AES of some packets runs beside the ALU-bound
+// SHA-1 of others.  Same arithmetic and results as esp_packet.
+constexpr uint32_t SPLIT_PROD = 192;          // producer threads (warps 0..5)
+constexpr uint32_t SPLIT_CONS = PIPE_MAX_PPC - SPLIT_PROD;          // 256 consumers
+
+// Producer: packet with datagram length D, sequence number q32: the 16 words
+// of T xor keystream (C <= 64) into the staging slot ct[0..3][j] (uint4 x 4).
+__device__ __forceinline__ void split_produce(const DevTable &T, const BatchArgs &B, FusedLo &L,
+                                              FusedHi &H, uint32_t lane4r, uint32_t slot, uint32_t sa,
+                                              uint32_t info, uint32_t q32, uint32_t inoff, uint32_t j)
+{
+    const uint32_t D = info & 0x7ffu;
+    const uint32_t pad = esp_pad(D);
+    const uint32_t C = D + pad + 2u;
+    const uint32_t Cw = C >> 2;
+    uint4 r0, hd, r1, r2;
+    const uint4 *line = T.sal + (size_t)sa * SAL_U4;
+    ldg_nc_v8(&line[0], r0, hd);
+    const uint8_t *src = B.in_buf + inoff;
+    // round keys 3..6 -> L.rkA[.][slot], 7..10 -> L.rkA[.][256 + slot]
+    uint4 *rkl = &L.rkA[0][0], *rkh = &L.rkA[0][256];
+    expand_key_slots(lane4r, r0, r1, r2, rkl, rkh, slot);
+    const CtrPre cp = ctr_precompute(lane4r, r0, r1, r2, hd.y, 0u, bswap32(q32));
+    Raw6 raw;      // the payload's loads in flight during the AES rounds
+    load_raw6(reinterpret_cast<uintptr_t>(src), reinterpret_cast<uintptr_t>(src) + D, raw);
+    uint32_t ks[16], ct[16];
+    aes4_keystream(lane4r, cp, 0u, rkl, rkh, slot, ks);
+    extract16(raw, ct);
+    {   // trailer (C = 0 mod 4): the last word and, when p = 3, the one before
+        const uint32_t lw = Cw - 1u;
+        const uint32_t keep = pad == 0 ? 0x0000ffffu : pad == 1 ? 0x000000ffu : 0u;
+        const uint32_t trl = pad == 0 ? 0x04000000u : pad == 1 ? 0x04010100u
+                           : pad == 2 ? 0x04020201u : 0x04030302u;
+#pragma unroll
+        for (int w = 0; w < 16; w++) {
+            if ((uint32_t)w == lw) ct[w] = (ct[w] & keep) | trl;
+            if (pad == 3u && (uint32_t)w + 1u == lw) ct[w] = (ct[w] & 0x00ffffffu) | 0x01000000u;
+        }
+    }
+#pragma unroll
+    for (int w = 0; w < 16; w++) ct[w] ^= ks[w];
+    uint4 *stg = &H.rkB[0][0];
+#pragma unroll
+    for (int k = 0; k < 4; k++)
+        stg[k * F_THREADS + j] = make_uint4(ct[4 * k], ct[4 * k + 1], ct[4 * k + 2], ct[4 * k + 3]);
+}
+
+// Consumer: the staged ciphertext of packet j -> outer header, ESP header,
+// ciphertext, HMAC-SHA1-96 (as esp_packet's SHA-1 part, one AES step).
+__device__ __forceinline__ void split_consume(const DevTable &T, const BatchArgs &B, FusedHi &H,
+                                              uint32_t sa, uint32_t info, uint32_t q32, uint32_t inoff,
+                                              uint32_t outoff, uint32_t j)
+{
+    const uint32_t D = info & 0x7ffu;
+    const uint32_t pad = esp_pad(D);
+    const uint32_t C = D + pad + 2u;
+    const uint32_t Lb = 48u + C;
+    const uint32_t Cw = C >> 2;
+    const uint32_t Mw = 4u + Cw;
+    const uint32_t nb_in = (4u * Mw + 8u) / 64u + 1u;
+    const uint32_t bitlen = (64u + 4u * Mw) * 8u;
+    uint4 hd, h0, h1, dummy;
+    const uint4 *line = T.sal + (size_t)sa * SAL_U4;
+    ldg_nc_v8(&line[0], dummy, hd);
+    ldg_nc_v8(&line[2], h0, h1);
+    const uint32_t tos = (uint32_t)__ldg(B.in_buf + inoff + 1);
+    const uint32_t qbe = bswap32(q32);
+    uint32_t ct[16];
+    {
+        const uint4 *stg = &H.rkB[0][0];
+#pragma unroll
+        for (int k = 0; k < 4; k++) {
+            const uint4 v = stg[k * F_THREADS + j];
+            ct[4 * k] = v.x;
+            ct[4 * k + 1] = v.y;
+            ct[4 * k + 2] = v.z;
+            ct[4 * k + 3] = v.w;
+        }
+    }
+    OutStream os;
+    os.init(B.out_buf + outoff);
+    {
+        const uint32_t src = bswap32(hd.z), dst = bswap32(hd.w);
+        uint32_t sum = (0x4500u | tos) + Lb + 0x4000u + ((64u << 8) | 50u) + (src >> 16) +
+                       (src & 0xffffu) + (dst >> 16) + (dst & 0xffffu);
+        sum = (sum & 0xffffu) + (sum >> 16);
+        sum = (sum & 0xffffu) + (sum >> 16);
+        const uint32_t cs = ~sum & 0xffffu;
+        os.put(0x45u | (tos << 8) | ((Lb >> 8) << 16) | ((Lb & 0xffu) << 24));
+        os.put(0x00400000u);
+        os.put(64u | (50u << 8) | ((cs >> 8) << 16) | ((cs & 0xffu) << 24));
+        os.put(hd.z);
+        os.put(hd.w);
+        os.put(hd.x);
+        os.put(qbe);
+        os.put(0u);
+        os.put(qbe);
+    }
+    if (Cw == 16u) {
+        os.put16(ct);
+    } else {
+#pragma unroll
+        for (int w = 0; w < 16; w++)
+            if ((uint32_t)w < Cw) os.put(ct[w]);
+    }
+    uint32_t carry[4] = {bswap32(hd.x), q32, 0u, q32};
+    uint32_t st[5] = {h0.x, h0.y, h0.z, h0.w, h1.x};
+#pragma unroll 1
+    for (uint32_t it = 0; it <= nb_in; it++) {
+        uint32_t W[16];
+        if (it < nb_in) {
+            const uint32_t m0 = 16u * it;
+#pragma unroll
+            for (int i = 0; i < 16; i++) {
+                const uint32_t m = m0 + i;
+                const uint32_t msg = i < 4 ? carry[i] : (it == 0 ? bswap32(ct[i - 4]) : 0u);
+                W[i] = m < Mw ? msg : (m == Mw ? 0x80000000u : 0u);
+            }
+            if (it == nb_in - 1u) W[15] = bitlen;
+#pragma unroll
+            for (int i = 0; i < 4; i++) carry[i] = bswap32(ct[12 + i]);
+        } else {
+#pragma unroll
+            for (int i = 0; i < 5; i++) W[i] = st[i];
+            W[5] = 0x80000000u;
+#pragma unroll
+            for (int i = 6; i < 15; i++) W[i] = 0u;
+            W[15] = (64u + 20u) * 8u;
+            uint4 g4, g5;
+            ldg_nc_v8(&T.sal[(size_t)sa * SAL_U4 + 4], g4, g5);
+            st[0] = g5.x; st[1] = g5.y; st[2] = g5.z; st[3] = g4.x; st[4] = g4.y;
+        }
+        sha1_compress_fma(st, W, T.n_sa != 0u ? 1u : 0u);
+    }
+    os.put(bswap32(st[0]));
+    os.put(bswap32(st[1]));
+    os.put(bswap32(st[2]));
+    os.finish(B.out_buf + outoff + Lb);
 }
 
 // ------------------------------------------- merged prologue (row a1 in-kernel)
@@ -1136,6 +1287,7 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
         L.stag_ns = 0u;
         L.stag_acc = 0u;
     }
+    for (uint32_t k = tid; k < PIPE_MAX_PPC; k += F_THREADS) L.tailf[k] = 0u;   // split: ready flags
     for (uint32_t k = tid; k < 2u * F_SUPER; k += F_THREADS) {
         L.hkey[k] = INVALID_SA;
         L.hmask[k] = 0u;
@@ -1183,8 +1335,10 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
         const bool early = NBA_PIPE_EARLY_KEYS == 1 ? true
                          : NBA_PIPE_EARLY_KEYS == 0 ? false : (L.pstat[2] & 1u) != 0u;
         const bool uniform = (L.pstat[2] & 4u) != 0u;    // the batch's packets share one length bin
+        // one AES step per packet (and at most 448): producer / consumer warps
+        const bool split = NBA_PIPE_SPLIT && L.pstat[1] <= 1u;
         PktPre pp = {};
-        if (!isP) {
+        if (!isP && !split) {
             const uint32_t run = L.wrun[warp];          // LPT placement of the runs
             const uint32_t pos = 32u * run + lane;
             have = run != 0xffu && pos < cnt;
@@ -1215,7 +1369,76 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
 #else
         pipe_sequence(T, work_of(bi), B, ppc, base0 + (bi + 1) * G, epoch_of(bi), L);
 #endif
-        if (!isP) {
+        if (!isP && split) {
+            const uint32_t ep = bi + 1u;                 // ready-flag value of this batch
+            volatile uint32_t *ready = L.tailf;
+            if (tid < SPLIT_PROD) {
+                // producer: packets tid, tid + 192, tid + 384
+                uint32_t f_info[3], f_sa[3], f_q[3], f_in[3];
+#pragma unroll
+                for (uint32_t k = 0; k < 3u; k++) {
+                    const uint32_t j = tid + k * SPLIT_PROD;
+                    f_info[k] = j < cnt ? L.info[j] : 0u;
+                    f_sa[k] = j < cnt ? L.sa[j] : 0u;
+                    f_q[k] = j < cnt ? L.seq[j] : 0u;
+                    f_in[k] = j < cnt ? L.inoff[j] : 0u;
+                }
+                bar_arrive_n(2, F_THREADS);              // fields taken: the arrays are free
+#define NBA_SEL3(a, k) ((k) == 0u ? a[0] : (k) == 1u ? a[1] : a[2])   // (no local memory)
+#pragma unroll 1
+                for (uint32_t k = 0; k < 3u; k++) {
+                    const uint32_t j = tid + k * SPLIT_PROD;
+                    const uint32_t info_k = NBA_SEL3(f_info, k), q_k = NBA_SEL3(f_q, k);
+                    if (j < cnt && (info_k & INFO_OK) && q_k != 0u && !NBA_PROLOGUE_ONLY) {
+                        split_produce(T, B, L, H, lane4r, tid, NBA_SEL3(f_sa, k), info_k, q_k,
+                                      NBA_SEL3(f_in, k), j);
+                        __threadfence_block();
+                        ready[j] = ep;
+                    }
+                }
+            } else {
+                // consumer: packets u, u + 256 (u = tid - 192)
+                const uint32_t u = tid - SPLIT_PROD;
+                uint32_t f_info[2], f_sa[2], f_q[2], f_in[2], f_out[2];
+#pragma unroll
+                for (uint32_t k = 0; k < 2u; k++) {
+                    const uint32_t j = u + k * SPLIT_CONS;
+                    f_info[k] = j < cnt ? L.info[j] : 0u;
+                    f_sa[k] = j < cnt ? L.sa[j] : 0u;
+                    f_q[k] = j < cnt ? L.seq[j] : 0u;
+                    f_in[k] = j < cnt ? L.inoff[j] : 0u;
+                    f_out[k] = j < cnt ? L.outoff[j] : 0u;
+                }
+                bar_arrive_n(2, F_THREADS);
+#define NBA_SEL2(a, k) ((k) == 0u ? a[0] : a[1])
+#pragma unroll 1
+                for (uint32_t k = 0; k < 2u; k++) {
+                    const uint32_t j = u + k * SPLIT_CONS;
+                    if (j >= cnt) continue;
+                    const uint32_t pkt = p_begin + j;
+                    const uint32_t info_k = NBA_SEL2(f_info, k), q_k = NBA_SEL2(f_q, k);
+                    if ((info_k & INFO_OK) && q_k != 0u) {
+                        if (!NBA_PROLOGUE_ONLY) {
+                            while (ready[j] != ep) __nanosleep(32);
+                            __threadfence_block();
+                            split_consume(T, B, H, NBA_SEL2(f_sa, k), info_k, q_k, NBA_SEL2(f_in, k),
+                                          NBA_SEL2(f_out, k), j);
+                        }
+                        const uint32_t Dp = info_k & 0x7ffu;
+                        const uint32_t Lp = 48u + esp_C(Dp);
+                        B.out_len[pkt] = (uint16_t)Lp;
+                        c_ok++;
+                        c_in += Dp;
+                        c_out += Lp;
+                    } else {
+                        B.out_len[pkt] = 0;
+                        c_drop++;
+                    }
+                }
+#undef NBA_SEL2
+#undef NBA_SEL3
+            }
+        } else if (!isP) {
             const uint32_t q32 = have ? L.seq[pk] : 0u;
             bar_arrive_n(2, F_THREADS);                  // fields taken: the arrays are free
             if (have) {

@@ -126,14 +126,14 @@ def main():
     ap.add_argument("--out", default=None)
     a = ap.parse_args()
     fc = os.path.join(CSRC, "fused_common.cuh")
-    rfc = func_ranges(fc, ["aes4_keystream", "ctr_precompute", "expand_key_lane"])
+    rfc = func_ranges(fc, ["aes4_keystream", "ctr_precompute", "expand_key_slots"])
     rsha = func_ranges(os.path.join(CSRC, "sha1.cuh"), ["sha1_compress_fma"])
     # the round loop of aes4_keystream: from its `for (int r = 0; r < 7` line to
-    # the line before `const uint4 rk = H.rkB[3]`
+    # the line before the final round's key load (`rkh[3 * F_THREADS`)
     src = open(fc).read().split("\n")
     a0, a1 = rfc["aes4_keystream"]
     loop0 = next(i + 1 for i in range(a0 - 1, a1) if "r < 7" in src[i])
-    loop1 = next(i + 1 for i in range(loop0, a1) if "H.rkB[3]" in src[i]) - 1
+    loop1 = next(i + 1 for i in range(loop0, a1) if "rkh[3 * F_THREADS" in src[i]) - 1
     ins = disassemble(a.kernel)
     regions = collections.OrderedDict(
         (k, collections.Counter()) for k in
@@ -152,7 +152,7 @@ def main():
             key = "aes_round_loop_body" if inner and loop0 <= inner[-1] <= loop1 else "aes_step_outside_loop"
         elif in_func(fr, "fused_common.cuh", rfc["ctr_precompute"]):
             key = "ctr_precompute"
-        elif in_func(fr, "fused_common.cuh", rfc["expand_key_lane"]):
+        elif in_func(fr, "fused_common.cuh", rfc["expand_key_slots"]):
             key = "expand_key_lane"
         if key:
             regions[key][p] += 1
