@@ -62,8 +62,8 @@ namespace nba {
 #define NBA_PIPE_STAGGER 128  //   STAGGER/256 x the time the lower warps took to their first AES
 #endif                        //   step (previous batch), so AES (LDS) and SHA-1 (ALU) overlap
 #ifndef NBA_PIPE_SPLIT        // pipelined ring: batches of one-AES-step packets run on producer
-#define NBA_PIPE_SPLIT 1      //   (AES) and consumer (SHA-1) warps (split_produce / _consume)
-#endif
+#define NBA_PIPE_SPLIT 0      //   (AES) and consumer (SHA-1) warps (split_produce / _consume);
+#endif                        //   measured slower (64 B 23.7 -> 27.4 us), off
 #ifndef NBA_PIPE_ONEBIN       // pipelined ring: one-length-bin batches keep index order (no sort)
 #define NBA_PIPE_ONEBIN 1
 #endif
