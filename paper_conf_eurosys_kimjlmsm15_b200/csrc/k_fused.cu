@@ -1481,6 +1481,12 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
 #endif
         } else {
             bar_sync_n(2, F_THREADS);                    // every lane took its fields
+#ifdef NBA_PRO_DELAY_NS   // experiment: start the next batch's prologue later (after the AES phase)
+            {
+                const uint32_t t0 = (uint32_t)gtimer();
+                while ((uint32_t)gtimer() - t0 < NBA_PRO_DELAY_NS) __nanosleep(256);
+            }
+#endif
             if (bi + 1 < n_batches) {
                 const BatchArgs Bn = slots[(first + bi + 1) % n_slots];
                 PipeMeta meta;
