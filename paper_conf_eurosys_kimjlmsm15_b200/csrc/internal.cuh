@@ -116,6 +116,8 @@ struct InState {                    // per-SA receive windows + per-batch worksp
     uint32_t *hval;                 // [hcap] smallest packet index with that key
     unsigned long long *counters;   // [N_IN_COUNTERS]
     uint32_t *ctl;                  // [8] ticket, barrier count / generation
+    unsigned long long *hk[2];      // one-kernel path: duplicate hashes by launch parity, the
+    uint32_t *hv[2];                //   current one filled by the lanes, the next one cleared
 };
 
 struct InBatchArgs {
@@ -193,7 +195,8 @@ cudaError_t launch_fused_ring(const DevTable &T, const DevWork &W, const BatchAr
 int aes_grid(int num_sms);
 int fused_grid(int num_sms);
 cudaError_t launch_in_fused(const DevTable &T, const InState &S, const InBatchArgs &B, int grid,
-                            uint32_t hmask, bool merged, uint32_t *bar_base, cudaStream_t st);
+                            uint32_t hmask, uint32_t hfull, bool merged, uint32_t *bar_base,
+                            cudaStream_t st);
 bool in_merged_ok(uint32_t n, int grid);
 cudaError_t launch_in_fused_ring(const DevTable &T, const InState &S, const InBatchArgs *slots,
                                  const RingRun &R, uint32_t hmask,

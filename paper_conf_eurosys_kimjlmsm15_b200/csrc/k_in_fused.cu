@@ -193,11 +193,35 @@ __device__ __forceinline__ void in_format(const DevTable &T, const InBatchArgs &
 // result as the sequential receiver.
 constexpr uint32_t CTLI_BAR = 4;   // S.ctl word: monotonic barrier arrivals
 constexpr uint32_t CTLI_BASE = 5;  // S.ctl word: arrivals before the current one-kernel launch
+constexpr uint32_t CTLI_PAR = 6;   // S.ctl word: one-kernel launches so far (hash parity)
+#ifndef NBA_IN_LANE_INSERT    // one-kernel inbound: duplicate-hash inserts by the lanes into a
+#define NBA_IN_LANE_INSERT 1  //   launch-parity pair of hashes (0: after the first barrier)
+#endif
 
-__device__ __forceinline__ void in_merged_tail(const DevTable &T, const InState &S, const InBatchArgs &B,
+// The one-kernel path's duplicate hashes (S.hk / S.hv by launch parity): the
+// lanes insert each authenticated packet into the current one right after
+// its ICV check, the tail clears the next launch's one between its two
+// barriers (over the whole capacity, `full`).  off: the hash S.hkey / S.hval
+// cleared at batch start and filled after the first barrier (plain ring).
+struct LaneIns {
+    bool on;
+    unsigned long long *ck;
+    uint32_t *cv;
+    unsigned long long *nk;
+    uint32_t *nv;
+    uint32_t full;
+};
+
+__device__ __forceinline__ void in_merged_tail(const DevTable &T, const InState &S0, const InBatchArgs &B,
                                                FusedLo &L, uint8_t *tabs, uint32_t p_begin,
-                                               uint32_t p_end, uint32_t hmask, uint32_t bar_base)
+                                               uint32_t p_end, uint32_t hmask, uint32_t bar_base,
+                                               const LaneIns &li)
 {
+    InState S = S0;
+    if (li.on) {                                  // the lanes' hash of this launch
+        S.hkey = li.ck;
+        S.hval = li.cv;
+    }
     constexpr uint32_t HS = 2u * F_SUPER, NW = F_THREADS / 32u;
     __shared__ unsigned long long s_cnt[N_IN_COUNTERS - 1];
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
@@ -251,10 +275,22 @@ __device__ __forceinline__ void in_merged_tail(const DevTable &T, const InState 
     __syncthreads();
     grid_arrive(&S.ctl[CTLI_BAR]);
     grid_wait(&S.ctl[CTLI_BAR], bar_base + G);
-    // every CTA has read the base (before arriving): advance it for the next launch
-    if (cta == 0 && tid == 0) S.ctl[CTLI_BASE] = bar_base + 2u * G;
-    // hash inserts (the hash was cleared before the barrier) and the row scans
-    if (inA) replay_hash_insert(S, key, q, i, hmask);
+    // every CTA has read the base and the parity (before arriving): advance
+    // them for the next launch
+    if (cta == 0 && tid == 0) {
+        S.ctl[CTLI_BASE] = bar_base + 2u * G;
+        if (li.on) S.ctl[CTLI_PAR] = S.ctl[CTLI_PAR] + 1u;
+    }
+    if (li.on) {
+        // the next launch's hash, cleared before this launch's second barrier
+        // (its previous user, the launch before this one, has completed)
+        for (uint32_t k = cta * F_THREADS + tid; k <= li.full; k += G * F_THREADS) {
+            li.nk[k] = ~0ull;
+            li.nv[k] = ~0u;
+        }
+    } else if (inA) {
+        replay_hash_insert(S, key, q, i, hmask);  // (the hash was cleared before the barrier)
+    }
     scan_all_rows(S, n_sa, cta * NW + warp, G * NW, G, lane);
     __syncthreads();
     grid_arrive(&S.ctl[CTLI_BAR]);
@@ -299,7 +335,8 @@ __device__ __forceinline__ void in_merged_tail(const DevTable &T, const InState 
 template <bool MERGED>
 __device__ __forceinline__ void in_fused_body(const DevTable &T, const InState &S,
                                               const InBatchArgs &B, uint32_t ppc, uint32_t hmask,
-                                              uint32_t bar_base, bool tinit, uint32_t tphase)
+                                              uint32_t bar_base, bool tinit, uint32_t tphase,
+                                              const LaneIns &li)
 {
     extern __shared__ __align__(16) uint8_t smem[];
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
@@ -318,10 +355,13 @@ __device__ __forceinline__ void in_fused_body(const DevTable &T, const InState &
     const uint32_t lane4r = (lane * 4u) | (smem_u32(tabs) & 0xffff0000u);
 
     // this batch's duplicate-detection hash (read by k_in_replay / k_in_decide
-    // of this batch only; the previous batch's kernels have completed)
-    for (uint32_t k = blockIdx.x * blockDim.x + tid; k <= hmask; k += gridDim.x * blockDim.x) {
-        S.hkey[k] = ~0ull;
-        S.hval[k] = ~0u;
+    // of this batch only; the previous batch's kernels have completed) -- with
+    // lane inserts the previous launch cleared it
+    if (!li.on) {
+        for (uint32_t k = blockIdx.x * blockDim.x + tid; k <= hmask; k += gridDim.x * blockDim.x) {
+            S.hkey[k] = ~0ull;
+            S.hval[k] = ~0u;
+        }
     }
     // T-tables by bulk copy (re-staged per batch: the replay merge of the
     // previous batch used their shared memory as scratch); waited for (phase
@@ -380,6 +420,8 @@ __device__ __forceinline__ void in_fused_body(const DevTable &T, const InState &
                 }
                 if (MERGED) {
                     L.aux1[pk] = flags;                 // for the in-kernel replay decision
+                    if (li.on && (flags & INF_ICV))     // (sa, q) -> first index, now
+                        replay_hash_insert(li.ck, li.cv, sa_me, L.seq[pk], base + pk, hmask);
                 } else {
                     S.flags[base + pk] = flags;
                     S.seq[base + pk] = L.seq[pk];
@@ -392,18 +434,25 @@ __device__ __forceinline__ void in_fused_body(const DevTable &T, const InState &
     // the tail uses the table region as scratch, and no copy may be in flight
     // when the CTA exits
     tables_bulk_wait(&L.tbar, tphase);
-    if constexpr (MERGED) in_merged_tail(T, S, B, L, tabs, p_begin, p_end, hmask, bar_base);
+    if constexpr (MERGED) in_merged_tail(T, S, B, L, tabs, p_begin, p_end, hmask, bar_base, li);
 }
 
 template <bool MERGED>
 __global__ void __launch_bounds__(F_THREADS, 1)
-k_in_fused(DevTable T, InState S, InBatchArgs B, uint32_t ppc, uint32_t hmask, uint32_t bar_base_h)
+k_in_fused(DevTable T, InState S, InBatchArgs B, uint32_t ppc, uint32_t hmask, uint32_t hfull,
+           uint32_t bar_base_h)
 {
-    // one-kernel form: the barrier base lives on the device (launches carry no
-    // host state and can be recorded in a graph); read before arriving
+    // one-kernel form: the barrier base and the hash parity live on the device
+    // (launches carry no host state and can be recorded in a graph); read
+    // before arriving
     const uint32_t bar_base =
         MERGED ? *reinterpret_cast<volatile uint32_t *>(&S.ctl[CTLI_BASE]) : bar_base_h;
-    in_fused_body<MERGED>(T, S, B, ppc, hmask, bar_base, true, 0u);
+    LaneIns li{false, nullptr, nullptr, nullptr, nullptr, 0u};
+    if (MERGED && NBA_IN_LANE_INSERT) {
+        const uint32_t par = *reinterpret_cast<volatile uint32_t *>(&S.ctl[CTLI_PAR]) & 1u;
+        li = LaneIns{true, S.hk[par], S.hv[par], S.hk[par ^ 1u], S.hv[par ^ 1u], hfull};
+    }
+    in_fused_body<MERGED>(T, S, B, ppc, hmask, bar_base, true, 0u, li);
 }
 
 // An inbound batch ring as ONE persistent launch: the grid walks the run's
@@ -430,7 +479,8 @@ k_in_fused_ring(DevTable T, InState S, const InBatchArgs *slots, RingRun R, uint
         uint32_t ppc = (B.n + G - 1) / G;
         ppc = (ppc + 31u) & ~31u;
         if (ppc < 32u) ppc = 32u;
-        in_fused_body<true>(T, Sb, B, ppc, hmask, base0 + 2u * bi * G, bi == 0, bi & 1u);
+        in_fused_body<true>(T, Sb, B, ppc, hmask, base0 + 2u * bi * G, bi == 0, bi & 1u,
+                            LaneIns{false, nullptr, nullptr, nullptr, nullptr, 0u});
         __syncthreads();   // shared memory is reused by the next batch
         if (R.ts && threadIdx.x == 0) atomicMax(&R.ts[1u + bi], gtimer());
     }
@@ -839,7 +889,8 @@ cudaError_t launch_in_fused_ring(const DevTable &T, const InState &S, const InBa
 }
 
 cudaError_t launch_in_fused(const DevTable &T, const InState &S, const InBatchArgs &B, int grid,
-                            uint32_t hmask, bool merged, uint32_t *bar_base, cudaStream_t st)
+                            uint32_t hmask, uint32_t hfull, bool merged, uint32_t *bar_base,
+                            cudaStream_t st)
 {
     uint32_t ppc = (B.n + grid - 1) / grid;
     ppc = (ppc + 31u) & ~31u;
@@ -856,8 +907,8 @@ cudaError_t launch_in_fused(const DevTable &T, const InState &S, const InBatchAr
     cfg.attrs = attr;
     cfg.numAttrs = merged ? 1 : 0;
     (void)bar_base;   // the one-kernel form keeps its barrier base on the device
-    cudaError_t e = merged ? cudaLaunchKernelEx(&cfg, k_in_fused<true>, T, S, B, ppc, hmask, 0u)
-                           : cudaLaunchKernelEx(&cfg, k_in_fused<false>, T, S, B, ppc, hmask, 0u);
+    cudaError_t e = merged ? cudaLaunchKernelEx(&cfg, k_in_fused<true>, T, S, B, ppc, hmask, hfull, 0u)
+                           : cudaLaunchKernelEx(&cfg, k_in_fused<false>, T, S, B, ppc, hmask, hfull, 0u);
     return e;
 }
 
