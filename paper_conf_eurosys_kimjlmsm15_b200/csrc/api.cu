@@ -77,6 +77,7 @@ struct nba_ipsec_sa_table {
     std::vector<uint32_t> seq0;     // the SAs' initial seq (window start, reading B6)
     bool in_enabled = false, in_gridsync = false;
     uint32_t in_hcap = 0;
+    InHashPair HP = {};           // the one-kernel inbound path's duplicate hashes
     uint32_t in_bar_base = 0;     // arrivals so far at the one-kernel inbound path's barriers
     uint32_t in_last_launches = 3;
     InState S{};
@@ -1125,8 +1126,8 @@ int nba_ipsec_enable_inbound(nba_ipsec_sa_table *t)
     chk(dalloc(t, &S.hkey, hcap));
     chk(dalloc(t, &S.hval, hcap));
     for (int k = 0; k < 2; k++) {
-        chk(dalloc(t, &S.hk[k], hcap));
-        chk(dalloc(t, &S.hv[k], hcap));
+        chk(dalloc(t, &t->HP.hk[k], hcap));
+        chk(dalloc(t, &t->HP.hv[k], hcap));
     }
     chk(dalloc(t, &S.counters, N_IN_COUNTERS));
     chk(dalloc(t, &S.ctl, 8));
@@ -1134,8 +1135,8 @@ int nba_ipsec_enable_inbound(nba_ipsec_sa_table *t)
     chk(dalloc(t, &t->in_bmp0, n_sa));
     if (e == cudaSuccess) {
         for (int k = 0; k < 2; k++) {          // the one-kernel path's hashes start empty
-            chk(cudaMemset(S.hk[k], 0xff, hcap * sizeof(unsigned long long)));
-            chk(cudaMemset(S.hv[k], 0xff, hcap * sizeof(uint32_t)));
+            chk(cudaMemset(t->HP.hk[k], 0xff, hcap * sizeof(unsigned long long)));
+            chk(cudaMemset(t->HP.hv[k], 0xff, hcap * sizeof(uint32_t)));
         }
         // reading B6: the window starts at the SA's seq, everything <= seq seen
         std::vector<unsigned long long> bmp(n_sa);
@@ -1191,8 +1192,8 @@ int nba_ipsec_process_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batch *b
     // decision inside, behind two grid barriers); else three kernels
     const bool merged = t->allow_merged && in_merged_ok(n, t->grid_fused);
     t->in_last_launches = merged ? 1 : 3;
-    if (launch_in_fused(t->T, t->S, B, t->grid_fused, hmask, t->in_hcap - 1u, merged, &t->in_bar_base,
-                        st) != cudaSuccess)
+    if (launch_in_fused(t->T, t->S, t->HP, B, t->grid_fused, hmask, t->in_hcap - 1u, merged,
+                        &t->in_bar_base, st) != cudaSuccess)
         return NBA_IPSEC_ECUDA;
     mark();
     if (merged) return NBA_IPSEC_OK;

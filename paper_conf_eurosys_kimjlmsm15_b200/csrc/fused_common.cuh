@@ -42,6 +42,9 @@ struct FusedLo {
     uint32_t tailf[448];           // inbound pipelined ring: a batch's per-packet flags and
     uint32_t tailq[448];           //   sequence numbers and SA indices (by packet index) for
     uint32_t tails[448];           //   its replay tail
+    uint32_t it0;                  // pipelined ring: this iteration's start (globaltimer, low word)
+    uint32_t lanes_acc;            //   the lanes' latest end relative to it (this batch)
+    uint32_t pro_delay;            //   the prologue warps' start delay for the next batch (ns)
     uint32_t stag_ns;              // pipelined ring: start delay of the upper lane warps
     uint32_t stag_acc;             //   (AES step 0 of the lower ones, measured per batch)
 };

@@ -116,8 +116,13 @@ struct InState {                    // per-SA receive windows + per-batch worksp
     uint32_t *hval;                 // [hcap] smallest packet index with that key
     unsigned long long *counters;   // [N_IN_COUNTERS]
     uint32_t *ctl;                  // [8] ticket, barrier count / generation
-    unsigned long long *hk[2];      // one-kernel path: duplicate hashes by launch parity, the
-    uint32_t *hv[2];                //   current one filled by the lanes, the next one cleared
+};
+
+// The one-kernel inbound path's duplicate hashes by launch parity (the
+// current one filled by the lanes, the next one cleared during the launch).
+struct InHashPair {
+    unsigned long long *hk[2];
+    uint32_t *hv[2];
 };
 
 struct InBatchArgs {
@@ -194,9 +199,9 @@ cudaError_t launch_fused_ring(const DevTable &T, const DevWork &W, const BatchAr
                               const RingRun &R, uint16_t *hist_b, int grid, cudaStream_t st);
 int aes_grid(int num_sms);
 int fused_grid(int num_sms);
-cudaError_t launch_in_fused(const DevTable &T, const InState &S, const InBatchArgs &B, int grid,
-                            uint32_t hmask, uint32_t hfull, bool merged, uint32_t *bar_base,
-                            cudaStream_t st);
+cudaError_t launch_in_fused(const DevTable &T, const InState &S, const InHashPair &HP,
+                            const InBatchArgs &B, int grid, uint32_t hmask, uint32_t hfull,
+                            bool merged, uint32_t *bar_base, cudaStream_t st);
 bool in_merged_ok(uint32_t n, int grid);
 cudaError_t launch_in_fused_ring(const DevTable &T, const InState &S, const InBatchArgs *slots,
                                  const RingRun &R, uint32_t hmask,

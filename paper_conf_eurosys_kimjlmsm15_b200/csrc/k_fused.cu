@@ -64,6 +64,9 @@ namespace nba {
 #ifndef NBA_PIPE_SPLIT        // pipelined ring: batches of one-AES-step packets run on producer
 #define NBA_PIPE_SPLIT 0      //   (AES) and consumer (SHA-1) warps (split_produce / _consume);
 #endif                        //   measured slower (64 B 23.7 -> 27.4 us), off
+#ifndef NBA_PIPE_PRO_DELAY    // pipelined ring: the prologue warps start the next batch's work
+#define NBA_PIPE_PRO_DELAY 1  //   min(4 us, 1/4 of the previous batch's lane phase) after the
+#endif                        //   lanes took their fields (off the AES phase's shared-memory load)
 #ifndef NBA_PIPE_ONEBIN       // pipelined ring: one-length-bin batches keep index order (no sort)
 #define NBA_PIPE_ONEBIN 1
 #endif
@@ -1286,6 +1289,8 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
     if (tid == 0) {
         L.stag_ns = 0u;
         L.stag_acc = 0u;
+        L.lanes_acc = 0u;
+        L.pro_delay = 0u;
     }
     for (uint32_t k = tid; k < PIPE_MAX_PPC; k += F_THREADS) L.tailf[k] = 0u;   // split: ready flags
     for (uint32_t k = tid; k < 2u * F_SUPER; k += F_THREADS) {
@@ -1322,6 +1327,7 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
 #if NBA_RING_TRACE
         if (tid == 0 && R.ts) *RTR(bi, 0) = gtimer();
 #endif
+        if (NBA_PIPE_PRO_DELAY && tid == 0) L.it0 = (uint32_t)gtimer();
         // lanes: the packet (known since the previous batch); its SA line and
         // round keys either before the barrier wait / scans / polls, whose
         // latency they then overlap (long or length-divergent batches, as
@@ -1476,11 +1482,16 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
                     c_drop++;
                 }
             }
+            if (NBA_PIPE_PRO_DELAY && lane == 0) atomicMax(&L.lanes_acc, (uint32_t)gtimer() - L.it0);
 #if NBA_RING_TRACE
             if (lane == 0 && R.ts) atomicMax(RTR(bi, 3), gtimer());
 #endif
         } else {
             bar_sync_n(2, F_THREADS);                    // every lane took its fields
+            if (NBA_PIPE_PRO_DELAY) {   // off the lanes' AES phase (its shared-memory load)
+                const uint32_t t0 = (uint32_t)gtimer(), d = L.pro_delay;
+                while ((uint32_t)gtimer() - t0 < d) __nanosleep(256);
+            }
 #ifdef NBA_PRO_DELAY_NS   // experiment: start the next batch's prologue later (after the AES phase)
             {
                 const uint32_t t0 = (uint32_t)gtimer();
@@ -1504,6 +1515,10 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
         if (NBA_PIPE_STAGGER && tid == 0) {               // next batch's delay of the upper warps
             L.stag_ns = (uint32_t)(((unsigned long long)L.stag_acc * NBA_PIPE_STAGGER) >> 8);
             L.stag_acc = 0u;
+        }
+        if (NBA_PIPE_PRO_DELAY && tid == 0) {             // and of the prologue warps
+            L.pro_delay = min(4000u, L.lanes_acc >> 2);
+            L.lanes_acc = 0u;
         }
 #if NBA_RING_TRACE
         if (tid == 0 && R.ts) *RTR(bi, 5) = gtimer();

@@ -439,8 +439,8 @@ __device__ __forceinline__ void in_fused_body(const DevTable &T, const InState &
 
 template <bool MERGED>
 __global__ void __launch_bounds__(F_THREADS, 1)
-k_in_fused(DevTable T, InState S, InBatchArgs B, uint32_t ppc, uint32_t hmask, uint32_t hfull,
-           uint32_t bar_base_h)
+k_in_fused(DevTable T, InState S, InHashPair HP, InBatchArgs B, uint32_t ppc, uint32_t hmask,
+           uint32_t hfull, uint32_t bar_base_h)
 {
     // one-kernel form: the barrier base and the hash parity live on the device
     // (launches carry no host state and can be recorded in a graph); read
@@ -450,7 +450,8 @@ k_in_fused(DevTable T, InState S, InBatchArgs B, uint32_t ppc, uint32_t hmask, u
     LaneIns li{false, nullptr, nullptr, nullptr, nullptr, 0u};
     if (MERGED && NBA_IN_LANE_INSERT) {
         const uint32_t par = *reinterpret_cast<volatile uint32_t *>(&S.ctl[CTLI_PAR]) & 1u;
-        li = LaneIns{true, S.hk[par], S.hv[par], S.hk[par ^ 1u], S.hv[par ^ 1u], hfull};
+        li = par ? LaneIns{true, HP.hk[1], HP.hv[1], HP.hk[0], HP.hv[0], hfull}
+                 : LaneIns{true, HP.hk[0], HP.hv[0], HP.hk[1], HP.hv[1], hfull};
     }
     in_fused_body<MERGED>(T, S, B, ppc, hmask, bar_base, true, 0u, li);
 }
@@ -888,9 +889,9 @@ cudaError_t launch_in_fused_ring(const DevTable &T, const InState &S, const InBa
     return cudaLaunchKernelEx(&cfg, k_in_fused_ring, T, S, slots, R, hmask, hkey_b, hval_b);
 }
 
-cudaError_t launch_in_fused(const DevTable &T, const InState &S, const InBatchArgs &B, int grid,
-                            uint32_t hmask, uint32_t hfull, bool merged, uint32_t *bar_base,
-                            cudaStream_t st)
+cudaError_t launch_in_fused(const DevTable &T, const InState &S, const InHashPair &HP,
+                            const InBatchArgs &B, int grid, uint32_t hmask, uint32_t hfull,
+                            bool merged, uint32_t *bar_base, cudaStream_t st)
 {
     uint32_t ppc = (B.n + grid - 1) / grid;
     ppc = (ppc + 31u) & ~31u;
@@ -907,8 +908,8 @@ cudaError_t launch_in_fused(const DevTable &T, const InState &S, const InBatchAr
     cfg.attrs = attr;
     cfg.numAttrs = merged ? 1 : 0;
     (void)bar_base;   // the one-kernel form keeps its barrier base on the device
-    cudaError_t e = merged ? cudaLaunchKernelEx(&cfg, k_in_fused<true>, T, S, B, ppc, hmask, hfull, 0u)
-                           : cudaLaunchKernelEx(&cfg, k_in_fused<false>, T, S, B, ppc, hmask, hfull, 0u);
+    cudaError_t e = merged ? cudaLaunchKernelEx(&cfg, k_in_fused<true>, T, S, HP, B, ppc, hmask, hfull, 0u)
+                           : cudaLaunchKernelEx(&cfg, k_in_fused<false>, T, S, HP, B, ppc, hmask, hfull, 0u);
     return e;
 }
 
