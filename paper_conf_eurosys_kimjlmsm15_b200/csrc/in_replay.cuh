@@ -30,10 +30,10 @@ __device__ __forceinline__ uint32_t group_prefix_max(uint32_t lt, uint32_t v)
     return mex;
 }
 
-__device__ __forceinline__ void window_advance(const InState &S, uint32_t sa, uint32_t batch_max)
+// (t0, b0: the SA's window, loaded by the caller beside the row)
+__device__ __forceinline__ void window_advance(const InState &S, uint32_t sa, uint32_t batch_max,
+                                               uint32_t t0, unsigned long long b0)
 {
-    const uint32_t t0 = S.top[sa];
-    const unsigned long long b0 = S.bmp[sa];
     S.top_prev[sa] = t0;
     S.bmp_prev[sa] = b0;
     const uint32_t t1 = max(t0, batch_max);
@@ -50,7 +50,12 @@ __device__ __forceinline__ void scan_max_row(const InState &S, uint32_t sa, uint
     constexpr int U = 8;
     uint32_t *row = S.hmax + (size_t)sa * n_tiles;
     uint32_t *pfx = S.pmx + (size_t)sa * n_tiles;
-    uint32_t carry = 0;
+    uint32_t carry = 0, w0 = 0;
+    unsigned long long b0 = 0;
+    if (lane == 0) {                                 // the window, beside the row's loads
+        w0 = S.top[sa];
+        b0 = S.bmp[sa];
+    }
     for (uint32_t t0 = 0; t0 < n_tiles; t0 += 32u * U) {
         uint32_t h[U];
 #pragma unroll
@@ -77,7 +82,7 @@ __device__ __forceinline__ void scan_max_row(const InState &S, uint32_t sa, uint
             carry = max(carry, __shfl_sync(0xffffffffu, x, 31));
         }
     }
-    if (lane == 0) window_advance(S, sa, carry);
+    if (lane == 0) window_advance(S, sa, carry, w0, b0);
 }
 
 // All SA rows by `nslots` warps (this one is `slot`): one warp per SA for long
@@ -95,6 +100,8 @@ __device__ __forceinline__ void scan_all_rows(const InState &S, uint32_t n_sa, u
         const uint32_t sa = (uint32_t)sa_l;
         uint32_t *row = S.hmax + (size_t)sa * n_tiles;
         uint32_t *pfx = S.pmx + (size_t)sa * n_tiles;
+        const uint32_t w0 = S.top[sa];
+        const unsigned long long b0 = S.bmp[sa];
         uint32_t h[32];
 #pragma unroll
         for (uint32_t t = 0; t < 32u; t++) h[t] = t < n_tiles ? __ldcg(&row[t]) : 0u;
@@ -107,7 +114,7 @@ __device__ __forceinline__ void scan_all_rows(const InState &S, uint32_t n_sa, u
             }
             carry = max(carry, h[t]);
         }
-        window_advance(S, sa, carry);
+        window_advance(S, sa, carry, w0, b0);
     }
 }
 

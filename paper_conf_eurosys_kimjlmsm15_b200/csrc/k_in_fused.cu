@@ -281,6 +281,7 @@ __device__ __forceinline__ void in_merged_tail(const DevTable &T, const InState 
         S.ctl[CTLI_BASE] = bar_base + 2u * G;
         if (li.on) S.ctl[CTLI_PAR] = S.ctl[CTLI_PAR] + 1u;
     }
+    scan_all_rows(S, n_sa, warp * G + cta, G * NW, G, lane);   // SA s on CTA s mod G
     if (li.on) {
         // the next launch's hash, cleared before this launch's second barrier
         // (its previous user, the launch before this one, has completed)
@@ -291,7 +292,6 @@ __device__ __forceinline__ void in_merged_tail(const DevTable &T, const InState 
     } else if (inA) {
         replay_hash_insert(S, key, q, i, hmask);  // (the hash was cleared before the barrier)
     }
-    scan_all_rows(S, n_sa, cta * NW + warp, G * NW, G, lane);
     __syncthreads();
     grid_arrive(&S.ctl[CTLI_BAR]);
     grid_wait(&S.ctl[CTLI_BAR], bar_base + 2u * G);
@@ -671,6 +671,8 @@ __device__ __forceinline__ void in_pipe_tail(const DevTable &T, const InState &S
     grid_arrive(&S.ctl[CTLI_BAR]);
     grid_wait(&S.ctl[CTLI_BAR], bar_base + G);
     if (tr && tid == 0) tr[1] = gtimer();
+    scan_all_rows(S, n_sa, warp * G + cta, G * NW, G, lane);   // SA s on CTA s mod G
+    if (tr && lane == 0) atomicMax(&tr[8], gtimer());
     // the next batch's hash: its last user (the batch before this one) made
     // its lookups before this batch's first barrier; every CTA clears its
     // slice before arriving at the second barrier, which the next batch's
@@ -683,8 +685,6 @@ __device__ __forceinline__ void in_pipe_tail(const DevTable &T, const InState &S
         __syncwarp();
         if (lane == 0) atomicMax(&tr[7], gtimer());
     }
-    scan_all_rows(S, n_sa, cta * NW + warp, G * NW, G, lane);
-    if (tr && lane == 0) atomicMax(&tr[8], gtimer());
     __syncthreads();
     if (tr && tid == 0) tr[9] = gtimer();
     grid_arrive(&S.ctl[CTLI_BAR]);

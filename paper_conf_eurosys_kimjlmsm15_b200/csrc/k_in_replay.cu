@@ -122,7 +122,7 @@ k_in_replay(DevTable T, InState S, InBatchArgs B, uint32_t n_tiles, uint32_t hma
     if (gridsync) {
         in_grid_barrier(&S.ctl[1], &S.ctl[2]);
         asm volatile("griddepcontrol.launch_dependents;");
-        scan_all_rows(S, n_sa, tile * (PTILE / 32u) + warp, gridDim.x * (PTILE / 32u), n_tiles, lane);
+        scan_all_rows(S, n_sa, warp * gridDim.x + tile, gridDim.x * (PTILE / 32u), n_tiles, lane);
     } else {
         __threadfence();
         __syncthreads();

@@ -403,7 +403,7 @@ def test_inbound_pipelined_ring_mixed_stream(n_sa, sizes, monkeypatch):
     with reordering, duplicates, stale replays, single-byte corruption,
     invalid SA indices and SPI mismatches: one rotation over the slots, then a
     partial rotation that replays the first two slots (every earlier packet
-    now a replay), each run against the oracle's sequential receiver
+    now a replay), then seven batches in one launch, each run against the oracle's sequential receiver
     continuing from the same state: statuses, lengths, inner bytes, windows
     and counters."""
     import torch
@@ -436,7 +436,7 @@ def test_inbound_pipelined_ring_mixed_stream(n_sa, sizes, monkeypatch):
         ring = t.ring_inbound([(*d.args(), st, ib.n) for d, st, ib in zip(ds, sts, bs)])
         assert ring.form == ring.PIPELINED
         k = 0
-        for nb in (len(bs), 2):
+        for nb in (len(bs), 2, 7):   # (7: every duplicate hash of the mod-3 rotation reused)
             ring.run_batches(nb)
             torch.cuda.synchronize()
             for _ in range(nb):

@@ -50,9 +50,12 @@ for size in %(sizes)r:
         ring.set_timestamps(ts)
         t.reset_inbound(); ring.run_batches(R); torch.cuda.synchronize()
         v = ts.cpu().numpy().reshape(R, G, 16).astype(np.int64)[1:-1]
-        rel = (v - v[:, :, :1]) / 1e3
-        names = {1: "bar1_passed", 2: "bar2_passed", 3: "lanes_done", 4: "side_done", 5: "iter_end",
-                 6: "tail_tile_done", 7: "inserts_done", 8: "row_scans_done", 9: "cta_done_mid"}
+        t0 = v[:, :, :1].min(axis=1, keepdims=True)       # the batch's first CTA start
+        v = np.where(v > 0, v, t0)                          # (stamps a form does not take)
+        rel = (v - t0) / 1e3
+        names = {0: "iter_start", 1: "bar1_passed", 2: "bar2_passed", 3: "lanes_done", 4: "side_done",
+                 5: "iter_end", 6: "tail_tile_done", 7: "next_hash_cleared", 8: "row_scans_done",
+                 9: "cta_done_mid"}
         out[str(size)] = {n: [round(float(np.median(rel[:, :, i])), 2),
                               round(float(np.median(np.max(rel[:, :, i], axis=1))), 2)]
                           for i, n in names.items()}
