@@ -374,8 +374,8 @@ def measure_inbound(ctx, args, cfg_id, steps, warmup, form=None):
     t_out.close()
     t = nba_ipsec.SATable(p, device=ctx.local, max_batch=PKTS_PER_GPU)
     t.enable_inbound()
-    if form == "pipelined":          # the opt-in software-pipelined inbound ring
-        os.environ["NBA_IPSEC_RING_IN_PIPE"] = "1"
+    if form is not None:             # force a form (default: the library's choice by length)
+        os.environ["NBA_IPSEC_RING_IN_PIPE"] = "1" if form == "pipelined" else "0"
     try:
         ring = t.ring_inbound([(e[0], db.out_off, e[1], db.sa_idx, e[2], db.out_off, e[3], None, b.n)
                                for e in esp])
@@ -724,10 +724,10 @@ def run_ours(args):
             inbound[size_key(CFG_SIZE[cfg_id])] = measure_inbound(ctx, args, cfg_id,
                                                                  max(10, steps // 4),
                                                                  max(3, warmup // 2))
-        # the opt-in software-pipelined inbound ring (faster for small packets,
-        # slower for large ones), on the same traffic
-        inbound["64_pipelined_ring"] = measure_inbound(ctx, args, 2, max(10, steps // 4),
-                                                       max(3, warmup // 2), form="pipelined")
+        # the other form at 64 B on the same traffic: the CUDA-graph ring of
+        # one-kernel launches (the library picks the pipelined ring there)
+        inbound["64_graph_ring"] = measure_inbound(ctx, args, 2, max(10, steps // 4),
+                                                   max(3, warmup // 2), form="graph")
     flows = None
     if not args.no_inbound:
         flows = measure_flows(ctx, args, main_cfg, max(10, steps // 4), max(3, warmup // 2))

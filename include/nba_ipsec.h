@@ -463,12 +463,18 @@ int nba_ipsec_enable_inbound(nba_ipsec_sa_table *t);
  * as process_batch.  NBA_IPSEC_EINVAL if inbound is not enabled, for NULL
  * arrays with n_pkts > 0 or n_pkts > max_batch_pkts. */
 int nba_ipsec_process_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batch *b, void *cuda_stream);
-/* A batch ring (nba_ipsec_ring_create) of ESP inbound slots: process_inbound
- * per slot recorded once as a CUDA graph (the one-kernel inbound path keeps
- * its barrier base on the device too), or -- opt-in, NBA_IPSEC_RING_IN_PERSIST
- * set at creation -- one persistent launch per run; run / destroy with
- * nba_ipsec_ring_run / nba_ipsec_ring_destroy.  Additionally NBA_IPSEC_EINVAL
- * if inbound is not enabled. */
+/* A batch ring (nba_ipsec_ring_create) of ESP inbound slots.  Form, chosen
+ * at creation: when every slot has <= 448 packets per SM and every packet's
+ * outer length is <= 640 B (read once from the slots' in_len, synchronously),
+ * one software-pipelined persistent launch per run (the next batch's
+ * metadata, the previous batch's replay row scans and decisions overlap the
+ * current batch's crypto); otherwise process_inbound per slot recorded once
+ * as a CUDA graph.  Environment overrides at creation:
+ * NBA_IPSEC_RING_IN_PIPE=1 / =0 (pipelined whenever it fits / never),
+ * NBA_IPSEC_RING_IN_PERSIST (a plain persistent launch per run),
+ * NBA_IPSEC_RING_GRAPH (the graph).  Run / destroy with nba_ipsec_ring_run[_batches]
+ * / nba_ipsec_ring_destroy.  Additionally NBA_IPSEC_EINVAL if inbound is not
+ * enabled; NBA_IPSEC_ECUDA if reading the lengths fails. */
 int nba_ipsec_ring_create_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batch *slots,
                                   uint32_t n_slots, nba_ipsec_ring **out);
 /* Enqueue (on `cuda_stream`) a reset of every receive window to its initial

@@ -404,6 +404,7 @@ struct nba_ipsec_ring {
     InBatchArgs *d_in_slots = nullptr;
     unsigned long long *hkey_b = nullptr;
     uint32_t *hval_b = nullptr;
+    InPipeBufs in_bufs = {};             // pipelined inbound form (hk1 / hv1 = hkey_b / hval_b)
     uint32_t in_hmask = 0;
     bool pipe = false;                   // software-pipelined form (k_fused_ring_pipe)
     bool in_pipe = false;                // inbound: software-pipelined form (k_in_fused_ring_pipe)
@@ -515,23 +516,39 @@ int nba_ipsec_ring_create_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batc
     r->n_slots = n_slots;
     r->flow_gen = t->flow_gen;
     r->h_in_slots.assign(slots, slots + n_slots);
-    // Forms: a CUDA graph of one-kernel launches (the default); opt-in, the
-    // software-pipelined persistent ring (NBA_IPSEC_RING_IN_PIPE, every slot
-    // <= 448 packets per SM) or the plain persistent ring
-    // (NBA_IPSEC_RING_IN_PERSIST).  Measured per batch, graph / plain /
-    // pipelined: 64 B 44.8 / 43.2 / 42.0 us, 1514 B 214 / 214 / 231 us, IMIX
-    // 107 / 112 / 140 us -- the replay tail's two grid barriers couple the
-    // CTAs every batch, so the pipelined form's lanes (slower under the side
-    // warps' loads) and stragglers are paid for in full.
-    bool pipe = std::getenv("NBA_IPSEC_RING_IN_PIPE") && !std::getenv("NBA_IPSEC_RING_GRAPH") &&
-                t->allow_merged;
-    bool persist = std::getenv("NBA_IPSEC_RING_IN_PERSIST") && !std::getenv("NBA_IPSEC_RING_GRAPH") &&
-                   t->allow_merged;
+    // Forms: the software-pipelined persistent ring (k_in_fused_ring_pipe)
+    // when every slot fits it (<= 448 packets per SM) and every packet is
+    // small (outer length <= IN_PIPE_MAX_LEN: uniform small-packet traffic),
+    // otherwise a CUDA graph of one-kernel launches.  Measured per batch,
+    // graph / pipelined (profiles/ab/r02aq_inbound_sweep.txt, r02ap):
+    // 64 B 39.7 / 31.8 us, 128 B 50.4 / 42.3, 256 B 63.6 / 58.2, 512 B
+    // 93.7 / 92.3, 1024 B 152.8 / 156.6, 1514 B 210 / 221, IMIX 101 / 130
+    // (the pipelined form has 14 lane warps, and its CTAs are coupled every
+    // batch through the replay's barriers, so a mix of lengths costs it the
+    // slowest CTA's lanes).  Overrides at creation: NBA_IPSEC_RING_IN_PIPE=1
+    // (pipelined whenever it fits) or =0 (never), NBA_IPSEC_RING_IN_PERSIST
+    // (the plain persistent ring), NBA_IPSEC_RING_GRAPH (the graph).
+    const char *pipe_env = std::getenv("NBA_IPSEC_RING_IN_PIPE");
+    const bool graph_only = std::getenv("NBA_IPSEC_RING_GRAPH") != nullptr || !t->allow_merged;
+    bool persist = std::getenv("NBA_IPSEC_RING_IN_PERSIST") && !graph_only;
+    bool pipe = !graph_only && !persist && !(pipe_env && pipe_env[0] == '0');
     uint32_t nmax = 0;
     for (uint32_t i = 0; i < n_slots; i++) {
         pipe = pipe && in_pipe_ok(slots[i].n_pkts, t->grid_fused);
         persist = persist && slots[i].n_pkts > 0 && in_merged_ok(slots[i].n_pkts, t->grid_fused);
         nmax = std::max(nmax, slots[i].n_pkts);
+    }
+    if (pipe && !(pipe_env && pipe_env[0] == '1')) {
+        // the automatic choice: the longest outer length over the slots
+        std::vector<uint16_t> len(nmax);
+        for (uint32_t i = 0; i < n_slots && pipe; i++) {
+            if (cudaMemcpy(len.data(), slots[i].in_len, slots[i].n_pkts * sizeof(uint16_t),
+                           cudaMemcpyDeviceToHost) != cudaSuccess) {
+                delete r;
+                return NBA_IPSEC_ECUDA;
+            }
+            for (uint32_t k = 0; k < slots[i].n_pkts && pipe; k++) pipe = len[k] <= IN_PIPE_MAX_LEN;
+        }
     }
     r->in_pipe = pipe;
     if (pipe || persist) {
@@ -552,6 +569,19 @@ int nba_ipsec_ring_create_inbound(nba_ipsec_sa_table *t, const nba_ipsec_in_batc
                        cudaMemcpyHostToDevice) != cudaSuccess) {
             nba_ipsec_ring_destroy(r);
             return NBA_IPSEC_ENOMEM;
+        }
+        if (pipe) {
+            InPipeBufs &P = r->in_bufs;
+            P.hk1 = r->hkey_b;
+            P.hv1 = r->hval_b;
+            if (cudaMalloc(&P.hk2, hc * sizeof(unsigned long long)) != cudaSuccess ||
+                cudaMalloc(&P.hv2, hc * sizeof(uint32_t)) != cudaSuccess ||
+                cudaMalloc(&P.hk3, hc * sizeof(unsigned long long)) != cudaSuccess ||
+                cudaMalloc(&P.hv3, hc * sizeof(uint32_t)) != cudaSuccess ||
+                cudaMalloc(&P.scr, (size_t)t->grid_fused * 448u /* PIPE_MAX_PPC */ * sizeof(uint4)) != cudaSuccess) {
+                nba_ipsec_ring_destroy(r);
+                return NBA_IPSEC_ENOMEM;
+            }
         }
         *out = r;
         return NBA_IPSEC_OK;
@@ -599,7 +629,7 @@ static int ring_launch(nba_ipsec_ring *r, uint32_t first, uint32_t n_batches, cu
     const RingRun R{r->n_slots, first, n_batches, r->ts};
     if (r->d_in_slots)
         return (r->in_pipe ? launch_in_fused_ring_pipe(t->T, t->S, r->d_in_slots, R, r->in_hmask,
-                                                       r->hkey_b, r->hval_b, t->grid_fused, st)
+                                                       r->in_bufs, t->grid_fused, st)
                            : launch_in_fused_ring(t->T, t->S, r->d_in_slots, R, r->in_hmask,
                                                   r->hkey_b, r->hval_b, t->grid_fused, st)) ==
                        cudaSuccess
@@ -702,6 +732,9 @@ int nba_ipsec_ring_destroy(nba_ipsec_ring *r)
         if (r->d_in_slots) cudaFree(r->d_in_slots);
         if (r->hkey_b) cudaFree(r->hkey_b);
         if (r->hval_b) cudaFree(r->hval_b);
+        for (void *q : {(void *)r->in_bufs.hk2, (void *)r->in_bufs.hv2, (void *)r->in_bufs.hk3,
+                        (void *)r->in_bufs.hv3, (void *)r->in_bufs.scr})
+            if (q) cudaFree(q);
     }
     delete r;
     return NBA_IPSEC_OK;

@@ -95,6 +95,7 @@ struct BatchArgs {
 // --- ESP inbound (readings B1..B9) ---------------
 constexpr uint32_t IN_MIN_LEN = 48u + 24u;      // outer 20 + ESP 16 + C >= 24 + ICV 12
 constexpr uint32_t IN_MAX_LEN = 48u + 1504u;
+constexpr uint32_t IN_PIPE_MAX_LEN = 640u;   // inbound rings: pipelined form up to this outer length
 constexpr uint32_t REPLAY_W = 64u;              // RFC 4303 §3.4.3 default window
 // per-packet flags written by k_in_fused: bits 0..15 inner length D
 constexpr uint32_t INF_FMT = 1u << 31, INF_ICV = 1u << 30, INF_TRL = 1u << 29;
@@ -123,6 +124,17 @@ struct InState {                    // per-SA receive windows + per-batch worksp
 struct InHashPair {
     unsigned long long *hk[2];
     uint32_t *hv[2];
+};
+
+// The pipelined inbound ring's own buffers: duplicate hashes 1..3 (hash 0 is
+// InState::hkey / hval), batch k's being hash k mod 4, and a scratch row of
+// PIPE_MAX_PPC per-packet decision inputs per CTA (flags, sequence number,
+// prefix max within the CTA, SA), written by batch k's tile part and read by
+// its decisions during batch k + 1.
+struct InPipeBufs {
+    unsigned long long *hk1, *hk2, *hk3;
+    uint32_t *hv1, *hv2, *hv3;
+    uint4 *scr;                      // [G][448]
 };
 
 struct InBatchArgs {
@@ -208,8 +220,8 @@ cudaError_t launch_in_fused_ring(const DevTable &T, const InState &S, const InBa
                                  unsigned long long *hkey_b, uint32_t *hval_b, int grid,
                                  cudaStream_t st);
 cudaError_t launch_in_fused_ring_pipe(const DevTable &T, const InState &S, const InBatchArgs *slots,
-                                      const RingRun &R, uint32_t hmask, unsigned long long *hkey_b,
-                                      uint32_t *hval_b, int grid, cudaStream_t st);
+                                      const RingRun &R, uint32_t hmask, const InPipeBufs &P, int grid,
+                                      cudaStream_t st);
 bool in_pipe_ok(uint32_t n, int grid);
 cudaError_t launch_in_replay(const DevTable &T, const InState &S, const InBatchArgs &B,
                              uint32_t n_tiles, uint32_t hmask, bool gridsync, cudaStream_t st);

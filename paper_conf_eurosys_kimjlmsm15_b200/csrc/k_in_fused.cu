@@ -194,6 +194,7 @@ __device__ __forceinline__ void in_format(const DevTable &T, const InBatchArgs &
 constexpr uint32_t CTLI_BAR = 4;   // S.ctl word: monotonic barrier arrivals
 constexpr uint32_t CTLI_BASE = 5;  // S.ctl word: arrivals before the current one-kernel launch
 constexpr uint32_t CTLI_PAR = 6;   // S.ctl word: one-kernel launches so far (hash parity)
+constexpr uint32_t CTLI_BAR2 = 7;  // S.ctl word: pipelined ring's row-scan arrivals (monotonic)
 #ifndef NBA_IN_LANE_INSERT    // one-kernel inbound: duplicate-hash inserts by the lanes into a
 #define NBA_IN_LANE_INSERT 1  //   launch-parity pair of hashes (0: after the first barrier)
 #endif
@@ -505,6 +506,15 @@ k_in_fused_ring(DevTable T, InState S, const InBatchArgs *slots, RingRun R, uint
 // batch k clears its buffer before its first barrier, and that buffer's last
 // user (batch k - 2) finished everywhere before batch k - 1's second barrier.
 
+#ifndef NBA_IN_LANE_FORMAT    // pipelined inbound ring: the outer-header format checks by the
+#define NBA_IN_LANE_FORMAT 0  //   lanes (1) or by the side warps' prologue (0)
+#endif
+#ifndef NBA_IN_PREFETCH       // pipelined inbound ring: L2 prefetches of the next batch's headers
+#define NBA_IN_PREFETCH 0     //   and the one after's metadata, ahead of the side warps' prologue
+#endif
+#ifndef NBA_IN_PRO_FIRST      // pipelined inbound ring: the side warps run the next batch's
+#define NBA_IN_PRO_FIRST 0    //   prologue before (1) or after (0) the previous batch's row scans
+#endif
 #ifndef NBA_RING_TRACE        // debug variant: per-(batch, CTA) phase stamps into RingRun::ts
 #define NBA_RING_TRACE 0
 #endif
@@ -512,10 +522,48 @@ k_in_fused_ring(DevTable T, InState S, const InBatchArgs *slots, RingRun R, uint
 #define IRTR(bi, k) (R.ts ? R.ts + ((size_t)(bi) * gridDim.x + blockIdx.x) * 16u + (k) : nullptr)
 #endif
 
+// Prefetches for the side warps' prologue, so its loads hit L2: the CTA's
+// range of a batch's metadata arrays (a batch ahead), and -- from the offsets,
+// then in L2 -- the outer headers of its packets (at the start of the
+// iteration before the prologue, ahead of the row scans).
+__device__ __forceinline__ void in_pipe_prefetch_meta(const InBatchArgs &B, uint32_t ppc, uint32_t pt)
+{
+    const uint32_t p_begin = blockIdx.x * ppc;
+    const uint32_t p_end = min(B.n, p_begin + ppc);
+    if (p_end <= p_begin) return;
+    auto lines = [&](const void *base, uint32_t esz) {
+        const uintptr_t a = reinterpret_cast<uintptr_t>(base) + (uintptr_t)p_begin * esz;
+        const uintptr_t e = reinterpret_cast<uintptr_t>(base) + (uintptr_t)p_end * esz;
+        for (uintptr_t x = (a & ~(uintptr_t)127) + 128u * pt; x < e; x += 128u * PIPE_P)
+            prefetch_l2(reinterpret_cast<const void *>(x));
+    };
+    lines(B.sa_idx, 4u);
+    lines(B.in_len, 2u);
+    lines(B.in_off, 4u);
+    lines(B.out_off, 4u);
+}
+
+__device__ __forceinline__ void in_pipe_prefetch_hdr(const InBatchArgs &B, uint32_t ppc, uint32_t pt)
+{
+    constexpr uint32_t PR = PIPE_MAX_PPC / PIPE_P;
+    const uint32_t p_begin = blockIdx.x * ppc;
+    const uint32_t p_end = min(B.n, p_begin + ppc);
+    const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
+    uint32_t off[PR];
+#pragma unroll
+    for (uint32_t r = 0; r < PR; r++) {
+        const uint32_t j = r * PIPE_P + pt;
+        off[r] = j < cnt ? B.in_off[p_begin + j] : 0u;
+    }
+#pragma unroll
+    for (uint32_t r = 0; r < PR; r++)
+        if (r * PIPE_P + pt < cnt) prefetch_l2(B.in_buf + off[r]);
+}
+
 // Metadata + format checks + length order of one inbound batch by the 64
 // prologue threads (pt = 0..63) of this CTA.
 __device__ __forceinline__ void in_pipe_prologue(const DevTable &T, const InBatchArgs &B, uint32_t ppc,
-                                                 FusedLo &L, uint32_t pt)
+                                                 FusedLo &L, uint32_t pt, unsigned long long *tr = nullptr)
 {
     constexpr uint32_t PR = PIPE_MAX_PPC / PIPE_P;                  // 7 rounds
     const uint32_t lane = pt & 31u, pw = pt >> 5;
@@ -523,37 +571,56 @@ __device__ __forceinline__ void in_pipe_prologue(const DevTable &T, const InBatc
     const uint32_t p_end = min(B.n, p_begin + ppc);
     const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
     const uint32_t rounds = (cnt + PIPE_P - 1u) / PIPE_P;
-    uint32_t mS[PR], mL[PR], mI[PR];
+    uint32_t mS[PR], mL[PR], mI[PR], mO[PR];
 #pragma unroll
     for (uint32_t r = 0; r < PR; r++) {                             // all loads issued together
         const uint32_t j = r * PIPE_P + pt, i = p_begin + j;
         mS[r] = j < cnt ? B.sa_idx[i] : INVALID_SA;
         mL[r] = j < cnt ? B.in_len[i] : 0u;
         mI[r] = j < cnt ? B.in_off[i] : 0u;
+        mO[r] = j < cnt ? B.out_off[i] : 0u;
     }
 #pragma unroll
     for (uint32_t r = 0; r < PR; r++)                               // outer headers -> L2 / L1
         if (r * PIPE_P + pt < cnt) prefetch_l2(B.in_buf + mI[r]);
+    // format checks, the header loads of several rounds in flight together
+    // (no shared-memory side effects in between), then the stores
+    // (NBA_IN_LANE_FORMAT: the lanes check the format themselves; here the
+    // payload length the length order and the LPT costs use, and the outer
+    // length in place of the sequence number)
+    uint32_t mF[PR], mQ[PR], mV0[PR], mV1[PR];
 #pragma unroll
-    for (uint32_t r = 0; r < PR; r++) {                             // (unrolled: mS[r] in registers)
+    for (uint32_t r = 0; r < PR; r++) {
+        mF[r] = mQ[r] = mV0[r] = mV1[r] = 0u;
+        if (NBA_IN_LANE_FORMAT) {
+            const uint32_t Lin = mL[r];
+            if (mS[r] < T.n_sa && Lin >= IN_MIN_LEN && Lin <= IN_MAX_LEN && ((Lin - 48u) & 3u) == 0)
+                mF[r] = (Lin - 48u) | INFO_OK;
+            mQ[r] = Lin;
+        } else if (r * PIPE_P + pt < cnt) {
+            in_format(T, B, mS[r], mL[r], mI[r], mF[r], mQ[r], mV0[r], mV1[r]);
+        }
+    }
+    if (tr && pt == 0) tr[10] = gtimer();
+#pragma unroll
+    for (uint32_t r = 0; r < PR; r++) {                             // (unrolled: arrays in registers)
         if (r >= rounds) break;
-        const uint32_t j = r * PIPE_P + pt, i = p_begin + j;
+        const uint32_t j = r * PIPE_P + pt;
         uint32_t bin = NBINS - 1;
         if (j < cnt) {
-            uint32_t info, q, iv0, iv1;
-            in_format(T, B, mS[r], mL[r], mI[r], info, q, iv0, iv1);
             L.sa[j] = mS[r];
-            L.info[j] = info;
-            L.seq[j] = q;
+            L.info[j] = mF[r];
+            L.seq[j] = mQ[r];
             L.inoff[j] = mI[r];
-            L.outoff[j] = B.out_off[i];
-            L.aux0[j] = iv0;
-            L.aux1[j] = iv1;
-            if (info) bin = hmac_bin(true, info & 0xffffu);
+            L.outoff[j] = mO[r];
+            L.aux0[j] = mV0[r];
+            L.aux1[j] = mV1[r];
+            if (mF[r]) bin = hmac_bin(true, mF[r] & 0xffffu);
         }
         warp_agg_add(L.bins, bin, j < cnt);
     }
     bar_sync_n(1, PIPE_P);
+    if (tr && pt == 0) tr[11] = gtimer();
     bool one_bin = false;
     if (pw == 0) {                                                  // bins -> cursors
         const uint32_t cb = L.bins[lane];
@@ -581,6 +648,7 @@ __device__ __forceinline__ void in_pipe_prologue(const DevTable &T, const InBatc
         if (j < cnt) L.perm[pos] = (uint16_t)j;
     }
     bar_sync_n(1, PIPE_P);
+    if (tr && pt == 0) tr[12] = gtimer();
     if (pt < NBINS) L.bins[pt] = 0u;
     if (pw == 0) {
         // runs of 32 sorted positions -> lane warps, longest first onto the
@@ -600,33 +668,31 @@ __device__ __forceinline__ void in_pipe_prologue(const DevTable &T, const InBatc
     }
 }
 
-// Batch k's anti-replay tail by the whole CTA (thread j <-> packet p_begin + j):
-// in_merged_tail with the flags / sequence numbers from L.tailf / L.tailq, the
-// group maxima in the round-key slots, and the duplicate hash cleared here.
-__device__ __forceinline__ void in_pipe_tail(const DevTable &T, const InState &S, const InBatchArgs &B,
-                                             FusedLo &L, FusedHi &H, uint32_t p_begin, uint32_t p_end,
-                                             uint32_t hmask, uint32_t bar_base,
-                                             unsigned long long *next_hkey, uint32_t *next_hval,
-                                             unsigned long long *tr = nullptr)
+// Batch k's tile part by the whole CTA (thread j <-> packet p_begin + j), the
+// first half of in_merged_tail: warp-segmented prefix maxima of the
+// authenticated sequence numbers per SA, the CTA's SA hash, the (SA, CTA)
+// tile maxima into S.hmax; each packet's decision inputs (flags, number,
+// prefix max within the CTA, SA) go to the CTA's scratch row, and the CTA
+// arrives at the batch's first barrier (SB1) without waiting for it.  The
+// per-warp group maxima live in the lanes' round-key slots (L.rkA / H.rkB,
+// free once the lanes are done), so the T-tables stay in shared memory.
+__device__ __forceinline__ void in_pipe_tile(const InState &S, FusedLo &L, FusedHi &H, uint32_t cnt,
+                                             uint4 *scr)
 {
-    __shared__ unsigned long long s_cnt[N_IN_COUNTERS - 1];
     constexpr uint32_t HS = 2u * F_SUPER, NW = F_THREADS / 32u;
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
-    const uint32_t G = gridDim.x, cta = blockIdx.x, n_sa = T.n_sa;
-    const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
-    const uint32_t j = tid, i = p_begin + j;
+    const uint32_t G = gridDim.x, cta = blockIdx.x;
+    const uint32_t j = tid;
     const bool live = j < cnt;
     const uint32_t f = live ? L.tailf[j] : 0u;
     const uint32_t sa = live ? L.tails[j] : INVALID_SA;
     const uint32_t q = (f & INF_FMT) ? L.tailq[j] : 0u;
     const uint32_t key = (f & INF_FMT) ? sa : INVALID_SA;
-    const bool inA = (f & INF_ICV) != 0u;
-    const uint32_t qa = inA ? q : 0u;
+    const uint32_t qa = (f & INF_ICV) ? q : 0u;
     for (uint32_t k = tid; k < HS; k += F_THREADS) {
         L.hkey[k] = INVALID_SA;
         L.hmask[k] = 0;
     }
-    if (tid < N_IN_COUNTERS - 1) s_cnt[tid] = 0;
     // per-warp group maxima [HS][NW] u32: slots < 512 in L.rkA, the rest in H.rkB
     auto gm = [&](uint32_t slot) -> uint32_t * {
         uint32_t *b = slot < 512u ? reinterpret_cast<uint32_t *>(&L.rkA[0][0])
@@ -663,44 +729,142 @@ __device__ __forceinline__ void in_pipe_tail(const DevTable &T, const InState &S
         if ((m >> (warp + 1u)) == 0u && lane == hi_lane && tmax != 0u)
             S.hmax[(size_t)key * G + cta] = tmax;
     }
-    const uint32_t lmax = max(base, mex);
-    // ((sa, q) -> first index of the authenticated packets went into this
-    // batch's hash from the lanes, right after each packet's ICV check)
+    if (live) scr[j] = make_uint4(f, q, max(base, mex), sa);
     __syncthreads();
-    if (tr && tid == 0) tr[6] = gtimer();
     grid_arrive(&S.ctl[CTLI_BAR]);
-    grid_wait(&S.ctl[CTLI_BAR], bar_base + G);
-    if (tr && tid == 0) tr[1] = gtimer();
-    scan_all_rows(S, n_sa, warp * G + cta, G * NW, G, lane);   // SA s on CTA s mod G
-    if (tr && lane == 0) atomicMax(&tr[8], gtimer());
-    // the next batch's hash: its last user (the batch before this one) made
-    // its lookups before this batch's first barrier; every CTA clears its
-    // slice before arriving at the second barrier, which the next batch's
-    // inserts follow
-    for (uint32_t k = cta * F_THREADS + tid; k <= hmask; k += G * F_THREADS) {
-        next_hkey[k] = ~0ull;
-        next_hval[k] = ~0u;
+}
+
+// Side-warp grid barrier: only the 64 prologue threads of each CTA wait.
+__device__ __forceinline__ void side_wait(const uint32_t *count, uint32_t target, uint32_t pt)
+{
+    if (pt == 0) {
+        uint32_t v;
+        do {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(count) : "memory");
+        } while ((int)(v - target) < 0);
     }
-    if (tr) {
-        __syncwarp();
-        if (lane == 0) atomicMax(&tr[7], gtimer());
+    bar_sync_n(1, PIPE_P);
+}
+
+// Row scans of SA rows sa0, sa0 + stride, ... by one warp, RW rows at a time
+// with every load of the RW rows issued first; n_tiles <= 160, lane l holding
+// tiles 5 l .. 5 l + 4 (a running max in registers, one warp scan of the lane
+// maxima).  The arithmetic of scan_max_row.
+__device__ __forceinline__ void scan_rows_batched(const InState &S, uint32_t sa0, uint32_t stride,
+                                                  uint32_t n_sa, uint32_t n_tiles, uint32_t lane)
+{
+    constexpr int RW = 4, U = 5;
+    for (uint32_t b = sa0; b < n_sa; b += RW * stride) {
+        uint32_t h[RW][U], w0[RW];
+        unsigned long long b0[RW];
+#pragma unroll
+        for (int r = 0; r < RW; r++) {
+            const uint32_t sa = b + r * stride;
+            const bool ok = sa < n_sa;
+#pragma unroll
+            for (int u = 0; u < U; u++) {
+                const uint32_t t = U * lane + u;
+                h[r][u] = ok && t < n_tiles ? __ldcg(&S.hmax[(size_t)sa * n_tiles + t]) : 0u;
+            }
+            w0[r] = ok && lane == 0 ? S.top[sa] : 0u;
+            b0[r] = ok && lane == 0 ? S.bmp[sa] : 0ull;
+        }
+#pragma unroll
+        for (int r = 0; r < RW; r++) {
+            const uint32_t sa = b + r * stride;
+            if (sa >= n_sa) break;
+            uint32_t lm = 0;                                       // this lane's tiles' max
+#pragma unroll
+            for (int u = 0; u < U; u++) lm = max(lm, h[r][u]);
+            uint32_t x = lm;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+                if (lane >= (uint32_t)o) x = max(x, y);
+            }
+            uint32_t run = __shfl_up_sync(0xffffffffu, x, 1);      // max over the earlier lanes
+            if (lane == 0) run = 0;
+            const uint32_t carry = __shfl_sync(0xffffffffu, x, 31);
+#pragma unroll
+            for (int u = 0; u < U; u++) {
+                const uint32_t t = U * lane + u;
+                if (t < n_tiles) {
+                    S.pmx[(size_t)sa * n_tiles + t] = run;
+                    if (h[r][u]) S.hmax[(size_t)sa * n_tiles + t] = 0;   // re-arm
+                }
+                run = max(run, h[r][u]);
+            }
+            if (lane == 0) window_advance(S, sa, carry, w0[r], b0[r]);
+        }
     }
-    __syncthreads();
-    if (tr && tid == 0) tr[9] = gtimer();
-    grid_arrive(&S.ctl[CTLI_BAR]);
-    grid_wait(&S.ctl[CTLI_BAR], bar_base + 2u * G);
-    if (tr && tid == 0) tr[2] = gtimer();
+}
+
+// Batch k's replay, second half, part 1 by the 64 side threads of the CTA
+// while the lanes run batch k + 1: wait for every CTA's tile part (SB1 =
+// sb1), this CTA's share of the SA row scans (prefix maxima down each
+// (SA, CTA) row, window edge update), arrival at SB2 (its own counter,
+// CTLI_BAR2: a CTA with no packets in batch k does not wait for SB2, so its
+// next tile arrival must not count towards it), and this CTA's slice of the
+// duplicate hash clr (batch k + 3's) cleared.
+__device__ __forceinline__ void in_pipe_rows(const DevTable &T, const InState &S, uint32_t hmask,
+                                             uint32_t sb1, unsigned long long *clr_k, uint32_t *clr_v,
+                                             uint32_t pt, unsigned long long *tr)
+{
+    const uint32_t lane = pt & 31u, pw = pt >> 5;
+    const uint32_t G = gridDim.x, cta = blockIdx.x;
+    side_wait(&S.ctl[CTLI_BAR], sb1, pt);
+    if (tr && pt == 0) tr[1] = gtimer();
+    scan_rows_batched(S, pw * G + cta, 2u * G, T.n_sa, G, lane);
+    bar_sync_n(1, PIPE_P);                           // (orders both warps' stores before the arrival)
+    if (pt == 0) asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&S.ctl[CTLI_BAR2]) : "memory");
+    if (tr && pt == 0) tr[8] = gtimer();
+    if (clr_k)
+        for (uint32_t k = cta * PIPE_P + pt; k <= hmask; k += G * PIPE_P) {
+            clr_k[k] = ~0ull;
+            clr_v[k] = ~0u;
+        }
+}
+
+// Part 2, by one warp for packets j = 32 w + lane of the CTA's batch-k range
+// (w: the warp's slot, 0..13 -- the lane warps once their own packets are
+// done): wait for SB2 (every row scanned, sb2), then the decisions:
+// statuses, lengths, counters into the CTA's shared counters.
+__device__ __forceinline__ void in_pipe_decide(const DevTable &T, const InState &S, const InBatchArgs &B,
+                                               uint32_t ppc, const uint4 *scr, uint32_t hmask,
+                                               const unsigned long long *hk, const uint32_t *hv,
+                                               uint32_t sb2, uint32_t w, unsigned long long *s_cnt)
+{
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t G = gridDim.x, cta = blockIdx.x, n_sa = T.n_sa;
+    const uint32_t p_begin = cta * ppc;
+    const uint32_t p_end = min(B.n, p_begin + ppc);
+    const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
+    if (32u * w >= cnt) return;
+    if (lane == 0) {
+        uint32_t v;
+        do {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(&S.ctl[CTLI_BAR2]) : "memory");
+        } while ((int)(v - sb2) < 0);
+    }
+    __syncwarp();
+    const uint32_t j = 32u * w + lane, i = p_begin + j;
     uint32_t st = 0xffu, D = 0, Lin = 0;
-    if (live) {
+    if (j < cnt) {
+        const uint4 d = scr[j];
+        const uint32_t f = d.x, q = d.y, sa = d.w;
         if (sa >= n_sa) {
             st = ST_DROP_SA;
         } else if (!(f & INF_FMT)) {
             st = ST_DROP_FORMAT;
         } else {
-            const uint32_t t0 = S.top_prev[sa];
-            const unsigned long long b0 = S.bmp_prev[sa];
-            const uint32_t tj = max(t0, max(S.pmx[(size_t)sa * G + cta], lmax));
-            st = replay_decide(S, sa, i, f, q, t0, b0, tj, S.top[sa], hmask);
+            const uint32_t t0 = __ldcg(&S.top_prev[sa]);
+            const unsigned long long b0 = __ldcg(&S.bmp_prev[sa]);
+            const uint32_t pm = __ldcg(&S.pmx[(size_t)sa * G + cta]);
+            const uint32_t t1 = __ldcg(&S.top[sa]);
+            InState Sd = S;
+            Sd.hkey = const_cast<unsigned long long *>(hk);
+            Sd.hval = const_cast<uint32_t *>(hv);
+            st = replay_decide(Sd, sa, i, f, q, t0, b0, max(t0, max(pm, d.z)), t1, hmask);
             if (st == ST_OK) {
                 D = f & 0xffffu;
                 Lin = B.in_len[i];
@@ -710,23 +874,21 @@ __device__ __forceinline__ void in_pipe_tail(const DevTable &T, const InState &S
         if (B.status) B.status[i] = (uint8_t)st;
     }
     // counters: pkts_ok, drop_sa, drop_format, drop_replay, drop_auth,
-    // drop_trailer, bytes_in, bytes_out (warp sums -> shared -> one atomic per CTA)
+    // drop_trailer, bytes_in, bytes_out (warp sums into the CTA's counters)
 #pragma unroll
     for (uint32_t k = 0; k < 6; k++) {
-        const uint32_t c = __reduce_add_sync(0xffffffffu, st == k ? 1u : 0u);
-        if (lane == 0 && c) atomicAdd(&s_cnt[k], (unsigned long long)c);
+        const uint32_t x = __reduce_add_sync(0xffffffffu, st == k ? 1u : 0u);
+        if (lane == 0 && x) atomicAdd(&s_cnt[k], (unsigned long long)x);
     }
-    const uint32_t bi_ = __reduce_add_sync(0xffffffffu, Lin);
-    const uint32_t bo_ = __reduce_add_sync(0xffffffffu, D);
-    if (lane == 0 && bi_) atomicAdd(&s_cnt[6], (unsigned long long)bi_);
-    if (lane == 0 && bo_) atomicAdd(&s_cnt[7], (unsigned long long)bo_);
-    __syncthreads();
-    if (tid < N_IN_COUNTERS - 1 && s_cnt[tid]) atomicAdd(&S.counters[tid], s_cnt[tid]);
+    const uint32_t xi = __reduce_add_sync(0xffffffffu, Lin);
+    const uint32_t xo = __reduce_add_sync(0xffffffffu, D);
+    if (lane == 0 && xi) atomicAdd(&s_cnt[6], (unsigned long long)xi);
+    if (lane == 0 && xo) atomicAdd(&s_cnt[7], (unsigned long long)xo);
 }
 
 __global__ void __launch_bounds__(F_THREADS, 1)
 k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R, uint32_t hmask,
-                     unsigned long long *hkey_b, uint32_t *hval_b)
+                     InPipeBufs P)
 {
     extern __shared__ __align__(16) uint8_t smem[];
     const uint32_t n_slots = R.n_slots, n_batches = R.n_batches, first = R.first;
@@ -735,6 +897,9 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
     if (n_batches == 0) return;
     if (!NBA_RING_TRACE && R.ts && cta == 0 && tid == 0) R.ts[0] = gtimer();
     const uint32_t base0 = *reinterpret_cast<volatile uint32_t *>(&S.ctl[CTLI_BASE]);
+    // (no row-scan arrival of this launch precedes every CTA's first tile
+    // arrival, which follows this read)
+    const uint32_t base2 = *reinterpret_cast<volatile uint32_t *>(&S.ctl[CTLI_BAR2]);
     const uint32_t sb = smem_u32(smem);
     const uint32_t toff = (0x10000u - (sb & 0xffffu)) & 0xffffu;
     uint32_t lo_off = 0;
@@ -746,13 +911,27 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
     FusedLo &L = *reinterpret_cast<FusedLo *>(smem + lo_off);
     FusedHi &H = *reinterpret_cast<FusedHi *>(smem + toff + AES_TABLE_BYTES);
     const uint32_t lane4r = (lane * 4u) | (smem_u32(tabs) & 0xffff0000u);
+    uint4 *scr = P.scr + (size_t)cta * PIPE_MAX_PPC;
+    // the duplicate hash of batch k: H[k mod 4] (H0 = S.hkey / S.hval)
+    auto hk_of = [&](uint32_t k) {
+        const uint32_t m = k & 3u;
+        return m == 0u ? S.hkey : m == 1u ? P.hk1 : m == 2u ? P.hk2 : P.hk3;
+    };
+    auto hv_of = [&](uint32_t k) {
+        const uint32_t m = k & 3u;
+        return m == 0u ? S.hval : m == 1u ? P.hv1 : m == 2u ? P.hv2 : P.hv3;
+    };
+    __shared__ unsigned long long s_cnt[N_IN_COUNTERS - 1];   // the CTA's decision counters
+    if (tid < N_IN_COUNTERS - 1) s_cnt[tid] = 0ull;
     tables_stage(tabs, T, &L.tbar, true);   // bulk copy, waited for before the first lookup
     if (tid < NBINS) L.bins[tid] = 0u;
-    // the first batch's duplicate hash, cleared by every CTA before a start
-    // barrier that the first inserts (after the first batch's lanes) follow
+    // batches 0 and 1's duplicate hashes, cleared by every CTA before a start
+    // barrier that the first inserts (after batch 0's lanes) follow
     for (uint32_t k = cta * F_THREADS + tid; k <= hmask; k += G * F_THREADS) {
         S.hkey[k] = ~0ull;
         S.hval[k] = ~0u;
+        P.hk1[k] = ~0ull;
+        P.hv1[k] = ~0u;
     }
     __syncthreads();
     grid_arrive(&S.ctl[CTLI_BAR]);
@@ -770,7 +949,10 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
     __syncthreads();
     tables_bulk_wait(&L.tbar, 0u);
     grid_wait(&S.ctl[CTLI_BAR], base0 + G);          // the start barrier (long since complete)
-    const uint32_t bbase = base0 + G;                 // batch bi: barriers bbase + 2 bi G + {G, 2G}
+    // per CTA and batch k: its tile part arrives at CTLI_BAR (SB1(k) complete
+    // at bbase + (k + 1) G) and its row scans at CTLI_BAR2 (SB2(k) at
+    // base2 + (k + 1) G)
+    const uint32_t bbase = base0 + G;
     for (uint32_t bi = 0; bi < n_batches; bi++) {
         const InBatchArgs B = slots[(first + bi) % n_slots];
         const uint32_t ppc = ppc_of(B);
@@ -784,17 +966,20 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
         unsigned long long *tr = nullptr;
 #endif
         if (!isP) {
+            unsigned long long *hk = hk_of(bi);
+            uint32_t *hv = hv_of(bi);
             const uint32_t run = L.wrun[warp];
             const uint32_t pos = 32u * run + lane;
             const bool have = run != 0xffu && pos < cnt;
             const uint32_t pk = have ? L.perm[pos] : 0u;
-            const uint32_t info = have ? L.info[pk] : 0u;
+            uint32_t info = have ? L.info[pk] : 0u;
             const uint32_t sa_raw = have ? L.sa[pk] : INVALID_SA;   // (the tail tells DROP_SA apart)
-            const uint32_t sa = (info & INFO_OK) ? sa_raw : INVALID_SA;
-            const uint32_t q = have ? L.seq[pk] : 0u;
-            const uint32_t iv0 = have ? L.aux0[pk] : 0u, iv1 = have ? L.aux1[pk] : 0u;
+            uint32_t q = have ? L.seq[pk] : 0u;          // (NBA_IN_LANE_FORMAT: the outer length)
+            uint32_t iv0 = have ? L.aux0[pk] : 0u, iv1 = have ? L.aux1[pk] : 0u;
             const uint32_t inoff = have ? L.inoff[pk] : 0u, outoff = have ? L.outoff[pk] : 0u;
             bar_arrive_n(2, F_THREADS);                  // fields taken: the arrays are free
+            if (NBA_IN_LANE_FORMAT && have) in_format(T, B, sa_raw, q, inoff, info, q, iv0, iv1);
+            const uint32_t sa = (info & INFO_OK) ? sa_raw : INVALID_SA;
             if (have) {
                 uint32_t flags = 0;
                 if (info & INFO_OK) {
@@ -805,51 +990,87 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
                     expand_key_lane(lane4r, r0, r1, r2, L, H, tid);
                     flags = INF_FMT | esp_in_packet(T, B, L, H, lane4r, tid, sa, info & 0xffffu, q, iv0,
                                                     iv1, inoff, outoff, r0, r1, r2, hd, h0, h1);
-                    // (sa, q) -> first index into this batch's duplicate hash
-                    // (cleared during the previous batch, before its second
-                    // barrier; read after this batch's first): the atomics'
-                    // latency overlaps the other lanes' crypto
-                    if (flags & INF_ICV)
-                        replay_hash_insert((bi & 1u) ? hkey_b : S.hkey, (bi & 1u) ? hval_b : S.hval, sa,
-                                           q, p_begin + pk, hmask);
+                    // (sa, q) -> first index into batch bi's duplicate hash
+                    // (cleared during batch bi - 2, read by batch bi's
+                    // decisions during batch bi + 1): the atomics' latency
+                    // overlaps the other lanes' crypto
+                    if (flags & INF_ICV) replay_hash_insert(hk, hv, sa, q, p_begin + pk, hmask);
                 }
                 L.tailf[pk] = flags;
                 L.tailq[pk] = q;
                 L.tails[pk] = sa_raw;
             }
             if (tr && lane == 0) atomicMax(&tr[3], gtimer());
+            if (bi > 0) {
+                // batch bi - 1's decisions for this warp's 32 packet slots,
+                // once every CTA's side warps scanned their rows (SB2)
+                const InBatchArgs Bp = slots[(first + bi - 1) % n_slots];
+                in_pipe_decide(T, S, Bp, ppc_of(Bp), scr, hmask, hk_of(bi - 1), hv_of(bi - 1),
+                               base2 + bi * G, warp, s_cnt);
+                if (tr && lane == 0) atomicMax(&tr[9], gtimer());
+            }
         } else {
             bar_sync_n(2, F_THREADS);                    // every lane took its fields
-            if (bi + 1 < n_batches) {
+            // batch bi - 1's row scans and batch bi + 2's hash cleared (its
+            // last user, batch bi - 2, decided before every CTA's tile part
+            // of batch bi - 1), and batch bi + 1's prologue
+            const bool more = bi + 1 < n_batches;
+            if (NBA_IN_PREFETCH && more) {
                 const InBatchArgs Bn = slots[(first + bi + 1) % n_slots];
-                in_pipe_prologue(T, Bn, ppc_of(Bn), L, pt);
+                in_pipe_prefetch_hdr(Bn, ppc_of(Bn), pt);
+                if (bi + 2 < n_batches) {
+                    const InBatchArgs Bm = slots[(first + bi + 2) % n_slots];
+                    in_pipe_prefetch_meta(Bm, ppc_of(Bm), pt);
+                }
+            }
+            if (NBA_IN_PRO_FIRST && more) {
+                const InBatchArgs Bn = slots[(first + bi + 1) % n_slots];
+                in_pipe_prologue(T, Bn, ppc_of(Bn), L, pt, tr);
+            }
+            if (bi > 0) {
+                in_pipe_rows(T, S, hmask, bbase + bi * G, hk_of(bi + 2), hv_of(bi + 2), pt, tr);
+            } else {
+                for (uint32_t k = cta * PIPE_P + pt; k <= hmask; k += G * PIPE_P) {
+                    P.hk2[k] = ~0ull;
+                    P.hv2[k] = ~0u;
+                }
+            }
+            if (!NBA_IN_PRO_FIRST && more) {
+                const InBatchArgs Bn = slots[(first + bi + 1) % n_slots];
+                in_pipe_prologue(T, Bn, ppc_of(Bn), L, pt, tr);
             }
             if (tr && pt == 0) tr[4] = gtimer();
         }
-        __syncthreads();                                  // lanes done, bi + 1 prepared
-        InState Sb = S;
-        if (bi & 1u) {
-            Sb.hkey = hkey_b;
-            Sb.hval = hval_b;
-        }
-        in_pipe_tail(T, Sb, B, L, H, p_begin, p_end, hmask, bbase + 2u * bi * G,
-                     (bi & 1u) ? S.hkey : hkey_b, (bi & 1u) ? S.hval : hval_b, tr);
-        __syncthreads();                                  // the tail's scratch is free again
+        __syncthreads();                                  // lanes done, bi - 1 decided, bi + 1 prepared
+        if (!NBA_RING_TRACE && R.ts && bi > 0 && tid == 0) atomicMax(&R.ts[bi], gtimer());
+        in_pipe_tile(S, L, H, cnt, scr);                  // (ends with the SB1(bi) arrival)
+        if (tr && tid == 0) tr[6] = gtimer();
+        __syncthreads();                                  // the tile part's scratch is free again
 #if NBA_RING_TRACE
         if (tr && tid == 0) tr[5] = gtimer();
-#else
-        if (R.ts && tid == 0) atomicMax(&R.ts[1u + bi], gtimer());
 #endif
     }
+    // the last batch's replay: row scans by the side warps, decisions by the lane warps
+    const uint32_t bl = n_batches - 1u;
+    if (isP) {
+        in_pipe_rows(T, S, hmask, bbase + (bl + 1u) * G, nullptr, nullptr, pt, nullptr);
+    } else {
+        const InBatchArgs Bp = slots[(first + bl) % n_slots];
+        in_pipe_decide(T, S, Bp, ppc_of(Bp), scr, hmask, hk_of(bl), hv_of(bl), base2 + (bl + 1u) * G, warp,
+                       s_cnt);
+    }
+    __syncthreads();
+    if (tid < N_IN_COUNTERS - 1 && s_cnt[tid]) atomicAdd(&S.counters[tid], s_cnt[tid]);
+    if (!NBA_RING_TRACE && R.ts && tid == 0) atomicMax(&R.ts[1u + bl], gtimer());
     if (tid == 0 && cta == 0) {
         atomicAdd(&S.counters[N_IN_COUNTERS - 1], (unsigned long long)n_batches);
-        S.ctl[CTLI_BASE] = bbase + 2u * n_batches * G;   // a start barrier, two per batch
+        S.ctl[CTLI_BASE] = bbase + n_batches * G;        // a start barrier, one tile arrival per batch
     }
 }
 
 cudaError_t launch_in_fused_ring_pipe(const DevTable &T, const InState &S, const InBatchArgs *slots,
-                                      const RingRun &R, uint32_t hmask, unsigned long long *hkey_b,
-                                      uint32_t *hval_b, int grid, cudaStream_t st)
+                                      const RingRun &R, uint32_t hmask, const InPipeBufs &P, int grid,
+                                      cudaStream_t st)
 {
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(grid);
@@ -861,7 +1082,7 @@ cudaError_t launch_in_fused_ring_pipe(const DevTable &T, const InState &S, const
     attr[0].val.cooperative = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    return cudaLaunchKernelEx(&cfg, k_in_fused_ring_pipe, T, S, slots, R, hmask, hkey_b, hval_b);
+    return cudaLaunchKernelEx(&cfg, k_in_fused_ring_pipe, T, S, slots, R, hmask, P);
 }
 
 bool in_pipe_ok(uint32_t n, int grid)

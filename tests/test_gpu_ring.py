@@ -126,10 +126,12 @@ def test_ring_two_kernel_and_unfused_paths(n, pipeline):
 @pytest.mark.parametrize("form", ["graph", "persistent", "pipelined"])
 def test_inbound_ring_equals_stream_launches_and_oracle(form, monkeypatch):
     """ESP inbound slots in a ring (graph form, the opt-in plain persistent form
-    and the default software-pipelined form): status, inner bytes, lengths,
+    and the software-pipelined form, each forced): status, inner bytes, lengths,
     windows and counters equal process_inbound from the stream and the
     oracle's receiver."""
     import torch
+    if form == "graph":
+        monkeypatch.setenv("NBA_IPSEC_RING_IN_PIPE", "0")
     if form == "persistent":
         monkeypatch.setenv("NBA_IPSEC_RING_IN_PERSIST", "1")
     if form == "pipelined":
@@ -453,4 +455,37 @@ def test_inbound_pipelined_ring_mixed_stream(n_sa, sizes, monkeypatch):
             o_top, o_bmp = oracle.window_state(win, n_sa)
             assert np.array_equal(top, o_top) and np.array_equal(bmp, o_bmp)
             assert t.in_counters() == ctr.as_dict()
+        ring.close()
+
+
+@pytest.mark.parametrize("size,form", [(64, "pipelined"), (512, "pipelined"), (1024, "graph"),
+                                       ("imix", "graph")])
+def test_inbound_ring_form_choice(size, form):
+    """Without overrides an inbound ring takes the pipelined form when every
+    packet's outer length is <= 640 B and the graph form otherwise (DESIGN
+    §5); either way the output equals the oracle's receiver."""
+    import torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    n_sa, n = 64, 3000
+    p = gen.make_sas(n_sa, cfg_id=77)
+    sas = oracle.make_sas(p)
+    b = gen.make_batch(n, size, n_sa, cfg_id=77)
+    e_out, e_len, _ = oracle.process_batch(sas, n_sa, b)
+    ib = gen.esp_batch(e_out, b.out_off, e_len, b.sa_idx, np.arange(n))
+    win = oracle.make_windows(oracle.make_sas(p), n_sa)
+    o_out, o_len, o_st, _ = oracle.process_inbound(oracle.make_sas(p), win, n_sa, ib)
+    with nba_ipsec.SATable(p, device=0, max_batch=n) as t:
+        t.enable_inbound()
+        d = device.to_device(ib, "cuda")
+        st = torch.zeros(n, dtype=torch.uint8, device="cuda")
+        ring = t.ring_inbound([(*d.args(), st, n)])
+        assert ring.form == {"graph": ring.GRAPH, "pipelined": ring.PIPELINED}[form]
+        ring.run_batches(1)
+        torch.cuda.synchronize()
+        g_out, g_len = device.fetch(d)
+        assert np.array_equal(st.cpu().numpy(), o_st)
+        assert np.array_equal(g_len, o_len)
+        for i in np.nonzero(o_len)[0]:
+            a, L = int(ib.out_off[i]), int(o_len[i])
+            assert np.array_equal(g_out[a:a + L], o_out[a:a + L])
         ring.close()

@@ -53,9 +53,12 @@ for size in %(sizes)r:
         t0 = v[:, :, :1].min(axis=1, keepdims=True)       # the batch's first CTA start
         v = np.where(v > 0, v, t0)                          # (stamps a form does not take)
         rel = (v - t0) / 1e3
-        names = {0: "iter_start", 1: "bar1_passed", 2: "bar2_passed", 3: "lanes_done", 4: "side_done",
-                 5: "iter_end", 6: "tail_tile_done", 7: "next_hash_cleared", 8: "row_scans_done",
-                 9: "cta_done_mid"}
+        # pipelined ring: 1 / 8 are the side warps' row scans of the PREVIOUS
+        # batch during this one (SB1 passed, scans done), 9 the lane warps'
+        # decisions of the previous batch
+        names = {0: "iter_start", 1: "prev_sb1_passed", 3: "lanes_done", 4: "side_done", 5: "iter_end",
+                 6: "tile_done", 8: "prev_row_scans_done", 9: "prev_decisions_done",
+                 10: "pro_formats_done", 11: "pro_stored", 12: "pro_sorted"}
         out[str(size)] = {n: [round(float(np.median(rel[:, :, i])), 2),
                               round(float(np.median(np.max(rel[:, :, i], axis=1))), 2)]
                           for i, n in names.items()}
