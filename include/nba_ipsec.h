@@ -109,8 +109,11 @@ int nba_ipsec_create_sa_table(const nba_ipsec_sa_params *sas, uint32_t n_sa, int
 int nba_ipsec_process_batch(nba_ipsec_sa_table *t, const nba_ipsec_batch *b, void *cuda_stream);
 
 /* Same computation with HOST buffers (end-to-end path): copies
- * in_buf[0, in_buf_bytes), in_off, in_len, sa_idx host->device, runs the
- * path, copies out_buf[0, out_buf_bytes) and out_len device->host.  The copies
+ * in_buf[0, in_buf_bytes) host->device, runs the path, copies
+ * out_buf[0, out_buf_bytes) device->host.  The per-packet arrays (in_off,
+ * in_len, sa_idx, out_off, out_len) are read / written by the kernels in place
+ * when all five are page-locked memory the device can address (cudaHostAlloc,
+ * cudaHostRegister), else staged with copies like in_buf.  The copies
  * and the kernels run on three internal streams with two staging slots, so
  * consecutive calls overlap batch k+1's copy-in and batch k-1's copy-out with
  * batch k's kernels (pinned host memory makes the copies asynchronous).

@@ -822,6 +822,37 @@ int nba_ipsec_process_batch_host(nba_ipsec_sa_table *t, const nba_ipsec_batch *b
     uint32_t *d_out_off = d_sa + t->max_batch;
     uint16_t *d_in_len = reinterpret_cast<uint16_t *>(d_out_off + t->max_batch);
     uint16_t *d_out_len = d_in_len + t->max_batch;
+    // Per-packet metadata in page-locked host memory the device can address
+    // (cudaHostAlloc'd or registered) is read -- and out_len written -- by the
+    // kernels in place over PCIe, once per packet, so only the two large
+    // buffers go through the copy engines: the four small copies in and one
+    // out cost ~50 us per 65,536-packet step in copy-engine time
+    // (tools/pcie_probe.py).  Otherwise the metadata is staged like in_buf.
+    auto mapped = [](const void *p) -> void * {
+        cudaPointerAttributes a;
+        if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+            cudaGetLastError();
+            return nullptr;
+        }
+        return a.type == cudaMemoryTypeHost ? a.devicePointer : nullptr;
+    };
+    bool zc = !std::getenv("NBA_IPSEC_HOST_STAGE_META");
+    void *z_in_off = nullptr, *z_sa = nullptr, *z_out_off = nullptr, *z_in_len = nullptr, *z_out_len = nullptr;
+    if (zc) {
+        z_in_off = mapped(b->in_off);
+        z_sa = mapped(b->sa_idx);
+        z_out_off = mapped(b->out_off);
+        z_in_len = mapped(b->in_len);
+        z_out_len = mapped(b->out_len);
+        zc = z_in_off && z_sa && z_out_off && z_in_len && z_out_len;
+    }
+    if (zc) {
+        d_in_off = static_cast<uint32_t *>(z_in_off);
+        d_sa = static_cast<uint32_t *>(z_sa);
+        d_out_off = static_cast<uint32_t *>(z_out_off);
+        d_in_len = static_cast<uint16_t *>(z_in_len);
+        d_out_len = static_cast<uint16_t *>(z_out_len);
+    }
     cudaError_t e = cudaSuccess;
     auto chk = [&](cudaError_t x) {
         if (e == cudaSuccess && x != cudaSuccess) e = x;
@@ -829,10 +860,12 @@ int nba_ipsec_process_batch_host(nba_ipsec_sa_table *t, const nba_ipsec_batch *b
     // copy-in: after this slot's previous copy-out has drained its buffers
     chk(cudaStreamWaitEvent(t->s_h2d, sl.out_done, 0));
     chk(cudaMemcpyAsync(sl.in, b->in_buf, in_buf_bytes, cudaMemcpyHostToDevice, t->s_h2d));
-    chk(cudaMemcpyAsync(d_in_off, b->in_off, n * 4ull, cudaMemcpyHostToDevice, t->s_h2d));
-    chk(cudaMemcpyAsync(d_sa, b->sa_idx, n * 4ull, cudaMemcpyHostToDevice, t->s_h2d));
-    chk(cudaMemcpyAsync(d_out_off, b->out_off, n * 4ull, cudaMemcpyHostToDevice, t->s_h2d));
-    chk(cudaMemcpyAsync(d_in_len, b->in_len, n * 2ull, cudaMemcpyHostToDevice, t->s_h2d));
+    if (!zc) {
+        chk(cudaMemcpyAsync(d_in_off, b->in_off, n * 4ull, cudaMemcpyHostToDevice, t->s_h2d));
+        chk(cudaMemcpyAsync(d_sa, b->sa_idx, n * 4ull, cudaMemcpyHostToDevice, t->s_h2d));
+        chk(cudaMemcpyAsync(d_out_off, b->out_off, n * 4ull, cudaMemcpyHostToDevice, t->s_h2d));
+        chk(cudaMemcpyAsync(d_in_len, b->in_len, n * 2ull, cudaMemcpyHostToDevice, t->s_h2d));
+    }
     chk(cudaEventRecord(sl.in_ready, t->s_h2d));
     // compute: after the inputs and after everything the caller's stream holds
     // (keeps the SA counters in call order with device-path batches)
@@ -848,7 +881,7 @@ int nba_ipsec_process_batch_host(nba_ipsec_sa_table *t, const nba_ipsec_batch *b
     // copy-out
     chk(cudaStreamWaitEvent(t->s_d2h, sl.done, 0));
     chk(cudaMemcpyAsync(b->out_buf, sl.out, out_buf_bytes, cudaMemcpyDeviceToHost, t->s_d2h));
-    chk(cudaMemcpyAsync(b->out_len, d_out_len, n * 2ull, cudaMemcpyDeviceToHost, t->s_d2h));
+    if (!zc) chk(cudaMemcpyAsync(b->out_len, d_out_len, n * 2ull, cudaMemcpyDeviceToHost, t->s_d2h));
     chk(cudaEventRecord(sl.out_done, t->s_d2h));
     return e == cudaSuccess ? NBA_IPSEC_OK : NBA_IPSEC_ECUDA;
 }

@@ -207,13 +207,20 @@ def test_concurrent_tables_on_two_streams():
         ts[k].close()
 
 
-def test_host_buffer_path_pipelined_and_mixed():
+@pytest.mark.parametrize("meta", ["in_place", "staged", "pageable"])
+def test_host_buffer_path_pipelined_and_mixed(meta, monkeypatch):
     """nba_ipsec_process_batch_host (the e2e API): pinned host buffers, three
     batches in flight through the copy-in / kernels / copy-out pipeline, then a
     device-path batch and another host batch on the same table: outputs, lengths,
-    counters and SA counters equal the oracle's sequential run."""
+    counters and SA counters equal the oracle's sequential run.  The per-packet
+    arrays read / written by the kernels in place (pinned), staged by copies
+    (forced), or staged because they are pageable."""
     import torch
     from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    if meta == "staged":
+        monkeypatch.setenv("NBA_IPSEC_HOST_STAGE_META", "1")
+    pin_meta = (lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()) if meta != "pageable" \
+        else (lambda a: torch.from_numpy(np.ascontiguousarray(a).copy()))
     n_sa = 48
     p = gen.make_sas(n_sa, cfg_id=60)
     bs = [gen.make_batch(5000, "imix", n_sa, cfg_id=60, batch=k, layout="packed") for k in range(5)]
@@ -227,20 +234,20 @@ def test_host_buffer_path_pipelined_and_mixed():
     hosts = []
     for k in (0, 1, 2):
         b = bs[k]
-        h = dict(i=pin(b.in_buf), o=pin(b.in_off.view(np.int32)), l=pin(b.in_len.view(np.int16)),
-                 s=pin(b.sa_idx.view(np.int32)), oo=pin(b.out_off.view(np.int32)),
+        h = dict(i=pin(b.in_buf), o=pin_meta(b.in_off.view(np.int32)), l=pin_meta(b.in_len.view(np.int16)),
+                 s=pin_meta(b.sa_idx.view(np.int32)), oo=pin_meta(b.out_off.view(np.int32)),
                  out=torch.zeros(b.out_pool_bytes, dtype=torch.uint8).pin_memory(),
-                 ol=torch.zeros(b.n, dtype=torch.int16).pin_memory())
+                 ol=pin_meta(np.zeros(b.n, dtype=np.int16)))
         hosts.append(h)
         t.process_host(h["i"], h["o"], h["l"], h["s"], h["out"], h["oo"], h["ol"],
                        int(b.in_off[-1]) + int(b.in_len[-1]), b.out_pool_bytes, n=b.n, stream=st)
     db = device.to_device(bs[3], "cuda")
     t.process(*db.args(), n=bs[3].n, stream=st)
     b = bs[4]
-    h = dict(i=pin(b.in_buf), o=pin(b.in_off.view(np.int32)), l=pin(b.in_len.view(np.int16)),
-             s=pin(b.sa_idx.view(np.int32)), oo=pin(b.out_off.view(np.int32)),
+    h = dict(i=pin(b.in_buf), o=pin_meta(b.in_off.view(np.int32)), l=pin_meta(b.in_len.view(np.int16)),
+             s=pin_meta(b.sa_idx.view(np.int32)), oo=pin_meta(b.out_off.view(np.int32)),
              out=torch.zeros(b.out_pool_bytes, dtype=torch.uint8).pin_memory(),
-             ol=torch.zeros(b.n, dtype=torch.int16).pin_memory())
+             ol=pin_meta(np.zeros(b.n, dtype=np.int16)))
     hosts.append(h)
     t.process_host(h["i"], h["o"], h["l"], h["s"], h["out"], h["oo"], h["ol"],
                    int(b.in_off[-1]) + int(b.in_len[-1]), b.out_pool_bytes, n=b.n, stream=st)

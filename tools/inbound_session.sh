@@ -1,6 +1,6 @@
 #!/bin/bash
 # inbound: GPU tests, ring forms side by side, phase trace of the pipelined ring
-TAG=${1:-r02ad}
+TAG=${1:-inb}
 mkdir -p gpurun_out
 python -m paper_conf_eurosys_kimjlmsm15_b200.build >/dev/null || exit 1
 timeout 900 python -m pytest tests -m gpu -x -q -k "inbound or replay" > gpurun_out/${TAG}_pytest_in.log 2>&1; tail -3 gpurun_out/${TAG}_pytest_in.log

@@ -1,6 +1,6 @@
 #!/bin/bash
 # GPU tests + the default bench line
-TAG=${1:-r02ar}
+TAG=${1:-tb}
 mkdir -p gpurun_out
 python -m paper_conf_eurosys_kimjlmsm15_b200.build >/dev/null || exit 1
 python -c "import oracle; oracle.build()"
