@@ -823,11 +823,14 @@ int nba_ipsec_process_batch_host(nba_ipsec_sa_table *t, const nba_ipsec_batch *b
     uint16_t *d_in_len = reinterpret_cast<uint16_t *>(d_out_off + t->max_batch);
     uint16_t *d_out_len = d_in_len + t->max_batch;
     // Per-packet metadata in page-locked host memory the device can address
-    // (cudaHostAlloc'd or registered) is read -- and out_len written -- by the
-    // kernels in place over PCIe, once per packet, so only the two large
-    // buffers go through the copy engines: the four small copies in and one
-    // out cost ~50 us per 65,536-packet step in copy-engine time
-    // (tools/pcie_probe.py).  Otherwise the metadata is staged like in_buf.
+    // (cudaHostAlloc'd or registered) does not go through the copy engines:
+    // the four small copies in and one out cost ~50 us per 65,536-packet step
+    // in copy-engine time (tools/pcie_probe.py).  The main kernels read the
+    // host arrays in place over PCIe and write out_len there.  Measured per
+    // 64 B step (profiles/ab/r02az_pcie.txt): in place 180.7 us, a pull
+    // kernel copying the four arrays into the staging slot first
+    // (NBA_IPSEC_HOST_META=pull) 192.7, copies (=stage) 199.3.  Pageable
+    // metadata is staged with copies like in_buf.
     auto mapped = [](const void *p) -> void * {
         cudaPointerAttributes a;
         if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
@@ -836,7 +839,9 @@ int nba_ipsec_process_batch_host(nba_ipsec_sa_table *t, const nba_ipsec_batch *b
         }
         return a.type == cudaMemoryTypeHost ? a.devicePointer : nullptr;
     };
-    bool zc = !std::getenv("NBA_IPSEC_HOST_STAGE_META");
+    const char *hm = std::getenv("NBA_IPSEC_HOST_META");
+    bool zc = !(hm && !std::strcmp(hm, "stage"));
+    const bool pull = hm && !std::strcmp(hm, "pull");
     void *z_in_off = nullptr, *z_sa = nullptr, *z_out_off = nullptr, *z_in_len = nullptr, *z_out_len = nullptr;
     if (zc) {
         z_in_off = mapped(b->in_off);
@@ -847,11 +852,13 @@ int nba_ipsec_process_batch_host(nba_ipsec_sa_table *t, const nba_ipsec_batch *b
         zc = z_in_off && z_sa && z_out_off && z_in_len && z_out_len;
     }
     if (zc) {
-        d_in_off = static_cast<uint32_t *>(z_in_off);
-        d_sa = static_cast<uint32_t *>(z_sa);
-        d_out_off = static_cast<uint32_t *>(z_out_off);
-        d_in_len = static_cast<uint16_t *>(z_in_len);
         d_out_len = static_cast<uint16_t *>(z_out_len);
+        if (!pull) {
+            d_in_off = static_cast<uint32_t *>(z_in_off);
+            d_sa = static_cast<uint32_t *>(z_sa);
+            d_out_off = static_cast<uint32_t *>(z_out_off);
+            d_in_len = static_cast<uint16_t *>(z_in_len);
+        }
     }
     cudaError_t e = cudaSuccess;
     auto chk = [&](cudaError_t x) {
@@ -872,6 +879,10 @@ int nba_ipsec_process_batch_host(nba_ipsec_sa_table *t, const nba_ipsec_batch *b
     chk(cudaEventRecord(t->ev_call, st));
     chk(cudaStreamWaitEvent(t->s_comp, t->ev_call, 0));
     chk(cudaStreamWaitEvent(t->s_comp, sl.in_ready, 0));
+    if (zc && pull)
+        chk(launch_pull_meta(static_cast<const uint32_t *>(z_in_off), static_cast<const uint32_t *>(z_sa),
+                             static_cast<const uint32_t *>(z_out_off), static_cast<const uint16_t *>(z_in_len),
+                             d_in_off, d_sa, d_out_off, d_in_len, n, t->num_sms, t->s_comp));
     if (e != cudaSuccess) return NBA_IPSEC_ECUDA;
     BatchArgs B{sl.in, d_in_off, d_in_len, d_sa, sl.out, d_out_off, d_out_len, n};
     int rc = enqueue(t, B, t->s_comp);
