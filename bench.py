@@ -64,6 +64,15 @@ def load_peaks():
         return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0, "source": "fallback (B200_PROFILING.md)"}
 
 
+def gpu_lead(torch, us: float = 100.0):
+    """A sleep kernel just before a timed region's start event: the GPU is busy
+    while the host enqueues the start event and the launches, so the events
+    measure device time, not the host's enqueue latency (the GIL, the NVML
+    sampler thread) -- with K = 20 ring batches (~0.5 ms) that jitter was
+    ~40 us per run (tools/ring_startup.py)."""
+    torch.cuda._sleep(int(us * 2000))       # cycles at <= 2 GHz: >= `us` microseconds
+
+
 class ClockSampler:
     """Samples SM clock + throttle reasons with NVML during the timed region."""
 
@@ -269,6 +278,7 @@ def measure_outbound(ctx, args, cfg_id, size, steps, warmup, full):
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(ctx.local) as clk:
         torch.cuda.synchronize()
+        gpu_lead(torch)
         e0.record()
         ring.run_batches(steps)            # ALL K timed batches: ONE persistent launch
         e1.record()
@@ -297,6 +307,7 @@ def measure_outbound(ctx, args, cfg_id, size, steps, warmup, full):
         for k in range(2 * R):
             runs[k % R]()
         torch.cuda.synchronize()
+        gpu_lead(torch)
         e0.record()
         for k in range(steps):
             runs[k % R]()
@@ -312,6 +323,7 @@ def measure_outbound(ctx, args, cfg_id, size, steps, warmup, full):
             del os.environ["NBA_IPSEC_RING_GRAPH"]
         g.run_batches(2 * R)
         torch.cuda.synchronize()
+        gpu_lead(torch)
         e0.record()
         g.run_batches(steps)
         e1.record()
@@ -395,6 +407,7 @@ def measure_inbound(ctx, args, cfg_id, steps, warmup, form=None):
     torch.cuda.synchronize()
     ctx.barrier()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    gpu_lead(torch)
     e0.record()
     timed_batches(steps)
     e1.record()
@@ -584,6 +597,7 @@ def run_e2e(ctx, args):
     ctx.barrier()
     steps = max(5, args.steps // 2)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    gpu_lead(torch, 50.0)
     e0.record()
     for _ in range(steps):
         step()
@@ -775,8 +789,10 @@ def run_ours(args):
                        "l2": f"inputs larger than L2: batches rotate over {head['R']} device copies "
                              "(> 2x L2 touched per rotation), SA table resident",
                        "timing": f"all {steps} timed batches in ONE nba_ipsec_ring_run_batches call "
-                                 f"({head['form']} persistent ring, 1 launch) between one CUDA event "
-                                 "pair, barrier + sync both sides, max over ranks"},
+                                 f"({head['form']} persistent ring, 1 launch, its start-up included) "
+                                 "between one CUDA event pair, barrier + sync both sides, max over "
+                                 "ranks; a sleep kernel ahead of the start event keeps host enqueue "
+                                 "latency out of the device time"},
             "roofline": roof_line,
             "gbps_by_size": {k: round(v["gbps"], 1) for k, v in by_size.items()},
             "us_by_size": {k: round(v["us"], 2) for k, v in by_size.items()},

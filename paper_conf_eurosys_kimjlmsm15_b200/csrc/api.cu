@@ -785,11 +785,19 @@ int nba_ipsec_reserve_host_io(nba_ipsec_sa_table *t, uint64_t in_buf_bytes, uint
     const uint64_t outb = std::max(out_buf_bytes, t->io_out_bytes);
     io_free(t);
     t->io_ready = false;
+    // (zeroed once: the lanes' 32-byte loads may cover up to 31 bytes past
+    // the copied input, and the copy-out takes the whole output range,
+    // including bytes between the slots the kernels never write)
     for (auto &sl : t->io) {
-        chk(cudaMalloc(&sl.in, inb + 16));
-        chk(cudaMalloc(&sl.out, outb + 16));
+        chk(cudaMalloc(&sl.in, inb + 64));
+        chk(cudaMalloc(&sl.out, outb + 64));
         chk(cudaMalloc(&sl.meta, (size_t)t->max_batch * 16 + 64));
+        if (e == cudaSuccess) {
+            chk(cudaMemset(sl.in, 0, inb + 64));
+            chk(cudaMemset(sl.out, 0, outb + 64));
+        }
     }
+    if (e == cudaSuccess) chk(cudaDeviceSynchronize());   // before the non-blocking streams' copies
     if (e != cudaSuccess) {
         cudaGetLastError();
         io_free(t);
@@ -827,10 +835,11 @@ int nba_ipsec_process_batch_host(nba_ipsec_sa_table *t, const nba_ipsec_batch *b
     // the four small copies in and one out cost ~50 us per 65,536-packet step
     // in copy-engine time (tools/pcie_probe.py).  The main kernels read the
     // host arrays in place over PCIe and write out_len there.  Measured per
-    // 64 B step (profiles/ab/r02az_pcie.txt): in place 180.7 us, a pull
-    // kernel copying the four arrays into the staging slot first
-    // (NBA_IPSEC_HOST_META=pull) 192.7, copies (=stage) 199.3.  Pageable
-    // metadata is staged with copies like in_buf.
+    // 64 B step (profiles/ab/r02az_pcie.txt): in place 180.7 us, copies
+    // (NBA_IPSEC_HOST_META=stage) 199.3; a pull kernel copying the four
+    // arrays into the staging slot first: 192.7 on the compute stream, 317 on
+    // the copy-in stream (it waits for the cooperative kernel's SMs).
+    // Pageable metadata is staged with copies like in_buf.
     auto mapped = [](const void *p) -> void * {
         cudaPointerAttributes a;
         if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
@@ -841,7 +850,6 @@ int nba_ipsec_process_batch_host(nba_ipsec_sa_table *t, const nba_ipsec_batch *b
     };
     const char *hm = std::getenv("NBA_IPSEC_HOST_META");
     bool zc = !(hm && !std::strcmp(hm, "stage"));
-    const bool pull = hm && !std::strcmp(hm, "pull");
     void *z_in_off = nullptr, *z_sa = nullptr, *z_out_off = nullptr, *z_in_len = nullptr, *z_out_len = nullptr;
     if (zc) {
         z_in_off = mapped(b->in_off);
@@ -852,13 +860,11 @@ int nba_ipsec_process_batch_host(nba_ipsec_sa_table *t, const nba_ipsec_batch *b
         zc = z_in_off && z_sa && z_out_off && z_in_len && z_out_len;
     }
     if (zc) {
+        d_in_off = static_cast<uint32_t *>(z_in_off);
+        d_sa = static_cast<uint32_t *>(z_sa);
+        d_out_off = static_cast<uint32_t *>(z_out_off);
+        d_in_len = static_cast<uint16_t *>(z_in_len);
         d_out_len = static_cast<uint16_t *>(z_out_len);
-        if (!pull) {
-            d_in_off = static_cast<uint32_t *>(z_in_off);
-            d_sa = static_cast<uint32_t *>(z_sa);
-            d_out_off = static_cast<uint32_t *>(z_out_off);
-            d_in_len = static_cast<uint16_t *>(z_in_len);
-        }
     }
     cudaError_t e = cudaSuccess;
     auto chk = [&](cudaError_t x) {
@@ -879,10 +885,6 @@ int nba_ipsec_process_batch_host(nba_ipsec_sa_table *t, const nba_ipsec_batch *b
     chk(cudaEventRecord(t->ev_call, st));
     chk(cudaStreamWaitEvent(t->s_comp, t->ev_call, 0));
     chk(cudaStreamWaitEvent(t->s_comp, sl.in_ready, 0));
-    if (zc && pull)
-        chk(launch_pull_meta(static_cast<const uint32_t *>(z_in_off), static_cast<const uint32_t *>(z_sa),
-                             static_cast<const uint32_t *>(z_out_off), static_cast<const uint16_t *>(z_in_len),
-                             d_in_off, d_sa, d_out_off, d_in_len, n, t->num_sms, t->s_comp));
     if (e != cudaSuccess) return NBA_IPSEC_ECUDA;
     BatchArgs B{sl.in, d_in_off, d_in_len, d_sa, sl.out, d_out_off, d_out_len, n};
     int rc = enqueue(t, B, t->s_comp);

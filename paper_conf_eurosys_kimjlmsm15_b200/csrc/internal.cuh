@@ -223,9 +223,6 @@ cudaError_t launch_in_fused_ring_pipe(const DevTable &T, const InState &S, const
                                       const RingRun &R, uint32_t hmask, const InPipeBufs &P, int grid,
                                       cudaStream_t st);
 bool in_pipe_ok(uint32_t n, int grid);
-cudaError_t launch_pull_meta(const uint32_t *h_in_off, const uint32_t *h_sa, const uint32_t *h_out_off,
-                             const uint16_t *h_in_len, uint32_t *in_off, uint32_t *sa, uint32_t *out_off,
-                             uint16_t *in_len, uint32_t n, int num_sms, cudaStream_t st);
 cudaError_t launch_in_replay(const DevTable &T, const InState &S, const InBatchArgs &B,
                              uint32_t n_tiles, uint32_t hmask, bool gridsync, cudaStream_t st);
 cudaError_t launch_in_decide(const DevTable &T, const InState &S, const InBatchArgs &B,

@@ -207,21 +207,18 @@ def test_concurrent_tables_on_two_streams():
         ts[k].close()
 
 
-@pytest.mark.parametrize("meta", ["pulled", "in_place", "staged", "pageable"])
+@pytest.mark.parametrize("meta", ["in_place", "staged", "pageable"])
 def test_host_buffer_path_pipelined_and_mixed(meta, monkeypatch):
     """nba_ipsec_process_batch_host (the e2e API): pinned host buffers, three
     batches in flight through the copy-in / kernels / copy-out pipeline, then a
     device-path batch and another host batch on the same table: outputs, lengths,
     counters and SA counters equal the oracle's sequential run.  The per-packet
-    arrays (pinned) read / written by the main kernels in place (default),
-    pulled by a kernel first, staged by copies (forced), or staged because they
-    are pageable."""
+    arrays (pinned) read / written by the kernels in place (default), staged
+    by copies (forced), or staged because they are pageable."""
     import torch
     from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
     if meta == "staged":
         monkeypatch.setenv("NBA_IPSEC_HOST_META", "stage")
-    if meta == "pulled":
-        monkeypatch.setenv("NBA_IPSEC_HOST_META", "pull")
     pin_meta = (lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()) if meta != "pageable" \
         else (lambda a: torch.from_numpy(np.ascontiguousarray(a).copy()))
     n_sa = 48
