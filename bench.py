@@ -615,8 +615,9 @@ def run_e2e(ctx, args):
             "mpps": tot["bytes_in"] * steps / (ms * 1e-3) / 1e6,
             "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
             "steps": steps, "ms_per_step": ms / steps,
-            "api": "nba_ipsec_process_batch_host (pinned H2D of packed datagrams + metadata, "
-                   "kernels, D2H of output pool + out_len every step, 2 staging slots pipelined)"}
+            "api": "nba_ipsec_process_batch_host (pinned host buffers: packed datagrams H2D by copy, "
+                   "per-packet metadata read and out_len written in place over PCIe by the kernels, "
+                   "output pool D2H by copy, every step; 2 staging slots pipelined)"}
 
 
 def cpu_model():
