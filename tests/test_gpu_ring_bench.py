@@ -10,7 +10,10 @@ the cursor, with and without per-batch timestamps.  The oracle runs the same
 batch sequence with carried SA state; each slot's WHOLE output pool must equal
 the oracle's output of the last batch that used that slot, and out_len, the
 final SA counters and the device counters must match.  The C5 sweep sizes
-(configs[4]: 128 / 256 / 512 / 1024 B) run the same way with R + 3 batches."""
+(configs[4]: 128 / 256 / 512 / 1024 B) run the same way with R + 3 batches.
+The bench's inbound protocol (R ESP batches through an inbound ring, windows
+reset per rotation) runs against the oracle's sequential receiver the same
+way, at 64 B (software-pipelined inbound ring) and IMIX (graph ring)."""
 import numpy as np
 import pytest
 
@@ -100,3 +103,73 @@ def test_sweep_sizes_process_batch(size):
     p, b = shard.rank_workload(5, N_PKTS, size, N_SA, 0, 1)
     batches = [b, gen.make_batch(N_PKTS, size, N_SA, cfg_id=5, batch=1), b]
     assert_same(gpu_run(p, batches), oracle_run(p, batches, n_threads=16))
+
+
+def _inbound_compare(ds, sts, last, tag):
+    from paper_conf_eurosys_kimjlmsm15_b200 import device
+    for s, (o_out, o_len, o_st, ib) in last.items():
+        g_out, g_len = device.fetch(ds[s])
+        assert np.array_equal(sts[s].cpu().numpy(), o_st), f"{tag} slot {s}: status differs"
+        assert np.array_equal(g_len, o_len), f"{tag} slot {s}: out_len differs"
+        mask = np.zeros(o_out.size, bool)
+        for i in np.nonzero(o_len)[0]:
+            a = int(ib.out_off[i])
+            mask[a:a + int(o_len[i])] = True
+        if not np.array_equal(g_out[:o_out.size][mask], o_out[mask]):
+            raise AssertionError(f"{tag} slot {s}: inner bytes differ")
+
+
+@pytest.mark.parametrize("cfg_id,size,form", [(2, 64, "pipelined"), (4, "imix", "graph")])
+def test_bench_inbound_ring_exact(cfg_id, size, form):
+    """bench.py's inbound protocol at full size against the oracle's sequential
+    receiver: R ESP batches from R consecutive outbound batches (the oracle's
+    output, with carried SA counters), an inbound ring over them in the form
+    the library picks by length (64 B: the software-pipelined ring; IMIX: the
+    graph ring); one rotation after reset_inbound (every packet accepted), then
+    three batches without a reset (every packet a replay).  Every slot's
+    statuses, out_len and the inner bytes of every accepted packet, the
+    windows and the counters equal the oracle's (RFC 4303 §3.4)."""
+    import torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    p, b = shard.rank_workload(cfg_id, N_PKTS, size, N_SA, 0, 1)
+    R = device.ring_slot_count(b.in_len, b.n, int(torch.cuda.get_device_properties(0).L2_cache_size))
+    sas = oracle.make_sas(p)
+    esp = []
+    for _ in range(R):
+        out, ol, _ = oracle.process_batch(sas, N_SA, b, n_threads=16)
+        esp.append(gen.Batch(n=b.n, in_buf=out, in_off=b.out_off.copy(), in_len=ol.copy(),
+                             sa_idx=b.sa_idx.copy(), out_off=b.out_off.copy(),
+                             out_pool_bytes=b.out_pool_bytes, frame_len=b.frame_len))
+    sas_in = oracle.make_sas(p)
+    ctr = oracle.InCounters()
+    with nba_ipsec.SATable(p, device=0, max_batch=N_PKTS) as t:
+        t.enable_inbound()
+        ds = [device.to_device(e, "cuda", out_fill=0xA5) for e in esp]
+        sts = [torch.full((b.n,), 0xff, dtype=torch.uint8, device="cuda") for _ in esp]
+        ring = t.ring_inbound([(*d.args(), st, e.n) for d, st, e in zip(ds, sts, esp)])
+        assert ring.form == {"graph": ring.GRAPH, "pipelined": ring.PIPELINED}[form]
+        # a rotation from fresh windows
+        t.reset_inbound()
+        ring.run_batches(R)
+        win = oracle.make_windows(oracle.make_sas(p), N_SA)
+        last = {}
+        for k in range(R):
+            o_out, o_len, o_st, _ = oracle.process_inbound(sas_in, win, N_SA, esp[k], counters=ctr)
+            assert np.all(o_st == 0)
+            last[k] = (o_out, o_len.copy(), o_st.copy(), esp[k])
+        torch.cuda.synchronize()
+        _inbound_compare(ds, sts, last, "rotation")
+        # three more batches, no reset: replays
+        ring.run_batches(3)
+        last = {}
+        for k in range(3):
+            o_out, o_len, o_st, _ = oracle.process_inbound(sas_in, win, N_SA, esp[k], counters=ctr)
+            assert np.all(o_st == 3)
+            last[k] = (o_out, o_len.copy(), o_st.copy(), esp[k])
+        torch.cuda.synchronize()
+        _inbound_compare(ds, sts, last, "replays")
+        top, bmp = t.replay_window()
+        o_top, o_bmp = oracle.window_state(win, N_SA)
+        assert np.array_equal(top, o_top) and np.array_equal(bmp, o_bmp)
+        assert t.in_counters() == ctr.as_dict()
+        ring.close()
