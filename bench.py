@@ -229,26 +229,39 @@ class Ctx:
             raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={self.world}: launch one "
                              f"process per GPU (bench.py re-launches itself under torchrun when "
                              f"WORLD_SIZE is unset)")
+        # BENCH_SHARE_GPU=1 (a plumbing check, not a measurement): every rank on
+        # cuda:0 and gloo for the reductions, so the multi-rank flow (shards,
+        # per-rank rings, barriers, max / sum over ranks) runs on a one-GPU box
+        self.share = os.environ.get("BENCH_SHARE_GPU") == "1" and self.world > 1
+        if self.share:
+            self.local = 0
         torch.cuda.set_device(self.local)
         self.dev = torch.device("cuda", self.local)
+        self.red_dev = torch.device("cpu") if self.share else self.dev
         if self.world > 1:
-            dist.init_process_group("nccl", device_id=self.dev)
+            if self.share:
+                dist.init_process_group("gloo")
+            else:
+                dist.init_process_group("nccl", device_id=self.dev)
         self.peaks = load_peaks()
         self.l2 = int(getattr(torch.cuda.get_device_properties(self.dev), "L2_cache_size", 126 << 20))
         self.flush_buf = torch.empty(256 << 20, dtype=torch.uint8, device=self.dev)
 
     def barrier(self):
         if self.world > 1:
-            self.dist.barrier(device_ids=[self.local])
+            if self.share:
+                self.dist.barrier()
+            else:
+                self.dist.barrier(device_ids=[self.local])
 
     def flush(self):
         self.flush_buf.zero_()
 
     def max_ms(self, ms):
-        return shard.max_over_ranks(ms, device=self.dev)
+        return shard.max_over_ranks(ms, device=self.red_dev)
 
     def sum_all(self, d):
-        return shard.reduce_counters(d, device=self.dev)
+        return shard.reduce_counters(d, device=self.red_dev)
 
 
 def measure_outbound(ctx, args, cfg_id, size, steps, warmup, full):
@@ -786,7 +799,10 @@ def run_ours(args):
             "config": {"workload": f"configs[{main_cfg - 1}]: {nm}", "frame_bytes": CFG_SIZE[main_cfg],
                        "packets_per_gpu": PKTS_PER_GPU, "n_sa_total": N_SA_TOTAL,
                        "global_batch": PKTS_PER_GPU * ctx.world,
-                       "parallelism": f"sa-hash shard x{ctx.world} (no data-path collective)",
+                       "parallelism": f"sa-hash shard x{ctx.world} (no data-path collective)"
+                                      + (" -- BENCH_SHARE_GPU: every rank on cuda:0 with gloo "
+                                         "reductions, a plumbing check, not a measurement"
+                                         if ctx.share else ""),
                        "l2": f"inputs larger than L2: batches rotate over {head['R']} device copies "
                              "(> 2x L2 touched per rotation), SA table resident",
                        "timing": f"all {steps} timed batches in ONE nba_ipsec_ring_run_batches call "
@@ -890,7 +906,7 @@ def relaunch_under_torchrun(args):
         have = torch.cuda.device_count()
     except Exception:
         have = 0
-    if have < args.gpus:
+    if have < args.gpus and os.environ.get("BENCH_SHARE_GPU") != "1":
         raise SystemExit(f"bench.py: --gpus {args.gpus} requested but {have} CUDA device(s) visible")
     with socket.socket() as s:
         s.bind(("127.0.0.1", 0))
