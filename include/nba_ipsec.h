@@ -195,10 +195,14 @@ int nba_ipsec_ring_cursor(const nba_ipsec_ring *r);          /* slot of the next
  * ns).  dev_ts == NULL switches it off.  NBA_IPSEC_EINVAL for a graph ring or
  * cap < 2. */
 int nba_ipsec_ring_set_timestamps(nba_ipsec_ring *r, unsigned long long *dev_ts, uint32_t cap);
-enum { NBA_IPSEC_RING_GRAPH = 0, NBA_IPSEC_RING_PERSISTENT = 1, NBA_IPSEC_RING_PIPELINED = 2 };
+enum { NBA_IPSEC_RING_GRAPH = 0, NBA_IPSEC_RING_PERSISTENT = 1, NBA_IPSEC_RING_PIPELINED = 2,
+       NBA_IPSEC_RING_FREE = 3 };
 /* The form a run takes (NBA_IPSEC_RING_*); set_form switches a persistent ring
- * between PERSISTENT and PIPELINED (NBA_IPSEC_EINVAL for graph rings or slots
- * the pipelined form does not fit).  Both give identical results. */
+ * between PERSISTENT, PIPELINED and FREE -- the pipelined form without the
+ * end-of-batch CTA barrier: a lane warp that finished its run starts the next
+ * batch while longer runs go on (mixed-length batches) -- (NBA_IPSEC_EINVAL
+ * for graph rings or slots the pipelined forms do not fit).  All give
+ * identical results. */
 int nba_ipsec_ring_form(const nba_ipsec_ring *r);
 int nba_ipsec_ring_set_form(nba_ipsec_ring *r, int form);
 int nba_ipsec_ring_destroy(nba_ipsec_ring *r);   /* NULL -> OK */

@@ -407,6 +407,7 @@ struct nba_ipsec_ring {
     InPipeBufs in_bufs = {};             // pipelined inbound form (hk1 / hv1 = hkey_b / hval_b)
     uint32_t in_hmask = 0;
     bool pipe = false;                   // software-pipelined form (k_fused_ring_pipe)
+    bool free_run = false;               //   its free-running-lanes variant (k_fused_ring_free)
     bool in_pipe = false;                // inbound: software-pipelined form (k_in_fused_ring_pipe)
     bool pipe_ok = false;                // every slot fits the pipelined form
     uint64_t flow_gen = 0;               // the table's flow-table generation when recorded
@@ -451,6 +452,7 @@ int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, u
         for (uint32_t i = 0; i < n_slots && r->pipe_ok; i++)
             r->pipe_ok = slots[i].sa_idx && fused_pipe_ok(slots[i].n_pkts, t->grid_fused);
         r->pipe = r->pipe_ok && !std::getenv("NBA_IPSEC_RING_NOPIPE");
+        r->free_run = r->pipe && std::getenv("NBA_IPSEC_RING_FREE");
         std::vector<BatchArgs> hb(n_slots);
         for (uint32_t i = 0; i < n_slots; i++) {
             const nba_ipsec_batch &b = slots[i];
@@ -636,10 +638,10 @@ static int ring_launch(nba_ipsec_ring *r, uint32_t first, uint32_t n_batches, cu
                    ? NBA_IPSEC_OK
                    : NBA_IPSEC_ECUDA;
     if (r->d_slots) {
-        const cudaError_t e = r->pipe ? launch_fused_ring_pipe(t->T, t->W, r->d_slots, R, r->hist_b,
-                                                               t->grid_fused, st)
-                                      : launch_fused_ring(t->T, t->W, r->d_slots, R, r->hist_b,
-                                                          t->grid_fused, st);
+        const cudaError_t e =
+            r->free_run ? launch_fused_ring_free(t->T, t->W, r->d_slots, R, r->hist_b, t->grid_fused, st)
+            : r->pipe   ? launch_fused_ring_pipe(t->T, t->W, r->d_slots, R, r->hist_b, t->grid_fused, st)
+                        : launch_fused_ring(t->T, t->W, r->d_slots, R, r->hist_b, t->grid_fused, st);
         return e == cudaSuccess ? NBA_IPSEC_OK : NBA_IPSEC_ECUDA;
     }
     uint32_t k = first, left = n_batches;
@@ -700,11 +702,12 @@ int nba_ipsec_ring_set_form(nba_ipsec_ring *r, int form)
 {
     if (!r || !r->d_slots) return NBA_IPSEC_EINVAL;   // graph rings have one form
     if (form == NBA_IPSEC_RING_PERSISTENT) {
-        r->pipe = false;
+        r->pipe = r->free_run = false;
         return NBA_IPSEC_OK;
     }
-    if (form == NBA_IPSEC_RING_PIPELINED && r->pipe_ok) {
+    if ((form == NBA_IPSEC_RING_PIPELINED || form == NBA_IPSEC_RING_FREE) && r->pipe_ok) {
         r->pipe = true;
+        r->free_run = form == NBA_IPSEC_RING_FREE;
         return NBA_IPSEC_OK;
     }
     return NBA_IPSEC_EINVAL;
@@ -714,8 +717,10 @@ int nba_ipsec_ring_form(const nba_ipsec_ring *r)
 {
     if (!r) return NBA_IPSEC_EINVAL;
     if (r->d_in_slots) return r->in_pipe ? NBA_IPSEC_RING_PIPELINED : NBA_IPSEC_RING_PERSISTENT;
-    return !r->d_slots ? NBA_IPSEC_RING_GRAPH : r->pipe ? NBA_IPSEC_RING_PIPELINED
-                                                         : NBA_IPSEC_RING_PERSISTENT;
+    return !r->d_slots ? NBA_IPSEC_RING_GRAPH
+           : r->free_run ? NBA_IPSEC_RING_FREE
+           : r->pipe    ? NBA_IPSEC_RING_PIPELINED
+                        : NBA_IPSEC_RING_PERSISTENT;
 }
 
 int nba_ipsec_ring_destroy(nba_ipsec_ring *r)

@@ -47,6 +47,9 @@ struct FusedLo {
     uint32_t pro_delay;            //   the prologue warps' start delay for the next batch (ns)
     uint32_t stag_ns;              // pipelined ring: start delay of the upper lane warps
     uint32_t stag_acc;             //   (AES step 0 of the lower ones, measured per batch)
+    uint32_t fr_ready;             // free-running ring: batches prepared (side -> lanes)
+    uint32_t fr_taken;             //   lane warps' field takes so far (lanes -> side)
+    uint32_t fr_load[16];          //   each lane warp's cumulative assigned cost
 };
 
 struct FusedHi {

@@ -206,6 +206,8 @@ struct RingRun {
 };
 cudaError_t launch_fused_ring_pipe(const DevTable &T, const DevWork &W, const BatchArgs *slots,
                                    const RingRun &R, uint16_t *hist_b, int grid, cudaStream_t st);
+cudaError_t launch_fused_ring_free(const DevTable &T, const DevWork &W, const BatchArgs *slots,
+                                   const RingRun &R, uint16_t *hist_b, int grid, cudaStream_t st);
 bool fused_pipe_ok(uint32_t n, int grid);
 cudaError_t launch_fused_ring(const DevTable &T, const DevWork &W, const BatchArgs *slots,
                               const RingRun &R, uint16_t *hist_b, int grid, cudaStream_t st);

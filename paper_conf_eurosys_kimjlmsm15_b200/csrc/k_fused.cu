@@ -1546,6 +1546,305 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
     }
 }
 
+// ----------------------------------------------- free-running lane warps
+// k_fused_ring_free: the pipelined ring without the end-of-batch CTA barrier,
+// for batches of mixed lengths, where one warp's run of long packets sets
+// the batch time while the others wait (profiles/r02be_imix_balance.md).
+// The two side warps run, per batch j: wait until every lane warp took its
+// fields of batch j - 1 (smem counter fr_taken), the prologue of batch j
+// (metadata, ranks, counts, arrival at its grid barrier), the run placement
+// (the batch's runs, longest first, onto the lane warps with the least
+// cumulative assigned cost: a long run goes to a warp that will be free
+// early), the grid barrier, this CTA's share of the row scans and the polls
+// of its packets' bases (the sequence numbers), then publish batch j (smem
+// flag fr_ready).  A lane warp, per batch: wait for fr_ready, take its run's
+// fields, count itself in fr_taken, encrypt its packets -- so a warp that
+// finished a short run starts the next batch while a long run is still
+// going.  Same results as k_fused_ring_pipe (the sequence numbers are the
+// per-SA order of the batch, not the order of completion).
+// Measured (profiles/ab/r02bh_forms.txt, the trace in DESIGN.md §9): SLOWER
+// than k_fused_ring_pipe at every size (64 B 42.1 vs 22.2 us, IMIX 169 vs 88):
+// the side warps' chain per batch (prologue ~32 us under the lanes' load,
+// grid barrier behind the slowest CTA, row scans and polls by two warps
+// ~12 us) becomes the period.  Opt-in only (nba_ipsec_ring_set_form FREE).
+constexpr uint32_t FR_SPIN_MAX = 1u << 26;    // bounded waits: a kernel error, never a hang
+
+__device__ __forceinline__ void fr_wait_ge(const uint32_t *p, uint32_t v)
+{
+    for (uint32_t k = 0; *reinterpret_cast<const volatile uint32_t *>(p) < v; k++) {
+        if (k > FR_SPIN_MAX) __trap();
+        __nanosleep(64);
+    }
+    __threadfence_block();
+}
+
+// The batch's grid barrier wait, this CTA's share of the row scans, and the
+// polls of its packets' published bases, by the 64 side threads: L.seq[j]
+// turns from the CTA rank into the ESP sequence number (0: dropped).
+__device__ __forceinline__ void fr_side_sequence(const DevTable &T, const DevWork &W, uint32_t cnt,
+                                                 uint32_t bar_target, uint32_t epoch, FusedLo &L,
+                                                 uint32_t pt)
+{
+    const uint32_t G = gridDim.x, cta = blockIdx.x, lane = pt & 31u, pw = pt >> 5;
+    if (pt == 0) {
+        uint32_t v;
+        for (uint32_t k = 0;; k++) {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(&W.ctl[CTL_BAR_MONO]) : "memory");
+            if ((int)(v - bar_target) >= 0) break;
+            if (k > FR_SPIN_MAX) __trap();
+            __nanosleep(64);
+        }
+    }
+    bar_sync_n(1, PIPE_P);
+    pipe_scan_rows(T, W, cta * 2u + pw, G * 2u, G, lane, epoch);
+    unsigned long long v[PR];
+    uint32_t sa_r[PR];
+#pragma unroll
+    for (uint32_t r = 0; r < PR; r++) {
+        const uint32_t j = r * PIPE_P + pt;
+        const bool ok = j < cnt && (L.info[j] & INFO_OK);
+        sa_r[r] = ok ? L.sa[j] : INVALID_SA;
+        v[r] = ok ? ld_relaxed_u64(&W.hbase[(size_t)sa_r[r] * G + cta]) : 0ull;
+    }
+#pragma unroll
+    for (uint32_t r = 0; r < PR; r++) {
+        const uint32_t j = r * PIPE_P + pt;
+        if (j >= cnt) continue;
+        uint32_t q32 = 0;
+        if (sa_r[r] != INVALID_SA) {
+            const unsigned long long *pb = &W.hbase[(size_t)sa_r[r] * G + cta];
+            for (uint32_t k = 0; (uint32_t)(v[r] >> 33) != epoch; k++) {
+                if (k > FR_SPIN_MAX) __trap();
+                v[r] = ld_relaxed_u64(pb);
+            }
+            const unsigned long long q = (v[r] & ((1ull << 33) - 1ull)) + 1ull + L.seq[j];
+            q32 = q <= 0xffffffffull ? (uint32_t)q : 0u;   // RFC 4303 §3.3.3: never cycle
+        }
+        L.seq[j] = q32;
+    }
+    bar_sync_n(1, PIPE_P);
+}
+
+// Run placement by cumulative cost (side warp 0): the lane warp with the
+// k-th smallest cumulative cost takes the run with the k-th largest cost
+// (run r = sorted positions 32 r ..; cost as the LPT placement's).
+__device__ __forceinline__ void fr_place(FusedLo &L, uint32_t cnt, uint32_t lane)
+{
+    const uint32_t nruns = (cnt + 31u) / 32u;
+    uint32_t cost = 0;
+    if (lane < nruns) {
+        const uint32_t info = L.info[L.perm[32u * lane]];
+        const uint32_t C = esp_C(info & 0x7ffu);
+        cost = (info & INFO_OK) ? 8u * (esp_nsha_inner(C) + 1u) + 3u * ((C + 15u) >> 4) : 1u;
+    }
+    uint32_t crank = 0;                            // runs costlier than this one (ties by index)
+#pragma unroll
+    for (uint32_t o = 0; o < PIPE_LANE_WARPS; o++) {
+        const uint32_t co = __shfl_sync(0xffffffffu, cost, o);
+        crank += (o < nruns && (co > cost || (co == cost && o < lane))) ? 1u : 0u;
+    }
+    const uint32_t w = lane;                       // lane w speaks for lane warp w
+    const uint32_t ld = w < PIPE_LANE_WARPS ? L.fr_load[w] : 0xffffffffu;
+    uint32_t rank = 0;                             // among the 14 warps, ties by index
+#pragma unroll
+    for (uint32_t o = 0; o < PIPE_LANE_WARPS; o++) {
+        const uint32_t lo = __shfl_sync(0xffffffffu, ld, o);
+        rank += (lo < ld || (lo == ld && o < w)) ? 1u : 0u;
+    }
+    uint32_t run = 0xffu, c_r = 0;                 // the run of cost rank `rank`
+#pragma unroll
+    for (uint32_t o = 0; o < PIPE_LANE_WARPS; o++) {
+        const uint32_t cr = __shfl_sync(0xffffffffu, crank, o);
+        const uint32_t co = __shfl_sync(0xffffffffu, cost, o);
+        if (o < nruns && cr == rank) {
+            run = o;
+            c_r = co;
+        }
+    }
+    if (w < PIPE_LANE_WARPS) {
+        L.wrun[w] = (uint8_t)run;
+        L.fr_load[w] = ld + c_r;
+    }
+    // keep the loads small: subtract the minimum
+    const uint32_t nl = w < PIPE_LANE_WARPS ? L.fr_load[w] : 0xffffffffu;
+    const uint32_t mn = __reduce_min_sync(0xffffffffu, nl);
+    if (w < PIPE_LANE_WARPS) L.fr_load[w] = nl - mn;
+}
+
+__global__ void __launch_bounds__(F_THREADS, 1)
+k_fused_ring_free(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint16_t *hist_b)
+{
+    const uint32_t n_slots = R.n_slots, n_batches = R.n_batches, first = R.first;
+    extern __shared__ __align__(16) uint8_t smem[];
+    const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
+    const uint32_t G = gridDim.x, cta = blockIdx.x;
+    if (n_batches == 0) return;
+    if (!NBA_RING_TRACE && R.ts && cta == 0 && tid == 0) R.ts[0] = gtimer();
+    const uint32_t base0 = *reinterpret_cast<volatile uint32_t *>(&W.ctl[CTL_BAR_BASE]);
+    const uint32_t ep0 = *reinterpret_cast<volatile uint32_t *>(&W.ctl[CTL_EPOCH]);
+    const uint32_t sb = smem_u32(smem);
+    const uint32_t toff = (0x10000u - (sb & 0xffffu)) & 0xffffu;
+    uint32_t lo_off = 0;
+    if (toff < sizeof(FusedLo)) {
+        if (toff + AES_TABLE_BYTES + sizeof(FusedHi) + sizeof(FusedLo) > F_SMEM) __trap();
+        lo_off = toff + AES_TABLE_BYTES + (uint32_t)sizeof(FusedHi);
+    }
+    uint8_t *tabs = smem + toff;
+    FusedLo &L = *reinterpret_cast<FusedLo *>(smem + lo_off);
+    FusedHi &H = *reinterpret_cast<FusedHi *>(smem + toff + AES_TABLE_BYTES);
+    const uint32_t lane4r = (lane * 4u) | (smem_u32(tabs) & 0xffff0000u);
+    tables_stage(tabs, T, &L.tbar, true);   // bulk copy, waited for before the first lookup
+    if (tid < NBINS) L.bins[tid] = 0u;
+    if (tid < 16) L.fr_load[tid] = 0u;
+    if (tid == 0) {
+        L.fr_ready = 0u;
+        L.fr_taken = 0u;
+    }
+    for (uint32_t k = tid; k < 2u * F_SUPER; k += F_THREADS) {
+        L.hkey[k] = INVALID_SA;
+        L.hmask[k] = 0u;
+        (&L.aux0[0])[k] = 0u;                     // the prologue's second count array
+    }
+    __syncthreads();
+    auto epoch_of = [&](uint32_t bi) { return ((ep0 + bi) % 0x7fffffffu) + 1u; };
+    auto work_of = [&](uint32_t bi) {
+        DevWork Wb = W;
+        if (bi & 1u) Wb.hist16 = hist_b;
+        return Wb;
+    };
+    unsigned long long c_ok = 0, c_drop = 0, c_in = 0, c_out = 0;
+    if (tid >= PIPE_MAX_PPC) {
+        // ---- side warps: prepare every batch of the run in order
+        const uint32_t pt = tid - PIPE_MAX_PPC;
+        for (uint32_t bi = 0; bi < n_batches; bi++) {
+            const BatchArgs B = slots[(first + bi) % n_slots];
+            const uint32_t ppc = fused_ppc(B.n, G);
+            const uint32_t p_begin = cta * ppc;
+            const uint32_t p_end = min(B.n, p_begin + ppc);
+            const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
+            if (bi > 0) {                          // the arrays are free: batch bi - 1 taken
+                if (pt == 0) fr_wait_ge(&L.fr_taken, PIPE_LANE_WARPS * bi);
+                bar_sync_n(1, PIPE_P);
+            }
+#if NBA_RING_TRACE
+            if (pt == 0 && R.ts) *RTR(bi, 0) = gtimer();
+#endif
+            PipeMeta meta;
+            pipe_load_meta(B, ppc, pt, meta);
+            if (bi + 1 < n_batches) {
+                const BatchArgs B1 = slots[(first + bi + 1) % n_slots];
+                pipe_prefetch_meta(B1, fused_ppc(B1.n, G), pt);
+            }
+            pipe_prologue(T, work_of(bi), B, ppc, base0 + (bi + 1) * G, epoch_of(bi), L, pt, bi & 1u, meta);
+            if (pt < 32u) fr_place(L, cnt, pt);
+#if NBA_RING_TRACE
+            if (pt == 0 && R.ts) *RTR(bi, 1) = gtimer();
+#endif
+            fr_side_sequence(T, work_of(bi), cnt, base0 + (bi + 1) * G, epoch_of(bi), L, pt);
+            if (pt == 0) {
+                __threadfence_block();
+                *reinterpret_cast<volatile uint32_t *>(&L.fr_ready) = bi + 1u;
+            }
+#if NBA_RING_TRACE
+            if (pt == 0 && R.ts) *RTR(bi, 2) = gtimer();
+#endif
+        }
+    } else {
+        // ---- lane warps: each batch as soon as it is prepared
+        tables_bulk_wait(&L.tbar, 0u);
+        for (uint32_t bi = 0; bi < n_batches; bi++) {
+            const BatchArgs B = slots[(first + bi) % n_slots];
+            const uint32_t ppc = fused_ppc(B.n, G);
+            const uint32_t p_begin = cta * ppc;
+            const uint32_t p_end = min(B.n, p_begin + ppc);
+            const uint32_t cnt = p_end > p_begin ? p_end - p_begin : 0u;
+#if NBA_RING_TRACE
+            const unsigned long long t_w = gtimer();
+#endif
+            if (lane == 0) fr_wait_ge(&L.fr_ready, bi + 1u);
+            __syncwarp();
+            __threadfence_block();
+#if NBA_RING_TRACE
+            if (lane == 0 && R.ts) {
+                atomicMax(RTR(bi, 3), gtimer());          // the latest take
+                atomicMax(RTR(bi, 6), gtimer() - t_w);    // the longest wait for the batch
+            }
+#endif
+            const uint32_t run = L.wrun[warp];
+            const uint32_t pos = 32u * run + lane;
+            const bool have = run != 0xffu && pos < cnt;
+            const uint32_t pk = have ? L.perm[pos] : 0u;
+            const uint32_t info = have ? L.info[pk] : 0u;
+            const uint32_t sa = (info & INFO_OK) ? L.sa[pk] : INVALID_SA;
+            const uint32_t inoff = have ? L.inoff[pk] : 0u;
+            const uint32_t outoff = have ? L.outoff[pk] : 0u;
+            const uint32_t q32 = have ? L.seq[pk] : 0u;
+            __syncwarp();
+            if (lane == 0) {                       // fields taken: the side may reuse the arrays
+                __threadfence_block();
+                atomicAdd(&L.fr_taken, 1u);
+            }
+            if (have) {
+                const uint32_t pkt = p_begin + pk;
+                if ((info & INFO_OK) && q32 != 0u) {
+                    PktPre pp = load_pkt_pre(T, B.in_buf, sa, inoff, true, 0u);
+                    expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
+                    esp_packet(T, B, L, H, lane4r, tid, sa, info, q32, inoff, outoff, pp, nullptr);
+                    const uint32_t Dp = info & 0x7ffu;
+                    const uint32_t Lp = 48u + esp_C(Dp);
+                    B.out_len[pkt] = (uint16_t)Lp;
+                    c_ok++;
+                    c_in += Dp;
+                    c_out += Lp;
+                } else {
+                    B.out_len[pkt] = 0;
+                    c_drop++;
+                }
+            }
+#if NBA_RING_TRACE
+            if (R.ts && lane == 0) atomicMax(RTR(bi, 4), gtimer());   // the latest lane finish
+#else
+            if (R.ts && lane == 0) atomicMax(&R.ts[1u + bi], gtimer());
+#endif
+        }
+    }
+    // counters (as fused_body), device state for the next launch
+    __syncthreads();
+    if (tid < 4) L.cnt[tid] = 0ull;
+    __syncthreads();
+    const unsigned long long s0 = warp_sum_u64(c_ok), s1 = warp_sum_u64(c_drop);
+    const unsigned long long s2 = warp_sum_u64(c_in), s3 = warp_sum_u64(c_out);
+    if (lane == 0) {
+        if (s0) atomicAdd(&L.cnt[0], s0);
+        if (s1) atomicAdd(&L.cnt[1], s1);
+        if (s2) atomicAdd(&L.cnt[2], s2);
+        if (s3) atomicAdd(&L.cnt[3], s3);
+    }
+    __syncthreads();
+    if (tid < 4 && L.cnt[tid]) atomicAdd(&W.counters[tid], L.cnt[tid]);
+    if (tid == 4 && cta == 0) {
+        atomicAdd(&W.counters[4], (unsigned long long)n_batches);
+        W.ctl[CTL_BAR_BASE] = base0 + n_batches * G;   // one barrier per batch
+        W.ctl[CTL_EPOCH] = epoch_of(n_batches - 1u);      // the last batch's epoch
+    }
+}
+
+cudaError_t launch_fused_ring_free(const DevTable &T, const DevWork &W, const BatchArgs *slots,
+                                   const RingRun &R, uint16_t *hist_b, int grid, cudaStream_t st)
+{
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(F_THREADS);
+    cfg.dynamicSmemBytes = F_SMEM;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeCooperative;   // grid barriers inside
+    attr[0].val.cooperative = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, k_fused_ring_free, T, W, slots, R, hist_b);
+}
+
 cudaError_t launch_fused_ring_pipe(const DevTable &T, const DevWork &W, const BatchArgs *slots,
                                    const RingRun &R, uint16_t *hist_b, int grid, cudaStream_t st)
 {
@@ -1630,6 +1929,9 @@ cudaError_t setup_fused_attributes()
                                           (int)F_SMEM);
     if (e0 != cudaSuccess) return e0;
     e0 = cudaFuncSetAttribute(k_fused_ring_pipe, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              (int)F_SMEM);
+    if (e0 != cudaSuccess) return e0;
+    e0 = cudaFuncSetAttribute(k_fused_ring_free, cudaFuncAttributeMaxDynamicSharedMemorySize,
                               (int)F_SMEM);
     if (e0 != cudaSuccess) return e0;
     cudaError_t e = cudaFuncSetAttribute(k_fused<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,

@@ -90,6 +90,19 @@ def test_sweep_sizes_ring(size):
     _ring_vs_oracle(size, 5, [R + 3])
 
 
+@pytest.mark.parametrize("cfg_id,size", [(2, 64), (3, 1514), (4, "imix")])
+def test_bench_ring_free_form(cfg_id, size):
+    """The free-running-lanes form (k_fused_ring_free, set_form) over the same
+    full-size ring: two rotations and a partial one, then a run continuing
+    mid-rotation, against the oracle."""
+    import torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    p, b = shard.rank_workload(cfg_id, N_PKTS, size, N_SA, 0, 1)
+    R = device.ring_slot_count(b.in_len, b.n, int(torch.cuda.get_device_properties(0).L2_cache_size))
+    _ring_vs_oracle(size, cfg_id, [2 * R + 5, max(1, R - 2)], timestamps=(cfg_id == 4),
+                    form=nba_ipsec.Ring.FREE)
+
+
 def test_bench_ring_plain_persistent_form():
     """The plain persistent form (set_form) over the same full-size 64-B ring."""
     from paper_conf_eurosys_kimjlmsm15_b200 import nba_ipsec
