@@ -512,6 +512,9 @@ k_in_fused_ring(DevTable T, InState S, const InBatchArgs *slots, RingRun R, uint
 #ifndef NBA_IN_PREFETCH       // pipelined inbound ring: L2 prefetches of the next batch's headers
 #define NBA_IN_PREFETCH 0     //   and the one after's metadata, ahead of the side warps' prologue
 #endif
+#ifndef NBA_IN_LANE_ROWS      // pipelined inbound ring: the previous batch's row scans by the
+#define NBA_IN_LANE_ROWS 0    //   lane warps at the start of the iteration (1) or the side warps (0)
+#endif
 #ifndef NBA_IN_PRO_FIRST      // pipelined inbound ring: the side warps run the next batch's
 #define NBA_IN_PRO_FIRST 0    //   prologue before (1) or after (0) the previous batch's row scans
 #endif
@@ -825,6 +828,38 @@ __device__ __forceinline__ void in_pipe_rows(const DevTable &T, const InState &S
         }
 }
 
+// The same by the 14 lane warps (NBA_IN_LANE_ROWS), at the start of batch
+// k + 1's iteration once they took their fields: wait for SB1 (one thread,
+// then named barrier 3 over the 448 lane threads), one SA row per warp at
+// most (SA s on CTA s mod G, warp s / G), batch k + 3's hash slice cleared,
+// arrival at SB2 once every lane warp's stores are ordered.
+__device__ __forceinline__ void in_pipe_rows_lanes(const DevTable &T, const InState &S, uint32_t hmask,
+                                                   uint32_t sb1, unsigned long long *clr_k, uint32_t *clr_v,
+                                                   unsigned long long *tr)
+{
+    const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
+    const uint32_t G = gridDim.x, cta = blockIdx.x;
+    if (tid == 0) {
+        uint32_t v;
+        do {
+            asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(&S.ctl[CTLI_BAR]) : "memory");
+        } while ((int)(v - sb1) < 0);
+        if (tr) tr[1] = gtimer();
+    }
+    bar_sync_n(3, PIPE_MAX_PPC);
+    scan_rows_batched(S, warp * G + cta, PIPE_LANE_WARPS * G, T.n_sa, G, lane);
+    if (clr_k)
+        for (uint32_t k = cta * PIPE_MAX_PPC + tid; k <= hmask; k += G * PIPE_MAX_PPC) {
+            clr_k[k] = ~0ull;
+            clr_v[k] = ~0u;
+        }
+    bar_sync_n(3, PIPE_MAX_PPC);                 // (orders every lane warp's stores before the arrival)
+    if (tid == 0) {
+        asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(&S.ctl[CTLI_BAR2]) : "memory");
+        if (tr) tr[8] = gtimer();
+    }
+}
+
 // Part 2, by one warp for packets j = 32 w + lane of the CTA's batch-k range
 // (w: the warp's slot, 0..13 -- the lane warps once their own packets are
 // done): wait for SB2 (every row scanned, sb2), then the decisions:
@@ -978,6 +1013,8 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
             uint32_t iv0 = have ? L.aux0[pk] : 0u, iv1 = have ? L.aux1[pk] : 0u;
             const uint32_t inoff = have ? L.inoff[pk] : 0u, outoff = have ? L.outoff[pk] : 0u;
             bar_arrive_n(2, F_THREADS);                  // fields taken: the arrays are free
+            if (NBA_IN_LANE_ROWS && bi > 0)              // batch bi - 1's row scans, bi + 2's hash
+                in_pipe_rows_lanes(T, S, hmask, bbase + bi * G, hk_of(bi + 2), hv_of(bi + 2), tr);
             if (NBA_IN_LANE_FORMAT && have) in_format(T, B, sa_raw, q, inoff, info, q, iv0, iv1);
             const uint32_t sa = (info & INFO_OK) ? sa_raw : INVALID_SA;
             if (have) {
@@ -1028,7 +1065,8 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
                 in_pipe_prologue(T, Bn, ppc_of(Bn), L, pt, tr);
             }
             if (bi > 0) {
-                in_pipe_rows(T, S, hmask, bbase + bi * G, hk_of(bi + 2), hv_of(bi + 2), pt, tr);
+                if (!NBA_IN_LANE_ROWS)
+                    in_pipe_rows(T, S, hmask, bbase + bi * G, hk_of(bi + 2), hv_of(bi + 2), pt, tr);
             } else {
                 for (uint32_t k = cta * PIPE_P + pt; k <= hmask; k += G * PIPE_P) {
                     P.hk2[k] = ~0ull;
@@ -1040,6 +1078,15 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
                 in_pipe_prologue(T, Bn, ppc_of(Bn), L, pt, tr);
             }
             if (tr && pt == 0) tr[4] = gtimer();
+        }
+        if (bi > 0 && tid == 0) {
+            // every CTA (also one without packets in batch bi - 1, whose lanes
+            // did not wait) passes SB2(bi - 1) before its tile part rewrites
+            // the tile maxima that batch bi - 1's row scans read
+            uint32_t v;
+            do {
+                asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(&S.ctl[CTLI_BAR2]) : "memory");
+            } while ((int)(v - (base2 + bi * G)) < 0);
         }
         __syncthreads();                                  // lanes done, bi - 1 decided, bi + 1 prepared
         if (!NBA_RING_TRACE && R.ts && bi > 0 && tid == 0) atomicMax(&R.ts[bi], gtimer());
@@ -1053,8 +1100,9 @@ k_in_fused_ring_pipe(DevTable T, InState S, const InBatchArgs *slots, RingRun R,
     // the last batch's replay: row scans by the side warps, decisions by the lane warps
     const uint32_t bl = n_batches - 1u;
     if (isP) {
-        in_pipe_rows(T, S, hmask, bbase + (bl + 1u) * G, nullptr, nullptr, pt, nullptr);
+        if (!NBA_IN_LANE_ROWS) in_pipe_rows(T, S, hmask, bbase + (bl + 1u) * G, nullptr, nullptr, pt, nullptr);
     } else {
+        if (NBA_IN_LANE_ROWS) in_pipe_rows_lanes(T, S, hmask, bbase + (bl + 1u) * G, nullptr, nullptr, nullptr);
         const InBatchArgs Bp = slots[(first + bl) % n_slots];
         in_pipe_decide(T, S, Bp, ppc_of(Bp), scr, hmask, hk_of(bl), hv_of(bl), base2 + (bl + 1u) * G, warp,
                        s_cnt);

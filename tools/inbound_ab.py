@@ -1,6 +1,6 @@
 #!/usr/bin/env python
-"""ESP inbound ring forms side by side (GPU): the CUDA-graph ring of one-kernel
-launches (default) and the persistent ring (NBA_IPSEC_RING_IN_PERSIST), on the
+"""ESP inbound ring forms side by side (GPU), each forced: the CUDA-graph ring of
+one-kernel launches, the plain persistent ring and the software-pipelined one, on the
 bench's inbound protocol (R ESP batches from R consecutive outbound batches,
 each rotation through nba_ipsec_ring_run_batches, windows reset per rotation),
 K = 100 batches between one CUDA event pair, per size; optionally per library
@@ -91,6 +91,8 @@ def main():
     for rep in range(2):
         for form in ("graph", "persistent", "pipelined"):
             env = dict(os.environ)
+            if form == "graph":
+                env["NBA_IPSEC_RING_IN_PIPE"] = "0"
             if form == "persistent":
                 env["NBA_IPSEC_RING_IN_PERSIST"] = "1"
             if form == "pipelined":
