@@ -1315,12 +1315,24 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
         const BatchArgs B0 = slots[first % n_slots];
         PipeMeta meta;
         pipe_load_meta(B0, fused_ppc(B0.n, G), pt, meta);
+#if NBA_RING_TRACE
+        if (pt == 0 && R.ts) *RTR(0, 13) = gtimer();      // start-up: batch 0's metadata issued
+#endif
         pipe_prologue(T, work_of(0), B0, fused_ppc(B0.n, G), base0 + G, epoch_of(0), L, pt, 0u, meta);
+#if NBA_RING_TRACE
+        if (pt == 0 && R.ts) *RTR(0, 14) = gtimer();      // start-up: batch 0's prologue done
+#endif
     }
+#if NBA_RING_TRACE
+    if (tid == 0 && R.ts) *RTR(0, 15) = gtimer();          // start-up: kernel start (CTA)
+#endif
     __syncthreads();
     // the T-table image landed (the bulk copy overlapped the first prologue);
     // every later lookup of the run finds it in place
     tables_bulk_wait(&L.tbar, 0u);
+#if NBA_RING_TRACE
+    if (tid == 0 && R.ts) *RTR(1, 15) = gtimer();          // start-up: tables landed (row 1)
+#endif
     unsigned long long c_ok = 0, c_drop = 0, c_in = 0, c_out = 0;
     for (uint32_t bi = 0; bi < n_batches; bi++) {
         const BatchArgs B = slots[(first + bi) % n_slots];

@@ -45,7 +45,15 @@ for size in %(sizes)r:
         ts = torch.zeros(K * G * 16, dtype=torch.int64, device="cuda")
         ring.set_timestamps(ts)
         ring.run_batches(K); torch.cuda.synchronize()
-        v = ts.cpu().numpy().reshape(K, G, 16).astype(np.int64)[2:-1]  # skip start-up, last
+        vall = ts.cpu().numpy().reshape(K, G, 16).astype(np.int64)
+        k0 = vall[0, :, 15].min()                 # the run's first CTA start
+        su = lambda a: round(float(np.median((a - k0) / 1e3)), 2)  # noqa: E731
+        startup = {"cta_start": su(vall[0, :, 15]), "b0_meta_issued": su(vall[0, :, 13]),
+                   "b0_prologue_done": su(vall[0, :, 14]), "tables_landed": su(vall[1, :, 15]),
+                   "it0_start": su(vall[0, :, 0]), "it0_barrier_seen": su(vall[0, :, 1]),
+                   "it0_polls_done": su(vall[0, :, 2]), "it0_lanes_done": su(vall[0, :, 3]),
+                   "it0_end": su(vall[0, :, 5]), "it1_end": su(vall[1, :, 5])}
+        v = vall[2:-1]                            # skip start-up, last
         rel = (v - v[:, :, :1]) / 1e3
         names = ["start", "barrier_seen", "polls_done", "lanes_done", "prologue_arrived",
                  "iter_end", "early_keys_done", "pseq_polls_done", "pro_meta", "pro_ranked",
@@ -58,7 +66,7 @@ for size in %(sizes)r:
         p90["slowest_ctas_lanes_us"] = [(int(c), round(float(np.median(lanes[:, c])), 2)) for c in order]
         p90["lanes_done_max_over_ctas"] = round(float(np.median(np.max(lanes, axis=1))), 2)
         it = np.diff(v[:, 0, 0]) / 1e3
-        out[str(size)] = {"median_us": med, "p90_us": p90, "iter_us": float(np.median(it))}
+        out[str(size)] = {"median_us": med, "p90_us": p90, "iter_us": float(np.median(it)), "startup": startup}
     else:
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(); ring.run_batches(K); e1.record(); torch.cuda.synchronize()

@@ -43,7 +43,7 @@ ring.set_timestamps(ts)
 ring.run_batches(20)
 torch.cuda.synchronize()
 v = ts.cpu().numpy().astype(np.int64)
-print(json.dumps({"us_by_K": {int(k): round(res[k], 2) for k in Ks}, "fit_a_us": round(float(afit), 2),
+print(json.dumps({"lib": os.environ.get("NBA_IPSEC_LIB", "default"), "us_by_K": {int(k): round(res[k], 2) for k in Ks}, "fit_a_us": round(float(afit), 2),
                   "fit_b_us": round(float(bfit), 3),
                   "ts_first_batch_us": round(float(v[1] - v[0]) / 1e3, 2),
                   "ts_batches_us": [round(float(x) / 1e3, 2) for x in np.diff(v)[1:6]]}), flush=True)
