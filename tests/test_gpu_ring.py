@@ -399,7 +399,8 @@ def test_pipelined_prologue_modes(n_sa, sizes):
         ring.close()
 
 
-@pytest.mark.parametrize("n_sa,sizes", [(16, [3000, 2500, 4000]), (1024, [20000, 20000, 9000])])
+@pytest.mark.parametrize("n_sa,sizes", [(16, [3000, 2500, 4000]), (1024, [20000, 20000, 9000]),
+                                        (5000, [30000, 12000, 25000])])
 def test_inbound_pipelined_ring_mixed_stream(n_sa, sizes, monkeypatch):
     """The software-pipelined inbound ring (k_in_fused_ring_pipe) on traffic
     with reordering, duplicates, stale replays, single-byte corruption,
