@@ -279,7 +279,7 @@ def measure_outbound(ctx, args, cfg_id, size, steps, warmup, full):
     dbs = [db] + [device.clone(db) for _ in range(R - 1)]
     slots = [(*d.args(), b.n) for d in dbs]
     ring = t.ring(slots)
-    form = {0: "graph", 1: "persistent", 2: "pipelined"}[ring.form]
+    form = {0: "graph", 1: "persistent", 2: "pipelined", 3: "free", 4: "roles"}[ring.form]
     # settle clocks (>= 0.3 s of back-to-back batches), then >= W warm-up batches
     t_end = time.time() + 0.3
     while time.time() < t_end:
@@ -430,7 +430,7 @@ def measure_inbound(ctx, args, cfg_id, steps, warmup, form=None):
     ctr = t.in_counters()
     ok_all = ctr["pkts_ok"] == ctr["batches"] * b.n
     same = bool(torch.equal(esp[-1][3][:b.n].to(torch.int32), db.in_len[:b.n].to(torch.int32)))
-    form = {0: "graph", 1: "persistent", 2: "pipelined"}[ring.form]
+    form = {0: "graph", 1: "persistent", 2: "pipelined", 3: "free", 4: "roles"}[ring.form]
     ring.close()
     del esp
     t.close()
@@ -714,8 +714,9 @@ def run_ours(args):
     w = work_model(head["b"])
     ms_batch = agg["ms_per_step"]
     roof = roofline(ms_batch, w, ctx.peaks, units)
-    kname = "fused_ring" if head["form"] != "graph" else "fused"
-    roof_line = {"kernel": "k_fused_ring_pipe" if head["form"] == "pipelined" else "k_fused_ring",
+    kname = {"graph": "fused", "roles": "fused_ring_roles"}.get(head["form"], "fused_ring")
+    roof_line = {"kernel": {"pipelined": "k_fused_ring_pipe", "roles": "k_fused_ring_roles",
+                            "free": "k_fused_ring_free"}.get(head["form"], "k_fused_ring"),
                  "bound": "alu", "achieved": roof["alu"]["achieved"], "peak": roof["alu"]["peak"],
                  "unit": "Tops/s", "frac": roof["alu"]["frac"],
                  "traffic": load_traffic(kname, gen.CONFIGS[main_cfg]["name"]),

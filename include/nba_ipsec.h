@@ -196,13 +196,22 @@ int nba_ipsec_ring_cursor(const nba_ipsec_ring *r);          /* slot of the next
  * cap < 2. */
 int nba_ipsec_ring_set_timestamps(nba_ipsec_ring *r, unsigned long long *dev_ts, uint32_t cap);
 enum { NBA_IPSEC_RING_GRAPH = 0, NBA_IPSEC_RING_PERSISTENT = 1, NBA_IPSEC_RING_PIPELINED = 2,
-       NBA_IPSEC_RING_FREE = 3 };
+       NBA_IPSEC_RING_FREE = 3, NBA_IPSEC_RING_ROLES = 4 };
 /* The form a run takes (NBA_IPSEC_RING_*); set_form switches a persistent ring
- * between PERSISTENT, PIPELINED and FREE -- the pipelined form without the
+ * between PERSISTENT, PIPELINED, FREE -- the pipelined form without the
  * end-of-batch CTA barrier: a lane warp that finished its run starts the next
- * batch while longer runs go on (mixed-length batches) -- (NBA_IPSEC_EINVAL
- * for graph rings or slots the pipelined forms do not fit).  All give
- * identical results. */
+ * batch while longer runs go on (mixed-length batches) -- and ROLES: CTA
+ * roles instead of warp roles, a few "sequencer" CTAs run every batch's
+ * prologue (validity, per-SA ranks over the whole batch, sequence numbers,
+ * PAPER.md:389-395 / RFC 4303 §3.3.3) and write one record per packet, the
+ * other CTAs encrypt as soon as a batch's records are out, with no grid-wide
+ * synchronisation between batches on their side.  ROLES fits slots with SA
+ * indices, <= 512 packets per encrypting CTA and <= 2048 SAs (its sequencer
+ * count: 6 for packets of <= 114 bytes, else 4; NBA_IPSEC_ROLES_P at creation
+ * overrides) and is the default form of rings whose every slot holds packets
+ * of one length, at most 1010 bytes (NBA_IPSEC_RING_ROLES=0/1 at creation
+ * overrides).  NBA_IPSEC_EINVAL for
+ * graph rings or slots a form does not fit.  All give identical results. */
 int nba_ipsec_ring_form(const nba_ipsec_ring *r);
 int nba_ipsec_ring_set_form(nba_ipsec_ring *r, int form);
 int nba_ipsec_ring_destroy(nba_ipsec_ring *r);   /* NULL -> OK */

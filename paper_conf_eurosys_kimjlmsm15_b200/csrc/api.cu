@@ -410,6 +410,9 @@ struct nba_ipsec_ring {
     bool free_run = false;               //   its free-running-lanes variant (k_fused_ring_free)
     bool in_pipe = false;                // inbound: software-pipelined form (k_in_fused_ring_pipe)
     bool pipe_ok = false;                // every slot fits the pipelined form
+    bool roles = false;                  // role-split form (k_fused_ring_roles)
+    bool roles_ok = false;               // every slot fits it (buffers allocated)
+    RolesBufs rq = {};                   //   its hand-off counters, records, per-SA totals
     uint64_t flow_gen = 0;               // the table's flow-table generation when recorded
     uint32_t cursor = 0;                 // the slot the next run_batches starts at
     unsigned long long *ts = nullptr;    // per-batch timestamps (caller's device buffer)
@@ -453,6 +456,51 @@ int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, u
             r->pipe_ok = slots[i].sa_idx && fused_pipe_ok(slots[i].n_pkts, t->grid_fused);
         r->pipe = r->pipe_ok && !std::getenv("NBA_IPSEC_RING_NOPIPE");
         r->free_run = r->pipe && std::getenv("NBA_IPSEC_RING_FREE");
+        // role-split form: sequencer CTAs + lane CTAs (every slot with SA indices,
+        // <= 512 packets per lane CTA, n_sa <= ROLES_MAX_SA).  The default for
+        // rings whose every slot holds packets of one length up to 1010 bytes
+        // (1024-B frames): measured per 65,536-packet batch against the
+        // pipelined form (tools/ring_forms.py, K = 200) 64 B 21.1 vs 21.9 us,
+        // 128 B 28.2 vs 32.7, 256 B 43.3 vs 47.3, 512 B 73.7 vs 76.4, 1024 B
+        // 132.9 vs 133.8, 1514 B 190.7 vs 189.0.  Sequencers: 6 for packets of
+        // <= 114 bytes (the 64-B batch needs them to keep ahead of the lanes),
+        // else 4 (NBA_IPSEC_ROLES_P overrides; NBA_IPSEC_RING_ROLES=0/1 forces).
+        {
+            bool one_len = true, idx = true;
+            uint32_t max_len = 0;
+            std::vector<uint16_t> lens;
+            for (uint32_t i = 0; i < n_slots && idx; i++) {
+                idx = slots[i].sa_idx != nullptr;
+                lens.resize(slots[i].n_pkts);
+                if (!idx || cudaMemcpy(lens.data(), slots[i].in_len, lens.size() * sizeof(uint16_t),
+                                       cudaMemcpyDefault) != cudaSuccess) {
+                    one_len = false;
+                    break;
+                }
+                for (uint16_t v : lens) {
+                    one_len = one_len && v == lens[0];
+                    max_len = std::max<uint32_t>(max_len, v);
+                }
+            }
+            const char *pe = std::getenv("NBA_IPSEC_ROLES_P");
+            const uint32_t npro = pe ? (uint32_t)std::max(1, std::atoi(pe)) : (max_len <= 114u ? 6u : 4u);
+            r->roles_ok = idx;
+            for (uint32_t i = 0; i < n_slots && r->roles_ok; i++)
+                r->roles_ok = fused_roles_ok(slots[i].n_pkts, t->n_sa, t->grid_fused, npro);
+            if (r->roles_ok) {
+                const uint32_t Lc = (uint32_t)t->grid_fused - npro;
+                r->rq.npro = npro;
+                if (cudaMalloc(&r->rq.ctl, ROLES_CTL_WORDS * sizeof(uint32_t)) != cudaSuccess ||
+                    cudaMemset(r->rq.ctl, 0, ROLES_CTL_WORDS * sizeof(uint32_t)) != cudaSuccess ||
+                    cudaMalloc(&r->rq.rec, (size_t)ROLES_NREC * Lc * 512u * sizeof(uint32_t)) != cudaSuccess ||
+                    cudaMalloc(&r->rq.ptot, (size_t)2u * npro * t->n_sa * sizeof(uint32_t)) != cudaSuccess) {
+                    nba_ipsec_ring_destroy(r);
+                    return NBA_IPSEC_ENOMEM;
+                }
+                const char *re = std::getenv("NBA_IPSEC_RING_ROLES");
+                r->roles = re ? std::atoi(re) != 0 : (one_len && max_len <= 1010u);
+            }
+        }
         std::vector<BatchArgs> hb(n_slots);
         for (uint32_t i = 0; i < n_slots; i++) {
             const nba_ipsec_batch &b = slots[i];
@@ -621,6 +669,8 @@ static int ring_launch(nba_ipsec_ring *r, uint32_t first, uint32_t n_batches, cu
     if (r->ts) {
 #ifdef NBA_RING_TRACE   // debug variant: [n_batches][grid][8] phase stamps
         const size_t need = (size_t)n_batches * t->grid_fused * 16u;
+#elif defined(NBA_ROLES_TRACE)
+        const size_t need = (size_t)n_batches * 9u + 1u;   // + the role-split ring's stamps
 #else
         const size_t need = (size_t)n_batches + 1u;
 #endif
@@ -639,7 +689,8 @@ static int ring_launch(nba_ipsec_ring *r, uint32_t first, uint32_t n_batches, cu
                    : NBA_IPSEC_ECUDA;
     if (r->d_slots) {
         const cudaError_t e =
-            r->free_run ? launch_fused_ring_free(t->T, t->W, r->d_slots, R, r->hist_b, t->grid_fused, st)
+            r->roles    ? launch_fused_ring_roles(t->T, t->W, r->d_slots, R, r->rq, t->grid_fused, st)
+            : r->free_run ? launch_fused_ring_free(t->T, t->W, r->d_slots, R, r->hist_b, t->grid_fused, st)
             : r->pipe   ? launch_fused_ring_pipe(t->T, t->W, r->d_slots, R, r->hist_b, t->grid_fused, st)
                         : launch_fused_ring(t->T, t->W, r->d_slots, R, r->hist_b, t->grid_fused, st);
         return e == cudaSuccess ? NBA_IPSEC_OK : NBA_IPSEC_ECUDA;
@@ -702,10 +753,16 @@ int nba_ipsec_ring_set_form(nba_ipsec_ring *r, int form)
 {
     if (!r || !r->d_slots) return NBA_IPSEC_EINVAL;   // graph rings have one form
     if (form == NBA_IPSEC_RING_PERSISTENT) {
+        r->pipe = r->free_run = r->roles = false;
+        return NBA_IPSEC_OK;
+    }
+    if (form == NBA_IPSEC_RING_ROLES && r->roles_ok) {
         r->pipe = r->free_run = false;
+        r->roles = true;
         return NBA_IPSEC_OK;
     }
     if ((form == NBA_IPSEC_RING_PIPELINED || form == NBA_IPSEC_RING_FREE) && r->pipe_ok) {
+        r->roles = false;
         r->pipe = true;
         r->free_run = form == NBA_IPSEC_RING_FREE;
         return NBA_IPSEC_OK;
@@ -718,6 +775,7 @@ int nba_ipsec_ring_form(const nba_ipsec_ring *r)
     if (!r) return NBA_IPSEC_EINVAL;
     if (r->d_in_slots) return r->in_pipe ? NBA_IPSEC_RING_PIPELINED : NBA_IPSEC_RING_PERSISTENT;
     return !r->d_slots ? NBA_IPSEC_RING_GRAPH
+           : r->roles    ? NBA_IPSEC_RING_ROLES
            : r->free_run ? NBA_IPSEC_RING_FREE
            : r->pipe    ? NBA_IPSEC_RING_PIPELINED
                         : NBA_IPSEC_RING_PERSISTENT;
@@ -730,8 +788,10 @@ int nba_ipsec_ring_destroy(nba_ipsec_ring *r)
         DeviceGuard g(r->t->device);
         if (r->exec) cudaGraphExecDestroy(r->exec);
         if (r->graph) cudaGraphDestroy(r->graph);
-        if (r->d_slots || r->hist_b || r->d_in_slots || r->hkey_b || r->hval_b)
+        if (r->d_slots || r->hist_b || r->d_in_slots || r->hkey_b || r->hval_b || r->rq.ctl)
             cudaDeviceSynchronize();   // a run may still be in flight
+        for (void *q : {(void *)r->rq.ctl, (void *)r->rq.rec, (void *)r->rq.ptot})
+            if (q) cudaFree(q);
         if (r->d_slots) cudaFree(r->d_slots);
         if (r->hist_b) cudaFree(r->hist_b);
         if (r->d_in_slots) cudaFree(r->d_in_slots);

@@ -209,6 +209,21 @@ cudaError_t launch_fused_ring_pipe(const DevTable &T, const DevWork &W, const Ba
 cudaError_t launch_fused_ring_free(const DevTable &T, const DevWork &W, const BatchArgs *slots,
                                    const RingRun &R, uint16_t *hist_b, int grid, cudaStream_t st);
 bool fused_pipe_ok(uint32_t n, int grid);
+// Role-split ring (k_fused_ring_roles): npro sequencer CTAs write one record
+// per packet into a ring of ROLES_NREC record buffers, the other CTAs encrypt.
+constexpr uint32_t ROLES_NREC = 4;          // batches of records in flight
+constexpr uint32_t ROLES_MAX_SA = 2048;     // per-warp SA counters in a sequencer's shared memory
+constexpr uint32_t ROLES_RPP_MAX = 16384;   // packets per sequencer and batch (shared stash)
+constexpr uint32_t ROLES_CTL_WORDS = 2u * ROLES_NREC + 2u;   // ready[], consumed[], pbar, exit
+struct RolesBufs {
+    uint32_t *ctl;      // [ROLES_CTL_WORDS] hand-off counters (zero between launches)
+    uint32_t *rec;      // [ROLES_NREC][(grid - npro) * 512] per-packet sequence numbers (0: drop)
+    uint32_t *ptot;     // [2][npro][n_sa] per-sequencer per-SA valid-packet totals
+    uint32_t npro;      // sequencer CTAs
+};
+bool fused_roles_ok(uint32_t n, uint32_t n_sa, int grid, uint32_t npro);
+cudaError_t launch_fused_ring_roles(const DevTable &T, const DevWork &W, const BatchArgs *slots,
+                                    const RingRun &R, const RolesBufs &Q, int grid, cudaStream_t st);
 cudaError_t launch_fused_ring(const DevTable &T, const DevWork &W, const BatchArgs *slots,
                               const RingRun &R, uint16_t *hist_b, int grid, cudaStream_t st);
 int aes_grid(int num_sms);

@@ -70,6 +70,9 @@ namespace nba {
 #ifndef NBA_PIPE_ONEBIN       // pipelined ring: one-length-bin batches keep index order (no sort)
 #define NBA_PIPE_ONEBIN 1
 #endif
+#ifndef NBA_PIPE_PRO_DELAY0   // the prologue warps' delay in the first iteration of a launch (ns)
+#define NBA_PIPE_PRO_DELAY0 0
+#endif
 #ifndef NBA_PIPE_META_PF      // pipelined ring: L2 prefetch of the metadata two batches ahead
 #define NBA_PIPE_META_PF 1
 #endif
@@ -1290,7 +1293,7 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
         L.stag_ns = 0u;
         L.stag_acc = 0u;
         L.lanes_acc = 0u;
-        L.pro_delay = 0u;
+        L.pro_delay = NBA_PIPE_PRO_DELAY0;
     }
     for (uint32_t k = tid; k < PIPE_MAX_PPC; k += F_THREADS) L.tailf[k] = 0u;   // split: ready flags
     for (uint32_t k = tid; k < 2u * F_SUPER; k += F_THREADS) {
@@ -1478,11 +1481,24 @@ k_fused_ring_pipe(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
                             while ((uint32_t)gtimer() - t_start < d) __nanosleep(256);
                         }
                     }
+#if NBA_RING_TRACE
+                    // lane timeline of the first batches (CTAs 0..3): esp_packet's clock64
+                    // segments, then globaltimer at its start / end
+                    unsigned long long *ldbg = (R.ts && cta < 4u && bi < 4u)
+                        ? R.ts + (size_t)n_batches * G * 16u + ((size_t)(bi * 4u + cta) * PIPE_MAX_PPC + tid) * 8u
+                        : nullptr;
+                    if (ldbg) ldbg[6] = gtimer();
+#else
+                    unsigned long long *ldbg = nullptr;
+#endif
                     if (!NBA_PROLOGUE_ONLY)   // (debug A/B: the ring without the lane work)
-                        esp_packet(T, B, L, H, lane4r, tid, sa, info, q32, inoff, outoff, pp, nullptr,
+                        esp_packet(T, B, L, H, lane4r, tid, sa, info, q32, inoff, outoff, pp, ldbg,
                                    (NBA_PIPE_STAGGER && uniform && warp < PIPE_LANE_WARPS / 2u)
                                        ? &L.stag_acc : nullptr,
                                    t_start);
+#if NBA_RING_TRACE
+                    if (ldbg) ldbg[7] = gtimer();
+#endif
                     const uint32_t Dp = info & 0x7ffu;
                     const uint32_t Lp = 48u + esp_C(Dp);
                     B.out_len[pkt] = (uint16_t)Lp;
@@ -1841,6 +1857,406 @@ k_fused_ring_free(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
     }
 }
 
+// ------------------------------------- role-split ring (SM specialisation)
+// k_fused_ring_roles: the batch ring with CTA roles instead of warp roles.
+// CTAs 0..P-1 ("sequencers") run every batch's prologue: validity (A15), the
+// stable rank of each valid packet among the batch's earlier valid packets of
+// its SA (index order over the whole batch), its sequence number q = seq + 1
+// + rank (RFC 4303 §3.3.3: dropped once q would pass 2^32 - 1, as the oracle's
+// step 2), and one 4-byte record per packet (q, 0 = drop) into a ring of
+// ROLES_NREC record buffers.  CTAs P..G-1
+// ("lanes", 16 warps) take batch b's records as soon as its sequencers
+// published them and encrypt their packets with the same esp_packet as every
+// other path.  Nothing synchronises the lane CTAs between two batches: a lane
+// warp that finished batch b starts batch b + 1 once its records are there, so
+// the shared-memory-bound AES and the ALU-bound SHA-1 of different warps drift
+// apart instead of running in lock step (the pipelined ring's lanes spend
+// most of a 64-B batch with every warp in the same phase), and the
+// per-batch critical section (grid barrier, row scans, polls) leaves the lane
+// SMs altogether.  Packet i of a batch always goes to the same lane (lane CTA
+// i / ppc, position j = i mod ppc -> warp j mod 16, lane j / 16, so every warp
+// carries ~ppc / 16 packets), so the uses of one ring slot write its output
+// slots in program order.  Records are stored by packet index (coalesced
+// sequencer stores; a lane's one 4-byte load per batch is scattered); a lane
+// reads its packet's SA, length and offsets from the batch itself one batch
+// ahead, so its SA line and round keys are ready before the record is read,
+// and prefetches its next payload line into L2.  The lanes' waits and counts
+// use no acquire / release fences (roles_lane_wait / roles_lane_consumed).
+//
+// Hand-offs (counters monotonic within a launch, zeroed by the last CTA to
+// leave; s = b mod ROLES_NREC, k = b / ROLES_NREC):
+//   ready[s]    += 1 per sequencer once batch b's records are written: the
+//                  lanes wait for (k + 1) P;
+//   consumed[s] += 1 per lane warp once it loaded its records of batch b: a
+//                  sequencer starts batch b only when it reads k * (lane warps);
+//   pbar        += 1 per sequencer and batch once its per-SA totals are out.
+__device__ __forceinline__ uint32_t roles_ld_acq(const uint32_t *p)
+{
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ void roles_red_rel(uint32_t *p, uint32_t v)
+{
+    asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+__device__ __forceinline__ void roles_wait_geq(const uint32_t *p, uint32_t target)
+{
+    while ((int32_t)(roles_ld_acq(p) - target) < 0) __nanosleep(32);
+}
+
+// The lanes' side of the hand-offs, without the acquire / release fences:
+// an acquire load invalidates the SM's L1 (CCTL.IVALL) and a release RMW waits
+// for every store the warp has in flight (MEMBAR + ERRBAR) -- together ~8% of
+// the lane warps' stall samples (ncu, 64 B).  Instead: lane 0 polls with a
+// relaxed load and the warp reads its records with L2 loads (ld.cg) issued
+// only after the poll returned (control dependency, in-order issue; L2 is the
+// point of coherence, and the sequencer's release made its records visible
+// there before its count); the "consumed" count is a relaxed add whose operand
+// depends, through a warp vote, on every lane's loaded record -- it cannot be
+// performed before those loads returned.
+__device__ __forceinline__ uint32_t roles_ld_relaxed(const uint32_t *p)
+{
+    uint32_t v;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ void roles_lane_wait(const uint32_t *p, uint32_t target)
+{
+    if ((threadIdx.x & 31u) == 0)
+        while ((int32_t)(roles_ld_relaxed(p) - target) < 0) __nanosleep(32);
+    __syncwarp();
+}
+
+__device__ __forceinline__ void roles_lane_consumed(uint32_t *p, uint32_t q)
+{
+    uint32_t z;
+    asm("and.b32 %0, %1, 0;" : "=r"(z) : "r"(q));     // 0, opaque: depends on the load of q
+    z = __ballot_sync(0xffffffffu, z != 0u);          // every lane's record has returned
+    if ((threadIdx.x & 31u) == 0)
+        asm volatile("red.relaxed.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(1u + z) : "memory");
+}
+
+#ifndef NBA_ROLES_TRACE       // debug variant: sequencer 0's phase stamps per batch and lane CTA 0's
+#define NBA_ROLES_TRACE 0     //   record arrival, after ts[0..n_batches] (tools/roles_trace.py)
+#endif
+#if NBA_ROLES_TRACE
+#define RLT(bi, k) (R.ts + 1u + R.n_batches + (size_t)(bi) * 8u + (k))
+#endif
+#ifndef NBA_ROLES_AG          // sequencer: rounds of 32 packets whose metadata loads are in flight together
+#define NBA_ROLES_AG 8
+#endif
+
+__device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchArgs *slots, const RingRun &R,
+                                                const RolesBufs &Q, uint8_t *smem, uint32_t p)
+{
+    const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
+    const uint32_t P = Q.npro, Lc = gridDim.x - P, LW = Lc * 16u, n_sa = T.n_sa;
+    // shared memory: per-packet stash of this sequencer's range, per-warp SA counters
+    uint16_t *rank = reinterpret_cast<uint16_t *>(smem);           // [ROLES_RPP_MAX]
+    uint16_t *sa16 = rank + ROLES_RPP_MAX;                         // [ROLES_RPP_MAX] 0xffff: drop
+    uint16_t *d16 = sa16 + ROLES_RPP_MAX;                          // [ROLES_RPP_MAX]
+    uint16_t *cnt = d16 + ROLES_RPP_MAX;                           // [16][ROLES_MAX_SA]
+    uint32_t *seqs = reinterpret_cast<uint32_t *>(cnt + 16u * ROLES_MAX_SA);   // [ROLES_MAX_SA]
+    unsigned long long *start = reinterpret_cast<unsigned long long *>(seqs + ROLES_MAX_SA);
+    uint32_t *ready = Q.ctl, *consumed = Q.ctl + ROLES_NREC, *pbar = Q.ctl + 2u * ROLES_NREC;
+    uint16_t *mycnt = cnt + warp * ROLES_MAX_SA;
+    for (uint32_t s = tid; s < n_sa; s += F_THREADS) seqs[s] = __ldcg(&T.seq[s]);
+    for (uint32_t s = lane; s < n_sa; s += 32u) mycnt[s] = 0;
+    __syncthreads();
+    for (uint32_t bi = 0; bi < R.n_batches; bi++) {
+        const BatchArgs B = slots[(R.first + bi) % R.n_slots];
+        const uint32_t n = B.n, rpp = (n + P - 1u) / P;
+        const uint32_t r0 = min(n, p * rpp), r1 = min(n, r0 + rpp);
+        const uint32_t spw = (((rpp + 15u) / 16u) + 31u) & ~31u;   // whole rounds per warp
+        const uint32_t w0 = min(r1, r0 + warp * spw), w1 = min(r1, w0 + spw);
+        // the next batch's metadata lines into L2 (ahead of its phase A)
+        if (bi + 1u < R.n_batches) {
+            const BatchArgs Bn = slots[(R.first + bi + 1u) % R.n_slots];
+            const uint32_t rn = (Bn.n + P - 1u) / P, a0 = min(Bn.n, p * rn), a1 = min(Bn.n, a0 + rn);
+            const uint32_t l16 = a1 > a0 ? (2u * (a1 - a0) + 127u) / 128u + 1u : 0u;
+            const uint32_t l32 = a1 > a0 ? (4u * (a1 - a0) + 127u) / 128u + 1u : 0u;
+            for (uint32_t k = tid; k < l16 + l32; k += F_THREADS) {   // in_len, sa_idx
+                const uint8_t *a, *e;
+                if (k < l16) {
+                    a = reinterpret_cast<const uint8_t *>(Bn.in_len + a0) + 128u * k;
+                    e = reinterpret_cast<const uint8_t *>(Bn.in_len + a1);
+                } else {
+                    a = reinterpret_cast<const uint8_t *>(Bn.sa_idx + a0) + 128u * (k - l16);
+                    e = reinterpret_cast<const uint8_t *>(Bn.sa_idx + a1);
+                }
+                if (a < e) prefetch_l2(a);
+            }
+        }
+#if NBA_ROLES_TRACE
+        if (R.ts && p == 0 && tid == 0) *RLT(bi, 0) = gtimer();
+#endif
+        // every lane warp has taken its records of batch bi - NREC (their buffer is reused)
+        if (bi >= ROLES_NREC) {
+            if (tid == 0) roles_wait_geq(&consumed[bi % ROLES_NREC], (bi / ROLES_NREC) * LW);
+            __syncthreads();
+        }
+        // A. validity, the packet's rank among the warp's earlier packets of its
+        //    SA (rounds of 32 in index order, match groups within a round)
+        for (uint32_t g0 = w0; g0 < w1; g0 += 32u * NBA_ROLES_AG) {
+            uint32_t s[NBA_ROLES_AG], D[NBA_ROLES_AG];
+#pragma unroll
+            for (uint32_t k = 0; k < NBA_ROLES_AG; k++) {
+                const uint32_t i = g0 + 32u * k + lane;
+                const bool in = i < w1;
+                s[k] = in ? B.sa_idx[i] : INVALID_SA;
+                D[k] = in ? (uint32_t)B.in_len[i] : 0u;
+            }
+#pragma unroll
+            for (uint32_t k = 0; k < NBA_ROLES_AG; k++) {
+                if (g0 + 32u * k >= w1) break;                       // (warp-uniform)
+                const uint32_t i = g0 + 32u * k + lane;
+                const bool in = i < w1;
+                const bool cand = in && s[k] < n_sa && D[k] >= MIN_D && D[k] <= MAX_D;
+                // lanes with the same SA (valid ones; SA < 2048): match by ballots
+                // over the 11 SA bits and the validity bit
+                const uint32_t key = cand ? s[k] : 0x800u;
+                uint32_t peers = 0xffffffffu;
+#pragma unroll
+                for (uint32_t bit = 0; bit < 12u; bit++) {
+                    const bool on = (key >> bit) & 1u;
+                    const uint32_t m = __ballot_sync(0xffffffffu, on);
+                    peers &= on ? m : ~m;
+                }
+                const uint32_t leader = (uint32_t)__ffs(peers) - 1u;
+                uint32_t c0 = (cand && lane == leader) ? (uint32_t)mycnt[s[k]] : 0u;
+                c0 = __shfl_sync(0xffffffffu, c0, leader);
+                if (cand) {
+                    rank[i - r0] = (uint16_t)(c0 + __popc(peers & lanemask_lt()));
+                    if (lane == leader) mycnt[s[k]] = (uint16_t)(c0 + __popc(peers));
+                }
+                if (in) {
+                    sa16[i - r0] = cand ? (uint16_t)s[k] : (uint16_t)0xffffu;
+                    d16[i - r0] = (uint16_t)D[k];
+                }
+            }
+        }
+        __syncthreads();
+#if NBA_ROLES_TRACE
+        if (R.ts && p == 0 && tid == 0) *RLT(bi, 1) = gtimer();
+#endif
+        // B. exclusive prefix of the warps' counts per SA; this sequencer's totals
+        uint32_t *ptot = Q.ptot + (size_t)(bi & 1u) * P * n_sa;
+        for (uint32_t s = tid; s < n_sa; s += F_THREADS) {
+            uint32_t run = 0;
+#pragma unroll
+            for (uint32_t w = 0; w < 16u; w++) {
+                const uint32_t c = cnt[w * ROLES_MAX_SA + s];
+                cnt[w * ROLES_MAX_SA + s] = (uint16_t)run;
+                run += c;
+            }
+            ptot[(size_t)p * n_sa + s] = run;
+        }
+        __syncthreads();
+#if NBA_ROLES_TRACE
+        if (R.ts && p == 0 && tid == 0) *RLT(bi, 2) = gtimer();
+#endif
+        if (tid == 0) {
+            __threadfence();
+            roles_red_rel(pbar, 1u);
+            roles_wait_geq(pbar, (bi + 1u) * P);
+        }
+        __syncthreads();
+#if NBA_ROLES_TRACE
+        if (R.ts && p == 0 && tid == 0) *RLT(bi, 3) = gtimer();
+#endif
+        // C. per SA: its sequence number before this sequencer's range, and
+        //    after the batch (saturating: a packet that would pass 2^32 - 1 is
+        //    dropped and consumes nothing)
+        for (uint32_t s = tid; s < n_sa; s += F_THREADS) {
+            uint32_t before = 0, all = 0;
+            for (uint32_t q = 0; q < P; q++) {
+                const uint32_t v = __ldcg(&ptot[(size_t)q * n_sa + s]);
+                before += q < p ? v : 0u;
+                all += v;
+            }
+            const unsigned long long sq = seqs[s];
+            start[s] = sq + before;
+            seqs[s] = (uint32_t)min(sq + all, 0xffffffffull);
+        }
+        __syncthreads();
+#if NBA_ROLES_TRACE
+        if (R.ts && p == 0 && tid == 0) *RLT(bi, 4) = gtimer();
+#endif
+        // D. the records (the sequence number, 0 = drop), by packet index
+        uint32_t *rec = Q.rec + (size_t)(bi % ROLES_NREC) * Lc * 512u;
+#pragma unroll 4
+        for (uint32_t g0 = w0; g0 < w1; g0 += 32u) {
+            const uint32_t i = g0 + lane;
+            if (i < w1) {
+                const uint32_t s = sa16[i - r0];
+                uint32_t r = 0u;
+                if (s != 0xffffu) {
+                    const unsigned long long q =
+                        start[s] + mycnt[s] + (unsigned long long)rank[i - r0] + 1ull;
+                    r = q <= 0xffffffffull ? (uint32_t)q : 0u;
+                }
+                rec[i] = r;
+            }
+        }
+        __syncwarp();
+        for (uint32_t s = lane; s < n_sa; s += 32u) mycnt[s] = 0;   // (the warp's own row)
+        __syncthreads();
+        if (tid == 0) {
+            __threadfence();
+            roles_red_rel(&ready[bi % ROLES_NREC], 1u);
+#if NBA_ROLES_TRACE
+            if (R.ts && p == 0) *RLT(bi, 5) = gtimer();
+#endif
+        }
+    }
+    if (p == 0)
+        for (uint32_t s = tid; s < n_sa; s += F_THREADS) T.seq[s] = seqs[s];
+}
+
+__device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W, const BatchArgs *slots,
+                                            const RingRun &R, const RolesBufs &Q, uint8_t *smem, uint32_t c)
+{
+    const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
+    const uint32_t P = Q.npro, Lc = gridDim.x - P, n_sa = T.n_sa;
+    const uint32_t sb = smem_u32(smem);
+    const uint32_t toff = (0x10000u - (sb & 0xffffu)) & 0xffffu;
+    uint32_t lo_off = 0;
+    if (toff < sizeof(FusedLo)) {
+        if (toff + AES_TABLE_BYTES + sizeof(FusedHi) + sizeof(FusedLo) > F_SMEM) __trap();
+        lo_off = toff + AES_TABLE_BYTES + (uint32_t)sizeof(FusedHi);
+    }
+    uint8_t *tabs = smem + toff;
+    FusedLo &L = *reinterpret_cast<FusedLo *>(smem + lo_off);
+    FusedHi &H = *reinterpret_cast<FusedHi *>(smem + toff + AES_TABLE_BYTES);
+    const uint32_t lane4r = (lane * 4u) | (smem_u32(tabs) & 0xffff0000u);
+    tables_stage(tabs, T, &L.tbar, true);
+    __syncthreads();
+    tables_bulk_wait(&L.tbar, 0u);
+    const uint32_t *ready = Q.ctl;
+    uint32_t *consumed = Q.ctl + ROLES_NREC;
+    const uint32_t jpos = lane * 16u + warp;         // position in the CTA's packet range
+    unsigned long long c_ok = 0, c_drop = 0, c_in = 0, c_out = 0;
+    // The lane's packet fields (batch inputs: SA, length, offsets) are known
+    // before its record (the sequence number): loaded one batch ahead, so that
+    // the SA line load and the round-key expansion run before the record wait.
+    // Its payload's first line goes into L2 one batch ahead too.
+    struct Fields { uint32_t i, sa, D, inoff, outoff; bool have; };
+    auto fields_of = [&](uint32_t bi) {
+        Fields f = {0u, INVALID_SA, 0u, 0u, 0u, false};
+        if (bi >= R.n_batches) return f;
+        const BatchArgs B = slots[(R.first + bi) % R.n_slots];
+        const uint32_t ppc = (B.n + Lc - 1u) / Lc;
+        f.i = c * ppc + jpos;
+        f.have = jpos < ppc && f.i < B.n;
+        if (f.have) {
+            f.sa = B.sa_idx[f.i];
+            f.D = B.in_len[f.i];
+            f.inoff = B.in_off[f.i];
+            f.outoff = B.out_off[f.i];
+        }
+        return f;
+    };
+    Fields f = fields_of(0u);
+    if (f.have) prefetch_l2(slots[R.first % R.n_slots].in_buf + f.inoff);
+    for (uint32_t bi = 0; bi < R.n_batches; bi++) {
+        const BatchArgs B = slots[(R.first + bi) % R.n_slots];
+        const Fields fn = fields_of(bi + 1u);
+        // the oracle's step 1 (A15): invalid SA or length -> drop, no number used
+        const bool cand = f.have && f.sa < n_sa && f.D >= MIN_D && f.D <= MAX_D;
+        PktPre pp = {};
+        if (cand) {
+            pp = load_pkt_pre(T, B.in_buf, f.sa, f.inoff, true, 0u);
+            expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
+        }
+#if NBA_ROLES_TRACE
+        if (R.ts && c == 0 && tid == 0) *RLT(bi, 6) = gtimer();
+#endif
+        roles_lane_wait(&ready[bi % ROLES_NREC], (bi / ROLES_NREC + 1u) * P);
+#if NBA_ROLES_TRACE
+        if (R.ts && c == 0 && tid == 0) *RLT(bi, 7) = gtimer();
+#endif
+        const uint32_t q = cand ? __ldcg(&Q.rec[(size_t)(bi % ROLES_NREC) * Lc * 512u + f.i]) : 0u;
+        roles_lane_consumed(&consumed[bi % ROLES_NREC], q);
+        if (f.have) {
+            if (q != 0u) {
+                esp_packet(T, B, L, H, lane4r, tid, f.sa, f.D | INFO_OK, q, f.inoff, f.outoff, pp, nullptr);
+                const uint32_t Lp = 48u + esp_C(f.D);
+                B.out_len[f.i] = (uint16_t)Lp;
+                c_ok++;
+                c_in += f.D;
+                c_out += Lp;
+            } else {
+                B.out_len[f.i] = 0;
+                c_drop++;
+            }
+        }
+        // the next packet's payload line into L2 (its offset has arrived by now)
+        if (fn.have) prefetch_l2(slots[(R.first + bi + 1u) % R.n_slots].in_buf + fn.inoff);
+        if (R.ts && lane == 0) atomicMax(&R.ts[1u + bi], gtimer());
+        f = fn;
+    }
+    if (tid < 4) L.cnt[tid] = 0ull;
+    __syncthreads();
+    const unsigned long long s0 = warp_sum_u64(c_ok), s1 = warp_sum_u64(c_drop);
+    const unsigned long long s2 = warp_sum_u64(c_in), s3 = warp_sum_u64(c_out);
+    if (lane == 0) {
+        if (s0) atomicAdd(&L.cnt[0], s0);
+        if (s1) atomicAdd(&L.cnt[1], s1);
+        if (s2) atomicAdd(&L.cnt[2], s2);
+        if (s3) atomicAdd(&L.cnt[3], s3);
+    }
+    __syncthreads();
+    if (tid < 4 && L.cnt[tid]) atomicAdd(&W.counters[tid], L.cnt[tid]);
+}
+
+__global__ void __launch_bounds__(F_THREADS, 1)
+k_fused_ring_roles(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, RolesBufs Q)
+{
+    extern __shared__ __align__(16) uint8_t smem[];
+    if (R.n_batches == 0) return;
+    if (R.ts && blockIdx.x == 0 && threadIdx.x == 0) R.ts[0] = gtimer();
+    if (blockIdx.x < Q.npro) roles_sequencer(T, slots, R, Q, smem, blockIdx.x);
+    else roles_lanes(T, W, slots, R, Q, smem, blockIdx.x - Q.npro);
+    // leave; the last CTA out zeroes the hand-off counters for the next launch
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        if (blockIdx.x == 0) atomicAdd(&W.counters[4], (unsigned long long)R.n_batches);
+        __threadfence();
+        const uint32_t t = atomicAdd(&Q.ctl[2u * ROLES_NREC + 1u], 1u);
+        if (t == gridDim.x - 1u) {
+            __threadfence();
+            for (uint32_t k = 0; k < ROLES_CTL_WORDS; k++) atomicExch(&Q.ctl[k], 0u);
+        }
+    }
+}
+
+bool fused_roles_ok(uint32_t n, uint32_t n_sa, int grid, uint32_t npro)
+{
+    if (npro == 0 || grid <= (int)npro || n == 0 || n_sa == 0 || n_sa > ROLES_MAX_SA) return false;
+    const uint32_t Lc = (uint32_t)grid - npro;
+    return n <= 512u * Lc && (n + npro - 1u) / npro <= ROLES_RPP_MAX;
+}
+
+cudaError_t launch_fused_ring_roles(const DevTable &T, const DevWork &W, const BatchArgs *slots,
+                                    const RingRun &R, const RolesBufs &Q, int grid, cudaStream_t st)
+{
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(F_THREADS);
+    cfg.dynamicSmemBytes = F_SMEM;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeCooperative;   // the roles wait on each other: co-resident
+    attr[0].val.cooperative = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, k_fused_ring_roles, T, W, slots, R, Q);
+}
+
 cudaError_t launch_fused_ring_free(const DevTable &T, const DevWork &W, const BatchArgs *slots,
                                    const RingRun &R, uint16_t *hist_b, int grid, cudaStream_t st)
 {
@@ -1944,6 +2360,9 @@ cudaError_t setup_fused_attributes()
                               (int)F_SMEM);
     if (e0 != cudaSuccess) return e0;
     e0 = cudaFuncSetAttribute(k_fused_ring_free, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              (int)F_SMEM);
+    if (e0 != cudaSuccess) return e0;
+    e0 = cudaFuncSetAttribute(k_fused_ring_roles, cudaFuncAttributeMaxDynamicSharedMemorySize,
                               (int)F_SMEM);
     if (e0 != cudaSuccess) return e0;
     cudaError_t e = cudaFuncSetAttribute(k_fused<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,

@@ -468,7 +468,7 @@ class Ring:
                                                  int(ts.numel()) if ts is not None else 0),
                "nba_ipsec_ring_set_timestamps")
 
-    GRAPH, PERSISTENT, PIPELINED, FREE = 0, 1, 2, 3
+    GRAPH, PERSISTENT, PIPELINED, FREE, ROLES = 0, 1, 2, 3, 4
 
     @property
     def form(self) -> int:

@@ -1,0 +1,141 @@
+"""GPU parity of the role-split batch ring (nba_ipsec_ring form ROLES,
+k_fused_ring_roles): sequencer CTAs assign every batch's sequence numbers
+(RFC 4303 §3.3.3 as the oracle's steps 1-2: invalid SA or
+length -> drop without consuming a number, a number that would pass 2^32 - 1
+-> drop) and the other CTAs encrypt.  Against the oracle processing the same
+batch sequence with carried SA state: whole output pools, out_len, final SA
+counters, device counters -- over sequencer counts, SA counts (1 .. 2048),
+batch sizes that leave most lane CTAs empty, one-slot rings (every batch
+rewrites the same output slots), runs stopping mid-rotation, runs longer than
+the record ring, invalid SAs / lengths and counters at 2^32 - 1."""
+import numpy as np
+import pytest
+
+import oracle
+from paper_conf_eurosys_kimjlmsm15_b200 import gen
+
+pytestmark = pytest.mark.gpu
+
+
+def _slot(db):
+    return (db.in_buf, db.in_off, db.in_len, db.sa_idx, db.out_buf, db.out_off, db.out_len, db.n)
+
+
+def _roles_vs_oracle(p, n_sa, hb, runs, force=True, defined_only=False):
+    import torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    sas = oracle.make_sas(p)
+    ctr = oracle.Counters()
+    R = len(hb)
+    with nba_ipsec.SATable(p, device=0, max_batch=max(b.n for b in hb)) as t:
+        dbs = [device.to_device(b, "cuda") for b in hb]
+        ring = t.ring([_slot(d) for d in dbs])
+        if force:
+            ring.set_form(nba_ipsec.Ring.ROLES)
+        assert ring.form == nba_ipsec.Ring.ROLES
+        last, k = {}, 0
+        for nb in runs:
+            ring.run_batches(nb)
+            for _ in range(nb):
+                o_out, o_len, _ = oracle.process_batch(sas, n_sa, hb[k % R], n_threads=8, counters=ctr)
+                last[k % R] = (o_out, o_len.copy())
+                k += 1
+            assert ring.cursor == k % R
+        torch.cuda.synchronize()
+        for s, (o_out, o_len) in last.items():
+            g_out, g_len = device.fetch(dbs[s])
+            assert np.array_equal(g_len, o_len), f"slot {s}: out_len differs"
+            if defined_only:
+                # only [0, out_len) of a packet's slot is defined: a packet dropped in
+                # a later round leaves the earlier round's bytes there
+                b = hb[s]
+                for i in np.nonzero(o_len)[0]:
+                    a, L = int(b.out_off[i]), int(o_len[i])
+                    assert np.array_equal(g_out[a:a + L], o_out[a:a + L]), f"slot {s} packet {i}"
+            elif not np.array_equal(g_out, o_out):
+                d = np.nonzero(g_out != o_out)[0]
+                raise AssertionError(f"slot {s}: {d.size} output bytes differ, first at {d[:8]}")
+        assert np.array_equal(t.sa_seq(), oracle.sa_seq(sas, n_sa)), "final SA counters differ"
+        assert t.counters() == ctr.as_dict()
+        ring.close()
+
+
+@pytest.mark.parametrize("npro", [1, 4, 9])
+@pytest.mark.parametrize("n_sa,n,sizes", [(61, 9000, (64, "imix", 300)), (2048, 30000, (1514, 64)),
+                                          (1, 20000, (64, 64))])
+def test_roles_ring_matches_oracle(npro, n_sa, n, sizes, monkeypatch):
+    """Sequencer counts 1 / 4 / 9, runs of 5 + 4 + 9 batches (past the record
+    ring of 4), invalid SAs and lengths in slot 0."""
+    if n > 16384 * npro:
+        pytest.skip("a sequencer stashes at most 16,384 packets per batch")
+    monkeypatch.setenv("NBA_IPSEC_ROLES_P", str(npro))
+    p = gen.make_sas(n_sa, cfg_id=71)
+    hb = [gen.make_batch(n, s, n_sa, cfg_id=71, batch=i) for i, s in enumerate(sizes)]
+    hb[0].sa_idx[::97] = n_sa + 1
+    hb[0].in_len[3::211] = 19
+    hb[0].in_len[7::223] = 1501
+    _roles_vs_oracle(p, n_sa, hb, [5, 4, 9])
+
+
+def test_roles_ring_one_slot(monkeypatch):
+    """One slot: every batch rewrites the same output slots with new sequence
+    numbers; the last batch's bytes must be what stays."""
+    p = gen.make_sas(16, cfg_id=72)
+    hb = [gen.make_batch(40000, 64, 16, cfg_id=72)]
+    _roles_vs_oracle(p, 16, hb, [7, 1, 6], force=False)     # one length: the default form
+
+
+@pytest.mark.parametrize("n", [1, 31, 100, 4737, 65536])
+def test_roles_ring_batch_sizes(n):
+    """Batches that leave most lane CTAs (and sequencer ranges) empty, up to
+    the bench's 65,536 packets."""
+    p = gen.make_sas(8, cfg_id=73)
+    hb = [gen.make_batch(n, s, 8, cfg_id=73, batch=k) for k, s in enumerate(("imix", 64))]
+    _roles_vs_oracle(p, 8, hb, [3, 2])
+
+
+def test_roles_ring_sequence_overflow():
+    """SA counters near 2^32 - 1 over consecutive batches: the sequencers drop
+    exactly the packets the oracle drops (and no later packet of that SA)."""
+    n_sa, n = 32, 20000
+    seq = np.full(n_sa, 0xFFFFFFFF - 700, np.uint32)
+    seq[::3] = 0xFFFFFFFF
+    seq[1::5] = 5
+    p = gen.make_sas(n_sa, cfg_id=74)
+    p = gen.SAParams(*[getattr(p, f) for f in ("spi", "tunnel_src", "tunnel_dst", "aes_key",
+                                               "ctr_nonce", "hmac_key")], seq=seq)
+    hb = [gen.make_batch(n, "imix", n_sa, cfg_id=74, batch=k) for k in range(2)]
+    _roles_vs_oracle(p, n_sa, hb, [2, 3], defined_only=True)
+
+
+def test_roles_ring_then_other_paths():
+    """A role-split run, then process_batch and a pipelined run on the same
+    table continue the SA counters exactly (the device state it leaves)."""
+    import torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    n_sa, n = 100, 25000
+    p = gen.make_sas(n_sa, cfg_id=75)
+    hb = [gen.make_batch(n, 64, n_sa, cfg_id=75, batch=k) for k in range(2)]
+    sas = oracle.make_sas(p)
+    with nba_ipsec.SATable(p, device=0, max_batch=n) as t:
+        dbs = [device.to_device(b, "cuda") for b in hb]
+        ring = t.ring([_slot(d) for d in dbs])
+        assert ring.form == nba_ipsec.Ring.ROLES
+        ring.run_batches(5)                    # slots 0 1 0 1 0
+        for k in range(5):
+            oracle.process_batch(sas, n_sa, hb[k % 2])
+        t.process(*dbs[1].args(), n=n)         # slot 1 through process_batch
+        o1 = oracle.process_batch(sas, n_sa, hb[1])
+        ring.set_form(nba_ipsec.Ring.PIPELINED)
+        ring.run_batches(1)                    # cursor 1: slot 1 again
+        o1 = oracle.process_batch(sas, n_sa, hb[1])
+        ring.set_form(nba_ipsec.Ring.ROLES)
+        ring.run_batches(2)                    # slots 0, 1
+        o0 = oracle.process_batch(sas, n_sa, hb[0])
+        o1 = oracle.process_batch(sas, n_sa, hb[1])
+        torch.cuda.synchronize()
+        for d, (o_out, o_len, _) in zip(dbs, (o0, o1)):
+            g_out, g_len = device.fetch(d)
+            assert np.array_equal(g_len, o_len) and np.array_equal(g_out, o_out)
+        assert np.array_equal(t.sa_seq(), oracle.sa_seq(sas, n_sa))
+        ring.close()

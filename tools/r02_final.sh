@@ -25,7 +25,7 @@ for C in 2 3 4; do
 done
 ls gpurun_out/ | grep $TAG | head -40
 for tool in memcheck racecheck synccheck initcheck; do
-  for c in c1 ring_small inbound inring host c4 ring64; do
+  for c in c1 ring_small roles inbound inring host c4 ring64; do
     timeout 420 compute-sanitizer --tool $tool python tools/sanitize_cases.py $c > gpurun_out/sanitizer/${TAG}_${tool}_${c}.txt 2>&1
     echo "$tool $c rc=$? $(grep -E 'SUMMARY|result ==' gpurun_out/sanitizer/${TAG}_${tool}_${c}.txt | tr '\n' ' ')"
   done

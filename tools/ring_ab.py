@@ -42,17 +42,32 @@ for size in %(sizes)r:
     ring.run_batches(max(40, 4 * R)); torch.cuda.synchronize()
     if %(trace)r:
         G = 148
-        ts = torch.zeros(K * G * 16, dtype=torch.int64, device="cuda")
+        ts = torch.zeros(K * G * 16 + 4 * 4 * 448 * 8, dtype=torch.int64, device="cuda")
         ring.set_timestamps(ts)
         ring.run_batches(K); torch.cuda.synchronize()
-        vall = ts.cpu().numpy().reshape(K, G, 16).astype(np.int64)
+        tsn = ts.cpu().numpy().astype(np.int64)
+        vall = tsn[:K * G * 16].reshape(K, G, 16)
+        # lane timelines of batches 0..3 (CTAs 0..3): clock64 segments (setup, AES step 0,
+        # emission, SHA block 0, rest) and globaltimer start / end of esp_packet
+        ld = tsn[K * G * 16:].reshape(4, 4, 448, 8)
+        lanes_tl = {}
+        for bb in range(4):
+            x = ld[bb].reshape(-1, 8)
+            x = x[x[:, 7] > 0]
+            if not len(x):
+                continue
+            it0 = vall[bb, :4, 0].min()
+            lanes_tl[bb] = {"n": int(len(x)), "seg_cycles_median": [int(np.median(x[:, j])) for j in range(5)],
+                            "seg_cycles_p90": [int(np.percentile(x[:, j], 90)) for j in range(5)],
+                            "start_us_p10_50_90": [round(float(np.percentile((x[:, 6] - it0) / 1e3, q)), 2) for q in (10, 50, 90)],
+                            "dur_us_p10_50_90": [round(float(np.percentile((x[:, 7] - x[:, 6]) / 1e3, q)), 2) for q in (10, 50, 90)]}
         k0 = vall[0, :, 15].min()                 # the run's first CTA start
         su = lambda a: round(float(np.median((a - k0) / 1e3)), 2)  # noqa: E731
         startup = {"cta_start": su(vall[0, :, 15]), "b0_meta_issued": su(vall[0, :, 13]),
                    "b0_prologue_done": su(vall[0, :, 14]), "tables_landed": su(vall[1, :, 15]),
                    "it0_start": su(vall[0, :, 0]), "it0_barrier_seen": su(vall[0, :, 1]),
                    "it0_polls_done": su(vall[0, :, 2]), "it0_lanes_done": su(vall[0, :, 3]),
-                   "it0_end": su(vall[0, :, 5]), "it1_end": su(vall[1, :, 5])}
+                   "it0_end": su(vall[0, :, 5]), "it1_end": su(vall[1, :, 5]), "lanes": lanes_tl}
         v = vall[2:-1]                            # skip start-up, last
         rel = (v - v[:, :, :1]) / 1e3
         names = ["start", "barrier_seen", "polls_done", "lanes_done", "prologue_arrived",

@@ -5,7 +5,7 @@ warm-up batches, then K = 200 batches in ONE nba_ipsec_ring_run_batches call
 between one CUDA event pair (a sleep kernel ahead of the start event), per
 form (nba_ipsec_ring_set_form), two passes interleaved.
 
-    python tools/ring_forms.py [sizes...]"""
+    FORMS=pipelined,roles RING_K=200 python tools/ring_forms.py [sizes...]"""
 import json
 import os
 import sys
@@ -17,7 +17,10 @@ from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec, shard  # noqa:
 
 K = 200
 sizes = [x if x == "imix" else int(x) for x in sys.argv[1:]] or [64, 1514, "imix"]
-forms = {"pipelined": nba_ipsec.Ring.PIPELINED, "free": nba_ipsec.Ring.FREE}
+ALL = {"pipelined": nba_ipsec.Ring.PIPELINED, "free": nba_ipsec.Ring.FREE, "roles": nba_ipsec.Ring.ROLES,
+       "persistent": nba_ipsec.Ring.PERSISTENT}
+forms = {f: ALL[f] for f in os.environ.get("FORMS", "pipelined,roles").split(",")}
+K = int(os.environ.get("RING_K", K))
 res = {f: {} for f in forms}
 for size in sizes:
     cfg = {64: 2, 1514: 3, "imix": 4}.get(size, 5)

@@ -1,0 +1,56 @@
+#!/usr/bin/env python
+"""Phase trace of the role-split ring (GPU; needs the NBA_ROLES_TRACE=1 build,
+`python tools/ring_ab.py build rtrace=NBA_ROLES_TRACE=1`, loaded through
+NBA_IPSEC_LIB): per batch, sequencer 0's phases (consumed wait, A = ranks,
+B = per-warp prefix, barrier among sequencers, C = per-SA bases, D = records
+out) and when lane CTA 0 started waiting for / received the batch's records;
+medians over batches 4..K-2 of each phase's duration and of the batch period.
+
+    NBA_IPSEC_LIB=build/variants/rtrace.so [NBA_IPSEC_ROLES_P=4] python tools/roles_trace.py [sizes...]"""
+import json
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec, shard  # noqa: E402
+
+K = 50
+out = {}
+for size in [x if x == "imix" else int(x) for x in sys.argv[1:]] or [64]:
+    cfg = {64: 2, 1514: 3, "imix": 4}.get(size, 5)
+    p, b = shard.rank_workload(cfg, 65536, size, 1024, 0, 1)
+    t = nba_ipsec.SATable(p, max_batch=65536)
+    d0 = device.to_device(b, "cuda")
+    R = device.ring_slot_count(b.in_len, b.n, torch.cuda.get_device_properties(0).L2_cache_size)
+    dbs = [d0] + [device.clone(d0) for _ in range(R - 1)]
+    ring = t.ring([(*d.args(), b.n) for d in dbs])
+    ring.set_form(nba_ipsec.Ring.ROLES)
+    ring.run_batches(2 * R)
+    ts = torch.zeros(K * 9 + 1, dtype=torch.int64, device="cuda")
+    ring.set_timestamps(ts)
+    ring.run_batches(K)
+    torch.cuda.synchronize()
+    v = ts.cpu().numpy().astype(np.int64)
+    ends = v[1:K + 1]
+    st = v[K + 1:].reshape(K, 8)
+    sl = slice(4, K - 1)
+    med = lambda a: round(float(np.median(a[sl])) / 1e3, 2)  # noqa: E731
+    out[str(size)] = {
+        "batch_period_us": med(np.diff(ends, prepend=ends[0])),
+        "seq_period_us": med(np.diff(st[:, 5], prepend=st[0, 5])),
+        "seq_A_ranks_incl_consumed_wait": med(st[:, 1] - st[:, 0]),
+        "seq_B_prefix": med(st[:, 2] - st[:, 1]),
+        "seq_barrier": med(st[:, 3] - st[:, 2]),
+        "seq_C_bases": med(st[:, 4] - st[:, 3]),
+        "seq_D_records": med(st[:, 5] - st[:, 4]),
+        "seq_idle_between": med(st[1:, 0] - st[:-1, 5]),
+        "lane0_wait_for_records": med(st[:, 7] - st[:, 6]),
+        "records_lead_over_lane0_us": med(st[:, 6] - st[:, 5]),
+        "first_batch_end_us": round(float(ends[0] - v[0]) / 1e3, 2),
+    }
+    ring.close()
+    t.close()
+print(json.dumps(out), flush=True)

@@ -1,12 +1,13 @@
 """Workloads for compute-sanitizer runs of the shipped kernels:
 
     compute-sanitizer --tool {memcheck,initcheck,racecheck,synccheck} \\
-        python tools/sanitize_cases.py {c1,c4,ring64,ring_small,inbound,inring,host}
+        python tools/sanitize_cases.py {c1,c4,ring64,roles,ring_small,inbound,inring,host}
 
 c1         BASELINE configs[0] (64 x 64 B, 1 SA) through process_batch (k_fused<1>)
 c4         configs[3] (IMIX, 65,536 packets, 1024 SAs) through process_batch
 ring64     the bench's ring: 2 full-size 64-B slots (65,536 packets, 1024 SAs),
-           3 batches in one run_batches (k_fused_ring_pipe)
+           3 batches in one run_batches (k_fused_ring_roles, then k_fused_ring_pipe)
+roles      a 3,000-packet 64 B / IMIX ring in the role-split form, runs of 5 and 3
 ring_small a 3,000-packet 64 B / IMIX ring in both persistent forms
 inbound    ESP inbound of an IMIX batch (k_in_fused<1>) with replays and a forgery
 inring     the software-pipelined inbound ring (k_in_fused_ring_pipe), 3 slots, runs of 3 and 6
@@ -65,7 +66,14 @@ def main():
         ok = outbound(p, [b])
     elif case == "ring64":
         p, b = shard.rank_workload(2, 65536, 64, 1024, 0, 1)
-        ok = outbound(p, [b, gen.make_batch(65536, 64, 1024, cfg_id=2, batch=1)], ring=True, runs=(3,))
+        bs = [b, gen.make_batch(65536, 64, 1024, cfg_id=2, batch=1)]
+        ok = outbound(p, bs, ring=True, runs=(3,))                               # role-split (default)
+        ok &= outbound(p, bs, ring=True, runs=(3,), form=nba_ipsec.Ring.PIPELINED)
+    elif case == "roles":           # role-split ring, mixed lengths, runs past the record ring
+        p = gen.make_sas(16, cfg_id=9)
+        bs = [gen.make_batch(3000, sz, 16, cfg_id=9, batch=k) for k, sz in enumerate((64, "imix"))]
+        bs[1].sa_idx[::53] = 99
+        ok = outbound(p, bs, ring=True, runs=(5, 3), form=nba_ipsec.Ring.ROLES)
     elif case == "ring_small":
         p = gen.make_sas(16, cfg_id=7)
         bs = [gen.make_batch(3000, sz, 16, cfg_id=7, batch=k) for k, sz in enumerate((64, "imix"))]
