@@ -50,6 +50,10 @@ for size in [x if x == "imix" else int(x) for x in sys.argv[1:]] or [64]:
         "lane0_wait_for_records": med(st[:, 7] - st[:, 6]),
         "records_lead_over_lane0_us": med(st[:, 6] - st[:, 5]),
         "first_batch_end_us": round(float(ends[0] - v[0]) / 1e3, 2),
+        # batches 0..2 from the kernel start: sequencer 0's stamps (phase start, A, B,
+        # barrier, C, D/published), lane CTA 0's wait start / records seen, batch end
+        "start_batches_0_2_us": [[round(float(x - v[0]) / 1e3, 2) for x in list(st[b]) + [ends[b]]]
+                                 for b in range(3)],
     }
     ring.close()
     t.close()
