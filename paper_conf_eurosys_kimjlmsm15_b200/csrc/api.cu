@@ -493,8 +493,7 @@ int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, u
                 if (cudaMalloc(&r->rq.ctl, ROLES_CTL_WORDS * sizeof(uint32_t)) != cudaSuccess ||
                     cudaMemset(r->rq.ctl, 0, ROLES_CTL_WORDS * sizeof(uint32_t)) != cudaSuccess ||
                     cudaMalloc(&r->rq.rec, (size_t)ROLES_NREC * Lc * 512u * sizeof(uint32_t)) != cudaSuccess ||
-                    cudaMalloc(&r->rq.ptot, (size_t)2u * npro * t->n_sa * sizeof(uint32_t)) != cudaSuccess ||
-                    cudaMalloc(&r->rq.scratch, (size_t)Lc * 256u) != cudaSuccess) {
+                    cudaMalloc(&r->rq.ptot, (size_t)2u * npro * t->n_sa * sizeof(uint32_t)) != cudaSuccess) {
                     nba_ipsec_ring_destroy(r);
                     return NBA_IPSEC_ENOMEM;
                 }
@@ -791,7 +790,7 @@ int nba_ipsec_ring_destroy(nba_ipsec_ring *r)
         if (r->graph) cudaGraphDestroy(r->graph);
         if (r->d_slots || r->hist_b || r->d_in_slots || r->hkey_b || r->hval_b || r->rq.ctl)
             cudaDeviceSynchronize();   // a run may still be in flight
-        for (void *q : {(void *)r->rq.ctl, (void *)r->rq.rec, (void *)r->rq.ptot, (void *)r->rq.scratch})
+        for (void *q : {(void *)r->rq.ctl, (void *)r->rq.rec, (void *)r->rq.ptot})
             if (q) cudaFree(q);
         if (r->d_slots) cudaFree(r->d_slots);
         if (r->hist_b) cudaFree(r->hist_b);

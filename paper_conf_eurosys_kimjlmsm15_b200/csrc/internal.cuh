@@ -219,7 +219,6 @@ struct RolesBufs {
     uint32_t *ctl;      // [ROLES_CTL_WORDS] hand-off counters (zero between launches)
     uint32_t *rec;      // [ROLES_NREC][(grid - npro) * 512] per-packet sequence numbers (0: drop)
     uint32_t *ptot;     // [2][npro][n_sa] per-sequencer per-SA valid-packet totals
-    uint8_t *scratch;   // [(grid - npro) * 256] the lanes' warm-up output lines
     uint32_t npro;      // sequencer CTAs
 };
 bool fused_roles_ok(uint32_t n, uint32_t n_sa, int grid, uint32_t npro);

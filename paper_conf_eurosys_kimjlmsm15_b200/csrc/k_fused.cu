@@ -1946,9 +1946,6 @@ __device__ __forceinline__ void roles_lane_consumed(uint32_t *p, uint32_t q)
 #if NBA_ROLES_TRACE
 #define RLT(bi, k) (R.ts + 1u + R.n_batches + (size_t)(bi) * 8u + (k))
 #endif
-#ifndef NBA_ROLES_WARM        // lanes: one dummy packet through the lane code while batch 0 is sequenced
-#define NBA_ROLES_WARM 0      //   (measured: batch 0 then runs at steady speed, 22.4 us, but the cold
-#endif                        //   dummy pass takes ~33 us against ~21 us of sequencing: a wash)
 #ifndef NBA_ROLES_AG          // sequencer: rounds of 32 packets whose metadata loads are in flight together
 #define NBA_ROLES_AG 8
 #endif
@@ -2137,6 +2134,17 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
     FusedLo &L = *reinterpret_cast<FusedLo *>(smem + lo_off);
     FusedHi &H = *reinterpret_cast<FusedHi *>(smem + toff + AES_TABLE_BYTES);
     const uint32_t lane4r = (lane * 4u) | (smem_u32(tabs) & 0xffff0000u);
+    // the ring's slot table in shared memory (the per-packet arrays L.sa ..
+    // L.aux1 are free in this form): a slot's arguments are read at every
+    // batch, and from global memory that load sat on the lanes' critical path
+    constexpr uint32_t SLOT_CACHE = (uint32_t)((7u * F_SUPER * sizeof(uint32_t)) / sizeof(BatchArgs));
+    static_assert(sizeof(BatchArgs) % 4 == 0, "slot copy by words");
+    BatchArgs *sc = reinterpret_cast<BatchArgs *>(&L.sa[0]);
+    const bool cached = R.n_slots <= SLOT_CACHE;
+    if (cached)
+        for (uint32_t k = tid; k < R.n_slots * (uint32_t)(sizeof(BatchArgs) / 4); k += F_THREADS)
+            reinterpret_cast<uint32_t *>(sc)[k] = reinterpret_cast<const uint32_t *>(slots)[k];
+    const BatchArgs *sl = cached ? sc : slots;
     tables_stage(tabs, T, &L.tbar, true);
     __syncthreads();
     tables_bulk_wait(&L.tbar, 0u);
@@ -2146,16 +2154,16 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
     unsigned long long c_ok = 0, c_drop = 0, c_in = 0, c_out = 0;
     // The lane's packet fields (batch inputs: SA, length, offsets) are known
     // before its record (the sequence number): loaded one batch ahead, so that
-    // the SA line load and the round-key expansion run before the record wait.
-    // Its payload's first line goes into L2 one batch ahead too.
+    // the SA line load and the round-key expansion run before the record is
+    // needed.  Its payload's first line goes into L2 one batch ahead too.
     struct Fields { uint32_t i, sa, D, inoff, outoff; bool have; };
     auto fields_of = [&](uint32_t bi) {
         Fields f = {0u, INVALID_SA, 0u, 0u, 0u, false};
         if (bi >= R.n_batches) return f;
-        const BatchArgs B = slots[(R.first + bi) % R.n_slots];
-        const uint32_t ppc = (B.n + Lc - 1u) / Lc;
+        const BatchArgs &B = sl[(R.first + bi) % R.n_slots];
+        const uint32_t n = B.n, ppc = (n + Lc - 1u) / Lc;
         f.i = c * ppc + jpos;
-        f.have = jpos < ppc && f.i < B.n;
+        f.have = jpos < ppc && f.i < n;
         if (f.have) {
             f.sa = B.sa_idx[f.i];
             f.D = B.in_len[f.i];
@@ -2164,35 +2172,26 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
         }
         return f;
     };
-    // Iteration -1 (NBA_ROLES_WARM): while the sequencers prepare batch 0, each
-    // lane runs its batch-0 packet's code path once on a dummy packet (SA 0,
-    // the same length up to 114 bytes, read from the T-table image, written to
-    // a per-CTA scratch line) through the SAME call sites: the first pass over
-    // the lane code is ~2x slower than the next ones (every lane alike,
-    // tools/ring_ab.py trace), and here it overlaps the sequencers' batch 0.
+    auto candidate = [&](const Fields &g) {   // the oracle's step 1 (A15)
+        return g.have && g.sa < n_sa && g.D >= MIN_D && g.D <= MAX_D;
+    };
     Fields f = fields_of(0u);
-    BatchArgs Bw = slots[R.first % R.n_slots];
-    if (NBA_ROLES_WARM) {
-        Bw.in_buf = reinterpret_cast<const uint8_t *>(T.timg);
-        Bw.out_buf = Q.scratch + (size_t)c * 256u;
-        f = Fields{0u, 0u, f.have ? min(max(f.D, MIN_D), 114u) : 50u, 0u, 14u, true};
-    } else if (f.have) {
-        prefetch_l2(slots[R.first % R.n_slots].in_buf + f.inoff);
-    }
-    for (int32_t bs = NBA_ROLES_WARM ? -1 : 0; bs < (int32_t)R.n_batches; bs++) {
-        const bool dummy = bs < 0;
-        const uint32_t bi = dummy ? 0u : (uint32_t)bs;
-        const BatchArgs B = dummy ? Bw : slots[(R.first + bi) % R.n_slots];
-        const Fields fn = fields_of(dummy ? 0u : bi + 1u);
-        // the oracle's step 1 (A15): invalid SA or length -> drop, no number used
-        const bool cand = f.have && f.sa < n_sa && f.D >= MIN_D && f.D <= MAX_D;
+    if (f.have) prefetch_l2(sl[R.first % R.n_slots].in_buf + f.inoff);
+    // batch bi's record when it was read ahead (at the end of iteration bi - 1,
+    // from a poll issued during it): neither the poll nor the record load then
+    // waits on the critical path
+    uint32_t q = 0u, rv_next = 0u;
+    bool got = false;
+    for (uint32_t bi = 0; bi < R.n_batches; bi++) {
+        const BatchArgs &B = sl[(R.first + bi) % R.n_slots];
+        const Fields fn = fields_of(bi + 1u);
+        const bool cand = candidate(f);
         PktPre pp = {};
         if (cand) {
             pp = load_pkt_pre(T, B.in_buf, f.sa, f.inoff, true, 0u);
             expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
         }
-        uint32_t q = 1u;
-        if (!dummy) {
+        if (!got) {
 #if NBA_ROLES_TRACE
             if (R.ts && c == 0 && tid == 0) *RLT(bi, 6) = gtimer();
 #endif
@@ -2201,26 +2200,35 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
             if (R.ts && c == 0 && tid == 0) *RLT(bi, 7) = gtimer();
 #endif
             q = cand ? __ldcg(&Q.rec[(size_t)(bi % ROLES_NREC) * Lc * 512u + f.i]) : 0u;
-            roles_lane_consumed(&consumed[bi % ROLES_NREC], q);
         }
+        roles_lane_consumed(&consumed[bi % ROLES_NREC], q);
+        if (lane == 0 && bi + 1u < R.n_batches) rv_next = roles_ld_relaxed(&ready[(bi + 1u) % ROLES_NREC]);
         if (f.have) {
             if (q != 0u) {
                 esp_packet(T, B, L, H, lane4r, tid, f.sa, f.D | INFO_OK, q, f.inoff, f.outoff, pp, nullptr);
-                if (!dummy) {
-                    const uint32_t Lp = 48u + esp_C(f.D);
-                    B.out_len[f.i] = (uint16_t)Lp;
-                    c_ok++;
-                    c_in += f.D;
-                    c_out += Lp;
-                }
+                const uint32_t Lp = 48u + esp_C(f.D);
+                B.out_len[f.i] = (uint16_t)Lp;
+                c_ok++;
+                c_in += f.D;
+                c_out += Lp;
             } else {
                 B.out_len[f.i] = 0;
                 c_drop++;
             }
         }
         // the next packet's payload line into L2 (its offset has arrived by now)
-        if (fn.have) prefetch_l2(slots[(R.first + (dummy ? 0u : bi + 1u)) % R.n_slots].in_buf + fn.inoff);
-        if (!dummy && R.ts && lane == 0) atomicMax(&R.ts[1u + bi], gtimer());
+        if (fn.have) prefetch_l2(sl[(R.first + bi + 1u) % R.n_slots].in_buf + fn.inoff);
+        if (R.ts && lane == 0) atomicMax(&R.ts[1u + bi], gtimer());
+        // the next batch's record, if its sequencers had published it when
+        // lane 0's poll (issued above) read the count
+        got = false;
+        if (bi + 1u < R.n_batches) {
+            const uint32_t rv = __shfl_sync(0xffffffffu, rv_next, 0);
+            if ((int32_t)(rv - ((bi + 1u) / ROLES_NREC + 1u) * P) >= 0) {
+                q = candidate(fn) ? __ldcg(&Q.rec[(size_t)((bi + 1u) % ROLES_NREC) * Lc * 512u + fn.i]) : 0u;
+                got = true;
+            }
+        }
         f = fn;
     }
     if (tid < 4) L.cnt[tid] = 0ull;
