@@ -459,12 +459,14 @@ int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, u
         // role-split form: sequencer CTAs + lane CTAs (every slot with SA indices,
         // <= 512 packets per lane CTA, n_sa <= ROLES_MAX_SA).  The default for
         // rings whose every slot holds packets of one length up to 1010 bytes
-        // (1024-B frames): measured per 65,536-packet batch against the
-        // pipelined form (tools/ring_forms.py, K = 200) 64 B 21.1 vs 21.9 us,
-        // 128 B 28.2 vs 32.7, 256 B 43.3 vs 47.3, 512 B 73.7 vs 76.4, 1024 B
-        // 132.9 vs 133.8, 1514 B 190.7 vs 189.0.  Sequencers: 6 for packets of
-        // <= 114 bytes (the 64-B batch needs them to keep ahead of the lanes),
-        // else 4 (NBA_IPSEC_ROLES_P overrides; NBA_IPSEC_RING_ROLES=0/1 forces).
+        // (1024-B frames) and for mixed-length rings of more than ROLES_NREC
+        // slots (sorted mode): measured per 65,536-packet batch against the
+        // pipelined form (tools/ring_forms.py, K = 200) 64 B 20.4 vs 22.2 us,
+        // 128 B 28.9 vs 33.1, 256 B 43.2 vs 47.4, 512 B 74.2 vs 76.5, 1024 B
+        // 132.9 vs 133.8, 1514 B 190.7 vs 189.0, IMIX (sorted) 69.2 vs 88.2.
+        // Sequencers: 6 for packets of <= 114 bytes and mixed rings (the
+        // sequencers must keep ahead of the lanes), else 4 (NBA_IPSEC_ROLES_P
+        // overrides; NBA_IPSEC_RING_ROLES=0/1 forces the form).
         {
             bool one_len = true, idx = true;
             uint32_t max_len = 0;
@@ -483,7 +485,8 @@ int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, u
                 }
             }
             const char *pe = std::getenv("NBA_IPSEC_ROLES_P");
-            const uint32_t npro = pe ? (uint32_t)std::max(1, std::atoi(pe)) : (max_len <= 114u ? 6u : 4u);
+            const uint32_t npro = pe ? (uint32_t)std::max(1, std::atoi(pe))
+                                     : (max_len <= 114u || !one_len ? 6u : 4u);
             r->roles_ok = idx;
             for (uint32_t i = 0; i < n_slots && r->roles_ok; i++)
                 r->roles_ok = fused_roles_ok(slots[i].n_pkts, t->n_sa, t->grid_fused, npro);
@@ -492,13 +495,21 @@ int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, u
                 r->rq.npro = npro;
                 if (cudaMalloc(&r->rq.ctl, ROLES_CTL_WORDS * sizeof(uint32_t)) != cudaSuccess ||
                     cudaMemset(r->rq.ctl, 0, ROLES_CTL_WORDS * sizeof(uint32_t)) != cudaSuccess ||
-                    cudaMalloc(&r->rq.rec, (size_t)ROLES_NREC * Lc * 512u * sizeof(uint32_t)) != cudaSuccess ||
-                    cudaMalloc(&r->rq.ptot, (size_t)2u * npro * t->n_sa * sizeof(uint32_t)) != cudaSuccess) {
+                    cudaMalloc(&r->rq.rec, (size_t)ROLES_NREC * Lc * 512u * sizeof(uint2)) != cudaSuccess ||
+                    cudaMalloc(&r->rq.cum, (size_t)Lc * 16u * sizeof(uint32_t)) != cudaSuccess ||
+                    cudaMemset(r->rq.cum, 0, (size_t)Lc * 16u * sizeof(uint32_t)) != cudaSuccess ||
+                    cudaMalloc(&r->rq.ptot, (size_t)2u * npro * t->n_sa * sizeof(uint32_t)) != cudaSuccess ||
+                    cudaMalloc(&r->rq.scratch, (size_t)Lc * 256u) != cudaSuccess) {
                     nba_ipsec_ring_destroy(r);
                     return NBA_IPSEC_ENOMEM;
                 }
+                // mixed lengths: per-batch length-sorted lane slots (a packet slot may
+                // change lanes between uses of a ring slot: needs n_slots > ROLES_NREC)
+                r->rq.sorted = (!one_len && n_slots > ROLES_NREC) ? 1u : 0u;
+                const char *rs = std::getenv("NBA_IPSEC_ROLES_SORTED");
+                if (rs) r->rq.sorted = (std::atoi(rs) != 0 && n_slots > ROLES_NREC) ? 1u : 0u;
                 const char *re = std::getenv("NBA_IPSEC_RING_ROLES");
-                r->roles = re ? std::atoi(re) != 0 : (one_len && max_len <= 1010u);
+                r->roles = re ? std::atoi(re) != 0 : ((one_len && max_len <= 1010u) || r->rq.sorted);
             }
         }
         std::vector<BatchArgs> hb(n_slots);
@@ -790,7 +801,8 @@ int nba_ipsec_ring_destroy(nba_ipsec_ring *r)
         if (r->graph) cudaGraphDestroy(r->graph);
         if (r->d_slots || r->hist_b || r->d_in_slots || r->hkey_b || r->hval_b || r->rq.ctl)
             cudaDeviceSynchronize();   // a run may still be in flight
-        for (void *q : {(void *)r->rq.ctl, (void *)r->rq.rec, (void *)r->rq.ptot})
+        for (void *q : {(void *)r->rq.ctl, (void *)r->rq.rec, (void *)r->rq.ptot, (void *)r->rq.scratch,
+                        (void *)r->rq.cum})
             if (q) cudaFree(q);
         if (r->d_slots) cudaFree(r->d_slots);
         if (r->hist_b) cudaFree(r->hist_b);

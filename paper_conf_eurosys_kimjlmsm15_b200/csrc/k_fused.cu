@@ -1946,9 +1946,96 @@ __device__ __forceinline__ void roles_lane_consumed(uint32_t *p, uint32_t q)
 #if NBA_ROLES_TRACE
 #define RLT(bi, k) (R.ts + 1u + R.n_batches + (size_t)(bi) * 8u + (k))
 #endif
+#ifndef NBA_ROLES_WARM        // experiment: lanes' warm-up pass (0 off, 1 all warps, 2 warp 0, 3 warps 0-3)
+#define NBA_ROLES_WARM 0
+#endif
+#ifndef NBA_ROLES_RK_ASYNC    // lanes: round keys 3..10 by cp.async from the SA's schedule instead of
+#define NBA_ROLES_RK_ASYNC 0  //   expanded from the key (1)
+#endif
 #ifndef NBA_ROLES_AG          // sequencer: rounds of 32 packets whose metadata loads are in flight together
 #define NBA_ROLES_AG 8
 #endif
+
+// Sorted mode (mixed-length rings), per lane CTA of this sequencer, one warp
+// each: the CTA's packets in a stable counting sort by HMAC length bin
+// (longest first, invalid last), cut into runs of 32 sorted positions; run r
+// goes to the lane warp with the least work assigned so far (LPT over the
+// warps' cumulative cost, Q.cum, so the long runs rotate among the warps from
+// batch to batch); d16[packet] becomes the packet's lane slot (warp * 32 +
+// position in the run).  Slots left without a packet get the record
+// {0, 0xffffffff}.  A run's cost: 8 (SHA-1 blocks + 1) + 3 AES steps of its
+// first (longest) packet, ~11 x inner SHA-1 blocks + 8.
+__device__ __noinline__ void roles_sort_slots(uint2 *rec, uint32_t *cumb, uint16_t *d16, const uint16_t *sa16,
+                                              uint32_t (*hw)[NBINS], uint32_t r0, uint32_t n,
+                                              uint32_t ppc, uint32_t cbeg, uint32_t cend)
+{
+    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+    for (uint32_t cc = cbeg + warp; cc < cend; cc += 16u) {
+        const uint32_t pb = min(n, cc * ppc), pe = min(n, pb + ppc), cnt = pe - pb;
+        auto bin_of = [&](uint32_t i) {
+            const bool ok = sa16[i - r0] != 0xffffu;
+            return hmac_bin(ok, esp_C(d16[i - r0]));
+        };
+        hw[warp][lane] = 0u;
+        __syncwarp();
+        for (uint32_t g = pb; g < pe; g += 32u)
+            warp_agg_add(hw[warp], g + lane < pe ? bin_of(g + lane) : 0u, g + lane < pe);
+        __syncwarp();
+        const uint32_t cb = hw[warp][lane];           // lane = bin: count, exclusive prefix
+        uint32_t x = cb;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+            if (lane >= (uint32_t)o) x += y;
+        }
+        const uint32_t base = x - cb;
+        hw[warp][lane] = base;
+        // runs: the bin of each run's first position, its cost; LPT onto the warps
+        const uint32_t nruns = (cnt + 31u) / 32u;
+        uint32_t binr = NBINS - 1u;
+        for (uint32_t b = 0; b < (uint32_t)NBINS; b++) {
+            const uint32_t bb = __shfl_sync(0xffffffffu, base, b), cbb = __shfl_sync(0xffffffffu, cb, b);
+            if (cbb > 0u && bb <= 32u * lane) binr = b;      // the last such bin holds position 32 lane
+        }
+        const uint32_t cost = binr == NBINS - 1u ? 1u : 11u * (NBINS - 1u - binr) + 8u;
+        uint32_t cum = lane < 16u ? cumb[cc * 16u + lane] : 0xffffffffu;
+        uint32_t wsl = 0xffu;                          // lane r: warp of run r
+        bool taken = lane >= 16u;                      // lane w: warp w holds a run of this batch
+        for (uint32_t r = 0; r < nruns; r++) {         // (nruns <= 16: one run per warp)
+            const uint32_t cr = __shfl_sync(0xffffffffu, cost, r);
+            const uint32_t v = __reduce_min_sync(0xffffffffu, taken ? 0xffffffffu
+                                                                    : (min(cum, 0x7ffffffu) << 5) | lane);
+            const uint32_t w = v & 31u;
+            if (lane == w) {
+                cum += cr;
+                taken = true;
+            }
+            if (lane == r) wsl = w;
+        }
+        const uint32_t m = __reduce_min_sync(0xffffffffu, lane < 16u ? cum : 0xffffffffu);
+        if (lane < 16u) cumb[cc * 16u + lane] = cum - m;   // (kept small)
+        // the run each warp holds (lane w: run or 0xffffffff)
+        uint32_t myrun = 0xffffffffu;
+        for (uint32_t r = 0; r < nruns; r++)
+            if (__shfl_sync(0xffffffffu, wsl, r) == lane) myrun = r;
+        __syncwarp();
+        // stable scatter: position = bin base + rank among the earlier packets of its bin
+        for (uint32_t g = pb; g < pe; g += 32u) {
+            const uint32_t i = g + lane;
+            const bool in = i < pe;
+            const uint32_t pos = warp_agg_add(hw[warp], in ? bin_of(i) : 0u, in);
+            const uint32_t w = __shfl_sync(0xffffffffu, wsl, in ? (pos >> 5) : 0u);
+            if (in) d16[i - r0] = (uint16_t)(w * 32u + (pos & 31u));
+        }
+        // slots without a packet
+        for (uint32_t sl = lane; sl < 512u; sl += 32u) {
+            const uint32_t r = __shfl_sync(0xffffffffu, myrun, sl >> 5);
+            if (r == 0xffffffffu || 32u * r + (sl & 31u) >= cnt)
+                rec[(size_t)cc * 512u + sl] = make_uint2(0u, 0xffffffffu);
+        }
+        __syncwarp();
+    }
+}
 
 __device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchArgs *slots, const RingRun &R,
                                                 const RolesBufs &Q, uint8_t *smem, uint32_t p)
@@ -1962,22 +2049,27 @@ __device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchAr
     uint16_t *cnt = d16 + ROLES_RPP_MAX;                           // [16][ROLES_MAX_SA]
     uint32_t *seqs = reinterpret_cast<uint32_t *>(cnt + 16u * ROLES_MAX_SA);   // [ROLES_MAX_SA]
     unsigned long long *start = reinterpret_cast<unsigned long long *>(seqs + ROLES_MAX_SA);
+    uint32_t (*sorth)[NBINS] = reinterpret_cast<uint32_t (*)[NBINS]>(start + ROLES_MAX_SA);   // [16][NBINS]
+    static_assert(3u * ROLES_RPP_MAX * 2u + 16u * ROLES_MAX_SA * 2u + ROLES_MAX_SA * 12u + 16u * NBINS * 4u
+                      <= F_SMEM, "sequencer shared memory");
     uint32_t *ready = Q.ctl, *consumed = Q.ctl + ROLES_NREC, *pbar = Q.ctl + 2u * ROLES_NREC;
     uint16_t *mycnt = cnt + warp * ROLES_MAX_SA;
     for (uint32_t s = tid; s < n_sa; s += F_THREADS) seqs[s] = __ldcg(&T.seq[s]);
     for (uint32_t s = lane; s < n_sa; s += 32u) mycnt[s] = 0;
     __syncthreads();
+    // this sequencer's lane CTAs [cbeg, cend): its packet range is theirs
+    const uint32_t cbeg = p * Lc / P, cend = (p + 1u) * Lc / P;
     for (uint32_t bi = 0; bi < R.n_batches; bi++) {
         const BatchArgs B = slots[(R.first + bi) % R.n_slots];
-        const uint32_t n = B.n, rpp = (n + P - 1u) / P;
-        const uint32_t r0 = min(n, p * rpp), r1 = min(n, r0 + rpp);
+        const uint32_t n = B.n, ppc = (n + Lc - 1u) / Lc;
+        const uint32_t r0 = min(n, cbeg * ppc), r1 = min(n, cend * ppc), rpp = r1 - r0;
         const uint32_t spw = (((rpp + 15u) / 16u) + 31u) & ~31u;   // whole rounds per warp
         const uint32_t w0 = min(r1, r0 + warp * spw), w1 = min(r1, w0 + spw);
         // the next batch's metadata lines into L2 (ahead of its phase A; batch 0's
         // at the start)
         for (uint32_t nb = bi == 0u ? 0u : bi + 1u; nb <= bi + 1u && nb < R.n_batches; nb++) {
             const BatchArgs Bn = slots[(R.first + nb) % R.n_slots];
-            const uint32_t rn = (Bn.n + P - 1u) / P, a0 = min(Bn.n, p * rn), a1 = min(Bn.n, a0 + rn);
+            const uint32_t pn = (Bn.n + Lc - 1u) / Lc, a0 = min(Bn.n, cbeg * pn), a1 = min(Bn.n, cend * pn);
             const uint32_t l16 = a1 > a0 ? (2u * (a1 - a0) + 127u) / 128u + 1u : 0u;
             const uint32_t l32 = a1 > a0 ? (4u * (a1 - a0) + 127u) / 128u + 1u : 0u;
             for (uint32_t k = tid; k < l16 + l32; k += F_THREADS) {   // in_len, sa_idx
@@ -2041,6 +2133,9 @@ __device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchAr
             }
         }
         __syncthreads();
+        if (Q.sorted)
+            roles_sort_slots(reinterpret_cast<uint2 *>(Q.rec) + (size_t)(bi % ROLES_NREC) * Lc * 512u, Q.cum,
+                             d16, sa16, sorth, r0, n, ppc, cbeg, cend);
 #if NBA_ROLES_TRACE
         if (R.ts && p == 0 && tid == 0) *RLT(bi, 1) = gtimer();
 #endif
@@ -2087,8 +2182,9 @@ __device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchAr
 #if NBA_ROLES_TRACE
         if (R.ts && p == 0 && tid == 0) *RLT(bi, 4) = gtimer();
 #endif
-        // D. the records (the sequence number, 0 = drop), by packet index
-        uint32_t *rec = Q.rec + (size_t)(bi % ROLES_NREC) * Lc * 512u;
+        // D. the records (the sequence number, 0 = drop): by packet index, or
+        //    (sorted mode) {q, packet} at the packet's lane slot
+        uint32_t *rec = Q.rec + (size_t)(bi % ROLES_NREC) * Lc * 512u * (Q.sorted ? 2u : 1u);
 #pragma unroll 4
         for (uint32_t g0 = w0; g0 < w1; g0 += 32u) {
             const uint32_t i = g0 + lane;
@@ -2100,7 +2196,13 @@ __device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchAr
                         start[s] + mycnt[s] + (unsigned long long)rank[i - r0] + 1ull;
                     r = q <= 0xffffffffull ? (uint32_t)q : 0u;
                 }
-                rec[i] = r;
+                if (Q.sorted) {
+                    const uint32_t c = i / ppc;
+                    reinterpret_cast<uint2 *>(rec)[(size_t)c * 512u + d16[i - r0]] = make_uint2(r, i - c * ppc);
+                    if (s != 0xffffu) prefetch_l2(B.in_buf + B.in_off[i]);   // its payload's first line
+                } else {
+                    rec[i] = r;
+                }
             }
         }
         __syncwarp();
@@ -2116,6 +2218,26 @@ __device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchAr
     }
     if (p == 0)
         for (uint32_t s = tid; s < n_sa; s += F_THREADS) T.seq[s] = seqs[s];
+}
+
+// A lane CTA's counters into the device counters (as fused_body).
+__device__ __forceinline__ void roles_lane_counters(const DevWork &W, FusedLo &L, unsigned long long c_ok,
+                                                    unsigned long long c_drop, unsigned long long c_in,
+                                                    unsigned long long c_out)
+{
+    const uint32_t tid = threadIdx.x, lane = tid & 31u;
+    if (tid < 4) L.cnt[tid] = 0ull;
+    __syncthreads();
+    const unsigned long long s0 = warp_sum_u64(c_ok), s1 = warp_sum_u64(c_drop);
+    const unsigned long long s2 = warp_sum_u64(c_in), s3 = warp_sum_u64(c_out);
+    if (lane == 0) {
+        if (s0) atomicAdd(&L.cnt[0], s0);
+        if (s1) atomicAdd(&L.cnt[1], s1);
+        if (s2) atomicAdd(&L.cnt[2], s2);
+        if (s3) atomicAdd(&L.cnt[3], s3);
+    }
+    __syncthreads();
+    if (tid < 4 && L.cnt[tid]) atomicAdd(&W.counters[tid], L.cnt[tid]);
 }
 
 __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W, const BatchArgs *slots,
@@ -2176,22 +2298,52 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
         return g.have && g.sa < n_sa && g.D >= MIN_D && g.D <= MAX_D;
     };
     Fields f = fields_of(0u);
-    if (f.have) prefetch_l2(sl[R.first % R.n_slots].in_buf + f.inoff);
+    const Fields f0 = f;
+    // experiment (NBA_ROLES_WARM 1 / 2 / 3: all warps / warp 0 / warps 0-3 of
+    // each lane CTA): iteration -1 runs the batch-0 code path on a dummy packet
+    // (SA 0, the lane's length up to 114 bytes, read from the T-table image,
+    // written to a per-CTA scratch line) through the same call sites, during
+    // the sequencers' batch 0 -- the first pass over the lane code in a launch
+    // is ~1.5x slower than the next ones
+    const bool warm_me = cached && R.n_slots < SLOT_CACHE &&
+                         (NBA_ROLES_WARM == 1 || (NBA_ROLES_WARM == 2 && warp == 0) ||
+                          (NBA_ROLES_WARM == 3 && warp < 4u));
+    if (NBA_ROLES_WARM && cached && R.n_slots < SLOT_CACHE && tid == 0) {
+        BatchArgs bw = sl[R.first % R.n_slots];
+        bw.in_buf = reinterpret_cast<const uint8_t *>(T.timg);
+        bw.out_buf = Q.scratch + (size_t)c * 256u;
+        sc[R.n_slots] = bw;
+    }
+    if (NBA_ROLES_WARM) __syncthreads();
+    if (warm_me) f = Fields{0u, 0u, f.have ? min(max(f.D, MIN_D), 114u) : 50u, 0u, 14u, true};
+    else if (f.have) prefetch_l2(sl[R.first % R.n_slots].in_buf + f.inoff);
     // batch bi's record when it was read ahead (at the end of iteration bi - 1,
     // from a poll issued during it): neither the poll nor the record load then
     // waits on the critical path
     uint32_t q = 0u, rv_next = 0u;
     bool got = false;
-    for (uint32_t bi = 0; bi < R.n_batches; bi++) {
-        const BatchArgs &B = sl[(R.first + bi) % R.n_slots];
-        const Fields fn = fields_of(bi + 1u);
+    for (int32_t bs = warm_me ? -1 : 0; bs < (int32_t)R.n_batches; bs++) {
+        const bool dummy = bs < 0;
+        const uint32_t bi = dummy ? 0u : (uint32_t)bs;
+        const BatchArgs &B = dummy ? sc[R.n_slots] : sl[(R.first + bi) % R.n_slots];
+        const Fields fn = dummy ? f0 : fields_of(bi + 1u);
         const bool cand = candidate(f);
         PktPre pp = {};
         if (cand) {
-            pp = load_pkt_pre(T, B.in_buf, f.sa, f.inoff, true, 0u);
-            expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
+            if (NBA_ROLES_RK_ASYNC) {
+                // round keys 3..10 copied from the SA's schedule (cp.async into the
+                // lane's own slots), 1..2 from its SA line: no expansion chain
+                rk_async_issue(T.rk, f.sa, L, H, tid);
+                pp = load_pkt_pre(T, B.in_buf, f.sa, f.inoff, true, 0u);
+                ldg_nc_v8(&T.sal[(size_t)f.sa * SAL_U4 + 6], pp.r1, pp.r2);
+            } else {
+                pp = load_pkt_pre(T, B.in_buf, f.sa, f.inoff, true, 0u);
+                expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
+            }
         }
-        if (!got) {
+        if (dummy) {
+            q = 1u;
+        } else if (!got) {
 #if NBA_ROLES_TRACE
             if (R.ts && c == 0 && tid == 0) *RLT(bi, 6) = gtimer();
 #endif
@@ -2201,11 +2353,18 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
 #endif
             q = cand ? __ldcg(&Q.rec[(size_t)(bi % ROLES_NREC) * Lc * 512u + f.i]) : 0u;
         }
-        roles_lane_consumed(&consumed[bi % ROLES_NREC], q);
-        if (lane == 0 && bi + 1u < R.n_batches) rv_next = roles_ld_relaxed(&ready[(bi + 1u) % ROLES_NREC]);
+        if (!dummy) roles_lane_consumed(&consumed[bi % ROLES_NREC], q);
+        if (!dummy && lane == 0 && bi + 1u < R.n_batches)
+            rv_next = roles_ld_relaxed(&ready[(bi + 1u) % ROLES_NREC]);
+        if (NBA_ROLES_RK_ASYNC && cand) rk_async_wait();
         if (f.have) {
             if (q != 0u) {
                 esp_packet(T, B, L, H, lane4r, tid, f.sa, f.D | INFO_OK, q, f.inoff, f.outoff, pp, nullptr);
+                if (dummy) {
+                    f = fn;
+                    if (f.have) prefetch_l2(sl[R.first % R.n_slots].in_buf + f.inoff);
+                    continue;
+                }
                 const uint32_t Lp = 48u + esp_C(f.D);
                 B.out_len[f.i] = (uint16_t)Lp;
                 c_ok++;
@@ -2231,18 +2390,98 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
         }
         f = fn;
     }
-    if (tid < 4) L.cnt[tid] = 0ull;
-    __syncthreads();
-    const unsigned long long s0 = warp_sum_u64(c_ok), s1 = warp_sum_u64(c_drop);
-    const unsigned long long s2 = warp_sum_u64(c_in), s3 = warp_sum_u64(c_out);
-    if (lane == 0) {
-        if (s0) atomicAdd(&L.cnt[0], s0);
-        if (s1) atomicAdd(&L.cnt[1], s1);
-        if (s2) atomicAdd(&L.cnt[2], s2);
-        if (s3) atomicAdd(&L.cnt[3], s3);
+    roles_lane_counters(W, L, c_ok, c_drop, c_in, c_out);
+}
+
+// Lane CTA, sorted mode (mixed-length rings): the record at the thread's own
+// lane slot names its packet {q, packet in the CTA's range} -- the packet's
+// fields are read after the record -- and a fence precedes the "consumed"
+// count: a packet slot may go to a different lane in a later batch of the
+// same ring slot, so this warp's earlier output stores must be visible before
+// the sequencers can publish a batch that reuses them (ring_create takes this
+// mode only with n_slots > ROLES_NREC: that batch is at least NREC + 1 later).
+__device__ __forceinline__ void roles_lanes_sorted(const DevTable &T, const DevWork &W, const BatchArgs *slots,
+                                                   const RingRun &R, const RolesBufs &Q, uint8_t *smem,
+                                                   uint32_t c)
+{
+    const uint32_t tid = threadIdx.x, lane = tid & 31u;
+    const uint32_t P = Q.npro, Lc = gridDim.x - P, n_sa = T.n_sa;
+    const uint32_t sb = smem_u32(smem);
+    const uint32_t toff = (0x10000u - (sb & 0xffffu)) & 0xffffu;
+    uint32_t lo_off = 0;
+    if (toff < sizeof(FusedLo)) {
+        if (toff + AES_TABLE_BYTES + sizeof(FusedHi) + sizeof(FusedLo) > F_SMEM) __trap();
+        lo_off = toff + AES_TABLE_BYTES + (uint32_t)sizeof(FusedHi);
     }
+    uint8_t *tabs = smem + toff;
+    FusedLo &L = *reinterpret_cast<FusedLo *>(smem + lo_off);
+    FusedHi &H = *reinterpret_cast<FusedHi *>(smem + toff + AES_TABLE_BYTES);
+    const uint32_t lane4r = (lane * 4u) | (smem_u32(tabs) & 0xffff0000u);
+    constexpr uint32_t SLOT_CACHE = (uint32_t)((7u * F_SUPER * sizeof(uint32_t)) / sizeof(BatchArgs));
+    BatchArgs *sc = reinterpret_cast<BatchArgs *>(&L.sa[0]);
+    const bool cached = R.n_slots <= SLOT_CACHE;
+    if (cached)
+        for (uint32_t k = tid; k < R.n_slots * (uint32_t)(sizeof(BatchArgs) / 4); k += F_THREADS)
+            reinterpret_cast<uint32_t *>(sc)[k] = reinterpret_cast<const uint32_t *>(slots)[k];
+    const BatchArgs *sl = cached ? sc : slots;
+    tables_stage(tabs, T, &L.tbar, true);
     __syncthreads();
-    if (tid < 4 && L.cnt[tid]) atomicAdd(&W.counters[tid], L.cnt[tid]);
+    tables_bulk_wait(&L.tbar, 0u);
+    const uint32_t *ready = Q.ctl;
+    uint32_t *consumed = Q.ctl + ROLES_NREC;
+    const uint2 *rec = reinterpret_cast<const uint2 *>(Q.rec);
+    unsigned long long c_ok = 0, c_drop = 0, c_in = 0, c_out = 0;
+    uint2 r = make_uint2(0u, 0xffffffffu);
+    uint32_t rv_next = 0u;
+    bool got = false;
+    for (uint32_t bi = 0; bi < R.n_batches; bi++) {
+        const BatchArgs &B = sl[(R.first + bi) % R.n_slots];
+        if (!got) {
+            roles_lane_wait(&ready[bi % ROLES_NREC], (bi / ROLES_NREC + 1u) * P);
+            r = __ldcg(&rec[((size_t)(bi % ROLES_NREC) * Lc + c) * 512u + tid]);
+        }
+        const bool have = r.y != 0xffffffffu;
+        const uint32_t i = c * ((B.n + Lc - 1u) / Lc) + (have ? r.y : 0u);
+        uint32_t sa = INVALID_SA, D = 0u, inoff = 0u, outoff = 0u;
+        if (have) {
+            sa = B.sa_idx[i];
+            D = B.in_len[i];
+            inoff = B.in_off[i];
+            outoff = B.out_off[i];
+        }
+        const bool cand = have && sa < n_sa && D >= MIN_D && D <= MAX_D;
+        PktPre pp = {};
+        if (cand) {
+            pp = load_pkt_pre(T, B.in_buf, sa, inoff, true, 0u);
+            expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
+        }
+        __threadfence();                                // this warp's earlier outputs (see above)
+        roles_lane_consumed(&consumed[bi % ROLES_NREC], r.x);
+        if (lane == 0 && bi + 1u < R.n_batches) rv_next = roles_ld_relaxed(&ready[(bi + 1u) % ROLES_NREC]);
+        if (have) {
+            if (r.x != 0u) {
+                esp_packet(T, B, L, H, lane4r, tid, sa, D | INFO_OK, r.x, inoff, outoff, pp, nullptr);
+                const uint32_t Lp = 48u + esp_C(D);
+                B.out_len[i] = (uint16_t)Lp;
+                c_ok++;
+                c_in += D;
+                c_out += Lp;
+            } else {
+                B.out_len[i] = 0;
+                c_drop++;
+            }
+        }
+        if (R.ts && lane == 0) atomicMax(&R.ts[1u + bi], gtimer());
+        got = false;
+        if (bi + 1u < R.n_batches) {
+            const uint32_t rv = __shfl_sync(0xffffffffu, rv_next, 0);
+            if ((int32_t)(rv - ((bi + 1u) / ROLES_NREC + 1u) * P) >= 0) {
+                r = __ldcg(&rec[((size_t)((bi + 1u) % ROLES_NREC) * Lc + c) * 512u + tid]);
+                got = true;
+            }
+        }
+    }
+    roles_lane_counters(W, L, c_ok, c_drop, c_in, c_out);
 }
 
 __global__ void __launch_bounds__(F_THREADS, 1)
@@ -2252,6 +2491,7 @@ k_fused_ring_roles(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, Rol
     if (R.n_batches == 0) return;
     if (R.ts && blockIdx.x == 0 && threadIdx.x == 0) R.ts[0] = gtimer();
     if (blockIdx.x < Q.npro) roles_sequencer(T, slots, R, Q, smem, blockIdx.x);
+    else if (Q.sorted) roles_lanes_sorted(T, W, slots, R, Q, smem, blockIdx.x - Q.npro);
     else roles_lanes(T, W, slots, R, Q, smem, blockIdx.x - Q.npro);
     // leave; the last CTA out zeroes the hand-off counters for the next launch
     __syncthreads();
@@ -2269,8 +2509,9 @@ k_fused_ring_roles(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, Rol
 bool fused_roles_ok(uint32_t n, uint32_t n_sa, int grid, uint32_t npro)
 {
     if (npro == 0 || grid <= (int)npro || n == 0 || n_sa == 0 || n_sa > ROLES_MAX_SA) return false;
-    const uint32_t Lc = (uint32_t)grid - npro;
-    return n <= 512u * Lc && (n + npro - 1u) / npro <= ROLES_RPP_MAX;
+    const uint32_t Lc = (uint32_t)grid - npro, ppc = (n + Lc - 1u) / Lc;
+    // a sequencer's range: its ceil(Lc / npro) lane CTAs' packets
+    return ppc <= 512u && ((Lc + npro - 1u) / npro) * ppc <= ROLES_RPP_MAX;
 }
 
 cudaError_t launch_fused_ring_roles(const DevTable &T, const DevWork &W, const BatchArgs *slots,

@@ -2,8 +2,8 @@
 oracle: memcmp of every slot ... on all configs"; §4.1).
 
 bench.py times the batch ring's default form (the role-split ring
-k_fused_ring_roles for one-length rings, the software-pipelined
-k_fused_ring_pipe for IMIX; each also run in the other form here) over R device copies of one full-size batch (65,536 packets, 1024 SAs; R from
+k_fused_ring_roles -- sorted mode at IMIX -- except the software-pipelined
+k_fused_ring_pipe at 1514 B; each also run in the other form here) over R device copies of one full-size batch (65,536 packets, 1024 SAs; R from
 device.ring_slot_count, the bench's own formula), every timed batch through
 nba_ipsec_ring_run_batches.  Here the same ring runs 2R + 5 batches (two
 rotations and a partial one), then a second run continues mid-rotation from
@@ -41,10 +41,11 @@ def _ring_vs_oracle(size, cfg_id, runs, timestamps=False, form=None):
         ring = t.ring([(*d.args(), b.n) for d in dbs])
         if form is not None:
             ring.set_form(form)
-        # default: the role-split form for one-length rings of frames up to 1024 B,
+        # default: the role-split form for one-length rings of frames up to 1024 B
+        # and for mixed rings of more than 4 slots (IMIX: R = 7, sorted mode),
         # else the pipelined one
         expect_form = form if form is not None else (
-            nba_ipsec.Ring.PIPELINED if size in ("imix", 1514) else nba_ipsec.Ring.ROLES)
+            nba_ipsec.Ring.PIPELINED if size == 1514 else nba_ipsec.Ring.ROLES)
         assert ring.form == expect_form
         ts = None
         if timestamps:
@@ -107,7 +108,7 @@ def test_bench_ring_free_form(cfg_id, size):
                     form=nba_ipsec.Ring.FREE)
 
 
-@pytest.mark.parametrize("cfg_id,size", [(2, 64), (5, 256)])
+@pytest.mark.parametrize("cfg_id,size", [(2, 64), (5, 256), (4, "imix")])
 def test_bench_ring_pipelined_form(cfg_id, size):
     """The software-pipelined form (set_form; the default before the role-split
     form) over the same full-size one-length rings, against the oracle."""
@@ -119,11 +120,11 @@ def test_bench_ring_pipelined_form(cfg_id, size):
                     form=nba_ipsec.Ring.PIPELINED)
 
 
-@pytest.mark.parametrize("cfg_id,size", [(4, "imix"), (3, 1514)])
+@pytest.mark.parametrize("cfg_id,size", [(3, 1514)])
 def test_bench_ring_roles_form(cfg_id, size):
-    """The role-split form (set_form) over the full-size IMIX ring (mixed
-    lengths in every warp) and 1514-B ring: two rotations and a partial one,
-    then a run continuing mid-rotation, with timestamps."""
+    """The role-split form (set_form) over the full-size 1514-B ring: two
+    rotations and a partial one, then a run continuing mid-rotation, with
+    timestamps."""
     import torch
     from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
     p, b = shard.rank_workload(cfg_id, N_PKTS, size, N_SA, 0, 1)

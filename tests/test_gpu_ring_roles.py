@@ -139,3 +139,31 @@ def test_roles_ring_then_other_paths():
             assert np.array_equal(g_len, o_len) and np.array_equal(g_out, o_out)
         assert np.array_equal(t.sa_seq(), oracle.sa_seq(sas, n_sa))
         ring.close()
+
+
+@pytest.mark.parametrize("npro,n_sa,n", [(4, 61, 9000), (6, 1024, 65536), (2, 2048, 30000), (5, 7, 100)])
+def test_roles_ring_sorted_mode(npro, n_sa, n, monkeypatch):
+    """Sorted mode (mixed-length rings with more slots than the record ring):
+    per batch the sequencers sort each lane CTA's packets by length and place
+    runs of 32 on the lane warps by cumulative cost, so a packet slot changes
+    lanes between uses of a ring slot -- 6 slots of mixed traffic (IMIX, 64 B,
+    1514 B), invalid SAs / lengths, runs of 7 + 5 + 13 batches."""
+    monkeypatch.setenv("NBA_IPSEC_ROLES_P", str(npro))
+    p = gen.make_sas(n_sa, cfg_id=76)
+    sizes = ("imix", 64, "imix", 1514, "imix", 300)
+    hb = [gen.make_batch(n, s, n_sa, cfg_id=76, batch=i) for i, s in enumerate(sizes)]
+    hb[0].sa_idx[::89] = n_sa + 2
+    hb[2].in_len[4::97] = 19
+    _roles_vs_oracle(p, n_sa, hb, [7, 5, 13])
+
+
+def test_roles_ring_sorted_mode_overflow():
+    """Sorted mode with SA counters at / near 2^32 - 1 over 6 slots."""
+    n_sa, n = 32, 20000
+    seq = np.full(n_sa, 0xFFFFFFFF - 1500, np.uint32)
+    seq[::3] = 0xFFFFFFFF
+    p = gen.make_sas(n_sa, cfg_id=77)
+    p = gen.SAParams(*[getattr(p, f) for f in ("spi", "tunnel_src", "tunnel_dst", "aes_key",
+                                               "ctr_nonce", "hmac_key")], seq=seq)
+    hb = [gen.make_batch(n, "imix", n_sa, cfg_id=77, batch=k) for k in range(6)]
+    _roles_vs_oracle(p, n_sa, hb, [6, 5], defined_only=True)
