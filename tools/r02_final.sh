@@ -19,14 +19,10 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --c
    --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 22 --warmup 3 --no-sweep --no-cpu --no-inbound --no-alb > /dev/null 2>&1
 for C in 2 3 4; do
   timeout 600 ncu --set full --clock-control none --import-source on -k regex:'k_fused_ring' \
-      -c 1 -o gpurun_out/prof_${TAG}_ring_c$C -f python tools/run_batches.py --config $C --batches 1 --ring 4 > /dev/null 2>&1
+      -c 1 -o gpurun_out/prof_${TAG}_ring_c$C -f python tools/run_batches.py --config $C --batches 1 --ring 6 > /dev/null 2>&1
   timeout 600 ncu --set full --clock-control none --import-source on -k regex:'k_in_' \
       -s 2 -c 1 -o gpurun_out/prof_${TAG}_in_c$C -f python tools/run_inbound.py --config $C --batches 3 > /dev/null 2>&1
 done
 ls gpurun_out/ | grep $TAG | head -40
-for tool in memcheck racecheck synccheck initcheck; do
-  for c in c1 ring_small roles inbound inring host c4 ring64; do
-    timeout 420 compute-sanitizer --tool $tool python tools/sanitize_cases.py $c > gpurun_out/sanitizer/${TAG}_${tool}_${c}.txt 2>&1
-    echo "$tool $c rc=$? $(grep -E 'SUMMARY|result ==' gpurun_out/sanitizer/${TAG}_${tool}_${c}.txt | tr '\n' ' ')"
-  done
-done
+# compute-sanitizer is closed on this GPU pool (runs under it left GPUs needing a reset);
+# the cases stay in tools/sanitize_cases.py for a pool where it is open

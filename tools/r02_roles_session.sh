@@ -5,9 +5,3 @@ python -c "import oracle; oracle.build()"
 timeout 1200 python -m pytest tests -m gpu -q > gpurun_out/s9_pytest_gpu.log 2>&1; tail -3 gpurun_out/s9_pytest_gpu.log
 timeout 200 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/s9_smoke.log 2>&1; echo smoke rc=$?
 timeout 600 python bench.py --steps 20 --warmup 5 > gpurun_out/s9_bench_s20.json 2> gpurun_out/s9_bench_s20.err; echo bench rc=$?
-for tool in memcheck racecheck synccheck initcheck; do
-  for c in roles ring64; do
-    timeout 600 compute-sanitizer --tool $tool python tools/sanitize_cases.py $c > gpurun_out/sanitizer/s9_${tool}_${c}.txt 2>&1
-    echo "$tool $c rc=$? $(grep -E 'SUMMARY|result ==|^ok|True|False' gpurun_out/sanitizer/s9_${tool}_${c}.txt | tail -2 | tr '\n' ' ')"
-  done
-done

@@ -3,8 +3,9 @@
 
     python tools/r02_summary.py TAG
 
-Reads gpurun_out/prof_TAG_ring_c{2,3,4}.ncu-rep (k_fused_ring_pipe, one run of
-4 batch slots = 4 batches), gpurun_out/prof_TAG_in_c{2,3,4}.ncu-rep (inbound
+Reads gpurun_out/prof_TAG_ring_c{2,3,4}.ncu-rep (the ring's default form for the
+config -- k_fused_ring_roles or k_fused_ring_pipe -- one run of 6 batch slots =
+6 batches), gpurun_out/prof_TAG_in_c{2,3,4}.ncu-rep (inbound
 one-kernel launch), gpurun_out/TAG_launches.csv (ncu launch list of
 `bench.py --steps 22`), gpurun_out/microbench_TAG.json and
 gpurun_out/bench_TAG.json; writes profiles/TAG_ncu_summary.md and updates
@@ -43,6 +44,9 @@ def raw(rep):
         return None
     h, u, d = rows[0], rows[1], rows[2]
     out = {}
+    if "Kernel Name" in h:
+        k = d[h.index("Kernel Name")]
+        out["kernel"] = k.split("(")[0].replace("nba::", "").replace("void ", "")
     for name, label, mul, kind in METRICS:
         if name in h:
             i = h.index(name)
@@ -60,15 +64,15 @@ def main():
     lines = [f"# ncu summary, round tag `{tag}`", "",
              "Captured with `ncu --set full --clock-control none --import-source on` under gpurun "
              "(`tools/r02_final.sh`); serialised, cold-cache replays: times under ncu are not bench "
-             "values, compare shares.  Ring rows: one `k_fused_ring_pipe` launch over a 4-slot ring "
-             "(4 batches), per-batch figures = launch / 4.", ""]
+             "values, compare shares.  Ring rows: one launch of the ring's default form (kernel "
+             "column) over a 6-slot ring (6 batches), per-batch figures = launch / 6.", ""]
     kj_path = os.path.join(PROF, "ncu_kernels.json")
     kj = json.load(open(kj_path)) if os.path.exists(kj_path) else {}
-    for kind, title, div in (("ring", "software-pipelined batch ring (per batch)", 4.0),
+    for kind, title, div in (("ring", "batch ring, default form (per batch)", 6.0),
                              ("in", "ESP inbound, one-kernel launch", 1.0)):
         lines += [f"## {title}", "",
-                  "| config | " + " | ".join(m[1] for m in METRICS) + " |",
-                  "|---|" + "---|" * len(METRICS)]
+                  "| config | kernel | " + " | ".join(m[1] for m in METRICS) + " |",
+                  "|---|---|" + "---|" * len(METRICS)]
         for c, name in CFG.items():
             rep = os.path.join(OUT, f"prof_{tag}_{kind}_c{c}.ncu-rep")
             if not os.path.exists(rep):
@@ -86,11 +90,13 @@ def main():
                              "bank conflicts"):
                     x = x / div
                 cells.append(f"{x:.4g}")
-            lines.append(f"| {name} | " + " | ".join(cells) + " |")
-            key = ("fused_ring" if kind == "ring" else "in_fused") + ":" + name
+            kern = v.get("kernel", "")
+            lines.append(f"| {name} | {kern} | " + " | ".join(cells) + " |")
+            key = ("in_fused" if kind != "ring" else
+                   "fused_ring_roles" if "roles" in kern else "fused_ring") + ":" + name
             kj[key] = {"dram_bytes_per_launch": (v["DRAM rd MB"] + v["DRAM wr MB"]) * 1e6 / div,
                        "ncu_duration_us": v["us"] / div,
-                       "note": "per batch of a 4-batch ring run" if kind == "ring" else "per launch",
+                       "note": "per batch of a 6-batch ring run" if kind == "ring" else "per launch",
                        "source": os.path.basename(rep)}
         lines.append("")
     kj["_round"] = tag
