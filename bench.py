@@ -150,10 +150,12 @@ def work_model(b):
 
 
 # Per-unit work, SASS-derived (tools/sass_hist.py over the shipped
-# k_fused_ring_pipe, committed as profiles/r02_sass_hist.txt): instructions per
-# AES-128 block (a quarter of the 4-block step, round loop x 7) and per SHA-1
-# compression, by issuing pipe.  Fallbacks = the r02 counts.
-SASS_HIST = os.path.join(ROOT, "profiles", "r02_sass_hist.txt")
+# k_fused_ring_roles -- the headline's kernel; k_fused_ring_pipe's counts,
+# profiles/r02_sass_hist.txt, differ by < 1% -- committed as
+# profiles/r02d_sass_hist.txt): instructions per AES-128 block (a quarter of the
+# 4-block step, round loop x 7) and per SHA-1 compression, by issuing pipe.
+# Fallbacks = the r02 counts.
+SASS_HIST = os.path.join(ROOT, "profiles", "r02d_sass_hist.txt")
 SASS_FALLBACK = {"aes_block": {"alu": 217.75, "fma": 19.5, "smem": 136.75},
                  "sha1_compression": {"alu": 434, "fma": 244, "smem": 0}}
 ALU_LANES_PER_CLK_SM = 64          # B300_MICROARCH "Pipe rates"; microbenchmarked 63.9 on B200
@@ -166,7 +168,7 @@ def sass_units():
             if line.startswith("JSON "):
                 d = json.loads(line[5:])
                 return {"aes_block": d["aes_block"], "sha1_compression": d["sha1_compression"],
-                        "source": "profiles/r02_sass_hist.txt"}
+                        "source": "profiles/r02d_sass_hist.txt"}
     except Exception:
         pass
     return dict(SASS_FALLBACK, source="fallback constants (r02 SASS counts)")

@@ -48,7 +48,7 @@ def test_imix_composition_and_invalid_packets_excluded():
 
 
 def test_roofline_arithmetic():
-    """ALU / LDS / HBM fractions from the SASS per-unit counts (profiles/r02_sass_hist.txt)."""
+    """ALU / LDS / HBM fractions from the SASS per-unit counts (profiles/r02d_sass_hist.txt)."""
     w = {"aes_blocks": 1000, "sha1_compressions": 100, "hbm_bytes": 5000}
     peaks = {"sm_max_mhz": 1965.0, "hbm_gbs": 6500.0, "source": "test"}
     units = bench.sass_units()

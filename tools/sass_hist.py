@@ -124,6 +124,9 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--kernel", default="k_fused_ring_pipe")
     ap.add_argument("--out", default=None)
+    ap.add_argument("--instances", type=int, default=1,
+                    help="inlined copies of the lane path in the kernel (k_fused_ring_roles: 2, its "
+                         "fixed-slot and sorted-slot lanes); per-unit counts are divided by it")
     a = ap.parse_args()
     fc = os.path.join(CSRC, "fused_common.cuh")
     rfc = func_ranges(fc, ["aes4_keystream", "ctr_precompute", "expand_key_slots"])
@@ -167,8 +170,10 @@ def main():
         return c
 
     aes4 = dyn(("aes_step_outside_loop", 1), ("aes_round_loop_body", 7))
-    per_block = {p: aes4[p] / 4.0 for p in pipes}
-    sha = dyn(("sha1_compress", 1))
+    per_block = {p: aes4[p] / 4.0 / a.instances for p in pipes}
+    sha = {p: v / a.instances for p, v in dyn(("sha1_compress", 1)).items()}
+    for k in ("ctr_precompute", "expand_key_lane"):
+        regions[k] = collections.Counter({p: v / a.instances for p, v in regions[k].items()})
     lines = [f"# SASS histogram of {a.kernel} (libnba_ipsec.so, nvdisasm -gi), by source function and pipe",
              f"# aes4_keystream fused_common.cuh:{a0}-{a1} (round loop {loop0}-{loop1}, x7); "
              f"sha1_compress_fma sha1.cuh:{rsha['sha1_compress_fma'][0]}-{rsha['sha1_compress_fma'][1]}",
@@ -177,13 +182,13 @@ def main():
         top = ", ".join(f"{o} {n}" for o, n in ops[k].most_common(8))
         lines.append(k.ljust(24) + "".join(str(c[p]).rjust(9) for p in pipes) + "   " + top)
     lines.append("")
-    lines.append("per unit (dynamic: loop body x 7)")
+    lines.append(f"per unit (dynamic: loop body x 7; / {a.instances} inlined copies of the lane path)")
     lines.append("AES-128 block (1/4 step)".ljust(24) + "".join(f"{per_block[p]:9.1f}" for p in pipes))
-    lines.append("SHA-1 compression".ljust(24) + "".join(str(sha[p]).rjust(9) for p in pipes))
+    lines.append("SHA-1 compression".ljust(24) + "".join(f"{sha.get(p, 0):9.1f}" for p in pipes))
     lines.append("per packet: ctr_precompute".ljust(24) + "".join(str(regions['ctr_precompute'][p]).rjust(9) for p in pipes))
     lines.append("per packet: key expansion".ljust(24) + "".join(str(regions['expand_key_lane'][p]).rjust(9) for p in pipes))
     summary = {"aes_block": {p: per_block[p] for p in pipes},
-               "sha1_compression": {p: sha[p] for p in pipes},
+               "sha1_compression": {p: sha.get(p, 0) for p in pipes},
                "ctr_precompute_per_packet": dict(regions["ctr_precompute"]),
                "expand_key_per_packet": dict(regions["expand_key_lane"])}
     lines.append("")
