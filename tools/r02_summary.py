@@ -33,7 +33,7 @@ METRICS = [("gpu__time_duration.sum", "us", 1e-3, "us"),
            ("l1tex__data_bank_conflicts_pipe_lsu_mem_shared.sum", "bank conflicts", 1, None),
            ("smsp__inst_executed.sum", "warp inst", 1, None),
            ("launch__registers_per_thread", "regs", 1, None)]
-SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "usecond": 1e3, "msecond": 1e6,
+SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "usecond": 1e3, "msecond": 1e6, "ms": 1e6,
          "nsecond": 1, "us": 1e3}
 
 
