@@ -503,6 +503,13 @@ int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, u
                     nba_ipsec_ring_destroy(r);
                     return NBA_IPSEC_ENOMEM;
                 }
+                // sequencers stage SA indices / lengths by bulk copy when every slot's
+                // arrays are 16-byte aligned
+                r->rq.stage = 1u;
+                for (uint32_t i = 0; i < n_slots; i++)
+                    if ((reinterpret_cast<uintptr_t>(slots[i].sa_idx) | reinterpret_cast<uintptr_t>(slots[i].in_len)) & 15u)
+                        r->rq.stage = 0u;
+                if (std::getenv("NBA_IPSEC_ROLES_NOSTAGE")) r->rq.stage = 0u;
                 // mixed lengths: per-batch length-sorted lane slots (a packet slot may
                 // change lanes between uses of a ring slot: needs n_slots > ROLES_NREC)
                 r->rq.sorted = (!one_len && n_slots > ROLES_NREC) ? 1u : 0u;

@@ -213,7 +213,8 @@ bool fused_pipe_ok(uint32_t n, int grid);
 // per packet into a ring of ROLES_NREC record buffers, the other CTAs encrypt.
 constexpr uint32_t ROLES_NREC = 4;          // batches of records in flight
 constexpr uint32_t ROLES_MAX_SA = 2048;     // per-warp SA counters in a sequencer's shared memory
-constexpr uint32_t ROLES_RPP_MAX = 18432;   // packets per sequencer and batch (shared stash)
+constexpr uint32_t ROLES_RPP_MAX = 16416;   // packets per sequencer and batch (shared stash: 36 lane
+                                            //   CTAs x 456 packets, a 65,536-packet batch at 4 sequencers)
 constexpr uint32_t ROLES_CTL_WORDS = 2u * ROLES_NREC + 2u;   // ready[], consumed[], pbar, exit
 struct RolesBufs {
     uint32_t *ctl;      // [ROLES_CTL_WORDS] hand-off counters (zero between launches)
@@ -222,6 +223,7 @@ struct RolesBufs {
                         //   range (0xffffffff: none)} by lane slot
     uint32_t *cum;      // [(grid - npro) * 16] sorted mode: each lane warp's assigned work so far
     uint32_t sorted;    // 1: per-batch length-sorted lane slots (mixed-length rings)
+    uint32_t stage;     // 1: sequencers stage SA indices / lengths by bulk copy (16-B aligned arrays)
     uint32_t *ptot;     // [2][npro][n_sa] per-sequencer per-SA valid-packet totals
     uint8_t *scratch;   // [(grid - npro) * 256] output lines of the lanes' warm-up experiment
     uint32_t npro;      // sequencer CTAs

@@ -1965,7 +1965,7 @@ __device__ __forceinline__ void roles_lane_consumed(uint32_t *p, uint32_t q)
 // position in the run).  Slots left without a packet get the record
 // {0, 0xffffffff}.  A run's cost: 8 (SHA-1 blocks + 1) + 3 AES steps of its
 // first (longest) packet, ~11 x inner SHA-1 blocks + 8.
-__device__ __noinline__ void roles_sort_slots(uint2 *rec, uint32_t *cumb, uint16_t *d16, const uint16_t *sa16,
+__device__ __noinline__ void roles_sort_slots(uint2 *rec, uint32_t *cumb, uint16_t *d16, const uint32_t *sav,
                                               uint32_t (*hw)[NBINS], uint32_t r0, uint32_t n,
                                               uint32_t ppc, uint32_t cbeg, uint32_t cend)
 {
@@ -1973,7 +1973,7 @@ __device__ __noinline__ void roles_sort_slots(uint2 *rec, uint32_t *cumb, uint16
     for (uint32_t cc = cbeg + warp; cc < cend; cc += 16u) {
         const uint32_t pb = min(n, cc * ppc), pe = min(n, pb + ppc), cnt = pe - pb;
         auto bin_of = [&](uint32_t i) {
-            const bool ok = sa16[i - r0] != 0xffffu;
+            const bool ok = sav[i - r0] != 0xffffffffu;
             return hmac_bin(ok, esp_C(d16[i - r0]));
         };
         hw[warp][lane] = 0u;
@@ -2042,20 +2042,27 @@ __device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchAr
 {
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
     const uint32_t P = Q.npro, Lc = gridDim.x - P, LW = Lc * 16u, n_sa = T.n_sa;
-    // shared memory: per-packet stash of this sequencer's range, per-warp SA counters
-    uint16_t *rank = reinterpret_cast<uint16_t *>(smem);           // [ROLES_RPP_MAX]
-    uint16_t *sa16 = rank + ROLES_RPP_MAX;                         // [ROLES_RPP_MAX] 0xffff: drop
-    uint16_t *d16 = sa16 + ROLES_RPP_MAX;                          // [ROLES_RPP_MAX]
-    uint16_t *cnt = d16 + ROLES_RPP_MAX;                           // [16][ROLES_MAX_SA]
-    uint32_t *seqs = reinterpret_cast<uint32_t *>(cnt + 16u * ROLES_MAX_SA);   // [ROLES_MAX_SA]
+    // shared memory: this sequencer's range of SA indices and lengths (staged by
+    // bulk copies from the batch; the SA index becomes 0xffffffff for a dropped
+    // packet, the length the lane slot in sorted mode), each packet's rank,
+    // per-warp SA counters, the SAs' counters and bases
+    uint16_t *rank = reinterpret_cast<uint16_t *>(smem);                          // [RPP_MAX]
+    uint32_t *raw_sa = reinterpret_cast<uint32_t *>(rank + ROLES_RPP_MAX);        // [RPP_MAX + 8]
+    uint16_t *raw_len = reinterpret_cast<uint16_t *>(raw_sa + ROLES_RPP_MAX + 8u); // [RPP_MAX + 16]
+    uint16_t *cnt = raw_len + ROLES_RPP_MAX + 16u;                                // [16][ROLES_MAX_SA]
+    uint32_t *seqs = reinterpret_cast<uint32_t *>(cnt + 16u * ROLES_MAX_SA);      // [ROLES_MAX_SA]
     unsigned long long *start = reinterpret_cast<unsigned long long *>(seqs + ROLES_MAX_SA);
     uint32_t (*sorth)[NBINS] = reinterpret_cast<uint32_t (*)[NBINS]>(start + ROLES_MAX_SA);   // [16][NBINS]
-    static_assert(3u * ROLES_RPP_MAX * 2u + 16u * ROLES_MAX_SA * 2u + ROLES_MAX_SA * 12u + 16u * NBINS * 4u
-                      <= F_SMEM, "sequencer shared memory");
+    unsigned long long *mbar = reinterpret_cast<unsigned long long *>(&sorth[16][0]);
+    static_assert(ROLES_RPP_MAX % 8u == 0u, "16-B aligned stash arrays");
+    static_assert(ROLES_RPP_MAX * 2u + (ROLES_RPP_MAX + 8u) * 4u + (ROLES_RPP_MAX + 16u) * 2u +
+                      16u * ROLES_MAX_SA * 2u + ROLES_MAX_SA * 12u + 16u * NBINS * 4u + 8u <= F_SMEM,
+                  "sequencer shared memory");
     uint32_t *ready = Q.ctl, *consumed = Q.ctl + ROLES_NREC, *pbar = Q.ctl + 2u * ROLES_NREC;
     uint16_t *mycnt = cnt + warp * ROLES_MAX_SA;
     for (uint32_t s = tid; s < n_sa; s += F_THREADS) seqs[s] = __ldcg(&T.seq[s]);
     for (uint32_t s = lane; s < n_sa; s += 32u) mycnt[s] = 0;
+    if (tid == 0) tbar_init(mbar);
     __syncthreads();
     // this sequencer's lane CTAs [cbeg, cend): its packet range is theirs
     const uint32_t cbeg = p * Lc / P, cend = (p + 1u) * Lc / P;
@@ -2092,6 +2099,45 @@ __device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchAr
             if (tid == 0) roles_wait_geq(&consumed[bi % ROLES_NREC], (bi / ROLES_NREC) * LW);
             __syncthreads();
         }
+        // the range's SA indices and lengths into shared memory: bulk async
+        // copies (TMA engine) of their 16-byte aligned cover, the few elements
+        // past its last whole 16 bytes by plain loads; or (arrays not 16-byte
+        // aligned) loads by all threads
+        const uint32_t hs = r0 & 3u, hl = r0 & 7u;
+        uint32_t *sav = raw_sa + hs;                       // sav[i - r0] = SA of packet i
+        uint16_t *lenv = raw_len + hl;                     // lenv[i - r0] = its length
+        if (Q.stage) {
+            const uint32_t nbs = r1 > r0 ? ((r1 - r0 + hs) * 4u) & ~15u : 0u;
+            const uint32_t nbl = r1 > r0 ? ((r1 - r0 + hl) * 2u) & ~15u : 0u;
+            if (tid == 0) {
+                const uint32_t mb = smem_u32(mbar);
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(nbs + nbl)
+                             : "memory");
+                const uint8_t *gs = reinterpret_cast<const uint8_t *>(B.sa_idx + (r0 - hs));
+                const uint8_t *gl = reinterpret_cast<const uint8_t *>(B.in_len + (r0 - hl));
+                for (uint32_t o = 0; o < nbs; o += 16384u)
+                    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                                 ::"r"(smem_u32(raw_sa) + o), "l"(gs + o), "r"(min(16384u, nbs - o)), "r"(mb)
+                                 : "memory");
+                for (uint32_t o = 0; o < nbl; o += 16384u)
+                    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                                 ::"r"(smem_u32(raw_len) + o), "l"(gl + o), "r"(min(16384u, nbl - o)), "r"(mb)
+                                 : "memory");
+            }
+            // the tails (< 4 SA indices, < 8 lengths)
+            for (uint32_t i = r0 - hs + nbs / 4u + tid; i < r1; i += F_THREADS) raw_sa[i - (r0 - hs)] = B.sa_idx[i];
+            for (uint32_t i = r0 - hl + nbl / 2u + tid; i < r1; i += F_THREADS)
+                raw_len[i - (r0 - hl)] = B.in_len[i];
+            __syncthreads();
+            tables_bulk_wait(mbar, bi & 1u);
+        } else {
+            for (uint32_t i = r0 + tid; i < r1; i += F_THREADS) {
+                sav[i - r0] = B.sa_idx[i];
+                lenv[i - r0] = B.in_len[i];
+            }
+            __syncthreads();
+        }
         // A. validity, the packet's rank among the warp's earlier packets of its
         //    SA (rounds of 32 in index order, match groups within a round)
         for (uint32_t g0 = w0; g0 < w1; g0 += 32u * NBA_ROLES_AG) {
@@ -2100,8 +2146,8 @@ __device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchAr
             for (uint32_t k = 0; k < NBA_ROLES_AG; k++) {
                 const uint32_t i = g0 + 32u * k + lane;
                 const bool in = i < w1;
-                s[k] = in ? B.sa_idx[i] : INVALID_SA;
-                D[k] = in ? (uint32_t)B.in_len[i] : 0u;
+                s[k] = in ? sav[i - r0] : INVALID_SA;
+                D[k] = in ? (uint32_t)lenv[i - r0] : 0u;
             }
 #pragma unroll
             for (uint32_t k = 0; k < NBA_ROLES_AG; k++) {
@@ -2126,16 +2172,13 @@ __device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchAr
                     rank[i - r0] = (uint16_t)(c0 + __popc(peers & lanemask_lt()));
                     if (lane == leader) mycnt[s[k]] = (uint16_t)(c0 + __popc(peers));
                 }
-                if (in) {
-                    sa16[i - r0] = cand ? (uint16_t)s[k] : (uint16_t)0xffffu;
-                    d16[i - r0] = (uint16_t)D[k];
-                }
+                if (in && !cand) sav[i - r0] = 0xffffffffu;    // dropped: no number
             }
         }
         __syncthreads();
         if (Q.sorted)
             roles_sort_slots(reinterpret_cast<uint2 *>(Q.rec) + (size_t)(bi % ROLES_NREC) * Lc * 512u, Q.cum,
-                             d16, sa16, sorth, r0, n, ppc, cbeg, cend);
+                             lenv, sav, sorth, r0, n, ppc, cbeg, cend);
 #if NBA_ROLES_TRACE
         if (R.ts && p == 0 && tid == 0) *RLT(bi, 1) = gtimer();
 #endif
@@ -2189,17 +2232,17 @@ __device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchAr
         for (uint32_t g0 = w0; g0 < w1; g0 += 32u) {
             const uint32_t i = g0 + lane;
             if (i < w1) {
-                const uint32_t s = sa16[i - r0];
+                const uint32_t s = sav[i - r0];
                 uint32_t r = 0u;
-                if (s != 0xffffu) {
+                if (s != 0xffffffffu) {
                     const unsigned long long q =
                         start[s] + mycnt[s] + (unsigned long long)rank[i - r0] + 1ull;
                     r = q <= 0xffffffffull ? (uint32_t)q : 0u;
                 }
                 if (Q.sorted) {
                     const uint32_t c = i / ppc;
-                    reinterpret_cast<uint2 *>(rec)[(size_t)c * 512u + d16[i - r0]] = make_uint2(r, i - c * ppc);
-                    if (s != 0xffffu) prefetch_l2(B.in_buf + B.in_off[i]);   // its payload's first line
+                    reinterpret_cast<uint2 *>(rec)[(size_t)c * 512u + lenv[i - r0]] = make_uint2(r, i - c * ppc);
+                    if (s != 0xffffffffu) prefetch_l2(B.in_buf + B.in_off[i]);   // its payload's first line
                 } else {
                     rec[i] = r;
                 }

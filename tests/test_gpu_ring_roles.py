@@ -167,3 +167,15 @@ def test_roles_ring_sorted_mode_overflow():
                                                "ctr_nonce", "hmac_key")], seq=seq)
     hb = [gen.make_batch(n, "imix", n_sa, cfg_id=77, batch=k) for k in range(6)]
     _roles_vs_oracle(p, n_sa, hb, [6, 5], defined_only=True)
+
+
+@pytest.mark.parametrize("sorted_mode", [False, True])
+def test_roles_ring_sequencer_plain_loads(sorted_mode, monkeypatch):
+    """The sequencers' fallback without bulk staging (SA index / length arrays
+    not 16-byte aligned take it; forced here), fixed and sorted lane slots."""
+    monkeypatch.setenv("NBA_IPSEC_ROLES_NOSTAGE", "1")
+    p = gen.make_sas(40, cfg_id=78)
+    sizes = ("imix", 64, "imix", 1514, 300) if sorted_mode else (64, 64)
+    hb = [gen.make_batch(7001, s, 40, cfg_id=78, batch=i) for i, s in enumerate(sizes)]
+    hb[0].sa_idx[::61] = 77
+    _roles_vs_oracle(p, 40, hb, [6, 7])
