@@ -298,7 +298,8 @@ struct OutStream {
     }
         switch (p) {
         case 0: {
-            stg_v4(cp, d[0], d[1], d[2], d[3]);
+            // (lo != 0 only at the stream's start: bytes [0, lo) are not ours)
+            store_chunk_range(cp, d[0], d[1], d[2], d[3], lo, 16);
             stg_v4(cp + 16, d[4], d[5], d[6], d[7]);
             stg_v4(cp + 32, d[8], d[9], d[10], d[11]);
             stg_v4(cp + 48, d[12], d[13], d[14], d[15]);

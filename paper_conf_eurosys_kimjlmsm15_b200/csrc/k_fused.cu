@@ -52,6 +52,9 @@ namespace nba {
 #ifndef NBA_CARRY             // 1: reuse the previous step's last 32-byte payload block
 #define NBA_CARRY 0
 #endif
+#ifndef NBA_HDR_DEFER         // 1: the outer header words go out with the first ciphertext words
+#define NBA_HDR_DEFER 0       //   (one put16 of header + 7 ciphertext words, its SA-line words and TOS
+#endif                        //   byte re-read; esp_packet<true>): measured per kernel
 #ifndef NBA_STG256            // 1: output through 32-byte chunks (256-bit stores)
 #define NBA_STG256 0
 #endif
@@ -105,6 +108,7 @@ __device__ __forceinline__ PktPre load_pkt_pre(const DevTable &T, const uint8_t 
     return p;
 }
 
+template <bool HDR_DEFER = (NBA_HDR_DEFER != 0)>
 __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B, FusedLo &L,
                                            FusedHi &H, uint32_t lane4r, uint32_t tid, uint32_t sa,
                                            uint32_t info, uint32_t q32, uint32_t inoff,
@@ -139,22 +143,53 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
     OutStream os;
 #endif
     os.init(B.out_buf + outoff);
-    {
+    // outer header words 0..8; emitted together with the first ciphertext words
+    // (NBA_HDR_DEFER: one 16-word put16 instead of 16 single-word puts for
+    // packets of >= 7 ciphertext words), else right here
+    auto header_words = [&](uint32_t (&h)[9]) {
         const uint32_t src = bswap32(hd.z), dst = bswap32(hd.w);
         uint32_t sum = (0x4500u | tos) + Lb + 0x4000u + ((64u << 8) | 50u) + (src >> 16) +
                        (src & 0xffffu) + (dst >> 16) + (dst & 0xffffu);
         sum = (sum & 0xffffu) + (sum >> 16);
         sum = (sum & 0xffffu) + (sum >> 16);
         const uint32_t cs = ~sum & 0xffffu;
-        os.put(0x45u | (tos << 8) | ((Lb >> 8) << 16) | ((Lb & 0xffu) << 24));
-        os.put(0x00400000u);
-        os.put(64u | (50u << 8) | ((cs >> 8) << 16) | ((cs & 0xffu) << 24));
-        os.put(hd.z);
-        os.put(hd.w);
-        os.put(hd.x);
-        os.put(qbe);
-        os.put(0u);
-        os.put(qbe);
+        h[0] = 0x45u | (tos << 8) | ((Lb >> 8) << 16) | ((Lb & 0xffu) << 24);
+        h[1] = 0x00400000u;
+        h[2] = 64u | (50u << 8) | ((cs >> 8) << 16) | ((cs & 0xffu) << 24);
+        h[3] = hd.z;
+        h[4] = hd.w;
+        h[5] = hd.x;
+        h[6] = qbe;
+        h[7] = 0u;
+        h[8] = qbe;
+    };
+    // (NBA_HDR_RELOAD: the deferred header re-reads its SA-line words and the
+    // inner TOS byte instead of keeping them live across the AES step)
+    auto header_words_reload = [&](uint32_t (&h)[9]) {
+        const uint4 hd2 = ldg_nc_v4(&T.sal[(size_t)sa * SAL_U4 + 1]);
+        const uint32_t tos2 = (uint32_t)__ldg(B.in_buf + inoff + 1);
+        const uint32_t src = bswap32(hd2.z), dst = bswap32(hd2.w);
+        uint32_t sum = (0x4500u | tos2) + Lb + 0x4000u + ((64u << 8) | 50u) + (src >> 16) +
+                       (src & 0xffffu) + (dst >> 16) + (dst & 0xffffu);
+        sum = (sum & 0xffffu) + (sum >> 16);
+        sum = (sum & 0xffffu) + (sum >> 16);
+        const uint32_t cs = ~sum & 0xffffu;
+        h[0] = 0x45u | (tos2 << 8) | ((Lb >> 8) << 16) | ((Lb & 0xffu) << 24);
+        h[1] = 0x00400000u;
+        h[2] = 64u | (50u << 8) | ((cs >> 8) << 16) | ((cs & 0xffu) << 24);
+        h[3] = hd2.z;
+        h[4] = hd2.w;
+        h[5] = hd2.x;
+        h[6] = qbe;
+        h[7] = 0u;
+        h[8] = qbe;
+    };
+    const bool hdr_defer = HDR_DEFER && Cw >= 7u;
+    if (!hdr_defer) {
+        uint32_t h[9];
+        header_words(h);
+#pragma unroll
+        for (int w = 0; w < 9; w++) os.put(h[w]);
     }
     // SHA-1 message words 0..3 = ESP header (big-endian words of the wire bytes)
     uint32_t carry[4] = {bswap32(hd.x), q32, 0u, q32};
@@ -246,7 +281,19 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
             // AES step (the upper ones start that much later next batch)
             if (aes0_mark && it == 0) atomicMax(aes0_mark, (uint32_t)gtimer() - t_start);
             // stream the ciphertext words of this step to the output slot
-            if (16u * it + 16u <= Cw) {
+            if (hdr_defer && it == 0u) {
+                uint32_t v[16];
+                uint32_t h[9];
+                header_words_reload(h);
+#pragma unroll
+                for (int w = 0; w < 9; w++) v[w] = h[w];
+#pragma unroll
+                for (int w = 0; w < 7; w++) v[9 + w] = ct[w];
+                os.put16(v);
+#pragma unroll
+                for (int w = 7; w < 16; w++)
+                    if ((uint32_t)w < Cw) os.put(ct[w]);
+            } else if (16u * it + 16u <= Cw) {
                 os.put16(ct);
             } else {
 #pragma unroll
@@ -2503,7 +2550,7 @@ __device__ __forceinline__ void roles_lanes_sorted(const DevTable &T, const DevW
         if (lane == 0 && bi + 1u < R.n_batches) rv_next = roles_ld_relaxed(&ready[(bi + 1u) % ROLES_NREC]);
         if (have) {
             if (r.x != 0u) {
-                esp_packet(T, B, L, H, lane4r, tid, sa, D | INFO_OK, r.x, inoff, outoff, pp, nullptr);
+                esp_packet<true>(T, B, L, H, lane4r, tid, sa, D | INFO_OK, r.x, inoff, outoff, pp, nullptr);
                 const uint32_t Lp = 48u + esp_C(D);
                 B.out_len[i] = (uint16_t)Lp;
                 c_ok++;
