@@ -1999,6 +1999,9 @@ __device__ __forceinline__ void roles_lane_consumed(uint32_t *p, uint32_t q)
 #ifndef NBA_ROLES_RK_ASYNC    // lanes: round keys 3..10 by cp.async from the SA's schedule instead of
 #define NBA_ROLES_RK_ASYNC 0  //   expanded from the key (1)
 #endif
+#ifndef NBA_ROLES_MATCH       // sequencer: equal-SA groups by MATCH.ANY (1) or 12 ballots (0)
+#define NBA_ROLES_MATCH 0
+#endif
 #ifndef NBA_ROLES_AG          // sequencer: rounds of 32 packets whose metadata loads are in flight together
 #define NBA_ROLES_AG 8
 #endif
@@ -2206,11 +2209,15 @@ __device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchAr
                 // over the 11 SA bits and the validity bit
                 const uint32_t key = cand ? s[k] : 0x800u;
                 uint32_t peers = 0xffffffffu;
+                if (NBA_ROLES_MATCH) {
+                    peers = __match_any_sync(0xffffffffu, key);
+                } else {
 #pragma unroll
-                for (uint32_t bit = 0; bit < 12u; bit++) {
-                    const bool on = (key >> bit) & 1u;
-                    const uint32_t m = __ballot_sync(0xffffffffu, on);
-                    peers &= on ? m : ~m;
+                    for (uint32_t bit = 0; bit < 12u; bit++) {
+                        const bool on = (key >> bit) & 1u;
+                        const uint32_t m = __ballot_sync(0xffffffffu, on);
+                        peers &= on ? m : ~m;
+                    }
                 }
                 const uint32_t leader = (uint32_t)__ffs(peers) - 1u;
                 uint32_t c0 = (cand && lane == leader) ? (uint32_t)mycnt[s[k]] : 0u;
