@@ -113,8 +113,13 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
                                            FusedHi &H, uint32_t lane4r, uint32_t tid, uint32_t sa,
                                            uint32_t info, uint32_t q32, uint32_t inoff,
                                            uint32_t outoff, const PktPre &pp, unsigned long long *dbg,
-                                           uint32_t *aes0_mark = nullptr, uint32_t t_start = 0)
+                                           uint32_t *aes0_mark = nullptr, uint32_t t_start = 0,
+                                           uint32_t skip = 0)
 {
+    // skip (the role-split lanes' warm-up pass only; 0 for every real packet):
+    // bit 0 the CTR precompute, 1 the AES step and its emission, 3 the SHA-1
+    // compressions -- warps entering the code at different points fetch its
+    // instruction lines in parallel
     long long ck_start = clock64(), ck_setup = 0, ck_aes = 0, ck_sha = 0, ck_emit = 0;
     const uint4 r0 = pp.r0, r1 = pp.r1, r2 = pp.r2, hd = pp.hd, h0 = pp.h0, h1 = pp.h1;
     const uint32_t D = info & 0x7ffu;
@@ -134,7 +139,8 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
     // u_c = T[row(t0)] ^ Z_c), header words, HMAC inner midstate
     // round keys 3..10 were expanded into L.rkA / H.rkB[.][tid] by expand_key_lane
     const uint32_t qbe = bswap32(q32);
-    const CtrPre cp = ctr_precompute(lane4r, r0, r1, r2, hd.y, 0u, qbe);   // IV = BE64(q), A6
+    CtrPre cp{};
+    if (!(skip & 1u)) cp = ctr_precompute(lane4r, r0, r1, r2, hd.y, 0u, qbe);   // IV = BE64(q), A6
 
     // outer IPv4 header (reading A13) + ESP header + IV: output words 0..8
 #if NBA_STG256
@@ -210,7 +216,7 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
         uint32_t ct[16];
 #pragma unroll
         for (int w = 0; w < 16; w++) ct[w] = 0u;
-        if (it < nsteps) {
+        if (it < nsteps && !(skip & 2u)) {
             // payload words of T bytes [64 it, 64 it + 64), realigned
             if (64u * (it + NBA_PF_AHEAD) < D)
                 prefetch_bytes(src + 64u * (it + NBA_PF_AHEAD), min(64u, D - 64u * (it + NBA_PF_AHEAD)));
@@ -332,7 +338,7 @@ __device__ __forceinline__ void esp_packet(const DevTable &T, const BatchArgs &B
             ldg_nc_v8(&T.sal[(size_t)sa * SAL_U4 + 4], g4, g5);
             st[0] = g5.x; st[1] = g5.y; st[2] = g5.z; st[3] = g4.x; st[4] = g4.y;
         }
-        sha1_compress_fma(st, W, T.n_sa != 0u ? 1u : 0u);   // (n_sa >= 1: an opaque 1)
+        if (!(skip & 8u)) sha1_compress_fma(st, W, T.n_sa != 0u ? 1u : 0u);   // (n_sa >= 1: an opaque 1)
         if (it == 0) ck_sha = clock64();
     }
     // ICV = first 96 bits of the outer digest (RFC 2404)
@@ -1996,6 +2002,9 @@ __device__ __forceinline__ void roles_lane_consumed(uint32_t *p, uint32_t q)
 #ifndef NBA_ROLES_WARM        // experiment: lanes' warm-up pass (0 off, 1 all warps, 2 warp 0, 3 warps 0-3)
 #define NBA_ROLES_WARM 0
 #endif
+#ifndef NBA_ROLES_WARM_D      // experiment: the warm-up packet's length (0: the lane's own, up to 114)
+#define NBA_ROLES_WARM_D 0
+#endif
 #ifndef NBA_ROLES_RK_ASYNC    // lanes: round keys 3..10 by cp.async from the SA's schedule instead of
 #define NBA_ROLES_RK_ASYNC 0  //   expanded from the key (1)
 #endif
@@ -2403,7 +2412,7 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
     // the sequencers' batch 0 -- the first pass over the lane code in a launch
     // is ~1.5x slower than the next ones
     const bool warm_me = cached && R.n_slots < SLOT_CACHE &&
-                         (NBA_ROLES_WARM == 1 || (NBA_ROLES_WARM == 2 && warp == 0) ||
+                         (NBA_ROLES_WARM == 1 || NBA_ROLES_WARM == 4 || (NBA_ROLES_WARM == 2 && warp == 0) ||
                           (NBA_ROLES_WARM == 3 && warp < 4u));
     if (NBA_ROLES_WARM && cached && R.n_slots < SLOT_CACHE && tid == 0) {
         BatchArgs bw = sl[R.first % R.n_slots];
@@ -2412,7 +2421,8 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
         sc[R.n_slots] = bw;
     }
     if (NBA_ROLES_WARM) __syncthreads();
-    if (warm_me) f = Fields{0u, 0u, f.have ? min(max(f.D, MIN_D), 114u) : 50u, 0u, 14u, true};
+    if (warm_me) f = Fields{0u, 0u, NBA_ROLES_WARM_D ? NBA_ROLES_WARM_D : (f.have ? min(max(f.D, MIN_D), 114u) : 50u),
+                            0u, 14u, true};
     else if (f.have) prefetch_l2(sl[R.first % R.n_slots].in_buf + f.inoff);
     // batch bi's record when it was read ahead (at the end of iteration bi - 1,
     // from a poll issued during it): neither the poll nor the record load then
@@ -2456,7 +2466,13 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
         if (NBA_ROLES_RK_ASYNC && cand) rk_async_wait();
         if (f.have) {
             if (q != 0u) {
-                esp_packet(T, B, L, H, lane4r, tid, f.sa, f.D | INFO_OK, q, f.inoff, f.outoff, pp, nullptr);
+                // (warm-up mode 4: warp groups enter the code at the CTR precompute,
+                // the AES step, the SHA-1 block, the tail)
+                const uint32_t g = warp & 3u;
+                const uint32_t skip = (NBA_ROLES_WARM == 4 && dummy) ? (g == 0u ? 0u : g == 1u ? 1u : g == 2u ? 3u : 11u)
+                                                                     : 0u;
+                esp_packet(T, B, L, H, lane4r, tid, f.sa, f.D | INFO_OK, q, f.inoff, f.outoff, pp, nullptr,
+                           nullptr, 0u, skip);
                 if (dummy) {
                     f = fn;
                     if (f.have) prefetch_l2(sl[R.first % R.n_slots].in_buf + f.inoff);
