@@ -499,7 +499,9 @@ int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, u
                     cudaMalloc(&r->rq.cum, (size_t)Lc * 16u * sizeof(uint32_t)) != cudaSuccess ||
                     cudaMemset(r->rq.cum, 0, (size_t)Lc * 16u * sizeof(uint32_t)) != cudaSuccess ||
                     cudaMalloc(&r->rq.ptot, (size_t)2u * npro * t->n_sa * sizeof(uint32_t)) != cudaSuccess ||
-                    cudaMalloc(&r->rq.scratch, (size_t)Lc * 256u) != cudaSuccess) {
+                    cudaMalloc(&r->rq.scratch, (size_t)Lc * 256u) != cudaSuccess ||
+                    cudaMalloc(&r->rq.hist0, (size_t)t->n_sa * t->grid_fused * sizeof(uint32_t)) != cudaSuccess ||
+                    cudaMalloc(&r->rq.tot0, (size_t)t->n_sa * sizeof(uint32_t)) != cudaSuccess) {
                     nba_ipsec_ring_destroy(r);
                     return NBA_IPSEC_ENOMEM;
                 }
@@ -515,6 +517,10 @@ int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, u
                 r->rq.sorted = (!one_len && n_slots > ROLES_NREC) ? 1u : 0u;
                 const char *rs = std::getenv("NBA_IPSEC_ROLES_SORTED");
                 if (rs) r->rq.sorted = (std::atoi(rs) != 0 && n_slots > ROLES_NREC) ? 1u : 0u;
+                // fixed-slot mode: every CTA numbers a launch's first batch (its row
+                // scans cover up to 160 CTAs)
+                r->rq.boot = (!r->rq.sorted && t->grid_fused <= 160 && !std::getenv("NBA_IPSEC_ROLES_NOBOOT"))
+                                 ? 1u : 0u;
                 const char *re = std::getenv("NBA_IPSEC_RING_ROLES");
                 r->roles = re ? std::atoi(re) != 0 : ((one_len && max_len <= 1010u) || r->rq.sorted);
             }
@@ -809,7 +815,7 @@ int nba_ipsec_ring_destroy(nba_ipsec_ring *r)
         if (r->d_slots || r->hist_b || r->d_in_slots || r->hkey_b || r->hval_b || r->rq.ctl)
             cudaDeviceSynchronize();   // a run may still be in flight
         for (void *q : {(void *)r->rq.ctl, (void *)r->rq.rec, (void *)r->rq.ptot, (void *)r->rq.scratch,
-                        (void *)r->rq.cum})
+                        (void *)r->rq.cum, (void *)r->rq.hist0, (void *)r->rq.tot0})
             if (q) cudaFree(q);
         if (r->d_slots) cudaFree(r->d_slots);
         if (r->hist_b) cudaFree(r->hist_b);

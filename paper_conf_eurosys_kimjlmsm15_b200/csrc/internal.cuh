@@ -215,7 +215,8 @@ constexpr uint32_t ROLES_NREC = 4;          // batches of records in flight
 constexpr uint32_t ROLES_MAX_SA = 2048;     // per-warp SA counters in a sequencer's shared memory
 constexpr uint32_t ROLES_RPP_MAX = 16416;   // packets per sequencer and batch (shared stash: 36 lane
                                             //   CTAs x 456 packets, a 65,536-packet batch at 4 sequencers)
-constexpr uint32_t ROLES_CTL_WORDS = 2u * ROLES_NREC + 2u;   // ready[], consumed[], pbar, exit
+constexpr uint32_t ROLES_CTL_WORDS = 2u * ROLES_NREC + 4u;   // ready[], consumed[], pbar, exit,
+                                                             //   batch-0 bootstrap barrier / count
 struct RolesBufs {
     uint32_t *ctl;      // [ROLES_CTL_WORDS] hand-off counters (zero between launches)
     uint32_t *rec;      // [ROLES_NREC][(grid - npro) * 512] per-packet sequence numbers (0: drop),
@@ -224,6 +225,9 @@ struct RolesBufs {
     uint32_t *cum;      // [(grid - npro) * 16] sorted mode: each lane warp's assigned work so far
     uint32_t sorted;    // 1: per-batch length-sorted lane slots (mixed-length rings)
     uint32_t stage;     // 1: sequencers stage SA indices / lengths by bulk copy (16-B aligned arrays)
+    uint32_t boot;      // 1: every CTA numbers batch 0 (fixed-slot mode), the sequencers start at batch 1
+    uint32_t *hist0;    // [n_sa][grid] bootstrap: per-(SA, CTA) counts -> exclusive prefixes over the CTAs
+    uint32_t *tot0;     // [n_sa] bootstrap: the SA's valid packets in batch 0
     uint32_t *ptot;     // [2][npro][n_sa] per-sequencer per-SA valid-packet totals
     uint8_t *scratch;   // [(grid - npro) * 256] output lines of the lanes' warm-up experiment
     uint32_t npro;      // sequencer CTAs

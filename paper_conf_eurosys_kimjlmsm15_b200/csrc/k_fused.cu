@@ -2015,6 +2015,120 @@ __device__ __forceinline__ void roles_lane_consumed(uint32_t *p, uint32_t q)
 #define NBA_ROLES_AG 8
 #endif
 
+// Batch-0 bootstrap (fixed-slot mode): the sequencers would need ~20 us for a
+// launch's first batch (their ranking is compute-bound and nothing overlaps
+// it), so every CTA numbers batch 0 instead, the pipelined ring's way: CTA c
+// takes packets [c ppc0, (c + 1) ppc0) (one per thread), ranks them per SA
+// (12-ballot groups in each warp, the warps' group sizes in shared-memory
+// rows) and writes its per-SA counts into column c of hist0 (zeroed by CTA c
+// first); after a grid barrier each warp turns one SA row into exclusive
+// prefixes over the CTAs in place (and the row total into tot0); after a
+// second one each CTA writes its packets' records (q = the SA's counter + 1 +
+// prefix + rank, 0 = drop, saturating as the sequencers) and the last CTA
+// publishes batch 0 as the sequencers would (ready[0] += P, pbar += P).  The
+// shared memory is scratch here: nothing else has used it yet in this launch.
+__device__ __noinline__ void roles_boot0(const DevTable &T, const BatchArgs *slots, RingRun R, RolesBufs Q,
+                                         uint8_t *smem)
+{
+    const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
+    const uint32_t G = gridDim.x, c = blockIdx.x, n_sa = T.n_sa;
+    const BatchArgs B = slots[R.first % R.n_slots];
+    const uint32_t n = B.n, ppc0 = (n + G - 1u) / G, i = c * ppc0 + tid;
+    const bool in = tid < ppc0 && i < n;
+    const uint32_t s = in ? B.sa_idx[i] : INVALID_SA, D = in ? (uint32_t)B.in_len[i] : 0u;
+    const bool cand = in && s < n_sa && D >= MIN_D && D <= MAX_D;
+    // the SA's counter before batch 0, read before the barriers: with no batch
+    // past the record ring, sequencer 0 can finish the run and write back T.seq
+    // while a slow CTA is still here
+    const uint32_t seq0 = cand ? __ldcg(&T.seq[s]) : 0u;
+    uint16_t *rows = reinterpret_cast<uint16_t *>(smem);                  // [16][n_sa]
+    uint32_t *bar = Q.ctl + 2u * ROLES_NREC + 2u, *done = bar + 1;
+    for (uint32_t k = tid; k < 16u * n_sa; k += F_THREADS) rows[k] = 0;
+    for (uint32_t sa = tid; sa < n_sa; sa += F_THREADS) Q.hist0[(size_t)sa * G + c] = 0u;
+    __syncthreads();
+    const uint32_t key = cand ? s : 0x800u;
+    uint32_t peers = 0xffffffffu;
+#pragma unroll
+    for (uint32_t bit = 0; bit < 12u; bit++) {
+        const bool on = (key >> bit) & 1u;
+        const uint32_t m = __ballot_sync(0xffffffffu, on);
+        peers &= on ? m : ~m;
+    }
+    const uint32_t leader = (uint32_t)__ffs(peers) - 1u;
+    if (cand && lane == leader) rows[warp * n_sa + s] = (uint16_t)__popc(peers);
+    __syncthreads();
+    uint32_t pre = 0u, tot = 0u;
+    bool first = true;                                   // the lowest warp holding the SA
+    if (cand)
+        for (uint32_t w = 0; w < 16u; w++) {
+            const uint32_t v = rows[w * n_sa + s];
+            if (w < warp) {
+                pre += v;
+                first = first && v == 0u;
+            }
+            tot += v;
+        }
+    const uint32_t rank = pre + __popc(peers & lanemask_lt());
+    if (cand && lane == leader && first) Q.hist0[(size_t)s * G + c] = tot;
+    __syncthreads();
+    if (tid == 0) {
+        __threadfence();
+        roles_red_rel(bar, 1u);
+        roles_wait_geq(bar, G);
+    }
+    __syncthreads();
+    // exclusive prefixes over the CTAs, one warp per SA row (lane l: columns [5l, 5l + 5))
+    for (uint32_t sa = c + warp * G; sa < n_sa; sa += 16u * G) {
+        uint32_t v[5], sum = 0;
+#pragma unroll
+        for (uint32_t k = 0; k < 5u; k++) {
+            const uint32_t col = 5u * lane + k;
+            v[k] = col < G ? __ldcg(&Q.hist0[(size_t)sa * G + col]) : 0u;
+            sum += v[k];
+        }
+        uint32_t x = sum;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+            if (lane >= (uint32_t)o) x += y;
+        }
+        uint32_t run = x - sum;
+#pragma unroll
+        for (uint32_t k = 0; k < 5u; k++) {
+            const uint32_t col = 5u * lane + k;
+            if (col < G) Q.hist0[(size_t)sa * G + col] = run;
+            run += v[k];
+        }
+        if (lane == 31u) Q.tot0[sa] = x;
+    }
+    __syncthreads();
+    if (tid == 0) {
+        __threadfence();
+        roles_red_rel(bar, 1u);
+        roles_wait_geq(bar, 2u * G);
+    }
+    __syncthreads();
+    if (in) {
+        uint32_t q = 0u;
+        if (cand) {
+            const unsigned long long q64 = (unsigned long long)seq0 + __ldcg(&Q.hist0[(size_t)s * G + c]) +
+                                           rank + 1ull;
+            q = q64 <= 0xffffffffull ? (uint32_t)q64 : 0u;
+        }
+        Q.rec[i] = q;                                    // record slot 0 (batch 0)
+    }
+    __syncthreads();
+    if (tid == 0) {
+        __threadfence();
+        if (atomicAdd(done, 1u) == G - 1u) {
+            __threadfence();
+            roles_red_rel(Q.ctl, Q.npro);                              // ready[0]
+            roles_red_rel(Q.ctl + 2u * ROLES_NREC, Q.npro);            // pbar: batch 0's arrivals
+        }
+    }
+    __syncthreads();
+}
+
 // Sorted mode (mixed-length rings), per lane CTA of this sequencer, one warp
 // each: the CTA's packets in a stable counting sort by HMAC length bin
 // (longest first, invalid last), cut into runs of 32 sorted positions; run r
@@ -2119,13 +2233,15 @@ __device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchAr
                   "sequencer shared memory");
     uint32_t *ready = Q.ctl, *consumed = Q.ctl + ROLES_NREC, *pbar = Q.ctl + 2u * ROLES_NREC;
     uint16_t *mycnt = cnt + warp * ROLES_MAX_SA;
-    for (uint32_t s = tid; s < n_sa; s += F_THREADS) seqs[s] = __ldcg(&T.seq[s]);
+    for (uint32_t s = tid; s < n_sa; s += F_THREADS)
+        seqs[s] = Q.boot ? (uint32_t)min((unsigned long long)__ldcg(&T.seq[s]) + __ldcg(&Q.tot0[s]), 0xffffffffull)
+                         : __ldcg(&T.seq[s]);
     for (uint32_t s = lane; s < n_sa; s += 32u) mycnt[s] = 0;
     if (tid == 0) tbar_init(mbar);
     __syncthreads();
     // this sequencer's lane CTAs [cbeg, cend): its packet range is theirs
     const uint32_t cbeg = p * Lc / P, cend = (p + 1u) * Lc / P;
-    for (uint32_t bi = 0; bi < R.n_batches; bi++) {
+    for (uint32_t bi = Q.boot ? 1u : 0u; bi < R.n_batches; bi++) {
         const BatchArgs B = slots[(R.first + bi) % R.n_slots];
         const uint32_t n = B.n, ppc = (n + Lc - 1u) / Lc;
         const uint32_t r0 = min(n, cbeg * ppc), r1 = min(n, cend * ppc), rpp = r1 - r0;
@@ -2133,7 +2249,7 @@ __device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchAr
         const uint32_t w0 = min(r1, r0 + warp * spw), w1 = min(r1, w0 + spw);
         // the next batch's metadata lines into L2 (ahead of its phase A; batch 0's
         // at the start)
-        for (uint32_t nb = bi == 0u ? 0u : bi + 1u; nb <= bi + 1u && nb < R.n_batches; nb++) {
+        for (uint32_t nb = bi == (Q.boot ? 1u : 0u) ? bi : bi + 1u; nb <= bi + 1u && nb < R.n_batches; nb++) {
             const BatchArgs Bn = slots[(R.first + nb) % R.n_slots];
             const uint32_t pn = (Bn.n + Lc - 1u) / Lc, a0 = min(Bn.n, cbeg * pn), a1 = min(Bn.n, cend * pn);
             const uint32_t l16 = a1 > a0 ? (2u * (a1 - a0) + 127u) / 128u + 1u : 0u;
@@ -2189,7 +2305,7 @@ __device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchAr
             for (uint32_t i = r0 - hl + nbl / 2u + tid; i < r1; i += F_THREADS)
                 raw_len[i - (r0 - hl)] = B.in_len[i];
             __syncthreads();
-            tables_bulk_wait(mbar, bi & 1u);
+            tables_bulk_wait(mbar, (bi - (Q.boot ? 1u : 0u)) & 1u);   // (one phase per staged batch)
         } else {
             for (uint32_t i = r0 + tid; i < r1; i += F_THREADS) {
                 sav[i - r0] = B.sa_idx[i];
@@ -2603,6 +2719,7 @@ k_fused_ring_roles(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, Rol
     extern __shared__ __align__(16) uint8_t smem[];
     if (R.n_batches == 0) return;
     if (R.ts && blockIdx.x == 0 && threadIdx.x == 0) R.ts[0] = gtimer();
+    if (Q.boot) roles_boot0(T, slots, R, Q, smem);
     if (blockIdx.x < Q.npro) roles_sequencer(T, slots, R, Q, smem, blockIdx.x);
     else if (Q.sorted) roles_lanes_sorted(T, W, slots, R, Q, smem, blockIdx.x - Q.npro);
     else roles_lanes(T, W, slots, R, Q, smem, blockIdx.x - Q.npro);

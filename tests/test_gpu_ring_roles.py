@@ -179,3 +179,15 @@ def test_roles_ring_sequencer_plain_loads(sorted_mode, monkeypatch):
     hb = [gen.make_batch(7001, s, 40, cfg_id=78, batch=i) for i, s in enumerate(sizes)]
     hb[0].sa_idx[::61] = 77
     _roles_vs_oracle(p, 40, hb, [6, 7])
+
+
+@pytest.mark.parametrize("sizes", [(64, 64, 64), ("imix", 300)])
+def test_roles_ring_without_bootstrap(sizes, monkeypatch):
+    """Fixed-slot rings with the sequencers numbering batch 0 too
+    (NBA_IPSEC_ROLES_NOBOOT; by default every CTA numbers a launch's first
+    batch), runs of 4 + 1 + 6 batches."""
+    monkeypatch.setenv("NBA_IPSEC_ROLES_NOBOOT", "1")
+    p = gen.make_sas(200, cfg_id=79)
+    hb = [gen.make_batch(12000, s, 200, cfg_id=79, batch=i) for i, s in enumerate(sizes)]
+    hb[0].sa_idx[::71] = 999
+    _roles_vs_oracle(p, 200, hb, [4, 1, 6])
