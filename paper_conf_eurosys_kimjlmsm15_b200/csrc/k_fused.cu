@@ -2005,6 +2005,9 @@ __device__ __forceinline__ void roles_lane_consumed(uint32_t *p, uint32_t q)
 #ifndef NBA_ROLES_WARM_D      // experiment: the warm-up packet's length (0: the lane's own, up to 114)
 #define NBA_ROLES_WARM_D 0
 #endif
+#ifndef NBA_ROLES_SAL_AHEAD   // lanes: the next packet's SA line loaded at the end of an iteration
+#define NBA_ROLES_SAL_AHEAD 0       // (measured: 64 B 20.5 -> 20.7 us, 128 B 29.3 -> 28.4, 512 B 73.6 -> 74.6, 1024 B 134 -> 137)
+#endif
 #ifndef NBA_ROLES_RK_ASYNC    // lanes: round keys 3..10 by cp.async from the SA's schedule instead of
 #define NBA_ROLES_RK_ASYNC 0  //   expanded from the key (1)
 #endif
@@ -2545,6 +2548,8 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
     // waits on the critical path
     uint32_t q = 0u, rv_next = 0u;
     bool got = false;
+    PktPre pp_ahead = {};                  // NBA_ROLES_SAL_AHEAD: the next packet's SA line
+    bool have_ahead = false;
     for (int32_t bs = warm_me ? -1 : 0; bs < (int32_t)R.n_batches; bs++) {
         const bool dummy = bs < 0;
         const uint32_t bi = dummy ? 0u : (uint32_t)bs;
@@ -2552,7 +2557,10 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
         const Fields fn = dummy ? f0 : fields_of(bi + 1u);
         const bool cand = candidate(f);
         PktPre pp = {};
-        if (cand) {
+        if (NBA_ROLES_SAL_AHEAD && cand && have_ahead) {
+            pp = pp_ahead;                                 // loaded at the end of the last iteration
+            expand_key_lane(lane4r, pp.r0, pp.r1, pp.r2, L, H, tid);
+        } else if (cand) {
             if (NBA_ROLES_RK_ASYNC) {
                 // round keys 3..10 copied from the SA's schedule (cp.async into the
                 // lane's own slots), 1..2 from its SA line: no expansion chain
@@ -2606,6 +2614,12 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
         }
         // the next packet's payload line into L2 (its offset has arrived by now)
         if (fn.have) prefetch_l2(sl[(R.first + bi + 1u) % R.n_slots].in_buf + fn.inoff);
+        // (NBA_ROLES_SAL_AHEAD) the next packet's SA line, in flight across the loop's tail
+        have_ahead = false;
+        if (NBA_ROLES_SAL_AHEAD && candidate(fn)) {
+            pp_ahead = load_pkt_pre(T, sl[(R.first + bi + 1u) % R.n_slots].in_buf, fn.sa, fn.inoff, true, 0u);
+            have_ahead = true;
+        }
         if (R.ts && lane == 0) atomicMax(&R.ts[1u + bi], gtimer());
         // the next batch's record, if its sequencers had published it when
         // lane 0's poll (issued above) read the count
