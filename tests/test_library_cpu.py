@@ -59,3 +59,16 @@ def test_host_hmac_midstates_rfc2202(name):
     inner = pysha1.finish([int(x) for x in hin], msg_of(r), 64)
     outer = pysha1.finish([int(x) for x in hout], inner, 64)
     assert outer.hex() == r["digest"]
+
+
+def test_ring_form_constants_match_header():
+    """The binding's ring-form constants are the header's NBA_IPSEC_RING_* values
+    (GRAPH, PERSISTENT, PIPELINED, FREE, ROLES)."""
+    import os
+    import re
+    from paper_conf_eurosys_kimjlmsm15_b200 import nba_ipsec
+    hdr = open(os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "include",
+                            "nba_ipsec.h")).read()
+    vals = {m.group(1): int(m.group(2)) for m in re.finditer(r"NBA_IPSEC_RING_([A-Z]+) = (\d+)", hdr)}
+    for name in ("GRAPH", "PERSISTENT", "PIPELINED", "FREE", "ROLES"):
+        assert getattr(nba_ipsec.Ring, name) == vals[name], name
