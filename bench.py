@@ -345,6 +345,21 @@ def measure_outbound(ctx, args, cfg_id, size, steps, warmup, full):
         torch.cuda.synchronize()
         res["graph_ms"] = e0.elapsed_time(e1)
         g.close()
+        # (b') the software-pipelined ring form on the same slots (the default
+        # before the role-split ring; set_form), when the ring's default is
+        # another persistent form
+        if form == "roles":
+            pr = t.ring(slots)
+            pr.set_form(nba_ipsec.Ring.PIPELINED)
+            pr.run_batches(2 * R)
+            torch.cuda.synchronize()
+            gpu_lead(torch)
+            e0.record()
+            pr.run_batches(steps)
+            e1.record()
+            torch.cuda.synchronize()
+            res["pipe_ring_ms"] = e0.elapsed_time(e1)
+            pr.close()
         # (c) isolated batches: L2 flushed before each, one event pair per batch
         iso = min(steps, 50)
         ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
@@ -772,6 +787,7 @@ def run_ours(args):
     ctr_all = ctx.sum_all(head["ctr"])
     launch_ms = ctx.max_ms(head.get("launch_loop_ms", 0.0))
     graph_ms = ctx.max_ms(head.get("graph_ms", 0.0))
+    pipe_ms = ctx.max_ms(head.get("pipe_ring_ms", 0.0))
     if ctx.rank == 0:
         clk = head["clk"].summary()
         nm = gen.CONFIGS[main_cfg]["name"]
@@ -824,6 +840,7 @@ def run_ours(args):
             "clocks": clk,
             "compare": {"process_batch_loop_us": 1e3 * launch_ms / steps,
                         "graph_replay_us": 1e3 * graph_ms / steps,
+                        "pipelined_ring_us": (1e3 * pipe_ms / steps) if pipe_ms else None,
                         "isolated_batch_us_mean": 1e3 * float(np.mean(head["iso_ms"])),
                         "ring_us": 1e3 * agg["ms_per_step"],
                         "launches_per_batch_unringed": head.get("lpb")},

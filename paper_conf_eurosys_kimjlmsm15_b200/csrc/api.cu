@@ -501,7 +501,9 @@ int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, u
                     cudaMalloc(&r->rq.ptot, (size_t)2u * npro * t->n_sa * sizeof(uint32_t)) != cudaSuccess ||
                     cudaMalloc(&r->rq.scratch, (size_t)Lc * 256u) != cudaSuccess ||
                     cudaMalloc(&r->rq.hist0, (size_t)t->n_sa * t->grid_fused * sizeof(uint32_t)) != cudaSuccess ||
-                    cudaMalloc(&r->rq.tot0, (size_t)t->n_sa * sizeof(uint32_t)) != cudaSuccess) {
+                    cudaMalloc(&r->rq.tot0, (size_t)t->n_sa * sizeof(uint32_t)) != cudaSuccess ||
+                    cudaMalloc(&r->rq.rows0, (size_t)t->grid_fused * 16u * t->n_sa * sizeof(uint16_t)) != cudaSuccess ||
+                    cudaMalloc(&r->rq.rank0, (size_t)t->grid_fused * 512u * sizeof(uint16_t)) != cudaSuccess) {
                     nba_ipsec_ring_destroy(r);
                     return NBA_IPSEC_ENOMEM;
                 }
@@ -815,7 +817,8 @@ int nba_ipsec_ring_destroy(nba_ipsec_ring *r)
         if (r->d_slots || r->hist_b || r->d_in_slots || r->hkey_b || r->hval_b || r->rq.ctl)
             cudaDeviceSynchronize();   // a run may still be in flight
         for (void *q : {(void *)r->rq.ctl, (void *)r->rq.rec, (void *)r->rq.ptot, (void *)r->rq.scratch,
-                        (void *)r->rq.cum, (void *)r->rq.hist0, (void *)r->rq.tot0})
+                        (void *)r->rq.cum, (void *)r->rq.hist0, (void *)r->rq.tot0, (void *)r->rq.rows0,
+                        (void *)r->rq.rank0})
             if (q) cudaFree(q);
         if (r->d_slots) cudaFree(r->d_slots);
         if (r->hist_b) cudaFree(r->hist_b);

@@ -228,6 +228,8 @@ struct RolesBufs {
     uint32_t boot;      // 1: every CTA numbers batch 0 (fixed-slot mode), the sequencers start at batch 1
     uint32_t *hist0;    // [n_sa][grid] bootstrap: per-(SA, CTA) counts -> exclusive prefixes over the CTAs
     uint32_t *tot0;     // [n_sa] bootstrap: the SA's valid packets in batch 0
+    uint16_t *rows0;    // [grid][16][n_sa] bootstrap: per-warp SA group sizes of each CTA
+    uint16_t *rank0;    // [grid * 512] bootstrap: each packet's rank among its CTA's packets of its SA
     uint32_t *ptot;     // [2][npro][n_sa] per-sequencer per-SA valid-packet totals
     uint8_t *scratch;   // [(grid - npro) * 256] output lines of the lanes' warm-up experiment
     uint32_t npro;      // sequencer CTAs

@@ -2022,16 +2022,18 @@ __device__ __forceinline__ void roles_lane_consumed(uint32_t *p, uint32_t q)
 // launch's first batch (their ranking is compute-bound and nothing overlaps
 // it), so every CTA numbers batch 0 instead, the pipelined ring's way: CTA c
 // takes packets [c ppc0, (c + 1) ppc0) (one per thread), ranks them per SA
-// (12-ballot groups in each warp, the warps' group sizes in shared-memory
-// rows) and writes its per-SA counts into column c of hist0 (zeroed by CTA c
-// first); after a grid barrier each warp turns one SA row into exclusive
-// prefixes over the CTAs in place (and the row total into tot0); after a
-// second one each CTA writes its packets' records (q = the SA's counter + 1 +
-// prefix + rank, 0 = drop, saturating as the sequencers) and the last CTA
-// publishes batch 0 as the sequencers would (ready[0] += P, pbar += P).  The
-// shared memory is scratch here: nothing else has used it yet in this launch.
-__device__ __noinline__ void roles_boot0(const DevTable &T, const BatchArgs *slots, RingRun R, RolesBufs Q,
-                                         uint8_t *smem)
+// (12-ballot groups in each warp, the warps' group sizes in rows in global
+// memory, so the lane CTAs' shared memory -- T-tables in flight, slot table --
+// is untouched), writes each packet's rank to rank0 and its per-SA counts into
+// column c of hist0 (zeroed by CTA c first); after a grid barrier each warp
+// turns one SA row into exclusive prefixes over the CTAs in place (and the row
+// total into tot0); after a second barrier batch 0's numbers are known: a lane
+// computes its packet's q = SA counter + 1 + hist0[sa][i / ppc0] + rank0[i]
+// (saturating as the sequencers) without a record, and the last CTA through
+// counts batch 0 as published for the sequencers' bookkeeping (ready[0] += P,
+// pbar += P).
+__device__ __forceinline__ uint32_t roles_boot0(const DevTable &T, const BatchArgs *slots, const RingRun &R,
+                                                const RolesBufs &Q, uint32_t sa_mine)
 {
     const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
     const uint32_t G = gridDim.x, c = blockIdx.x, n_sa = T.n_sa;
@@ -2040,15 +2042,21 @@ __device__ __noinline__ void roles_boot0(const DevTable &T, const BatchArgs *slo
     const bool in = tid < ppc0 && i < n;
     const uint32_t s = in ? B.sa_idx[i] : INVALID_SA, D = in ? (uint32_t)B.in_len[i] : 0u;
     const bool cand = in && s < n_sa && D >= MIN_D && D <= MAX_D;
-    // the SA's counter before batch 0, read before the barriers: with no batch
-    // past the record ring, sequencer 0 can finish the run and write back T.seq
-    // while a slow CTA is still here
-    const uint32_t seq0 = cand ? __ldcg(&T.seq[s]) : 0u;
-    uint16_t *rows = reinterpret_cast<uint16_t *>(smem);                  // [16][n_sa]
+    uint16_t *rows = Q.rows0 + (size_t)c * 16u * n_sa;                   // [16][n_sa]
     uint32_t *bar = Q.ctl + 2u * ROLES_NREC + 2u, *done = bar + 1;
-    for (uint32_t k = tid; k < 16u * n_sa; k += F_THREADS) rows[k] = 0;
+#if NBA_ROLES_TRACE
+    if (R.ts && tid == 0) atomicMax(RLT(1, 6), gtimer());   // the latest boot start
+#endif
+#if NBA_ROLES_TRACE
+    if (R.ts && c == 0 && tid == 0) *RLT(0, 0) = gtimer();
+#endif
+    for (uint32_t k = tid; k < 2u * n_sa; k += F_THREADS)               // 16 x n_sa u16 = 2 n_sa uint4
+        reinterpret_cast<uint4 *>(rows)[k] = make_uint4(0u, 0u, 0u, 0u);
     for (uint32_t sa = tid; sa < n_sa; sa += F_THREADS) Q.hist0[(size_t)sa * G + c] = 0u;
     __syncthreads();
+#if NBA_ROLES_TRACE
+    if (R.ts && c == 0 && tid == 0) *RLT(0, 1) = gtimer();
+#endif
     const uint32_t key = cand ? s : 0x800u;
     uint32_t peers = 0xffffffffu;
 #pragma unroll
@@ -2064,22 +2072,31 @@ __device__ __noinline__ void roles_boot0(const DevTable &T, const BatchArgs *slo
     bool first = true;                                   // the lowest warp holding the SA
     if (cand)
         for (uint32_t w = 0; w < 16u; w++) {
-            const uint32_t v = rows[w * n_sa + s];
+            const uint32_t v = __ldcg(&rows[w * n_sa + s]);
             if (w < warp) {
                 pre += v;
                 first = first && v == 0u;
             }
             tot += v;
         }
-    const uint32_t rank = pre + __popc(peers & lanemask_lt());
+    if (in) Q.rank0[i] = (uint16_t)(pre + __popc(peers & lanemask_lt()));
     if (cand && lane == leader && first) Q.hist0[(size_t)s * G + c] = tot;
     __syncthreads();
+#if NBA_ROLES_TRACE
+    if (R.ts && c == 0 && tid == 0) *RLT(0, 2) = gtimer();
+#endif
     if (tid == 0) {
+#if NBA_ROLES_TRACE
+        if (R.ts) atomicMax(RLT(0, 6), gtimer());       // the latest arrival (any CTA)
+#endif
         __threadfence();
         roles_red_rel(bar, 1u);
         roles_wait_geq(bar, G);
     }
     __syncthreads();
+#if NBA_ROLES_TRACE
+    if (R.ts && c == 0 && tid == 0) *RLT(0, 3) = gtimer();
+#endif
     // exclusive prefixes over the CTAs, one warp per SA row (lane l: columns [5l, 5l + 5))
     for (uint32_t sa = c + warp * G; sa < n_sa; sa += 16u * G) {
         uint32_t v[5], sum = 0;
@@ -2104,32 +2121,39 @@ __device__ __noinline__ void roles_boot0(const DevTable &T, const BatchArgs *slo
         }
         if (lane == 31u) Q.tot0[sa] = x;
     }
+    const uint32_t seq_mine = sa_mine < n_sa ? __ldcg(&T.seq[sa_mine]) : 0u;   // (before barrier 2)
     __syncthreads();
+#if NBA_ROLES_TRACE
+    if (R.ts && c == 0 && tid == 0) *RLT(0, 4) = gtimer();
+#endif
     if (tid == 0) {
+#if NBA_ROLES_TRACE
+        if (R.ts) atomicMax(RLT(0, 7), gtimer());
+#endif
         __threadfence();
         roles_red_rel(bar, 1u);
         roles_wait_geq(bar, 2u * G);
-    }
-    __syncthreads();
-    if (in) {
-        uint32_t q = 0u;
-        if (cand) {
-            const unsigned long long q64 = (unsigned long long)seq0 + __ldcg(&Q.hist0[(size_t)s * G + c]) +
-                                           rank + 1ull;
-            q = q64 <= 0xffffffffull ? (uint32_t)q64 : 0u;
-        }
-        Q.rec[i] = q;                                    // record slot 0 (batch 0)
-    }
-    __syncthreads();
-    if (tid == 0) {
-        __threadfence();
         if (atomicAdd(done, 1u) == G - 1u) {
-            __threadfence();
             roles_red_rel(Q.ctl, Q.npro);                              // ready[0]
             roles_red_rel(Q.ctl + 2u * ROLES_NREC, Q.npro);            // pbar: batch 0's arrivals
         }
     }
     __syncthreads();
+#if NBA_ROLES_TRACE
+    if (R.ts && c == 0 && tid == 0) *RLT(0, 5) = gtimer();
+#endif
+    return seq_mine;
+}
+
+// A lane's batch-0 sequence number after the bootstrap (0 = drop); seq0 = the
+// SA's counter, read before the bootstrap's barriers.
+__device__ __forceinline__ uint32_t roles_boot_q(const RolesBufs &Q, const BatchArgs &B, uint32_t i,
+                                                 uint32_t sa, uint32_t seq0)
+{
+    const uint32_t G = gridDim.x, ppc0 = (B.n + G - 1u) / G;
+    const unsigned long long q64 = (unsigned long long)seq0 + __ldcg(&Q.hist0[(size_t)sa * G + i / ppc0]) +
+                                   __ldcg(&Q.rank0[i]) + 1ull;
+    return q64 <= 0xffffffffull ? (uint32_t)q64 : 0u;
 }
 
 // Sorted mode (mixed-length rings), per lane CTA of this sequencer, one warp
@@ -2236,6 +2260,7 @@ __device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchAr
                   "sequencer shared memory");
     uint32_t *ready = Q.ctl, *consumed = Q.ctl + ROLES_NREC, *pbar = Q.ctl + 2u * ROLES_NREC;
     uint16_t *mycnt = cnt + warp * ROLES_MAX_SA;
+    if (Q.boot) roles_boot0(T, slots, R, Q, INVALID_SA);
     for (uint32_t s = tid; s < n_sa; s += F_THREADS)
         seqs[s] = Q.boot ? (uint32_t)min((unsigned long long)__ldcg(&T.seq[s]) + __ldcg(&Q.tot0[s]), 0xffffffffull)
                          : __ldcg(&T.seq[s]);
@@ -2488,13 +2513,7 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
     static_assert(sizeof(BatchArgs) % 4 == 0, "slot copy by words");
     BatchArgs *sc = reinterpret_cast<BatchArgs *>(&L.sa[0]);
     const bool cached = R.n_slots <= SLOT_CACHE;
-    if (cached)
-        for (uint32_t k = tid; k < R.n_slots * (uint32_t)(sizeof(BatchArgs) / 4); k += F_THREADS)
-            reinterpret_cast<uint32_t *>(sc)[k] = reinterpret_cast<const uint32_t *>(slots)[k];
-    const BatchArgs *sl = cached ? sc : slots;
     tables_stage(tabs, T, &L.tbar, true);
-    __syncthreads();
-    tables_bulk_wait(&L.tbar, 0u);
     const uint32_t *ready = Q.ctl;
     uint32_t *consumed = Q.ctl + ROLES_NREC;
     const uint32_t jpos = lane * 16u + warp;         // position in the CTA's packet range
@@ -2504,6 +2523,7 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
     // the SA line load and the round-key expansion run before the record is
     // needed.  Its payload's first line goes into L2 one batch ahead too.
     struct Fields { uint32_t i, sa, D, inoff, outoff; bool have; };
+    const BatchArgs *sl = slots;                     // -> the shared-memory copy below
     auto fields_of = [&](uint32_t bi) {
         Fields f = {0u, INVALID_SA, 0u, 0u, 0u, false};
         if (bi >= R.n_batches) return f;
@@ -2522,8 +2542,20 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
     auto candidate = [&](const Fields &g) {   // the oracle's step 1 (A15)
         return g.have && g.sa < n_sa && g.D >= MIN_D && g.D <= MAX_D;
     };
+    // batch 0's fields from the slot array itself (loads in flight across the
+    // bootstrap, in which every CTA numbers batch 0 while the T-table copy
+    // lands); the bootstrap also returns the packet SA's counter, read between
+    // its barriers (sequencer 0 may finish a short run and write it back after
+    // them); then the slot table into shared memory
     Fields f = fields_of(0u);
     const Fields f0 = f;
+    const uint32_t seq0 = Q.boot ? roles_boot0(T, slots, R, Q, candidate(f) ? f.sa : INVALID_SA) : 0u;
+    if (cached)
+        for (uint32_t k = tid; k < R.n_slots * (uint32_t)(sizeof(BatchArgs) / 4); k += F_THREADS)
+            reinterpret_cast<uint32_t *>(sc)[k] = reinterpret_cast<const uint32_t *>(slots)[k];
+    __syncthreads();
+    if (cached) sl = sc;
+    tables_bulk_wait(&L.tbar, 0u);
     // experiment (NBA_ROLES_WARM 1 / 2 / 3: all warps / warp 0 / warps 0-3 of
     // each lane CTA): iteration -1 runs the batch-0 code path on a dummy packet
     // (SA 0, the lane's length up to 114 bytes, read from the T-table image,
@@ -2574,6 +2606,8 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
         }
         if (dummy) {
             q = 1u;
+        } else if (Q.boot && bi == 0u) {
+            q = cand ? roles_boot_q(Q, B, f.i, f.sa, seq0) : 0u;    // (no record for batch 0)
         } else if (!got) {
 #if NBA_ROLES_TRACE
             if (R.ts && c == 0 && tid == 0) *RLT(bi, 6) = gtimer();
@@ -2733,7 +2767,6 @@ k_fused_ring_roles(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, Rol
     extern __shared__ __align__(16) uint8_t smem[];
     if (R.n_batches == 0) return;
     if (R.ts && blockIdx.x == 0 && threadIdx.x == 0) R.ts[0] = gtimer();
-    if (Q.boot) roles_boot0(T, slots, R, Q, smem);
     if (blockIdx.x < Q.npro) roles_sequencer(T, slots, R, Q, smem, blockIdx.x);
     else if (Q.sorted) roles_lanes_sorted(T, W, slots, R, Q, smem, blockIdx.x - Q.npro);
     else roles_lanes(T, W, slots, R, Q, smem, blockIdx.x - Q.npro);
