@@ -1955,9 +1955,15 @@ __device__ __forceinline__ void roles_red_rel(uint32_t *p, uint32_t v)
     asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
+__device__ __forceinline__ uint32_t roles_ld_relaxed(const uint32_t *p);
+
+// Wait until *p >= target (wrapping compare) with acquire semantics: relaxed
+// polls (an acquire load invalidates the SM's L1 on every iteration), then one
+// acquire load of the count that satisfied it.
 __device__ __forceinline__ void roles_wait_geq(const uint32_t *p, uint32_t target)
 {
-    while ((int32_t)(roles_ld_acq(p) - target) < 0) __nanosleep(32);
+    while ((int32_t)(roles_ld_relaxed(p) - target) < 0) __nanosleep(32);
+    (void)roles_ld_acq(p);
 }
 
 // The lanes' side of the hand-offs, without the acquire / release fences:
