@@ -1935,14 +1935,20 @@ k_fused_ring_free(DevTable T, DevWork W, const BatchArgs *slots, RingRun R, uint
 // ahead, so its SA line and round keys are ready before the record is read,
 // and prefetches its next payload line into L2.  The lanes' waits and counts
 // use no acquire / release fences (roles_lane_wait / roles_lane_consumed).
+// Mixed-length rings of more than ROLES_NREC slots take the sorted mode (per
+// batch length-sorted runs placed on the lane warps by cumulative cost,
+// roles_sort_slots / roles_lanes_sorted); in the fixed-slot mode a launch's
+// first batch is numbered by every CTA (roles_boot0) and the sequencers start
+// at batch 1.
 //
 // Hand-offs (counters monotonic within a launch, zeroed by the last CTA to
 // leave; s = b mod ROLES_NREC, k = b / ROLES_NREC):
 //   ready[s]    += 1 per sequencer once batch b's records are written: the
-//                  lanes wait for (k + 1) P;
+//                  lanes wait for (k + 1) P (the bootstrap counts batch 0 as P);
 //   consumed[s] += 1 per lane warp once it loaded its records of batch b: a
 //                  sequencer starts batch b only when it reads k * (lane warps);
-//   pbar        += 1 per sequencer and batch once its per-SA totals are out.
+//   pbar        += 1 per sequencer and batch once its per-SA totals are out;
+//   boot bar / done: the bootstrap's two grid barriers and its completion count.
 __device__ __forceinline__ uint32_t roles_ld_acq(const uint32_t *p)
 {
     uint32_t v;
