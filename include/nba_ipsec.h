@@ -207,10 +207,12 @@ enum { NBA_IPSEC_RING_GRAPH = 0, NBA_IPSEC_RING_PERSISTENT = 1, NBA_IPSEC_RING_P
  * other CTAs encrypt as soon as a batch's records are out, with no grid-wide
  * synchronisation between batches on their side.  ROLES fits slots with SA
  * indices, <= 512 packets per encrypting CTA and <= 2048 SAs (its sequencer
- * count: 6 for packets of <= 114 bytes, else 4; NBA_IPSEC_ROLES_P at creation
- * overrides) and is the default form of rings whose every slot holds packets
- * of one length, at most 1010 bytes (NBA_IPSEC_RING_ROLES=0/1 at creation
- * overrides).  NBA_IPSEC_EINVAL for
+ * count: 6 for packets of <= 114 bytes and for mixed lengths, else 4;
+ * NBA_IPSEC_ROLES_P at creation overrides) and is the default form of rings
+ * whose every slot holds packets of one length, at most 1010 bytes, and of
+ * mixed-length rings of more than 4 slots (there each batch's packets are
+ * sorted by length onto the encrypting warps; NBA_IPSEC_RING_ROLES=0/1 at
+ * creation overrides).  NBA_IPSEC_EINVAL for
  * graph rings or slots a form does not fit.  All give identical results. */
 int nba_ipsec_ring_form(const nba_ipsec_ring *r);
 int nba_ipsec_ring_set_form(nba_ipsec_ring *r, int form);
