@@ -696,7 +696,7 @@ static int ring_launch(nba_ipsec_ring *r, uint32_t first, uint32_t n_batches, cu
 #ifdef NBA_RING_TRACE   // debug variant: [n_batches][grid][8] phase stamps
         const size_t need = (size_t)n_batches * t->grid_fused * 16u;
 #elif defined(NBA_ROLES_TRACE)
-        const size_t need = (size_t)n_batches * 9u + 1u;   // + the role-split ring's stamps
+        const size_t need = (size_t)n_batches * 9u + 1u + 4u * 4u * 512u * 2u;   // + roles stamps, lanes
 #else
         const size_t need = (size_t)n_batches + 1u;
 #endif

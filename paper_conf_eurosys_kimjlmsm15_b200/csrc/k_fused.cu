@@ -2641,8 +2641,17 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
                 const uint32_t g = warp & 3u;
                 const uint32_t skip = (NBA_ROLES_WARM == 4 && dummy) ? (g == 0u ? 0u : g == 1u ? 1u : g == 2u ? 3u : 11u)
                                                                      : 0u;
+#if NBA_ROLES_TRACE
+                // lane timelines of batches 0..3 in lane CTAs 0..3: esp_packet start / end
+                unsigned long long *lt = (R.ts && c < 4u && bi < 4u && !dummy)
+                    ? R.ts + 1u + 9u * R.n_batches + ((size_t)(bi * 4u + c) * 512u + tid) * 2u : nullptr;
+                if (lt) lt[0] = gtimer();
+#endif
                 esp_packet(T, B, L, H, lane4r, tid, f.sa, f.D | INFO_OK, q, f.inoff, f.outoff, pp, nullptr,
                            nullptr, 0u, skip);
+#if NBA_ROLES_TRACE
+                if (lt) lt[1] = gtimer();
+#endif
                 if (dummy) {
                     f = fn;
                     if (f.have) prefetch_l2(sl[R.first % R.n_slots].in_buf + f.inoff);

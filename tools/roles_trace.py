@@ -29,13 +29,24 @@ for size in [x if x == "imix" else int(x) for x in sys.argv[1:]] or [64]:
     ring = t.ring([(*d.args(), b.n) for d in dbs])
     ring.set_form(nba_ipsec.Ring.ROLES)
     ring.run_batches(2 * R)
-    ts = torch.zeros(K * 9 + 1, dtype=torch.int64, device="cuda")
+    ts = torch.zeros(K * 9 + 1 + 4 * 4 * 512 * 2, dtype=torch.int64, device="cuda")
     ring.set_timestamps(ts)
     ring.run_batches(K)
     torch.cuda.synchronize()
     v = ts.cpu().numpy().astype(np.int64)
     ends = v[1:K + 1]
-    st = v[K + 1:].reshape(K, 8)
+    st = v[K + 1:K + 1 + 8 * K].reshape(K, 8)
+    lt = v[1 + 9 * K:].reshape(4, 4, 512, 2)
+    lanes_tl = {}
+    for bb in range(4):
+        x = lt[bb].reshape(-1, 2)
+        x = x[(x[:, 0] > 0) & (x[:, 1] > 0)]
+        if len(x):
+            rel0 = (x[:, 0] - v[0]) / 1e3
+            dur = (x[:, 1] - x[:, 0]) / 1e3
+            lanes_tl[bb] = {"n": int(len(x)), "start_us_p10_50_90": [round(float(np.percentile(rel0, q)), 2) for q in (10, 50, 90)],
+                            "dur_us_p10_50_90": [round(float(np.percentile(dur, q)), 2) for q in (10, 50, 90)],
+                            "end_us_max": round(float(((x[:, 1] - v[0]) / 1e3).max()), 2)}
     sl = slice(4, K - 1)
     med = lambda a: round(float(np.median(a[sl])) / 1e3, 2)  # noqa: E731
     out[str(size)] = {
@@ -50,6 +61,7 @@ for size in [x if x == "imix" else int(x) for x in sys.argv[1:]] or [64]:
         "lane0_wait_for_records": med(st[:, 7] - st[:, 6]),
         "records_lead_over_lane0_us": med(st[:, 6] - st[:, 5]),
         "first_batch_end_us": round(float(ends[0] - v[0]) / 1e3, 2),
+        "lanes_first_batches": lanes_tl,
         # batches 0..2 from the kernel start: sequencer 0's stamps (phase start, A, B,
         # barrier, C, D/published), lane CTA 0's wait start / records seen, batch end
         "start_batches_0_2_us": [[round(float(x - v[0]) / 1e3, 2) for x in list(st[b]) + [ends[b]]]
