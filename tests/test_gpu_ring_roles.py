@@ -191,3 +191,30 @@ def test_roles_ring_without_bootstrap(sizes, monkeypatch):
     hb = [gen.make_batch(12000, s, 200, cfg_id=79, batch=i) for i, s in enumerate(sizes)]
     hb[0].sa_idx[::71] = 999
     _roles_vs_oracle(p, 200, hb, [4, 1, 6])
+
+
+def test_roles_form_refused_where_it_does_not_fit():
+    """set_form(ROLES) is refused (NBA_IPSEC_EINVAL) for slots it does not fit:
+    more than 2048 SAs, or more than 512 packets per encrypting CTA; the ring
+    keeps its form and still equals the oracle."""
+    import torch
+    from paper_conf_eurosys_kimjlmsm15_b200 import device, nba_ipsec
+    for n_sa, n in ((2500, 5000), (16, 100_000)):
+        p = gen.make_sas(n_sa, cfg_id=80)
+        b = gen.make_batch(n, 64, n_sa, cfg_id=80)
+        sas = oracle.make_sas(p)
+        with nba_ipsec.SATable(p, device=0, max_batch=n) as t:
+            d = device.to_device(b, "cuda")
+            ring = t.ring([_slot(d)])
+            form = ring.form
+            assert form != nba_ipsec.Ring.ROLES
+            with pytest.raises(nba_ipsec.NbaIpsecError):
+                ring.set_form(nba_ipsec.Ring.ROLES)
+            assert ring.form == form
+            ring.run_batches(2)
+            torch.cuda.synchronize()
+            oracle.process_batch(sas, n_sa, b)
+            o_out, o_len, _ = oracle.process_batch(sas, n_sa, b)
+            g_out, g_len = device.fetch(d)
+            assert np.array_equal(g_len, o_len) and np.array_equal(g_out, o_out)
+            ring.close()
