@@ -495,7 +495,7 @@ int nba_ipsec_ring_create(nba_ipsec_sa_table *t, const nba_ipsec_batch *slots, u
                 r->rq.npro = npro;
                 if (cudaMalloc(&r->rq.ctl, ROLES_CTL_WORDS * sizeof(uint32_t)) != cudaSuccess ||
                     cudaMemset(r->rq.ctl, 0, ROLES_CTL_WORDS * sizeof(uint32_t)) != cudaSuccess ||
-                    cudaMalloc(&r->rq.rec, (size_t)ROLES_NREC * Lc * 512u * sizeof(uint2)) != cudaSuccess ||
+                    cudaMalloc(&r->rq.rec, (size_t)ROLES_NREC * Lc * 512u * sizeof(uint4)) != cudaSuccess ||
                     cudaMalloc(&r->rq.cum, (size_t)Lc * 16u * sizeof(uint32_t)) != cudaSuccess ||
                     cudaMemset(r->rq.cum, 0, (size_t)Lc * 16u * sizeof(uint32_t)) != cudaSuccess ||
                     cudaMalloc(&r->rq.ptot, (size_t)2u * npro * t->n_sa * sizeof(uint32_t)) != cudaSuccess ||

@@ -220,8 +220,9 @@ constexpr uint32_t ROLES_CTL_WORDS = 2u * ROLES_NREC + 4u;   // ready[], consume
 struct RolesBufs {
     uint32_t *ctl;      // [ROLES_CTL_WORDS] hand-off counters (zero between launches)
     uint32_t *rec;      // [ROLES_NREC][(grid - npro) * 512] per-packet sequence numbers (0: drop),
-                        //   by packet index; sorted mode: uint2 {q, packet in the lane CTA's
-                        //   range (0xffffffff: none)} by lane slot
+                        //   by packet index; sorted mode: uint4 {q, packet in the lane CTA's
+                        //   range | D << 9 | SA << 20 (0xffffffff: none), in_off, out_off}
+                        //   by lane slot
     uint32_t *cum;      // [(grid - npro) * 16] sorted mode: each lane warp's assigned work so far
     uint32_t sorted;    // 1: per-batch length-sorted lane slots (mixed-length rings)
     uint32_t stage;     // 1: sequencers stage SA indices / lengths by bulk copy (16-B aligned arrays)

@@ -2177,7 +2177,7 @@ __device__ __forceinline__ uint32_t roles_boot_q(const RolesBufs &Q, const Batch
 // position in the run).  Slots left without a packet get the record
 // {0, 0xffffffff}.  A run's cost: 8 (SHA-1 blocks + 1) + 3 AES steps of its
 // first (longest) packet, ~11 x inner SHA-1 blocks + 8.
-__device__ __noinline__ void roles_sort_slots(uint2 *rec, uint32_t *cumb, uint16_t *d16, const uint32_t *sav,
+__device__ __noinline__ void roles_sort_slots(uint4 *rec, uint32_t *cumb, uint16_t *d16, const uint32_t *sav,
                                               uint32_t (*hw)[NBINS], uint32_t r0, uint32_t n,
                                               uint32_t ppc, uint32_t cbeg, uint32_t cend)
 {
@@ -2243,7 +2243,7 @@ __device__ __noinline__ void roles_sort_slots(uint2 *rec, uint32_t *cumb, uint16
         for (uint32_t sl = lane; sl < 512u; sl += 32u) {
             const uint32_t r = __shfl_sync(0xffffffffu, myrun, sl >> 5);
             if (r == 0xffffffffu || 32u * r + (sl & 31u) >= cnt)
-                rec[(size_t)cc * 512u + sl] = make_uint2(0u, 0xffffffffu);
+                rec[(size_t)cc * 512u + sl] = make_uint4(0u, 0xffffffffu, 0u, 0u);
         }
         __syncwarp();
     }
@@ -2396,7 +2396,7 @@ __device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchAr
         }
         __syncthreads();
         if (Q.sorted)
-            roles_sort_slots(reinterpret_cast<uint2 *>(Q.rec) + (size_t)(bi % ROLES_NREC) * Lc * 512u, Q.cum,
+            roles_sort_slots(reinterpret_cast<uint4 *>(Q.rec) + (size_t)(bi % ROLES_NREC) * Lc * 512u, Q.cum,
                              lenv, sav, sorth, r0, n, ppc, cbeg, cend);
 #if NBA_ROLES_TRACE
         if (R.ts && p == 0 && tid == 0) *RLT(bi, 1) = gtimer();
@@ -2446,7 +2446,7 @@ __device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchAr
 #endif
         // D. the records (the sequence number, 0 = drop): by packet index, or
         //    (sorted mode) {q, packet} at the packet's lane slot
-        uint32_t *rec = Q.rec + (size_t)(bi % ROLES_NREC) * Lc * 512u * (Q.sorted ? 2u : 1u);
+        uint32_t *rec = Q.rec + (size_t)(bi % ROLES_NREC) * Lc * 512u * (Q.sorted ? 4u : 1u);   // (uint4 records)
 #pragma unroll 4
         for (uint32_t g0 = w0; g0 < w1; g0 += 32u) {
             const uint32_t i = g0 + lane;
@@ -2459,9 +2459,13 @@ __device__ __forceinline__ void roles_sequencer(const DevTable &T, const BatchAr
                     r = q <= 0xffffffffull ? (uint32_t)q : 0u;
                 }
                 if (Q.sorted) {
+                    // {q, packet | D << 9 | SA << 20 (D, SA: valid packets only), in_off, out_off}:
+                    // the lane needs no load of the packet's fields
                     const uint32_t c = i / ppc;
-                    reinterpret_cast<uint2 *>(rec)[(size_t)c * 512u + lenv[i - r0]] = make_uint2(r, i - c * ppc);
-                    if (s != 0xffffffffu) prefetch_l2(B.in_buf + B.in_off[i]);   // its payload's first line
+                    const uint32_t io = B.in_off[i], oo = B.out_off[i];
+                    const uint32_t y = (i - c * ppc) | (s != 0xffffffffu ? ((uint32_t)B.in_len[i] << 9) | (s << 20) : 0u);
+                    reinterpret_cast<uint4 *>(rec)[(size_t)c * 512u + lenv[i - r0]] = make_uint4(r, y, io, oo);
+                    if (s != 0xffffffffu) prefetch_l2(B.in_buf + io);   // its payload's first line
                 } else {
                     rec[i] = r;
                 }
@@ -2693,7 +2697,8 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
 
 // Lane CTA, sorted mode (mixed-length rings): the record at the thread's own
 // lane slot names its packet {q, packet in the CTA's range} -- the packet's
-// fields are read after the record -- and a fence precedes the "consumed"
+// fields come in the record: {q, j | D << 9 | SA << 20, in_off, out_off} --
+// and a fence precedes the "consumed"
 // count: a packet slot may go to a different lane in a later batch of the
 // same ring slot, so this warp's earlier output stores must be visible before
 // the sequencers can publish a batch that reuses them (ring_create takes this
@@ -2727,9 +2732,9 @@ __device__ __forceinline__ void roles_lanes_sorted(const DevTable &T, const DevW
     tables_bulk_wait(&L.tbar, 0u);
     const uint32_t *ready = Q.ctl;
     uint32_t *consumed = Q.ctl + ROLES_NREC;
-    const uint2 *rec = reinterpret_cast<const uint2 *>(Q.rec);
+    const uint4 *rec = reinterpret_cast<const uint4 *>(Q.rec);
     unsigned long long c_ok = 0, c_drop = 0, c_in = 0, c_out = 0;
-    uint2 r = make_uint2(0u, 0xffffffffu);
+    uint4 r = make_uint4(0u, 0xffffffffu, 0u, 0u);
     uint32_t rv_next = 0u;
     bool got = false;
     for (uint32_t bi = 0; bi < R.n_batches; bi++) {
@@ -2739,15 +2744,10 @@ __device__ __forceinline__ void roles_lanes_sorted(const DevTable &T, const DevW
             r = __ldcg(&rec[((size_t)(bi % ROLES_NREC) * Lc + c) * 512u + tid]);
         }
         const bool have = r.y != 0xffffffffu;
-        const uint32_t i = c * ((B.n + Lc - 1u) / Lc) + (have ? r.y : 0u);
-        uint32_t sa = INVALID_SA, D = 0u, inoff = 0u, outoff = 0u;
-        if (have) {
-            sa = B.sa_idx[i];
-            D = B.in_len[i];
-            inoff = B.in_off[i];
-            outoff = B.out_off[i];
-        }
-        const bool cand = have && sa < n_sa && D >= MIN_D && D <= MAX_D;
+        const uint32_t i = c * ((B.n + Lc - 1u) / Lc) + (have ? (r.y & 0x1ffu) : 0u);
+        // the packet's fields come with its record (q != 0: a valid packet)
+        const bool cand = have && r.x != 0u;
+        const uint32_t sa = r.y >> 20, D = (r.y >> 9) & 0x7ffu, inoff = r.z, outoff = r.w;
         PktPre pp = {};
         if (cand) {
             pp = load_pkt_pre(T, B.in_buf, sa, inoff, true, 0u);
