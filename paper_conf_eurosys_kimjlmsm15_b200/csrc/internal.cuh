@@ -211,7 +211,10 @@ cudaError_t launch_fused_ring_free(const DevTable &T, const DevWork &W, const Ba
 bool fused_pipe_ok(uint32_t n, int grid);
 // Role-split ring (k_fused_ring_roles): npro sequencer CTAs write one record
 // per packet into a ring of ROLES_NREC record buffers, the other CTAs encrypt.
-constexpr uint32_t ROLES_NREC = 4;          // batches of records in flight
+#ifndef NBA_ROLES_NREC
+#define NBA_ROLES_NREC 4
+#endif
+constexpr uint32_t ROLES_NREC = NBA_ROLES_NREC;   // batches of records in flight
 constexpr uint32_t ROLES_MAX_SA = 2048;     // per-warp SA counters in a sequencer's shared memory
 constexpr uint32_t ROLES_RPP_MAX = 16416;   // packets per sequencer and batch (shared stash: 36 lane
                                             //   CTAs x 456 packets, a 65,536-packet batch at 4 sequencers)
