@@ -2020,6 +2020,9 @@ __device__ __forceinline__ void roles_lane_consumed(uint32_t *p, uint32_t q)
 #ifndef NBA_ROLES_SAL_AHEAD   // lanes: the next packet's SA line loaded at the end of an iteration
 #define NBA_ROLES_SAL_AHEAD 0       // (measured: 64 B 20.5 -> 20.7 us, 128 B 29.3 -> 28.4, 512 B 73.6 -> 74.6, 1024 B 134 -> 137)
 #endif
+#ifndef NBA_ROLES_SAL_L1      // lanes: L1 prefetch of the next packet's SA line after each packet
+#define NBA_ROLES_SAL_L1 0
+#endif
 #ifndef NBA_ROLES_RK_ASYNC    // lanes: round keys 3..10 by cp.async from the SA's schedule instead of
 #define NBA_ROLES_RK_ASYNC 0  //   expanded from the key (1)
 #endif
@@ -2660,6 +2663,12 @@ __device__ __forceinline__ void roles_lanes(const DevTable &T, const DevWork &W,
                     f = fn;
                     if (f.have) prefetch_l2(sl[R.first % R.n_slots].in_buf + f.inoff);
                     continue;
+                }
+                // (NBA_ROLES_SAL_L1) the next packet's SA line into L1 right away
+                if (NBA_ROLES_SAL_L1 && candidate(fn)) {
+                    const uint4 *ln = T.sal + (size_t)fn.sa * SAL_U4;
+                    asm volatile("prefetch.global.L1 [%0];" ::"l"(ln));
+                    asm volatile("prefetch.global.L1 [%0];" ::"l"(ln + 2));
                 }
                 const uint32_t Lp = 48u + esp_C(f.D);
                 B.out_len[f.i] = (uint16_t)Lp;
