@@ -218,3 +218,14 @@ def test_roles_form_refused_where_it_does_not_fit():
             g_out, g_len = device.fetch(d)
             assert np.array_equal(g_len, o_len) and np.array_equal(g_out, o_out)
             ring.close()
+
+
+@pytest.mark.parametrize("sizes", [(64,), (64, "imix")])
+def test_roles_ring_many_slots(sizes):
+    """More slots than the lanes' shared-memory slot table holds (179): the
+    lanes read the slot arguments from global memory; 190 small slots,
+    fixed-slot (one length) and sorted (mixed) modes, 250 + 140 batches."""
+    n_sa, n, R = 24, 300, 190
+    p = gen.make_sas(n_sa, cfg_id=81)
+    hb = [gen.make_batch(n, sizes[k % len(sizes)], n_sa, cfg_id=81, batch=k) for k in range(R)]
+    _roles_vs_oracle(p, n_sa, hb, [250, 140], force=False)
