@@ -229,3 +229,13 @@ def test_roles_ring_many_slots(sizes):
     p = gen.make_sas(n_sa, cfg_id=81)
     hb = [gen.make_batch(n, sizes[k % len(sizes)], n_sa, cfg_id=81, batch=k) for k in range(R)]
     _roles_vs_oracle(p, n_sa, hb, [250, 140], force=False)
+
+
+def test_roles_ring_slots_of_different_sizes():
+    """Slots of 65,536 / 1,000 / 30,000 / 7 packets in one ring (the lanes'
+    packet -> lane mapping changes from slot to slot, the bootstrap takes the
+    first batch's), 9 + 6 batches."""
+    n_sa = 300
+    p = gen.make_sas(n_sa, cfg_id=82)
+    hb = [gen.make_batch(n, 64, n_sa, cfg_id=82, batch=k) for k, n in enumerate((65536, 1000, 30000, 7))]
+    _roles_vs_oracle(p, n_sa, hb, [9, 6], force=False)
